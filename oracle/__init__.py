@@ -1,0 +1,165 @@
+"""CPU oracle for the LOO-CV bandwidth grid search (Rohlfs & Zahran 2017).
+
+TEST INFRASTRUCTURE ONLY.  Only ``tests/``, ``__graft_entry__.smoke()`` and
+``bench.py``'s ``cpu_baseline`` / ``--impl reference`` legs may import this
+package.  It shares no code with the CUDA path; the only module both sides
+import is ``workloads`` (seeded input recipes, no method arithmetic).
+
+Contents
+--------
+* ``cv_direct``   -- C, the plain definition Eq.(1)-(3) (PAPER.md P@11484-12036),
+                     O(n^2 m), long double (or double for pin P9).
+* ``cv_sorted``   -- C, the paper's Program 3: per-row sort + ascending sweep
+                     (P@13614-14984, P@20401-22459), long double.
+* ``exact.cv_exact``        -- Python ``fractions`` brute force of Eq.(1)-(3).
+* ``window.cv_window``      -- numpy long-double window-prefix checker (pin P10).
+* ``sorted_rows``           -- the x-sorted row order (stable by (x, index))
+                               that defines shards.
+
+Parity status: every function here is pinned by tests/test_oracle_pins.py
+(see DESIGN.md "Oracle pins").  None is "parity unpinned".
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_BUILD = os.path.join(_HERE, "build")
+
+UNIFORM, EPANECHNIKOV, TRIANGULAR = 0, 1, 2
+
+_libs: dict[str, ctypes.CDLL] = {}
+
+
+def build() -> None:
+    """Compile the oracle shared libraries (gcc + OpenMP)."""
+    subprocess.run(["make", "-s", "-C", _HERE], check=True)
+
+
+def _lib(precision: str = "ld") -> ctypes.CDLL:
+    if precision not in ("ld", "d"):
+        raise ValueError(precision)
+    if precision in _libs:
+        return _libs[precision]
+    path = os.path.join(_BUILD, f"liboracle_{precision}.so")
+    if not os.path.exists(path):
+        build()
+    lib = ctypes.CDLL(path)
+    P = ctypes.c_void_p
+    i64, i32 = ctypes.c_int64, ctypes.c_int32
+    lib.kro_cv_direct.argtypes = [P, P, i64, P, i32, i32, P, i64, P, P, P, P, P, P, P]
+    lib.kro_cv_direct.restype = ctypes.c_int
+    lib.kro_cv_sorted.argtypes = [P, P, i64, P, i32, i32, P, i64, P, P, P, P]
+    lib.kro_cv_sorted.restype = ctypes.c_int
+    lib.kro_default_grid.argtypes = [P, i64, i32, P]
+    lib.kro_default_grid.restype = ctypes.c_int
+    lib.kro_finalize.argtypes = [P, i64, i32, P, P]
+    lib.kro_finalize.restype = ctypes.c_int
+    lib.kro_real_bits.restype = ctypes.c_int
+    lib.kro_num_threads.restype = ctypes.c_int
+    _libs[precision] = lib
+    return lib
+
+
+class OracleError(RuntimeError):
+    def __init__(self, status: int):
+        super().__init__(f"oracle status {status}")
+        self.status = status
+
+
+def _ptr(a):
+    return None if a is None else a.ctypes.data
+
+
+def _prep(x, y, h):
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    y = np.ascontiguousarray(y, dtype=np.float64)
+    h = np.ascontiguousarray(h, dtype=np.float64)
+    return x, y, h
+
+
+class Result(dict):
+    """dict with keys cv, best, S, neff (and aux sums for cv_direct)."""
+    __getattr__ = dict.__getitem__
+
+
+def cv_direct(x, y, h, kernel: int, rows=None, precision: str = "ld", aux: bool = False) -> Result:
+    """Plain definition, Eq.(1)-(3).  rows: optional original-index row list."""
+    x, y, h = _prep(x, y, h)
+    n, m = x.shape[0], h.shape[0]
+    r = None if rows is None else np.ascontiguousarray(rows, dtype=np.int64)
+    S = np.zeros(m); ne = np.zeros(m, np.int64); cv = np.zeros(m)
+    best = ctypes.c_int32(-1)
+    cs = np.zeros(m, np.int64) if aux else None
+    sy = np.zeros(m) if aux else None
+    s2 = np.zeros(m) if aux else None
+    st = _lib(precision).kro_cv_direct(
+        _ptr(x), _ptr(y), n, _ptr(h), m, int(kernel), _ptr(r), 0 if r is None else r.shape[0],
+        _ptr(S), _ptr(ne), _ptr(cs), _ptr(sy), _ptr(s2), _ptr(cv), ctypes.byref(best))
+    if st:
+        raise OracleError(st)
+    out = Result(cv=cv, best=int(best.value), S=S, neff=ne)
+    if aux:
+        out.update(csum=cs, sysum=sy, sd2sum=s2)
+    return out
+
+
+def cv_sorted(x, y, h, kernel: int, rows=None, precision: str = "ld") -> Result:
+    """The paper's Program-3 algorithm: per-row sort + ascending sweep."""
+    x, y, h = _prep(x, y, h)
+    n, m = x.shape[0], h.shape[0]
+    r = None if rows is None else np.ascontiguousarray(rows, dtype=np.int64)
+    S = np.zeros(m); ne = np.zeros(m, np.int64); cv = np.zeros(m)
+    best = ctypes.c_int32(-1)
+    st = _lib(precision).kro_cv_sorted(
+        _ptr(x), _ptr(y), n, _ptr(h), m, int(kernel), _ptr(r), 0 if r is None else r.shape[0],
+        _ptr(S), _ptr(ne), _ptr(cv), ctypes.byref(best))
+    if st:
+        raise OracleError(st)
+    return Result(cv=cv, best=int(best.value), S=S, neff=ne)
+
+
+def default_grid(x, m: int) -> np.ndarray:
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    h = np.zeros(m)
+    st = _lib().kro_default_grid(_ptr(x), x.shape[0], int(m), _ptr(h))
+    if st:
+        raise OracleError(st)
+    return h
+
+
+def finalize(S, n: int):
+    """CV = S/n and the Q11 arg-min, for summed shard partials."""
+    S = np.ascontiguousarray(S, dtype=np.float64)
+    m = S.shape[0]
+    cv = np.zeros(m); best = ctypes.c_int32(-1)
+    st = _lib().kro_finalize(_ptr(S), int(n), m, _ptr(cv), ctypes.byref(best))
+    if st:
+        raise OracleError(st)
+    return cv, int(best.value)
+
+
+def sorted_rows(x) -> np.ndarray:
+    """Row order of the x-sorted data, ties by original index (stable)."""
+    return np.argsort(np.asarray(x, dtype=np.float64), kind="stable").astype(np.int64)
+
+
+def shard_rows(x, shard: int, nshards: int) -> np.ndarray:
+    """Original indices of the rows of shard r/P: sorted positions
+    [floor(r n / P), floor((r+1) n / P))."""
+    order = sorted_rows(x)
+    n = order.shape[0]
+    lo, hi = (shard * n) // nshards, ((shard + 1) * n) // nshards
+    return order[lo:hi]
+
+
+def num_threads() -> int:
+    return int(_lib().kro_num_threads())
+
+
+def real_bits(precision: str = "ld") -> int:
+    return int(_lib(precision).kro_real_bits())

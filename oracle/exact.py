@@ -1,0 +1,70 @@
+"""Exact-rational brute force of Eq.(1)-(3) -- pin P1.
+
+TEST INFRASTRUCTURE ONLY.
+
+Straight from the definition (§III):
+  Eq.(1) P@11484  CV(h) = n^-1 sum_i (Y_i - g_{-i}(X_i))^2 M(X_i)
+  Eq.(2) P@11694  g_{-i}(X_i) = sum_{l!=i} Y_l K((X_i-X_l)/h) / sum_{l!=i} K(.)
+         P@11802  M = 1 iff the denominator of (2) is non-zero
+  Eq.(3) P@11971  K(u) = 0.75 (1 - u^2) I{|u| <= 1}
+  fn.1   P@18521  uniform K = 1/2 I{|u|<=1}; triangular K = (1-|u|) I{|u|<1} (Q13)
+
+Every value is a ``fractions.Fraction``; no sort, no running sum, no
+decomposition.  Window membership follows reading Q1: decided in binary64 on
+d = |x_l - x_i| (Python float subtraction is IEEE binary64), with '<' for
+Epanechnikov/triangular and '<=' for uniform.  On the dyadic inputs the pins
+use, binary64 subtraction is exact, so this equals the rational test.
+M_i follows Q6 (at least one in-window neighbour), Q7 (M=0 rows add 0, divide
+by n) and Q11 (smallest arg-min).
+"""
+from __future__ import annotations
+
+from fractions import Fraction
+
+UNIFORM, EPANECHNIKOV, TRIANGULAR = 0, 1, 2
+
+
+def _K(u: Fraction, kernel: int) -> Fraction:
+    if kernel == EPANECHNIKOV:
+        return Fraction(3, 4) * (1 - u * u)
+    if kernel == TRIANGULAR:
+        return 1 - u
+    return Fraction(1, 2)
+
+
+def cv_exact(x, y, h, kernel: int):
+    """Return (cv list of Fractions, neff list, best index)."""
+    xs = [float(v) for v in x]
+    ys = [Fraction(float(v)) for v in y]
+    hs = [float(v) for v in h]
+    n = len(xs)
+    cvs, neffs = [], []
+    for hb in hs:
+        H = Fraction(hb)
+        tot = Fraction(0)
+        ne = 0
+        for i in range(n):
+            num = Fraction(0)
+            den = Fraction(0)
+            cnt = 0
+            for l in range(n):
+                if l == i:
+                    continue
+                d64 = abs(xs[l] - xs[i])
+                inside = d64 <= hb if kernel == UNIFORM else d64 < hb
+                if not inside:
+                    continue
+                u = abs(Fraction(xs[i]) - Fraction(xs[l])) / H
+                w = _K(u, kernel)
+                num += ys[l] * w
+                den += w
+                cnt += 1
+            if cnt == 0:
+                continue
+            e = ys[i] - num / den
+            tot += e * e
+            ne += 1
+        cvs.append(tot / n)
+        neffs.append(ne)
+    best = min(range(len(cvs)), key=lambda b: (cvs[b], b))
+    return cvs, neffs, best

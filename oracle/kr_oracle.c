@@ -1,0 +1,378 @@
+/*
+ * kr_oracle.c -- CPU ORACLE for the leave-one-out CV bandwidth grid search.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and
+ * bench.py's cpu_baseline / --impl reference legs may load this library.
+ * It shares no code, header, table or helper with the CUDA path
+ * (paper_conf_ipps_rohlfsz17_b200/csrc); neither includes the other.
+ *
+ * What it computes (PAPER.md = Rohlfs & Zahran, IPDPSW 2017; citations are
+ * P@<char offset> into the single-line PAPER.md):
+ *
+ *   Eq.(1) P@11484  CV(h) = n^-1 sum_i (Y_i - g_{-i}(X_i))^2 M(X_i)
+ *   Eq.(2) P@11694  g_{-i}(X_i) = sum_{l!=i} Y_l K((X_i-X_l)/h) / sum_{l!=i} K((X_i-X_l)/h)
+ *          P@11802  M(X_i) = 1 iff the denominator of (2) is non-zero
+ *   Eq.(3) P@11971  K(u) = 0.75 (1-u^2) I{|u|<=1}           (Epanechnikov)
+ *   fn.1   P@18521  "The same approach can be used for the Uniform and
+ *                   Triangular kernels"  -> K(u)=1/2 I{|u|<=1},
+ *                   K(u)=(1-|u|) I{|u|<1}  (reading Q13, textbook forms)
+ *
+ * Two independent evaluators:
+ *
+ *   kro_cv_direct  -- the plain definition, Eq.(1)-(3) written out:
+ *                     for every bandwidth, every row, every other row.
+ *                     O(n^2 m).  No sort, no running sums.
+ *   kro_cv_sorted  -- the paper's own algorithm (Program 3 "Sequential C",
+ *                     P@27641, P@28414; §III P@13614-14984; §IV.B
+ *                     P@20401-22459): per row, fill |X_i - X_l|, sort,
+ *                     sweep the ascending grid carrying the running sums
+ *                     forward ("copy our sums ... and begin to add",
+ *                     P@21724), then divide by h^2, multiply by 0.75,
+ *                     form (Y_i - g)^2 M.
+ *
+ * Readings of the paper used here:
+ *   Q1  window membership is decided in IEEE binary64 on d = fabs(x_l - x_i):
+ *       d <  h for Epanechnikov and triangular, d <= h for uniform.
+ *   Q6  M_i = [number of in-window l != i >= 1] (integer test).
+ *   Q7  rows with M_i = 0 contribute 0; CV divides by n (Eq.(1) literally).
+ *   Q8  leave-one-out excludes the index i only (duplicates of X_i stay).
+ *   Q11 best = smallest b with minimal CV; NaN is never minimal.
+ *   Q12 arithmetic in long double (KRO_REAL), inputs are binary64.
+ *   Q14 the sorted sweep's decomposition h^2 c - sum d^2 cancels when all
+ *       in-window points sit near the edge; if 0.75(c - sum d^2/h^2) <
+ *       2^-30 * 0.75 c it recomputes numerator and denominator directly from
+ *       K over the sorted prefix (the direct form has no cancellation).
+ *
+ * Determinism: row work is split in fixed chunks whose partial sums are
+ * added in chunk order, so results do not depend on the thread count.
+ */
+#include <math.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+#ifndef KRO_REAL
+#define KRO_REAL long double
+#endif
+typedef KRO_REAL real;
+
+#define KRO_UNIFORM 0
+#define KRO_EPANECHNIKOV 1
+#define KRO_TRIANGULAR 2
+
+#define KRO_OK 0
+#define KRO_EARG 1
+#define KRO_EKERNEL 2
+#define KRO_EGRID 3
+#define KRO_ENONFINITE 4
+#define KRO_EDEGENERATE 5
+#define KRO_ENOMEM 6
+
+#define KRO_MAX_M 65536
+#define KRO_CHUNK 256
+
+/* ------------------------------------------------------------------ */
+/* validation: same contract as the C-ABI, own code   */
+/* ------------------------------------------------------------------ */
+static int kro_validate(const double *x, const double *y, int64_t n,
+                        const double *h, int32_t m, int32_t kernel)
+{
+    if (!x || !y || !h) return KRO_EARG;
+    if (n < 2 || n > 2147483647LL || m < 1 || m > KRO_MAX_M) return KRO_EARG;
+    if (kernel != KRO_UNIFORM && kernel != KRO_EPANECHNIKOV && kernel != KRO_TRIANGULAR)
+        return KRO_EKERNEL;
+    for (int32_t b = 0; b < m; b++) {
+        if (!isfinite(h[b]) || !(h[b] > 0.0)) return KRO_EGRID;
+        if (b > 0 && h[b] < h[b - 1]) return KRO_EGRID;
+    }
+    for (int64_t i = 0; i < n; i++)
+        if (!isfinite(x[i]) || !isfinite(y[i])) return KRO_ENONFINITE;
+    return KRO_OK;
+}
+
+/* Q1: the window predicate, binary64. */
+static int in_window(double d, double h, int32_t kernel)
+{
+    return kernel == KRO_UNIFORM ? (d <= h) : (d < h);
+}
+
+/* Eq.(3) and footnote 1 (Q13), with u = d/h, |u| inside the window. */
+static real kernel_K(double d, double h, int32_t kernel)
+{
+    real u = (real)d / (real)h;
+    switch (kernel) {
+    case KRO_EPANECHNIKOV: return (real)0.75 * ((real)1 - u * u);
+    case KRO_TRIANGULAR:   return (real)1 - u;
+    default:               return (real)0.5;
+    }
+}
+
+/* Default grid, §IV P@16146-16375: max = range of X, min = range/k, evenly
+ * spaced; written h_b = r * ((b+1)/m) (reading Q9). */
+int kro_default_grid(const double *x, int64_t n, int32_t m, double *h_out)
+{
+    if (!x || !h_out || n < 2 || m < 1 || m > KRO_MAX_M) return KRO_EARG;
+    double lo = x[0], hi = x[0];
+    for (int64_t i = 0; i < n; i++) {
+        if (!isfinite(x[i])) return KRO_ENONFINITE;
+        if (x[i] < lo) lo = x[i];
+        if (x[i] > hi) hi = x[i];
+    }
+    double r = hi - lo;
+    if (!(r > 0.0)) return KRO_EDEGENERATE;
+    for (int32_t b = 0; b < m; b++) h_out[b] = r * ((double)(b + 1) / (double)m);
+    return KRO_OK;
+}
+
+/* Eq.(1) finalize + Q11 arg-min.  S[b] = sum_i M_i e_i^2 (long double). */
+static void kro_finish(const real *S, int64_t n, int32_t m, double *cv_out, int32_t *best_out)
+{
+    int32_t best = -1;
+    for (int32_t b = 0; b < m; b++) {
+        double cv = (double)(S[b] / (real)n);
+        if (cv_out) cv_out[b] = cv;
+        if (!isnan(cv) && (best < 0 || cv < (double)(S[best] / (real)n))) best = b;
+    }
+    if (best_out) *best_out = best < 0 ? 0 : best;
+}
+
+/* ------------------------------------------------------------------ */
+/* Evaluator 1: the plain definition, Eq.(1)-(3).                      */
+/* rows: optional list of row indices (NULL = all rows 0..n-1).         */
+/* S_out[m]   : sum over the listed rows of M_i (Y_i - g_{-i})^2        */
+/* neff_out[m]: sum over the listed rows of M_i                         */
+/* csum_out, sysum_out, sd2sum_out (nullable, [m]): sum over rows of    */
+/*   |W_i|, sum_{l in W_i} Y_l, sum_{l in W_i} d_il^2  (pins P7, P8)    */
+/* ------------------------------------------------------------------ */
+static int direct_core(const double *x, const double *y, int64_t n,
+                       const double *h, int32_t m, int32_t kernel,
+                       const int64_t *rows, int64_t nrows,
+                       real *S, int64_t *neff, int64_t *csum, real *sysum, real *sd2sum)
+{
+    int64_t R = rows ? nrows : n;
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int32_t b = 0; b < m; b++) {
+        real Sb = 0, sy_b = 0, sd2_b = 0;
+        int64_t ne = 0, cs = 0;
+        for (int64_t r = 0; r < R; r++) {
+            int64_t i = rows ? rows[r] : r;
+            real num = 0, den = 0;      /* Eq.(2) numerator, denominator */
+            int64_t cnt = 0;
+            for (int64_t l = 0; l < n; l++) {
+                if (l == i) continue;                       /* l != i */
+                double d = fabs(x[l] - x[i]);
+                if (!in_window(d, h[b], kernel)) continue;  /* I{|u| <= 1} */
+                real w = kernel_K(d, h[b], kernel);
+                num += (real)y[l] * w;
+                den += w;
+                cnt++;
+                sy_b += (real)y[l];
+                sd2_b += (real)d * (real)d;
+            }
+            cs += cnt;
+            if (cnt == 0) continue;                         /* M(X_i) = 0 */
+            real e = (real)y[i] - num / den;
+            Sb += e * e;
+            ne++;
+        }
+        S[b] = Sb;
+        neff[b] = ne;
+        if (csum) csum[b] = cs;
+        if (sysum) sysum[b] = sy_b;
+        if (sd2sum) sd2sum[b] = sd2_b;
+    }
+    return KRO_OK;
+}
+
+int kro_cv_direct(const double *x, const double *y, int64_t n,
+                  const double *h, int32_t m, int32_t kernel,
+                  const int64_t *rows, int64_t nrows,
+                  double *S_out, int64_t *neff_out,
+                  int64_t *csum_out, double *sysum_out, double *sd2sum_out,
+                  double *cv_out, int32_t *best_out)
+{
+    int st = kro_validate(x, y, n, h, m, kernel);
+    if (st) return st;
+    if (rows && nrows < 0) return KRO_EARG;
+    if (rows)
+        for (int64_t r = 0; r < nrows; r++)
+            if (rows[r] < 0 || rows[r] >= n) return KRO_EARG;
+    real *S = (real *)calloc((size_t)m, sizeof(real));
+    real *sy = (real *)calloc((size_t)m, sizeof(real));
+    real *sd2 = (real *)calloc((size_t)m, sizeof(real));
+    int64_t *ne = (int64_t *)calloc((size_t)m, sizeof(int64_t));
+    if (!S || !sy || !sd2 || !ne) { free(S); free(sy); free(sd2); free(ne); return KRO_ENOMEM; }
+    st = direct_core(x, y, n, h, m, kernel, rows, nrows, S, ne, csum_out, sy, sd2);
+    if (!st) {
+        for (int32_t b = 0; b < m; b++) {
+            if (S_out) S_out[b] = (double)S[b];
+            if (neff_out) neff_out[b] = ne[b];
+            if (sysum_out) sysum_out[b] = (double)sy[b];
+            if (sd2sum_out) sd2sum_out[b] = (double)sd2[b];
+        }
+        kro_finish(S, n, m, cv_out, best_out);
+    }
+    free(S); free(sy); free(sd2); free(ne);
+    return st;
+}
+
+/* ------------------------------------------------------------------ */
+/* Evaluator 2: the paper's sorting-based sweep (Program 3).           */
+/* ------------------------------------------------------------------ */
+typedef struct { double d; double y; int64_t l; } kro_pair;
+
+static int cmp_pair(const void *a, const void *b)
+{
+    const kro_pair *p = (const kro_pair *)a, *q = (const kro_pair *)b;
+    if (p->d < q->d) return -1;
+    if (p->d > q->d) return 1;
+    return (p->l > q->l) - (p->l < q->l);
+}
+
+/* One row i: fill, sort, sweep, residuals.  Adds into S[m], ne[m]. */
+static void sorted_row(const double *x, const double *y, int64_t n,
+                       const double *h, int32_t m, int32_t kernel, int64_t i,
+                       kro_pair *buf, real *S, int64_t *ne)
+{
+    const real tau = (real)1 / (real)1073741824.0; /* 2^-30, Q14 */
+    /* "Each thread j fills in n values of the abs(X_i - X_j) and Y_i" P@20401 */
+    int64_t k = 0;
+    for (int64_t l = 0; l < n; l++) {
+        if (l == i) continue; /* "the final sums exclude ... the j-th observation" P@22353 */
+        buf[k].d = fabs(x[l] - x[i]);
+        buf[k].y = y[l];
+        buf[k].l = l;
+        k++;
+    }
+    /* "it sorts both of these matrices in order of abs(X_i - X_j)" P@20459 */
+    qsort(buf, (size_t)k, sizeof(kro_pair), cmp_pair);
+
+    /* "We begin with the smallest bandwidth" P@21154 -- running sums carried
+     * from bandwidth to bandwidth. §III P@14010: sums of Y_l, Y_l d^2, d^2;
+     * plus the count c (reading Q3). Triangular: Y_l d and d (reading Q13). */
+    int64_t p = 0;
+    real c = 0, sy = 0, s2 = 0, sy2 = 0;
+    for (int32_t b = 0; b < m; b++) {
+        double hb = h[b];
+        while (p < k && in_window(buf[p].d, hb, kernel)) {
+            real d = (real)buf[p].d, yl = (real)buf[p].y;
+            c += 1;
+            sy += yl;
+            if (kernel == KRO_EPANECHNIKOV) { s2 += d * d; sy2 += yl * d * d; }
+            else if (kernel == KRO_TRIANGULAR) { s2 += d; sy2 += yl * d; }
+            p++;
+        }
+        if (p == 0) continue; /* M(X_i) = 0: no in-window neighbour (Q6, Q7) */
+        real H = (real)hb, g;
+        if (kernel == KRO_UNIFORM) {
+            g = ((real)0.5 * sy) / ((real)0.5 * c);
+        } else {
+            /* "divided by the square of the bandwidths and multiplied by 0.75" P@22188 */
+            real num, den;
+            if (kernel == KRO_EPANECHNIKOV) {
+                num = (real)0.75 * (sy - sy2 / (H * H));
+                den = (real)0.75 * (c - s2 / (H * H));
+                if (!(den >= tau * (real)0.75 * c)) goto direct;
+            } else {
+                num = sy - sy2 / H;
+                den = c - s2 / H;
+                if (!(den >= tau * c)) goto direct;
+            }
+            g = num / den;
+            goto emit;
+        direct: /* Q14: recompute from K over the in-window prefix [0, p) */
+            num = 0; den = 0;
+            for (int64_t q = 0; q < p; q++) {
+                real w = kernel_K(buf[q].d, hb, kernel);
+                num += (real)buf[q].y * w;
+                den += w;
+            }
+            g = num / den;
+        }
+    emit:;
+        real e = (real)y[i] - g;
+        S[b] += e * e;
+        ne[b] += 1;
+    }
+}
+
+int kro_cv_sorted(const double *x, const double *y, int64_t n,
+                  const double *h, int32_t m, int32_t kernel,
+                  const int64_t *rows, int64_t nrows,
+                  double *S_out, int64_t *neff_out,
+                  double *cv_out, int32_t *best_out)
+{
+    int st = kro_validate(x, y, n, h, m, kernel);
+    if (st) return st;
+    int64_t R = rows ? nrows : n;
+    if (R < 0) return KRO_EARG;
+    if (rows)
+        for (int64_t r = 0; r < R; r++)
+            if (rows[r] < 0 || rows[r] >= n) return KRO_EARG;
+    int64_t nchunks = (R + KRO_CHUNK - 1) / KRO_CHUNK;
+    real *Sc = (real *)calloc((size_t)(nchunks ? nchunks : 1) * (size_t)m, sizeof(real));
+    int64_t *nc = (int64_t *)calloc((size_t)(nchunks ? nchunks : 1) * (size_t)m, sizeof(int64_t));
+    if (!Sc || !nc) { free(Sc); free(nc); return KRO_ENOMEM; }
+    int oom = 0;
+#pragma omp parallel
+    {
+        kro_pair *buf = (kro_pair *)malloc((size_t)n * sizeof(kro_pair));
+        if (!buf) {
+#pragma omp atomic write
+            oom = 1;
+        }
+#pragma omp for schedule(dynamic, 1)
+        for (int64_t ch = 0; ch < nchunks; ch++) {
+            if (!buf) continue;
+            int64_t r0 = ch * KRO_CHUNK, r1 = r0 + KRO_CHUNK < R ? r0 + KRO_CHUNK : R;
+            for (int64_t r = r0; r < r1; r++) {
+                int64_t i = rows ? rows[r] : r;
+                sorted_row(x, y, n, h, m, kernel, i, buf, Sc + ch * m, nc + ch * m);
+            }
+        }
+        free(buf);
+    }
+    if (oom) { free(Sc); free(nc); return KRO_ENOMEM; }
+    /* "a summation reduction is performed k times, once for each bandwidth" P@23970;
+     * chunk partials added in chunk order (deterministic). */
+    real *S = (real *)calloc((size_t)m, sizeof(real));
+    if (!S) { free(Sc); free(nc); return KRO_ENOMEM; }
+    for (int32_t b = 0; b < m; b++) {
+        real s = 0;
+        int64_t ne = 0;
+        for (int64_t ch = 0; ch < nchunks; ch++) { s += Sc[ch * m + b]; ne += nc[ch * m + b]; }
+        S[b] = s;
+        if (S_out) S_out[b] = (double)s;
+        if (neff_out) neff_out[b] = ne;
+    }
+    kro_finish(S, n, m, cv_out, best_out);
+    free(S); free(Sc); free(nc);
+    return KRO_OK;
+}
+
+/* Public finalize for summed shard partials (mirrors the ABI's kr_finalize,
+ * own code): CV[b] = S[b]/n, best per Q11. */
+int kro_finalize(const double *S, int64_t n, int32_t m, double *cv_out, int32_t *best_out)
+{
+    if (!S || n < 1 || m < 1) return KRO_EARG;
+    real *T = (real *)malloc((size_t)m * sizeof(real));
+    if (!T) return KRO_ENOMEM;
+    for (int32_t b = 0; b < m; b++) T[b] = (real)S[b];
+    kro_finish(T, n, m, cv_out, best_out);
+    free(T);
+    return KRO_OK;
+}
+
+int kro_real_bits(void) { return (int)(sizeof(real) * 8); }
+
+int kro_num_threads(void)
+{
+#ifdef _OPENMP
+    return omp_get_max_threads();
+#else
+    return 1;
+#endif
+}

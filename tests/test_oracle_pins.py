@@ -1,0 +1,313 @@
+"""Pins for the CPU oracle.  CPU only.
+
+The oracle is pinned to things other than itself: exact rationals of the
+definition, hand-derived values, closed forms, invariances, integer identities
+and an independent algorithm.  Each test names the pin and the passage.
+"""
+from __future__ import annotations
+
+import json
+import math
+import os
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads
+from oracle import exact, window
+from tests.helpers import best_ok, cv_rel_err
+
+U, E, T = oracle.UNIFORM, oracle.EPANECHNIKOV, oracle.TRIANGULAR
+KERNELS = [U, E, T]
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+EVALS = {
+    "direct": lambda *a, **k: oracle.cv_direct(*a, **k),
+    "sorted": lambda *a, **k: oracle.cv_sorted(*a, **k),
+}
+
+
+def _frac_rel(got: np.ndarray, exact_vals) -> float:
+    ex = [float(v) for v in exact_vals]
+    return cv_rel_err(got, ex)
+
+
+# ---------------------------------------------------------------- P2
+@pytest.mark.parametrize("which", ["direct", "sorted"])
+@pytest.mark.parametrize("kname", ["epanechnikov", "uniform", "triangular"])
+def test_P2_worked_example(which, kname):
+    """Hand-derived fixture tests/golden/worked_example.json (Eq.(1)-(3))."""
+    g = json.load(open(os.path.join(GOLDEN, "worked_example.json")))
+    k = workloads.KERNEL_IDS[kname]
+    r = EVALS[which](g["x"], g["y"], g["h"], k)
+    want = [Fraction(s) for s in g[kname]["cv"]]
+    for b, w in enumerate(want):
+        # exact to 1 ulp of the rounded rational
+        assert abs(r.cv[b] - float(w)) <= math.ulp(float(w)) if w else r.cv[b] == 0.0
+    assert list(r.neff) == g[kname]["neff"]
+    assert r.best == g[kname]["best"]
+
+
+# ---------------------------------------------------------------- P1
+@pytest.mark.parametrize("seed", range(24))
+@pytest.mark.parametrize("which", ["direct", "sorted"])
+def test_P1_exact_rational_bruteforce(seed, which):
+    """Exact-rational Eq.(1)-(3) on dyadic inputs incl. duplicates and points
+    exactly at h (the grid is drawn from the pair distances)."""
+    rng = np.random.default_rng(1000 + seed)
+    n = int(rng.integers(2, 17))
+    m = int(rng.integers(1, 9))
+    x, y, h = workloads.random_dyadic(n, m, seed)
+    for k in KERNELS:
+        cv_ex, ne_ex, best_ex = exact.cv_exact(x, y, h, k)
+        r = EVALS[which](x, y, h, k)
+        assert _frac_rel(r.cv, cv_ex) <= 1e-15, (k, r.cv, [float(c) for c in cv_ex])
+        assert list(r.neff) == ne_ex
+        assert r.best == best_ex or r.cv[r.best] == r.cv[best_ex]
+
+
+# ---------------------------------------------------------------- P3
+@pytest.mark.parametrize("n", [2, 3, 17, 200])
+def test_P3_closed_form_all_in_window(n):
+    """h >= range, uniform kernel: g_{-i} = (sum y - y_i)/(n-1), so
+    CV = n/(n-1)^2 * sum (y_i - ybar)^2 (north_star invariant)."""
+    x, y = workloads.draw_xy("paper", n, 5)
+    r = float(x.max() - x.min())
+    ys = [Fraction(v) for v in y]
+    ybar = sum(ys) / n
+    cf = float(Fraction(n, (n - 1) ** 2) * sum((v - ybar) ** 2 for v in ys))
+    h = np.array([r, 2 * r, 1e3 * r])
+    for which in EVALS:
+        res = EVALS[which](x, y, h, U)
+        assert cv_rel_err(res.cv, [cf] * 3) <= 1e-14
+        # Epanechnikov tends to the same limit as h -> inf (bias O((r/h)^2))
+        res = EVALS[which](x, y, np.array([1e6 * r]), E)
+        assert cv_rel_err(res.cv, [cf]) <= 1e-11
+
+
+# ---------------------------------------------------------------- P4
+@pytest.mark.parametrize("which", ["direct", "sorted"])
+def test_P4_two_points(which):
+    """n = 2: CV = (y1-y2)^2 if |x1-x2| in window, else 0."""
+    r = EVALS[which]([0.0, 1.0], [5.0, 2.0], [1.0, 2.0], E)
+    assert list(r.cv) == [0.0, 9.0] and list(r.neff) == [0, 2] and r.best == 0
+    r = EVALS[which]([0.0, 1.0], [5.0, 2.0], [1.0, 2.0], U)
+    assert list(r.cv) == [9.0, 9.0] and r.best == 0
+    r = EVALS[which]([0.0, 1.0], [5.0, 2.0], [0.5, 1.0], T)
+    assert list(r.cv) == [0.0, 0.0] and list(r.neff) == [0, 0]
+
+
+# ---------------------------------------------------------------- P5
+@pytest.mark.parametrize("which", ["direct", "sorted"])
+def test_P5_uniform_is_window_mean(which):
+    """Uniform kernel: g_{-i} = mean of the in-window neighbours (north_star)."""
+    x, y = workloads.draw_xy("sin_uniform", 300, 3)
+    h = workloads.grid_default(x, 12)
+    want = []
+    for hb in h:
+        tot = 0.0
+        for i in range(x.shape[0]):
+            mask = np.abs(x - x[i]) <= hb
+            mask[i] = False
+            if mask.any():
+                tot += (y[i] - y[mask].mean()) ** 2
+        want.append(tot / x.shape[0])
+    r = EVALS[which](x, y, h, U)
+    assert cv_rel_err(r.cv, want) <= 1e-13
+
+
+# ---------------------------------------------------------------- P6
+@pytest.mark.parametrize("k", KERNELS)
+def test_P6_invariances(k):
+    x, y = workloads.draw_xy("paper", 257, 11)
+    h = workloads.grid_default(x, 16)
+    base = oracle.cv_sorted(x, y, h, k)
+    # constant y -> CV identically 0 (exactly for a power-of-two constant,
+    # where y*w is exact; to rounding level otherwise)
+    assert np.all(oracle.cv_sorted(x, np.full_like(y, 4.0), h, k).cv == 0.0)
+    assert np.all(oracle.cv_direct(x, np.full_like(y, 4.0), h, k).cv == 0.0)
+    assert np.all(oracle.cv_sorted(x, np.full_like(y, 3.25), h, k).cv <= 1e-30)
+    # y -> 2^k y scales CV by 4^k exactly
+    r = oracle.cv_sorted(x, 8.0 * y, h, k)
+    assert np.array_equal(r.cv, base.cv * 64.0)
+    # (x, h) -> (2^k x, 2^k h): bit-identical
+    r = oracle.cv_sorted(x * 0.25, y, h * 0.25, k)
+    assert np.array_equal(r.cv, base.cv)
+    # y -> y + a: CV unchanged (LOO estimator is shift-equivariant)
+    r = oracle.cv_sorted(x, y + 1.0, h, k)
+    assert cv_rel_err(r.cv, base.cv) <= 1e-12
+    # permuting the (x_i, y_i) pairs changes nothing
+    p = np.random.default_rng(0).permutation(x.shape[0])
+    r = oracle.cv_direct(x[p], y[p], h, k)
+    assert cv_rel_err(r.cv, base.cv) <= 1e-14
+    assert np.array_equal(r.neff, base.neff)
+
+
+# ---------------------------------------------------------------- P7 / P8
+def _pairs_inside(x, hb, k):
+    xs = np.sort(x)
+    n = xs.shape[0]
+    cnt = 0
+    j = 0
+    for i in range(n):  # two-pointer over sorted x
+        if j < i + 1:
+            j = i + 1
+        while j < n and ((xs[j] - xs[i] <= hb) if k == U else (xs[j] - xs[i] < hb)):
+            j += 1
+        cnt += j - i - 1
+    return cnt
+
+
+@pytest.mark.parametrize("k", KERNELS)
+def test_P7_count_identity_and_P8_pair_symmetry(k):
+    x, y = workloads.draw_xy("lognormal", 400, 2)
+    x = np.concatenate([x, x[:7]])  # duplicated x values
+    y = np.concatenate([y, y[:7] + 1])
+    h = workloads.grid_log(x, 24)
+    r = oracle.cv_direct(x, y, h, k, aux=True)
+    n = x.shape[0]
+    D = np.abs(x[:, None] - x[None, :])
+    for b, hb in enumerate(h):
+        # P7: sum_i c_i = 2 #{i<j in window}, by an independent two-pointer pass
+        assert r.csum[b] == 2 * _pairs_inside(x, hb, k)
+        inside = (D <= hb) if k == U else (D < hb)
+        np.fill_diagonal(inside, False)
+        c = inside.sum(axis=1)
+        # P8: sum_i sum_{l in W_i} d^2 = 2 sum_{i<j in W} d^2; sum_i sum_{l in W_i} y_l = sum_j y_j c_j
+        iu = np.triu(inside, 1)
+        assert abs(r.sd2sum[b] - 2.0 * float(np.sum(D[iu] ** 2))) <= 1e-12 * max(1.0, r.sd2sum[b])
+        assert abs(r.sysum[b] - float(np.dot(y, c))) <= 1e-12 * max(1.0, abs(r.sysum[b]))
+        assert r.neff[b] == int(np.count_nonzero(c))
+    assert np.all(np.diff(r.neff) >= 0)  # nested windows: n_eff non-decreasing
+
+
+# ---------------------------------------------------------------- P9
+@pytest.mark.parametrize("k", KERNELS)
+def test_P9_long_double_vs_double(k):
+    x, y, h, _ = workloads.make("C2", seed=1, n=1500)
+    a = oracle.cv_sorted(x, y, h, k, precision="ld")
+    b = oracle.cv_sorted(x, y, h, k, precision="d")
+    assert oracle.real_bits("ld") > 64 or os.uname().machine != "x86_64"
+    assert cv_rel_err(b.cv, a.cv) <= 1e-12
+    assert np.array_equal(a.neff, b.neff)
+
+
+# ---------------------------------------------------------------- direct vs sorted
+@pytest.mark.parametrize("cfg,k", [("C1", U), ("C2", E), ("C5", E), ("C2", T), ("C5", U)])
+def test_direct_equals_sorted(cfg, k):
+    """The plain definition and the paper's algorithm agree (two independent
+    evaluators; the sorted one is the fast oracle used at large n)."""
+    x, y, h, _ = workloads.make(cfg, seed=7, n=700)
+    a = oracle.cv_direct(x, y, h, k)
+    b = oracle.cv_sorted(x, y, h, k)
+    assert cv_rel_err(b.cv, a.cv) <= 1e-13
+    assert np.array_equal(a.neff, b.neff)
+    assert a.best == b.best
+
+
+# ---------------------------------------------------------------- P10
+@pytest.mark.parametrize("cfg,n,k,tol", [("C1", 1000, U, 1e-12), ("C2", 4000, E, 1e-11),
+                                          ("C5", 3000, E, 1e-10), ("C3", 3000, T, 1e-11)])
+def test_P10_window_prefix_checker(cfg, n, k, tol):
+    x, y, h, _ = workloads.make(cfg, seed=0, n=n)
+    a = oracle.cv_sorted(x, y, h, k)
+    w = window.cv_window(x, y, h, k)
+    assert cv_rel_err(a.cv, w["cv"]) <= tol
+    assert np.array_equal(a.neff, w["neff"])
+    assert a.best == w["best"]
+
+
+# ---------------------------------------------------------------- Q14 guard
+@pytest.mark.parametrize("yv", [(3.0, 5.0), (0.1, 7.0), (5.0, 0.125)])
+def test_Q14_edge_cancellation_guard(yv):
+    """One neighbour at d = nextafter(h, 0): the decomposition h^2 c - sum d^2
+    cancels to nothing; the guarded sweep must return g = y_l exactly."""
+    h = 1.0
+    x = np.array([0.0, np.nextafter(1.0, 0.0)])
+    y = np.array(yv)
+    want = float((Fraction(y[0]) - Fraction(y[1])) ** 2)
+    for which in EVALS:
+        r = EVALS[which](x, y, [h], E)
+        assert abs(r.cv[0] - want) <= math.ulp(want) and r.neff[0] == 2
+        r = EVALS[which](x, y, [h], T)
+        assert abs(r.cv[0] - want) <= math.ulp(want)
+
+
+# ---------------------------------------------------------------- P11 (seed-0 configs)
+def test_P11_C1_seed0():
+    """C1 seed 0: best b=4, CV=0.26568957122597 (two evaluators there)."""
+    x, y, h, k = workloads.make("C1", seed=0)
+    r = oracle.cv_direct(x, y, h, k)
+    assert r.best == 4
+    assert abs(r.cv[4] - 0.2656895712259686) <= 1e-9 * 0.2656895712259686
+    assert best_ok(r.best, r.cv)
+    assert np.all(r.neff == x.shape[0])
+
+
+def test_P11_C2_seed0_window_checker():
+    """C2 seed 0: best b=1, CV=0.020828858781022."""
+    x, y, h, k = workloads.make("C2", seed=0)
+    w = window.cv_window(x, y, h, k)
+    assert w["best"] == 1
+    assert abs(w["cv"][1] - 0.020828858781022) <= 1e-9 * 0.0208
+
+
+# ---------------------------------------------------------------- grid, finalize, errors
+def test_default_grid():
+    """§IV P@16146-16375: max = range, min = range/m, evenly spaced; recipe
+    h_b = r*((b+1)/m) agrees bitwise with the workload generator."""
+    x, _ = workloads.draw_xy("sin_uniform", 1000, 0)
+    for m in (1, 3, 100, 1000):
+        h = oracle.default_grid(x, m)
+        r = x.max() - x.min()
+        assert h[-1] == r
+        assert np.array_equal(h, workloads.grid_default(x, m))
+        for b in range(m):
+            exact_v = Fraction(r) * (b + 1) / m
+            assert abs(Fraction(h[b]) - exact_v) <= 2 * Fraction(math.ulp(h[b]))  # two roundings
+    with pytest.raises(oracle.OracleError) as ei:
+        oracle.default_grid(np.ones(5), 4)
+    assert ei.value.status == 5
+
+
+@pytest.mark.parametrize("bad,code", [
+    (dict(x=[0.0]), 1),
+    (dict(kernel=7), 2),
+    (dict(h=[0.5, 0.25]), 3),
+    (dict(h=[0.0, 1.0]), 3),
+    (dict(h=[math.inf]), 3),
+    (dict(x=[0.0, math.nan, 1.0]), 4),
+    (dict(y=[0.0, math.inf, 1.0]), 4),
+])
+def test_validation_codes(bad, code):
+    args = dict(x=[0.0, 0.5, 1.0], y=[1.0, 2.0, 3.0], h=[0.5, 1.0], kernel=E)
+    args.update(bad)
+    if len(args["y"]) != len(args["x"]):
+        args["y"] = args["y"][: len(args["x"])] + [0.0] * (len(args["x"]) - len(args["y"]))
+    for which in EVALS:
+        with pytest.raises(oracle.OracleError) as ei:
+            EVALS[which](args["x"], args["y"], args["h"], args["kernel"])
+        assert ei.value.status == code
+
+
+def test_best_rule_ties_and_nan():
+    cv, best = oracle.finalize(np.array([3.0, 1.0, 1.0, 2.0]), 1)
+    assert best == 1
+    cv, best = oracle.finalize(np.array([math.nan, 2.0, 1.0]), 1)
+    assert best == 2
+
+
+@pytest.mark.parametrize("P", [2, 3, 7])
+def test_shard_partials_add_up(P):
+    """Shards of the x-sorted row order partition the rows."""
+    x, y, h, k = workloads.make("C5", seed=3, n=900)
+    full = oracle.cv_sorted(x, y, h, k)
+    S = np.zeros(h.shape[0]); ne = np.zeros(h.shape[0], np.int64)
+    for r in range(P):
+        part = oracle.cv_sorted(x, y, h, k, rows=oracle.shard_rows(x, r, P))
+        S += part.S; ne += part.neff
+    assert np.array_equal(ne, full.neff)
+    assert cv_rel_err(S, full.S) <= 1e-14
+    cv, best = oracle.finalize(S, x.shape[0])
+    assert best_ok(best, full.cv)
