@@ -1,0 +1,391 @@
+#!/usr/bin/env python
+"""Benchmark: LOO-CV bandwidth grid search (Rohlfs & Zahran 2017) on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl ours|reference]
+
+A "step" is one full grid search (every SURVEY.md §8(a) row: pack, sort,
+sweep + LOO emit, reduce, [all-reduce], finalize/arg-min) over the config's
+synthetic input, inputs resident in HBM.  Prints ONE JSON line (rank 0).
+
+Metric (BASELINE.json): pair-bandwidth CV evaluations per second,
+n (n-1) m / T_step, plus the wall time per full grid search (e2e).
+For N > 1 (torchrun) rows are sharded across ranks with one NCCL all-reduce
+of the 2m+2 partial vector; the job is fixed (strong scaling); time is the
+max over ranks of CUDA-event time.
+
+--impl reference times the CPU oracle (the paper's Program-3 algorithm,
+oracle/kr_oracle.c) on the host cores on a bounded row sample of the same
+workload (this tier's reference arm; there is no reference code).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import workloads  # noqa: E402
+
+METRIC = json.load(open(os.path.join(ROOT, "BASELINE.json")))["metric"]
+UNIT = "pair·bandwidth evals/s"
+SM_COUNT = 148
+FP64_LANES_PER_SM = 64          # FP64 FMA lanes per SM per clock
+SM_MAX_MHZ_NOMINAL = 1965.0     # B200 clocks.max.sm (B200_PROFILING.md)
+# Algorithmic FP64 flops (FMA = 2) per ordered pair and per (row, bandwidth)
+# emit, per kernel.
+FLOPS_PER_PAIR = {0: 2, 1: 6, 2: 5}
+FLOPS_PER_EMIT = {0: 4, 1: 9, 2: 9}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="C2", choices=sorted(workloads.CONFIGS))
+    ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=8.0,
+                    help="target wall seconds of the bounded oracle sample")
+    return ap.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def workload_desc(cfg, seed):
+    kname = workloads.KERNEL_NAMES[cfg.kernel]
+    return (f"{cfg.name}: n={cfg.n}, m={cfg.m} ({cfg.grid} grid), {kname} kernel, "
+            f"x~{cfg.x_dist}, seed {seed}")
+
+
+# --------------------------------------------------------------------- clocks
+class ClockSampler:
+    """Samples SM clock and throttle reasons through NVML during the timed region."""
+
+    REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+        0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+        0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
+    }
+
+    def __init__(self, index: int):
+        self.samples, self.reasons = [], 0
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self.ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover - no NVML
+            self.err = str(e)
+
+    def _run(self):
+        nv = self.nv
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                self.reasons |= int(r) & ~0x1
+            except Exception:
+                pass
+            time.sleep(0.002)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+            time.sleep(0.01)
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+
+    def summary(self):
+        if not self.ok:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml_unavailable"]}
+        names = [v for k, v in self.REASONS.items() if self.reasons & k]
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": names, "samples": len(self.samples)}
+
+
+# --------------------------------------------------------------- cpu oracle
+def oracle_sample(x, y, h, k, target_s: float):
+    """Time the oracle (Program-3 algorithm) on a bounded row sample of the
+    workload; returns (pair_bw_per_s, seconds, rows, threads)."""
+    import oracle
+
+    n, m = x.shape[0], h.shape[0]
+    order = oracle.sorted_rows(x)
+    threads = oracle.num_threads()
+    rows = max(2 * threads, 16)
+    t0 = time.perf_counter()
+    oracle.cv_sorted(x, y, h, k, rows=order[:rows])
+    dt = time.perf_counter() - t0
+    per_row = dt / rows
+    rows = int(min(n, max(rows, target_s / max(per_row, 1e-9))))
+    stride = max(1, n // rows)
+    sample = order[::stride][:rows]  # spread over the sorted order
+    t0 = time.perf_counter()
+    oracle.cv_sorted(x, y, h, k, rows=sample)
+    dt = time.perf_counter() - t0
+    return sample.shape[0] * (n - 1) * m / dt, dt, int(sample.shape[0]), threads
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+# ------------------------------------------------------------ reference arm
+def run_reference(args):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return 0
+    cfg = workloads.CONFIGS[args.config]
+    x, y, h, k = workloads.make(cfg, seed=args.seed)
+    n, m = x.shape[0], h.shape[0]
+    per_step_target = max(0.5, min(args.cpu_seconds, 120.0 / max(1, args.steps + args.warmup)))
+    vals, secs, rows = [], [], 0
+    threads = 1
+    for s in range(args.warmup + args.steps):
+        v, dt, rows, threads = oracle_sample(x, y, h, k, per_step_target)
+        if s >= args.warmup:
+            vals.append(v)
+            secs.append(dt)
+    value = statistics.median(vals)
+    full_search_s = n * (n - 1) * m / value
+    sample = (f"kro_cv_sorted (long double, per-row qsort + sweep) on {rows} of {n} rows "
+              f"(strided over the x-sorted order), {threads} OpenMP threads; value extrapolated "
+              f"to the full job; {cpu_model()}")
+    out = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * full_search_s,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f80",
+        "data": "synthetic",
+        "config": {"workload": workload_desc(cfg, args.seed), "n": n, "m": m,
+                   "kernel": workloads.KERNEL_NAMES[k], "seed": args.seed},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "wall_s_per_full_search_extrapolated": full_search_s,
+    }
+    print(json.dumps(out), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ our arm
+def run_ours(args):
+    import torch
+
+    rank, world, local = dist_env()
+    if world != args.gpus:
+        if world == 1 and args.gpus > 1:
+            raise SystemExit("--gpus N>1 must be launched with torchrun (one rank per GPU)")
+    if not torch.cuda.is_available():
+        raise SystemExit("bench.py needs a CUDA device")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+    from paper_conf_ipps_rohlfsz17_b200 import krcv
+    from paper_conf_ipps_rohlfsz17_b200.api import GridSearch
+
+    cfg = workloads.CONFIGS[args.config]
+    x, y, h, k = workloads.make(cfg, seed=args.seed)
+    n, m = x.shape[0], h.shape[0]
+    units = n * (n - 1) * m  # pair-bandwidth evaluations of one full grid search
+
+    d_x = torch.as_tensor(x, device=dev)
+    d_y = torch.as_tensor(y, device=dev)
+    plan = GridSearch(n, h, k, device=dev, rank=rank, world=world)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+    stream = torch.cuda.current_stream(dev)
+
+    def barrier():
+        if world > 1:
+            torch.distributed.barrier()
+
+    for _ in range(args.warmup):
+        plan.run(d_x, d_y)
+    r = plan.result()
+    torch.cuda.synchronize()
+
+    # ---- device-timed steps (value); L2 flushed between steps, outside the events
+    krcv.kr_profile_enable(True)
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    sweep_ms, sort_ms = [], []
+    launches = 0
+    barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        for s in range(args.steps):
+            flush.fill_(s & 0xFF)
+            starts[s].record(stream)
+            plan.run(d_x, d_y)
+            ends[s].record(stream)
+            a, b, _c = krcv.kr_profile_read()  # syncs on this step's events
+            sort_ms.append(a)
+            sweep_ms.append(b)
+            launches += krcv.kr_launch_count() + 1  # + finalize kernel
+        torch.cuda.synchronize()
+    barrier()
+    krcv.kr_profile_enable(False)
+    step_ms = [starts[s].elapsed_time(ends[s]) for s in range(args.steps)]
+    total_ms = sum(step_ms)
+    if world > 1:
+        t = torch.tensor([total_ms, sum(sweep_ms)], dtype=torch.float64, device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        total_ms, sweep_total = float(t[0]), float(t[1])
+    else:
+        sweep_total = sum(sweep_ms)
+    res = plan.result()
+    value = units * args.steps / (total_ms * 1e-3)
+
+    # ---- end-to-end through the public API, host buffers, H2D/D2H inside
+    e2e = e2e_measure(args, x, y, h, k, n, m, units, dev, rank, world, plan)
+
+    # ---- roofline of the dominant kernel (sweep)
+    fl_pair, fl_emit = FLOPS_PER_PAIR[k], FLOPS_PER_EMIT[k]
+    rows_mine = ((rank + 1) * n) // world - (rank * n) // world
+    flops_per_launch = rows_mine * (n - 1) * fl_pair + rows_mine * m * fl_emit
+    sweep_avg_s = (sweep_total / args.steps) * 1e-3
+    peak = SM_COUNT * FP64_LANES_PER_SM * 2 * SM_MAX_MHZ_NOMINAL * 1e6 / 1e12  # TFLOP/s
+    achieved = flops_per_launch / sweep_avg_s / 1e12
+    traffic = None
+    ncu_json = os.path.join(ROOT, "profiles", "sweep_ncu.json")
+    if os.path.exists(ncu_json):
+        try:
+            prof = json.load(open(ncu_json)).get(args.config)
+            if prof:
+                traffic = prof.get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+
+    out = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": workload_desc(cfg, args.seed), "n": n, "m": m,
+                   "kernel": workloads.KERNEL_NAMES[k], "seed": args.seed,
+                   "parallelism": f"row-shard x{world}" + (" + nccl all_reduce(2m+2 fp64)" if world > 1 else ""),
+                   "l2": "flushed between timed steps (256 MiB write, outside the events)"},
+        "roofline": {"bound": "alu", "kernel": "sweep_kernel (a3+a4)", "achieved": achieved,
+                     "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak, "traffic": traffic,
+                     "peak_note": "FP64: 148 SM x 64 FMA lanes x 2 flop x 1965 MHz (derived, DESIGN.md)",
+                     "flops_per_launch": flops_per_launch, "sweep_ms": sweep_total / args.steps,
+                     "sweep_share_of_step": (sweep_total / args.steps) / (total_ms / args.steps)},
+        "stage_ms": {"pack_sort_gather": sum(sort_ms) / args.steps, "sweep": sum(sweep_ms) / args.steps},
+        "result": {"best": res.best, "h_best": float(h[res.best]), "cv_best": float(res.cv[res.best])},
+        "e2e": e2e,
+        "clocks": clk.summary(),
+        "gpu_launches": launches,
+        "wall_time_per_grid_search_ms": e2e.get("ms_per_search"),
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        v, dt, rows, threads = oracle_sample(x, y, h, k, args.cpu_seconds)
+        out["cpu_baseline"] = {
+            "value": v, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "sample": (f"kro_cv_sorted on {rows} of {n} rows (strided over the x-sorted order), "
+                       f"{dt:.1f} s, {threads} OpenMP threads, {cpu_model()}; extrapolated to the full job")}
+    if world > 1:
+        torch.distributed.barrier()
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        torch.distributed.destroy_process_group()
+    return 0
+
+
+def e2e_measure(args, x, y, h, k, n, m, units, dev, rank, world, plan):
+    """Same metric through the public API from pinned host buffers, per step:
+    H2D of x, y (and h), the grid search, D2H of the CV curve and best."""
+    import ctypes
+
+    import torch
+
+    from paper_conf_ipps_rohlfsz17_b200 import krcv
+
+    hx = torch.from_numpy(x).pin_memory()
+    hy = torch.from_numpy(y).pin_memory()
+    hh = torch.from_numpy(h).pin_memory()
+    hcv = torch.empty(m, dtype=torch.float64).pin_memory()
+    times = []
+    if world == 1:
+        best = ctypes.c_int32(-1)
+        for s in range(args.warmup + args.steps):
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            st = krcv.kr_cv_grid_ptr(hx.data_ptr(), hy.data_ptr(), n, hh.data_ptr(), m, k, hcv.data_ptr(),
+                                     ctypes.byref(best))
+            t1 = time.perf_counter()
+            if st != 0:
+                raise krcv.KrcvError(st, "kr_cv_grid")
+            if s >= args.warmup:
+                times.append(t1 - t0)
+        api = "kr_cv_grid (C-ABI, host pointers, synchronous)"
+        d2h = 8 * m + 8
+    else:
+        d_x = torch.empty(n, dtype=torch.float64, device=dev)
+        d_y = torch.empty(n, dtype=torch.float64, device=dev)
+        for s in range(args.warmup + args.steps):
+            torch.distributed.barrier()
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            d_x.copy_(hx, non_blocking=True)
+            d_y.copy_(hy, non_blocking=True)
+            plan.run(d_x, d_y)
+            hcv.copy_(plan.cv, non_blocking=True)
+            bs = plan.best_status.cpu()
+            t1 = time.perf_counter()
+            if int(bs[1]) != 0:
+                raise krcv.KrcvError(int(bs[1]), "device status")
+            if s >= args.warmup:
+                times.append(t1 - t0)
+        t = torch.tensor([sum(times)], dtype=torch.float64, device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        times = [float(t[0]) / len(times)] * len(times)
+        api = "GridSearch.run (row-sharded, NCCL all-reduce) with pinned H2D/D2H per step"
+        d2h = 8 * m + 8
+    tot = sum(times)
+    return {"value": units * len(times) / tot, "unit": UNIT, "h2d_bytes_per_step": 16 * n + 8 * m,
+            "d2h_bytes_per_step": d2h, "ms_per_search": 1e3 * tot / len(times), "api": api,
+            "timing": "host wall clock around the synchronous call"}
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

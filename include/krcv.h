@@ -1,0 +1,180 @@
+/*
+ * krcv.h -- C-ABI of the B200-native leave-one-out cross-validation
+ * bandwidth grid search for univariate Nadaraya-Watson regression
+ * (Rohlfs & Zahran, "Optimal Bandwidth Selection for Kernel Regression Using
+ * a Fast Grid Search and a GPU", IPDPSW 2017).
+ *
+ * Citations are P@<char offset> into the single-line reference PAPER.md
+ * (SURVEY.md §0).
+ *
+ * What is computed (§III):
+ *   Eq.(1) P@11484  CV(h) = n^-1 sum_i (Y_i - g_{-i}(X_i))^2 M(X_i)
+ *   Eq.(2) P@11694  g_{-i}(X_i) = sum_{l!=i} Y_l K((X_i-X_l)/h) / sum_{l!=i} K((X_i-X_l)/h)
+ *          P@11802  M(X_i) = 1 iff the denominator of (2) is non-zero
+ *   Eq.(3) P@11971  Epanechnikov K(u) = 0.75 (1-u^2) I{|u|<=1}
+ *   fn.1   P@18521  uniform K = 1/2 I{|u|<=1}, triangular K = (1-|u|) I{|u|<1}
+ * for every bandwidth h_b of a non-decreasing grid, then the arg-min
+ * (§IV.B P@23454-26269; footnote 2 P@25449: return the index).
+ *
+ * Conventions:
+ *   - Window membership is decided in IEEE binary64 on d = |x_l - x_i|:
+ *     d < h for Epanechnikov / triangular, d <= h for uniform (Q1).
+ *   - M_i = 1 iff at least one l != i is in the window (Q6).  Rows with
+ *     M_i = 0 contribute 0 and CV divides by n (Eq.(1) literally, Q7).
+ *   - Leave-one-out excludes index i only; duplicates of x_i stay (Q8).
+ *   - best = smallest b whose CV equals the minimum; NaN is never minimal (Q11).
+ *   - Arithmetic is fp64 (the paper's fp32, P@19633, misses 1e-6 parity).
+ *   - Indices are 0-based.  The grid must be finite, > 0, non-decreasing;
+ *     duplicates are allowed (equal CV, lower index wins).  No 2,048 cap
+ *     (the paper's cap is a constant-memory artefact, P@20037).
+ *
+ * Ownership: the caller owns every buffer.  The library keeps no pointer to
+ * caller memory after a call returns (async calls: until the enqueued stream
+ * work completes).  Outputs are written only when a call returns KR_OK
+ * (async calls: see the status slots of the partial vector).
+ *
+ * Threading: every entry point is re-entrant.  kr_cv_grid serialises on a
+ * per-device context (lazily created workspace + stream) guarded by a mutex.
+ */
+#ifndef KRCV_H
+#define KRCV_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Kernel functions K (Eq.(3), footnote 1 P@18521). */
+enum {
+    KR_UNIFORM = 0,
+    KR_EPANECHNIKOV = 1,
+    KR_TRIANGULAR = 2
+};
+
+/* Status codes returned by every int-valued entry point. */
+enum {
+    KR_OK = 0,
+    KR_EARG = 1,        /* null pointer, n < 2, n > INT32_MAX, m < 1, m > KR_MAX_M,
+                           bad shard/nshards, workspace too small */
+    KR_EKERNEL = 2,     /* unknown kernel id */
+    KR_EGRID = 3,       /* h non-finite, h <= 0, or decreasing */
+    KR_ENONFINITE = 4,  /* NaN / Inf in x or y */
+    KR_EDEGENERATE = 5, /* default grid requested with max(x) == min(x) */
+    KR_ENOMEM = 6,      /* device or host allocation failed */
+    KR_ECUDA = 7        /* any other CUDA runtime error (see kr_last_cuda_error) */
+};
+
+#define KR_MAX_M 65536
+
+/* Length of the partial vector of the device path: [ S[0..m) | neff[0..m) |
+ * n_bad_grid | n_nonfinite ].  S[b] = sum over the shard's rows of
+ * M_i (y_i - g_{-i}(h_b))^2, neff[b] = sum of M_i (exact in fp64), and two
+ * status counters.  All entries add under an all-reduce(SUM) across shards. */
+#define KR_PARTIAL_LEN(m) (2 * (int64_t)(m) + 2)
+
+/*
+ * kr_cv_grid -- the whole grid search on the current CUDA device, host
+ * pointers, synchronous.  (BASELINE.json north_star signature.)
+ *   x, y     [n] fp64 host arrays (any order; any pageable or pinned memory)
+ *   h_grid   [m] fp64 host, non-decreasing, finite, > 0
+ *   kernel   KR_UNIFORM | KR_EPANECHNIKOV | KR_TRIANGULAR
+ *   cv_out   [m] host: CV(h_b) per Eq.(1) (already divided by n)
+ *   best_out host: smallest arg-min index
+ * Errors: KR_EARG, KR_EKERNEL, KR_EGRID, KR_ENONFINITE (validated on the host
+ * before any device work), KR_ENOMEM, KR_ECUDA.  Outputs untouched on error.
+ */
+int kr_cv_grid(const double *x, const double *y, int64_t n,
+               const double *h_grid, int32_t m, int32_t kernel,
+               double *cv_out, int32_t *best_out);
+
+/* kr_cv_grid plus the per-bandwidth count of rows with M_i = 1
+ * (neff_out [m] int64, nullable). */
+int kr_cv_grid_ex(const double *x, const double *y, int64_t n,
+                  const double *h_grid, int32_t m, int32_t kernel,
+                  double *cv_out, int64_t *neff_out, int32_t *best_out);
+
+/* Host-side grid check (finite, > 0, non-decreasing, 1 <= m <= KR_MAX_M). */
+int kr_validate_grid(const double *h_grid, int32_t m);
+
+/* Device workspace size in bytes for kr_cv_shard_async at (n, m).  Returns 0
+ * for invalid (n, m).  Requires a CUDA device (the radix-sort scratch size
+ * is queried from the runtime). */
+size_t kr_workspace_bytes(int64_t n, int32_t m);
+
+/*
+ * kr_cv_shard_async -- device path for caller-owned device memory and row
+ * sharding.  Enqueues on `cuda_stream` (a cudaStream_t; NULL = legacy default
+ * stream) and returns without synchronising; capturable in a CUDA graph.
+ *   d_x, d_y     [n] fp64 DEVICE arrays, unsorted; every shard sees all n
+ *   d_h          [m] fp64 DEVICE grid (validate it on the host first with
+ *                kr_validate_grid; it is re-checked on the device and a bad
+ *                grid is reported through the n_bad_grid slot)
+ *   shard, nshards  rows [floor(shard*n/nshards), floor((shard+1)*n/nshards))
+ *                of the x-sorted order (stable: ties by original index)
+ *   d_partial    [KR_PARTIAL_LEN(m)] fp64 DEVICE output, fully overwritten
+ *   d_workspace  >= kr_workspace_bytes(n, m) bytes of device memory, 256-B aligned
+ * Host-checked errors (returned): KR_EARG, KR_EKERNEL, KR_ECUDA (launch).
+ * Device-detected errors (non-finite x/y, bad device grid) are counted in the
+ * status slots and turned into KR_ENONFINITE / KR_EGRID by kr_finalize.
+ */
+int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n,
+                      const double *d_h, int32_t m, int32_t kernel,
+                      int32_t shard, int32_t nshards,
+                      double *d_partial, void *d_workspace, size_t workspace_bytes,
+                      void *cuda_stream);
+
+/*
+ * kr_finalize -- host finalize of a partial vector already summed over all
+ * shards: cv_out[b] = S[b]/n, neff_out[b] = neff[b] (nullable), best_out per
+ * Q11.  Returns KR_EGRID / KR_ENONFINITE if the status slots are non-zero.
+ */
+int kr_finalize(const double *partial, int64_t n, int32_t m,
+                double *cv_out, int64_t *neff_out, int32_t *best_out);
+
+/*
+ * kr_finalize_async -- the same on the device (one CTA; the paper's
+ * min-reduction kernel, P@24653): d_cv [m] fp64, d_neff [m] int64 (nullable),
+ * d_best int32, d_status int32 (KR_OK / KR_EGRID / KR_ENONFINITE).
+ */
+int kr_finalize_async(const double *d_partial, int64_t n, int32_t m,
+                      double *d_cv, int64_t *d_neff, int32_t *d_best, int32_t *d_status,
+                      void *cuda_stream);
+
+/*
+ * kr_default_grid -- §IV P@16146-16375: max = range of x, min = range/m,
+ * evenly spaced; h_b = r * ((double)(b+1)/m), r = max(x) - min(x), so the
+ * last point is exactly r (reading Q9).  Host pointers.
+ * Errors: KR_EARG, KR_ENONFINITE, KR_EDEGENERATE (r == 0).
+ */
+int kr_default_grid(const double *x, int64_t n, int32_t m, double *h_out);
+
+/* Static message for a status code (never NULL). */
+const char *kr_strerror(int status);
+
+/* The last CUDA runtime error string seen by this thread ("" if none). */
+const char *kr_last_cuda_error(void);
+
+/*
+ * Optional stage timing for benchmarks (thread-local state).
+ * kr_profile_enable(1): subsequent kr_cv_shard_async calls on this thread
+ * record CUDA events on their stream around (a1+a2) pack+sort+gather,
+ * (a3+a4) sweep and (a5) reduce.  Do not enable while capturing a graph.
+ * kr_profile_read waits for the last call's events and writes ms[3]
+ * = {sort, sweep, reduce} in milliseconds; returns KR_EARG if nothing was
+ * recorded.  kr_launch_count returns the number of kernel launches the last
+ * kr_cv_shard_async call on this thread enqueued (CUB passes included).
+ */
+int kr_profile_enable(int on);
+int kr_profile_read(float *ms);
+int64_t kr_launch_count(void);
+
+/* Library version, e.g. "krcv 0.1.0 sm_100a". */
+const char *kr_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* KRCV_H */

@@ -1,0 +1,100 @@
+"""Python-level API over the C-ABI: single- and multi-GPU grid search.
+
+PyTorch supplies device memory (caching allocator), streams and the process
+group; the computation is the C-ABI's (libkrcv.so).  Row sharding follows
+SURVEY.md §8(e): rank r of P sweeps sorted rows [floor(r n/P), floor((r+1) n/P)),
+then ONE all-reduce(SUM) of the partial vector [S | neff | status] (2m+2
+fp64) over NCCL, then every rank finalizes identically on its device.
+"""
+from __future__ import annotations
+
+import dataclasses
+
+import numpy as np
+
+from . import krcv
+
+
+@dataclasses.dataclass
+class CVResult:
+    cv: "object"       # torch.Tensor float64 [m] (device) or np.ndarray
+    neff: "object"     # int64 [m]
+    best: int
+    h: np.ndarray
+
+    @property
+    def h_best(self) -> float:
+        return float(self.h[self.best])
+
+
+class GridSearch:
+    """Reusable device plan for one (n, m, kernel) on one GPU / one rank.
+
+    ``run(x, y)`` enqueues: sharded pipeline -> (all-reduce) -> device
+    finalize, on the current stream; nothing synchronises until ``result()``.
+    """
+
+    def __init__(self, n: int, h, kernel="epanechnikov", device=None, rank: int = 0, world: int = 1,
+                 group=None):
+        import torch
+
+        self.torch = torch
+        self.device = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+        h_host = np.ascontiguousarray(h, dtype=np.float64)
+        st = krcv.kr_validate_grid(h_host)
+        if st != krcv.KR_OK:
+            raise krcv.KrcvError(st, "grid")
+        self.n, self.m = int(n), int(h_host.shape[0])
+        self.kernel = krcv._kernel_id(kernel)
+        self.rank, self.world, self.group = int(rank), int(world), group
+        self.h = h_host
+        self.d_h = torch.as_tensor(h_host, device=self.device)
+        self._ws_raw = krcv.workspace(self.n, self.m, self.device)
+        self.ws = krcv.aligned(self._ws_raw)
+        self.partial = torch.empty(krcv.partial_len(self.m), dtype=torch.float64, device=self.device)
+        self.cv = torch.empty(self.m, dtype=torch.float64, device=self.device)
+        self.neff = torch.empty(self.m, dtype=torch.int64, device=self.device)
+        self.best_status = torch.empty(2, dtype=torch.int32, device=self.device)
+
+    def run(self, d_x, d_y) -> None:
+        if d_x.numel() != self.n or d_y.numel() != self.n:
+            raise ValueError("x, y must have n elements")
+        krcv.kr_cv_shard_async(d_x, d_y, self.d_h, self.kernel, self.rank, self.world, self.partial, self.ws)
+        if self.world > 1:
+            import torch.distributed as dist
+
+            dist.all_reduce(self.partial, op=dist.ReduceOp.SUM, group=self.group)
+        krcv.kr_finalize_async(self.partial, self.n, self.m, self.cv, self.neff, self.best_status)
+
+    def result(self) -> CVResult:
+        bs = self.best_status.cpu()
+        st = int(bs[1])
+        if st != krcv.KR_OK:
+            raise krcv.KrcvError(st, "device status")
+        return CVResult(cv=self.cv, neff=self.neff, best=int(bs[0]), h=self.h)
+
+
+def cv_grid(x, y, h=None, m: int | None = None, kernel="epanechnikov", device=None, distributed: bool = False,
+            group=None) -> CVResult:
+    """LOO-CV grid search.  x, y: numpy arrays or CUDA tensors; h: grid array,
+    or None with m for the default grid (§IV P@16146).  With distributed=True
+    every rank of the default (or given) process group must call it with the
+    same inputs; the result is identical on every rank."""
+    import torch
+
+    if h is None:
+        if m is None:
+            raise ValueError("give h or m")
+        xh = x.detach().cpu().numpy() if torch.is_tensor(x) else np.asarray(x, np.float64)
+        h = krcv.kr_default_grid(xh, int(m))
+    rank, world = 0, 1
+    if distributed:
+        import torch.distributed as dist
+
+        rank, world = dist.get_rank(group), dist.get_world_size(group)
+    dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+    d_x = torch.as_tensor(x, dtype=torch.float64, device=dev).contiguous()
+    d_y = torch.as_tensor(y, dtype=torch.float64, device=dev).contiguous()
+    plan = GridSearch(d_x.numel(), h, kernel, dev, rank, world, group)
+    plan.run(d_x, d_y)
+    return plan.result()

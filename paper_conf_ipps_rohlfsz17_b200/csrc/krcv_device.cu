@@ -1,0 +1,493 @@
+// krcv_device.cu -- sm_100a kernels of the LOO-CV bandwidth grid search and
+// the device half of the C-ABI (kr_workspace_bytes, kr_cv_shard_async,
+// kr_finalize_async).  See include/krcv.h and DESIGN.md.
+//
+// Hot path, one pass per call:
+//   a1 pack      x -> order-preserving uint64 key, index; validity counters
+//   a2 sort      CUB onesweep radix sort of (key, index), stable; gather (x,y)
+//   a3 sweep     per sorted row: fused distance + window test + running sums,
+//                bandwidths ascending (§III P@14010-14984,
+//                §IV.B P@21154-22104), realised on the globally sorted array:
+//                row i's right neighbours i+1, i+2, ... and left neighbours
+//                i-1, i-2, ... are already in increasing |x_l - x_i| order.
+//   a4 emit      LOO estimate Eq.(2), M, squared error Eq.(1) per (row, h_b)
+//   a5 reduce    per-warp-tile partials -> fixed-order column sums -> partial
+// All arithmetic fp64; no tensor cores (not a contraction).
+#include <cuda_runtime.h>
+#include <cub/device/device_radix_sort.cuh>
+
+#include <cmath>
+#include <cstdint>
+
+#include "krcv.h"
+#include "krcv_internal.h"
+
+namespace krcv {
+
+// ---------------------------------------------------------------------------
+// a1: pack + device-side validation
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t order_key(double v)
+{
+    // IEEE-754 total order on non-NaN values as an unsigned integer.
+    uint64_t u = static_cast<uint64_t>(__double_as_longlong(v));
+    return (u & 0x8000000000000000ull) ? ~u : (u | 0x8000000000000000ull);
+}
+
+__global__ void pack_kernel(const double *__restrict__ x, const double *__restrict__ y, int n,
+                            const double *__restrict__ h, int m,
+                            uint64_t *__restrict__ keys, uint32_t *__restrict__ vals,
+                            unsigned *__restrict__ status)
+{
+    const int stride = gridDim.x * blockDim.x;
+    const int tid = blockIdx.x * blockDim.x + threadIdx.x;
+    unsigned bad = 0, gbad = 0;
+    for (int i = tid; i < n; i += stride) {
+        double xv = x[i], yv = y[i];
+        bad += (!isfinite(xv) || !isfinite(yv)) ? 1u : 0u;
+        keys[i] = order_key(xv);
+        vals[i] = static_cast<uint32_t>(i);
+    }
+    for (int b = tid; b < m; b += stride) {
+        double hb = h[b];
+        gbad += (!isfinite(hb) || !(hb > 0.0) || (b > 0 && hb < h[b - 1])) ? 1u : 0u;
+    }
+    if (bad) atomicAdd(&status[1], bad);
+    if (gbad) atomicAdd(&status[0], gbad);
+}
+
+// a2 (second half): gather (x, y) into sorted order as one 16-byte record.
+__global__ void gather_kernel(const double *__restrict__ x, const double *__restrict__ y,
+                              const uint32_t *__restrict__ order, int n, double2 *__restrict__ xy)
+{
+    const int stride = gridDim.x * blockDim.x;
+    for (int k = blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+        uint32_t i = order[k];
+        xy[k] = make_double2(x[i], y[i]);
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a3 + a4: the sweep
+// ---------------------------------------------------------------------------
+template <int KERN>
+__device__ __forceinline__ bool inside(double d, double h)
+{
+    // Q1: open window for Epanechnikov / triangular, closed for uniform.
+    return KERN == KR_UNIFORM ? (d <= h) : (d < h);
+}
+
+// Running sums of one row.  Epanechnikov: sum y, sum d^2, sum y d^2 (§III
+// P@14010; the count comes from the pointers, reading Q3).  Triangular: sum y,
+// sum d, sum y d.  Uniform: sum y.
+struct Sums {
+    double sy, s1, sy1;
+};
+
+template <int KERN>
+__device__ __forceinline__ void acc(Sums &s, double yv, double d)
+{
+    s.sy += yv;
+    if (KERN == KR_EPANECHNIKOV) {
+        double d2 = d * d;
+        s.s1 += d2;
+        s.sy1 = fma(yv, d2, s.sy1);
+    } else if (KERN == KR_TRIANGULAR) {
+        s.s1 += d;
+        s.sy1 = fma(yv, d, s.sy1);
+    }
+}
+
+__device__ __forceinline__ double warp_sum(double v)
+{
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+constexpr int kSweepWarps = 4;
+constexpr int kSweepThreads = kSweepWarps * 32;
+
+// One warp = 32 consecutive sorted rows (one per lane); bandwidths ascend in
+// lock-step across the warp (warp-uniform b).  Per (tile, b) the warp writes
+// sum M e^2 and sum M to tileS/tileN[b][tile]; nothing per pair is stored.
+template <int KERN>
+__global__ void __launch_bounds__(kSweepThreads)
+sweep_kernel(const double2 *__restrict__ xy, int n, const double *__restrict__ hg, int m,
+             int row_lo, int row_hi, int ntiles,
+             double *__restrict__ tileS, uint8_t *__restrict__ tileN)
+{
+    const int tile = blockIdx.x * kSweepWarps + (threadIdx.x >> 5);
+    const int lane = threadIdx.x & 31;
+    if (tile >= ntiles) return;  // warp-uniform
+    const int i = row_lo + tile * kTile + lane;
+    const bool valid = i < row_hi;
+    double xi = 0.0, yi = 0.0;
+    if (valid) {
+        double2 v = xy[i];
+        xi = v.x;
+        yi = v.y;
+    }
+    int R = valid ? i + 1 : n;   // next right candidate
+    int L = valid ? i - 1 : -1;  // next left candidate
+    Sums s{0.0, 0.0, 0.0};
+
+    for (int b = 0; b < m; b++) {
+        const double h = __ldg(hg + b);
+        // Right side: x[R] - x_i is non-decreasing in R.  4-wide fast path:
+        // if the 4th candidate is inside, all four are (monotone order).
+        while (R + 3 < n) {
+            double2 v0 = xy[R], v1 = xy[R + 1], v2 = xy[R + 2], v3 = xy[R + 3];
+            double d3 = v3.x - xi;
+            if (!inside<KERN>(d3, h)) break;
+            acc<KERN>(s, v0.y, v0.x - xi);
+            acc<KERN>(s, v1.y, v1.x - xi);
+            acc<KERN>(s, v2.y, v2.x - xi);
+            acc<KERN>(s, v3.y, d3);
+            R += 4;
+        }
+        while (R < n) {
+            double2 v = xy[R];
+            double d = v.x - xi;
+            if (!inside<KERN>(d, h)) break;
+            acc<KERN>(s, v.y, d);
+            R++;
+        }
+        // Left side: x_i - x[L] is non-decreasing as L decreases.
+        while (L >= 3) {
+            double2 v0 = xy[L], v1 = xy[L - 1], v2 = xy[L - 2], v3 = xy[L - 3];
+            double d3 = xi - v3.x;
+            if (!inside<KERN>(d3, h)) break;
+            acc<KERN>(s, v0.y, xi - v0.x);
+            acc<KERN>(s, v1.y, xi - v1.x);
+            acc<KERN>(s, v2.y, xi - v2.x);
+            acc<KERN>(s, v3.y, d3);
+            L -= 4;
+        }
+        while (L >= 0) {
+            double2 v = xy[L];
+            double d = xi - v.x;
+            if (!inside<KERN>(d, h)) break;
+            acc<KERN>(s, v.y, d);
+            L--;
+        }
+
+        // a4: LOO estimate (Eq.(2)); 0.75 and 1/h^2 cancel (reading Q5).
+        const int c = (R - i - 1) + (i - L - 1);
+        const bool M = valid && c > 0;  // Q6
+        double e2 = 0.0;
+        if (M) {
+            double g;
+            if (KERN == KR_UNIFORM) {
+                g = s.sy / (double)c;
+            } else {
+                const double hk = (KERN == KR_EPANECHNIKOV) ? h * h : h;
+                double num = fma(hk, s.sy, -s.sy1);
+                double den = fma(hk, (double)c, -s.s1);
+                // Q14 conditioning guard: the decomposition cancels when every
+                // in-window point sits near the edge; recompute directly over
+                // the contiguous window [L+1, R-1] \ {i} with exact factors.
+                if (!(den >= 0x1p-20 * hk * (double)c)) {
+                    num = 0.0;
+                    den = 0.0;
+                    for (int q = L + 1; q < R; q++) {
+                        if (q == i) continue;
+                        double2 v = xy[q];
+                        double d = fabs(v.x - xi);
+                        double w = (KERN == KR_EPANECHNIKOV) ? (h - d) * (h + d) : (h - d);
+                        num = fma(v.y, w, num);
+                        den += w;
+                    }
+                }
+                g = num / den;
+            }
+            const double e = yi - g;
+            e2 = e * e;
+        }
+        // a5 (warp level): lanes are rows; fixed shuffle tree.
+        e2 = warp_sum(e2);
+        const unsigned ball = __ballot_sync(0xffffffffu, M);
+        if (lane == 0) {
+            tileS[(size_t)b * ntiles + tile] = e2;
+            tileN[(size_t)b * ntiles + tile] = (uint8_t)__popc(ball);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a5: fixed-order column reduction of the tile partials (the paper's
+// "summation reduction ... performed k times", P@23970, as one launch).
+// ---------------------------------------------------------------------------
+constexpr int kReduceThreads = 256;
+
+__global__ void __launch_bounds__(kReduceThreads)
+reduce_kernel(const double *__restrict__ tileS, const uint8_t *__restrict__ tileN, int ntiles, int m,
+              const unsigned *__restrict__ status, double *__restrict__ partial)
+{
+    __shared__ double sS[kReduceThreads];
+    __shared__ long long sN[kReduceThreads];
+    for (int b = blockIdx.x; b < m; b += gridDim.x) {
+        double a = 0.0;
+        long long cnt = 0;
+        const double *col = tileS + (size_t)b * ntiles;
+        const uint8_t *ncol = tileN + (size_t)b * ntiles;
+        for (int t = threadIdx.x; t < ntiles; t += kReduceThreads) {
+            a += col[t];
+            cnt += ncol[t];
+        }
+        sS[threadIdx.x] = a;
+        sN[threadIdx.x] = cnt;
+        __syncthreads();
+        for (int s = kReduceThreads / 2; s > 0; s >>= 1) {
+            if (threadIdx.x < s) {
+                sS[threadIdx.x] += sS[threadIdx.x + s];
+                sN[threadIdx.x] += sN[threadIdx.x + s];
+            }
+            __syncthreads();
+        }
+        if (threadIdx.x == 0) {
+            partial[b] = sS[0];
+            partial[m + b] = (double)sN[0];
+        }
+        __syncthreads();
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        partial[2 * m] = (double)status[0];
+        partial[2 * m + 1] = (double)status[1];
+    }
+}
+
+// ---------------------------------------------------------------------------
+// finalize on the device: CV = S/n, arg-min (Q11), status.  One CTA.
+// ---------------------------------------------------------------------------
+constexpr int kFinThreads = 1024;
+
+__global__ void __launch_bounds__(kFinThreads)
+finalize_kernel(const double *__restrict__ partial, long long n, int m, double *__restrict__ cv,
+                long long *__restrict__ neff, int *__restrict__ best, int *__restrict__ status)
+{
+    __shared__ double sv[kFinThreads];
+    __shared__ int si[kFinThreads];
+    double bv = 0.0;
+    int bi = -1;
+    for (int b = threadIdx.x; b < m; b += kFinThreads) {
+        double v = partial[b] / (double)n;
+        cv[b] = v;
+        if (neff) neff[b] = (long long)partial[m + b];
+        if (!isnan(v) && (bi < 0 || v < bv)) {  // strided order: b ascending per thread
+            bv = v;
+            bi = b;
+        }
+    }
+    sv[threadIdx.x] = bv;
+    si[threadIdx.x] = bi;
+    __syncthreads();
+    for (int s = kFinThreads / 2; s > 0; s >>= 1) {
+        if (threadIdx.x < s) {
+            double ov = sv[threadIdx.x + s];
+            int oi = si[threadIdx.x + s];
+            int mi = si[threadIdx.x];
+            double mv = sv[threadIdx.x];
+            if (oi >= 0 && (mi < 0 || ov < mv || (ov == mv && oi < mi))) {
+                sv[threadIdx.x] = ov;
+                si[threadIdx.x] = oi;
+            }
+        }
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) {
+        *best = si[0] < 0 ? 0 : si[0];
+        int st = KR_OK;
+        if (partial[2 * m] != 0.0) st = KR_EGRID;
+        else if (partial[2 * m + 1] != 0.0) st = KR_ENONFINITE;
+        *status = st;
+    }
+}
+
+// ---------------------------------------------------------------------------
+// host-side launch helpers
+// ---------------------------------------------------------------------------
+// CUB onesweep falls back to a single-tile kernel below this many keys
+// (policy-dependent; verified from the ncu launch list).
+constexpr int64_t kCubSingleTile = 0;
+
+static inline size_t align256(size_t v) { return (v + 255) & ~size_t(255); }
+
+bool ws_layout(int64_t n, int32_t m, WsLayout *L)
+{
+    size_t cub_bytes = 0;
+    cudaError_t e = cub::DeviceRadixSort::SortPairs(
+        nullptr, cub_bytes, (const uint64_t *)nullptr, (uint64_t *)nullptr,
+        (const uint32_t *)nullptr, (uint32_t *)nullptr, (int)n, 0, 64, (cudaStream_t)0);
+    if (e != cudaSuccess) {
+        set_cuda_error("cub::DeviceRadixSort::SortPairs(size query)", (int)e);
+        return false;
+    }
+    const int64_t ntiles = (n + kTile - 1) / kTile;
+    size_t off = 0;
+    L->keys_in = off;  off = align256(off + sizeof(uint64_t) * (size_t)n);
+    L->keys_out = off; off = align256(off + sizeof(uint64_t) * (size_t)n);
+    L->vals_in = off;  off = align256(off + sizeof(uint32_t) * (size_t)n);
+    L->vals_out = off; off = align256(off + sizeof(uint32_t) * (size_t)n);
+    L->xy = off;       off = align256(off + sizeof(double2) * (size_t)n);
+    L->tileS = off;    off = align256(off + sizeof(double) * (size_t)ntiles * (size_t)m);
+    L->tileN = off;    off = align256(off + sizeof(uint8_t) * (size_t)ntiles * (size_t)m);
+    L->status = off;   off = align256(off + 2 * sizeof(unsigned));
+    L->cub = off;      off = align256(off + cub_bytes);
+    L->cub_bytes = cub_bytes;
+    L->total = off;
+    L->ntiles_max = ntiles;
+    return true;
+}
+
+static int grid_for(int64_t work, int threads)
+{
+    int64_t b = (work + threads - 1) / threads;
+    if (b < 1) b = 1;
+    if (b > 148 * 16) b = 148 * 16;
+    return (int)b;
+}
+
+template <int KERN>
+static void launch_sweep(const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
+                         double *tileS, uint8_t *tileN, cudaStream_t st)
+{
+    const int blocks = (ntiles + kSweepWarps - 1) / kSweepWarps;
+    sweep_kernel<KERN><<<blocks, kSweepThreads, 0, st>>>(xy, n, h, m, lo, hi, ntiles, tileS, tileN);
+}
+
+// Optional stage timing (kr_profile_enable / kr_profile_read), thread-local.
+struct Prof {
+    bool on = false;
+    bool recorded = false;
+    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+    int64_t launches = 0;
+};
+static thread_local Prof g_prof;
+
+static void prof_mark(int k, cudaStream_t st)
+{
+    if (!g_prof.on) return;
+    if (!g_prof.ev[k]) cudaEventCreate(&g_prof.ev[k]);
+    cudaEventRecord(g_prof.ev[k], st);
+}
+
+// Kernel launches CUB's radix sort makes for `n` 64-bit keys.  Onesweep:
+// one histogram kernel + one exclusive-scan kernel + one pass per 8-bit
+// digit; below the single-tile threshold a single kernel.  (Cross-checked
+// against the ncu launch list, profiles/.)
+static int64_t cub_sort_launches(int64_t n) { return n <= kCubSingleTile ? 1 : 2 + 64 / 8; }
+
+}  // namespace krcv
+
+using namespace krcv;
+
+extern "C" int kr_profile_enable(int on)
+{
+    g_prof.on = on != 0;
+    g_prof.recorded = false;
+    return KR_OK;
+}
+
+extern "C" int kr_profile_read(float *ms)
+{
+    if (!ms || !g_prof.recorded) return KR_EARG;
+    cudaError_t e = cudaEventSynchronize(g_prof.ev[3]);
+    if (e != cudaSuccess) { set_cuda_error("cudaEventSynchronize", (int)e); return KR_ECUDA; }
+    for (int k = 0; k < 3; k++) {
+        e = cudaEventElapsedTime(&ms[k], g_prof.ev[k], g_prof.ev[k + 1]);
+        if (e != cudaSuccess) { set_cuda_error("cudaEventElapsedTime", (int)e); return KR_ECUDA; }
+    }
+    return KR_OK;
+}
+
+extern "C" int64_t kr_launch_count(void) { return g_prof.launches; }
+
+extern "C" size_t kr_workspace_bytes(int64_t n, int32_t m)
+{
+    if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return 0;
+    WsLayout L;
+    if (!ws_layout(n, m, &L)) return 0;
+    return L.total;
+}
+
+extern "C" int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n,
+                                 const double *d_h, int32_t m, int32_t kernel,
+                                 int32_t shard, int32_t nshards,
+                                 double *d_partial, void *d_workspace, size_t workspace_bytes,
+                                 void *cuda_stream)
+{
+    if (!d_x || !d_y || !d_h || !d_partial || !d_workspace) return KR_EARG;
+    if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return KR_EARG;
+    if (kernel != KR_UNIFORM && kernel != KR_EPANECHNIKOV && kernel != KR_TRIANGULAR) return KR_EKERNEL;
+    if (nshards < 1 || shard < 0 || shard >= nshards) return KR_EARG;
+    if ((reinterpret_cast<uintptr_t>(d_workspace) & 255u) != 0) return KR_EARG;
+    WsLayout L;
+    if (!ws_layout(n, m, &L)) return KR_ECUDA;
+    if (workspace_bytes < L.total) return KR_EARG;
+
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    char *ws = static_cast<char *>(d_workspace);
+    uint64_t *keys_in = reinterpret_cast<uint64_t *>(ws + L.keys_in);
+    uint64_t *keys_out = reinterpret_cast<uint64_t *>(ws + L.keys_out);
+    uint32_t *vals_in = reinterpret_cast<uint32_t *>(ws + L.vals_in);
+    uint32_t *vals_out = reinterpret_cast<uint32_t *>(ws + L.vals_out);
+    double2 *xy = reinterpret_cast<double2 *>(ws + L.xy);
+    double *tileS = reinterpret_cast<double *>(ws + L.tileS);
+    uint8_t *tileN = reinterpret_cast<uint8_t *>(ws + L.tileN);
+    unsigned *status = reinterpret_cast<unsigned *>(ws + L.status);
+    const int nn = (int)n;
+
+    // Rows of this shard in sorted order.
+    const int lo = (int)(((int64_t)shard * n) / nshards);
+    const int hi = (int)(((int64_t)(shard + 1) * n) / nshards);
+    const int ntiles = (hi - lo + kTile - 1) / kTile;
+
+    int64_t launches = 0;
+    prof_mark(0, st);
+    cudaError_t e = cudaMemsetAsync(status, 0, 2 * sizeof(unsigned), st);
+    if (e != cudaSuccess) { set_cuda_error("cudaMemsetAsync(status)", (int)e); return KR_ECUDA; }
+    pack_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, nn, d_h, m, keys_in, vals_in, status);
+    size_t cub_bytes = L.cub_bytes;
+    e = cub::DeviceRadixSort::SortPairs(ws + L.cub, cub_bytes, keys_in, keys_out, vals_in, vals_out,
+                                        nn, 0, 64, st);
+    if (e != cudaSuccess) { set_cuda_error("cub::DeviceRadixSort::SortPairs", (int)e); return KR_ECUDA; }
+    gather_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, vals_out, nn, xy);
+    launches += 2 + cub_sort_launches(n);
+    prof_mark(1, st);
+    if (ntiles > 0) {
+        launches += 1;
+        switch (kernel) {
+        case KR_UNIFORM:
+            launch_sweep<KR_UNIFORM>(xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, st);
+            break;
+        case KR_EPANECHNIKOV:
+            launch_sweep<KR_EPANECHNIKOV>(xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, st);
+            break;
+        default:
+            launch_sweep<KR_TRIANGULAR>(xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, st);
+            break;
+        }
+    }
+    prof_mark(2, st);
+    reduce_kernel<<<m < 148 * 8 ? m : 148 * 8, kReduceThreads, 0, st>>>(tileS, tileN, ntiles, m, status,
+                                                                        d_partial);
+    launches += 1;
+    prof_mark(3, st);
+    g_prof.recorded = g_prof.on;
+    g_prof.launches = launches;
+    e = cudaGetLastError();
+    if (e != cudaSuccess) { set_cuda_error("kernel launch", (int)e); return KR_ECUDA; }
+    return KR_OK;
+}
+
+extern "C" int kr_finalize_async(const double *d_partial, int64_t n, int32_t m, double *d_cv,
+                                 int64_t *d_neff, int32_t *d_best, int32_t *d_status, void *cuda_stream)
+{
+    if (!d_partial || !d_cv || !d_best || !d_status || n < 1 || m < 1 || m > KR_MAX_M) return KR_EARG;
+    finalize_kernel<<<1, kFinThreads, 0, static_cast<cudaStream_t>(cuda_stream)>>>(
+        d_partial, (long long)n, m, d_cv, reinterpret_cast<long long *>(d_neff), d_best, d_status);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) { set_cuda_error("finalize_kernel launch", (int)e); return KR_ECUDA; }
+    return KR_OK;
+}

@@ -1,0 +1,33 @@
+// krcv_internal.h -- declarations shared by the host (krcv_host.cpp) and
+// device (krcv_device.cu) halves of libkrcv.so.  Not part of the C-ABI.
+#pragma once
+
+#include <cstddef>
+#include <cstdint>
+
+namespace krcv {
+
+// Rows per warp tile in the sweep kernel (one sorted row per lane).
+constexpr int kTile = 32;
+
+// Byte layout of the device workspace (kr_workspace_bytes / kr_cv_shard_async).
+struct WsLayout {
+    size_t keys_in, keys_out;   // uint64 [n]  order-preserving keys of x
+    size_t vals_in, vals_out;   // uint32 [n]  original indices
+    size_t xy;                  // double2 [n] (x, y) in sorted order
+    size_t tileS;               // double  [m][ntiles]  per-tile sum of M e^2
+    size_t tileN;               // uint8   [m][ntiles]  per-tile sum of M
+    size_t status;              // uint32  [2]  n_bad_grid, n_nonfinite
+    size_t cub;                 // radix-sort scratch
+    size_t cub_bytes;
+    size_t total;
+    int64_t ntiles_max;
+};
+
+// Fills `out`; returns false if the CUDA runtime refuses the sort-size query.
+bool ws_layout(int64_t n, int32_t m, WsLayout *out);
+
+// Records a CUDA error string for kr_last_cuda_error (thread-local).
+void set_cuda_error(const char *what, int code);
+
+}  // namespace krcv

@@ -1,0 +1,231 @@
+"""Thin ctypes binding of ``libkrcv.so`` (include/krcv.h).
+
+Argument marshalling only: every step of the hot path runs in the sm_100a
+kernels of ``csrc/krcv_device.cu``.  There is no CPU fallback: if the shared
+library is missing the import fails loudly (build it with
+``python -c "import __graft_entry__ as g; g.build()"``).
+
+The functions keep the C names (``kr_cv_grid``, ``kr_cv_shard_async``,
+``kr_finalize``, ``kr_finalize_async``, ``kr_default_grid``,
+``kr_workspace_bytes``, ``kr_validate_grid``, ``kr_strerror``).
+Host-pointer calls take numpy arrays; device-pointer calls take
+``torch.Tensor`` objects on a CUDA device (PyTorch provides device memory and
+streams only).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libkrcv.so")
+
+UNIFORM, EPANECHNIKOV, TRIANGULAR = 0, 1, 2
+KERNELS = {"uniform": UNIFORM, "epanechnikov": EPANECHNIKOV, "triangular": TRIANGULAR}
+
+KR_OK, KR_EARG, KR_EKERNEL, KR_EGRID, KR_ENONFINITE, KR_EDEGENERATE, KR_ENOMEM, KR_ECUDA = range(8)
+KR_MAX_M = 65536
+
+# Every symbol include/krcv.h declares (checked by tests/test_abi.py).
+EXPORTS = (
+    "kr_cv_grid", "kr_cv_grid_ex", "kr_validate_grid", "kr_workspace_bytes",
+    "kr_cv_shard_async", "kr_finalize", "kr_finalize_async", "kr_default_grid",
+    "kr_strerror", "kr_last_cuda_error", "kr_version",
+    "kr_profile_enable", "kr_profile_read", "kr_launch_count",
+)
+
+
+def partial_len(m: int) -> int:
+    return 2 * int(m) + 2
+
+
+class KrcvError(RuntimeError):
+    def __init__(self, status: int, where: str = ""):
+        msg = _lib().kr_strerror(status).decode()
+        if status == KR_ECUDA:
+            msg += f": {_lib().kr_last_cuda_error().decode()}"
+        super().__init__(f"{where}: {msg} (status {status})" if where else msg)
+        self.status = status
+
+
+_LIB = None
+
+
+def _lib() -> ctypes.CDLL:
+    global _LIB
+    if _LIB is not None:
+        return _LIB
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(
+            f"libkrcv.so not found at {LIB_PATH}; build it with __graft_entry__.build() "
+            "(there is no CPU fallback)")
+    lib = ctypes.CDLL(LIB_PATH)
+    P, i64, i32, sz = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_size_t
+    lib.kr_cv_grid.argtypes = [P, P, i64, P, i32, i32, P, P]
+    lib.kr_cv_grid_ex.argtypes = [P, P, i64, P, i32, i32, P, P, P]
+    lib.kr_validate_grid.argtypes = [P, i32]
+    lib.kr_workspace_bytes.argtypes = [i64, i32]
+    lib.kr_workspace_bytes.restype = sz
+    lib.kr_cv_shard_async.argtypes = [P, P, i64, P, i32, i32, i32, i32, P, P, sz, P]
+    lib.kr_finalize.argtypes = [P, i64, i32, P, P, P]
+    lib.kr_finalize_async.argtypes = [P, i64, i32, P, P, P, P, P]
+    lib.kr_default_grid.argtypes = [P, i64, i32, P]
+    for f in ("kr_cv_grid", "kr_cv_grid_ex", "kr_validate_grid", "kr_cv_shard_async",
+              "kr_finalize", "kr_finalize_async", "kr_default_grid"):
+        getattr(lib, f).restype = ctypes.c_int
+    lib.kr_strerror.argtypes = [ctypes.c_int]
+    lib.kr_strerror.restype = ctypes.c_char_p
+    lib.kr_last_cuda_error.restype = ctypes.c_char_p
+    lib.kr_version.restype = ctypes.c_char_p
+    lib.kr_profile_enable.argtypes = [ctypes.c_int]
+    lib.kr_profile_enable.restype = ctypes.c_int
+    lib.kr_profile_read.argtypes = [P]
+    lib.kr_profile_read.restype = ctypes.c_int
+    lib.kr_launch_count.restype = ctypes.c_int64
+    _LIB = lib
+    return lib
+
+
+def _kernel_id(kernel) -> int:
+    if isinstance(kernel, str):
+        return KERNELS[kernel.lower()]
+    return int(kernel)
+
+
+def _host(a) -> np.ndarray:
+    return np.ascontiguousarray(a, dtype=np.float64)
+
+
+def _check(st: int, where: str) -> None:
+    if st != KR_OK:
+        raise KrcvError(st, where)
+
+
+# ------------------------------------------------------------------ host API
+def kr_cv_grid(x, y, h, kernel="epanechnikov", with_neff: bool = False):
+    """Whole grid search on the current CUDA device from host arrays.
+    Returns (cv[m], best) or (cv, neff, best)."""
+    x, y, h = _host(x), _host(y), _host(h)
+    if x.shape != y.shape or x.ndim != 1:
+        raise ValueError("x and y must be 1-D arrays of equal length")
+    n, m = x.shape[0], h.shape[0]
+    cv = np.empty(m, np.float64)
+    best = ctypes.c_int32(-1)
+    if with_neff:
+        neff = np.empty(m, np.int64)
+        st = _lib().kr_cv_grid_ex(x.ctypes.data, y.ctypes.data, n, h.ctypes.data, m, _kernel_id(kernel),
+                                  cv.ctypes.data, neff.ctypes.data, ctypes.byref(best))
+        _check(st, "kr_cv_grid_ex")
+        return cv, neff, int(best.value)
+    st = _lib().kr_cv_grid(x.ctypes.data, y.ctypes.data, n, h.ctypes.data, m, _kernel_id(kernel),
+                           cv.ctypes.data, ctypes.byref(best))
+    _check(st, "kr_cv_grid")
+    return cv, int(best.value)
+
+
+def kr_cv_grid_ptr(x_ptr: int, y_ptr: int, n: int, h_ptr: int, m: int, kernel: int,
+                   cv_ptr: int, best_ref) -> int:
+    """Raw-pointer form (used by bench.py's end-to-end leg with pinned buffers)."""
+    return _lib().kr_cv_grid(x_ptr, y_ptr, n, h_ptr, m, kernel, cv_ptr, best_ref)
+
+
+def kr_default_grid(x, m: int) -> np.ndarray:
+    x = _host(x)
+    h = np.empty(int(m), np.float64)
+    _check(_lib().kr_default_grid(x.ctypes.data, x.shape[0], int(m), h.ctypes.data), "kr_default_grid")
+    return h
+
+
+def kr_validate_grid(h) -> int:
+    h = _host(h)
+    return int(_lib().kr_validate_grid(h.ctypes.data if h.size else None, h.shape[0]))
+
+
+def kr_finalize(partial, n: int, m: int):
+    """Host finalize of summed partials -> (cv, neff, best)."""
+    p = _host(partial)
+    if p.shape[0] != partial_len(m):
+        raise ValueError("partial must have length 2m+2")
+    cv = np.empty(m, np.float64)
+    neff = np.empty(m, np.int64)
+    best = ctypes.c_int32(-1)
+    _check(_lib().kr_finalize(p.ctypes.data, int(n), int(m), cv.ctypes.data, neff.ctypes.data,
+                              ctypes.byref(best)), "kr_finalize")
+    return cv, neff, int(best.value)
+
+
+def kr_strerror(status: int) -> str:
+    return _lib().kr_strerror(int(status)).decode()
+
+
+def kr_version() -> str:
+    return _lib().kr_version().decode()
+
+
+def kr_workspace_bytes(n: int, m: int) -> int:
+    return int(_lib().kr_workspace_bytes(int(n), int(m)))
+
+
+# ---------------------------------------------------------------- device API
+def kr_cv_shard_async(d_x, d_y, d_h, kernel, shard: int, nshards: int, d_partial, d_ws, stream=None) -> None:
+    """Enqueue the sharded device pipeline.  All tensor arguments are CUDA
+    torch tensors (float64 for x, y, h, partial; uint8 for the workspace)."""
+    import torch
+
+    n, m = d_x.numel(), d_h.numel()
+    for t, name in ((d_x, "x"), (d_y, "y"), (d_h, "h"), (d_partial, "partial")):
+        if not (t.is_cuda and t.dtype == torch.float64 and t.is_contiguous()):
+            raise ValueError(f"{name} must be a contiguous float64 CUDA tensor")
+    if d_partial.numel() != partial_len(m):
+        raise ValueError("partial must have 2m+2 elements")
+    s = torch.cuda.current_stream(d_x.device) if stream is None else stream
+    st = _lib().kr_cv_shard_async(d_x.data_ptr(), d_y.data_ptr(), n, d_h.data_ptr(), m, _kernel_id(kernel),
+                                  int(shard), int(nshards), d_partial.data_ptr(), d_ws.data_ptr(),
+                                  d_ws.numel() * d_ws.element_size(), ctypes.c_void_p(s.cuda_stream))
+    _check(st, "kr_cv_shard_async")
+
+
+def kr_finalize_async(d_partial, n: int, m: int, d_cv, d_neff, d_best_status, stream=None) -> None:
+    """Device finalize: d_cv float64[m], d_neff int64[m] (or None),
+    d_best_status int32[2] -> (best, status)."""
+    import torch
+
+    s = torch.cuda.current_stream(d_partial.device) if stream is None else stream
+    st = _lib().kr_finalize_async(d_partial.data_ptr(), int(n), int(m), d_cv.data_ptr(),
+                                  None if d_neff is None else d_neff.data_ptr(),
+                                  d_best_status.data_ptr(), d_best_status.data_ptr() + 4,
+                                  ctypes.c_void_p(s.cuda_stream))
+    _check(st, "kr_finalize_async")
+
+
+def kr_profile_enable(on: bool) -> None:
+    _lib().kr_profile_enable(1 if on else 0)
+
+
+def kr_profile_read():
+    """(sort_ms, sweep_ms, reduce_ms) of the last kr_cv_shard_async on this thread."""
+    ms = np.zeros(3, np.float32)
+    _check(_lib().kr_profile_read(ms.ctypes.data), "kr_profile_read")
+    return float(ms[0]), float(ms[1]), float(ms[2])
+
+
+def kr_launch_count() -> int:
+    return int(_lib().kr_launch_count())
+
+
+def workspace(n: int, m: int, device=None):
+    """A device workspace tensor (PyTorch caching allocator, 256-B aligned)."""
+    import torch
+
+    nbytes = kr_workspace_bytes(n, m)
+    if nbytes == 0:
+        raise KrcvError(KR_ECUDA, "kr_workspace_bytes")
+    return torch.empty(nbytes + 256, dtype=torch.uint8, device=device)
+
+
+def aligned(ws):
+    """View of ws starting at a 256-byte boundary."""
+    off = (-ws.data_ptr()) % 256
+    return ws[off:]

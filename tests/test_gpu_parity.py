@@ -1,0 +1,231 @@
+"""GPU parity: the CUDA path (through the C-ABI) vs the CPU oracle (T3, T4, T8).
+
+Bar (BASELINE.json north_star): relative error <= 1e-6 on CV(h) with the
+floor of SURVEY.md §8(c); n_eff identical; best identical unless the oracle's
+two best values lie within 1e-6.  On well-conditioned workloads we also assert
+a much tighter 1e-10 (fp64 vs long double is ~1e-14).
+"""
+from __future__ import annotations
+
+import json
+import math
+import os
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads
+from oracle import exact
+from paper_conf_ipps_rohlfsz17_b200 import krcv
+from paper_conf_ipps_rohlfsz17_b200.api import GridSearch
+from tests.helpers import best_ok, cv_rel_err
+
+pytestmark = pytest.mark.gpu
+
+U, E, T = 0, 1, 2
+TOL = 1e-6
+TIGHT = 1e-10
+
+
+def _gpu(x, y, h, k):
+    cv, neff, best = krcv.kr_cv_grid(x, y, h, k, with_neff=True)
+    return cv, neff, best
+
+
+def _check(x, y, h, k, ref=None, tight=True):
+    cv, neff, best = _gpu(x, y, h, k)
+    if ref is None:
+        ref = oracle.cv_sorted(x, y, h, k) if x.shape[0] > 400 else oracle.cv_direct(x, y, h, k)
+    err = cv_rel_err(cv, ref.cv)
+    assert err <= (TIGHT if tight else TOL), err
+    assert np.array_equal(neff, ref.neff)
+    assert best_ok(best, ref.cv), (best, ref.best)
+    return err
+
+
+@pytest.mark.parametrize("kname", ["epanechnikov", "uniform", "triangular"])
+def test_worked_example_exact(kname):
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "worked_example.json")))
+    k = workloads.KERNEL_IDS[kname]
+    cv, neff, best = _gpu(np.array(g["x"]), np.array(g["y"]), np.array(g["h"]), k)
+    want = [float(Fraction(s)) for s in g[kname]["cv"]]
+    for b in range(len(want)):
+        assert abs(cv[b] - want[b]) <= 4 * math.ulp(want[b]) if want[b] else cv[b] == 0.0
+    assert list(neff) == g[kname]["neff"] and best == g[kname]["best"]
+
+
+@pytest.mark.parametrize("seed", range(16))
+def test_exact_rational_dyadic(seed):
+    """Dyadic inputs with points exactly at h and duplicated x: window
+    membership must be bit-exact (n_eff identical), CV to fp64 rounding."""
+    rng = np.random.default_rng(50 + seed)
+    n = int(rng.integers(2, 17))
+    m = int(rng.integers(1, 9))
+    x, y, h = workloads.random_dyadic(n, m, seed)
+    for k in (U, E, T):
+        cv_ex, ne_ex, best_ex = exact.cv_exact(x, y, h, k)
+        cv, neff, best = _gpu(x, y, h, k)
+        assert cv_rel_err(cv, [float(v) for v in cv_ex]) <= 1e-13
+        assert list(neff) == ne_ex
+        assert best == best_ex or cv[best] == cv[best_ex]
+
+
+@pytest.mark.parametrize("n", [2, 3, 31, 32, 33, 64, 65, 127, 1000])
+@pytest.mark.parametrize("dist", ["paper", "sin_uniform", "lognormal"])
+@pytest.mark.parametrize("k", [U, E, T])
+def test_small_sizes_tiles_and_ragged_tails(n, dist, k):
+    x, y = workloads.draw_xy(dist, n, 3)
+    m = 37
+    h = workloads.grid_log(x, m) if dist == "lognormal" else workloads.grid_default(x, m)
+    _check(x, y, h, k)
+
+
+@pytest.mark.parametrize("k", [U, E, T])
+def test_user_grid_with_duplicates_and_small_h(k):
+    x, y = workloads.draw_xy("paper", 777, 8)
+    h = np.sort(np.concatenate([np.linspace(1e-4, 0.02, 20), [0.01, 0.01, 0.5, 0.5], np.linspace(0.3, 2.0, 9)]))
+    _check(x, y, h, k)
+
+
+@pytest.mark.parametrize("k", [U, E, T])
+def test_duplicate_x_constant_y_and_equal_x(k):
+    x, y = workloads.draw_xy("paper", 300, 9)
+    x = np.round(x * 20) / 20  # heavy ties in x
+    h = workloads.grid_default(x, 25)
+    _check(x, y, h, k)
+    cv, neff, best = _gpu(x, np.full_like(y, 4.0), h, k)
+    assert np.all(cv == 0.0)
+    # every x equal: all pairs at d = 0 -> g is the LOO mean
+    xe = np.full(50, 0.75)
+    ref = oracle.cv_direct(xe, y[:50], [0.1, 1.0], k)
+    cv, neff, best = _gpu(xe, y[:50], np.array([0.1, 1.0]), k)
+    assert cv_rel_err(cv, ref.cv) <= TIGHT and np.array_equal(neff, ref.neff)
+
+
+@pytest.mark.parametrize("k", [E, T])
+@pytest.mark.parametrize("yv", [(3.0, 5.0), (0.1, 7.0), (5.0, 0.125)])
+def test_edge_cancellation_guard(k, yv):
+    """One neighbour at d = nextafter(h, 0): guarded path returns g = y_l."""
+    x = np.array([0.0, np.nextafter(1.0, 0.0)])
+    y = np.array(yv)
+    cv, neff, _ = _gpu(x, y, np.array([1.0]), k)
+    want = float((Fraction(y[0]) - Fraction(y[1])) ** 2)
+    assert abs(cv[0] - want) <= 2 * math.ulp(want) and neff[0] == 2
+
+
+def test_boundary_exactly_at_h_uniform():
+    """Default grid's last point h = r puts (min, max) exactly on the closed
+    uniform window: GPU and oracle must agree bit-level on n_eff
+    and the closed form."""
+    x, y, h, k = workloads.make("C1", seed=0)
+    _check(x, y, h, k)
+
+
+def test_C1_seed0_full():
+    x, y, h, k = workloads.make("C1", seed=0)
+    cv, neff, best = _gpu(x, y, h, k)
+    ref = oracle.cv_direct(x, y, h, k)
+    assert cv_rel_err(cv, ref.cv) <= TIGHT and best == ref.best == 4
+
+
+def test_C2_seed0_full():
+    x, y, h, k = workloads.make("C2", seed=0)
+    cv, neff, best = _gpu(x, y, h, k)
+    ref = oracle.cv_sorted(x, y, h, k)
+    assert cv_rel_err(cv, ref.cv) <= TIGHT
+    assert np.array_equal(neff, ref.neff)
+    assert best == ref.best == 1
+
+
+def _device_partial(x, y, h, k, shard, nshards):
+    import torch
+    d_x = torch.as_tensor(x, device="cuda")
+    d_y = torch.as_tensor(y, device="cuda")
+    d_h = torch.as_tensor(h, device="cuda")
+    part = torch.empty(krcv.partial_len(h.shape[0]), dtype=torch.float64, device="cuda")
+    ws = krcv.aligned(krcv.workspace(x.shape[0], h.shape[0], "cuda"))
+    krcv.kr_cv_shard_async(d_x, d_y, d_h, k, shard, nshards, part, ws)
+    torch.cuda.synchronize()
+    return part.cpu().numpy()
+
+
+@pytest.mark.parametrize("cfg,P,shard", [("C3", 64, 17), ("C5", 64, 0), ("C5", 64, 63), ("C4", 4096, 2048)])
+def test_full_size_sampled_shard(cfg, P, shard):
+    """Full BASELINE sizes in the bench launch configuration: one row shard of
+    the sorted order, checked against the oracle on exactly those rows."""
+    x, y, h, k = workloads.make(cfg, seed=0)
+    part = _device_partial(x, y, h, k, shard, P)
+    m = h.shape[0]
+    ref = oracle.cv_sorted(x, y, h, k, rows=oracle.shard_rows(x, shard, P))
+    assert cv_rel_err(part[:m], ref.S) <= TIGHT
+    assert np.array_equal(part[m:2 * m].astype(np.int64), ref.neff)
+    assert part[2 * m] == 0 and part[2 * m + 1] == 0
+
+
+@pytest.mark.parametrize("P", [2, 3, 8, 64])
+def test_shard_emulation_sums_to_unsharded(P):
+    """T4: shards 0..P-1 on one GPU, summed on the host == unsharded run."""
+    x, y, h, k = workloads.make("C5", seed=1, n=5000)
+    full = _device_partial(x, y, h, k, 0, 1)
+    tot = sum(_device_partial(x, y, h, k, r, P) for r in range(P))
+    m = h.shape[0]
+    assert cv_rel_err(tot[:m], full[:m]) <= 1e-14
+    assert np.array_equal(tot[m:], full[m:])
+    cv, neff, best = krcv.kr_finalize(tot, x.shape[0], m)
+    ref = oracle.cv_sorted(x, y, h, k)
+    assert cv_rel_err(cv, ref.cv) <= TIGHT and best_ok(best, ref.cv)
+
+
+def test_determinism_bitwise():
+    """T8: repeated runs are bit-identical (static row->warp map, fixed-order reductions)."""
+    x, y, h, k = workloads.make("C2", seed=2, n=6000)
+    a = _gpu(x, y, h, k)[0]
+    for _ in range(3):
+        assert np.array_equal(_gpu(x, y, h, k)[0], a)
+
+
+def test_device_status_nonfinite_and_bad_grid():
+    import torch
+    x, y, h, k = workloads.make("C2", seed=0, n=500)
+    x = x.copy()
+    x[10] = np.nan
+    part = _device_partial(x, y, h, k, 0, 1)
+    with pytest.raises(krcv.KrcvError) as e:
+        krcv.kr_finalize(part, x.shape[0], h.shape[0])
+    assert e.value.status == krcv.KR_ENONFINITE
+    x[10] = 0.5
+    hb = h.copy()
+    hb[3] = -1.0
+    part = _device_partial(x, y, hb, k, 0, 1)
+    with pytest.raises(krcv.KrcvError) as e:
+        krcv.kr_finalize(part, x.shape[0], h.shape[0])
+    assert e.value.status == krcv.KR_EGRID
+    # device finalize reports the same status
+    plan = GridSearch(x.shape[0], h, k)
+    xd = torch.as_tensor(x, device="cuda")
+    yd = torch.as_tensor(y, device="cuda")
+    xd[10] = float("inf")
+    plan.run(xd, yd)
+    with pytest.raises(krcv.KrcvError) as e:
+        plan.result()
+    assert e.value.status == krcv.KR_ENONFINITE
+
+
+def test_device_api_matches_host_api():
+    import torch
+    x, y, h, k = workloads.make("C5", seed=0, n=20000)
+    plan = GridSearch(x.shape[0], h, k)
+    plan.run(torch.as_tensor(x, device="cuda"), torch.as_tensor(y, device="cuda"))
+    r = plan.result()
+    cv, neff, best = _gpu(x, y, h, k)
+    assert np.array_equal(r.cv.cpu().numpy(), cv)
+    assert np.array_equal(r.neff.cpu().numpy(), neff) and r.best == best
+
+
+@pytest.mark.parametrize("m", [1, 2, 4099])
+def test_grid_sizes(m):
+    x, y = workloads.draw_xy("paper", 900, 1)
+    h = workloads.grid_default(x, m)
+    _check(x, y, h, E)
