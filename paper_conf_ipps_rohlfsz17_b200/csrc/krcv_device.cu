@@ -18,9 +18,12 @@
 
 #include <cmath>
 #include <cstdint>
+#include <cstdlib>
 
 #include "krcv.h"
 #include "krcv_internal.h"
+#include "krcv_sweep.cuh"
+#include "krcv_sweep_gxg.cuh"
 
 namespace krcv {
 
@@ -56,164 +59,29 @@ __global__ void pack_kernel(const double *__restrict__ x, const double *__restri
     if (gbad) atomicAdd(&status[0], gbad);
 }
 
-// a2 (second half): gather (x, y) into sorted order as one 16-byte record.
+// a2 (second half): gather (x, y) into sorted order as one 16-byte record,
+// with kPad (-inf, 0) / (+inf, 0) sentinels before and after (xy points at
+// the first real record).  Also resets the sweep's tile counter.
 __global__ void gather_kernel(const double *__restrict__ x, const double *__restrict__ y,
-                              const uint32_t *__restrict__ order, int n, double2 *__restrict__ xy)
+                              const uint32_t *__restrict__ order, int n, double2 *__restrict__ xy,
+                              int *__restrict__ tile_counter)
 {
     const int stride = gridDim.x * blockDim.x;
-    for (int k = blockIdx.x * blockDim.x + threadIdx.x; k < n; k += stride) {
+    const int tid = blockIdx.x * blockDim.x + threadIdx.x;
+    for (int k = tid; k < n; k += stride) {
         uint32_t i = order[k];
         xy[k] = make_double2(x[i], y[i]);
     }
+    if (tid < kPad) {
+        xy[-1 - tid] = make_double2(-INFINITY, 0.0);
+        xy[n + tid] = make_double2(INFINITY, 0.0);
+    }
+    if (tid == 0) *tile_counter = 0;
 }
 
 // ---------------------------------------------------------------------------
-// a3 + a4: the sweep
+// a3 + a4: the sweep -- see krcv_sweep.cuh
 // ---------------------------------------------------------------------------
-template <int KERN>
-__device__ __forceinline__ bool inside(double d, double h)
-{
-    // Q1: open window for Epanechnikov / triangular, closed for uniform.
-    return KERN == KR_UNIFORM ? (d <= h) : (d < h);
-}
-
-// Running sums of one row.  Epanechnikov: sum y, sum d^2, sum y d^2 (§III
-// P@14010; the count comes from the pointers, reading Q3).  Triangular: sum y,
-// sum d, sum y d.  Uniform: sum y.
-struct Sums {
-    double sy, s1, sy1;
-};
-
-template <int KERN>
-__device__ __forceinline__ void acc(Sums &s, double yv, double d)
-{
-    s.sy += yv;
-    if (KERN == KR_EPANECHNIKOV) {
-        double d2 = d * d;
-        s.s1 += d2;
-        s.sy1 = fma(yv, d2, s.sy1);
-    } else if (KERN == KR_TRIANGULAR) {
-        s.s1 += d;
-        s.sy1 = fma(yv, d, s.sy1);
-    }
-}
-
-__device__ __forceinline__ double warp_sum(double v)
-{
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-    return v;
-}
-
-constexpr int kSweepWarps = 4;
-constexpr int kSweepThreads = kSweepWarps * 32;
-
-// One warp = 32 consecutive sorted rows (one per lane); bandwidths ascend in
-// lock-step across the warp (warp-uniform b).  Per (tile, b) the warp writes
-// sum M e^2 and sum M to tileS/tileN[b][tile]; nothing per pair is stored.
-template <int KERN>
-__global__ void __launch_bounds__(kSweepThreads)
-sweep_kernel(const double2 *__restrict__ xy, int n, const double *__restrict__ hg, int m,
-             int row_lo, int row_hi, int ntiles,
-             double *__restrict__ tileS, uint8_t *__restrict__ tileN)
-{
-    const int tile = blockIdx.x * kSweepWarps + (threadIdx.x >> 5);
-    const int lane = threadIdx.x & 31;
-    if (tile >= ntiles) return;  // warp-uniform
-    const int i = row_lo + tile * kTile + lane;
-    const bool valid = i < row_hi;
-    double xi = 0.0, yi = 0.0;
-    if (valid) {
-        double2 v = xy[i];
-        xi = v.x;
-        yi = v.y;
-    }
-    int R = valid ? i + 1 : n;   // next right candidate
-    int L = valid ? i - 1 : -1;  // next left candidate
-    Sums s{0.0, 0.0, 0.0};
-
-    for (int b = 0; b < m; b++) {
-        const double h = __ldg(hg + b);
-        // Right side: x[R] - x_i is non-decreasing in R.  4-wide fast path:
-        // if the 4th candidate is inside, all four are (monotone order).
-        while (R + 3 < n) {
-            double2 v0 = xy[R], v1 = xy[R + 1], v2 = xy[R + 2], v3 = xy[R + 3];
-            double d3 = v3.x - xi;
-            if (!inside<KERN>(d3, h)) break;
-            acc<KERN>(s, v0.y, v0.x - xi);
-            acc<KERN>(s, v1.y, v1.x - xi);
-            acc<KERN>(s, v2.y, v2.x - xi);
-            acc<KERN>(s, v3.y, d3);
-            R += 4;
-        }
-        while (R < n) {
-            double2 v = xy[R];
-            double d = v.x - xi;
-            if (!inside<KERN>(d, h)) break;
-            acc<KERN>(s, v.y, d);
-            R++;
-        }
-        // Left side: x_i - x[L] is non-decreasing as L decreases.
-        while (L >= 3) {
-            double2 v0 = xy[L], v1 = xy[L - 1], v2 = xy[L - 2], v3 = xy[L - 3];
-            double d3 = xi - v3.x;
-            if (!inside<KERN>(d3, h)) break;
-            acc<KERN>(s, v0.y, xi - v0.x);
-            acc<KERN>(s, v1.y, xi - v1.x);
-            acc<KERN>(s, v2.y, xi - v2.x);
-            acc<KERN>(s, v3.y, d3);
-            L -= 4;
-        }
-        while (L >= 0) {
-            double2 v = xy[L];
-            double d = xi - v.x;
-            if (!inside<KERN>(d, h)) break;
-            acc<KERN>(s, v.y, d);
-            L--;
-        }
-
-        // a4: LOO estimate (Eq.(2)); 0.75 and 1/h^2 cancel (reading Q5).
-        const int c = (R - i - 1) + (i - L - 1);
-        const bool M = valid && c > 0;  // Q6
-        double e2 = 0.0;
-        if (M) {
-            double g;
-            if (KERN == KR_UNIFORM) {
-                g = s.sy / (double)c;
-            } else {
-                const double hk = (KERN == KR_EPANECHNIKOV) ? h * h : h;
-                double num = fma(hk, s.sy, -s.sy1);
-                double den = fma(hk, (double)c, -s.s1);
-                // Q14 conditioning guard: the decomposition cancels when every
-                // in-window point sits near the edge; recompute directly over
-                // the contiguous window [L+1, R-1] \ {i} with exact factors.
-                if (!(den >= 0x1p-20 * hk * (double)c)) {
-                    num = 0.0;
-                    den = 0.0;
-                    for (int q = L + 1; q < R; q++) {
-                        if (q == i) continue;
-                        double2 v = xy[q];
-                        double d = fabs(v.x - xi);
-                        double w = (KERN == KR_EPANECHNIKOV) ? (h - d) * (h + d) : (h - d);
-                        num = fma(v.y, w, num);
-                        den += w;
-                    }
-                }
-                g = num / den;
-            }
-            const double e = yi - g;
-            e2 = e * e;
-        }
-        // a5 (warp level): lanes are rows; fixed shuffle tree.
-        e2 = warp_sum(e2);
-        const unsigned ball = __ballot_sync(0xffffffffu, M);
-        if (lane == 0) {
-            tileS[(size_t)b * ntiles + tile] = e2;
-            tileN[(size_t)b * ntiles + tile] = (uint8_t)__popc(ball);
-        }
-    }
-}
-
 // ---------------------------------------------------------------------------
 // a5: fixed-order column reduction of the tile partials (the paper's
 // "summation reduction ... performed k times", P@23970, as one launch).
@@ -323,13 +191,14 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
         set_cuda_error("cub::DeviceRadixSort::SortPairs(size query)", (int)e);
         return false;
     }
-    const int64_t ntiles = (n + kTile - 1) / kTile;
+    const int64_t ntiles = max_tiles(n);
     size_t off = 0;
     L->keys_in = off;  off = align256(off + sizeof(uint64_t) * (size_t)n);
     L->keys_out = off; off = align256(off + sizeof(uint64_t) * (size_t)n);
     L->vals_in = off;  off = align256(off + sizeof(uint32_t) * (size_t)n);
     L->vals_out = off; off = align256(off + sizeof(uint32_t) * (size_t)n);
-    L->xy = off;       off = align256(off + sizeof(double2) * (size_t)n);
+    L->xy = off;       off = align256(off + sizeof(double2) * ((size_t)n + 2 * kPad));
+    L->counter = off;  off = align256(off + sizeof(int));
     L->tileS = off;    off = align256(off + sizeof(double) * (size_t)ntiles * (size_t)m);
     L->tileN = off;    off = align256(off + sizeof(uint8_t) * (size_t)ntiles * (size_t)m);
     L->status = off;   off = align256(off + 2 * sizeof(unsigned));
@@ -340,6 +209,34 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     return true;
 }
 
+// Rows per lane-group: G lanes share one row (both sides split by residue
+// class).  Small shards need G > 1 to fill 148 SMs with warps.
+int sweep_G(int64_t rows)
+{
+    static int forced = -1;
+    if (forced < 0) {
+        const char *e = getenv("KRCV_SWEEP_G");
+        int g = e ? atoi(e) : 0;
+        forced = (g == 1 || g == 2 || g == 4 || g == 8) ? g : 0;
+    }
+    if (forced) return forced;
+    if (rows <= kG4Rows) return 4;
+    if (rows <= kG2Rows) return 2;
+    return 1;
+}
+
+static int64_t tiles_for(int64_t rows, int G) { return (rows * G + 31) / 32; }
+
+// Upper bound of tile slots over every shard size rows <= n (G shrinks as
+// rows grow, so the maximum is at a threshold or at n) and any forced G.
+int64_t max_tiles(int64_t n)
+{
+    int64_t t = tiles_for(n, sweep_G(n));
+    t = t > tiles_for(n < kG4Rows ? n : kG4Rows, 4) ? t : tiles_for(n < kG4Rows ? n : kG4Rows, 4);
+    t = t > tiles_for(n < kG2Rows ? n : kG2Rows, 2) ? t : tiles_for(n < kG2Rows ? n : kG2Rows, 2);
+    return t > tiles_for(n, sweep_G(n)) ? t : tiles_for(n, sweep_G(n));
+}
+
 static int grid_for(int64_t work, int threads)
 {
     int64_t b = (work + threads - 1) / threads;
@@ -348,12 +245,64 @@ static int grid_for(int64_t work, int threads)
     return (int)b;
 }
 
-template <int KERN>
-static void launch_sweep(const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
-                         double *tileS, uint8_t *tileN, cudaStream_t st)
+// Sweep variant: 0 = split (G lanes per row), 1 = gxg (G lanes x G rows).
+int sweep_variant()
 {
-    const int blocks = (ntiles + kSweepWarps - 1) / kSweepWarps;
-    sweep_kernel<KERN><<<blocks, kSweepThreads, 0, st>>>(xy, n, h, m, lo, hi, ntiles, tileS, tileN);
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("KRCV_SWEEP");
+        v = (e && e[0] == 's') ? 0 : 1;
+    }
+    return v;
+}
+
+template <int KERN, int G, bool GXG>
+static void launch_sweep_g(const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
+                           double *tileS, uint8_t *tileN, int *counter, cudaStream_t st)
+{
+    static int resident = 0;  // CTAs per SM at full occupancy (persistent grid)
+    if (!resident) {
+        int b = 0;
+        if (GXG)
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sweep_gxg_kernel<KERN, G>, kSweepThreads, 0);
+        else
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sweep_kernel<KERN, G>, kSweepThreads, 0);
+        resident = b > 0 ? b : 1;
+    }
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (sms <= 0) sms = 148;
+    }
+    int blocks = (ntiles + kSweepWarps - 1) / kSweepWarps;
+    if (blocks > sms * resident) blocks = sms * resident;
+    if (GXG)
+        sweep_gxg_kernel<KERN, G><<<blocks, kSweepThreads, 0, st>>>(xy, n, h, m, lo, hi, ntiles, tileS, tileN,
+                                                                    counter);
+    else
+        sweep_kernel<KERN, G><<<blocks, kSweepThreads, 0, st>>>(xy, n, h, m, lo, hi, ntiles, tileS, tileN, counter);
+}
+
+template <int KERN>
+static void launch_sweep(int G, const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
+                         double *tileS, uint8_t *tileN, int *counter, cudaStream_t st)
+{
+    if (sweep_variant() == 1) {
+        switch (G) {
+        case 1: launch_sweep_g<KERN, 1, true>(xy, n, h, m, lo, hi, ntiles, tileS, tileN, counter, st); break;
+        case 2: launch_sweep_g<KERN, 2, true>(xy, n, h, m, lo, hi, ntiles, tileS, tileN, counter, st); break;
+        default: launch_sweep_g<KERN, 4, true>(xy, n, h, m, lo, hi, ntiles, tileS, tileN, counter, st); break;
+        }
+        return;
+    }
+    switch (G) {
+    case 1: launch_sweep_g<KERN, 1, false>(xy, n, h, m, lo, hi, ntiles, tileS, tileN, counter, st); break;
+    case 2: launch_sweep_g<KERN, 2, false>(xy, n, h, m, lo, hi, ntiles, tileS, tileN, counter, st); break;
+    case 4: launch_sweep_g<KERN, 4, false>(xy, n, h, m, lo, hi, ntiles, tileS, tileN, counter, st); break;
+    default: launch_sweep_g<KERN, 8, false>(xy, n, h, m, lo, hi, ntiles, tileS, tileN, counter, st); break;
+    }
 }
 
 // Optional stage timing (kr_profile_enable / kr_profile_read), thread-local.
@@ -432,7 +381,8 @@ extern "C" int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n
     uint64_t *keys_out = reinterpret_cast<uint64_t *>(ws + L.keys_out);
     uint32_t *vals_in = reinterpret_cast<uint32_t *>(ws + L.vals_in);
     uint32_t *vals_out = reinterpret_cast<uint32_t *>(ws + L.vals_out);
-    double2 *xy = reinterpret_cast<double2 *>(ws + L.xy);
+    double2 *xy = reinterpret_cast<double2 *>(ws + L.xy) + kPad;  // first real record
+    int *counter = reinterpret_cast<int *>(ws + L.counter);
     double *tileS = reinterpret_cast<double *>(ws + L.tileS);
     uint8_t *tileN = reinterpret_cast<uint8_t *>(ws + L.tileN);
     unsigned *status = reinterpret_cast<unsigned *>(ws + L.status);
@@ -441,7 +391,9 @@ extern "C" int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n
     // Rows of this shard in sorted order.
     const int lo = (int)(((int64_t)shard * n) / nshards);
     const int hi = (int)(((int64_t)(shard + 1) * n) / nshards);
-    const int ntiles = (hi - lo + kTile - 1) / kTile;
+    int G = sweep_G(hi - lo);
+    if (sweep_variant() == 1 && G > 4) G = 4;
+    const int ntiles = sweep_variant() == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G);
 
     int64_t launches = 0;
     prof_mark(0, st);
@@ -452,20 +404,20 @@ extern "C" int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n
     e = cub::DeviceRadixSort::SortPairs(ws + L.cub, cub_bytes, keys_in, keys_out, vals_in, vals_out,
                                         nn, 0, 64, st);
     if (e != cudaSuccess) { set_cuda_error("cub::DeviceRadixSort::SortPairs", (int)e); return KR_ECUDA; }
-    gather_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, vals_out, nn, xy);
+    gather_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, vals_out, nn, xy, counter);
     launches += 2 + cub_sort_launches(n);
     prof_mark(1, st);
     if (ntiles > 0) {
         launches += 1;
         switch (kernel) {
         case KR_UNIFORM:
-            launch_sweep<KR_UNIFORM>(xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, st);
+            launch_sweep<KR_UNIFORM>(G, xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, counter, st);
             break;
         case KR_EPANECHNIKOV:
-            launch_sweep<KR_EPANECHNIKOV>(xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, st);
+            launch_sweep<KR_EPANECHNIKOV>(G, xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, counter, st);
             break;
         default:
-            launch_sweep<KR_TRIANGULAR>(xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, st);
+            launch_sweep<KR_TRIANGULAR>(G, xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, counter, st);
             break;
         }
     }

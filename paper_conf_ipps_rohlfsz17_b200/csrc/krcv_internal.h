@@ -7,14 +7,18 @@
 
 namespace krcv {
 
-// Rows per warp tile in the sweep kernel (one sorted row per lane).
-constexpr int kTile = 32;
+// Shard sizes (rows) up to which the sweep uses G = 4 / G = 2 lanes per row.
+constexpr int64_t kG4Rows = 60000;
+constexpr int64_t kG2Rows = 250000;
+int sweep_G(int64_t rows);
+int64_t max_tiles(int64_t n);
 
 // Byte layout of the device workspace (kr_workspace_bytes / kr_cv_shard_async).
 struct WsLayout {
     size_t keys_in, keys_out;   // uint64 [n]  order-preserving keys of x
     size_t vals_in, vals_out;   // uint32 [n]  original indices
-    size_t xy;                  // double2 [n] (x, y) in sorted order
+    size_t xy;                  // double2 [n + 2 kPad] (x, y) in sorted order, +-inf sentinels
+    size_t counter;             // int: sweep tile counter
     size_t tileS;               // double  [m][ntiles]  per-tile sum of M e^2
     size_t tileN;               // uint8   [m][ntiles]  per-tile sum of M
     size_t status;              // uint32  [2]  n_bad_grid, n_nonfinite

@@ -1,0 +1,37 @@
+"""Summarise an .ncu-rep (raw page) into the metrics we track."""
+import csv, subprocess, sys, json
+
+KEYS = [
+    "gpu__time_duration.sum", "sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active",
+    "sm__inst_executed_pipe_fp64.avg.pct_of_peak_sustained_active",
+    "smsp__inst_executed.sum", "smsp__thread_inst_executed_per_inst_executed.ratio",
+    "sm__warps_active.avg.pct_of_peak_sustained_active", "smsp__issue_active.avg.pct_of_peak_sustained_active",
+    "l1tex__data_pipe_lsu_wavefronts.sum.pct_of_peak_sustained_elapsed", "l1tex__t_sector_hit_rate.pct",
+    "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum", "l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum",
+    "dram__bytes_read.sum", "dram__bytes_write.sum", "lts__t_bytes.sum", "launch__registers_per_thread",
+    "launch__grid_size", "launch__block_size", "sm__throughput.avg.pct_of_peak_sustained_elapsed",
+]
+STALLS = "smsp__average_warps_issue_stalled_"
+
+def main(path):
+    out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(out.splitlines()))
+    hdr, units = rows[0], rows[1]
+    res = []
+    for r in rows[2:]:
+        d = {}
+        name = r[hdr.index("Kernel Name")]
+        for k in KEYS:
+            if k in hdr:
+                d[k] = r[hdr.index(k)] + " " + units[hdr.index(k)]
+        st = {h[len(STALLS):].replace("_per_issue_active.ratio", ""): float(v)
+              for h, v in zip(hdr, r) if h.startswith(STALLS) and h.endswith("per_issue_active.ratio") and v}
+        d["stalls_per_issue"] = {k: round(v, 3) for k, v in sorted(st.items(), key=lambda kv: -kv[1]) if v > 0.02}
+        res.append((name[:80], d))
+    return res
+
+if __name__ == "__main__":
+    for name, d in main(sys.argv[1]):
+        print(name)
+        for k, v in d.items():
+            print("   ", k, v)
