@@ -27,6 +27,43 @@ class CVResult:
         return float(self.h[self.best])
 
 
+def shard_bounds(n: int, shard: int, nshards: int) -> tuple[int, int]:
+    """Sorted-order rows [floor(r n / P), floor((r+1) n / P)) of shard r of P
+    (the same rule kr_cv_shard_async applies on the device)."""
+    if not (0 <= shard < nshards):
+        raise ValueError("shard out of range")
+    return (shard * n) // nshards, ((shard + 1) * n) // nshards
+
+
+def allreduce_partial(partial, group=None) -> None:
+    """The path's one exchange step: all-reduce(SUM) of the
+    2m+2 partial vector [S | n_eff | n_bad_grid | n_nonfinite]; every entry
+    is additive, so the reduced vector is the unsharded one."""
+    import torch.distributed as dist
+
+    if dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
+        dist.all_reduce(partial, op=dist.ReduceOp.SUM, group=group)
+
+
+def finalize_partial(partial, n: int, m: int):
+    """CV = S/n, n_eff and the arg-min from a reduced partial vector.  CUDA
+    tensors are finalized on the device (kr_finalize_async), CPU tensors with
+    the host entry point kr_finalize.  Returns (cv, neff, best)."""
+    import torch
+
+    if partial.is_cuda:
+        cv = torch.empty(m, dtype=torch.float64, device=partial.device)
+        neff = torch.empty(m, dtype=torch.int64, device=partial.device)
+        bs = torch.empty(2, dtype=torch.int32, device=partial.device)
+        krcv.kr_finalize_async(partial, n, m, cv, neff, bs)
+        bs = bs.cpu()
+        if int(bs[1]) != krcv.KR_OK:
+            raise krcv.KrcvError(int(bs[1]), "device status")
+        return cv, neff, int(bs[0])
+    cv, neff, best = krcv.kr_finalize(partial.detach().numpy(), n, m)
+    return torch.from_numpy(cv), torch.from_numpy(neff), best
+
+
 class GridSearch:
     """Reusable device plan for one (n, m, kernel) on one GPU / one rank.
 
@@ -61,9 +98,7 @@ class GridSearch:
             raise ValueError("x, y must have n elements")
         krcv.kr_cv_shard_async(d_x, d_y, self.d_h, self.kernel, self.rank, self.world, self.partial, self.ws)
         if self.world > 1:
-            import torch.distributed as dist
-
-            dist.all_reduce(self.partial, op=dist.ReduceOp.SUM, group=self.group)
+            allreduce_partial(self.partial, self.group)
         krcv.kr_finalize_async(self.partial, self.n, self.m, self.cv, self.neff, self.best_status)
 
     def result(self) -> CVResult:

@@ -24,19 +24,13 @@
 #include "krcv_internal.h"
 #include "krcv_sweep.cuh"
 #include "krcv_sweep_gxg.cuh"
+#include "krcv_sort.cuh"
 
 namespace krcv {
 
 // ---------------------------------------------------------------------------
 // a1: pack + device-side validation
 // ---------------------------------------------------------------------------
-__device__ __forceinline__ uint64_t order_key(double v)
-{
-    // IEEE-754 total order on non-NaN values as an unsigned integer.
-    uint64_t u = static_cast<uint64_t>(__double_as_longlong(v));
-    return (u & 0x8000000000000000ull) ? ~u : (u | 0x8000000000000000ull);
-}
-
 __global__ void pack_kernel(const double *__restrict__ x, const double *__restrict__ y, int n,
                             const double *__restrict__ h, int m,
                             uint64_t *__restrict__ keys, uint32_t *__restrict__ vals,
@@ -193,10 +187,11 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     }
     const int64_t ntiles = max_tiles(n);
     size_t off = 0;
-    L->keys_in = off;  off = align256(off + sizeof(uint64_t) * (size_t)n);
-    L->keys_out = off; off = align256(off + sizeof(uint64_t) * (size_t)n);
-    L->vals_in = off;  off = align256(off + sizeof(uint32_t) * (size_t)n);
-    L->vals_out = off; off = align256(off + sizeof(uint32_t) * (size_t)n);
+    const size_t npad = (size_t)((n + kChunk - 1) / kChunk) * kChunk;  // chunked rank sort
+    L->keys_in = off;  off = align256(off + sizeof(uint64_t) * npad);
+    L->keys_out = off; off = align256(off + sizeof(uint64_t) * npad);
+    L->vals_in = off;  off = align256(off + sizeof(uint32_t) * npad);
+    L->vals_out = off; off = align256(off + sizeof(uint32_t) * npad);
     L->xy = off;       off = align256(off + sizeof(double2) * ((size_t)n + 2 * kPad));
     L->counter = off;  off = align256(off + sizeof(int));
     L->tileS = off;    off = align256(off + sizeof(double) * (size_t)ntiles * (size_t)m);
@@ -209,9 +204,11 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     return true;
 }
 
-// Rows per lane-group: G lanes share one row (both sides split by residue
-// class).  Small shards need G > 1 to fill 148 SMs with warps.
-int sweep_G(int64_t rows)
+// Lanes per row group.  Measured on B200 (profiles/): G = 4
+// is fastest for both sweep variants on C2-C5 (G = 1/2 leave the FP64 pipe
+// idle at 1-2 warps per scheduler on small shards; G = 8 adds epilogue and
+// combine overhead).  KRCV_SWEEP_G overrides (1, 2, 4; 8 for split).
+int sweep_G(int64_t /*rows*/)
 {
     static int forced = -1;
     if (forced < 0) {
@@ -219,22 +216,19 @@ int sweep_G(int64_t rows)
         int g = e ? atoi(e) : 0;
         forced = (g == 1 || g == 2 || g == 4 || g == 8) ? g : 0;
     }
-    if (forced) return forced;
-    if (rows <= kG4Rows) return 4;
-    if (rows <= kG2Rows) return 2;
-    return 1;
+    return forced ? forced : 4;
 }
 
 static int64_t tiles_for(int64_t rows, int G) { return (rows * G + 31) / 32; }
 
-// Upper bound of tile slots over every shard size rows <= n (G shrinks as
-// rows grow, so the maximum is at a threshold or at n) and any forced G.
-int64_t max_tiles(int64_t n)
+// Upper bound of tile slots for any shard of n rows and either variant:
+// split uses 32/G rows per tile, gxg 32.
+int64_t max_tiles(int64_t n) { return tiles_for(n, sweep_G(n)); }
+
+static bool getenv_flag(const char *name)
 {
-    int64_t t = tiles_for(n, sweep_G(n));
-    t = t > tiles_for(n < kG4Rows ? n : kG4Rows, 4) ? t : tiles_for(n < kG4Rows ? n : kG4Rows, 4);
-    t = t > tiles_for(n < kG2Rows ? n : kG2Rows, 2) ? t : tiles_for(n < kG2Rows ? n : kG2Rows, 2);
-    return t > tiles_for(n, sweep_G(n)) ? t : tiles_for(n, sweep_G(n));
+    const char *e = getenv(name);
+    return e && e[0] && e[0] != '0';
 }
 
 static int grid_for(int64_t work, int threads)
@@ -245,15 +239,20 @@ static int grid_for(int64_t work, int threads)
     return (int)b;
 }
 
-// Sweep variant: 0 = split (G lanes per row), 1 = gxg (G lanes x G rows).
-int sweep_variant()
+// Sweep variant for a shard of `rows` rows: 0 = split (G lanes per row),
+// 1 = gxg (G lanes x G adjacent rows with shared moments).  gxg halves the
+// C4 sweep (1e6 rows) but degrades on heavy-tailed data with few rows per
+// unit of x (C5) and on small shards (C2); measured crossover ~4e5 rows
+// (DESIGN.md §6).  KRCV_SWEEP=split|gxg overrides.
+int sweep_variant(int64_t rows)
 {
     static int v = -1;
     if (v < 0) {
         const char *e = getenv("KRCV_SWEEP");
-        v = (e && e[0] == 's') ? 0 : 1;
+        v = !e ? 2 : (e[0] == 's' ? 0 : (e[0] == 'g' ? 1 : 2));
     }
-    return v;
+    if (v != 2) return v;
+    return rows >= kGxgRows ? 1 : 0;
 }
 
 template <int KERN, int G, bool GXG>
@@ -289,7 +288,7 @@ template <int KERN>
 static void launch_sweep(int G, const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
                          double *tileS, uint8_t *tileN, int *counter, cudaStream_t st)
 {
-    if (sweep_variant() == 1) {
+    if (sweep_variant(hi - lo) == 1) {
         switch (G) {
         case 1: launch_sweep_g<KERN, 1, true>(xy, n, h, m, lo, hi, ntiles, tileS, tileN, counter, st); break;
         case 2: launch_sweep_g<KERN, 2, true>(xy, n, h, m, lo, hi, ntiles, tileS, tileN, counter, st); break;
@@ -391,21 +390,31 @@ extern "C" int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n
     // Rows of this shard in sorted order.
     const int lo = (int)(((int64_t)shard * n) / nshards);
     const int hi = (int)(((int64_t)(shard + 1) * n) / nshards);
+    const int variant = sweep_variant(hi - lo);
     int G = sweep_G(hi - lo);
-    if (sweep_variant() == 1 && G > 4) G = 4;
-    const int ntiles = sweep_variant() == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G);
+    if (variant == 1 && G > 4) G = 4;
+    const int ntiles = variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G);
 
     int64_t launches = 0;
     prof_mark(0, st);
     cudaError_t e = cudaMemsetAsync(status, 0, 2 * sizeof(unsigned), st);
     if (e != cudaSuccess) { set_cuda_error("cudaMemsetAsync(status)", (int)e); return KR_ECUDA; }
-    pack_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, nn, d_h, m, keys_in, vals_in, status);
-    size_t cub_bytes = L.cub_bytes;
-    e = cub::DeviceRadixSort::SortPairs(ws + L.cub, cub_bytes, keys_in, keys_out, vals_in, vals_out,
-                                        nn, 0, 64, st);
-    if (e != cudaSuccess) { set_cuda_error("cub::DeviceRadixSort::SortPairs", (int)e); return KR_ECUDA; }
-    gather_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, vals_out, nn, xy, counter);
-    launches += 2 + cub_sort_launches(n);
+    if (n <= kRankSortMaxN && !getenv_flag("KRCV_CUB_SORT")) {
+        // a1 + a2 fused: chunk bitonic sort + rank-by-search scatter (krcv_sort.cuh)
+        const int nchunks = (int)((n + kChunk - 1) / kChunk);
+        chunk_sort_kernel<<<nchunks, kChunkThreads, 0, st>>>(d_x, d_y, nn, d_h, m, keys_in, vals_in, status);
+        rank_scatter_kernel<<<(nchunks * kChunk + 255) / 256, 256, 0, st>>>(keys_in, vals_in, nn, nchunks, d_x,
+                                                                          d_y, xy, counter);
+        launches += 2;
+    } else {
+        pack_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, nn, d_h, m, keys_in, vals_in, status);
+        size_t cub_bytes = L.cub_bytes;
+        e = cub::DeviceRadixSort::SortPairs(ws + L.cub, cub_bytes, keys_in, keys_out, vals_in, vals_out,
+                                            nn, 0, 64, st);
+        if (e != cudaSuccess) { set_cuda_error("cub::DeviceRadixSort::SortPairs", (int)e); return KR_ECUDA; }
+        gather_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, vals_out, nn, xy, counter);
+        launches += 2 + cub_sort_launches(n);
+    }
     prof_mark(1, st);
     if (ntiles > 0) {
         launches += 1;

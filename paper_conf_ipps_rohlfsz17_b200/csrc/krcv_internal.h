@@ -7,10 +7,10 @@
 
 namespace krcv {
 
-// Shard sizes (rows) up to which the sweep uses G = 4 / G = 2 lanes per row.
-constexpr int64_t kG4Rows = 60000;
-constexpr int64_t kG2Rows = 250000;
+// Shards with at least this many rows use the gxg sweep variant.
+constexpr int64_t kGxgRows = 400000;
 int sweep_G(int64_t rows);
+int sweep_variant(int64_t rows);
 int64_t max_tiles(int64_t n);
 
 // Byte layout of the device workspace (kr_workspace_bytes / kr_cv_shard_async).

@@ -67,12 +67,14 @@ __device__ __forceinline__ void acc(Sums &s, double yv, double d)
 }
 
 // Consume one quad of a side.  p = next candidate index of this lane's
-// residue class, step = +G (right) or -G (left).  Returns true if the side
-// may still have in-window elements for this bandwidth.
+// residue class, step = +G (right) or -G (left).  Elements alternate between
+// two accumulator sets (sa: 0, 2; sb: 1, 3) to halve the dependency chains.
+// Returns true if the side may still have in-window elements for this
+// bandwidth.
 template <int KERN, int G, bool RIGHT>
-__device__ __forceinline__ bool quad(const double2 *__restrict__ xy, int &p, int &cnt, Sums &s,
-                                     double xi, double h, const double2 &v0, const double2 &v1,
-                                     const double2 &v2, const double2 &v3)
+__device__ __forceinline__ bool quad(int &p, int &cnt, Sums &sa, Sums &sb, double xi, double h,
+                                     const double2 &v0, const double2 &v1, const double2 &v2,
+                                     const double2 &v3)
 {
     const double d0 = RIGHT ? v0.x - xi : xi - v0.x;
     const double d1 = RIGHT ? v1.x - xi : xi - v1.x;
@@ -80,25 +82,25 @@ __device__ __forceinline__ bool quad(const double2 *__restrict__ xy, int &p, int
     const double d3 = RIGHT ? v3.x - xi : xi - v3.x;
     constexpr int step = RIGHT ? G : -G;
     if (inside<KERN>(d3, h)) {  // monotone: all four inside
-        acc<KERN>(s, v0.y, d0);
-        acc<KERN>(s, v1.y, d1);
-        acc<KERN>(s, v2.y, d2);
-        acc<KERN>(s, v3.y, d3);
+        acc<KERN>(sa, v0.y, d0);
+        acc<KERN>(sb, v1.y, d1);
+        acc<KERN>(sa, v2.y, d2);
+        acc<KERN>(sb, v3.y, d3);
         p += 4 * step;
         cnt += 4;
         return true;
     }
     // partial quad: the inside elements form a prefix
     if (inside<KERN>(d0, h)) {
-        acc<KERN>(s, v0.y, d0);
+        acc<KERN>(sa, v0.y, d0);
         p += step;
         cnt += 1;
         if (inside<KERN>(d1, h)) {
-            acc<KERN>(s, v1.y, d1);
+            acc<KERN>(sb, v1.y, d1);
             p += step;
             cnt += 1;
             if (inside<KERN>(d2, h)) {
-                acc<KERN>(s, v2.y, d2);
+                acc<KERN>(sa, v2.y, d2);
                 p += step;
                 cnt += 1;
             }
@@ -161,7 +163,7 @@ sweep_kernel(const double2 *__restrict__ xy, int n, const double *__restrict__ h
         }
         int R = i + 1 + k, L = i - 1 - k;  // this lane's next right / left candidates
         int cR = 0, cL = 0;                // this lane's in-window counts
-        Sums sR{0.0, 0.0, 0.0}, sL{0.0, 0.0, 0.0};
+        Sums sRa{0.0, 0.0, 0.0}, sRb{0.0, 0.0, 0.0}, sLa{0.0, 0.0, 0.0}, sLb{0.0, 0.0, 0.0};
 
         for (int b = 0; b < m; b++) {
             const double h = __ldg(hg + b);
@@ -180,18 +182,18 @@ sweep_kernel(const double2 *__restrict__ xy, int n, const double *__restrict__ h
                     c2 = xy[L - 2 * G];
                     c3 = xy[L - 3 * G];
                 }
-                if (rgo) rgo = quad<KERN, G, true>(xy, R, cR, sR, xi, h, a0, a1, a2, a3);
-                if (lgo) lgo = quad<KERN, G, false>(xy, L, cL, sL, xi, h, c0, c1, c2, c3);
+                if (rgo) rgo = quad<KERN, G, true>(R, cR, sRa, sRb, xi, h, a0, a1, a2, a3);
+                if (lgo) lgo = quad<KERN, G, false>(L, cL, sLa, sLb, xi, h, c0, c1, c2, c3);
             }
 
             // ---- a4: combine the row's G lanes, LOO estimate, squared error
             const int cRt = group_sum_i<G>(cR);
             const int cLt = group_sum_i<G>(cL);
-            const double sy = group_sum<G>(sR.sy + sL.sy);
+            const double sy = group_sum<G>((sRa.sy + sRb.sy) + (sLa.sy + sLb.sy));
             double s1 = 0.0, sy1 = 0.0;
             if (KERN != KR_UNIFORM) {
-                s1 = group_sum<G>(sR.s1 + sL.s1);
-                sy1 = group_sum<G>(sR.sy1 + sL.sy1);
+                s1 = group_sum<G>((sRa.s1 + sRb.s1) + (sLa.s1 + sLb.s1));
+                sy1 = group_sum<G>((sRa.sy1 + sRb.sy1) + (sLa.sy1 + sLb.sy1));
             }
             const int c = cRt + cLt;
             const bool M = valid && c > 0;  // reading Q6

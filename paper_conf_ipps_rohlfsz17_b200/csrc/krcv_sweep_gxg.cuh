@@ -49,6 +49,33 @@ __device__ __forceinline__ T reduce_scatter(const T (&v)[G], int k)
     }
 }
 
+// Moments of the elements that lie inside ALL G rows' windows, taken about
+// x0 = x of the group's first row: u = x_j - x0.  Row r (delta = x_r - x0)
+// recovers its own sums exactly in real arithmetic:
+//   sum (x_j - x_r)^2     = u2 - 2 delta u1 + delta^2 c
+//   sum y_j (x_j - x_r)^2 = y2 - 2 delta y1 + delta^2 y0
+// Such elements satisfy |x_j - x_r| < h for every row, so delta < h and the
+// shift adds no cancellation beyond a small constant factor.
+struct Shared {
+    double c, u1, u2, y0, y1, y2;
+};
+
+template <int KERN>
+__device__ __forceinline__ void sh_add(Shared &s, double yv, double u)
+{
+    s.c += 1.0;
+    s.y0 += yv;
+    if (KERN != KR_UNIFORM) {
+        s.u1 += u;
+        s.y1 = fma(yv, u, s.y1);
+        if (KERN == KR_EPANECHNIKOV) {
+            const double u2 = u * u;
+            s.u2 += u2;
+            s.y2 = fma(yv, u2, s.y2);
+        }
+    }
+}
+
 template <int KERN, int G>
 __global__ void __launch_bounds__(kSweepThreads)
 sweep_gxg_kernel(const double2 *__restrict__ xy, int n, const double *__restrict__ hg, int m,
@@ -88,6 +115,12 @@ sweep_gxg_kernel(const double2 *__restrict__ xy, int n, const double *__restrict
             sR[r] = Sums{0.0, 0.0, 0.0};
             sL[r] = Sums{0.0, 0.0, 0.0};
         }
+        // Shared-element moments.  Epanechnikov and uniform need only |d|^2
+        // or nothing, so both sides share one set; triangular needs the sign
+        // of (x_j - x_r), so it keeps one set per side.
+        Shared sh0{0, 0, 0, 0, 0, 0}, sh1{0, 0, 0, 0, 0, 0};
+        Shared &shR = sh0;
+        Shared &shL = (KERN == KR_TRIANGULAR) ? sh1 : sh0;
 
         for (int b = 0; b < m; b++) {
             const double h = __ldg(hg + b);
@@ -105,8 +138,24 @@ sweep_gxg_kernel(const double2 *__restrict__ xy, int n, const double *__restrict
 #pragma unroll
                     for (int q = 0; q < 4; q++) c[q] = xy[pL - q * G];
                 }
+                // Fast path (right): row 0 is the laggard; if its 4th element is
+                // inside and no row has already counted any of the quad, every
+                // row takes all four -> shared moments (7 FP64 per element for
+                // G pairs).
+                bool rfast = false;
+                double u3 = 0.0;
                 if (rgo) {
-                    bool lead_in = false;
+                    u3 = a[3].x - xr[0];
+                    rfast = pR >= nx[G - 1] && inside<KERN>(u3, h);
+                }
+                if (rfast) {
+#pragma unroll
+                    for (int q = 0; q < 4; q++) sh_add<KERN>(shR, a[q].y, q == 3 ? u3 : a[q].x - xr[0]);
+                    pR += 4 * G;
+#pragma unroll
+                    for (int r = 0; r < G; r++) nx[r] = pR;
+                } else if (rgo) {
+                    int ndone = 0;  // rows whose window ended: a prefix 0..ndone-1
 #pragma unroll
                     for (int r = 0; r < G; r++) {
                         int cnt = 0;
@@ -116,20 +165,35 @@ sweep_gxg_kernel(const double2 *__restrict__ xy, int n, const double *__restrict
                             const bool in = inside<KERN>(d, h);
                             cnt += in ? 1 : 0;
                             if (in && pR + q * G >= nx[r]) acc<KERN>(sR[r], a[q].y, d);
-                            if (r == G - 1 && q == 3) lead_in = in;
                         }
                         // first outside element of row r = pR + cnt*G, but only in
                         // the quad where row r's inside-prefix ends (cnt > 0);
                         // later quads of this bucket lie wholly outside row r.
                         if (cnt) nx[r] = max(nx[r], pR + cnt * G);
+                        if (cnt < 4) ndone = r + 1;
                     }
-                    pR += 4 * G;
-                    rgo = lead_in;
-                }
-                if (lgo) {
-                    bool lead_in = false;
+                    // continue from the laggard among the rows still inside;
+                    // jump over elements every active row has already counted
+                    rgo = ndone < G;
+                    int nxt = pR + 4 * G;
 #pragma unroll
-                    for (int r = 0; r < G; r++) {
+                    for (int r = 0; r < G; r++)
+                        if (r == ndone) nxt = max(nxt, nx[r]);
+                    pR = nxt;
+                }
+                // Fast path (left): row G-1 is the laggard.
+                bool lfast = false;
+                if (lgo) lfast = pL <= pv[0] && inside<KERN>(xr[G - 1] - c[3].x, h);
+                if (lfast) {
+#pragma unroll
+                    for (int q = 0; q < 4; q++) sh_add<KERN>(shL, c[q].y, c[q].x - xr[0]);
+                    pL -= 4 * G;
+#pragma unroll
+                    for (int r = 0; r < G; r++) pv[r] = pL;
+                } else if (lgo) {
+                    int nact = G;  // rows still inside: a prefix 0..nact-1
+#pragma unroll
+                    for (int r = G - 1; r >= 0; r--) {
                         int cnt = 0;
 #pragma unroll
                         for (int q = 0; q < 4; q++) {
@@ -137,12 +201,16 @@ sweep_gxg_kernel(const double2 *__restrict__ xy, int n, const double *__restrict
                             const bool in = inside<KERN>(d, h);
                             cnt += in ? 1 : 0;
                             if (in && pL - q * G <= pv[r]) acc<KERN>(sL[r], c[q].y, d);
-                            if (r == 0 && q == 3) lead_in = in;
                         }
                         if (cnt) pv[r] = min(pv[r], pL - cnt * G);
+                        if (cnt < 4) nact = r;
                     }
-                    pL -= 4 * G;
-                    lgo = lead_in;
+                    lgo = nact > 0;
+                    int nxt = pL - 4 * G;
+#pragma unroll
+                    for (int r = 0; r < G; r++)
+                        if (r == nact - 1) nxt = min(nxt, pv[r]);
+                    pL = nxt;
                 }
             }
 
@@ -153,9 +221,18 @@ sweep_gxg_kernel(const double2 *__restrict__ xy, int n, const double *__restrict
             for (int r = 0; r < G; r++) {
                 cRv[r] = (nx[r] - first_n[r]) / G;
                 cLv[r] = (first_p[r] - pv[r]) / G;
-                syv[r] = sR[r].sy + sL[r].sy;
+                syv[r] = sR[r].sy + sL[r].sy + shR.y0;
                 s1v[r] = sR[r].s1 + sL[r].s1;
                 sy1v[r] = sR[r].sy1 + sL[r].sy1;
+                const double dl = xr[r] - xr[0];  // delta_r
+                if (KERN == KR_EPANECHNIKOV) {
+                    s1v[r] += fma(dl * dl, shR.c, fma(-2.0 * dl, shR.u1, shR.u2));
+                    sy1v[r] += fma(dl * dl, shR.y0, fma(-2.0 * dl, shR.y1, shR.y2));
+                } else if (KERN == KR_TRIANGULAR) {
+                    syv[r] += shL.y0;
+                    s1v[r] += fma(-dl, shR.c, shR.u1) + fma(dl, shL.c, -shL.u1);
+                    sy1v[r] += fma(-dl, shR.y0, shR.y1) + fma(dl, shL.y0, -shL.y1);
+                }
             }
             const int cRt = reduce_scatter<G>(cRv, k);
             const int cLt = reduce_scatter<G>(cLv, k);

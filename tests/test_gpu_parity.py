@@ -229,3 +229,23 @@ def test_grid_sizes(m):
     x, y = workloads.draw_xy("paper", 900, 1)
     h = workloads.grid_default(x, m)
     _check(x, y, h, E)
+
+
+@pytest.mark.parametrize("cfg,n", [("C2", 20000), ("C5", 5000), ("C1", 1000), ("C2", 4097), ("C2", 131072)])
+def test_rank_sort_matches_cub_sort_bitwise(cfg, n, monkeypatch):
+    """The two a2 implementations (chunked rank sort for n <= 131072, CUB
+    onesweep otherwise) produce the same total order (x, index), hence
+    bit-identical CV curves."""
+    x, y, h, k = workloads.make(cfg, seed=5, n=n)
+    a = _gpu(x, y, h, k)
+    monkeypatch.setenv("KRCV_CUB_SORT", "1")
+    b = _gpu(x, y, h, k)
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1]) and a[2] == b[2]
+
+
+def test_rank_sort_heavy_duplicates():
+    """Many equal x (ties broken by original index) through the rank sort."""
+    x, y = workloads.draw_xy("paper", 9000, 2)
+    x = np.floor(x * 7) / 7
+    h = workloads.grid_default(x, 20)
+    _check(x, y, h, E)
