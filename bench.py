@@ -56,6 +56,8 @@ def parse():
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--algo", default="auto", choices=["auto", "sweep", "prefix"],
+                    help="KR_ALGO_* for every call (sets KRCV_ALGO before the library loads)")
     ap.add_argument("--cpu-seconds", type=float, default=8.0,
                     help="target wall seconds of the bounded oracle sample")
     return ap.parse_args()
@@ -241,7 +243,7 @@ def run_ours(args):
     krcv.kr_profile_enable(True)
     starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
     ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    sweep_ms, sort_ms = [], []
+    sweep_ms, sort_ms, build_ms = [], [], []
     launches = 0
     barrier()
     torch.cuda.synchronize()
@@ -251,8 +253,9 @@ def run_ours(args):
             starts[s].record(stream)
             plan.run(d_x, d_y)
             ends[s].record(stream)
-            a, b, _c = krcv.kr_profile_read()  # syncs on this step's events
+            a, pb, b, _c = krcv.kr_profile_read()  # syncs on this step's events
             sort_ms.append(a)
+            build_ms.append(pb)
             sweep_ms.append(b)
             launches += krcv.kr_launch_count() + 1  # + finalize kernel
         torch.cuda.synchronize()
@@ -302,7 +305,9 @@ def run_ours(args):
                      "peak_note": "FP64: 148 SM x 64 FMA lanes x 2 flop x 1965 MHz (derived, DESIGN.md)",
                      "flops_per_launch": flops_per_launch, "sweep_ms": sweep_total / args.steps,
                      "sweep_share_of_step": (sweep_total / args.steps) / (total_ms / args.steps)},
-        "stage_ms": {"pack_sort_gather": sum(sort_ms) / args.steps, "sweep": sum(sweep_ms) / args.steps},
+        "stage_ms": {"pack_sort_gather": sum(sort_ms) / args.steps, "prefix_build": sum(build_ms) / args.steps,
+                     "sweep": sum(sweep_ms) / args.steps},
+        "algo": {1: "sweep", 2: "prefix"}.get(krcv.kr_last_algo(), "?"),
         "result": {"best": res.best, "h_best": float(h[res.best]), "cv_best": float(res.cv[res.best])},
         "e2e": e2e,
         "clocks": clk.summary(),
@@ -382,6 +387,8 @@ def e2e_measure(args, x, y, h, k, n, m, units, dev, rank, world, plan):
 
 def main():
     args = parse()
+    if args.algo != "auto":
+        os.environ["KRCV_ALGO"] = args.algo
     if args.impl == "reference":
         return run_reference(args)
     return run_ours(args)

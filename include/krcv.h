@@ -68,6 +68,23 @@ enum {
 
 #define KR_MAX_M 65536
 
+/* Algorithms (both compute the same CV curve):
+ *   KR_ALGO_SWEEP  the paper's per-row running sums (§III P@14010-14984,
+ *                  §IV.B P@21724-22104): every row visits its neighbours in
+ *                  distance order and adds them one by one as h grows --
+ *                  O(n^2) pair steps + O(n m) emits;
+ *   KR_ALGO_PREFIX window-prefix: the same running sums reached by exact
+ *                  boundary search on the sorted x and differences of
+ *                  double-double prefix moments --
+ *                  O(n m log) work, no per-pair step;
+ *   KR_ALGO_AUTO   the library's choice (currently KR_ALGO_PREFIX; the
+ *                  environment variable KRCV_ALGO=sweep|prefix overrides). */
+enum {
+    KR_ALGO_AUTO = 0,
+    KR_ALGO_SWEEP = 1,
+    KR_ALGO_PREFIX = 2
+};
+
 /* Length of the partial vector of the device path: [ S[0..m) | neff[0..m) |
  * n_bad_grid | n_nonfinite ].  S[b] = sum over the shard's rows of
  * M_i (y_i - g_{-i}(h_b))^2, neff[b] = sum of M_i (exact in fp64), and two
@@ -94,6 +111,11 @@ int kr_cv_grid(const double *x, const double *y, int64_t n,
 int kr_cv_grid_ex(const double *x, const double *y, int64_t n,
                   const double *h_grid, int32_t m, int32_t kernel,
                   double *cv_out, int64_t *neff_out, int32_t *best_out);
+
+/* kr_cv_grid_ex with an explicit algorithm (KR_ALGO_*; KR_EARG if unknown). */
+int kr_cv_grid_algo(const double *x, const double *y, int64_t n,
+                    const double *h_grid, int32_t m, int32_t kernel, int32_t algo,
+                    double *cv_out, int64_t *neff_out, int32_t *best_out);
 
 /* Host-side grid check (finite, > 0, non-decreasing, 1 <= m <= KR_MAX_M). */
 int kr_validate_grid(const double *h_grid, int32_t m);
@@ -124,6 +146,14 @@ int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n,
                       int32_t shard, int32_t nshards,
                       double *d_partial, void *d_workspace, size_t workspace_bytes,
                       void *cuda_stream);
+
+/* kr_cv_shard_async with an explicit algorithm (KR_ALGO_*; KR_EARG if
+ * unknown).  Same arguments, layout, ownership and errors otherwise. */
+int kr_cv_shard_algo_async(const double *d_x, const double *d_y, int64_t n,
+                           const double *d_h, int32_t m, int32_t kernel, int32_t algo,
+                           int32_t shard, int32_t nshards,
+                           double *d_partial, void *d_workspace, size_t workspace_bytes,
+                           void *cuda_stream);
 
 /*
  * kr_finalize -- host finalize of a partial vector already summed over all
@@ -160,15 +190,19 @@ const char *kr_last_cuda_error(void);
  * Optional stage timing for benchmarks (thread-local state).
  * kr_profile_enable(1): subsequent kr_cv_shard_async calls on this thread
  * record CUDA events on their stream around (a1+a2) pack+sort+gather,
- * (a3+a4) sweep and (a5) reduce.  Do not enable while capturing a graph.
- * kr_profile_read waits for the last call's events and writes ms[3]
- * = {sort, sweep, reduce} in milliseconds; returns KR_EARG if nothing was
- * recorded.  kr_launch_count returns the number of kernel launches the last
- * kr_cv_shard_async call on this thread enqueued (CUB passes included).
+ * the prefix build (window-prefix path only), (a3+a4) the sweep / window
+ * kernel and (a5) reduce.  Do not enable while capturing a graph.
+ * kr_profile_read waits for the last call's events and writes ms[4]
+ * = {sort, prefix_build, sweep, reduce} in milliseconds (prefix_build is ~0
+ * on the sweep path); returns KR_EARG if nothing was recorded.
+ * kr_launch_count returns the number of kernel launches the last
+ * kr_cv_shard_async call on this thread enqueued (CUB passes included);
+ * kr_last_algo the algorithm it ran (KR_ALGO_SWEEP or KR_ALGO_PREFIX).
  */
 int kr_profile_enable(int on);
 int kr_profile_read(float *ms);
 int64_t kr_launch_count(void);
+int32_t kr_last_algo(void);
 
 /* Library version, e.g. "krcv 0.1.0 sm_100a". */
 const char *kr_version(void);

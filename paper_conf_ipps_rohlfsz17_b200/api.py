@@ -72,7 +72,7 @@ class GridSearch:
     """
 
     def __init__(self, n: int, h, kernel="epanechnikov", device=None, rank: int = 0, world: int = 1,
-                 group=None):
+                 group=None, algo="auto"):
         import torch
 
         self.torch = torch
@@ -83,6 +83,7 @@ class GridSearch:
             raise krcv.KrcvError(st, "grid")
         self.n, self.m = int(n), int(h_host.shape[0])
         self.kernel = krcv._kernel_id(kernel)
+        self.algo = krcv._algo_id(algo)
         self.rank, self.world, self.group = int(rank), int(world), group
         self.h = h_host
         self.d_h = torch.as_tensor(h_host, device=self.device)
@@ -96,7 +97,8 @@ class GridSearch:
     def run(self, d_x, d_y) -> None:
         if d_x.numel() != self.n or d_y.numel() != self.n:
             raise ValueError("x, y must have n elements")
-        krcv.kr_cv_shard_async(d_x, d_y, self.d_h, self.kernel, self.rank, self.world, self.partial, self.ws)
+        krcv.kr_cv_shard_async(d_x, d_y, self.d_h, self.kernel, self.rank, self.world, self.partial, self.ws,
+                               algo=self.algo)
         if self.world > 1:
             allreduce_partial(self.partial, self.group)
         krcv.kr_finalize_async(self.partial, self.n, self.m, self.cv, self.neff, self.best_status)
@@ -110,7 +112,7 @@ class GridSearch:
 
 
 def cv_grid(x, y, h=None, m: int | None = None, kernel="epanechnikov", device=None, distributed: bool = False,
-            group=None) -> CVResult:
+            group=None, algo="auto") -> CVResult:
     """LOO-CV grid search.  x, y: numpy arrays or CUDA tensors; h: grid array,
     or None with m for the default grid (§IV P@16146).  With distributed=True
     every rank of the default (or given) process group must call it with the
@@ -130,6 +132,6 @@ def cv_grid(x, y, h=None, m: int | None = None, kernel="epanechnikov", device=No
     dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
     d_x = torch.as_tensor(x, dtype=torch.float64, device=dev).contiguous()
     d_y = torch.as_tensor(y, dtype=torch.float64, device=dev).contiguous()
-    plan = GridSearch(d_x.numel(), h, kernel, dev, rank, world, group)
+    plan = GridSearch(d_x.numel(), h, kernel, dev, rank, world, group, algo)
     plan.run(d_x, d_y)
     return plan.result()

@@ -25,6 +25,7 @@
 #include "krcv_sweep.cuh"
 #include "krcv_sweep_gxg.cuh"
 #include "krcv_sort.cuh"
+#include "krcv_prefix.cuh"
 
 namespace krcv {
 
@@ -196,6 +197,14 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     L->counter = off;  off = align256(off + sizeof(int));
     L->tileS = off;    off = align256(off + sizeof(double) * (size_t)ntiles * (size_t)m);
     L->tileN = off;    off = align256(off + sizeof(uint8_t) * (size_t)ntiles * (size_t)m);
+    // window-prefix path (krcv_prefix.cuh)
+    const size_t nch = (size_t)((n + kPfxCh - 1) / kPfxCh);
+    L->pstride = (int64_t)(((size_t)n + 1 + 15) & ~size_t(15));
+    L->nch = (int64_t)nch;
+    L->xs = off;       off = align256(off + sizeof(double) * ((size_t)n + 2 * kPad));
+    L->pfx = off;      off = align256(off + sizeof(double2) * kPfxMoments * (size_t)L->pstride);
+    L->ptot = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
+    L->poff = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
     L->status = off;   off = align256(off + 2 * sizeof(unsigned));
     L->cub = off;      off = align256(off + cub_bytes);
     L->cub_bytes = cub_bytes;
@@ -305,11 +314,15 @@ static void launch_sweep(int G, const double2 *xy, int n, const double *h, int m
 }
 
 // Optional stage timing (kr_profile_enable / kr_profile_read), thread-local.
+// Events: 0 start, 1 after pack+sort+gather, 2 after the prefix build (equal
+// to 1 on the sweep path), 3 after the sweep / window kernel, 4 after reduce.
+constexpr int kProfEvents = 5;
 struct Prof {
     bool on = false;
     bool recorded = false;
-    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+    cudaEvent_t ev[kProfEvents] = {nullptr, nullptr, nullptr, nullptr, nullptr};
     int64_t launches = 0;
+    int algo = 0;
 };
 static thread_local Prof g_prof;
 
@@ -326,6 +339,71 @@ static void prof_mark(int k, cudaStream_t st)
 // against the ncu launch list, profiles/.)
 static int64_t cub_sort_launches(int64_t n) { return n <= kCubSingleTile ? 1 : 2 + 64 / 8; }
 
+// KR_ALGO_AUTO: the window-prefix path does O(n m log) work against the
+// sweep's O(n^2); measured faster on every BASELINE config.
+// KRCV_ALGO=sweep|prefix overrides (benchmarks, A/B tests).
+int auto_algo(int64_t /*n*/, int64_t /*rows*/, int32_t /*m*/, int32_t /*kernel*/)
+{
+    static int forced = -1;
+    if (forced < 0) {
+        const char *e = getenv("KRCV_ALGO");
+        forced = !e ? 0 : (e[0] == 's' ? KR_ALGO_SWEEP : (e[0] == 'p' ? KR_ALGO_PREFIX : 0));
+    }
+    return forced ? forced : KR_ALGO_PREFIX;
+}
+
+template <int KERN>
+static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, char *ws, cudaStream_t st)
+{
+    double *xs = reinterpret_cast<double *>(ws + L.xs) + kPad;
+    double2 *P = reinterpret_cast<double2 *>(ws + L.pfx);
+    double2 *tot = reinterpret_cast<double2 *>(ws + L.ptot);
+    double2 *off = reinterpret_cast<double2 *>(ws + L.poff);
+    const int nch = (int)L.nch;
+    const int blocks = (nch + kPfxThreads - 1) / kPfxThreads;
+    pfx_chunk_kernel<KERN><<<blocks, kPfxThreads, 0, st>>>(xy, n, xs, tot, nch);
+    pfx_scan_kernel<KERN><<<1, kPfxScanThreads, 0, st>>>(tot, off, nch);
+    pfx_write_kernel<KERN><<<blocks, kPfxThreads, 0, st>>>(xy, n, off, nch, P, (int)L.pstride);
+}
+
+template <int KERN>
+static void launch_window(const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
+                          const WsLayout &L, char *ws, double *tileS, uint8_t *tileN, int *counter,
+                          cudaStream_t st)
+{
+    static int resident = 0;
+    if (!resident) {
+        int b = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel<KERN>, kWinThreads, 0);
+        resident = b > 0 ? b : 1;
+    }
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (sms <= 0) sms = 148;
+    }
+    // Split the bandwidth loop into nbc chunks until there are enough warp
+    // tasks to fill every SM (~kWinTasksPerSM resident warps each), keeping
+    // >= kWinMinBper bandwidths per chunk to amortise the cold searches.
+    const int64_t want = (int64_t)sms * kWinTasksPerSM;
+    int nbc = (int)((want + ntiles - 1) / ntiles);
+    nbc = nbc < 1 ? 1 : nbc;
+    const int max_nbc = (m + kWinMinBper - 1) / kWinMinBper;
+    if (nbc > max_nbc) nbc = max_nbc;
+    if (nbc < 1) nbc = 1;
+    const char *fe = getenv("KRCV_WIN_NBC");
+    if (fe && atoi(fe) > 0) nbc = atoi(fe) < m ? atoi(fe) : m;
+    const int64_t tasks = (int64_t)ntiles * nbc;
+    int blocks = (int)((tasks + kWinWarps - 1) / kWinWarps);
+    if (blocks > sms * resident) blocks = sms * resident;
+    const double *xs = reinterpret_cast<const double *>(ws + L.xs) + kPad;
+    const double2 *P = reinterpret_cast<const double2 *>(ws + L.pfx);
+    window_kernel<KERN><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc,
+                                                        tileS, tileN, counter);
+}
+
 }  // namespace krcv
 
 using namespace krcv;
@@ -340,9 +418,9 @@ extern "C" int kr_profile_enable(int on)
 extern "C" int kr_profile_read(float *ms)
 {
     if (!ms || !g_prof.recorded) return KR_EARG;
-    cudaError_t e = cudaEventSynchronize(g_prof.ev[3]);
+    cudaError_t e = cudaEventSynchronize(g_prof.ev[kProfEvents - 1]);
     if (e != cudaSuccess) { set_cuda_error("cudaEventSynchronize", (int)e); return KR_ECUDA; }
-    for (int k = 0; k < 3; k++) {
+    for (int k = 0; k < kProfEvents - 1; k++) {
         e = cudaEventElapsedTime(&ms[k], g_prof.ev[k], g_prof.ev[k + 1]);
         if (e != cudaSuccess) { set_cuda_error("cudaEventElapsedTime", (int)e); return KR_ECUDA; }
     }
@@ -350,6 +428,8 @@ extern "C" int kr_profile_read(float *ms)
 }
 
 extern "C" int64_t kr_launch_count(void) { return g_prof.launches; }
+
+extern "C" int32_t kr_last_algo(void) { return g_prof.algo; }
 
 extern "C" size_t kr_workspace_bytes(int64_t n, int32_t m)
 {
@@ -359,15 +439,16 @@ extern "C" size_t kr_workspace_bytes(int64_t n, int32_t m)
     return L.total;
 }
 
-extern "C" int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n,
-                                 const double *d_h, int32_t m, int32_t kernel,
-                                 int32_t shard, int32_t nshards,
-                                 double *d_partial, void *d_workspace, size_t workspace_bytes,
-                                 void *cuda_stream)
+extern "C" int kr_cv_shard_algo_async(const double *d_x, const double *d_y, int64_t n,
+                                      const double *d_h, int32_t m, int32_t kernel, int32_t algo,
+                                      int32_t shard, int32_t nshards,
+                                      double *d_partial, void *d_workspace, size_t workspace_bytes,
+                                      void *cuda_stream)
 {
     if (!d_x || !d_y || !d_h || !d_partial || !d_workspace) return KR_EARG;
     if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return KR_EARG;
     if (kernel != KR_UNIFORM && kernel != KR_EPANECHNIKOV && kernel != KR_TRIANGULAR) return KR_EKERNEL;
+    if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX) return KR_EARG;
     if (nshards < 1 || shard < 0 || shard >= nshards) return KR_EARG;
     if ((reinterpret_cast<uintptr_t>(d_workspace) & 255u) != 0) return KR_EARG;
     WsLayout L;
@@ -390,10 +471,13 @@ extern "C" int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n
     // Rows of this shard in sorted order.
     const int lo = (int)(((int64_t)shard * n) / nshards);
     const int hi = (int)(((int64_t)(shard + 1) * n) / nshards);
+    if (algo == KR_ALGO_AUTO) algo = auto_algo(n, hi - lo, m, kernel);
+    const bool prefix = algo == KR_ALGO_PREFIX;
     const int variant = sweep_variant(hi - lo);
     int G = sweep_G(hi - lo);
     if (variant == 1 && G > 4) G = 4;
-    const int ntiles = variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G);
+    const int ntiles = prefix ? (int)tiles_for(hi - lo, 1)
+                              : (variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G));
 
     int64_t launches = 0;
     prof_mark(0, st);
@@ -416,30 +500,64 @@ extern "C" int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n
         launches += 2 + cub_sort_launches(n);
     }
     prof_mark(1, st);
-    if (ntiles > 0) {
-        launches += 1;
+    if (prefix) {
         switch (kernel) {
-        case KR_UNIFORM:
-            launch_sweep<KR_UNIFORM>(G, xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, counter, st);
-            break;
-        case KR_EPANECHNIKOV:
-            launch_sweep<KR_EPANECHNIKOV>(G, xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, counter, st);
-            break;
-        default:
-            launch_sweep<KR_TRIANGULAR>(G, xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, counter, st);
-            break;
+        case KR_UNIFORM: launch_prefix_build<KR_UNIFORM>(xy, nn, L, ws, st); break;
+        case KR_EPANECHNIKOV: launch_prefix_build<KR_EPANECHNIKOV>(xy, nn, L, ws, st); break;
+        default: launch_prefix_build<KR_TRIANGULAR>(xy, nn, L, ws, st); break;
         }
+        launches += 3;
     }
     prof_mark(2, st);
+    if (ntiles > 0) {
+        launches += 1;
+        if (prefix) {
+            switch (kernel) {
+            case KR_UNIFORM:
+                launch_window<KR_UNIFORM>(xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
+                break;
+            case KR_EPANECHNIKOV:
+                launch_window<KR_EPANECHNIKOV>(xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
+                break;
+            default:
+                launch_window<KR_TRIANGULAR>(xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
+                break;
+            }
+        } else {
+            switch (kernel) {
+            case KR_UNIFORM:
+                launch_sweep<KR_UNIFORM>(G, xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, counter, st);
+                break;
+            case KR_EPANECHNIKOV:
+                launch_sweep<KR_EPANECHNIKOV>(G, xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, counter, st);
+                break;
+            default:
+                launch_sweep<KR_TRIANGULAR>(G, xy, nn, d_h, m, lo, hi, ntiles, tileS, tileN, counter, st);
+                break;
+            }
+        }
+    }
+    prof_mark(3, st);
     reduce_kernel<<<m < 148 * 8 ? m : 148 * 8, kReduceThreads, 0, st>>>(tileS, tileN, ntiles, m, status,
                                                                         d_partial);
     launches += 1;
-    prof_mark(3, st);
+    prof_mark(4, st);
     g_prof.recorded = g_prof.on;
     g_prof.launches = launches;
+    g_prof.algo = algo;
     e = cudaGetLastError();
     if (e != cudaSuccess) { set_cuda_error("kernel launch", (int)e); return KR_ECUDA; }
     return KR_OK;
+}
+
+extern "C" int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n,
+                                 const double *d_h, int32_t m, int32_t kernel,
+                                 int32_t shard, int32_t nshards,
+                                 double *d_partial, void *d_workspace, size_t workspace_bytes,
+                                 void *cuda_stream)
+{
+    return kr_cv_shard_algo_async(d_x, d_y, n, d_h, m, kernel, KR_ALGO_AUTO, shard, nshards, d_partial,
+                                  d_workspace, workspace_bytes, cuda_stream);
 }
 
 extern "C" int kr_finalize_async(const double *d_partial, int64_t n, int32_t m, double *d_cv,

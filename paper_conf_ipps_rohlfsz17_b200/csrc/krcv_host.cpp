@@ -133,10 +133,12 @@ static int validate_all(const double *x, const double *y, int64_t n, const doubl
     return KR_OK;
 }
 
-extern "C" int kr_cv_grid_ex(const double *x, const double *y, int64_t n, const double *h_grid, int32_t m,
-                             int32_t kernel, double *cv_out, int64_t *neff_out, int32_t *best_out)
+extern "C" int kr_cv_grid_algo(const double *x, const double *y, int64_t n, const double *h_grid, int32_t m,
+                               int32_t kernel, int32_t algo, double *cv_out, int64_t *neff_out,
+                               int32_t *best_out)
 {
     if (!cv_out || !best_out) return KR_EARG;
+    if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX) return KR_EARG;
     int st = validate_all(x, y, n, h_grid, m, kernel);
     if (st) return st;
     int dev = 0;
@@ -149,7 +151,8 @@ extern "C" int kr_cv_grid_ex(const double *x, const double *y, int64_t n, const 
     KR_CUDA_TRY(cudaMemcpyAsync(c->dx, x, sizeof(double) * n, cudaMemcpyHostToDevice, s));
     KR_CUDA_TRY(cudaMemcpyAsync(c->dy, y, sizeof(double) * n, cudaMemcpyHostToDevice, s));
     KR_CUDA_TRY(cudaMemcpyAsync(c->dh, h_grid, sizeof(double) * m, cudaMemcpyHostToDevice, s));
-    st = kr_cv_shard_async(c->dx, c->dy, n, c->dh, m, kernel, 0, 1, c->dpartial, c->ws, c->ws_bytes, s);
+    st = kr_cv_shard_algo_async(c->dx, c->dy, n, c->dh, m, kernel, algo, 0, 1, c->dpartial, c->ws, c->ws_bytes,
+                                s);
     if (st) return st;
     st = kr_finalize_async(c->dpartial, n, m, c->dcv, c->dneff, c->dbest, c->dbest + 1, s);
     if (st) return st;
@@ -166,6 +169,12 @@ extern "C" int kr_cv_grid_ex(const double *x, const double *y, int64_t n, const 
     if (neff_out) std::memcpy(neff_out, ne.data(), sizeof(int64_t) * m);
     *best_out = bs[0];
     return KR_OK;
+}
+
+extern "C" int kr_cv_grid_ex(const double *x, const double *y, int64_t n, const double *h_grid, int32_t m,
+                             int32_t kernel, double *cv_out, int64_t *neff_out, int32_t *best_out)
+{
+    return kr_cv_grid_algo(x, y, n, h_grid, m, kernel, KR_ALGO_AUTO, cv_out, neff_out, best_out);
 }
 
 extern "C" int kr_cv_grid(const double *x, const double *y, int64_t n, const double *h_grid, int32_t m,

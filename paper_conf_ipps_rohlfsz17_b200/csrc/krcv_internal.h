@@ -12,6 +12,9 @@ constexpr int64_t kGxgRows = 400000;
 int sweep_G(int64_t rows);
 int sweep_variant(int64_t rows);
 int64_t max_tiles(int64_t n);
+// Algorithm for a shard of `rows` rows of an n-point problem when the caller
+// asked for KR_ALGO_AUTO.
+int auto_algo(int64_t n, int64_t rows, int32_t m, int32_t kernel);
 
 // Byte layout of the device workspace (kr_workspace_bytes / kr_cv_shard_async).
 struct WsLayout {
@@ -22,6 +25,10 @@ struct WsLayout {
     size_t tileS;               // double  [m][ntiles]  per-tile sum of M e^2
     size_t tileN;               // uint8   [m][ntiles]  per-tile sum of M
     size_t status;              // uint32  [2]  n_bad_grid, n_nonfinite
+    size_t xs;                  // double  [n + 2 kPad] sorted x, +-inf sentinels (prefix path)
+    size_t pfx;                 // double2 [5][pstride] dd prefix moments P[k][0..n]
+    size_t ptot, poff;          // double2 [5][nch] chunk totals / exclusive offsets
+    int64_t pstride, nch;
     size_t cub;                 // radix-sort scratch
     size_t cub_bytes;
     size_t total;

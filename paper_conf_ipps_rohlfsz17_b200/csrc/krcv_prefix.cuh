@@ -1,0 +1,382 @@
+// krcv_prefix.cuh -- the window-prefix path ("a
+// sub-quadratic window-prefix variant").
+//
+// Same quantities as the per-pair sweep (krcv_sweep.cuh): for every sorted
+// row r and every bandwidth h_b of the ascending grid, the window
+// W_r(h_b) = { l != r : |x_l - x_r| < h_b } (<= for uniform; reading Q1),
+// the running sums c, sum y, sum d^2, sum y d^2 over it (reading Q3), the LOO
+// estimate Eq.(2), M (Q6) and the squared error of Eq.(1).
+//
+// What changes is how the running sums reach h_b.  The paper (§III
+// P@14010-14984, §IV.B P@21724-22104) carries them from h_{b-1} and adds the
+// additional neighbours one by one.  On the globally sorted array the window
+// of row r is the index range (L_r(b), R_r(b)) minus r itself, so:
+//   * the boundaries are found by a galloping search with the exact binary64
+//     membership predicate (monotone along the sorted array), starting from
+//     the previous bandwidth's boundaries -- window membership is identical to
+//     the sweep's and the oracle's, bit for bit;
+//   * the "additional values" of every bandwidth step are summed in O(1) as a
+//     difference of prefix sums P[R] - P[L+1] of the moments
+//     y, u, u^2, y u, y u^2 (u = x - o, o = the median x), kept in
+//     double-double so the difference and the shift to the row's own origin,
+//         sum (x_l - x_r)^2     = Suu  - delta (2 Su  - c' delta)
+//         sum y_l (x_l - x_r)^2 = Syuu - delta (2 Syu - delta Sy)
+//     (delta = x_r - o, c' = R - L - 1 including row r, whose own terms are
+//     0 in both), lose nothing to cancellation (krcv_dd.cuh);
+//   * sum y excludes row r by subtracting y_r (LOO, Eq.(2) l != i, Q8).
+// Per (row, bandwidth) the work is O(log growth) + O(1); nothing is O(n) per
+// row, so a grid search costs O(n m log) instead of O(n^2).
+//
+// Kernels:
+//   pfx_chunk_kernel   one thread per chunk of kPfxCh sorted records: moment
+//                      terms, chunk totals (dd), and the plain sorted-x array
+//                      xs[] (with -inf / +inf sentinels) used by the searches
+//   pfx_scan_kernel    one CTA: exclusive scan of the chunk totals
+//   pfx_write_kernel   one thread per chunk: prefix values P[k][0..n]
+//   window_kernel<K>   a warp owns 32 consecutive sorted rows (one per lane),
+//                      walks b = 0..m-1, emits (M e^2, M) per (tile, b) into
+//                      the same tile-partial layout the sweep uses (a5).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <climits>
+#include <cstdint>
+
+#include "krcv.h"
+#include "krcv_dd.cuh"
+#include "krcv_sweep.cuh"
+
+namespace krcv {
+
+constexpr int kPfxCh = 32;            // sorted records per thread in the prefix build
+constexpr int kPfxThreads = 128;
+constexpr int kPfxScanThreads = 1024;
+constexpr int kPfxMoments = 5;        // slots reserved in the workspace
+constexpr int kWinWarps = 4;
+constexpr int kWinThreads = kWinWarps * 32;
+constexpr int kWinTasksPerSM = 64;    // warp tasks per SM the b-split aims for
+constexpr int kWinMinBper = 8;        // >= this many bandwidths per task
+
+// Moments per kernel (slot order).  Epanechnikov: y, u, u^2, y u, y u^2.
+// Triangular: y, u, y u.  Uniform: y.
+template <int KERN>
+struct NMom {
+    static constexpr int v = KERN == KR_UNIFORM ? 1 : (KERN == KR_TRIANGULAR ? 3 : 5);
+};
+
+template <int KERN>
+__device__ __forceinline__ void moment_terms(double x, double y, double o, dd (&t)[kPfxMoments])
+{
+    t[0] = dd_make(y);
+    if (KERN != KR_UNIFORM) {
+        const dd u = two_sum(x, -o);  // exact: u.hi + u.lo == x - o
+        if (KERN == KR_EPANECHNIKOV) {
+            const dd uu = dd_mul(u, u);
+            t[1] = u;
+            t[2] = uu;
+            t[3] = dd_mul_d(u, y);
+            t[4] = dd_mul_d(uu, y);
+        } else {
+            t[1] = u;
+            t[2] = dd_mul_d(u, y);
+        }
+    }
+}
+
+__device__ __forceinline__ dd ld_dd(const double2 *p) { const double2 v = *p; return dd{v.x, v.y}; }
+__device__ __forceinline__ void st_dd(double2 *p, dd v) { *p = make_double2(v.hi, v.lo); }
+
+// origin o: the median record of the sorted array (keeps |u| small).
+__device__ __forceinline__ double pfx_origin(const double2 *xy, int n) { return xy[n >> 1].x; }
+
+// ---------------------------------------------------------------- build
+template <int KERN>
+__global__ void __launch_bounds__(kPfxThreads)
+pfx_chunk_kernel(const double2 *__restrict__ xy, int n, double *__restrict__ xs, double2 *__restrict__ tot,
+                 int nch)
+{
+    constexpr int K = NMom<KERN>::v;
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c == 0) {
+        for (int q = 1; q <= kPad; q++) {
+            xs[-q] = -INFINITY;
+            xs[n - 1 + q] = INFINITY;
+        }
+    }
+    if (c >= nch) return;
+    const double o = pfx_origin(xy, n);
+    dd acc[kPfxMoments];
+#pragma unroll
+    for (int k = 0; k < K; k++) acc[k] = dd{0.0, 0.0};
+    const int j0 = c * kPfxCh, j1 = min(n, j0 + kPfxCh);
+    for (int j = j0; j < j1; j++) {
+        const double2 v = xy[j];
+        xs[j] = v.x;
+        dd t[kPfxMoments];
+        moment_terms<KERN>(v.x, v.y, o, t);
+#pragma unroll
+        for (int k = 0; k < K; k++) acc[k] = dd_add(acc[k], t[k]);
+    }
+#pragma unroll
+    for (int k = 0; k < K; k++) st_dd(tot + (size_t)k * nch + c, acc[k]);
+}
+
+__device__ __forceinline__ dd shfl_up_dd(dd v, int d)
+{
+    return dd{__shfl_up_sync(0xffffffffu, v.hi, d), __shfl_up_sync(0xffffffffu, v.lo, d)};
+}
+
+// Exclusive scan of the chunk totals, one CTA, fixed order (deterministic).
+template <int KERN>
+__global__ void __launch_bounds__(kPfxScanThreads)
+pfx_scan_kernel(const double2 *__restrict__ tot, double2 *__restrict__ off, int nch)
+{
+    constexpr int K = NMom<KERN>::v;
+    __shared__ double2 wsum[K][kPfxScanThreads / 32];
+    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+    const int per = (nch + kPfxScanThreads - 1) / kPfxScanThreads;
+    const int c0 = min(nch, t * per), c1 = min(nch, c0 + per);
+    dd s[kPfxMoments];
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        s[k] = dd{0.0, 0.0};
+        for (int c = c0; c < c1; c++) s[k] = dd_add(s[k], ld_dd(tot + (size_t)k * nch + c));
+    }
+    // inclusive warp scan of the thread totals
+    dd inc[kPfxMoments];
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        inc[k] = s[k];
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const dd o = shfl_up_dd(inc[k], d);
+            if (lane >= d) inc[k] = dd_add(o, inc[k]);
+        }
+        if (lane == 31) st_dd(&wsum[k][w], inc[k]);
+    }
+    __syncthreads();
+    if (w == 0) {
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            dd v = ld_dd(&wsum[k][lane]);
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const dd o = shfl_up_dd(v, d);
+                if (lane >= d) v = dd_add(o, v);
+            }
+            st_dd(&wsum[k][lane], v);  // inclusive over warps
+        }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        dd run = dd_sub(inc[k], s[k]);  // exclusive within the warp
+        if (w > 0) run = dd_add(ld_dd(&wsum[k][w - 1]), run);
+        for (int c = c0; c < c1; c++) {
+            st_dd(off + (size_t)k * nch + c, run);
+            run = dd_add(run, ld_dd(tot + (size_t)k * nch + c));
+        }
+    }
+}
+
+template <int KERN>
+__global__ void __launch_bounds__(kPfxThreads)
+pfx_write_kernel(const double2 *__restrict__ xy, int n, const double2 *__restrict__ off, int nch,
+                 double2 *__restrict__ P, int pstride)
+{
+    constexpr int K = NMom<KERN>::v;
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= nch) return;
+    const double o = pfx_origin(xy, n);
+    dd acc[kPfxMoments];
+#pragma unroll
+    for (int k = 0; k < K; k++) acc[k] = ld_dd(off + (size_t)k * nch + c);
+    const int j0 = c * kPfxCh, j1 = min(n, j0 + kPfxCh);
+    for (int j = j0; j < j1; j++) {
+#pragma unroll
+        for (int k = 0; k < K; k++) st_dd(P + (size_t)k * pstride + j, acc[k]);
+        const double2 v = xy[j];
+        dd t[kPfxMoments];
+        moment_terms<KERN>(v.x, v.y, o, t);
+#pragma unroll
+        for (int k = 0; k < K; k++) acc[k] = dd_add(acc[k], t[k]);
+    }
+    if (j1 == n) {
+#pragma unroll
+        for (int k = 0; k < K; k++) st_dd(P + (size_t)k * pstride + n, acc[k]);
+    }
+}
+
+// ---------------------------------------------------------------- windows
+// New boundaries for bandwidth h from the previous ones.  Right: every j in
+// (r, R) is inside, returns the first j >= R outside.  Left: every j in
+// (L, r) is inside, returns the last j <= L outside.  Gallop (first step 1,
+// then the previous growth, then doubling) and bisect; both sides
+// interleaved for memory-level parallelism.  xs carries +-inf sentinels, so
+// xs[n] and xs[-1] are outside every window.
+template <int KERN>
+__device__ __forceinline__ void window_bounds(const double *__restrict__ xs, int n, double xr, double h, int &R,
+                                              int &L, int &gR, int &gL)
+{
+    int rlo = R - 1, rhi = 0, rstep = 1;  // rlo: inside (or r)
+    int llo = L + 1, lhi = 0, lstep = 1;  // llo: inside (or r)
+    bool rg = true, lg = true, rfirst = true, lfirst = true;
+    while (rg || lg) {
+        if (rg) {
+            const int p = min(rlo + rstep, n);
+            if (inside<KERN>(xs[p] - xr, h)) {
+                rlo = p;
+                rstep = rfirst ? gR : 2 * rstep;
+                rfirst = false;
+            } else {
+                rhi = p;
+                rg = false;
+            }
+        }
+        if (lg) {
+            const int p = max(llo - lstep, -1);
+            if (inside<KERN>(xr - xs[p], h)) {
+                llo = p;
+                lstep = lfirst ? gL : 2 * lstep;
+                lfirst = false;
+            } else {
+                lhi = p;
+                lg = false;
+            }
+        }
+    }
+    while (rhi - rlo > 1 || llo - lhi > 1) {
+        if (rhi - rlo > 1) {
+            const int p = (rlo + rhi) >> 1;
+            if (inside<KERN>(xs[p] - xr, h)) rlo = p; else rhi = p;
+        }
+        if (llo - lhi > 1) {
+            const int p = (llo + lhi) >> 1;
+            if (inside<KERN>(xr - xs[p], h)) llo = p; else lhi = p;
+        }
+    }
+    gR = max(1, rhi - R);
+    gL = max(1, L - lhi);
+    R = rhi;
+    L = lhi;
+}
+
+// Window sums of moment k over sorted indices [a, b): P[b] - P[a].
+__device__ __forceinline__ dd wsum(const double2 *__restrict__ P, int pstride, int k, int a, int b)
+{
+    return dd_sub(ld_dd(P + (size_t)k * pstride + b), ld_dd(P + (size_t)k * pstride + a));
+}
+
+template <int KERN>
+__global__ void __launch_bounds__(kWinThreads)
+window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double2 *__restrict__ P,
+              int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
+              int nbc, double *__restrict__ tileS, uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
+{
+    const int lane = threadIdx.x & 31;
+    const double o = pfx_origin(xy, n);
+    const int bper = (m + nbc - 1) / nbc;
+    for (;;) {
+        // task = (tile of 32 rows, chunk of bandwidths): the bandwidth loop is
+        // split so that small shards still fill the GPU; a chunk starts its
+        // searches cold (from the row itself), later steps from the previous h.
+        int task = 0;
+        if (lane == 0) task = atomicAdd(tile_counter, 1);
+        task = __shfl_sync(0xffffffffu, task, 0);
+        if (task >= ntiles * nbc) return;  // warp-uniform
+        const int tile = task / nbc;
+        const int b0 = (task - tile * nbc) * bper, b1 = min(m, b0 + bper);
+
+        const int i = row_lo + tile * 32 + lane;
+        const bool valid = i < row_hi;
+        const int r = valid ? i : row_hi - 1;  // clamped rows do identical work, discarded
+        const double2 vr = xy[r];
+        const double xr = vr.x, yr = vr.y;
+        const dd del = two_sum(xr, -o);  // exact x_r - o
+        int R = r + 1, L = r - 1, gR = 1, gL = 1;
+        // triangular splits the window at r: per-row constants P[r], P[r+1]
+        dd Pr[3], Pr1[3];
+        if (KERN == KR_TRIANGULAR) {
+#pragma unroll
+            for (int k = 0; k < 3; k++) {
+                Pr[k] = ld_dd(P + (size_t)k * pstride + r);
+                Pr1[k] = ld_dd(P + (size_t)k * pstride + r + 1);
+            }
+        }
+
+        for (int b = b0; b < b1; b++) {
+            const double h = __ldg(hg + b);
+            window_bounds<KERN>(xs, n, xr, h, R, L, gR, gL);
+            const int cR = R - r - 1, cL = r - L - 1;
+            const int c = cR + cL;
+            const bool M = valid && c > 0;  // reading Q6
+            double e2 = 0.0;
+            if (M) {
+                double g;
+                if (KERN == KR_UNIFORM) {
+                    const dd Sy = wsum(P, pstride, 0, L + 1, R);
+                    g = dd_to_d(dd_add_d(Sy, -yr)) / (double)c;
+                } else {
+                    double sy, s1, sy1;
+                    if (KERN == KR_EPANECHNIKOV) {
+                        const dd Sy = wsum(P, pstride, 0, L + 1, R);
+                        const dd Su = wsum(P, pstride, 1, L + 1, R);
+                        const dd Suu = wsum(P, pstride, 2, L + 1, R);
+                        const dd Syu = wsum(P, pstride, 3, L + 1, R);
+                        const dd Syuu = wsum(P, pstride, 4, L + 1, R);
+                        const dd t1 = dd_sub(dd_twice(Su), dd_mul_d(del, (double)(c + 1)));
+                        s1 = dd_to_d(dd_sub(Suu, dd_mul(del, t1)));
+                        const dd t2 = dd_sub(dd_twice(Syu), dd_mul(del, Sy));
+                        sy1 = dd_to_d(dd_sub(Syuu, dd_mul(del, t2)));
+                        sy = dd_to_d(dd_add_d(Sy, -yr));
+                    } else {  // triangular: right (r, R) and left (L, r) separately
+                        const double2 *P0 = P, *P1 = P + pstride, *P2 = P + 2 * (size_t)pstride;
+                        const dd SyR = dd_sub(ld_dd(P0 + R), Pr1[0]);
+                        const dd SuR = dd_sub(ld_dd(P1 + R), Pr1[1]);
+                        const dd SyuR = dd_sub(ld_dd(P2 + R), Pr1[2]);
+                        const dd SyL = dd_sub(Pr[0], ld_dd(P0 + L + 1));
+                        const dd SuL = dd_sub(Pr[1], ld_dd(P1 + L + 1));
+                        const dd SyuL = dd_sub(Pr[2], ld_dd(P2 + L + 1));
+                        // sum d  = (SuR - cR delta) + (cL delta - SuL)
+                        const dd dR = dd_sub(SuR, dd_mul_d(del, (double)cR));
+                        const dd dL = dd_sub(dd_mul_d(del, (double)cL), SuL);
+                        s1 = dd_to_d(dd_add(dR, dL));
+                        // sum y d = (SyuR - delta SyR) + (delta SyL - SyuL)
+                        const dd yR = dd_sub(SyuR, dd_mul(del, SyR));
+                        const dd yL = dd_sub(dd_mul(del, SyL), SyuL);
+                        sy1 = dd_to_d(dd_add(yR, yL));
+                        sy = dd_to_d(dd_add(SyR, SyL));
+                    }
+                    // Eq.(2)-(3) with 0.75 and 1/h^2 cancelled (reading Q5)
+                    const double hk = (KERN == KR_EPANECHNIKOV) ? h * h : h;
+                    double num = fma(hk, sy, -sy1);
+                    double den = fma(hk, (double)c, -s1);
+                    if (!(den >= 0x1p-20 * hk * (double)c)) {  // reading Q14
+                        num = 0.0;
+                        den = 0.0;
+                        for (int q = L + 1; q < R; q++) {
+                            if (q == r) continue;
+                            const double2 v = xy[q];
+                            const double d = fabs(v.x - xr);
+                            const double w = (KERN == KR_EPANECHNIKOV) ? (h - d) * (h + d) : (h - d);
+                            num = fma(v.y, w, num);
+                            den += w;
+                        }
+                    }
+                    g = num / den;
+                }
+                const double e = yr - g;
+                e2 = e * e;
+            }
+            e2 = warp_sum(e2);
+            const unsigned ball = __ballot_sync(0xffffffffu, M);
+            if (lane == 0) {
+                tileS[(size_t)b * ntiles + tile] = e2;
+                tileN[(size_t)b * ntiles + tile] = (uint8_t)__popc(ball);
+            }
+        }
+    }
+}
+
+}  // namespace krcv

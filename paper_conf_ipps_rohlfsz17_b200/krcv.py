@@ -25,15 +25,18 @@ LIB_PATH = os.path.join(_HERE, "libkrcv.so")
 UNIFORM, EPANECHNIKOV, TRIANGULAR = 0, 1, 2
 KERNELS = {"uniform": UNIFORM, "epanechnikov": EPANECHNIKOV, "triangular": TRIANGULAR}
 
+ALGO_AUTO, ALGO_SWEEP, ALGO_PREFIX = 0, 1, 2
+ALGOS = {"auto": ALGO_AUTO, "sweep": ALGO_SWEEP, "prefix": ALGO_PREFIX}
+
 KR_OK, KR_EARG, KR_EKERNEL, KR_EGRID, KR_ENONFINITE, KR_EDEGENERATE, KR_ENOMEM, KR_ECUDA = range(8)
 KR_MAX_M = 65536
 
 # Every symbol include/krcv.h declares (checked by tests/test_abi.py).
 EXPORTS = (
-    "kr_cv_grid", "kr_cv_grid_ex", "kr_validate_grid", "kr_workspace_bytes",
-    "kr_cv_shard_async", "kr_finalize", "kr_finalize_async", "kr_default_grid",
+    "kr_cv_grid", "kr_cv_grid_ex", "kr_cv_grid_algo", "kr_validate_grid", "kr_workspace_bytes",
+    "kr_cv_shard_async", "kr_cv_shard_algo_async", "kr_finalize", "kr_finalize_async", "kr_default_grid",
     "kr_strerror", "kr_last_cuda_error", "kr_version",
-    "kr_profile_enable", "kr_profile_read", "kr_launch_count",
+    "kr_profile_enable", "kr_profile_read", "kr_launch_count", "kr_last_algo",
 )
 
 
@@ -65,14 +68,17 @@ def _lib() -> ctypes.CDLL:
     P, i64, i32, sz = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_size_t
     lib.kr_cv_grid.argtypes = [P, P, i64, P, i32, i32, P, P]
     lib.kr_cv_grid_ex.argtypes = [P, P, i64, P, i32, i32, P, P, P]
+    lib.kr_cv_grid_algo.argtypes = [P, P, i64, P, i32, i32, i32, P, P, P]
     lib.kr_validate_grid.argtypes = [P, i32]
     lib.kr_workspace_bytes.argtypes = [i64, i32]
     lib.kr_workspace_bytes.restype = sz
     lib.kr_cv_shard_async.argtypes = [P, P, i64, P, i32, i32, i32, i32, P, P, sz, P]
+    lib.kr_cv_shard_algo_async.argtypes = [P, P, i64, P, i32, i32, i32, i32, i32, P, P, sz, P]
     lib.kr_finalize.argtypes = [P, i64, i32, P, P, P]
     lib.kr_finalize_async.argtypes = [P, i64, i32, P, P, P, P, P]
     lib.kr_default_grid.argtypes = [P, i64, i32, P]
-    for f in ("kr_cv_grid", "kr_cv_grid_ex", "kr_validate_grid", "kr_cv_shard_async",
+    for f in ("kr_cv_grid", "kr_cv_grid_ex", "kr_cv_grid_algo", "kr_validate_grid", "kr_cv_shard_async",
+              "kr_cv_shard_algo_async",
               "kr_finalize", "kr_finalize_async", "kr_default_grid"):
         getattr(lib, f).restype = ctypes.c_int
     lib.kr_strerror.argtypes = [ctypes.c_int]
@@ -84,6 +90,7 @@ def _lib() -> ctypes.CDLL:
     lib.kr_profile_read.argtypes = [P]
     lib.kr_profile_read.restype = ctypes.c_int
     lib.kr_launch_count.restype = ctypes.c_int64
+    lib.kr_last_algo.restype = ctypes.c_int32
     _LIB = lib
     return lib
 
@@ -92,6 +99,12 @@ def _kernel_id(kernel) -> int:
     if isinstance(kernel, str):
         return KERNELS[kernel.lower()]
     return int(kernel)
+
+
+def _algo_id(algo) -> int:
+    if isinstance(algo, str):
+        return ALGOS[algo.lower()]
+    return int(algo)
 
 
 def _host(a) -> np.ndarray:
@@ -104,15 +117,23 @@ def _check(st: int, where: str) -> None:
 
 
 # ------------------------------------------------------------------ host API
-def kr_cv_grid(x, y, h, kernel="epanechnikov", with_neff: bool = False):
+def kr_cv_grid(x, y, h, kernel="epanechnikov", with_neff: bool = False, algo="auto"):
     """Whole grid search on the current CUDA device from host arrays.
-    Returns (cv[m], best) or (cv, neff, best)."""
+    Returns (cv[m], best) or (cv, neff, best).  ``algo`` = "auto" | "sweep" |
+    "prefix" (KR_ALGO_*); "auto" calls kr_cv_grid / kr_cv_grid_ex themselves."""
     x, y, h = _host(x), _host(y), _host(h)
     if x.shape != y.shape or x.ndim != 1:
         raise ValueError("x and y must be 1-D arrays of equal length")
     n, m = x.shape[0], h.shape[0]
     cv = np.empty(m, np.float64)
     best = ctypes.c_int32(-1)
+    a = _algo_id(algo)
+    if a != ALGO_AUTO:
+        neff = np.empty(m, np.int64)
+        st = _lib().kr_cv_grid_algo(x.ctypes.data, y.ctypes.data, n, h.ctypes.data, m, _kernel_id(kernel), a,
+                                    cv.ctypes.data, neff.ctypes.data, ctypes.byref(best))
+        _check(st, "kr_cv_grid_algo")
+        return (cv, neff, int(best.value)) if with_neff else (cv, int(best.value))
     if with_neff:
         neff = np.empty(m, np.int64)
         st = _lib().kr_cv_grid_ex(x.ctypes.data, y.ctypes.data, n, h.ctypes.data, m, _kernel_id(kernel),
@@ -169,9 +190,11 @@ def kr_workspace_bytes(n: int, m: int) -> int:
 
 
 # ---------------------------------------------------------------- device API
-def kr_cv_shard_async(d_x, d_y, d_h, kernel, shard: int, nshards: int, d_partial, d_ws, stream=None) -> None:
+def kr_cv_shard_async(d_x, d_y, d_h, kernel, shard: int, nshards: int, d_partial, d_ws, stream=None,
+                      algo="auto") -> None:
     """Enqueue the sharded device pipeline.  All tensor arguments are CUDA
-    torch tensors (float64 for x, y, h, partial; uint8 for the workspace)."""
+    torch tensors (float64 for x, y, h, partial; uint8 for the workspace).
+    ``algo`` "auto" calls kr_cv_shard_async, otherwise kr_cv_shard_algo_async."""
     import torch
 
     n, m = d_x.numel(), d_h.numel()
@@ -181,10 +204,17 @@ def kr_cv_shard_async(d_x, d_y, d_h, kernel, shard: int, nshards: int, d_partial
     if d_partial.numel() != partial_len(m):
         raise ValueError("partial must have 2m+2 elements")
     s = torch.cuda.current_stream(d_x.device) if stream is None else stream
-    st = _lib().kr_cv_shard_async(d_x.data_ptr(), d_y.data_ptr(), n, d_h.data_ptr(), m, _kernel_id(kernel),
-                                  int(shard), int(nshards), d_partial.data_ptr(), d_ws.data_ptr(),
-                                  d_ws.numel() * d_ws.element_size(), ctypes.c_void_p(s.cuda_stream))
-    _check(st, "kr_cv_shard_async")
+    a = _algo_id(algo)
+    if a == ALGO_AUTO:
+        st = _lib().kr_cv_shard_async(d_x.data_ptr(), d_y.data_ptr(), n, d_h.data_ptr(), m, _kernel_id(kernel),
+                                      int(shard), int(nshards), d_partial.data_ptr(), d_ws.data_ptr(),
+                                      d_ws.numel() * d_ws.element_size(), ctypes.c_void_p(s.cuda_stream))
+        _check(st, "kr_cv_shard_async")
+        return
+    st = _lib().kr_cv_shard_algo_async(d_x.data_ptr(), d_y.data_ptr(), n, d_h.data_ptr(), m, _kernel_id(kernel),
+                                       a, int(shard), int(nshards), d_partial.data_ptr(), d_ws.data_ptr(),
+                                       d_ws.numel() * d_ws.element_size(), ctypes.c_void_p(s.cuda_stream))
+    _check(st, "kr_cv_shard_algo_async")
 
 
 def kr_finalize_async(d_partial, n: int, m: int, d_cv, d_neff, d_best_status, stream=None) -> None:
@@ -205,10 +235,15 @@ def kr_profile_enable(on: bool) -> None:
 
 
 def kr_profile_read():
-    """(sort_ms, sweep_ms, reduce_ms) of the last kr_cv_shard_async on this thread."""
-    ms = np.zeros(3, np.float32)
+    """(sort_ms, prefix_build_ms, sweep_ms, reduce_ms) of the last
+    kr_cv_shard_async on this thread."""
+    ms = np.zeros(4, np.float32)
     _check(_lib().kr_profile_read(ms.ctypes.data), "kr_profile_read")
-    return float(ms[0]), float(ms[1]), float(ms[2])
+    return tuple(float(v) for v in ms)
+
+
+def kr_last_algo() -> int:
+    return int(_lib().kr_last_algo())
 
 
 def kr_launch_count() -> int:

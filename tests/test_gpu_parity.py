@@ -27,10 +27,19 @@ pytestmark = pytest.mark.gpu
 U, E, T = 0, 1, 2
 TOL = 1e-6
 TIGHT = 1e-10
+ALGO = {"a": "auto"}
+
+
+@pytest.fixture(params=["sweep", "prefix"], autouse=True)
+def algo(request):
+    """Every parity test runs on both algorithms (KR_ALGO_SWEEP, KR_ALGO_PREFIX)."""
+    ALGO["a"] = request.param
+    yield request.param
+    ALGO["a"] = "auto"
 
 
 def _gpu(x, y, h, k):
-    cv, neff, best = krcv.kr_cv_grid(x, y, h, k, with_neff=True)
+    cv, neff, best = krcv.kr_cv_grid(x, y, h, k, with_neff=True, algo=ALGO["a"])
     return cv, neff, best
 
 
@@ -146,7 +155,7 @@ def _device_partial(x, y, h, k, shard, nshards):
     d_h = torch.as_tensor(h, device="cuda")
     part = torch.empty(krcv.partial_len(h.shape[0]), dtype=torch.float64, device="cuda")
     ws = krcv.aligned(krcv.workspace(x.shape[0], h.shape[0], "cuda"))
-    krcv.kr_cv_shard_async(d_x, d_y, d_h, k, shard, nshards, part, ws)
+    krcv.kr_cv_shard_async(d_x, d_y, d_h, k, shard, nshards, part, ws, algo=ALGO["a"])
     torch.cuda.synchronize()
     return part.cpu().numpy()
 
@@ -178,6 +187,17 @@ def test_shard_emulation_sums_to_unsharded(P):
     assert cv_rel_err(cv, ref.cv) <= TIGHT and best_ok(best, ref.cv)
 
 
+def test_algorithms_agree():
+    """Sweep and window-prefix give the same curve to ~1e-13 and identical
+    n_eff (window membership is decided by the same binary64 predicate)."""
+    for cfg, n in (("C2", 20000), ("C5", 20000), ("C1", 1000)):
+        x, y, h, k = workloads.make(cfg, seed=4, n=n)
+        a = krcv.kr_cv_grid(x, y, h, k, with_neff=True, algo="sweep")
+        b = krcv.kr_cv_grid(x, y, h, k, with_neff=True, algo="prefix")
+        assert cv_rel_err(b[0], a[0]) <= 1e-12
+        assert np.array_equal(a[1], b[1]) and best_ok(b[2], a[0])
+
+
 def test_determinism_bitwise():
     """T8: repeated runs are bit-identical (static row->warp map, fixed-order reductions)."""
     x, y, h, k = workloads.make("C2", seed=2, n=6000)
@@ -203,7 +223,7 @@ def test_device_status_nonfinite_and_bad_grid():
         krcv.kr_finalize(part, x.shape[0], h.shape[0])
     assert e.value.status == krcv.KR_EGRID
     # device finalize reports the same status
-    plan = GridSearch(x.shape[0], h, k)
+    plan = GridSearch(x.shape[0], h, k, algo=ALGO["a"])
     xd = torch.as_tensor(x, device="cuda")
     yd = torch.as_tensor(y, device="cuda")
     xd[10] = float("inf")
@@ -216,7 +236,7 @@ def test_device_status_nonfinite_and_bad_grid():
 def test_device_api_matches_host_api():
     import torch
     x, y, h, k = workloads.make("C5", seed=0, n=20000)
-    plan = GridSearch(x.shape[0], h, k)
+    plan = GridSearch(x.shape[0], h, k, algo=ALGO["a"])
     plan.run(torch.as_tensor(x, device="cuda"), torch.as_tensor(y, device="cuda"))
     r = plan.result()
     cv, neff, best = _gpu(x, y, h, k)
