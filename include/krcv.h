@@ -156,6 +156,25 @@ int kr_cv_shard_algo_async(const double *d_x, const double *d_y, int64_t n,
                            void *cuda_stream);
 
 /*
+ * kr_cv_grid_async -- the whole single-GPU grid search on caller-owned device
+ * memory, enqueued on `cuda_stream` without synchronising (capturable):
+ * kr_cv_shard_algo_async(shard 0 of 1) with the finalize fused into the
+ * reduction's last CTA (one launch fewer than shard + kr_finalize_async).
+ *   d_x, d_y, d_h, n, m, kernel, algo, d_workspace, workspace_bytes: as
+ *                  kr_cv_shard_algo_async (the partial vector lives in the
+ *                  workspace)
+ *   d_cv           [m] fp64 DEVICE: CV(h_b) per Eq.(1)
+ *   d_neff         [m] int64 DEVICE, nullable: rows with M_i = 1 per bandwidth
+ *   d_best_status  [2] int32 DEVICE: { best index (Q11), KR_OK | KR_EGRID |
+ *                  KR_ENONFINITE } -- read it after the stream work completes
+ * Host-checked errors (returned): KR_EARG, KR_EKERNEL, KR_ECUDA.
+ */
+int kr_cv_grid_async(const double *d_x, const double *d_y, int64_t n,
+                     const double *d_h, int32_t m, int32_t kernel, int32_t algo,
+                     double *d_cv, int64_t *d_neff, int32_t *d_best_status,
+                     void *d_workspace, size_t workspace_bytes, void *cuda_stream);
+
+/*
  * kr_finalize -- host finalize of a partial vector already summed over all
  * shards: cv_out[b] = S[b]/n, neff_out[b] = neff[b] (nullable), best_out per
  * Q11.  Returns KR_EGRID / KR_ENONFINITE if the status slots are non-zero.

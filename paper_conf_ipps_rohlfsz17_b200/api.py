@@ -97,10 +97,13 @@ class GridSearch:
     def run(self, d_x, d_y) -> None:
         if d_x.numel() != self.n or d_y.numel() != self.n:
             raise ValueError("x, y must have n elements")
+        if self.world == 1:  # whole search in one enqueue, finalize fused into the reduction
+            krcv.kr_cv_grid_async(d_x, d_y, self.d_h, self.kernel, self.cv, self.neff, self.best_status, self.ws,
+                                  algo=self.algo)
+            return
         krcv.kr_cv_shard_async(d_x, d_y, self.d_h, self.kernel, self.rank, self.world, self.partial, self.ws,
                                algo=self.algo)
-        if self.world > 1:
-            allreduce_partial(self.partial, self.group)
+        allreduce_partial(self.partial, self.group)
         krcv.kr_finalize_async(self.partial, self.n, self.m, self.cv, self.neff, self.best_status)
 
     def result(self) -> CVResult:

@@ -84,6 +84,30 @@ __device__ __forceinline__ dd dd_mul(dd a, dd b)
     return quick_two_sum(p.hi, p.lo);
 }
 
+// a * b and a * (double) b without the final renormalisation: |lo| stays
+// O(eps |hi|), which every consumer below (dd_add / dd_sub_to_d) accepts.
+__device__ __forceinline__ dd dd_mul_raw(dd a, dd b)
+{
+    dd p = two_prod(a.hi, b.hi);
+    p.lo = __fma_rn(a.hi, b.lo, __fma_rn(a.lo, b.hi, p.lo));
+    return p;
+}
+
+__device__ __forceinline__ dd dd_mul_d_raw(dd a, double b)
+{
+    dd p = two_prod(a.hi, b);
+    p.lo = __fma_rn(a.lo, b, p.lo);
+    return p;
+}
+
+// a - b rounded to the nearest double (within 1 ulp): the last step of a
+// dd computation whose result is consumed in double.
+__device__ __forceinline__ double dd_sub_to_d(dd a, dd b)
+{
+    const dd s = two_sum(a.hi, -b.hi);
+    return __dadd_rn(s.hi, __dadd_rn(s.lo, __dsub_rn(a.lo, b.lo)));
+}
+
 // 2^k scaling is exact.
 __device__ __forceinline__ dd dd_twice(dd a) { return dd{__dmul_rn(2.0, a.hi), __dmul_rn(2.0, a.lo)}; }
 

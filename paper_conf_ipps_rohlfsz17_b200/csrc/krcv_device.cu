@@ -78,17 +78,87 @@ __global__ void gather_kernel(const double *__restrict__ x, const double *__rest
 // a3 + a4: the sweep -- see krcv_sweep.cuh
 // ---------------------------------------------------------------------------
 // ---------------------------------------------------------------------------
+// finalize: CV = S/n, arg-min (Q11), status.  One CTA of THREADS threads;
+// the paper's min-reduction kernel (P@24653).  Reads the partial vector with
+// ld.global.cg (it may have been written by other CTAs of the same launch).
+// ---------------------------------------------------------------------------
+template <int THREADS>
+__device__ __forceinline__ void finalize_body(const double *partial, long long n, int m, double *__restrict__ cv,
+                                              long long *__restrict__ neff, int *__restrict__ best,
+                                              int *__restrict__ status, double *sv, int *si)
+{
+    double bv = 0.0;
+    int bi = -1;
+    for (int b = threadIdx.x; b < m; b += THREADS) {
+        const double v = __ldcg(partial + b) / (double)n;
+        cv[b] = v;
+        if (neff) neff[b] = (long long)__ldcg(partial + m + b);
+        if (!isnan(v) && (bi < 0 || v < bv)) {  // strided order: b ascending per thread
+            bv = v;
+            bi = b;
+        }
+    }
+    sv[threadIdx.x] = bv;
+    si[threadIdx.x] = bi;
+    __syncthreads();
+    for (int s = THREADS / 2; s > 0; s >>= 1) {
+        if (threadIdx.x < s) {
+            const double ov = sv[threadIdx.x + s];
+            const int oi = si[threadIdx.x + s];
+            const int mi = si[threadIdx.x];
+            const double mv = sv[threadIdx.x];
+            if (oi >= 0 && (mi < 0 || ov < mv || (ov == mv && oi < mi))) {
+                sv[threadIdx.x] = ov;
+                si[threadIdx.x] = oi;
+            }
+        }
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) {
+        *best = si[0] < 0 ? 0 : si[0];
+        int st = KR_OK;
+        if (__ldcg(partial + 2 * m) != 0.0) st = KR_EGRID;
+        else if (__ldcg(partial + 2 * m + 1) != 0.0) st = KR_ENONFINITE;
+        *status = st;
+    }
+}
+
+constexpr int kFinThreads = 1024;
+
+__global__ void __launch_bounds__(kFinThreads)
+finalize_kernel(const double *__restrict__ partial, long long n, int m, double *__restrict__ cv,
+                long long *__restrict__ neff, int *__restrict__ best, int *__restrict__ status)
+{
+    __shared__ double sv[kFinThreads];
+    __shared__ int si[kFinThreads];
+    finalize_body<kFinThreads>(partial, n, m, cv, neff, best, status, sv, si);
+}
+
+// ---------------------------------------------------------------------------
 // a5: fixed-order column reduction of the tile partials (the paper's
 // "summation reduction ... performed k times", P@23970, as one launch).
+// With fin != nullptr (single-GPU whole search, kr_cv_grid_async) the last
+// CTA to finish also runs the finalize (threadfence + completion counter),
+// saving a launch; the counter is reset for the next call.
 // ---------------------------------------------------------------------------
 constexpr int kReduceThreads = 256;
 
+struct FinOut {
+    long long n;
+    double *cv;
+    long long *neff;
+    int *best, *status;
+    unsigned *done;
+};
+
 __global__ void __launch_bounds__(kReduceThreads)
 reduce_kernel(const double *__restrict__ tileS, const uint8_t *__restrict__ tileN, int ntiles, int m,
-              const unsigned *__restrict__ status, double *__restrict__ partial)
+              const unsigned *__restrict__ status, double *__restrict__ partial, FinOut fin)
 {
     __shared__ double sS[kReduceThreads];
     __shared__ long long sN[kReduceThreads];
+    __shared__ int sI[kReduceThreads];
+    __shared__ bool last;
     for (int b = blockIdx.x; b < m; b += gridDim.x) {
         double a = 0.0;
         long long cnt = 0;
@@ -118,53 +188,15 @@ reduce_kernel(const double *__restrict__ tileS, const uint8_t *__restrict__ tile
         partial[2 * m] = (double)status[0];
         partial[2 * m + 1] = (double)status[1];
     }
-}
-
-// ---------------------------------------------------------------------------
-// finalize on the device: CV = S/n, arg-min (Q11), status.  One CTA.
-// ---------------------------------------------------------------------------
-constexpr int kFinThreads = 1024;
-
-__global__ void __launch_bounds__(kFinThreads)
-finalize_kernel(const double *__restrict__ partial, long long n, int m, double *__restrict__ cv,
-                long long *__restrict__ neff, int *__restrict__ best, int *__restrict__ status)
-{
-    __shared__ double sv[kFinThreads];
-    __shared__ int si[kFinThreads];
-    double bv = 0.0;
-    int bi = -1;
-    for (int b = threadIdx.x; b < m; b += kFinThreads) {
-        double v = partial[b] / (double)n;
-        cv[b] = v;
-        if (neff) neff[b] = (long long)partial[m + b];
-        if (!isnan(v) && (bi < 0 || v < bv)) {  // strided order: b ascending per thread
-            bv = v;
-            bi = b;
-        }
-    }
-    sv[threadIdx.x] = bv;
-    si[threadIdx.x] = bi;
+    if (fin.cv == nullptr) return;
+    __threadfence();
     __syncthreads();
-    for (int s = kFinThreads / 2; s > 0; s >>= 1) {
-        if (threadIdx.x < s) {
-            double ov = sv[threadIdx.x + s];
-            int oi = si[threadIdx.x + s];
-            int mi = si[threadIdx.x];
-            double mv = sv[threadIdx.x];
-            if (oi >= 0 && (mi < 0 || ov < mv || (ov == mv && oi < mi))) {
-                sv[threadIdx.x] = ov;
-                si[threadIdx.x] = oi;
-            }
-        }
-        __syncthreads();
-    }
-    if (threadIdx.x == 0) {
-        *best = si[0] < 0 ? 0 : si[0];
-        int st = KR_OK;
-        if (partial[2 * m] != 0.0) st = KR_EGRID;
-        else if (partial[2 * m + 1] != 0.0) st = KR_ENONFINITE;
-        *status = st;
-    }
+    if (threadIdx.x == 0) last = atomicAdd(fin.done, 1u) == gridDim.x - 1;
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    finalize_body<kReduceThreads>(partial, fin.n, m, fin.cv, fin.neff, fin.best, fin.status, sS, sI);
+    if (threadIdx.x == 0) *fin.done = 0u;
 }
 
 // ---------------------------------------------------------------------------
@@ -198,14 +230,15 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     L->tileS = off;    off = align256(off + sizeof(double) * (size_t)ntiles * (size_t)m);
     L->tileN = off;    off = align256(off + sizeof(uint8_t) * (size_t)ntiles * (size_t)m);
     // window-prefix path (krcv_prefix.cuh)
-    const size_t nch = (size_t)((n + kPfxCh - 1) / kPfxCh);
+    const size_t nch = (size_t)((n + kPfxTile) / kPfxTile);  // tiles covering P[0..n]
     L->pstride = (int64_t)(((size_t)n + 1 + 15) & ~size_t(15));
     L->nch = (int64_t)nch;
     L->xs = off;       off = align256(off + sizeof(double) * ((size_t)n + 2 * kPad));
     L->pfx = off;      off = align256(off + sizeof(double2) * kPfxMoments * (size_t)L->pstride);
     L->ptot = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
     L->poff = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
-    L->status = off;   off = align256(off + 2 * sizeof(unsigned));
+    L->status = off;   off = align256(off + 4 * sizeof(unsigned));  // bad grid, non-finite, done, pad
+    L->partial = off;  off = align256(off + sizeof(double) * (size_t)KR_PARTIAL_LEN(m));
     L->cub = off;      off = align256(off + cub_bytes);
     L->cub_bytes = cub_bytes;
     L->total = off;
@@ -359,11 +392,10 @@ static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, cha
     double2 *P = reinterpret_cast<double2 *>(ws + L.pfx);
     double2 *tot = reinterpret_cast<double2 *>(ws + L.ptot);
     double2 *off = reinterpret_cast<double2 *>(ws + L.poff);
-    const int nch = (int)L.nch;
-    const int blocks = (nch + kPfxThreads - 1) / kPfxThreads;
-    pfx_chunk_kernel<KERN><<<blocks, kPfxThreads, 0, st>>>(xy, n, xs, tot, nch);
-    pfx_scan_kernel<KERN><<<1, kPfxScanThreads, 0, st>>>(tot, off, nch);
-    pfx_write_kernel<KERN><<<blocks, kPfxThreads, 0, st>>>(xy, n, off, nch, P, (int)L.pstride);
+    const int ntiles = (int)L.nch;
+    pfx_tile_reduce_kernel<KERN><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles);
+    pfx_scan_kernel<KERN><<<1, kPfxScanThreads, 0, st>>>(tot, off, ntiles);
+    pfx_tile_scan_kernel<KERN><<<ntiles, kPfxThreads, 0, st>>>(xy, n, off, ntiles, P, (int)L.pstride, xs);
 }
 
 template <int KERN>
@@ -439,13 +471,13 @@ extern "C" size_t kr_workspace_bytes(int64_t n, int32_t m)
     return L.total;
 }
 
-extern "C" int kr_cv_shard_algo_async(const double *d_x, const double *d_y, int64_t n,
-                                      const double *d_h, int32_t m, int32_t kernel, int32_t algo,
-                                      int32_t shard, int32_t nshards,
-                                      double *d_partial, void *d_workspace, size_t workspace_bytes,
-                                      void *cuda_stream)
+// The whole device pipeline of one shard: a1 .. a5, and with fin.cv set the
+// fused finalize (single-GPU whole search).
+static int enqueue(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m, int32_t kernel,
+                   int32_t algo, int32_t shard, int32_t nshards, double *d_partial, FinOut fin,
+                   void *d_workspace, size_t workspace_bytes, void *cuda_stream)
 {
-    if (!d_x || !d_y || !d_h || !d_partial || !d_workspace) return KR_EARG;
+    if (!d_x || !d_y || !d_h || !d_workspace) return KR_EARG;
     if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return KR_EARG;
     if (kernel != KR_UNIFORM && kernel != KR_EPANECHNIKOV && kernel != KR_TRIANGULAR) return KR_EKERNEL;
     if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX) return KR_EARG;
@@ -466,6 +498,8 @@ extern "C" int kr_cv_shard_algo_async(const double *d_x, const double *d_y, int6
     double *tileS = reinterpret_cast<double *>(ws + L.tileS);
     uint8_t *tileN = reinterpret_cast<uint8_t *>(ws + L.tileN);
     unsigned *status = reinterpret_cast<unsigned *>(ws + L.status);
+    if (!d_partial) d_partial = reinterpret_cast<double *>(ws + L.partial);
+    fin.done = status + 2;
     const int nn = (int)n;
 
     // Rows of this shard in sorted order.
@@ -481,14 +515,20 @@ extern "C" int kr_cv_shard_algo_async(const double *d_x, const double *d_y, int6
 
     int64_t launches = 0;
     prof_mark(0, st);
-    cudaError_t e = cudaMemsetAsync(status, 0, 2 * sizeof(unsigned), st);
+    cudaError_t e = cudaMemsetAsync(status, 0, 3 * sizeof(unsigned), st);
     if (e != cudaSuccess) { set_cuda_error("cudaMemsetAsync(status)", (int)e); return KR_ECUDA; }
     if (n <= kRankSortMaxN && !getenv_flag("KRCV_CUB_SORT")) {
-        // a1 + a2 fused: chunk bitonic sort + rank-by-search scatter (krcv_sort.cuh)
+        // a1 + a2: chunk merge sort, rank by counting across chunk pairs, scatter (krcv_sort.cuh)
         const int nchunks = (int)((n + kChunk - 1) / kChunk);
-        chunk_sort_kernel<<<nchunks, kChunkThreads, 0, st>>>(d_x, d_y, nn, d_h, m, keys_in, vals_in, status);
-        rank_scatter_kernel<<<(nchunks * kChunk + 255) / 256, 256, 0, st>>>(keys_in, vals_in, nn, nchunks, d_x,
-                                                                          d_y, xy, counter);
+        uint32_t *khi = reinterpret_cast<uint32_t *>(keys_out);          // keys_out is free on this path
+        int *rank = reinterpret_cast<int *>(vals_out);                    // so is vals_out
+        chunk_sort_kernel<<<nchunks, kChunkThreads, 0, st>>>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank,
+                                                            status);
+        if (nchunks > 1)
+            rank_count_kernel<<<dim3(nchunks, nchunks), kChunkThreads, 0, st>>>(keys_in, khi, vals_in, rank);
+        const int npad = nchunks * kChunk;
+        rank_scatter_kernel<<<(npad + 255) / 256, 256, 0, st>>>(vals_in, rank, nn, npad, d_x, d_y, xy, counter);
+        launches += nchunks > 1 ? 1 : 0;
         launches += 2;
     } else {
         pack_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, nn, d_h, m, keys_in, vals_in, status);
@@ -539,7 +579,7 @@ extern "C" int kr_cv_shard_algo_async(const double *d_x, const double *d_y, int6
     }
     prof_mark(3, st);
     reduce_kernel<<<m < 148 * 8 ? m : 148 * 8, kReduceThreads, 0, st>>>(tileS, tileN, ntiles, m, status,
-                                                                        d_partial);
+                                                                        d_partial, fin);
     launches += 1;
     prof_mark(4, st);
     g_prof.recorded = g_prof.on;
@@ -548,6 +588,34 @@ extern "C" int kr_cv_shard_algo_async(const double *d_x, const double *d_y, int6
     e = cudaGetLastError();
     if (e != cudaSuccess) { set_cuda_error("kernel launch", (int)e); return KR_ECUDA; }
     return KR_OK;
+}
+
+extern "C" int kr_cv_shard_algo_async(const double *d_x, const double *d_y, int64_t n,
+                                      const double *d_h, int32_t m, int32_t kernel, int32_t algo,
+                                      int32_t shard, int32_t nshards,
+                                      double *d_partial, void *d_workspace, size_t workspace_bytes,
+                                      void *cuda_stream)
+{
+    if (!d_partial) return KR_EARG;
+    FinOut fin{};
+    return enqueue(d_x, d_y, n, d_h, m, kernel, algo, shard, nshards, d_partial, fin, d_workspace,
+                   workspace_bytes, cuda_stream);
+}
+
+extern "C" int kr_cv_grid_async(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m,
+                                int32_t kernel, int32_t algo, double *d_cv, int64_t *d_neff,
+                                int32_t *d_best_status, void *d_workspace, size_t workspace_bytes,
+                                void *cuda_stream)
+{
+    if (!d_cv || !d_best_status) return KR_EARG;
+    FinOut fin{};
+    fin.n = (long long)n;
+    fin.cv = d_cv;
+    fin.neff = reinterpret_cast<long long *>(d_neff);
+    fin.best = d_best_status;
+    fin.status = d_best_status + 1;
+    return enqueue(d_x, d_y, n, d_h, m, kernel, algo, 0, 1, nullptr, fin, d_workspace, workspace_bytes,
+                   cuda_stream);
 }
 
 extern "C" int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n,

@@ -151,10 +151,8 @@ extern "C" int kr_cv_grid_algo(const double *x, const double *y, int64_t n, cons
     KR_CUDA_TRY(cudaMemcpyAsync(c->dx, x, sizeof(double) * n, cudaMemcpyHostToDevice, s));
     KR_CUDA_TRY(cudaMemcpyAsync(c->dy, y, sizeof(double) * n, cudaMemcpyHostToDevice, s));
     KR_CUDA_TRY(cudaMemcpyAsync(c->dh, h_grid, sizeof(double) * m, cudaMemcpyHostToDevice, s));
-    st = kr_cv_shard_algo_async(c->dx, c->dy, n, c->dh, m, kernel, algo, 0, 1, c->dpartial, c->ws, c->ws_bytes,
-                                s);
-    if (st) return st;
-    st = kr_finalize_async(c->dpartial, n, m, c->dcv, c->dneff, c->dbest, c->dbest + 1, s);
+    st = kr_cv_grid_async(c->dx, c->dy, n, c->dh, m, kernel, algo, c->dcv, c->dneff, c->dbest, c->ws, c->ws_bytes,
+                          s);
     if (st) return st;
     std::vector<double> cv(m);
     std::vector<int64_t> ne(neff_out ? m : 0);

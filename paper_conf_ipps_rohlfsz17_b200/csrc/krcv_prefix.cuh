@@ -28,11 +28,12 @@
 // row, so a grid search costs O(n m log) instead of O(n^2).
 //
 // Kernels:
-//   pfx_chunk_kernel   one thread per chunk of kPfxCh sorted records: moment
-//                      terms, chunk totals (dd), and the plain sorted-x array
-//                      xs[] (with -inf / +inf sentinels) used by the searches
-//   pfx_scan_kernel    one CTA: exclusive scan of the chunk totals
-//   pfx_write_kernel   one thread per chunk: prefix values P[k][0..n]
+//   pfx_tile_reduce_kernel  per tile of kPfxTile sorted records: moment terms
+//                           and their dd totals
+//   pfx_scan_kernel         one CTA: exclusive scan of the tile totals
+//   pfx_tile_scan_kernel    per tile: prefix values P[k][0..n] and the plain
+//                           sorted-x array xs[] (+-inf sentinels) the
+//                           searches read
 //   window_kernel<K>   a warp owns 32 consecutive sorted rows (one per lane),
 //                      walks b = 0..m-1, emits (M e^2, M) per (tile, b) into
 //                      the same tile-partial layout the sweep uses (a5).
@@ -49,8 +50,7 @@
 
 namespace krcv {
 
-constexpr int kPfxCh = 32;            // sorted records per thread in the prefix build
-constexpr int kPfxThreads = 128;
+constexpr int kPfxThreads = 256;      // prefix build CTA
 constexpr int kPfxScanThreads = 1024;
 constexpr int kPfxMoments = 5;        // slots reserved in the workspace
 constexpr int kWinWarps = 4;
@@ -91,43 +91,60 @@ __device__ __forceinline__ void st_dd(double2 *p, dd v) { *p = make_double2(v.hi
 __device__ __forceinline__ double pfx_origin(const double2 *xy, int n) { return xy[n >> 1].x; }
 
 // ---------------------------------------------------------------- build
-template <int KERN>
-__global__ void __launch_bounds__(kPfxThreads)
-pfx_chunk_kernel(const double2 *__restrict__ xy, int n, double *__restrict__ xs, double2 *__restrict__ tot,
-                 int nch)
-{
-    constexpr int K = NMom<KERN>::v;
-    const int c = blockIdx.x * blockDim.x + threadIdx.x;
-    if (c == 0) {
-        for (int q = 1; q <= kPad; q++) {
-            xs[-q] = -INFINITY;
-            xs[n - 1 + q] = INFINITY;
-        }
-    }
-    if (c >= nch) return;
-    const double o = pfx_origin(xy, n);
-    dd acc[kPfxMoments];
-#pragma unroll
-    for (int k = 0; k < K; k++) acc[k] = dd{0.0, 0.0};
-    const int j0 = c * kPfxCh, j1 = min(n, j0 + kPfxCh);
-    for (int j = j0; j < j1; j++) {
-        const double2 v = xy[j];
-        xs[j] = v.x;
-        dd t[kPfxMoments];
-        moment_terms<KERN>(v.x, v.y, o, t);
-#pragma unroll
-        for (int k = 0; k < K; k++) acc[k] = dd_add(acc[k], t[k]);
-    }
-#pragma unroll
-    for (int k = 0; k < K; k++) st_dd(tot + (size_t)k * nch + c, acc[k]);
-}
+// Three-phase fixed-order scan (bit-reproducible; a decoupled look-back
+// would make the dd rounding depend on timing).  A tile is kPfxTile sorted
+// records; thread t of its CTA owns records 4t .. 4t+3 of the tile.
+constexpr int kPfxItems = 4;
+constexpr int kPfxTile = kPfxThreads * kPfxItems;
 
 __device__ __forceinline__ dd shfl_up_dd(dd v, int d)
 {
     return dd{__shfl_up_sync(0xffffffffu, v.hi, d), __shfl_up_sync(0xffffffffu, v.lo, d)};
 }
 
-// Exclusive scan of the chunk totals, one CTA, fixed order (deterministic).
+__device__ __forceinline__ dd shfl_xor_dd(dd v, int d)
+{
+    return dd{__shfl_xor_sync(0xffffffffu, v.hi, d), __shfl_xor_sync(0xffffffffu, v.lo, d)};
+}
+
+// Phase 1: per-tile totals of the moment terms -> tot[k][tile].
+template <int KERN>
+__global__ void __launch_bounds__(kPfxThreads)
+pfx_tile_reduce_kernel(const double2 *__restrict__ xy, int n, double2 *__restrict__ tot, int ntiles)
+{
+    constexpr int K = NMom<KERN>::v;
+    __shared__ double2 wsum[K][kPfxThreads / 32];
+    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+    const int j0 = blockIdx.x * kPfxTile + t * kPfxItems;
+    const double o = pfx_origin(xy, n);
+    dd acc[kPfxMoments];
+#pragma unroll
+    for (int k = 0; k < K; k++) acc[k] = dd{0.0, 0.0};
+#pragma unroll
+    for (int q = 0; q < kPfxItems; q++) {
+        if (j0 + q < n) {
+            const double2 v = xy[j0 + q];
+            dd tm[kPfxMoments];
+            moment_terms<KERN>(v.x, v.y, o, tm);
+#pragma unroll
+            for (int k = 0; k < K; k++) acc[k] = dd_add(acc[k], tm[k]);
+        }
+    }
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+#pragma unroll
+        for (int d = 16; d > 0; d >>= 1) acc[k] = dd_add(acc[k], shfl_xor_dd(acc[k], d));
+        if (lane == 0) st_dd(&wsum[k][w], acc[k]);
+    }
+    __syncthreads();
+    if (t < K) {
+        dd a = dd{0.0, 0.0};
+        for (int q = 0; q < kPfxThreads / 32; q++) a = dd_add(a, ld_dd(&wsum[t][q]));
+        st_dd(tot + (size_t)t * ntiles + blockIdx.x, a);
+    }
+}
+
+// Phase 2: exclusive scan of the tile totals, one CTA, fixed order.
 template <int KERN>
 __global__ void __launch_bounds__(kPfxScanThreads)
 pfx_scan_kernel(const double2 *__restrict__ tot, double2 *__restrict__ off, int nch)
@@ -143,15 +160,14 @@ pfx_scan_kernel(const double2 *__restrict__ tot, double2 *__restrict__ off, int 
         s[k] = dd{0.0, 0.0};
         for (int c = c0; c < c1; c++) s[k] = dd_add(s[k], ld_dd(tot + (size_t)k * nch + c));
     }
-    // inclusive warp scan of the thread totals
     dd inc[kPfxMoments];
 #pragma unroll
     for (int k = 0; k < K; k++) {
         inc[k] = s[k];
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
-            const dd o = shfl_up_dd(inc[k], d);
-            if (lane >= d) inc[k] = dd_add(o, inc[k]);
+            const dd u = shfl_up_dd(inc[k], d);
+            if (lane >= d) inc[k] = dd_add(u, inc[k]);
         }
         if (lane == 31) st_dd(&wsum[k][w], inc[k]);
     }
@@ -162,8 +178,8 @@ pfx_scan_kernel(const double2 *__restrict__ tot, double2 *__restrict__ off, int 
             dd v = ld_dd(&wsum[k][lane]);
 #pragma unroll
             for (int d = 1; d < 32; d <<= 1) {
-                const dd o = shfl_up_dd(v, d);
-                if (lane >= d) v = dd_add(o, v);
+                const dd u = shfl_up_dd(v, d);
+                if (lane >= d) v = dd_add(u, v);
             }
             st_dd(&wsum[k][lane], v);  // inclusive over warps
         }
@@ -180,86 +196,124 @@ pfx_scan_kernel(const double2 *__restrict__ tot, double2 *__restrict__ off, int 
     }
 }
 
+// Phase 3: in-tile exclusive scan + tile offset -> P[k][j] = sum_{l<j} t_k(l)
+// for j in the tile (and P[k][n] by the last tile), plus the plain sorted-x
+// array xs (with -inf / +inf sentinels) used by the window searches.
 template <int KERN>
 __global__ void __launch_bounds__(kPfxThreads)
-pfx_write_kernel(const double2 *__restrict__ xy, int n, const double2 *__restrict__ off, int nch,
-                 double2 *__restrict__ P, int pstride)
+pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__restrict__ off, int ntiles,
+                     double2 *__restrict__ P, int pstride, double *__restrict__ xs)
 {
     constexpr int K = NMom<KERN>::v;
-    const int c = blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= nch) return;
+    __shared__ double2 wsum[K][kPfxThreads / 32];
+    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+    const int j0 = blockIdx.x * kPfxTile + t * kPfxItems;
+    if (blockIdx.x == 0 && t < kPad) {
+        xs[-1 - t] = -INFINITY;
+        xs[n + t] = INFINITY;
+    }
     const double o = pfx_origin(xy, n);
+    dd tm[kPfxItems][kPfxMoments];
     dd acc[kPfxMoments];
 #pragma unroll
-    for (int k = 0; k < K; k++) acc[k] = ld_dd(off + (size_t)k * nch + c);
-    const int j0 = c * kPfxCh, j1 = min(n, j0 + kPfxCh);
-    for (int j = j0; j < j1; j++) {
+    for (int k = 0; k < K; k++) acc[k] = dd{0.0, 0.0};
 #pragma unroll
-        for (int k = 0; k < K; k++) st_dd(P + (size_t)k * pstride + j, acc[k]);
-        const double2 v = xy[j];
-        dd t[kPfxMoments];
-        moment_terms<KERN>(v.x, v.y, o, t);
+    for (int q = 0; q < kPfxItems; q++) {
+        if (j0 + q < n) {
+            const double2 v = xy[j0 + q];
+            xs[j0 + q] = v.x;
+            moment_terms<KERN>(v.x, v.y, o, tm[q]);
+        } else {
 #pragma unroll
-        for (int k = 0; k < K; k++) acc[k] = dd_add(acc[k], t[k]);
+            for (int k = 0; k < K; k++) tm[q][k] = dd{0.0, 0.0};
+        }
+#pragma unroll
+        for (int k = 0; k < K; k++) acc[k] = dd_add(acc[k], tm[q][k]);
     }
-    if (j1 == n) {
+    // exclusive scan of the thread totals across the CTA
+    dd ex[kPfxMoments];
 #pragma unroll
-        for (int k = 0; k < K; k++) st_dd(P + (size_t)k * pstride + n, acc[k]);
+    for (int k = 0; k < K; k++) {
+        dd inc = acc[k];
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const dd u = shfl_up_dd(inc, d);
+            if (lane >= d) inc = dd_add(u, inc);
+        }
+        if (lane == 31) st_dd(&wsum[k][w], inc);
+        const dd u = shfl_up_dd(inc, 1);
+        ex[k] = lane == 0 ? dd{0.0, 0.0} : u;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        dd base = ld_dd(off + (size_t)k * ntiles + blockIdx.x);
+        for (int q = 0; q < w; q++) base = dd_add(base, ld_dd(&wsum[k][q]));
+        dd run = dd_add(base, ex[k]);
+#pragma unroll
+        for (int q = 0; q < kPfxItems; q++) {
+            if (j0 + q <= n) st_dd(P + (size_t)k * pstride + j0 + q, run);
+            run = dd_add(run, tm[q][k]);
+        }
     }
 }
 
 // ---------------------------------------------------------------- windows
-// New boundaries for bandwidth h from the previous ones.  Right: every j in
-// (r, R) is inside, returns the first j >= R outside.  Left: every j in
-// (L, r) is inside, returns the last j <= L outside.  Gallop (first step 1,
-// then the previous growth, then doubling) and bisect; both sides
-// interleaved for memory-level parallelism.  xs carries +-inf sentinels, so
-// xs[n] and xs[-1] are outside every window.
+// New boundaries for bandwidth h from the previous ones, in offsets from the
+// row: the right side probes xs[r + k], the left side xs[r - k]; "inside" is
+// the exact binary64 predicate of reading Q1 and is monotone in k.  On entry
+// every offset in (0, kR) / (0, kL) is inside (the previous windows); on exit
+// kR / kL are the first offsets outside.  xs carries +-inf sentinels, so
+// offset n - r (right) and r + 1 (left) are outside every window.
+// Gallop (first step 1, then the previous growth gR / gL, then doubling) and
+// bisect; both sides advance in the same loop iteration (memory-level
+// parallelism).  (A predicted-bracket variant issued more instructions than
+// it saved probes: profiles/r01f_*.)
 template <int KERN>
-__device__ __forceinline__ void window_bounds(const double *__restrict__ xs, int n, double xr, double h, int &R,
-                                              int &L, int &gR, int &gL)
+__device__ __forceinline__ void window_bounds(const double *__restrict__ xs, int n, int r, double xr, double h,
+                                              int &kR, int &kL, int gR, int gL)
 {
-    int rlo = R - 1, rhi = 0, rstep = 1;  // rlo: inside (or r)
-    int llo = L + 1, lhi = 0, lstep = 1;  // llo: inside (or r)
+    const double *__restrict__ xsr = xs + r;
+    int rlo = kR - 1, rhi = 0, rstep = 1;  // rlo: inside (or the row itself)
+    int llo = kL - 1, lhi = 0, lstep = 1;
+    const int kRmax = n - r, kLmax = r + 1;
     bool rg = true, lg = true, rfirst = true, lfirst = true;
     while (rg || lg) {
         if (rg) {
-            const int p = min(rlo + rstep, n);
-            if (inside<KERN>(xs[p] - xr, h)) {
-                rlo = p;
+            const int k = min(rlo + rstep, kRmax);
+            if (inside<KERN>(xsr[k] - xr, h)) {
+                rlo = k;
                 rstep = rfirst ? gR : 2 * rstep;
                 rfirst = false;
             } else {
-                rhi = p;
+                rhi = k;
                 rg = false;
             }
         }
         if (lg) {
-            const int p = max(llo - lstep, -1);
-            if (inside<KERN>(xr - xs[p], h)) {
-                llo = p;
+            const int k = min(llo + lstep, kLmax);
+            if (inside<KERN>(xr - xsr[-k], h)) {
+                llo = k;
                 lstep = lfirst ? gL : 2 * lstep;
                 lfirst = false;
             } else {
-                lhi = p;
+                lhi = k;
                 lg = false;
             }
         }
     }
-    while (rhi - rlo > 1 || llo - lhi > 1) {
+    while (rhi - rlo > 1 || lhi - llo > 1) {
         if (rhi - rlo > 1) {
-            const int p = (rlo + rhi) >> 1;
-            if (inside<KERN>(xs[p] - xr, h)) rlo = p; else rhi = p;
+            const int k = (rlo + rhi) >> 1;
+            if (inside<KERN>(xsr[k] - xr, h)) rlo = k; else rhi = k;
         }
-        if (llo - lhi > 1) {
-            const int p = (llo + lhi) >> 1;
-            if (inside<KERN>(xr - xs[p], h)) llo = p; else lhi = p;
+        if (lhi - llo > 1) {
+            const int k = (llo + lhi) >> 1;
+            if (inside<KERN>(xr - xsr[-k], h)) llo = k; else lhi = k;
         }
     }
-    gR = max(1, rhi - R);
-    gL = max(1, L - lhi);
-    R = rhi;
-    L = lhi;
+    kR = rhi;
+    kL = lhi;
 }
 
 // Window sums of moment k over sorted indices [a, b): P[b] - P[a].
@@ -294,7 +348,8 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
         const double2 vr = xy[r];
         const double xr = vr.x, yr = vr.y;
         const dd del = two_sum(xr, -o);  // exact x_r - o
-        int R = r + 1, L = r - 1, gR = 1, gL = 1;
+        int kR = 1, kL = 1;  // first offsets not yet known inside
+        int gR = 1, gL = 1;  // previous growth of each side (first gallop step)
         // triangular splits the window at r: per-row constants P[r], P[r+1]
         dd Pr[3], Pr1[3];
         if (KERN == KR_TRIANGULAR) {
@@ -307,7 +362,11 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
 
         for (int b = b0; b < b1; b++) {
             const double h = __ldg(hg + b);
-            window_bounds<KERN>(xs, n, xr, h, R, L, gR, gL);
+            const int kR0 = kR, kL0 = kL;
+            window_bounds<KERN>(xs, n, r, xr, h, kR, kL, gR, gL);
+            gR = max(1, kR - kR0);
+            gL = max(1, kL - kL0);
+            const int R = r + kR, L = r - kL;
             const int cR = R - r - 1, cL = r - L - 1;
             const int c = cR + cL;
             const bool M = valid && c > 0;  // reading Q6
@@ -316,7 +375,7 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
                 double g;
                 if (KERN == KR_UNIFORM) {
                     const dd Sy = wsum(P, pstride, 0, L + 1, R);
-                    g = dd_to_d(dd_add_d(Sy, -yr)) / (double)c;
+                    g = dd_sub_to_d(Sy, dd_make(yr)) / (double)c;
                 } else {
                     double sy, s1, sy1;
                     if (KERN == KR_EPANECHNIKOV) {
@@ -325,11 +384,11 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
                         const dd Suu = wsum(P, pstride, 2, L + 1, R);
                         const dd Syu = wsum(P, pstride, 3, L + 1, R);
                         const dd Syuu = wsum(P, pstride, 4, L + 1, R);
-                        const dd t1 = dd_sub(dd_twice(Su), dd_mul_d(del, (double)(c + 1)));
-                        s1 = dd_to_d(dd_sub(Suu, dd_mul(del, t1)));
-                        const dd t2 = dd_sub(dd_twice(Syu), dd_mul(del, Sy));
-                        sy1 = dd_to_d(dd_sub(Syuu, dd_mul(del, t2)));
-                        sy = dd_to_d(dd_add_d(Sy, -yr));
+                        const dd t1 = dd_sub(dd_twice(Su), dd_mul_d_raw(del, (double)(c + 1)));
+                        s1 = dd_sub_to_d(Suu, dd_mul_raw(del, t1));
+                        const dd t2 = dd_sub(dd_twice(Syu), dd_mul_raw(del, Sy));
+                        sy1 = dd_sub_to_d(Syuu, dd_mul_raw(del, t2));
+                        sy = dd_sub_to_d(Sy, dd_make(yr));
                     } else {  // triangular: right (r, R) and left (L, r) separately
                         const double2 *P0 = P, *P1 = P + pstride, *P2 = P + 2 * (size_t)pstride;
                         const dd SyR = dd_sub(ld_dd(P0 + R), Pr1[0]);
@@ -339,12 +398,12 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
                         const dd SuL = dd_sub(Pr[1], ld_dd(P1 + L + 1));
                         const dd SyuL = dd_sub(Pr[2], ld_dd(P2 + L + 1));
                         // sum d  = (SuR - cR delta) + (cL delta - SuL)
-                        const dd dR = dd_sub(SuR, dd_mul_d(del, (double)cR));
-                        const dd dL = dd_sub(dd_mul_d(del, (double)cL), SuL);
+                        const dd dR = dd_sub(SuR, dd_mul_d_raw(del, (double)cR));
+                        const dd dL = dd_sub(dd_mul_d_raw(del, (double)cL), SuL);
                         s1 = dd_to_d(dd_add(dR, dL));
                         // sum y d = (SyuR - delta SyR) + (delta SyL - SyuL)
-                        const dd yR = dd_sub(SyuR, dd_mul(del, SyR));
-                        const dd yL = dd_sub(dd_mul(del, SyL), SyuL);
+                        const dd yR = dd_sub(SyuR, dd_mul_raw(del, SyR));
+                        const dd yL = dd_sub(dd_mul_raw(del, SyL), SyuL);
                         sy1 = dd_to_d(dd_add(yR, yL));
                         sy = dd_to_d(dd_add(SyR, SyL));
                     }

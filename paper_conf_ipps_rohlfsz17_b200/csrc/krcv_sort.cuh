@@ -8,21 +8,23 @@
 //
 //   K1 chunk_sort_kernel:  each CTA packs kChunk records (order-preserving
 //      u64 key of x, u32 index), counts non-finite inputs and bad grid
-//      entries, and radix-sorts the chunk in registers/shared memory
-//      (cub::BlockRadixSort, stable, so ties stay in index order);
-//   K2 rank_scatter_kernel: every record's final position is its position in
-//      its chunk plus, for every other chunk, the number of records that
-//      compare less (branchless binary search); it writes (x, y) straight to
-//      that position of the sorted array -- no merge passes, no separate
-//      gather.  (key, index) pairs are unique, so the order is total and
-//      identical to a stable sort by x.
+//      entries, and sorts the chunk in registers/shared memory
+//      (cub::BlockMergeSort::StableSort, so ties stay in index order);
+//   K2 rank_count_kernel: one CTA per ordered chunk pair (c, cc): the count
+//      of chunk cc's records that compare less than each record of chunk c
+//      (fixed-depth binary searches), added to the record's rank;
+//   K3 rank_scatter_kernel: writes (x, y) straight to that rank in the
+//      sorted array -- no merge passes, no separate gather.  (key, index)
+//      pairs are unique, so the order is total and identical to a stable
+//      sort by x.
 #pragma once
 
 #include <cuda_runtime.h>
 
 #include <cstdint>
 
-#include <cub/block/block_radix_sort.cuh>
+#include <cub/block/block_merge_sort.cuh>
+
 
 #include "krcv_sweep.cuh"
 
@@ -45,13 +47,18 @@ __device__ __forceinline__ bool kv_less(uint64_t ka, uint32_t ia, uint64_t kb, u
     return ka < kb || (ka == kb && ia < ib);
 }
 
+struct KeyLess {
+    __device__ __forceinline__ bool operator()(const uint64_t &a, const uint64_t &b) const { return a < b; }
+};
+
 __global__ void __launch_bounds__(kChunkThreads)
 chunk_sort_kernel(const double *__restrict__ x, const double *__restrict__ y, int n,
                   const double *__restrict__ h, int m, uint64_t *__restrict__ keys,
-                  uint32_t *__restrict__ idx, unsigned *__restrict__ status)
+                  uint32_t *__restrict__ khi, uint32_t *__restrict__ idx, int *__restrict__ rank,
+                  unsigned *__restrict__ status)
 {
-    using BRS = cub::BlockRadixSort<uint64_t, kChunkThreads, kChunkItems, uint32_t, 6>;
-    __shared__ typename BRS::TempStorage ts;
+    using BMS = cub::BlockMergeSort<uint64_t, kChunkThreads, kChunkItems, uint32_t>;
+    __shared__ typename BMS::TempStorage ts;
     const int base = blockIdx.x * kChunk;
     uint64_t k[kChunkItems];
     uint32_t v[kChunkItems];
@@ -77,98 +84,88 @@ chunk_sort_kernel(const double *__restrict__ x, const double *__restrict__ y, in
         }
     if (bad) atomicAdd(&status[1], bad);
     if (gbad) atomicAdd(&status[0], gbad);
-    BRS(ts).Sort(k, v);  // stable LSD radix: equal keys keep index order
+    BMS(ts).StableSort(k, v, KeyLess());  // stable: equal keys keep index order
 #pragma unroll
     for (int q = 0; q < kChunkItems; q++) {
         keys[base + threadIdx.x * kChunkItems + q] = k[q];
+        khi[base + threadIdx.x * kChunkItems + q] = (uint32_t)(k[q] >> 32);
+        rank[base + threadIdx.x * kChunkItems + q] = threadIdx.x * kChunkItems + q;  // + counts (K2)
         idx[base + threadIdx.x * kChunkItems + q] = v[q];
     }
 }
 
-constexpr int kSearchBatch = 8;      // binary searches advanced in lock-step (ILP)
-constexpr int kRankThreads = 256;    // a CTA ranks 256 consecutive records of one chunk
-constexpr int kMaxChunks = (int)(kRankSortMaxN / kChunk);
-
-// Branchless count of records < (k, i) in the sorted range [lo, lo + len) of
-// the chunked arrays, for kSearchBatch chunks at once.
-__device__ __forceinline__ bool rec_less(const uint64_t *__restrict__ keys, const uint32_t *__restrict__ idx,
-                                         int p, uint64_t k, uint32_t i)
+// K2: counts of chunk c's records in chunk cc, one CTA per ordered pair
+// (c, cc != c) so the whole GPU shares the O(n * nchunks * log kChunk)
+// searches.  Thread t owns records t, t + 256, ... of chunk c (striped: the
+// lanes of a warp search nearby words of the other chunk's high key words,
+// which stay L1-resident); kChunkItems fixed-depth branchless binary searches
+// run in lock-step (ILP) on the high 32 key bits and fall back to the full
+// (key, index) order only when high words tie.  The counts are added to the
+// record's rank with integer atomics (exact, so the result is deterministic).
+__global__ void __launch_bounds__(kChunkThreads)
+rank_count_kernel(const uint64_t *__restrict__ keys, const uint32_t *__restrict__ khi,
+                  const uint32_t *__restrict__ idx, int *__restrict__ rank)
 {
-    const uint64_t kp = keys[p];
-    return kp < k || (kp == k && idx[p] < i);  // idx only read on key ties
+    const int c = blockIdx.x, cc = blockIdx.y;
+    if (c == cc) return;
+    const int t = threadIdx.x;
+    const uint32_t *ch = khi + (size_t)cc * kChunk;
+    const uint64_t *ck = keys + (size_t)cc * kChunk;
+    const uint32_t *ci = idx + (size_t)cc * kChunk;
+    uint64_t k[kChunkItems];
+    uint32_t v[kChunkItems], kh[kChunkItems];
+    int pos[kChunkItems];
+#pragma unroll
+    for (int q = 0; q < kChunkItems; q++) {
+        const int g = c * kChunk + t + q * kChunkThreads;
+        k[q] = keys[g];
+        v[q] = idx[g];
+        kh[q] = (uint32_t)(k[q] >> 32);
+        pos[q] = 0;
+    }
+    // pos = #{records of cc that are (key, idx)-less}; invariant: [0, pos) less
+#pragma unroll
+    for (int half = kChunk / 2; half > 0; half >>= 1) {
+#pragma unroll
+        for (int q = 0; q < kChunkItems; q++) {
+            const int p = pos[q] + half - 1;
+            const uint32_t hp = __ldg(ch + p);
+            bool less = hp < kh[q];
+            if (hp == kh[q]) {  // rare: compare the full order
+                const uint64_t kp = __ldg(ck + p);
+                less = kp < k[q] || (kp == k[q] && __ldg(ci + p) < v[q]);
+            }
+            pos[q] += less ? half : 0;
+        }
+    }
+#pragma unroll
+    for (int q = 0; q < kChunkItems; q++) {
+        const int p = pos[q];  // <= kChunk - 1
+        const uint32_t hp = __ldg(ch + p);
+        bool less = hp < kh[q];
+        if (hp == kh[q]) {
+            const uint64_t kp = __ldg(ck + p);
+            less = kp < k[q] || (kp == k[q] && __ldg(ci + p) < v[q]);
+        }
+        if (v[q] != 0xffffffffu) atomicAdd(rank + c * kChunk + t + q * kChunkThreads, p + (less ? 1 : 0));
+    }
 }
 
-__global__ void __launch_bounds__(kRankThreads)
-rank_scatter_kernel(const uint64_t *__restrict__ keys, const uint32_t *__restrict__ idx, int n, int nchunks,
+// K3: scatter (x, y) to the sorted positions; sentinels; sweep counter reset.
+__global__ void __launch_bounds__(256)
+rank_scatter_kernel(const uint32_t *__restrict__ idx, const int *__restrict__ rank, int n, int npad,
                     const double *__restrict__ x, const double *__restrict__ y, double2 *__restrict__ xy,
                     int *__restrict__ tile_counter)
 {
-    __shared__ int s_lo[kMaxChunks], s_len[kMaxChunks];
-    const int g0 = blockIdx.x * kRankThreads;  // first record of this CTA (sorted within chunk c)
-    const int g = g0 + threadIdx.x;
-    const int c = g0 / kChunk;
-    if (g < kPad && blockIdx.x == 0) {
+    const int g = blockIdx.x * blockDim.x + threadIdx.x;
+    if (g < kPad) {
         xy[-1 - g] = make_double2(-INFINITY, 0.0);
         xy[n + g] = make_double2(INFINITY, 0.0);
     }
     if (g == 0) *tile_counter = 0;
-    // 1) For every other chunk, bracket where this CTA's records fall: the
-    //    counts of its first and last record (2 full searches per chunk, one
-    //    thread each).  Every record's count then lies in that bracket, which
-    //    the whole CTA searches next -- a small, L1-resident range.
-    {
-        const int t = threadIdx.x;
-        if (t < 2 * nchunks) {
-            const int cc = t >> 1;
-            const int gq = (t & 1) ? g0 + kRankThreads - 1 : g0;
-            const uint64_t kq = keys[gq];
-            const uint32_t iq = idx[gq];
-            int base = 0;
-#pragma unroll
-            for (int half = kChunk / 2; half > 0; half >>= 1)
-                if (rec_less(keys, idx, cc * kChunk + base + half - 1, kq, iq)) base += half;
-            base += rec_less(keys, idx, cc * kChunk + base, kq, iq) ? 1 : 0;
-            if (t & 1) s_len[cc] = base;  // count for the last record (upper end)
-            else s_lo[cc] = base;
-        }
-    }
-    __syncthreads();
-    if (g >= nchunks * kChunk) return;
+    if (g >= npad) return;
     const uint32_t i = idx[g];
-    if (i >= (uint32_t)n) return;  // padding
-    const uint64_t k = keys[g];
-    int rank = g - c * kChunk;
-    // 2) count within [lo, hi] of each other chunk; kSearchBatch searches in
-    //    lock-step; ranges are short, so fixed-depth searches over pow2 spans.
-    for (int c0 = 0; c0 < nchunks; c0 += kSearchBatch) {
-        int basev[kSearchBatch], hiv[kSearchBatch];
-#pragma unroll
-        for (int j = 0; j < kSearchBatch; j++) {
-            const int cc = min(c0 + j, nchunks - 1);
-            basev[j] = s_lo[cc];        // count >= this
-            hiv[j] = s_len[cc];         // count <= this
-        }
-        // widest bracket of the batch decides the depth (warp-uniform loop)
-        int span = 0;
-#pragma unroll
-        for (int j = 0; j < kSearchBatch; j++) span = max(span, hiv[j] - basev[j]);
-        int step = 1;
-        while (step <= span) step <<= 1;
-        for (step >>= 1; step > 0; step >>= 1) {
-#pragma unroll
-            for (int j = 0; j < kSearchBatch; j++) {
-                const int cc = min(c0 + j, nchunks - 1);
-                const int q = basev[j] + step;  // candidate count
-                if (q <= hiv[j] && rec_less(keys, idx, cc * kChunk + q - 1, k, i)) basev[j] = q;
-            }
-        }
-#pragma unroll
-        for (int j = 0; j < kSearchBatch; j++) {
-            const int cc = c0 + j;
-            if (cc < nchunks && cc != c) rank += basev[j];
-        }
-    }
-    xy[rank] = make_double2(x[i], y[i]);
+    if (i < (uint32_t)n) xy[rank[g]] = make_double2(x[i], y[i]);
 }
 
 }  // namespace krcv

@@ -34,7 +34,7 @@ KR_MAX_M = 65536
 # Every symbol include/krcv.h declares (checked by tests/test_abi.py).
 EXPORTS = (
     "kr_cv_grid", "kr_cv_grid_ex", "kr_cv_grid_algo", "kr_validate_grid", "kr_workspace_bytes",
-    "kr_cv_shard_async", "kr_cv_shard_algo_async", "kr_finalize", "kr_finalize_async", "kr_default_grid",
+    "kr_cv_shard_async", "kr_cv_shard_algo_async", "kr_cv_grid_async", "kr_finalize", "kr_finalize_async", "kr_default_grid",
     "kr_strerror", "kr_last_cuda_error", "kr_version",
     "kr_profile_enable", "kr_profile_read", "kr_launch_count", "kr_last_algo",
 )
@@ -74,11 +74,12 @@ def _lib() -> ctypes.CDLL:
     lib.kr_workspace_bytes.restype = sz
     lib.kr_cv_shard_async.argtypes = [P, P, i64, P, i32, i32, i32, i32, P, P, sz, P]
     lib.kr_cv_shard_algo_async.argtypes = [P, P, i64, P, i32, i32, i32, i32, i32, P, P, sz, P]
+    lib.kr_cv_grid_async.argtypes = [P, P, i64, P, i32, i32, i32, P, P, P, P, sz, P]
     lib.kr_finalize.argtypes = [P, i64, i32, P, P, P]
     lib.kr_finalize_async.argtypes = [P, i64, i32, P, P, P, P, P]
     lib.kr_default_grid.argtypes = [P, i64, i32, P]
     for f in ("kr_cv_grid", "kr_cv_grid_ex", "kr_cv_grid_algo", "kr_validate_grid", "kr_cv_shard_async",
-              "kr_cv_shard_algo_async",
+              "kr_cv_shard_algo_async", "kr_cv_grid_async",
               "kr_finalize", "kr_finalize_async", "kr_default_grid"):
         getattr(lib, f).restype = ctypes.c_int
     lib.kr_strerror.argtypes = [ctypes.c_int]
@@ -215,6 +216,25 @@ def kr_cv_shard_async(d_x, d_y, d_h, kernel, shard: int, nshards: int, d_partial
                                        a, int(shard), int(nshards), d_partial.data_ptr(), d_ws.data_ptr(),
                                        d_ws.numel() * d_ws.element_size(), ctypes.c_void_p(s.cuda_stream))
     _check(st, "kr_cv_shard_algo_async")
+
+
+def kr_cv_grid_async(d_x, d_y, d_h, kernel, d_cv, d_neff, d_best_status, d_ws, stream=None, algo="auto") -> None:
+    """Enqueue the whole single-GPU search (fused finalize): d_cv float64[m],
+    d_neff int64[m] (or None), d_best_status int32[2] -> (best, status)."""
+    import torch
+
+    n, m = d_x.numel(), d_h.numel()
+    for t, name in ((d_x, "x"), (d_y, "y"), (d_h, "h"), (d_cv, "cv")):
+        if not (t.is_cuda and t.dtype == torch.float64 and t.is_contiguous()):
+            raise ValueError(f"{name} must be a contiguous float64 CUDA tensor")
+    if d_cv.numel() != m or d_best_status.numel() != 2 or d_best_status.dtype != torch.int32:
+        raise ValueError("cv must have m elements, best_status 2 int32")
+    s = torch.cuda.current_stream(d_x.device) if stream is None else stream
+    st = _lib().kr_cv_grid_async(d_x.data_ptr(), d_y.data_ptr(), n, d_h.data_ptr(), m, _kernel_id(kernel),
+                                 _algo_id(algo), d_cv.data_ptr(), None if d_neff is None else d_neff.data_ptr(),
+                                 d_best_status.data_ptr(), d_ws.data_ptr(), d_ws.numel() * d_ws.element_size(),
+                                 ctypes.c_void_p(s.cuda_stream))
+    _check(st, "kr_cv_grid_async")
 
 
 def kr_finalize_async(d_partial, n: int, m: int, d_cv, d_neff, d_best_status, stream=None) -> None:

@@ -244,6 +244,23 @@ def test_device_api_matches_host_api():
     assert np.array_equal(r.neff.cpu().numpy(), neff) and r.best == best
 
 
+def test_fused_finalize_matches_shard_plus_finalize():
+    """kr_cv_grid_async (finalize fused into the reduction's last CTA) ==
+    kr_cv_shard_async + host kr_finalize, bit for bit, over repeated calls
+    (the completion counter must reset)."""
+    import torch
+    x, y, h, k = workloads.make("C5", seed=3, n=7000)
+    part = _device_partial(x, y, h, k, 0, 1)
+    cv0, ne0, b0 = krcv.kr_finalize(part, x.shape[0], h.shape[0])
+    plan = GridSearch(x.shape[0], h, k, algo=ALGO["a"])
+    xd, yd = torch.as_tensor(x, device="cuda"), torch.as_tensor(y, device="cuda")
+    for _ in range(3):
+        plan.run(xd, yd)
+        r = plan.result()
+        assert np.array_equal(r.cv.cpu().numpy(), cv0) and np.array_equal(r.neff.cpu().numpy(), ne0)
+        assert r.best == b0
+
+
 @pytest.mark.parametrize("m", [1, 2, 4099])
 def test_grid_sizes(m):
     x, y = workloads.draw_xy("paper", 900, 1)
