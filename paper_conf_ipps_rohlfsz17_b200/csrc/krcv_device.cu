@@ -237,7 +237,7 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     L->pfx = off;      off = align256(off + sizeof(double2) * kPfxMoments * (size_t)L->pstride);
     L->ptot = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
     L->poff = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
-    L->status = off;   off = align256(off + 4 * sizeof(unsigned));  // bad grid, non-finite, done, pad
+    L->status = off;   off = align256(off + 8 * sizeof(unsigned));  // bad grid, non-finite, done, pad, u64 max|y| bits
     L->partial = off;  off = align256(off + sizeof(double) * (size_t)KR_PARTIAL_LEN(m));
     L->cub = off;      off = align256(off + cub_bytes);
     L->cub_bytes = cub_bytes;
@@ -389,11 +389,12 @@ template <int KERN>
 static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, char *ws, cudaStream_t st)
 {
     double *xs = reinterpret_cast<double *>(ws + L.xs) + kPad;
-    double2 *P = reinterpret_cast<double2 *>(ws + L.pfx);
+    double *P = reinterpret_cast<double *>(ws + L.pfx);
     double2 *tot = reinterpret_cast<double2 *>(ws + L.ptot);
+    unsigned long long *ymax = reinterpret_cast<unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
     double2 *off = reinterpret_cast<double2 *>(ws + L.poff);
     const int ntiles = (int)L.nch;
-    pfx_tile_reduce_kernel<KERN><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles);
+    pfx_tile_reduce_kernel<KERN><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, ymax);
     pfx_scan_kernel<KERN><<<1, kPfxScanThreads, 0, st>>>(tot, off, ntiles);
     pfx_tile_scan_kernel<KERN><<<ntiles, kPfxThreads, 0, st>>>(xy, n, off, ntiles, P, (int)L.pstride, xs);
 }
@@ -431,9 +432,11 @@ static void launch_window(const double2 *xy, int n, const double *h, int m, int 
     int blocks = (int)((tasks + kWinWarps - 1) / kWinWarps);
     if (blocks > sms * resident) blocks = sms * resident;
     const double *xs = reinterpret_cast<const double *>(ws + L.xs) + kPad;
-    const double2 *P = reinterpret_cast<const double2 *>(ws + L.pfx);
+    const double *P = reinterpret_cast<const double *>(ws + L.pfx);
+    const unsigned long long *ymax =
+        reinterpret_cast<const unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
     window_kernel<KERN><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc,
-                                                        tileS, tileN, counter);
+                                                        ymax, tileS, tileN, counter);
 }
 
 }  // namespace krcv
@@ -515,7 +518,7 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
 
     int64_t launches = 0;
     prof_mark(0, st);
-    cudaError_t e = cudaMemsetAsync(status, 0, 3 * sizeof(unsigned), st);
+    cudaError_t e = cudaMemsetAsync(status, 0, 8 * sizeof(unsigned), st);
     if (e != cudaSuccess) { set_cuda_error("cudaMemsetAsync(status)", (int)e); return KR_ECUDA; }
     if (n <= kRankSortMaxN && !getenv_flag("KRCV_CUB_SORT")) {
         // a1 + a2: chunk merge sort, rank by counting across chunk pairs, scatter (krcv_sort.cuh)

@@ -24,10 +24,11 @@ struct WsLayout {
     size_t counter;             // int: sweep tile counter
     size_t tileS;               // double  [m][ntiles]  per-tile sum of M e^2
     size_t tileN;               // uint8   [m][ntiles]  per-tile sum of M
-    size_t status;              // uint32  [4]  n_bad_grid, n_nonfinite, reduce completion counter, pad
+    size_t status;              // uint32  [8]  n_bad_grid, n_nonfinite, reduce completion counter, pad,
+                                //              u64 bits of max |y| (window-prefix fast-path bound)
     size_t partial;             // double  [2m+2] partial vector of kr_cv_grid_async
     size_t xs;                  // double  [n + 2 kPad] sorted x, +-inf sentinels (prefix path)
-    size_t pfx;                 // double2 [5][pstride] dd prefix moments P[k][0..n]
+    size_t pfx;                 // double [5][2][pstride] dd prefix moments P[k][0..n], hi / lo planes
     size_t ptot, poff;          // double2 [5][nch] chunk totals / exclusive offsets
     int64_t pstride, nch;
     size_t cub;                 // radix-sort scratch

@@ -110,7 +110,8 @@ __device__ __forceinline__ dd shfl_xor_dd(dd v, int d)
 // Phase 1: per-tile totals of the moment terms -> tot[k][tile].
 template <int KERN>
 __global__ void __launch_bounds__(kPfxThreads)
-pfx_tile_reduce_kernel(const double2 *__restrict__ xy, int n, double2 *__restrict__ tot, int ntiles)
+pfx_tile_reduce_kernel(const double2 *__restrict__ xy, int n, double2 *__restrict__ tot, int ntiles,
+                       unsigned long long *__restrict__ ymax_bits)
 {
     constexpr int K = NMom<KERN>::v;
     __shared__ double2 wsum[K][kPfxThreads / 32];
@@ -120,10 +121,12 @@ pfx_tile_reduce_kernel(const double2 *__restrict__ xy, int n, double2 *__restric
     dd acc[kPfxMoments];
 #pragma unroll
     for (int k = 0; k < K; k++) acc[k] = dd{0.0, 0.0};
+    double ym = 0.0;
 #pragma unroll
     for (int q = 0; q < kPfxItems; q++) {
         if (j0 + q < n) {
             const double2 v = xy[j0 + q];
+            ym = fmax(ym, fabs(v.y));
             dd tm[kPfxMoments];
             moment_terms<KERN>(v.x, v.y, o, tm);
 #pragma unroll
@@ -136,6 +139,11 @@ pfx_tile_reduce_kernel(const double2 *__restrict__ xy, int n, double2 *__restric
         for (int d = 16; d > 0; d >>= 1) acc[k] = dd_add(acc[k], shfl_xor_dd(acc[k], d));
         if (lane == 0) st_dd(&wsum[k][w], acc[k]);
     }
+    // max |y| over all records (the window kernel's fast-path bound);
+    // non-negative doubles order like their bit patterns
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) ym = fmax(ym, __shfl_xor_sync(0xffffffffu, ym, d));
+    if (lane == 0 && ym > 0.0) atomicMax(ymax_bits, (unsigned long long)__double_as_longlong(ym));
     __syncthreads();
     if (t < K) {
         dd a = dd{0.0, 0.0};
@@ -202,7 +210,7 @@ pfx_scan_kernel(const double2 *__restrict__ tot, double2 *__restrict__ off, int 
 template <int KERN>
 __global__ void __launch_bounds__(kPfxThreads)
 pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__restrict__ off, int ntiles,
-                     double2 *__restrict__ P, int pstride, double *__restrict__ xs)
+                     double *__restrict__ P, int pstride, double *__restrict__ xs)
 {
     constexpr int K = NMom<KERN>::v;
     __shared__ double2 wsum[K][kPfxThreads / 32];
@@ -252,7 +260,10 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
         dd run = dd_add(base, ex[k]);
 #pragma unroll
         for (int q = 0; q < kPfxItems; q++) {
-            if (j0 + q <= n) st_dd(P + (size_t)k * pstride + j0 + q, run);
+            if (j0 + q <= n) {
+                P[(size_t)(2 * k) * pstride + j0 + q] = run.hi;
+                P[(size_t)(2 * k + 1) * pstride + j0 + q] = run.lo;
+            }
             run = dd_add(run, tm[q][k]);
         }
     }
@@ -267,8 +278,8 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
 // offset n - r (right) and r + 1 (left) are outside every window.
 // Gallop (first step 1, then the previous growth gR / gL, then doubling) and
 // bisect; both sides advance in the same loop iteration (memory-level
-// parallelism).  (A predicted-bracket variant issued more instructions than
-// it saved probes: profiles/r01f_*.)
+// parallelism).  (Predicted-bracket and interpolation variants issued more
+// instructions than they saved probes: profiles/r01f_*, r01l_*.)
 template <int KERN>
 __device__ __forceinline__ void window_bounds(const double *__restrict__ xs, int n, int r, double xr, double h,
                                               int &kR, int &kL, int gR, int gL)
@@ -316,21 +327,49 @@ __device__ __forceinline__ void window_bounds(const double *__restrict__ xs, int
     kL = lhi;
 }
 
-// Window sums of moment k over sorted indices [a, b): P[b] - P[a].
-__device__ __forceinline__ dd wsum(const double2 *__restrict__ P, int pstride, int k, int a, int b)
+// Prefix storage: structure of arrays, moment k's hi parts at
+// P + 2k pstride, lo parts at P + (2k+1) pstride (the fast path below reads
+// only the hi words).
+__device__ __forceinline__ double ld_hi(const double *__restrict__ P, int ps, int k, int j)
 {
-    return dd_sub(ld_dd(P + (size_t)k * pstride + b), ld_dd(P + (size_t)k * pstride + a));
+    return P[(size_t)(2 * k) * ps + j];
 }
+
+__device__ __forceinline__ dd ld_pdd(const double *__restrict__ P, int ps, int k, int j)
+{
+    return dd{P[(size_t)(2 * k) * ps + j], P[(size_t)(2 * k + 1) * ps + j]};
+}
+
+// Window sums of moment k over sorted indices [a, b): P[b] - P[a], in dd.
+__device__ __forceinline__ dd wsum(const double *__restrict__ P, int ps, int k, int a, int b)
+{
+    return dd_sub(ld_pdd(P, ps, k, b), ld_pdd(P, ps, k, a));
+}
+
+// Fast-path acceptance.  The hi words are the prefix sums
+// rounded to nearest, so a difference of two of them carries an absolute
+// error <= eps/2 (|P[b]| + |P[a]|) + eps |diff|; the shift to the row adds
+// errors of the order of the magnitudes it combines.  E1 / E2 / E0 bound
+// those magnitudes for sum d^2, sum y d^2 and sum y; the fast result is
+// kept only if kFastSlack eps times them is below kFastTol of the
+// denominator (and, for the numerator, of den * max|y|), which bounds the
+// fast path's relative error in den and its absolute error in g_{-i} by
+// kFastTol (times max|y|).  Otherwise the window is recomputed in dd.
+constexpr double kFastSlack = 16.0 * 0x1p-53;
+constexpr double kFastTol = 0x1p-44;
 
 template <int KERN>
 __global__ void __launch_bounds__(kWinThreads)
-window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double2 *__restrict__ P,
+window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
               int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
-              int nbc, double *__restrict__ tileS, uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
+              int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
+              uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
 {
     const int lane = threadIdx.x & 31;
     const double o = pfx_origin(xy, n);
+    const double ymax = __longlong_as_double((long long)*ymax_bits);
     const int bper = (m + nbc - 1) / nbc;
+    const int ps = pstride;
     for (;;) {
         // task = (tile of 32 rows, chunk of bandwidths): the bandwidth loop is
         // split so that small shards still fill the GPU; a chunk starts its
@@ -348,6 +387,7 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
         const double2 vr = xy[r];
         const double xr = vr.x, yr = vr.y;
         const dd del = two_sum(xr, -o);  // exact x_r - o
+        const double dl = del.hi, adl = fabs(del.hi);
         int kR = 1, kL = 1;  // first offsets not yet known inside
         int gR = 1, gL = 1;  // previous growth of each side (first gallop step)
         // triangular splits the window at r: per-row constants P[r], P[r+1]
@@ -355,8 +395,8 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
         if (KERN == KR_TRIANGULAR) {
 #pragma unroll
             for (int k = 0; k < 3; k++) {
-                Pr[k] = ld_dd(P + (size_t)k * pstride + r);
-                Pr1[k] = ld_dd(P + (size_t)k * pstride + r + 1);
+                Pr[k] = ld_pdd(P, ps, k, r);
+                Pr1[k] = ld_pdd(P, ps, k, r + 1);
             }
         }
 
@@ -366,55 +406,84 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
             window_bounds<KERN>(xs, n, r, xr, h, kR, kL, gR, gL);
             gR = max(1, kR - kR0);
             gL = max(1, kL - kL0);
-            const int R = r + kR, L = r - kL;
-            const int cR = R - r - 1, cL = r - L - 1;
-            const int c = cR + cL;
+            const int R = r + kR, L = r - kL, A = L + 1;  // window = [A, R) \ {r}
+            const int c = R - A - 1;
             const bool M = valid && c > 0;  // reading Q6
             double e2 = 0.0;
             if (M) {
                 double g;
                 if (KERN == KR_UNIFORM) {
-                    const dd Sy = wsum(P, pstride, 0, L + 1, R);
-                    g = dd_sub_to_d(Sy, dd_make(yr)) / (double)c;
+                    const double pb = ld_hi(P, ps, 0, R), pa = ld_hi(P, ps, 0, A);
+                    double sy = (pb - pa) - yr;
+                    if (!(kFastSlack * (fabs(pb) + fabs(pa) + fabs(yr)) <= kFastTol * (double)c * ymax))
+                        sy = dd_sub_to_d(wsum(P, ps, 0, A, R), dd_make(yr));
+                    g = sy / (double)c;
                 } else {
-                    double sy, s1, sy1;
-                    if (KERN == KR_EPANECHNIKOV) {
-                        const dd Sy = wsum(P, pstride, 0, L + 1, R);
-                        const dd Su = wsum(P, pstride, 1, L + 1, R);
-                        const dd Suu = wsum(P, pstride, 2, L + 1, R);
-                        const dd Syu = wsum(P, pstride, 3, L + 1, R);
-                        const dd Syuu = wsum(P, pstride, 4, L + 1, R);
-                        const dd t1 = dd_sub(dd_twice(Su), dd_mul_d_raw(del, (double)(c + 1)));
-                        s1 = dd_sub_to_d(Suu, dd_mul_raw(del, t1));
-                        const dd t2 = dd_sub(dd_twice(Syu), dd_mul_raw(del, Sy));
-                        sy1 = dd_sub_to_d(Syuu, dd_mul_raw(del, t2));
-                        sy = dd_sub_to_d(Sy, dd_make(yr));
-                    } else {  // triangular: right (r, R) and left (L, r) separately
-                        const double2 *P0 = P, *P1 = P + pstride, *P2 = P + 2 * (size_t)pstride;
-                        const dd SyR = dd_sub(ld_dd(P0 + R), Pr1[0]);
-                        const dd SuR = dd_sub(ld_dd(P1 + R), Pr1[1]);
-                        const dd SyuR = dd_sub(ld_dd(P2 + R), Pr1[2]);
-                        const dd SyL = dd_sub(Pr[0], ld_dd(P0 + L + 1));
-                        const dd SuL = dd_sub(Pr[1], ld_dd(P1 + L + 1));
-                        const dd SyuL = dd_sub(Pr[2], ld_dd(P2 + L + 1));
-                        // sum d  = (SuR - cR delta) + (cL delta - SuL)
-                        const dd dR = dd_sub(SuR, dd_mul_d_raw(del, (double)cR));
-                        const dd dL = dd_sub(dd_mul_d_raw(del, (double)cL), SuL);
-                        s1 = dd_to_d(dd_add(dR, dL));
-                        // sum y d = (SyuR - delta SyR) + (delta SyL - SyuL)
-                        const dd yR = dd_sub(SyuR, dd_mul_raw(del, SyR));
-                        const dd yL = dd_sub(dd_mul_raw(del, SyL), SyuL);
-                        sy1 = dd_to_d(dd_add(yR, yL));
-                        sy = dd_to_d(dd_add(SyR, SyL));
-                    }
-                    // Eq.(2)-(3) with 0.75 and 1/h^2 cancelled (reading Q5)
                     const double hk = (KERN == KR_EPANECHNIKOV) ? h * h : h;
-                    double num = fma(hk, sy, -sy1);
-                    double den = fma(hk, (double)c, -s1);
+                    double sy, s1, sy1, num, den;
+                    bool fast = false;
+                    if (KERN == KR_EPANECHNIKOV) {
+                        // fast path: hi words only, plain double
+                        const double y_b = ld_hi(P, ps, 0, R), y_a = ld_hi(P, ps, 0, A);
+                        const double u_b = ld_hi(P, ps, 1, R), u_a = ld_hi(P, ps, 1, A);
+                        const double uu_b = ld_hi(P, ps, 2, R), uu_a = ld_hi(P, ps, 2, A);
+                        const double yu_b = ld_hi(P, ps, 3, R), yu_a = ld_hi(P, ps, 3, A);
+                        const double yuu_b = ld_hi(P, ps, 4, R), yuu_a = ld_hi(P, ps, 4, A);
+                        const double c1 = (double)(c + 1);  // range count, row r included (its terms vanish)
+                        const double Sy = y_b - y_a, Su = u_b - u_a, Suu = uu_b - uu_a;
+                        const double Syu = yu_b - yu_a, Syuu = yuu_b - yuu_a;
+                        s1 = fma(-dl, fma(-c1, dl, 2.0 * Su), Suu);
+                        sy1 = fma(-dl, fma(-dl, Sy, 2.0 * Syu), Syuu);
+                        sy = Sy - yr;
+                        num = fma(hk, sy, -sy1);
+                        den = fma(hk, (double)c, -s1);
+                        const double ay = fabs(y_b) + fabs(y_a);
+                        const double E1 = fabs(uu_b) + fabs(uu_a) + 2.0 * adl * (fabs(u_b) + fabs(u_a)) +
+                                          2.0 * c1 * adl * (adl + h);
+                        const double E2 = fabs(yuu_b) + fabs(yuu_a) + 2.0 * adl * (fabs(yu_b) + fabs(yu_a)) +
+                                          2.0 * adl * adl * ay + 2.0 * c1 * ymax * adl * (adl + h);
+                        const double E0 = ay + fabs(yr);
+                        fast = kFastSlack * E1 <= kFastTol * den &&
+                               kFastSlack * fma(hk, E0, E2) <= kFastTol * den * ymax;
+                    }
+                    if (!fast) {
+                        if (KERN == KR_EPANECHNIKOV) {
+                            const dd Sy = wsum(P, ps, 0, A, R);
+                            const dd Su = wsum(P, ps, 1, A, R);
+                            const dd Suu = wsum(P, ps, 2, A, R);
+                            const dd Syu = wsum(P, ps, 3, A, R);
+                            const dd Syuu = wsum(P, ps, 4, A, R);
+                            const dd t1 = dd_sub(dd_twice(Su), dd_mul_d_raw(del, (double)(c + 1)));
+                            s1 = dd_sub_to_d(Suu, dd_mul_raw(del, t1));
+                            const dd t2 = dd_sub(dd_twice(Syu), dd_mul_raw(del, Sy));
+                            sy1 = dd_sub_to_d(Syuu, dd_mul_raw(del, t2));
+                            sy = dd_sub_to_d(Sy, dd_make(yr));
+                        } else {  // triangular: right (r, R) and left (L, r) separately
+                            const dd SyR = dd_sub(ld_pdd(P, ps, 0, R), Pr1[0]);
+                            const dd SuR = dd_sub(ld_pdd(P, ps, 1, R), Pr1[1]);
+                            const dd SyuR = dd_sub(ld_pdd(P, ps, 2, R), Pr1[2]);
+                            const dd SyL = dd_sub(Pr[0], ld_pdd(P, ps, 0, A));
+                            const dd SuL = dd_sub(Pr[1], ld_pdd(P, ps, 1, A));
+                            const dd SyuL = dd_sub(Pr[2], ld_pdd(P, ps, 2, A));
+                            const int cR = R - r - 1, cL = r - L - 1;
+                            // sum d  = (SuR - cR delta) + (cL delta - SuL)
+                            const dd dR = dd_sub(SuR, dd_mul_d_raw(del, (double)cR));
+                            const dd dL = dd_sub(dd_mul_d_raw(del, (double)cL), SuL);
+                            s1 = dd_to_d(dd_add(dR, dL));
+                            // sum y d = (SyuR - delta SyR) + (delta SyL - SyuL)
+                            const dd yR = dd_sub(SyuR, dd_mul_raw(del, SyR));
+                            const dd yL = dd_sub(dd_mul_raw(del, SyL), SyuL);
+                            sy1 = dd_to_d(dd_add(yR, yL));
+                            sy = dd_to_d(dd_add(SyR, SyL));
+                        }
+                        // Eq.(2)-(3) with 0.75 and 1/h^2 cancelled (reading Q5)
+                        num = fma(hk, sy, -sy1);
+                        den = fma(hk, (double)c, -s1);
+                    }
                     if (!(den >= 0x1p-20 * hk * (double)c)) {  // reading Q14
                         num = 0.0;
                         den = 0.0;
-                        for (int q = L + 1; q < R; q++) {
+                        for (int q = A; q < R; q++) {
                             if (q == r) continue;
                             const double2 v = xy[q];
                             const double d = fabs(v.x - xr);
