@@ -45,6 +45,10 @@ SM_MAX_MHZ_NOMINAL = 1965.0     # B200 clocks.max.sm (B200_PROFILING.md)
 # emit, per kernel.
 FLOPS_PER_PAIR = {0: 2, 1: 6, 2: 5}
 FLOPS_PER_EMIT = {0: 4, 1: 9, 2: 9}
+# Window-prefix path: flops per (row, bandwidth) of its double-precision
+# formula (prefix differences, shift to the row frame, estimate, error);
+# DESIGN.md §6.2.
+FLOPS_PER_WINDOW = {0: 6, 1: 25, 2: 30}
 
 
 def parse():
@@ -56,6 +60,7 @@ def parse():
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-alt", action="store_true", help="skip timing the other algorithm (alt_algo)")
     ap.add_argument("--algo", default="auto", choices=["auto", "sweep", "prefix"],
                     help="KR_ALGO_* for every call (sets KRCV_ALGO before the library loads)")
     ap.add_argument("--cpu-seconds", type=float, default=8.0,
@@ -226,94 +231,113 @@ def run_ours(args):
 
     d_x = torch.as_tensor(x, device=dev)
     d_y = torch.as_tensor(y, device=dev)
-    plan = GridSearch(n, h, k, device=dev, rank=rank, world=world)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
     stream = torch.cuda.current_stream(dev)
+    rows_mine = ((rank + 1) * n) // world - (rank * n) // world
 
     def barrier():
         if world > 1:
             torch.distributed.barrier()
 
-    for _ in range(args.warmup):
-        plan.run(d_x, d_y)
-    r = plan.result()
-    torch.cuda.synchronize()
-
-    # ---- device-timed steps (value); L2 flushed between steps, outside the events
-    krcv.kr_profile_enable(True)
-    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    sweep_ms, sort_ms, build_ms = [], [], []
-    launches = 0
-    barrier()
-    torch.cuda.synchronize()
-    with ClockSampler(local) as clk:
-        for s in range(args.steps):
-            flush.fill_(s & 0xFF)
-            starts[s].record(stream)
+    def timed(algo):
+        """W warm-up + K device-timed grid searches with `algo`; L2 flushed
+        between steps (outside the events); max over ranks."""
+        plan = GridSearch(n, h, k, device=dev, rank=rank, world=world, algo=algo)
+        for _ in range(args.warmup):
             plan.run(d_x, d_y)
-            ends[s].record(stream)
-            a, pb, b, _c = krcv.kr_profile_read()  # syncs on this step's events
-            sort_ms.append(a)
-            build_ms.append(pb)
-            sweep_ms.append(b)
-            launches += krcv.kr_launch_count() + (1 if world > 1 else 0)  # + finalize kernel (fused at N=1)
+        plan.result()
         torch.cuda.synchronize()
-    barrier()
-    krcv.kr_profile_enable(False)
-    step_ms = [starts[s].elapsed_time(ends[s]) for s in range(args.steps)]
-    total_ms = sum(step_ms)
-    if world > 1:
-        t = torch.tensor([total_ms, sum(sweep_ms)], dtype=torch.float64, device=dev)
-        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-        total_ms, sweep_total = float(t[0]), float(t[1])
-    else:
-        sweep_total = sum(sweep_ms)
-    res = plan.result()
-    value = units * args.steps / (total_ms * 1e-3)
+        krcv.kr_profile_enable(True)
+        starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+        ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+        main_ms, sort_ms, build_ms, red_ms = [], [], [], []
+        launches = 0
+        barrier()
+        torch.cuda.synchronize()
+        with ClockSampler(local) as clk:
+            for s in range(args.steps):
+                flush.fill_(s & 0xFF)
+                starts[s].record(stream)
+                plan.run(d_x, d_y)
+                ends[s].record(stream)
+                a, pb, b, c = krcv.kr_profile_read()  # syncs on this step's events
+                sort_ms.append(a)
+                build_ms.append(pb)
+                main_ms.append(b)
+                red_ms.append(c)
+                launches += krcv.kr_launch_count() + (1 if world > 1 else 0)  # + finalize (fused at N=1)
+            torch.cuda.synchronize()
+        barrier()
+        krcv.kr_profile_enable(False)
+        used = {1: "sweep", 2: "prefix"}.get(krcv.kr_last_algo(), "?")
+        total_ms = sum(starts[s].elapsed_time(ends[s]) for s in range(args.steps))
+        main_total = sum(main_ms)
+        if world > 1:
+            t = torch.tensor([total_ms, main_total], dtype=torch.float64, device=dev)
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            total_ms, main_total = float(t[0]), float(t[1])
+        res = plan.result()
+        main_s = (main_total / args.steps) * 1e-3
+        peak = SM_COUNT * FP64_LANES_PER_SM * 2 * SM_MAX_MHZ_NOMINAL * 1e6 / 1e12  # TFLOP/s
+        if used == "sweep":
+            kname = "sweep_kernel (a3+a4, per-pair running sums)"
+            flops = rows_mine * (n - 1) * FLOPS_PER_PAIR[k] + rows_mine * m * FLOPS_PER_EMIT[k]
+            basis = (f"{FLOPS_PER_PAIR[k]} flops per ordered pair x rows x (n-1) + {FLOPS_PER_EMIT[k]} per "
+                     "(row, bandwidth) emit")
+        else:
+            kname = "window_kernel (a3+a4, window-prefix)"
+            flops = rows_mine * m * FLOPS_PER_WINDOW[k]
+            basis = (f"{FLOPS_PER_WINDOW[k]} flops per (row, bandwidth): prefix differences, shift to the "
+                     "row, LOO estimate, squared error (DESIGN.md §6.2); searches not counted")
+        achieved = flops / main_s / 1e12
+        return {
+            "algo": used, "value": units * args.steps / (total_ms * 1e-3), "ms_per_step": total_ms / args.steps,
+            "stage_ms": {"pack_sort_gather": sum(sort_ms) / args.steps, "prefix_build": sum(build_ms) / args.steps,
+                         "sweep": sum(main_ms) / args.steps, "reduce_finalize": sum(red_ms) / args.steps},
+            "roofline": {"bound": "alu", "kernel": kname, "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
+                         "frac": achieved / peak, "traffic": None, "flops_per_launch": flops, "flops_basis": basis,
+                         "peak_note": "FP64: 148 SM x 64 FMA lanes x 2 flop x 1965 MHz (derived, DESIGN.md)",
+                         "kernel_ms": main_total / args.steps,
+                         "kernel_share_of_step": main_total / total_ms},
+            "result": {"best": res.best, "h_best": float(h[res.best]), "cv_best": float(res.cv[res.best])},
+            "clocks": clk.summary(), "gpu_launches": launches, "plan": plan,
+        }
+
+    main = timed(args.algo)
+    plan = main.pop("plan")
 
     # ---- end-to-end through the public API, host buffers, H2D/D2H inside
     e2e = e2e_measure(args, x, y, h, k, n, m, units, dev, rank, world, plan)
-
-    # ---- roofline of the dominant kernel (sweep)
-    fl_pair, fl_emit = FLOPS_PER_PAIR[k], FLOPS_PER_EMIT[k]
-    rows_mine = ((rank + 1) * n) // world - (rank * n) // world
-    flops_per_launch = rows_mine * (n - 1) * fl_pair + rows_mine * m * fl_emit
-    sweep_avg_s = (sweep_total / args.steps) * 1e-3
-    peak = SM_COUNT * FP64_LANES_PER_SM * 2 * SM_MAX_MHZ_NOMINAL * 1e6 / 1e12  # TFLOP/s
-    achieved = flops_per_launch / sweep_avg_s / 1e12
-    traffic = None
-    ncu_json = os.path.join(ROOT, "profiles", "sweep_ncu.json")
-    if os.path.exists(ncu_json):
+    traffic_json = os.path.join(ROOT, "profiles", "dram_traffic.json")
+    if os.path.exists(traffic_json):
         try:
-            prof = json.load(open(ncu_json)).get(args.config)
-            if prof:
-                traffic = prof.get("dram_bytes_per_launch")
+            main["roofline"]["traffic"] = json.load(open(traffic_json)).get(args.config, {}).get(main["algo"])
         except Exception:
-            traffic = None
+            pass
 
     out = {
-        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+        "metric": METRIC, "value": main["value"], "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": main["ms_per_step"], "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": workload_desc(cfg, args.seed), "n": n, "m": m,
                    "kernel": workloads.KERNEL_NAMES[k], "seed": args.seed,
                    "parallelism": f"row-shard x{world}" + (" + nccl all_reduce(2m+2 fp64)" if world > 1 else ""),
                    "l2": "flushed between timed steps (256 MiB write, outside the events)"},
-        "roofline": {"bound": "alu", "kernel": "sweep_kernel (a3+a4)", "achieved": achieved,
-                     "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak, "traffic": traffic,
-                     "peak_note": "FP64: 148 SM x 64 FMA lanes x 2 flop x 1965 MHz (derived, DESIGN.md)",
-                     "flops_per_launch": flops_per_launch, "sweep_ms": sweep_total / args.steps,
-                     "sweep_share_of_step": (sweep_total / args.steps) / (total_ms / args.steps)},
-        "stage_ms": {"pack_sort_gather": sum(sort_ms) / args.steps, "prefix_build": sum(build_ms) / args.steps,
-                     "sweep": sum(sweep_ms) / args.steps},
-        "algo": {1: "sweep", 2: "prefix"}.get(krcv.kr_last_algo(), "?"),
-        "result": {"best": res.best, "h_best": float(h[res.best]), "cv_best": float(res.cv[res.best])},
+        "algo": main["algo"],
+        "roofline": main["roofline"],
+        "stage_ms": main["stage_ms"],
+        "result": main["result"],
         "e2e": e2e,
-        "clocks": clk.summary(),
-        "gpu_launches": launches,
+        "clocks": main["clocks"],
+        "gpu_launches": main["gpu_launches"],
         "wall_time_per_grid_search_ms": e2e.get("ms_per_search"),
     }
+    if not args.no_alt:
+        other = "sweep" if main["algo"] == "prefix" else "prefix"
+        alt = timed(other)
+        alt.pop("plan")
+        out["alt_algo"] = {key: alt[key] for key in ("algo", "value", "ms_per_step", "stage_ms", "roofline",
+                                                      "result", "clocks")}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         v, dt, rows, threads = oracle_sample(x, y, h, k, args.cpu_seconds)
         out["cpu_baseline"] = {
