@@ -117,6 +117,26 @@ int kr_cv_grid_algo(const double *x, const double *y, int64_t n,
                     const double *h_grid, int32_t m, int32_t kernel, int32_t algo,
                     double *cv_out, int64_t *neff_out, int32_t *best_out);
 
+/*
+ * kr_cv_refine -- coarse-to-fine grid search.  §IV.A P@20112-20269: "the
+ * user can run the optimization code multiple times with progressively
+ * smaller ranges of possible bandwidths".  Level 0 evaluates h_grid[m];
+ * level l+1 evaluates m_fine evenly spaced bandwidths on [lo, hi] around level
+ * l's best index b (reading Q22): lo = h[b-1] (h[b]/2 if b == 0),
+ * hi = h[b+1] (2 h[b] if b is the last index),
+ * h_j = lo + (hi - lo) * ((double)j / (m_fine - 1)), h_{m_fine-1} = hi.
+ * Levels after the first reuse the device-side sort and prefix moments.
+ *   x, y, n, h_grid, m, kernel, algo  as kr_cv_grid_algo (host pointers)
+ *   levels       1 .. 64; m_fine 3 .. KR_MAX_M (ignored if levels == 1)
+ *   h_best_out   [levels] host: best bandwidth of each level
+ *   cv_best_out  [levels] host: its CV
+ * Synchronous.  Errors: as kr_cv_grid, KR_EARG for bad levels / m_fine.
+ */
+int kr_cv_refine(const double *x, const double *y, int64_t n,
+                 const double *h_grid, int32_t m, int32_t kernel, int32_t algo,
+                 int32_t levels, int32_t m_fine,
+                 double *h_best_out, double *cv_best_out);
+
 /* Host-side grid check (finite, > 0, non-decreasing, 1 <= m <= KR_MAX_M). */
 int kr_validate_grid(const double *h_grid, int32_t m);
 

@@ -163,3 +163,40 @@ def num_threads() -> int:
 
 def real_bits(precision: str = "ld") -> int:
     return int(_lib(precision).kro_real_bits())
+
+
+def refine_grid(h, best: int, m_fine: int) -> np.ndarray:
+    """Level l+1 grid of the coarse-to-fine search (§IV.A P@20112-20269:
+    "run the optimization code multiple times with progressively smaller
+    ranges of possible bandwidths"; the range rule is reading Q22, DESIGN.md
+    §2): m_fine evenly spaced points on [lo, hi], lo = h[b-1] (h[b]/2 if b is
+    the first index), hi = h[b+1] (2 h[b] if b is the last), both ends
+    included: h_j = lo + (hi - lo) * (j / (m_fine - 1)), the last point = hi."""
+    h = [float(v) for v in h]
+    m = len(h)
+    lo = h[best - 1] if best > 0 else h[best] / 2.0
+    hi = h[best + 1] if best < m - 1 else 2.0 * h[best]
+    out = []
+    for j in range(m_fine):
+        t = float(j) / float(m_fine - 1)
+        out.append(lo + (hi - lo) * t)
+    out[-1] = hi
+    return np.array(out, dtype=np.float64)
+
+
+def cv_refine(x, y, h, kernel: int, levels: int, m_fine: int, evaluate=None):
+    """Coarse-to-fine search: level 0 on h, each next level on refine_grid
+    around the previous level's best index.  `evaluate(x, y, h, kernel)`
+    returns an object with .cv and .best (default: cv_sorted).  Returns
+    (h_best[levels], cv_best[levels], grids)."""
+    evaluate = evaluate or (lambda a, b, g, k: cv_sorted(a, b, g, k))
+    grid = np.asarray(h, dtype=np.float64)
+    hb, cb, grids = [], [], []
+    for level in range(levels):
+        grids.append(grid)
+        r = evaluate(x, y, grid, kernel)
+        hb.append(float(grid[r.best]))
+        cb.append(float(r.cv[r.best]))
+        if level + 1 < levels:
+            grid = refine_grid(grid, r.best, m_fine)
+    return np.array(hb), np.array(cb), grids

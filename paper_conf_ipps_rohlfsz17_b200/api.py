@@ -138,3 +138,16 @@ def cv_grid(x, y, h=None, m: int | None = None, kernel="epanechnikov", device=No
     plan = GridSearch(d_x.numel(), h, kernel, dev, rank, world, group, algo)
     plan.run(d_x, d_y)
     return plan.result()
+
+
+def cv_refine(x, y, h=None, m: int | None = None, kernel="epanechnikov", levels: int = 3, m_fine: int = 65,
+              algo="auto"):
+    """Coarse-to-fine search (§IV.A P@20112-20269; reading Q22) on the
+    current CUDA device through kr_cv_refine: returns (h_best, cv_best), one
+    entry per level.  h: level-0 grid, or None with m for the default grid."""
+    xh = np.asarray(x, np.float64)
+    if h is None:
+        if m is None:
+            raise ValueError("give h or m")
+        h = krcv.kr_default_grid(xh, int(m))
+    return krcv.kr_cv_refine(xh, np.asarray(y, np.float64), h, kernel, levels, m_fine, algo)

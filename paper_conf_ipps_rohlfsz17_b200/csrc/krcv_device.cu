@@ -227,8 +227,6 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     L->vals_out = off; off = align256(off + sizeof(uint32_t) * npad);
     L->xy = off;       off = align256(off + sizeof(double2) * ((size_t)n + 2 * kPad));
     L->counter = off;  off = align256(off + sizeof(int));
-    L->tileS = off;    off = align256(off + sizeof(double) * (size_t)ntiles * (size_t)m);
-    L->tileN = off;    off = align256(off + sizeof(uint8_t) * (size_t)ntiles * (size_t)m);
     // window-prefix path (krcv_prefix.cuh)
     const size_t nch = (size_t)((n + kPfxTile) / kPfxTile);  // tiles covering P[0..n]
     L->pstride = (int64_t)(((size_t)n + 1 + 15) & ~size_t(15));
@@ -238,8 +236,13 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     L->ptot = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
     L->poff = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
     L->status = off;   off = align256(off + 8 * sizeof(unsigned));  // bad grid, non-finite, done, pad, u64 max|y| bits
-    L->partial = off;  off = align256(off + sizeof(double) * (size_t)KR_PARTIAL_LEN(m));
     L->cub = off;      off = align256(off + cub_bytes);
+    // m-dependent buffers last: everything above has the same offset for any
+    // m, so a refinement level with another grid size can reuse the sorted
+    // arrays and prefix moments in place (kr_cv_refine)
+    L->tileS = off;    off = align256(off + sizeof(double) * (size_t)ntiles * (size_t)m);
+    L->tileN = off;    off = align256(off + sizeof(uint8_t) * (size_t)ntiles * (size_t)m);
+    L->partial = off;  off = align256(off + sizeof(double) * (size_t)KR_PARTIAL_LEN(m));
     L->cub_bytes = cub_bytes;
     L->total = off;
     L->ntiles_max = ntiles;
@@ -476,9 +479,13 @@ extern "C" size_t kr_workspace_bytes(int64_t n, int32_t m)
 
 // The whole device pipeline of one shard: a1 .. a5, and with fin.cv set the
 // fused finalize (single-GPU whole search).
+// reuse_sorted: the workspace already holds this (x, y)'s sorted arrays (and,
+// for the window-prefix path, its prefix moments for this kernel) from the
+// previous call on it -- only the bandwidth-dependent stages run (the
+// coarse-to-fine refinement, kr_cv_refine).
 static int enqueue(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m, int32_t kernel,
                    int32_t algo, int32_t shard, int32_t nshards, double *d_partial, FinOut fin,
-                   void *d_workspace, size_t workspace_bytes, void *cuda_stream)
+                   void *d_workspace, size_t workspace_bytes, void *cuda_stream, bool reuse_sorted = false)
 {
     if (!d_x || !d_y || !d_h || !d_workspace) return KR_EARG;
     if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return KR_EARG;
@@ -518,9 +525,13 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
 
     int64_t launches = 0;
     prof_mark(0, st);
-    cudaError_t e = cudaMemsetAsync(status, 0, 8 * sizeof(unsigned), st);
+    // reuse keeps max|y| (words 4-5); the host validated x, y and the grid
+    cudaError_t e = cudaMemsetAsync(status, 0, (reuse_sorted ? 3 : 8) * sizeof(unsigned), st);
     if (e != cudaSuccess) { set_cuda_error("cudaMemsetAsync(status)", (int)e); return KR_ECUDA; }
-    if (n <= kRankSortMaxN && !getenv_flag("KRCV_CUB_SORT")) {
+    if (reuse_sorted) {
+        e = cudaMemsetAsync(counter, 0, sizeof(int), st);
+        if (e != cudaSuccess) { set_cuda_error("cudaMemsetAsync(counter)", (int)e); return KR_ECUDA; }
+    } else if (n <= kRankSortMaxN && !getenv_flag("KRCV_CUB_SORT")) {
         // a1 + a2: chunk merge sort, rank by counting across chunk pairs, scatter (krcv_sort.cuh)
         const int nchunks = (int)((n + kChunk - 1) / kChunk);
         uint32_t *khi = reinterpret_cast<uint32_t *>(keys_out);          // keys_out is free on this path
@@ -543,7 +554,7 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         launches += 2 + cub_sort_launches(n);
     }
     prof_mark(1, st);
-    if (prefix) {
+    if (prefix && !reuse_sorted) {
         switch (kernel) {
         case KR_UNIFORM: launch_prefix_build<KR_UNIFORM>(xy, nn, L, ws, st); break;
         case KR_EPANECHNIKOV: launch_prefix_build<KR_EPANECHNIKOV>(xy, nn, L, ws, st); break;
@@ -605,10 +616,9 @@ extern "C" int kr_cv_shard_algo_async(const double *d_x, const double *d_y, int6
                    workspace_bytes, cuda_stream);
 }
 
-extern "C" int kr_cv_grid_async(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m,
-                                int32_t kernel, int32_t algo, double *d_cv, int64_t *d_neff,
-                                int32_t *d_best_status, void *d_workspace, size_t workspace_bytes,
-                                void *cuda_stream)
+int krcv::enqueue_grid(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m,
+                       int32_t kernel, int32_t algo, double *d_cv, int64_t *d_neff, int32_t *d_best_status, void *d_workspace,
+                 size_t workspace_bytes, void *cuda_stream, bool reuse_sorted)
 {
     if (!d_cv || !d_best_status) return KR_EARG;
     FinOut fin{};
@@ -618,7 +628,16 @@ extern "C" int kr_cv_grid_async(const double *d_x, const double *d_y, int64_t n,
     fin.best = d_best_status;
     fin.status = d_best_status + 1;
     return enqueue(d_x, d_y, n, d_h, m, kernel, algo, 0, 1, nullptr, fin, d_workspace, workspace_bytes,
-                   cuda_stream);
+                   cuda_stream, reuse_sorted);
+}
+
+extern "C" int kr_cv_grid_async(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m,
+                                int32_t kernel, int32_t algo, double *d_cv, int64_t *d_neff,
+                                int32_t *d_best_status, void *d_workspace, size_t workspace_bytes,
+                                void *cuda_stream)
+{
+    return enqueue_grid(d_x, d_y, n, d_h, m, kernel, algo, d_cv, d_neff, d_best_status, d_workspace,
+                        workspace_bytes, cuda_stream, false);
 }
 
 extern "C" int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n,

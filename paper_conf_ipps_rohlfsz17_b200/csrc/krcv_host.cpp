@@ -181,6 +181,69 @@ extern "C" int kr_cv_grid(const double *x, const double *y, int64_t n, const dou
     return kr_cv_grid_ex(x, y, n, h_grid, m, kernel, cv_out, nullptr, best_out);
 }
 
+// Level l+1's grid around level l's best index (reading Q22):
+// [lo, hi] = [h[b-1], h[b+1]] (h[b]/2 below the first, 2 h[b] above the
+// last point), m_fine evenly spaced points with both ends included.
+static void refine_grid(const std::vector<double> &h, int32_t best, int32_t m_fine, std::vector<double> &out)
+{
+    const int32_t m = (int32_t)h.size();
+    const double lo = best > 0 ? h[best - 1] : h[best] / 2.0;
+    const double hi = best < m - 1 ? h[best + 1] : 2.0 * h[best];
+    out.resize(m_fine);
+    const double w = hi - lo;
+    for (int32_t j = 0; j < m_fine; j++) {
+        const double t = (double)j / (double)(m_fine - 1);
+        const double p = w * t;
+        out[j] = lo + p;
+    }
+    out[m_fine - 1] = hi;
+}
+
+extern "C" int kr_cv_refine(const double *x, const double *y, int64_t n, const double *h_grid, int32_t m,
+                            int32_t kernel, int32_t algo, int32_t levels, int32_t m_fine, double *h_best_out,
+                            double *cv_best_out)
+{
+    if (!h_best_out || !cv_best_out || levels < 1 || levels > 64) return KR_EARG;
+    if (levels > 1 && (m_fine < 3 || m_fine > KR_MAX_M)) return KR_EARG;
+    if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX) return KR_EARG;
+    int st = validate_all(x, y, n, h_grid, m, kernel);
+    if (st) return st;
+    int dev = 0;
+    KR_CUDA_TRY(cudaGetDevice(&dev));
+    DevCtx *c = get_ctx(dev);
+    std::lock_guard<std::mutex> g(c->mu);
+    const int32_t mcap = levels > 1 && m_fine > m ? m_fine : m;
+    st = ensure_capacity(c, n, mcap);
+    if (st) return st;
+    cudaStream_t s = c->stream;
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dx, x, sizeof(double) * n, cudaMemcpyHostToDevice, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dy, y, sizeof(double) * n, cudaMemcpyHostToDevice, s));
+    std::vector<double> h(h_grid, h_grid + m), next, cv;
+    for (int32_t l = 0; l < levels; l++) {
+        const int32_t ml = (int32_t)h.size();
+        st = kr_validate_grid(h.data(), ml);
+        if (st) return st;  // a refined grid of a degenerate level (lo == hi) is still valid
+        KR_CUDA_TRY(cudaMemcpyAsync(c->dh, h.data(), sizeof(double) * ml, cudaMemcpyHostToDevice, s));
+        // level 0 sorts and builds the prefix moments; later levels reuse them
+        st = enqueue_grid(c->dx, c->dy, n, c->dh, ml, kernel, algo, c->dcv, nullptr, c->dbest, c->ws, c->ws_bytes,
+                          s, l > 0);
+        if (st) return st;
+        cv.resize(ml);
+        int32_t bs[2] = {0, 0};
+        KR_CUDA_TRY(cudaMemcpyAsync(cv.data(), c->dcv, sizeof(double) * ml, cudaMemcpyDeviceToHost, s));
+        KR_CUDA_TRY(cudaMemcpyAsync(bs, c->dbest, sizeof(int32_t) * 2, cudaMemcpyDeviceToHost, s));
+        KR_CUDA_TRY(cudaStreamSynchronize(s));
+        if (bs[1] != KR_OK) return bs[1];
+        h_best_out[l] = h[bs[0]];
+        cv_best_out[l] = cv[bs[0]];
+        if (l + 1 < levels) {
+            refine_grid(h, bs[0], m_fine, next);
+            h.swap(next);
+        }
+    }
+    return KR_OK;
+}
+
 extern "C" int kr_finalize(const double *partial, int64_t n, int32_t m, double *cv_out, int64_t *neff_out,
                            int32_t *best_out)
 {

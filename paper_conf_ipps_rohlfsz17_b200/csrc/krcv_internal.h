@@ -40,6 +40,13 @@ struct WsLayout {
 // Fills `out`; returns false if the CUDA runtime refuses the sort-size query.
 bool ws_layout(int64_t n, int32_t m, WsLayout *out);
 
+// Whole single-GPU search (kr_cv_grid_async) with an optional reuse of the
+// sorted arrays / prefix moments already in the workspace (kr_cv_refine).
+// Defined outside namespace krcv's anonymous parts, in krcv_device.cu.
+int enqueue_grid(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m, int32_t kernel,
+                 int32_t algo, double *d_cv, int64_t *d_neff, int32_t *d_best_status, void *d_workspace,
+                 size_t workspace_bytes, void *cuda_stream, bool reuse_sorted);
+
 // Records a CUDA error string for kr_last_cuda_error (thread-local).
 void set_cuda_error(const char *what, int code);
 

@@ -276,7 +276,7 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
 // every offset in (0, kR) / (0, kL) is inside (the previous windows); on exit
 // kR / kL are the first offsets outside.  xs carries +-inf sentinels, so
 // offset n - r (right) and r + 1 (left) are outside every window.
-// Gallop (first step 1, then the previous growth gR / gL, then doubling) and
+// Gallop (first step = the previous growth gR / gL, then doubling) and
 // bisect; both sides advance in the same loop iteration (memory-level
 // parallelism).  (Predicted-bracket and interpolation variants issued more
 // instructions than they saved probes: profiles/r01f_*, r01l_*.)
@@ -285,17 +285,16 @@ __device__ __forceinline__ void window_bounds(const double *__restrict__ xs, int
                                               int &kR, int &kL, int gR, int gL)
 {
     const double *__restrict__ xsr = xs + r;
-    int rlo = kR - 1, rhi = 0, rstep = 1;  // rlo: inside (or the row itself)
-    int llo = kL - 1, lhi = 0, lstep = 1;
+    int rlo = kR - 1, rhi = 0, rstep = gR;  // rlo: inside (or the row itself)
+    int llo = kL - 1, lhi = 0, lstep = gL;
     const int kRmax = n - r, kLmax = r + 1;
-    bool rg = true, lg = true, rfirst = true, lfirst = true;
+    bool rg = true, lg = true;
     while (rg || lg) {
         if (rg) {
             const int k = min(rlo + rstep, kRmax);
             if (inside<KERN>(xsr[k] - xr, h)) {
                 rlo = k;
-                rstep = rfirst ? gR : 2 * rstep;
-                rfirst = false;
+                rstep *= 2;
             } else {
                 rhi = k;
                 rg = false;
@@ -305,8 +304,7 @@ __device__ __forceinline__ void window_bounds(const double *__restrict__ xs, int
             const int k = min(llo + lstep, kLmax);
             if (inside<KERN>(xr - xsr[-k], h)) {
                 llo = k;
-                lstep = lfirst ? gL : 2 * lstep;
-                lfirst = false;
+                lstep *= 2;
             } else {
                 lhi = k;
                 lg = false;

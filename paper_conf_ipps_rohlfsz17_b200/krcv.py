@@ -33,7 +33,7 @@ KR_MAX_M = 65536
 
 # Every symbol include/krcv.h declares (checked by tests/test_abi.py).
 EXPORTS = (
-    "kr_cv_grid", "kr_cv_grid_ex", "kr_cv_grid_algo", "kr_validate_grid", "kr_workspace_bytes",
+    "kr_cv_grid", "kr_cv_grid_ex", "kr_cv_grid_algo", "kr_cv_refine", "kr_validate_grid", "kr_workspace_bytes",
     "kr_cv_shard_async", "kr_cv_shard_algo_async", "kr_cv_grid_async", "kr_finalize", "kr_finalize_async", "kr_default_grid",
     "kr_strerror", "kr_last_cuda_error", "kr_version",
     "kr_profile_enable", "kr_profile_read", "kr_launch_count", "kr_last_algo",
@@ -69,6 +69,7 @@ def _lib() -> ctypes.CDLL:
     lib.kr_cv_grid.argtypes = [P, P, i64, P, i32, i32, P, P]
     lib.kr_cv_grid_ex.argtypes = [P, P, i64, P, i32, i32, P, P, P]
     lib.kr_cv_grid_algo.argtypes = [P, P, i64, P, i32, i32, i32, P, P, P]
+    lib.kr_cv_refine.argtypes = [P, P, i64, P, i32, i32, i32, i32, i32, P, P]
     lib.kr_validate_grid.argtypes = [P, i32]
     lib.kr_workspace_bytes.argtypes = [i64, i32]
     lib.kr_workspace_bytes.restype = sz
@@ -78,7 +79,7 @@ def _lib() -> ctypes.CDLL:
     lib.kr_finalize.argtypes = [P, i64, i32, P, P, P]
     lib.kr_finalize_async.argtypes = [P, i64, i32, P, P, P, P, P]
     lib.kr_default_grid.argtypes = [P, i64, i32, P]
-    for f in ("kr_cv_grid", "kr_cv_grid_ex", "kr_cv_grid_algo", "kr_validate_grid", "kr_cv_shard_async",
+    for f in ("kr_cv_grid", "kr_cv_grid_ex", "kr_cv_grid_algo", "kr_cv_refine", "kr_validate_grid", "kr_cv_shard_async",
               "kr_cv_shard_algo_async", "kr_cv_grid_async",
               "kr_finalize", "kr_finalize_async", "kr_default_grid"):
         getattr(lib, f).restype = ctypes.c_int
@@ -145,6 +146,19 @@ def kr_cv_grid(x, y, h, kernel="epanechnikov", with_neff: bool = False, algo="au
                            cv.ctypes.data, ctypes.byref(best))
     _check(st, "kr_cv_grid")
     return cv, int(best.value)
+
+
+def kr_cv_refine(x, y, h, kernel="epanechnikov", levels: int = 3, m_fine: int = 65, algo="auto"):
+    """Coarse-to-fine search (§IV.A P@20112): returns (h_best[levels], cv_best[levels])."""
+    x, y, h = _host(x), _host(y), _host(h)
+    if x.shape != y.shape or x.ndim != 1:
+        raise ValueError("x and y must be 1-D arrays of equal length")
+    hb = np.empty(int(levels), np.float64)
+    cb = np.empty(int(levels), np.float64)
+    st = _lib().kr_cv_refine(x.ctypes.data, y.ctypes.data, x.shape[0], h.ctypes.data, h.shape[0], _kernel_id(kernel),
+                             _algo_id(algo), int(levels), int(m_fine), hb.ctypes.data, cb.ctypes.data)
+    _check(st, "kr_cv_refine")
+    return hb, cb
 
 
 def kr_cv_grid_ptr(x_ptr: int, y_ptr: int, n: int, h_ptr: int, m: int, kernel: int,

@@ -286,3 +286,18 @@ def test_rank_sort_heavy_duplicates():
     x = np.floor(x * 7) / 7
     h = workloads.grid_default(x, 20)
     _check(x, y, h, E)
+
+
+@pytest.mark.parametrize("k", [U, E, T])
+@pytest.mark.parametrize("cfg", ["C2", "C5"])
+def test_refine_matches_oracle(cfg, k):
+    """kr_cv_refine (levels > 0 reuse the device-side sort / prefix moments,
+    with grid sizes different from level 0) == the oracle's coarse-to-fine
+    loop (oracle.cv_refine, reading Q22) level by level."""
+    x, y, h, _ = workloads.make(cfg, seed=6, n=3000)
+    hb, cb = krcv.kr_cv_refine(x, y, h, k, levels=4, m_fine=33, algo=ALGO["a"])
+    hb_or, cb_or, _ = oracle.cv_refine(x, y, h, k, levels=4, m_fine=33)
+    assert np.array_equal(hb, hb_or), (hb, hb_or)
+    assert cv_rel_err(cb, cb_or) <= TIGHT
+    with pytest.raises(krcv.KrcvError):
+        krcv.kr_cv_refine(x, y, h, k, levels=3, m_fine=2)

@@ -311,3 +311,41 @@ def test_shard_partials_add_up(P):
     assert cv_rel_err(S, full.S) <= 1e-14
     cv, best = oracle.finalize(S, x.shape[0])
     assert best_ok(best, full.cv)
+
+
+# ---------------------------------------------------------------- Q22 (coarse-to-fine, §IV.A P@20112)
+def test_Q22_refine_grid_rule_hand_values():
+    """The refinement range rule, worked by hand on dyadic grids (exact)."""
+    h = [1.0, 2.0, 3.0, 4.0]
+    assert list(oracle.refine_grid(h, 2, 5)) == [2.0, 2.5, 3.0, 3.5, 4.0]   # [h1, h3]
+    assert list(oracle.refine_grid(h, 0, 4)) == [0.5, 1.0, 1.5, 2.0]        # [h0/2, h1]
+    assert list(oracle.refine_grid(h, 3, 6)) == [3.0, 4.0, 5.0, 6.0, 7.0, 8.0]  # [h2, 2 h3]
+    g = oracle.refine_grid([0.1, 0.2, 0.3], 1, 7)
+    assert g[0] == 0.1 and g[-1] == 0.3 and np.all(np.diff(g) > 0)
+
+
+class _Exact:
+    def __init__(self, cv, best):
+        self.cv = np.array([float(v) for v in cv])
+        self.best = best
+
+
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("k", KERNELS)
+def test_Q22_refine_loop_against_exact(seed, k):
+    """The coarse-to-fine loop driven by the exact-rational evaluator (P1)
+    and by the oracle's Program-3 evaluator pick the same bandwidths; dyadic
+    grids keep every refined point exact, so the exact run is the truth."""
+    x, y, _ = workloads.random_dyadic(12, 4, 300 + seed)
+    h0 = np.array([0.25, 0.75, 1.25, 1.75, 2.25])
+
+    def ex_eval(a, b, g, kk):
+        cv, _ne, best = exact.cv_exact(a, b, g, kk)
+        return _Exact(cv, best)
+
+    hb_ex, cb_ex, grids_ex = oracle.cv_refine(x, y, h0, k, levels=3, m_fine=5, evaluate=ex_eval)
+    hb, cb, grids = oracle.cv_refine(x, y, h0, k, levels=3, m_fine=5)
+    for g1, g2 in zip(grids, grids_ex):
+        assert np.array_equal(g1, g2)
+    assert np.array_equal(hb, hb_ex)
+    assert cv_rel_err(cb, cb_ex) <= 1e-15
