@@ -30,7 +30,7 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _BUILD = os.path.join(_HERE, "build")
 
-UNIFORM, EPANECHNIKOV, TRIANGULAR = 0, 1, 2
+UNIFORM, EPANECHNIKOV, TRIANGULAR, GAUSSIAN = 0, 1, 2, 3
 
 _libs: dict[str, ctypes.CDLL] = {}
 

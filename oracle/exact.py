@@ -68,3 +68,39 @@ def cv_exact(x, y, h, kernel: int):
         neffs.append(ne)
     best = min(range(len(cvs)), key=lambda b: (cvs[b], b))
     return cvs, neffs, best
+
+
+def cv_gauss_decimal(x, y, h, digits: int = 50):
+    """Gaussian-kernel CV by the definition in decimal arithmetic with `digits`
+    significant digits (exp by Decimal.exp): pin P1-G for the long-double
+    oracle.  Eq.(2) with K(u) = exp(-u^2/2) (the normalising constant
+    cancels); every l != i is in the window; no rescaling (the decimal exponent
+    range makes underflow impossible here).  Returns (cv list of Decimal,
+    best index)."""
+    from decimal import Decimal, localcontext
+
+    with localcontext() as ctx:
+        ctx.prec = digits
+        xs = [Decimal(float(v)) for v in x]
+        ys = [Decimal(float(v)) for v in y]
+        n = len(xs)
+        cvs = []
+        for hv in h:
+            hh = Decimal(float(hv))
+            two_h2 = 2 * hh * hh
+            S = Decimal(0)
+            for i in range(n):
+                num = Decimal(0)
+                den = Decimal(0)
+                for l in range(n):
+                    if l == i:
+                        continue
+                    d = xs[l] - xs[i]
+                    w = (-(d * d) / two_h2).exp()
+                    num += ys[l] * w
+                    den += w
+                e = ys[i] - num / den
+                S += e * e
+            cvs.append(S / n)
+        best = min(range(len(cvs)), key=lambda b: (cvs[b], b))
+        return cvs, best

@@ -16,6 +16,9 @@
  *   fn.1   P@18521  "The same approach can be used for the Uniform and
  *                   Triangular kernels"  -> K(u)=1/2 I{|u|<=1},
  *                   K(u)=(1-|u|) I{|u|<1}  (reading Q13, textbook forms)
+ *   P@10203         "straightforward to add additional ones" -> Gaussian
+ *                   K(u) = exp(-u^2/2) (the 1/sqrt(2 pi) cancels in (2));
+ *                   direct evaluator only (reading Q23).
  *
  * Two independent evaluators:
  *
@@ -38,6 +41,11 @@
  *   Q8  leave-one-out excludes the index i only (duplicates of X_i stay).
  *   Q11 best = smallest b with minimal CV; NaN is never minimal.
  *   Q12 arithmetic in long double (KRO_REAL), inputs are binary64.
+ *   Q23 Gaussian: every l != i is in the window (full support), M_i = 1 for
+ *       n >= 2; numerator and denominator of (2) are both multiplied by
+ *       exp(dmin_i^2 / (2 h^2)), dmin_i = min_{l != i} |x_l - x_i| (an exact
+ *       identity), so the nearest neighbour has weight 1 and no weight
+ *       underflow can turn (2) into 0/0.
  *   Q14 the sorted sweep's decomposition h^2 c - sum d^2 cancels when all
  *       in-window points sit near the edge; if 0.75(c - sum d^2/h^2) <
  *       2^-30 * 0.75 c it recomputes numerator and denominator directly from
@@ -62,6 +70,7 @@ typedef KRO_REAL real;
 #define KRO_UNIFORM 0
 #define KRO_EPANECHNIKOV 1
 #define KRO_TRIANGULAR 2
+#define KRO_GAUSSIAN 3
 
 #define KRO_OK 0
 #define KRO_EARG 1
@@ -82,7 +91,8 @@ static int kro_validate(const double *x, const double *y, int64_t n,
 {
     if (!x || !y || !h) return KRO_EARG;
     if (n < 2 || n > 2147483647LL || m < 1 || m > KRO_MAX_M) return KRO_EARG;
-    if (kernel != KRO_UNIFORM && kernel != KRO_EPANECHNIKOV && kernel != KRO_TRIANGULAR)
+    if (kernel != KRO_UNIFORM && kernel != KRO_EPANECHNIKOV && kernel != KRO_TRIANGULAR &&
+        kernel != KRO_GAUSSIAN)
         return KRO_EKERNEL;
     for (int32_t b = 0; b < m; b++) {
         if (!isfinite(h[b]) || !(h[b] > 0.0)) return KRO_EGRID;
@@ -93,9 +103,10 @@ static int kro_validate(const double *x, const double *y, int64_t n,
     return KRO_OK;
 }
 
-/* Q1: the window predicate, binary64. */
+/* Q1: the window predicate, binary64 (Gaussian: full support, Q23). */
 static int in_window(double d, double h, int32_t kernel)
 {
+    if (kernel == KRO_GAUSSIAN) return 1;
     return kernel == KRO_UNIFORM ? (d <= h) : (d < h);
 }
 
@@ -161,11 +172,20 @@ static int direct_core(const double *x, const double *y, int64_t n,
             int64_t i = rows ? rows[r] : r;
             real num = 0, den = 0;      /* Eq.(2) numerator, denominator */
             int64_t cnt = 0;
+            real dmin2 = 0;             /* Gaussian scaling, Q23 */
+            if (kernel == KRO_GAUSSIAN) {
+                double dmin = INFINITY;
+                for (int64_t l = 0; l < n; l++)
+                    if (l != i && fabs(x[l] - x[i]) < dmin) dmin = fabs(x[l] - x[i]);
+                dmin2 = (real)dmin * (real)dmin;
+            }
             for (int64_t l = 0; l < n; l++) {
                 if (l == i) continue;                       /* l != i */
                 double d = fabs(x[l] - x[i]);
                 if (!in_window(d, h[b], kernel)) continue;  /* I{|u| <= 1} */
-                real w = kernel_K(d, h[b], kernel);
+                real w = kernel == KRO_GAUSSIAN
+                             ? expl(-((real)d * (real)d - dmin2) / ((real)2 * (real)h[b] * (real)h[b]))
+                             : kernel_K(d, h[b], kernel);
                 num += (real)y[l] * w;
                 den += w;
                 cnt++;
@@ -307,6 +327,7 @@ int kro_cv_sorted(const double *x, const double *y, int64_t n,
 {
     int st = kro_validate(x, y, n, h, m, kernel);
     if (st) return st;
+    if (kernel == KRO_GAUSSIAN) return KRO_EKERNEL; /* no finite window to sweep (Q23) */
     int64_t R = rows ? nrows : n;
     if (R < 0) return KRO_EARG;
     if (rows)

@@ -349,3 +349,61 @@ def test_Q22_refine_loop_against_exact(seed, k):
         assert np.array_equal(g1, g2)
     assert np.array_equal(hb, hb_ex)
     assert cv_rel_err(cb, cb_ex) <= 1e-15
+
+
+# ---------------------------------------------------------------- Gaussian (Q23, P@10203)
+G = oracle.GAUSSIAN
+
+
+@pytest.mark.parametrize("seed", range(5))
+def test_P1G_gaussian_vs_decimal_definition(seed):
+    """Long-double oracle (with the Q23 nearest-neighbour rescaling) vs the
+    plain definition evaluated in 50-digit decimal arithmetic, including
+    bandwidths so small that far weights underflow binary64."""
+    rng = np.random.default_rng(700 + seed)
+    n = int(rng.integers(2, 11))
+    x = rng.uniform(0, 1, n)
+    y = rng.normal(0, 1, n)
+    h = np.array([0.003, 0.02, 0.1, 0.5, 4.0])
+    r = oracle.cv_direct(x, y, h, G)
+    cv, best = exact.cv_gauss_decimal(x, y, h)
+    assert cv_rel_err(r.cv, [float(v) for v in cv]) <= 1e-15
+    assert r.best == best and list(r.neff) == [n] * h.shape[0]  # M_i = 1 always (Q23)
+
+
+def test_PG_two_points_and_constant_y():
+    """n = 2: the LOO estimate is the other point's y for every h, CV = (y1 - y2)^2."""
+    r = oracle.cv_direct(np.array([0.0, 1.0]), np.array([5.0, 2.0]), np.array([1e-3, 1.0, 1e3]), G)
+    assert np.all(r.cv == 9.0)
+    x, y = workloads.draw_xy("paper", 50, 2)
+    assert np.all(oracle.cv_direct(x, np.full(50, 1.5), np.array([0.01, 0.3]), G).cv <= 1e-30)  # long-double rounding
+
+
+def test_PG_large_h_closed_form():
+    """h -> infinity: every weight -> 1, CV -> n/(n-1)^2 sum (y - ybar)^2 (P3)."""
+    x, y = workloads.draw_xy("sin_uniform", 200, 4)
+    r = oracle.cv_direct(x, y, np.array([1e6 * (x.max() - x.min())]), G)
+    n = x.shape[0]
+    ref = n / (n - 1) ** 2 * float(np.sum((y - y.mean()) ** 2))
+    assert abs(r.cv[0] - ref) / ref <= 1e-10
+
+
+def test_PG_small_h_nearest_neighbour():
+    """h -> 0: the nearest neighbour dominates exponentially; on x with
+    well-separated neighbour distances CV = mean (y_i - y_nn(i))^2."""
+    x = np.array([0.0, 1.0, 3.0, 7.0, 15.0])
+    y = np.array([1.0, -2.0, 0.5, 4.0, 3.0])
+    nn = [1, 0, 1, 2, 3]
+    r = oracle.cv_direct(x, y, np.array([0.05]), G)
+    ref = float(np.mean((y - y[nn]) ** 2))
+    assert abs(r.cv[0] - ref) <= 1e-15 * ref
+
+
+def test_PG_scaling_invariance_and_sorted_rejects():
+    x, y = workloads.draw_xy("paper", 120, 7)
+    h = np.array([0.01, 0.05, 0.2])
+    a = oracle.cv_direct(x, y, h, G).cv
+    b = oracle.cv_direct(x * 8.0, y, h * 8.0, G).cv
+    assert np.array_equal(a, b)
+    with pytest.raises(oracle.OracleError):
+        oracle.cv_sorted(x, y, h, G)

@@ -34,7 +34,9 @@ import numpy as np
 UNIFORM = 0
 EPANECHNIKOV = 1
 TRIANGULAR = 2
-KERNEL_NAMES = {UNIFORM: "uniform", EPANECHNIKOV: "epanechnikov", TRIANGULAR: "triangular"}
+GAUSSIAN = 3
+KERNEL_NAMES = {UNIFORM: "uniform", EPANECHNIKOV: "epanechnikov", TRIANGULAR: "triangular",
+                GAUSSIAN: "gaussian"}
 KERNEL_IDS = {v: k for k, v in KERNEL_NAMES.items()}
 
 
