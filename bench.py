@@ -20,6 +20,7 @@ workload (this tier's reference arm; there is no reference code).
 from __future__ import annotations
 
 import argparse
+import dataclasses
 import json
 import math
 import os
@@ -49,6 +50,10 @@ FLOPS_PER_EMIT = {0: 4, 1: 9, 2: 9}
 # formula (prefix differences, shift to the row frame, estimate, error);
 # DESIGN.md §6.2.
 FLOPS_PER_WINDOW = {0: 6, 1: 25, 2: 30}
+# Dense Gaussian path: per (pair, bandwidth) x = t c (1), e^-x evaluated on
+# the FP64 pipe (Cody-Waite 2 FMA + degree-12 Horner 12 FMA + rounding trick
+# 2 + scale 1 = 31 flops), num FMA (2), den add (1).  DESIGN.md §6.5.
+FLOPS_PER_PAIR_BW_DENSE = 35
 
 
 def parse():
@@ -61,6 +66,8 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-alt", action="store_true", help="skip timing the other algorithm (alt_algo)")
+    ap.add_argument("--kernel", default=None, choices=["uniform", "epanechnikov", "triangular", "gaussian"],
+                    help="override the config's kernel (e.g. the Gaussian dense path on C2's data)")
     ap.add_argument("--algo", default="auto", choices=["auto", "sweep", "prefix"],
                     help="KR_ALGO_* for every call (sets KRCV_ALGO before the library loads)")
     ap.add_argument("--cpu-seconds", type=float, default=8.0,
@@ -147,15 +154,16 @@ def oracle_sample(x, y, h, k, target_s: float):
     order = oracle.sorted_rows(x)
     threads = oracle.num_threads()
     rows = max(2 * threads, 16)
+    evaluate = oracle.cv_direct if k == oracle.GAUSSIAN else oracle.cv_sorted  # no window to sweep (Q23)
     t0 = time.perf_counter()
-    oracle.cv_sorted(x, y, h, k, rows=order[:rows])
+    evaluate(x, y, h, k, rows=order[:rows])
     dt = time.perf_counter() - t0
     per_row = dt / rows
     rows = int(min(n, max(rows, target_s / max(per_row, 1e-9))))
     stride = max(1, n // rows)
     sample = order[::stride][:rows]  # spread over the sorted order
     t0 = time.perf_counter()
-    oracle.cv_sorted(x, y, h, k, rows=sample)
+    evaluate(x, y, h, k, rows=sample)
     dt = time.perf_counter() - t0
     return sample.shape[0] * (n - 1) * m / dt, dt, int(sample.shape[0]), threads
 
@@ -177,6 +185,9 @@ def run_reference(args):
         return 0
     cfg = workloads.CONFIGS[args.config]
     x, y, h, k = workloads.make(cfg, seed=args.seed)
+    if args.kernel:
+        k = workloads.KERNEL_IDS[args.kernel]
+        cfg = dataclasses.replace(cfg, kernel=k)
     n, m = x.shape[0], h.shape[0]
     per_step_target = max(0.5, min(args.cpu_seconds, 120.0 / max(1, args.steps + args.warmup)))
     vals, secs, rows = [], [], 0
@@ -226,6 +237,9 @@ def run_ours(args):
 
     cfg = workloads.CONFIGS[args.config]
     x, y, h, k = workloads.make(cfg, seed=args.seed)
+    if args.kernel:
+        k = workloads.KERNEL_IDS[args.kernel]
+        cfg = dataclasses.replace(cfg, kernel=k)
     n, m = x.shape[0], h.shape[0]
     units = n * (n - 1) * m  # pair-bandwidth evaluations of one full grid search
 
@@ -269,7 +283,7 @@ def run_ours(args):
             torch.cuda.synchronize()
         barrier()
         krcv.kr_profile_enable(False)
-        used = {1: "sweep", 2: "prefix"}.get(krcv.kr_last_algo(), "?")
+        used = {1: "sweep", 2: "prefix", 3: "dense"}.get(krcv.kr_last_algo(), "?")
         total_ms = sum(starts[s].elapsed_time(ends[s]) for s in range(args.steps))
         main_total = sum(main_ms)
         if world > 1:
@@ -279,7 +293,12 @@ def run_ours(args):
         res = plan.result()
         main_s = (main_total / args.steps) * 1e-3
         peak = SM_COUNT * FP64_LANES_PER_SM * 2 * SM_MAX_MHZ_NOMINAL * 1e6 / 1e12  # TFLOP/s
-        if used == "sweep":
+        if used == "dense":
+            kname = "gauss_kernel (a3+a4, tiled all-pairs, Gaussian)"
+            flops = rows_mine * (n - 1) * m * FLOPS_PER_PAIR_BW_DENSE
+            basis = (f"{FLOPS_PER_PAIR_BW_DENSE} flops per (ordered pair, bandwidth) incl. the fp64 exp; "
+                     "column truncation (weights < e^-64) not credited")
+        elif used == "sweep":
             kname = "sweep_kernel (a3+a4, per-pair running sums)"
             flops = rows_mine * (n - 1) * FLOPS_PER_PAIR[k] + rows_mine * m * FLOPS_PER_EMIT[k]
             basis = (f"{FLOPS_PER_PAIR[k]} flops per ordered pair x rows x (n-1) + {FLOPS_PER_EMIT[k]} per "
@@ -332,7 +351,7 @@ def run_ours(args):
         "gpu_launches": main["gpu_launches"],
         "wall_time_per_grid_search_ms": e2e.get("ms_per_search"),
     }
-    if not args.no_alt:
+    if not args.no_alt and main["algo"] != "dense":
         other = "sweep" if main["algo"] == "prefix" else "prefix"
         alt = timed(other)
         alt.pop("plan")
@@ -342,7 +361,8 @@ def run_ours(args):
         v, dt, rows, threads = oracle_sample(x, y, h, k, args.cpu_seconds)
         out["cpu_baseline"] = {
             "value": v, "unit": UNIT, "cores": threads, "kind": "oracle",
-            "sample": (f"kro_cv_sorted on {rows} of {n} rows (strided over the x-sorted order), "
+            "sample": (f"{'kro_cv_direct' if k == 3 else 'kro_cv_sorted'} on {rows} of {n} rows "
+                       "(strided over the x-sorted order), "
                        f"{dt:.1f} s, {threads} OpenMP threads, {cpu_model()}; extrapolated to the full job")}
     if world > 1:
         torch.distributed.barrier()

@@ -50,7 +50,10 @@ extern "C" {
 enum {
     KR_UNIFORM = 0,
     KR_EPANECHNIKOV = 1,
-    KR_TRIANGULAR = 2
+    KR_TRIANGULAR = 2,
+    KR_GAUSSIAN = 3  /* K(u) = exp(-u^2/2), P@10203 "additional [kernels]"; reading Q23:
+                        full support, M_i = 1, weights rescaled by the nearest
+                        neighbour's (exact for Eq.(2)); dense path only */
 };
 
 /* Status codes returned by every int-valued entry point. */
@@ -82,7 +85,11 @@ enum {
 enum {
     KR_ALGO_AUTO = 0,
     KR_ALGO_SWEEP = 1,
-    KR_ALGO_PREFIX = 2
+    KR_ALGO_PREFIX = 2,
+    KR_ALGO_DENSE = 3   /* tiled all-pairs x all-bandwidths, the only path for
+                           KR_GAUSSIAN (AUTO picks it); KR_EARG with the
+                           compact kernels, and SWEEP / PREFIX give KR_EARG
+                           with KR_GAUSSIAN */
 };
 
 /* Length of the partial vector of the device path: [ S[0..m) | neff[0..m) |

@@ -26,6 +26,7 @@
 #include "krcv_sweep_gxg.cuh"
 #include "krcv_sort.cuh"
 #include "krcv_prefix.cuh"
+#include "krcv_dense.cuh"
 
 namespace krcv {
 
@@ -489,8 +490,14 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
 {
     if (!d_x || !d_y || !d_h || !d_workspace) return KR_EARG;
     if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return KR_EARG;
-    if (kernel != KR_UNIFORM && kernel != KR_EPANECHNIKOV && kernel != KR_TRIANGULAR) return KR_EKERNEL;
-    if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX) return KR_EARG;
+    if (kernel != KR_UNIFORM && kernel != KR_EPANECHNIKOV && kernel != KR_TRIANGULAR && kernel != KR_GAUSSIAN)
+        return KR_EKERNEL;
+    if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX && algo != KR_ALGO_DENSE)
+        return KR_EARG;
+    // the Gaussian has no compact support: only the dense path applies, and
+    // the dense path is only for it
+    if ((kernel == KR_GAUSSIAN) != (algo == KR_ALGO_DENSE || (algo == KR_ALGO_AUTO && kernel == KR_GAUSSIAN)))
+        return KR_EARG;
     if (nshards < 1 || shard < 0 || shard >= nshards) return KR_EARG;
     if ((reinterpret_cast<uintptr_t>(d_workspace) & 255u) != 0) return KR_EARG;
     WsLayout L;
@@ -515,13 +522,14 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     // Rows of this shard in sorted order.
     const int lo = (int)(((int64_t)shard * n) / nshards);
     const int hi = (int)(((int64_t)(shard + 1) * n) / nshards);
-    if (algo == KR_ALGO_AUTO) algo = auto_algo(n, hi - lo, m, kernel);
+    if (algo == KR_ALGO_AUTO) algo = kernel == KR_GAUSSIAN ? KR_ALGO_DENSE : auto_algo(n, hi - lo, m, kernel);
     const bool prefix = algo == KR_ALGO_PREFIX;
+    const bool dense = algo == KR_ALGO_DENSE;
     const int variant = sweep_variant(hi - lo);
     int G = sweep_G(hi - lo);
     if (variant == 1 && G > 4) G = 4;
-    const int ntiles = prefix ? (int)tiles_for(hi - lo, 1)
-                              : (variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G));
+    const int ntiles = (prefix || dense) ? (int)tiles_for(hi - lo, 1)
+                                         : (variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G));
 
     int64_t launches = 0;
     prof_mark(0, st);
@@ -565,7 +573,11 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     prof_mark(2, st);
     if (ntiles > 0) {
         launches += 1;
-        if (prefix) {
+        if (dense) {
+            const int nrt = (hi - lo + kGThreads - 1) / kGThreads;
+            const int nbc = (m + kGB - 1) / kGB;
+            gauss_kernel<<<nrt * nbc, kGThreads, 0, st>>>(xy, nn, d_h, m, lo, hi, nbc, ntiles, tileS, tileN);
+        } else if (prefix) {
             switch (kernel) {
             case KR_UNIFORM:
                 launch_window<KR_UNIFORM>(xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);

@@ -22,11 +22,11 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libkrcv.so")
 
-UNIFORM, EPANECHNIKOV, TRIANGULAR = 0, 1, 2
-KERNELS = {"uniform": UNIFORM, "epanechnikov": EPANECHNIKOV, "triangular": TRIANGULAR}
+UNIFORM, EPANECHNIKOV, TRIANGULAR, GAUSSIAN = 0, 1, 2, 3
+KERNELS = {"uniform": UNIFORM, "epanechnikov": EPANECHNIKOV, "triangular": TRIANGULAR, "gaussian": GAUSSIAN}
 
-ALGO_AUTO, ALGO_SWEEP, ALGO_PREFIX = 0, 1, 2
-ALGOS = {"auto": ALGO_AUTO, "sweep": ALGO_SWEEP, "prefix": ALGO_PREFIX}
+ALGO_AUTO, ALGO_SWEEP, ALGO_PREFIX, ALGO_DENSE = 0, 1, 2, 3
+ALGOS = {"auto": ALGO_AUTO, "sweep": ALGO_SWEEP, "prefix": ALGO_PREFIX, "dense": ALGO_DENSE}
 
 KR_OK, KR_EARG, KR_EKERNEL, KR_EGRID, KR_ENONFINITE, KR_EDEGENERATE, KR_ENOMEM, KR_ECUDA = range(8)
 KR_MAX_M = 65536

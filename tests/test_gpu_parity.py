@@ -155,7 +155,7 @@ def _device_partial(x, y, h, k, shard, nshards):
     d_h = torch.as_tensor(h, device="cuda")
     part = torch.empty(krcv.partial_len(h.shape[0]), dtype=torch.float64, device="cuda")
     ws = krcv.aligned(krcv.workspace(x.shape[0], h.shape[0], "cuda"))
-    krcv.kr_cv_shard_async(d_x, d_y, d_h, k, shard, nshards, part, ws, algo=ALGO["a"])
+    krcv.kr_cv_shard_async(d_x, d_y, d_h, k, shard, nshards, part, ws, algo="auto" if k == 3 else ALGO["a"])
     torch.cuda.synchronize()
     return part.cpu().numpy()
 
@@ -301,3 +301,58 @@ def test_refine_matches_oracle(cfg, k):
     assert cv_rel_err(cb, cb_or) <= TIGHT
     with pytest.raises(krcv.KrcvError):
         krcv.kr_cv_refine(x, y, h, k, levels=3, m_fine=2)
+
+
+# ---------------------------------------------------------------- Gaussian (dense path, Q23)
+GA = 3
+
+
+@pytest.mark.parametrize("n", [2, 33, 257, 1000])
+@pytest.mark.parametrize("dist", ["paper", "sin_uniform", "lognormal"])
+def test_gaussian_dense_parity(n, dist):
+    """KR_GAUSSIAN through the tiled all-pairs kernel vs the oracle's direct
+    long-double definition (with the Q23 rescaling); M_i = 1 for every row."""
+    x, y = workloads.draw_xy(dist, n, 11)
+    m = 21
+    h = workloads.grid_log(x, m) if dist == "lognormal" else workloads.grid_default(x, m)
+    cv, neff, best = krcv.kr_cv_grid(x, y, h, GA, with_neff=True)
+    ref = oracle.cv_direct(x, y, h, GA)
+    assert cv_rel_err(cv, ref.cv) <= TIGHT
+    assert np.all(neff == n) and best_ok(best, ref.cv)
+
+
+def test_gaussian_tiny_h_and_duplicates():
+    """Bandwidths so small that unscaled weights would underflow fp64, and
+    heavy ties in x (dmin = 0)."""
+    x, y = workloads.draw_xy("paper", 600, 12)
+    x = np.round(x * 50) / 50
+    h = np.array([1e-5, 1e-3, 0.02, 0.3])
+    cv, neff, best = krcv.kr_cv_grid(x, y, h, GA, with_neff=True)
+    ref = oracle.cv_direct(x, y, h, GA)
+    assert cv_rel_err(cv, ref.cv) <= TIGHT and np.all(neff == 600)
+
+
+def test_gaussian_C2_sampled_shard():
+    """Full C2 size (n = 20,000, 200 bandwidths) with the Gaussian kernel: one
+    sorted-order shard checked row-exactly against the oracle."""
+    x, y, h, _ = workloads.make("C2", seed=0)
+    P, shard = 64, 21
+    part = _device_partial(x, y, h, GA, shard, P)
+    m = h.shape[0]
+    ref = oracle.cv_direct(x, y, h, GA, rows=oracle.shard_rows(x, shard, P))
+    assert cv_rel_err(part[:m], ref.S) <= TIGHT
+    assert np.array_equal(part[m:2 * m].astype(np.int64), ref.neff)
+
+
+def test_gaussian_algorithm_contract():
+    x, y = workloads.draw_xy("paper", 100, 13)
+    h = workloads.grid_default(x, 5)
+    for a in ("sweep", "prefix"):
+        with pytest.raises(krcv.KrcvError) as e:
+            krcv.kr_cv_grid(x, y, h, GA, algo=a)
+        assert e.value.status == krcv.KR_EARG
+    with pytest.raises(krcv.KrcvError):
+        krcv.kr_cv_grid(x, y, h, E, algo="dense")
+    a = krcv.kr_cv_grid(x, y, h, GA, algo="dense")
+    b = krcv.kr_cv_grid(x, y, h, GA)
+    assert np.array_equal(a[0], b[0])
