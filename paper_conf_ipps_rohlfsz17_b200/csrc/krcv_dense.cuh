@@ -19,10 +19,11 @@
 //     and every bandwidth of the chunk (|x_j - x_r| >= sqrt(dmin_max^2 +
 //     128 h_max^2)) are skipped: their total is < n e^-64 relative to the
 //     denominator, far below fp64 rounding;
-//   * exp is evaluated in fp64 on the FP64 pipe (2^k scaling + degree-12
-//     Taylor on |r| <= ln2/2, truncation error < 2e-16).
-// The LOO term j == r gets weight 0.  Per (row, column, bandwidth): 1 DMUL,
-// the exp (17 FP64 ops), 1 DFMA, 1 DADD.
+//   * exp is evaluated in fp64 on the FP64 pipe: a 16-entry 2^(-j/16) table
+//     in shared memory (conflict-free), Cody-Waite reduction, degree-7
+//     Taylor (exp_neg_tab; the table-free exp_neg is kept as its reference).
+// The LOO term j == r gets weight ~1e-304 (see the loop).  Per (row, column, bandwidth): 1 DMUL,
+// the exp (13 FP64 ops + 1 LDS), 1 DFMA, 1 DADD.
 #pragma once
 
 #include <cuda_runtime.h>
@@ -68,6 +69,46 @@ __device__ __forceinline__ double exp_neg(double x)
     return __dmul_rn(p, __hiloint2double((k + 1023) << 20, 0));
 }
 
+// 2^(-j/16), j = 0..15, correctly rounded.  16 doubles = 128 B: staged in
+// shared memory they occupy each of the 32 banks exactly once, so any
+// per-lane index pattern is conflict-free (equal indices broadcast).
+__device__ __constant__ double kExp2Tab[16] = {
+    1.0, 0.9576032806985737, 0.9170040432046712, 0.8781260801866497,
+    0.8408964152537145, 0.8052451659746271, 0.7711054127039704, 0.7384130729697497,
+    0.7071067811865476, 0.6771277734684463, 0.6484197773255048, 0.620928906036742,
+    0.5946035575013605, 0.5693943173783458, 0.5452538663326288, 0.5221368912137069};
+
+// e^{-x} for 0 <= x <= 9e7, table-driven: N = round(16 x / ln2) (1.5 * 2^52
+// trick, N in the low word: an int up to 2^31), r = x - N ln2/16
+// (Cody-Waite, ln2/16 split so N * hi is exact), |r| <= ln2/32;
+// e^{-x} = 2^{-(N>>4)} * 2^{-(N&15)/16} * e^{-r} with e^{-r} by the degree-7
+// Taylor series (truncation < 1.3e-18).  The 2^{-(N>>4)} scaling subtracts
+// from the table value's exponent field, N>>4 clamped at 1010 in the integer
+// domain: for x > 700 the result is ~1e-304 instead of e^{-x}, i.e. zero next
+// to the nearest-neighbour weight 1.  13 FP64-pipe ops + 1 conflict-free LDS
+// (vs 18 FP64 for exp_neg).
+__device__ __forceinline__ double exp_neg_tab(double x, const double *__restrict__ tab)
+{
+    const double kMagic = 6755399441055744.0;  // 1.5 * 2^52
+    const double t = __fma_rn(x, 23.083120654223414, kMagic);
+    const double Nd = __dsub_rn(t, kMagic);
+    const int N = __double2loint(t);
+    double r = __fma_rn(Nd, -0.04332169877307024, x);
+    r = __fma_rn(Nd, -1.1926343307941173e-11, r);
+    double p = -1.98412698412698412698e-04;  // (-1)^7 / 7!
+    p = __fma_rn(p, r, 1.38888888888888888889e-03);
+    p = __fma_rn(p, r, -8.33333333333333333333e-03);
+    p = __fma_rn(p, r, 4.16666666666666666667e-02);
+    p = __fma_rn(p, r, -1.66666666666666666667e-01);
+    p = __fma_rn(p, r, 0.5);
+    p = __fma_rn(p, r, -1.0);
+    p = __fma_rn(p, r, 1.0);
+    const double tb = tab[N & 15];
+    const int q = min(N >> 4, 1010);
+    const double sc = __hiloint2double(__double2hiint(tb) - (q << 20), __double2loint(tb));
+    return __dmul_rn(p, sc);
+}
+
 // First index j in [0, n) with x_j >= v (UPPER: x_j > v) on the sorted x
 // (the sentinels are outside [0, n)).
 template <bool UPPER>
@@ -92,6 +133,7 @@ gauss_kernel(const double2 *__restrict__ xy, int n, const double *__restrict__ h
              int nbc, int ntiles, double *__restrict__ tileS, uint8_t *__restrict__ tileN)
 {
     __shared__ double2 col[kGTile];
+    __shared__ double s_tab[16];
     __shared__ double s_max[kGThreads / 32];
     __shared__ int s_range[2];
     const int rt = blockIdx.x / nbc, bc = blockIdx.x - rt * nbc;
@@ -106,17 +148,27 @@ gauss_kernel(const double2 *__restrict__ xy, int n, const double *__restrict__ h
     const double dmin = fmin(xr - xy[r - 1].x, xy[r + 1].x - xr);
     const double dmin2 = dmin * dmin;
     double c[kGB], num[kGB], den[kGB];
-    double hmax = 0.0;
+    double hmax = 0.0, hmin = INFINITY;
 #pragma unroll
     for (int q = 0; q < kGB; q++) {
         const double h = __ldg(hg + min(b0 + q, m - 1));
         hmax = fmax(hmax, h);
+        hmin = fmin(hmin, h);
         c[q] = 0.5 / (h * h);
         num[q] = 0.0;
         den[q] = 0.0;
     }
+    // cap of t = d^2 - dmin^2 keeping every x = t c <= 9e7 (exp_neg_tab's
+    // range: N = 16 x / ln2 must fit an int); a capped column still has
+    // x >= 9e7 hmin^2/hmax^2 >= 700 for every bandwidth of the chunk when
+    // hmax/hmin <= 300, so its weight stays ~1e-304.  Chunks spanning a wider
+    // bandwidth ratio (extreme grids) clamp x per bandwidth instead (slow
+    // path, block-uniform branch).
+    const bool wide = hmax > 300.0 * hmin;
+    const double ttcap = wide ? INFINITY : 1.8e8 * hmin * hmin;
     // column range that can matter for any row of the tile and bandwidth of
     // the chunk
+    if (t < 16) s_tab[t] = kExp2Tab[t];
     double dm = valid ? dmin2 : 0.0;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) dm = fmax(dm, __shfl_xor_sync(0xffffffffu, dm, o));
@@ -143,14 +195,24 @@ gauss_kernel(const double2 *__restrict__ xy, int n, const double *__restrict__ h
         for (int q = 0; q < cnt; q++) {
             const double2 v = col[q];
             const double d = v.x - xr;
-            const double tt = __fma_rn(d, d, -dmin2);
-            const bool is_self = q == self;  // leave-one-out (Eq.(2) l != i)
+            // leave-one-out (Eq.(2) l != i): the row itself gets t = ttcap, i.e.
+            // weight ~1e-304 next to the nearest neighbour's 1 -- below half
+            // an ulp of every sum it joins, so the sums are unchanged
+            const double tt = q == self ? ttcap : fmin(__fma_rn(d, d, -dmin2), ttcap);
+            if (!wide) {
 #pragma unroll
-            for (int k = 0; k < kGB; k++) {
-                double wgt = exp_neg(tt * c[k]);
-                wgt = is_self ? 0.0 : wgt;
-                num[k] = __fma_rn(wgt, v.y, num[k]);
-                den[k] += wgt;
+                for (int k = 0; k < kGB; k++) {
+                    const double wgt = exp_neg_tab(tt * c[k], s_tab);
+                    num[k] = __fma_rn(wgt, v.y, num[k]);
+                    den[k] += wgt;
+                }
+            } else {
+#pragma unroll
+                for (int k = 0; k < kGB; k++) {
+                    const double wgt = exp_neg_tab(fmin(tt * c[k], 1e4), s_tab);
+                    num[k] = __fma_rn(wgt, v.y, num[k]);
+                    den[k] += wgt;
+                }
             }
         }
     }

@@ -356,3 +356,13 @@ def test_gaussian_algorithm_contract():
     a = krcv.kr_cv_grid(x, y, h, GA, algo="dense")
     b = krcv.kr_cv_grid(x, y, h, GA)
     assert np.array_equal(a[0], b[0])
+
+
+def test_gaussian_wide_bandwidth_chunk():
+    """A chunk of bandwidths spanning more than 1e5 (the kernel's per-bandwidth
+    clamp path) and the normal path give the oracle's curve."""
+    x, y = workloads.draw_xy("lognormal", 700, 14)
+    h = np.array([1e-7, 3e-6, 1e-4, 1e-2, 0.3, 2.0, 30.0, 200.0, 210.0])
+    cv, neff, best = krcv.kr_cv_grid(x, y, h, GA, with_neff=True)
+    ref = oracle.cv_direct(x, y, h, GA)
+    assert cv_rel_err(cv, ref.cv) <= TIGHT and np.all(neff == 700)
