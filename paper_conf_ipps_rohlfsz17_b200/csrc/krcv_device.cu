@@ -403,15 +403,30 @@ static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, cha
     pfx_tile_scan_kernel<KERN><<<ntiles, kPfxThreads, 0, st>>>(xy, n, off, ntiles, P, (int)L.pstride, xs);
 }
 
-template <int KERN>
-static void launch_window(const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
-                          const WsLayout &L, char *ws, double *tileS, uint8_t *tileN, int *counter,
-                          cudaStream_t st)
+// Rows per lane of the window kernel (K consecutive rows; rows 2..K advance
+// from their predecessor's boundaries).  KRCV_WIN_K overrides (1, 2, 4).
+int win_rows_per_lane(int64_t rows)
+{
+    static int forced = -1;
+    if (forced < 0) {
+        const char *e = getenv("KRCV_WIN_K");
+        const int k = e ? atoi(e) : 0;
+        forced = (k == 1 || k == 2 || k == 4) ? k : 0;
+    }
+    if (forced) return forced;
+    // measured (profiles/r01s_*): K = 2 best up to ~1e5 rows, K = 1 above
+    return rows <= 150000 ? 2 : 1;
+}
+
+template <int KERN, int K>
+static void launch_window_k(const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
+                            const WsLayout &L, char *ws, double *tileS, uint8_t *tileN, int *counter,
+                            cudaStream_t st)
 {
     static int resident = 0;
     if (!resident) {
         int b = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel<KERN>, kWinThreads, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel<KERN, K>, kWinThreads, 0);
         resident = b > 0 ? b : 1;
     }
     static int sms = 0;
@@ -439,8 +454,20 @@ static void launch_window(const double2 *xy, int n, const double *h, int m, int 
     const double *P = reinterpret_cast<const double *>(ws + L.pfx);
     const unsigned long long *ymax =
         reinterpret_cast<const unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
-    window_kernel<KERN><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc,
-                                                        ymax, tileS, tileN, counter);
+    window_kernel<KERN, K><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc,
+                                                           ymax, tileS, tileN, counter);
+}
+
+template <int KERN>
+static void launch_window(int K, const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
+                          const WsLayout &L, char *ws, double *tileS, uint8_t *tileN, int *counter,
+                          cudaStream_t st)
+{
+    switch (K) {
+    case 1: launch_window_k<KERN, 1>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    case 2: launch_window_k<KERN, 2>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    default: launch_window_k<KERN, 4>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    }
 }
 
 }  // namespace krcv
@@ -528,8 +555,10 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     const int variant = sweep_variant(hi - lo);
     int G = sweep_G(hi - lo);
     if (variant == 1 && G > 4) G = 4;
-    const int ntiles = (prefix || dense) ? (int)tiles_for(hi - lo, 1)
-                                         : (variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G));
+    const int winK = win_rows_per_lane(hi - lo);
+    const int ntiles = prefix ? (int)((hi - lo + 32 * winK - 1) / (32 * winK))
+                              : dense ? (int)tiles_for(hi - lo, 1)
+                                      : (variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G));
 
     int64_t launches = 0;
     prof_mark(0, st);
@@ -580,13 +609,13 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         } else if (prefix) {
             switch (kernel) {
             case KR_UNIFORM:
-                launch_window<KR_UNIFORM>(xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
+                launch_window<KR_UNIFORM>(winK, xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
                 break;
             case KR_EPANECHNIKOV:
-                launch_window<KR_EPANECHNIKOV>(xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
+                launch_window<KR_EPANECHNIKOV>(winK, xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
                 break;
             default:
-                launch_window<KR_TRIANGULAR>(xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
+                launch_window<KR_TRIANGULAR>(winK, xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
                 break;
             }
         } else {

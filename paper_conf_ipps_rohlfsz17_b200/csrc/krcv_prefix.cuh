@@ -356,7 +356,153 @@ __device__ __forceinline__ dd wsum(const double *__restrict__ P, int ps, int k, 
 constexpr double kFastSlack = 16.0 * 0x1p-53;
 constexpr double kFastTol = 0x1p-44;
 
+// Per-row state of the window kernel.
+struct WinRow {
+    int r;       // sorted row index
+    double xr, yr;
+    dd del;      // x_r - o, exact
+};
+
+// Squared LOO error of row `w` at bandwidth h with window [A, R) \ {r}
+// (c = R - A - 1 >= 1): prefix differences (fast path or dd), Q14 guard,
+// Eq.(2), Eq.(1)'s (y_r - g)^2.  Triangular needs P[r], P[r+1] (pr, pr1).
 template <int KERN>
+__device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c, double h,
+                                            const double2 *__restrict__ xy, const double *__restrict__ P, int ps,
+                                            double ymax)
+{
+    const int r = w.r;
+    const double xr = w.xr, yr = w.yr;
+    const dd del = w.del;
+    const double dl = del.hi, adl = fabs(del.hi);
+    double g;
+    if (KERN == KR_UNIFORM) {
+        const double pb = ld_hi(P, ps, 0, R), pa = ld_hi(P, ps, 0, A);
+        double sy = (pb - pa) - yr;
+        if (!(kFastSlack * (fabs(pb) + fabs(pa) + fabs(yr)) <= kFastTol * (double)c * ymax))
+            sy = dd_sub_to_d(wsum(P, ps, 0, A, R), dd_make(yr));
+        g = sy / (double)c;
+    } else {
+        const double hk = (KERN == KR_EPANECHNIKOV) ? h * h : h;
+        double sy, s1, sy1, num, den;
+        bool fast = false;
+        if (KERN == KR_EPANECHNIKOV) {
+            // fast path: hi words only, plain double (error test: see kFastTol)
+            const double y_b = ld_hi(P, ps, 0, R), y_a = ld_hi(P, ps, 0, A);
+            const double u_b = ld_hi(P, ps, 1, R), u_a = ld_hi(P, ps, 1, A);
+            const double uu_b = ld_hi(P, ps, 2, R), uu_a = ld_hi(P, ps, 2, A);
+            const double yu_b = ld_hi(P, ps, 3, R), yu_a = ld_hi(P, ps, 3, A);
+            const double yuu_b = ld_hi(P, ps, 4, R), yuu_a = ld_hi(P, ps, 4, A);
+            const double c1 = (double)(c + 1);  // range count, row r included (its terms vanish)
+            const double Sy = y_b - y_a, Su = u_b - u_a, Suu = uu_b - uu_a;
+            const double Syu = yu_b - yu_a, Syuu = yuu_b - yuu_a;
+            s1 = fma(-dl, fma(-c1, dl, 2.0 * Su), Suu);
+            sy1 = fma(-dl, fma(-dl, Sy, 2.0 * Syu), Syuu);
+            sy = Sy - yr;
+            num = fma(hk, sy, -sy1);
+            den = fma(hk, (double)c, -s1);
+            const double ay = fabs(y_b) + fabs(y_a);
+            const double E1 = fabs(uu_b) + fabs(uu_a) + 2.0 * adl * (fabs(u_b) + fabs(u_a)) +
+                              2.0 * c1 * adl * (adl + h);
+            const double E2 = fabs(yuu_b) + fabs(yuu_a) + 2.0 * adl * (fabs(yu_b) + fabs(yu_a)) +
+                              2.0 * adl * adl * ay + 2.0 * c1 * ymax * adl * (adl + h);
+            const double E0 = ay + fabs(yr);
+            fast = kFastSlack * E1 <= kFastTol * den && kFastSlack * fma(hk, E0, E2) <= kFastTol * den * ymax;
+        }
+        if (!fast) {
+            if (KERN == KR_EPANECHNIKOV) {
+                const dd Sy = wsum(P, ps, 0, A, R);
+                const dd Su = wsum(P, ps, 1, A, R);
+                const dd Suu = wsum(P, ps, 2, A, R);
+                const dd Syu = wsum(P, ps, 3, A, R);
+                const dd Syuu = wsum(P, ps, 4, A, R);
+                const dd t1 = dd_sub(dd_twice(Su), dd_mul_d_raw(del, (double)(c + 1)));
+                s1 = dd_sub_to_d(Suu, dd_mul_raw(del, t1));
+                const dd t2 = dd_sub(dd_twice(Syu), dd_mul_raw(del, Sy));
+                sy1 = dd_sub_to_d(Syuu, dd_mul_raw(del, t2));
+                sy = dd_sub_to_d(Sy, dd_make(yr));
+            } else {  // triangular: right (r, R) and left [A, r) separately
+                const dd SyR = wsum(P, ps, 0, r + 1, R);
+                const dd SuR = wsum(P, ps, 1, r + 1, R);
+                const dd SyuR = wsum(P, ps, 2, r + 1, R);
+                const dd SyL = wsum(P, ps, 0, A, r);
+                const dd SuL = wsum(P, ps, 1, A, r);
+                const dd SyuL = wsum(P, ps, 2, A, r);
+                const int cR = R - r - 1, cL = r - A;
+                // sum d  = (SuR - cR delta) + (cL delta - SuL)
+                const dd dR = dd_sub(SuR, dd_mul_d_raw(del, (double)cR));
+                const dd dL = dd_sub(dd_mul_d_raw(del, (double)cL), SuL);
+                s1 = dd_to_d(dd_add(dR, dL));
+                // sum y d = (SyuR - delta SyR) + (delta SyL - SyuL)
+                const dd yR = dd_sub(SyuR, dd_mul_raw(del, SyR));
+                const dd yL = dd_sub(dd_mul_raw(del, SyL), SyuL);
+                sy1 = dd_to_d(dd_add(yR, yL));
+                sy = dd_to_d(dd_add(SyR, SyL));
+            }
+            // Eq.(2)-(3) with 0.75 and 1/h^2 cancelled (reading Q5)
+            num = fma(hk, sy, -sy1);
+            den = fma(hk, (double)c, -s1);
+        }
+        if (!(den >= 0x1p-20 * hk * (double)c)) {  // reading Q14
+            num = 0.0;
+            den = 0.0;
+            for (int q = A; q < R; q++) {
+                if (q == r) continue;
+                const double2 v = xy[q];
+                const double d = fabs(v.x - xr);
+                const double wt = (KERN == KR_EPANECHNIKOV) ? (h - d) * (h + d) : (h - d);
+                num = fma(v.y, wt, num);
+                den += wt;
+            }
+        }
+        g = num / den;
+    }
+    const double e = yr - g;
+    return e * e;
+}
+
+// Boundaries of row r + 1 from row r's at the same bandwidth (sorted x:
+// R_{r+1} >= R_r, L_{r+1} >= L_r).  Right: every j in (r+1, R) is inside for
+// row r+1; find the first j >= max(R, r+2) outside.  Left: every j <= L is
+// outside for row r+1; find the last j <= r outside.  Gallop from the known
+// end with steps 1, 2, 4, ... and bisect (typical advance: about one index).
+template <int KERN>
+__device__ __forceinline__ void window_advance(const double *__restrict__ xs, int n, int r1, double xr1, double h,
+                                               int &R, int &L)
+{
+    int rlo = max(R, r1 + 1) - 1, rhi = 0, rstep = 1;  // rlo: inside for r1 (or r1 itself)
+    int llo = L, lhi = 0, lstep = 1;                   // llo: outside for r1
+    bool rg = true, lg = true;
+    while (rg || lg) {
+        if (rg) {
+            const int k = min(rlo + rstep, n);
+            if (inside<KERN>(xs[k] - xr1, h)) { rlo = k; rstep *= 2; } else { rhi = k; rg = false; }
+        }
+        if (lg) {
+            const int k = min(llo + lstep, r1);  // r1 itself is "inside" (d = 0)
+            if (k < r1 && !inside<KERN>(xr1 - xs[k], h)) { llo = k; lstep *= 2; } else { lhi = k; lg = false; }
+        }
+    }
+    while (rhi - rlo > 1 || lhi - llo > 1) {
+        if (rhi - rlo > 1) {
+            const int k = (rlo + rhi) >> 1;
+            if (inside<KERN>(xs[k] - xr1, h)) rlo = k; else rhi = k;
+        }
+        if (lhi - llo > 1) {
+            const int k = (llo + lhi) >> 1;
+            if (!inside<KERN>(xr1 - xs[k], h)) llo = k; else lhi = k;
+        }
+    }
+    R = rhi;
+    L = llo;
+}
+
+// A warp owns 32 * K consecutive sorted rows: lane l the K rows
+// base + l K .. base + l K + K - 1, and a chunk of the bandwidth loop.  Per
+// bandwidth the lane's first row searches from its previous bandwidth's
+// boundaries (window_bounds); each next row starts from its predecessor's
+// boundaries at the same bandwidth (window_advance, ~1 probe per side).
+template <int KERN, int K>
 __global__ void __launch_bounds__(kWinThreads)
 window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
               int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
@@ -369,137 +515,61 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
     const int bper = (m + nbc - 1) / nbc;
     const int ps = pstride;
     for (;;) {
-        // task = (tile of 32 rows, chunk of bandwidths): the bandwidth loop is
+        // task = (tile of 32 K rows, chunk of bandwidths): the bandwidth loop is
         // split so that small shards still fill the GPU; a chunk starts its
         // searches cold (from the row itself), later steps from the previous h.
         int task = 0;
         if (lane == 0) task = atomicAdd(tile_counter, 1);
         task = __shfl_sync(0xffffffffu, task, 0);
         if (task >= ntiles * nbc) return;  // warp-uniform
-        const int tile = task / nbc;
-        const int b0 = (task - tile * nbc) * bper, b1 = min(m, b0 + bper);
+        // chunk-major order: concurrently running warps hold adjacent tiles at
+        // the same bandwidths, so their windows (and probes) overlap in L1/L2
+        const int chunk = task / ntiles;
+        const int tile = task - chunk * ntiles;
+        const int b0 = chunk * bper, b1 = min(m, b0 + bper);
 
-        const int i = row_lo + tile * 32 + lane;
-        const bool valid = i < row_hi;
-        const int r = valid ? i : row_hi - 1;  // clamped rows do identical work, discarded
-        const double2 vr = xy[r];
-        const double xr = vr.x, yr = vr.y;
-        const dd del = two_sum(xr, -o);  // exact x_r - o
-        const double dl = del.hi, adl = fabs(del.hi);
-        int kR = 1, kL = 1;  // first offsets not yet known inside
-        int gR = 1, gL = 1;  // previous growth of each side (first gallop step)
-        // triangular splits the window at r: per-row constants P[r], P[r+1]
-        dd Pr[3], Pr1[3];
-        if (KERN == KR_TRIANGULAR) {
+        const int i0 = row_lo + tile * 32 * K + lane * K;  // this lane's first row
+        WinRow rows[K];
+        int nvalid = 0;
 #pragma unroll
-            for (int k = 0; k < 3; k++) {
-                Pr[k] = ld_pdd(P, ps, k, r);
-                Pr1[k] = ld_pdd(P, ps, k, r + 1);
-            }
+        for (int k = 0; k < K; k++) {
+            const int i = i0 + k;
+            nvalid += i < row_hi ? 1 : 0;
+            rows[k].r = min(i, row_hi - 1);  // clamped rows do identical work, discarded
+            const double2 v = xy[rows[k].r];
+            rows[k].xr = v.x;
+            rows[k].yr = v.y;
+            rows[k].del = two_sum(v.x, -o);  // exact x_r - o
         }
+        int kR = 1, kL = 1;  // first row: first offsets not yet known inside
+        int gR = 1, gL = 1;  // first row: previous growth of each side
 
         for (int b = b0; b < b1; b++) {
             const double h = __ldg(hg + b);
             const int kR0 = kR, kL0 = kL;
-            window_bounds<KERN>(xs, n, r, xr, h, kR, kL, gR, gL);
+            window_bounds<KERN>(xs, n, rows[0].r, rows[0].xr, h, kR, kL, gR, gL);
             gR = max(1, kR - kR0);
             gL = max(1, kL - kL0);
-            const int R = r + kR, L = r - kL, A = L + 1;  // window = [A, R) \ {r}
-            const int c = R - A - 1;
-            const bool M = valid && c > 0;  // reading Q6
+            int R = rows[0].r + kR, L = rows[0].r - kL;
             double e2 = 0.0;
-            if (M) {
-                double g;
-                if (KERN == KR_UNIFORM) {
-                    const double pb = ld_hi(P, ps, 0, R), pa = ld_hi(P, ps, 0, A);
-                    double sy = (pb - pa) - yr;
-                    if (!(kFastSlack * (fabs(pb) + fabs(pa) + fabs(yr)) <= kFastTol * (double)c * ymax))
-                        sy = dd_sub_to_d(wsum(P, ps, 0, A, R), dd_make(yr));
-                    g = sy / (double)c;
-                } else {
-                    const double hk = (KERN == KR_EPANECHNIKOV) ? h * h : h;
-                    double sy, s1, sy1, num, den;
-                    bool fast = false;
-                    if (KERN == KR_EPANECHNIKOV) {
-                        // fast path: hi words only, plain double
-                        const double y_b = ld_hi(P, ps, 0, R), y_a = ld_hi(P, ps, 0, A);
-                        const double u_b = ld_hi(P, ps, 1, R), u_a = ld_hi(P, ps, 1, A);
-                        const double uu_b = ld_hi(P, ps, 2, R), uu_a = ld_hi(P, ps, 2, A);
-                        const double yu_b = ld_hi(P, ps, 3, R), yu_a = ld_hi(P, ps, 3, A);
-                        const double yuu_b = ld_hi(P, ps, 4, R), yuu_a = ld_hi(P, ps, 4, A);
-                        const double c1 = (double)(c + 1);  // range count, row r included (its terms vanish)
-                        const double Sy = y_b - y_a, Su = u_b - u_a, Suu = uu_b - uu_a;
-                        const double Syu = yu_b - yu_a, Syuu = yuu_b - yuu_a;
-                        s1 = fma(-dl, fma(-c1, dl, 2.0 * Su), Suu);
-                        sy1 = fma(-dl, fma(-dl, Sy, 2.0 * Syu), Syuu);
-                        sy = Sy - yr;
-                        num = fma(hk, sy, -sy1);
-                        den = fma(hk, (double)c, -s1);
-                        const double ay = fabs(y_b) + fabs(y_a);
-                        const double E1 = fabs(uu_b) + fabs(uu_a) + 2.0 * adl * (fabs(u_b) + fabs(u_a)) +
-                                          2.0 * c1 * adl * (adl + h);
-                        const double E2 = fabs(yuu_b) + fabs(yuu_a) + 2.0 * adl * (fabs(yu_b) + fabs(yu_a)) +
-                                          2.0 * adl * adl * ay + 2.0 * c1 * ymax * adl * (adl + h);
-                        const double E0 = ay + fabs(yr);
-                        fast = kFastSlack * E1 <= kFastTol * den &&
-                               kFastSlack * fma(hk, E0, E2) <= kFastTol * den * ymax;
-                    }
-                    if (!fast) {
-                        if (KERN == KR_EPANECHNIKOV) {
-                            const dd Sy = wsum(P, ps, 0, A, R);
-                            const dd Su = wsum(P, ps, 1, A, R);
-                            const dd Suu = wsum(P, ps, 2, A, R);
-                            const dd Syu = wsum(P, ps, 3, A, R);
-                            const dd Syuu = wsum(P, ps, 4, A, R);
-                            const dd t1 = dd_sub(dd_twice(Su), dd_mul_d_raw(del, (double)(c + 1)));
-                            s1 = dd_sub_to_d(Suu, dd_mul_raw(del, t1));
-                            const dd t2 = dd_sub(dd_twice(Syu), dd_mul_raw(del, Sy));
-                            sy1 = dd_sub_to_d(Syuu, dd_mul_raw(del, t2));
-                            sy = dd_sub_to_d(Sy, dd_make(yr));
-                        } else {  // triangular: right (r, R) and left (L, r) separately
-                            const dd SyR = dd_sub(ld_pdd(P, ps, 0, R), Pr1[0]);
-                            const dd SuR = dd_sub(ld_pdd(P, ps, 1, R), Pr1[1]);
-                            const dd SyuR = dd_sub(ld_pdd(P, ps, 2, R), Pr1[2]);
-                            const dd SyL = dd_sub(Pr[0], ld_pdd(P, ps, 0, A));
-                            const dd SuL = dd_sub(Pr[1], ld_pdd(P, ps, 1, A));
-                            const dd SyuL = dd_sub(Pr[2], ld_pdd(P, ps, 2, A));
-                            const int cR = R - r - 1, cL = r - L - 1;
-                            // sum d  = (SuR - cR delta) + (cL delta - SuL)
-                            const dd dR = dd_sub(SuR, dd_mul_d_raw(del, (double)cR));
-                            const dd dL = dd_sub(dd_mul_d_raw(del, (double)cL), SuL);
-                            s1 = dd_to_d(dd_add(dR, dL));
-                            // sum y d = (SyuR - delta SyR) + (delta SyL - SyuL)
-                            const dd yR = dd_sub(SyuR, dd_mul_raw(del, SyR));
-                            const dd yL = dd_sub(dd_mul_raw(del, SyL), SyuL);
-                            sy1 = dd_to_d(dd_add(yR, yL));
-                            sy = dd_to_d(dd_add(SyR, SyL));
-                        }
-                        // Eq.(2)-(3) with 0.75 and 1/h^2 cancelled (reading Q5)
-                        num = fma(hk, sy, -sy1);
-                        den = fma(hk, (double)c, -s1);
-                    }
-                    if (!(den >= 0x1p-20 * hk * (double)c)) {  // reading Q14
-                        num = 0.0;
-                        den = 0.0;
-                        for (int q = A; q < R; q++) {
-                            if (q == r) continue;
-                            const double2 v = xy[q];
-                            const double d = fabs(v.x - xr);
-                            const double w = (KERN == KR_EPANECHNIKOV) ? (h - d) * (h + d) : (h - d);
-                            num = fma(v.y, w, num);
-                            den += w;
-                        }
-                    }
-                    g = num / den;
+            int cntM = 0;
+#pragma unroll
+            for (int k = 0; k < K; k++) {
+                if (k > 0) {
+                    if (rows[k].r != rows[k - 1].r)
+                        window_advance<KERN>(xs, n, rows[k].r, rows[k].xr, h, R, L);
                 }
-                const double e = yr - g;
-                e2 = e * e;
+                const int c = R - L - 2;
+                if (k < nvalid && c > 0) {  // reading Q6
+                    e2 += window_e2<KERN>(rows[k], L + 1, R, c, h, xy, P, ps, ymax);
+                    cntM += 1;
+                }
             }
             e2 = warp_sum(e2);
-            const unsigned ball = __ballot_sync(0xffffffffu, M);
+            const int cnt = __reduce_add_sync(0xffffffffu, cntM);  // <= 32 K <= 128: fits the u8 slot
             if (lane == 0) {
                 tileS[(size_t)b * ntiles + tile] = e2;
-                tileN[(size_t)b * ntiles + tile] = (uint8_t)__popc(ball);
+                tileN[(size_t)b * ntiles + tile] = (uint8_t)cnt;
             }
         }
     }
