@@ -411,11 +411,13 @@ int win_rows_per_lane(int64_t rows)
     if (forced < 0) {
         const char *e = getenv("KRCV_WIN_K");
         const int k = e ? atoi(e) : 0;
-        forced = (k == 1 || k == 2 || k == 4) ? k : 0;
+        forced = (k == 1 || k == 2 || k == 3 || k == 4) ? k : 0;  // 3: window_kernel_b2
     }
     if (forced) return forced;
-    // measured (profiles/r01s_*): K = 2 best up to ~1e5 rows, K = 1 above
-    return rows <= 150000 ? 2 : 1;
+    // measured (profiles/r01t_*, r01u_*): two consecutive rows per lane up to
+    // ~1.5e5 rows (C2, C3); above, one row per lane with two bandwidths per
+    // step (window_kernel_b2: C4 22.9 -> 20.9 ms, C5 2.57 -> 2.43 ms)
+    return rows <= 150000 ? 2 : 3;
 }
 
 template <int KERN, int K>
@@ -426,7 +428,10 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
     static int resident = 0;
     if (!resident) {
         int b = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel<KERN, K>, kWinThreads, 0);
+        if (K == 3)
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_b2<KERN>, kWinThreads, 0);
+        else
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel<KERN, K>, kWinThreads, 0);
         resident = b > 0 ? b : 1;
     }
     static int sms = 0;
@@ -454,8 +459,13 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
     const double *P = reinterpret_cast<const double *>(ws + L.pfx);
     const unsigned long long *ymax =
         reinterpret_cast<const unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
-    window_kernel<KERN, K><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc,
-                                                           ymax, tileS, tileN, counter);
+    if (K == 3)
+        window_kernel_b2<KERN><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
+                                                               nbc, ymax, tileS, tileN, counter);
+    else
+        window_kernel<KERN, K == 3 ? 1 : K><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo,
+                                                                            hi, ntiles, nbc, ymax, tileS, tileN,
+                                                                            counter);
 }
 
 template <int KERN>
@@ -466,6 +476,7 @@ static void launch_window(int K, const double2 *xy, int n, const double *h, int 
     switch (K) {
     case 1: launch_window_k<KERN, 1>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     case 2: launch_window_k<KERN, 2>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    case 3: launch_window_k<KERN, 3>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     default: launch_window_k<KERN, 4>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     }
 }
@@ -556,7 +567,8 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     int G = sweep_G(hi - lo);
     if (variant == 1 && G > 4) G = 4;
     const int winK = win_rows_per_lane(hi - lo);
-    const int ntiles = prefix ? (int)((hi - lo + 32 * winK - 1) / (32 * winK))
+    const int rows_per_tile = 32 * (winK == 3 ? 1 : winK);
+    const int ntiles = prefix ? (int)((hi - lo + rows_per_tile - 1) / rows_per_tile)
                               : dense ? (int)tiles_for(hi - lo, 1)
                                       : (variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G));
 

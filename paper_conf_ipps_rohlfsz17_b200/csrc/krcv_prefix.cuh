@@ -575,4 +575,113 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
     }
 }
 
+// Two bandwidths per step: the boundary searches of h_b and h_{b+1} (both
+// sides) start from the same previous boundaries and run as four independent
+// probe chains in one loop -- twice the memory-level parallelism per warp of
+// window_bounds, for a kernel whose time is the latency of dependent probes.
+template <int KERN>
+__device__ __forceinline__ void window_bounds2(const double *__restrict__ xs, int n, int r, double xr, double ha,
+                                               double hb, int kR, int kL, int gR, int gL, int (&kout)[4])
+{
+    const double *__restrict__ xsr = xs + r;
+    // chains: 0 right@ha, 1 left@ha, 2 right@hb, 3 left@hb
+    int lo[4] = {kR - 1, kL - 1, kR - 1, kL - 1};
+    int hi[4] = {0, 0, 0, 0};
+    int st[4] = {gR, gL, 2 * gR, 2 * gL};
+    bool go[4] = {true, true, true, true};
+    const int kmax[4] = {n - r, r + 1, n - r, r + 1};
+    const double hh[4] = {ha, ha, hb, hb};
+    while (go[0] || go[1] || go[2] || go[3]) {
+#pragma unroll
+        for (int c = 0; c < 4; c++) {
+            if (go[c]) {
+                const int k = min(lo[c] + st[c], kmax[c]);
+                const double d = (c & 1) ? xr - xsr[-k] : xsr[k] - xr;
+                if (inside<KERN>(d, hh[c])) { lo[c] = k; st[c] *= 2; } else { hi[c] = k; go[c] = false; }
+            }
+        }
+    }
+    while (hi[0] - lo[0] > 1 || hi[1] - lo[1] > 1 || hi[2] - lo[2] > 1 || hi[3] - lo[3] > 1) {
+#pragma unroll
+        for (int c = 0; c < 4; c++) {
+            if (hi[c] - lo[c] > 1) {
+                const int k = (lo[c] + hi[c]) >> 1;
+                const double d = (c & 1) ? xr - xsr[-k] : xsr[k] - xr;
+                if (inside<KERN>(d, hh[c])) lo[c] = k; else hi[c] = k;
+            }
+        }
+    }
+#pragma unroll
+    for (int c = 0; c < 4; c++) kout[c] = hi[c];
+}
+
+template <int KERN>
+__global__ void __launch_bounds__(kWinThreads)
+window_kernel_b2(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
+                 int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
+                 int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
+                 uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
+{
+    const int lane = threadIdx.x & 31;
+    const double o = pfx_origin(xy, n);
+    const double ymax = __longlong_as_double((long long)*ymax_bits);
+    const int bper = (m + nbc - 1) / nbc;
+    const int ps = pstride;
+    for (;;) {
+        int task = 0;
+        if (lane == 0) task = atomicAdd(tile_counter, 1);
+        task = __shfl_sync(0xffffffffu, task, 0);
+        if (task >= ntiles * nbc) return;  // warp-uniform
+        const int chunk = task / ntiles;  // chunk-major (see window_kernel)
+        const int tile = task - chunk * ntiles;
+        const int b0 = chunk * bper, b1 = min(m, b0 + bper);
+
+        const int i = row_lo + tile * 32 + lane;
+        const bool valid = i < row_hi;
+        WinRow w;
+        w.r = valid ? i : row_hi - 1;  // clamped rows do identical work, discarded
+        const double2 v = xy[w.r];
+        w.xr = v.x;
+        w.yr = v.y;
+        w.del = two_sum(v.x, -o);
+        int kR = 1, kL = 1, gR = 1, gL = 1;
+        for (int b = b0; b < b1; b += 2) {
+            const bool two = b + 1 < b1;
+            const double ha = __ldg(hg + b), hb = two ? __ldg(hg + b + 1) : ha;
+            int ko[4];
+            window_bounds2<KERN>(xs, n, w.r, w.xr, ha, hb, kR, kL, gR, gL, ko);
+            gR = max(1, (ko[2] - kR + 1) / 2);
+            gL = max(1, (ko[3] - kL + 1) / 2);
+            kR = ko[2];
+            kL = ko[3];
+            double e2a = 0.0, e2b = 0.0;
+            bool Ma, Mb;
+            {
+                const int R = w.r + ko[0], L = w.r - ko[1], c = R - L - 2;
+                Ma = valid && c > 0;  // reading Q6
+                if (Ma) e2a = window_e2<KERN>(w, L + 1, R, c, ha, xy, P, ps, ymax);
+            }
+            {
+                const int R = w.r + ko[2], L = w.r - ko[3], c = R - L - 2;
+                Mb = two && valid && c > 0;
+                if (Mb) e2b = window_e2<KERN>(w, L + 1, R, c, hb, xy, P, ps, ymax);
+            }
+#pragma unroll
+            for (int o2 = 16; o2 > 0; o2 >>= 1) {
+                e2a += __shfl_xor_sync(0xffffffffu, e2a, o2);
+                e2b += __shfl_xor_sync(0xffffffffu, e2b, o2);
+            }
+            const unsigned balla = __ballot_sync(0xffffffffu, Ma), ballb = __ballot_sync(0xffffffffu, Mb);
+            if (lane == 0) {
+                tileS[(size_t)b * ntiles + tile] = e2a;
+                tileN[(size_t)b * ntiles + tile] = (uint8_t)__popc(balla);
+                if (two) {
+                    tileS[(size_t)(b + 1) * ntiles + tile] = e2b;
+                    tileN[(size_t)(b + 1) * ntiles + tile] = (uint8_t)__popc(ballb);
+                }
+            }
+        }
+    }
+}
+
 }  // namespace krcv
