@@ -235,7 +235,6 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     L->xs = off;       off = align256(off + sizeof(double) * ((size_t)n + 2 * kPad));
     L->pfx = off;      off = align256(off + sizeof(double2) * kPfxMoments * (size_t)L->pstride);
     L->ptot = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
-    L->poff = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
     L->status = off;   off = align256(off + 8 * sizeof(unsigned));  // bad grid, non-finite, done, pad, u64 max|y| bits
     L->cub = off;      off = align256(off + cub_bytes);
     // m-dependent buffers last: everything above has the same offset for any
@@ -376,6 +375,31 @@ static void prof_mark(int k, cudaStream_t st)
 // against the ncu launch list, profiles/.)
 static int64_t cub_sort_launches(int64_t n) { return n <= kCubSingleTile ? 1 : 2 + 64 / 8; }
 
+// Small-n sort chunk configuration: 0 = 256x4 (1024), 1 = 256x8 (2048),
+// 2 = 512x8 (4096), 3 = 256x2 (512) records per CTA.  Measured
+// (profiles/r01v_*): 1024 fastest for C2 and C3 -- smaller chunks sort faster
+// on more SMs, the extra chunk pairs of the rank step are cheap.
+// KRCV_CHUNK=0..3 overrides.
+int chunk_config(int64_t n)
+{
+    static int forced = -1;
+    if (forced < 0) {
+        const char *e = getenv("KRCV_CHUNK");
+        forced = (e && e[0] >= '0' && e[0] <= '3') ? e[0] - '0' : 4;
+    }
+    if (forced != 4) return forced;
+    (void)n;
+    return 0;
+}
+
+template <int T, int I>
+static void launch_rank_sort(const double *d_x, const double *d_y, int n, const double *d_h, int m, uint64_t *keys,
+                             uint32_t *khi, uint32_t *idx, int *rank, unsigned *status, int nchunks, cudaStream_t st)
+{
+    chunk_sort_kernel<T, I><<<nchunks, T, 0, st>>>(d_x, d_y, n, d_h, m, keys, khi, idx, rank, status);
+    if (nchunks > 1) rank_count_kernel<T, I><<<dim3(nchunks, nchunks), T, 0, st>>>(keys, khi, idx, rank);
+}
+
 // KR_ALGO_AUTO: the window-prefix path does O(n m log) work against the
 // sweep's O(n^2); measured faster on every BASELINE config.
 // KRCV_ALGO=sweep|prefix overrides (benchmarks, A/B tests).
@@ -396,11 +420,9 @@ static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, cha
     double *P = reinterpret_cast<double *>(ws + L.pfx);
     double2 *tot = reinterpret_cast<double2 *>(ws + L.ptot);
     unsigned long long *ymax = reinterpret_cast<unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
-    double2 *off = reinterpret_cast<double2 *>(ws + L.poff);
     const int ntiles = (int)L.nch;
     pfx_tile_reduce_kernel<KERN><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, ymax);
-    pfx_scan_kernel<KERN><<<1, kPfxScanThreads, 0, st>>>(tot, off, ntiles);
-    pfx_tile_scan_kernel<KERN><<<ntiles, kPfxThreads, 0, st>>>(xy, n, off, ntiles, P, (int)L.pstride, xs);
+    pfx_tile_scan_kernel<KERN><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, P, (int)L.pstride, xs);
 }
 
 // Rows per lane of the window kernel (K consecutive rows; rows 2..K advance
@@ -582,14 +604,18 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         if (e != cudaSuccess) { set_cuda_error("cudaMemsetAsync(counter)", (int)e); return KR_ECUDA; }
     } else if (n <= kRankSortMaxN && !getenv_flag("KRCV_CUB_SORT")) {
         // a1 + a2: chunk merge sort, rank by counting across chunk pairs, scatter (krcv_sort.cuh)
-        const int nchunks = (int)((n + kChunk - 1) / kChunk);
+        const int cfg = chunk_config(n);
+        const int chunk = cfg == 0 ? 1024 : (cfg == 1 ? 2048 : (cfg == 2 ? 4096 : 512));
+        const int nchunks = (int)((n + chunk - 1) / chunk);
         uint32_t *khi = reinterpret_cast<uint32_t *>(keys_out);          // keys_out is free on this path
         int *rank = reinterpret_cast<int *>(vals_out);                    // so is vals_out
-        chunk_sort_kernel<<<nchunks, kChunkThreads, 0, st>>>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank,
-                                                            status);
-        if (nchunks > 1)
-            rank_count_kernel<<<dim3(nchunks, nchunks), kChunkThreads, 0, st>>>(keys_in, khi, vals_in, rank);
-        const int npad = nchunks * kChunk;
+        switch (cfg) {
+        case 0: launch_rank_sort<256, 4>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
+        case 1: launch_rank_sort<256, 8>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
+        case 2: launch_rank_sort<512, 8>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
+        default: launch_rank_sort<256, 2>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
+        }
+        const int npad = nchunks * chunk;
         rank_scatter_kernel<<<(npad + 255) / 256, 256, 0, st>>>(vals_in, rank, nn, npad, d_x, d_y, xy, counter);
         launches += nchunks > 1 ? 1 : 0;
         launches += 2;
@@ -609,7 +635,7 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         case KR_EPANECHNIKOV: launch_prefix_build<KR_EPANECHNIKOV>(xy, nn, L, ws, st); break;
         default: launch_prefix_build<KR_TRIANGULAR>(xy, nn, L, ws, st); break;
         }
-        launches += 3;
+        launches += 2;
     }
     prof_mark(2, st);
     if (ntiles > 0) {

@@ -30,8 +30,9 @@
 // Kernels:
 //   pfx_tile_reduce_kernel  per tile of kPfxTile sorted records: moment terms
 //                           and their dd totals
-//   pfx_scan_kernel         one CTA: exclusive scan of the tile totals
-//   pfx_tile_scan_kernel    per tile: prefix values P[k][0..n] and the plain
+//   pfx_tile_scan_kernel    per tile: its offset (fixed-order sum of the
+//                           earlier tiles' totals), prefix values P[k][0..n]
+//                           and the plain
 //                           sorted-x array xs[] (+-inf sentinels) the
 //                           searches read
 //   window_kernel<K>   a warp owns 32 consecutive sorted rows (one per lane),
@@ -51,7 +52,6 @@
 namespace krcv {
 
 constexpr int kPfxThreads = 256;      // prefix build CTA
-constexpr int kPfxScanThreads = 1024;
 constexpr int kPfxMoments = 5;        // slots reserved in the workspace
 constexpr int kWinWarps = 4;
 constexpr int kWinThreads = kWinWarps * 32;
@@ -91,8 +91,9 @@ __device__ __forceinline__ void st_dd(double2 *p, dd v) { *p = make_double2(v.hi
 __device__ __forceinline__ double pfx_origin(const double2 *xy, int n) { return xy[n >> 1].x; }
 
 // ---------------------------------------------------------------- build
-// Three-phase fixed-order scan (bit-reproducible; a decoupled look-back
-// would make the dd rounding depend on timing).  A tile is kPfxTile sorted
+// Two-phase fixed-order scan (bit-reproducible; a decoupled look-back
+// would make the dd rounding depend on timing): tile totals, then every tile
+// sums its predecessors' totals itself and scans its records.  A tile is kPfxTile sorted
 // records; thread t of its CTA owns records 4t .. 4t+3 of the tile.
 constexpr int kPfxItems = 4;
 constexpr int kPfxTile = kPfxThreads * kPfxItems;
@@ -152,68 +153,38 @@ pfx_tile_reduce_kernel(const double2 *__restrict__ xy, int n, double2 *__restric
     }
 }
 
-// Phase 2: exclusive scan of the tile totals, one CTA, fixed order.
-template <int KERN>
-__global__ void __launch_bounds__(kPfxScanThreads)
-pfx_scan_kernel(const double2 *__restrict__ tot, double2 *__restrict__ off, int nch)
-{
-    constexpr int K = NMom<KERN>::v;
-    __shared__ double2 wsum[K][kPfxScanThreads / 32];
-    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-    const int per = (nch + kPfxScanThreads - 1) / kPfxScanThreads;
-    const int c0 = min(nch, t * per), c1 = min(nch, c0 + per);
-    dd s[kPfxMoments];
-#pragma unroll
-    for (int k = 0; k < K; k++) {
-        s[k] = dd{0.0, 0.0};
-        for (int c = c0; c < c1; c++) s[k] = dd_add(s[k], ld_dd(tot + (size_t)k * nch + c));
-    }
-    dd inc[kPfxMoments];
-#pragma unroll
-    for (int k = 0; k < K; k++) {
-        inc[k] = s[k];
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const dd u = shfl_up_dd(inc[k], d);
-            if (lane >= d) inc[k] = dd_add(u, inc[k]);
-        }
-        if (lane == 31) st_dd(&wsum[k][w], inc[k]);
-    }
-    __syncthreads();
-    if (w == 0) {
-#pragma unroll
-        for (int k = 0; k < K; k++) {
-            dd v = ld_dd(&wsum[k][lane]);
-#pragma unroll
-            for (int d = 1; d < 32; d <<= 1) {
-                const dd u = shfl_up_dd(v, d);
-                if (lane >= d) v = dd_add(u, v);
-            }
-            st_dd(&wsum[k][lane], v);  // inclusive over warps
-        }
-    }
-    __syncthreads();
-#pragma unroll
-    for (int k = 0; k < K; k++) {
-        dd run = dd_sub(inc[k], s[k]);  // exclusive within the warp
-        if (w > 0) run = dd_add(ld_dd(&wsum[k][w - 1]), run);
-        for (int c = c0; c < c1; c++) {
-            st_dd(off + (size_t)k * nch + c, run);
-            run = dd_add(run, ld_dd(tot + (size_t)k * nch + c));
-        }
-    }
-}
-
 // Phase 3: in-tile exclusive scan + tile offset -> P[k][j] = sum_{l<j} t_k(l)
 // for j in the tile (and P[k][n] by the last tile), plus the plain sorted-x
 // array xs (with -inf / +inf sentinels) used by the window searches.
 template <int KERN>
 __global__ void __launch_bounds__(kPfxThreads)
-pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__restrict__ off, int ntiles,
+pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__restrict__ tot, int ntiles,
                      double *__restrict__ P, int pstride, double *__restrict__ xs)
 {
     constexpr int K = NMom<KERN>::v;
     __shared__ double2 wsum[K][kPfxThreads / 32];
+    __shared__ double2 base_s[K];
+    // this tile's offset: the totals of all earlier tiles, summed in a fixed
+    // order (strided per thread, then a fixed tree) -- no separate scan launch
+    {
+        const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+        dd a[kPfxMoments];
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            a[k] = dd{0.0, 0.0};
+            for (int q = t; q < (int)blockIdx.x; q += kPfxThreads) a[k] = dd_add(a[k], ld_dd(tot + (size_t)k * ntiles + q));
+#pragma unroll
+            for (int d = 16; d > 0; d >>= 1) a[k] = dd_add(a[k], shfl_xor_dd(a[k], d));
+            if (lane == 0) st_dd(&wsum[k][w], a[k]);
+        }
+        __syncthreads();
+        if (t < K) {
+            dd b = dd{0.0, 0.0};
+            for (int q = 0; q < kPfxThreads / 32; q++) b = dd_add(b, ld_dd(&wsum[t][q]));
+            st_dd(&base_s[t], b);
+        }
+        __syncthreads();
+    }
     const int t = threadIdx.x, lane = t & 31, w = t >> 5;
     const int j0 = blockIdx.x * kPfxTile + t * kPfxItems;
     if (blockIdx.x == 0 && t < kPad) {
@@ -255,7 +226,7 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
     __syncthreads();
 #pragma unroll
     for (int k = 0; k < K; k++) {
-        dd base = ld_dd(off + (size_t)k * ntiles + blockIdx.x);
+        dd base = ld_dd(&base_s[k]);
         for (int q = 0; q < w; q++) base = dd_add(base, ld_dd(&wsum[k][q]));
         dd run = dd_add(base, ex[k]);
 #pragma unroll

@@ -30,10 +30,11 @@
 
 namespace krcv {
 
-constexpr int kChunkThreads = 256;
-constexpr int kChunkItems = 8;
-constexpr int kChunk = kChunkThreads * kChunkItems;  // 2048 records per CTA in K1
-constexpr int64_t kRankSortMaxN = 64 * kChunk;     // 131072: <= 63 searches per record
+// Chunk configurations (threads x items): 256x4 = 1024, 256x8 = 2048,
+// 512x8 = 4096 records per CTA (chunk_config()).  kChunk is the largest, used
+// to pad the workspace arrays so every configuration fits.
+constexpr int kChunk = 4096;
+constexpr int64_t kRankSortMaxN = 131072;
 
 __device__ __forceinline__ uint64_t order_key(double v)
 {
@@ -51,12 +52,14 @@ struct KeyLess {
     __device__ __forceinline__ bool operator()(const uint64_t &a, const uint64_t &b) const { return a < b; }
 };
 
+template <int kChunkThreads, int kChunkItems>
 __global__ void __launch_bounds__(kChunkThreads)
 chunk_sort_kernel(const double *__restrict__ x, const double *__restrict__ y, int n,
                   const double *__restrict__ h, int m, uint64_t *__restrict__ keys,
                   uint32_t *__restrict__ khi, uint32_t *__restrict__ idx, int *__restrict__ rank,
                   unsigned *__restrict__ status)
 {
+    constexpr int kChunk = kChunkThreads * kChunkItems;
     using BMS = cub::BlockMergeSort<uint64_t, kChunkThreads, kChunkItems, uint32_t>;
     __shared__ typename BMS::TempStorage ts;
     const int base = blockIdx.x * kChunk;
@@ -102,10 +105,12 @@ chunk_sort_kernel(const double *__restrict__ x, const double *__restrict__ y, in
 // run in lock-step (ILP) on the high 32 key bits and fall back to the full
 // (key, index) order only when high words tie.  The counts are added to the
 // record's rank with integer atomics (exact, so the result is deterministic).
+template <int kChunkThreads, int kChunkItems>
 __global__ void __launch_bounds__(kChunkThreads)
 rank_count_kernel(const uint64_t *__restrict__ keys, const uint32_t *__restrict__ khi,
                   const uint32_t *__restrict__ idx, int *__restrict__ rank)
 {
+    constexpr int kChunk = kChunkThreads * kChunkItems;
     const int c = blockIdx.x, cc = blockIdx.y;
     if (c == cc) return;
     const int t = threadIdx.x;
