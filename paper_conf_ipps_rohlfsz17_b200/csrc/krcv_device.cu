@@ -433,7 +433,7 @@ int win_rows_per_lane(int64_t rows)
     if (forced < 0) {
         const char *e = getenv("KRCV_WIN_K");
         const int k = e ? atoi(e) : 0;
-        forced = (k == 1 || k == 2 || k == 3 || k == 4) ? k : 0;  // 3: window_kernel_b2
+        forced = (k >= 1 && k <= 5) ? k : 0;  // 3: window_kernel_b2, 5: window_kernel_coop
     }
     if (forced) return forced;
     // measured (profiles/r01t_*, r01u_*): two consecutive rows per lane up to
@@ -452,6 +452,8 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
         int b = 0;
         if (K == 3)
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_b2<KERN>, kWinThreads, 0);
+        else if (K == 5)
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_coop<KERN>, kCoopRows, 0);
         else
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel<KERN, K>, kWinThreads, 0);
         resident = b > 0 ? b : 1;
@@ -475,7 +477,7 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
     const char *fe = getenv("KRCV_WIN_NBC");
     if (fe && atoi(fe) > 0) nbc = atoi(fe) < m ? atoi(fe) : m;
     const int64_t tasks = (int64_t)ntiles * nbc;
-    int blocks = (int)((tasks + kWinWarps - 1) / kWinWarps);
+    int blocks = (int)((tasks + kWinWarps - 1) / kWinWarps);  // kWinWarps == kCoopRows / 32
     if (blocks > sms * resident) blocks = sms * resident;
     const double *xs = reinterpret_cast<const double *>(ws + L.xs) + kPad;
     const double *P = reinterpret_cast<const double *>(ws + L.pfx);
@@ -484,8 +486,11 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
     if (K == 3)
         window_kernel_b2<KERN><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
                                                                nbc, ymax, tileS, tileN, counter);
+    else if (K == 5)
+        window_kernel_coop<KERN><<<blocks, kCoopRows, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
+                                                               nbc, ymax, tileS, tileN, counter);
     else
-        window_kernel<KERN, K == 3 ? 1 : K><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo,
+        window_kernel<KERN, (K == 3 || K == 5) ? 1 : K><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo,
                                                                             hi, ntiles, nbc, ymax, tileS, tileN,
                                                                             counter);
 }
@@ -499,6 +504,7 @@ static void launch_window(int K, const double2 *xy, int n, const double *h, int 
     case 1: launch_window_k<KERN, 1>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     case 2: launch_window_k<KERN, 2>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     case 3: launch_window_k<KERN, 3>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    case 5: launch_window_k<KERN, 5>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     default: launch_window_k<KERN, 4>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     }
 }
@@ -589,7 +595,7 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     int G = sweep_G(hi - lo);
     if (variant == 1 && G > 4) G = 4;
     const int winK = win_rows_per_lane(hi - lo);
-    const int rows_per_tile = 32 * (winK == 3 ? 1 : winK);
+    const int rows_per_tile = 32 * ((winK == 3 || winK == 5) ? 1 : winK);
     const int ntiles = prefix ? (int)((hi - lo + rows_per_tile - 1) / rows_per_tile)
                               : dense ? (int)tiles_for(hi - lo, 1)
                                       : (variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G));

@@ -655,4 +655,160 @@ window_kernel_b2(const double *__restrict__ xs, const double2 *__restrict__ xy, 
     }
 }
 
+// ---------------------------------------------------------------------------
+// Cooperative variant (window_kernel_coop): a CTA owns kCoopRows = 128
+// consecutive sorted rows and a chunk of the bandwidth loop.  Per bandwidth:
+//   1. four "leader" boundaries -- right and left boundary of the tile's first
+//      and last row -- each found by one warp with 32 parallel probes per
+//      round (a 32-ary search from the previous bandwidth's boundary: one or
+//      two dependent round trips instead of ~8);
+//   2. since every row's boundaries lie between its tile's leaders (both are
+//      monotone in the row), the two segments [R_first, R_last] and
+//      [L_first, L_last] of the sorted x are staged in shared memory
+//      (coalesced) and every thread bisects its own boundaries there;
+//   3. the window arithmetic and the per-warp partials are window_e2's.
+// Segments longer than kCoopSeg (sparse data: a tile spanning a wide x range)
+// fall back, CTA-uniformly, to every thread's own global search.
+constexpr int kCoopRows = 128;
+constexpr int kCoopSeg = 1024;
+
+// 32-ary search by one warp: the first offset k > lo (offsets from row r,
+// direction by RIGHT) that is outside the window of row (r, xr) at h, given
+// that lo is inside (0 = the row itself) and the boundary is expected about
+// g past lo.  Returns the same value in every lane.
+template <int KERN, bool RIGHT>
+__device__ __forceinline__ int warp_boundary(const double *__restrict__ xs, int n, int r, double xr, double h, int lo,
+                                             int g, int lane)
+{
+    const int kmax = RIGHT ? n - r : r + 1;  // sentinel offset: outside
+    int s = max(1, (2 * g + 31) / 32);
+    for (;;) {
+        const int k = min(lo + (lane + 1) * s, kmax);
+        const double d = RIGHT ? xs[r + k] - xr : xr - xs[r - k];
+        const unsigned in = __ballot_sync(0xffffffffu, inside<KERN>(d, h));
+        const int cnt = __popc(in);  // inside probes form a prefix
+        if (cnt == 32) {             // all 32 inside: move on, widen
+            lo = min(lo + 32 * s, kmax);
+            s *= 2;
+            continue;
+        }
+        const int hi = min(lo + (cnt + 1) * s, kmax);  // first probed outside
+        lo = lo + cnt * s;                              // last probed inside
+        if (hi - lo <= 1) return hi;
+        s = (hi - lo + 31) / 32;  // refine inside (lo, hi)
+        if (s == 1) {
+            const int k2 = min(lo + lane + 1, hi);
+            const double d2 = RIGHT ? xs[r + k2] - xr : xr - xs[r - k2];
+            const unsigned in2 = __ballot_sync(0xffffffffu, k2 < hi && inside<KERN>(d2, h));
+            return lo + __popc(in2) + 1;
+        }
+    }
+}
+
+template <int KERN>
+__global__ void __launch_bounds__(kCoopRows)
+window_kernel_coop(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
+                   int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
+                   int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
+                   uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
+{
+    __shared__ double segR[kCoopSeg], segL[kCoopSeg];
+    __shared__ int s_lead[4];  // R_first, R_last (absolute), L_first, L_last (absolute)
+    __shared__ int s_task;
+    const int t = threadIdx.x, lane = t & 31, wp = t >> 5;
+    const double o = pfx_origin(xy, n);
+    const double ymax = __longlong_as_double((long long)*ymax_bits);
+    const int bper = (m + nbc - 1) / nbc;
+    const int ps = pstride;
+    const int ctiles = (ntiles + 3) / 4;  // CTA tiles of 128 rows (ntiles counts 32-row tiles)
+    for (;;) {
+        __syncthreads();
+        if (t == 0) s_task = atomicAdd(tile_counter, 1);
+        __syncthreads();
+        const int task = s_task;
+        if (task >= ctiles * nbc) return;  // block-uniform
+        const int chunk = task / ctiles;
+        const int ct = task - chunk * ctiles;
+        const int b0 = chunk * bper, b1 = min(m, b0 + bper);
+        const int first = row_lo + ct * kCoopRows;
+        const int last = min(row_hi, first + kCoopRows) - 1;
+
+        const int i = first + t;
+        const bool valid = i <= last;
+        WinRow w;
+        w.r = valid ? i : last;
+        const double2 v = xy[w.r];
+        w.xr = v.x;
+        w.yr = v.y;
+        w.del = two_sum(v.x, -o);
+        int kR = 1, kL = 1, gR = 1, gL = 1;  // this row's previous boundaries (offsets) and growth
+        // leader state (offsets from the leader row): warp 0 R of first, 1 R of
+        // last, 2 L of first, 3 L of last
+        const int lrow = (wp & 1) ? last : first;
+        const double lx = xy[lrow].x;
+        int lk = 1, lg = 1;
+
+        for (int b = b0; b < b1; b++) {
+            const double h = __ldg(hg + b);
+            // 1. leaders
+            {
+                const int k = (wp < 2) ? warp_boundary<KERN, true>(xs, n, lrow, lx, h, lk - 1, lg, lane)
+                                       : warp_boundary<KERN, false>(xs, n, lrow, lx, h, lk - 1, lg, lane);
+                lg = max(1, k - lk);
+                lk = k;
+                if (lane == 0) s_lead[wp] = (wp < 2) ? lrow + k : lrow - k;
+            }
+            __syncthreads();
+            const int Rf = s_lead[0], Rl = s_lead[1], Lf = s_lead[2], Ll = s_lead[3];
+            const int lenR = Rl - Rf + 1, lenL = Ll - Lf + 1;
+            const bool seg = lenR <= kCoopSeg && lenL <= kCoopSeg;  // block-uniform
+            if (seg) {
+                for (int q = t; q < lenR; q += kCoopRows) segR[q] = xs[Rf + q];
+                for (int q = t; q < lenL; q += kCoopRows) segL[q] = xs[Lf + q];
+            }
+            __syncthreads();
+            int R, L;
+            if (seg) {
+                // right: first index in [Rf, Rl] outside for this row (Rl is)
+                int lo = -1, hi = lenR - 1;  // lo: inside (virtual), hi: outside
+                while (hi - lo > 1) {
+                    const int q = (lo + hi) >> 1;
+                    if (inside<KERN>(segR[q] - w.xr, h)) lo = q; else hi = q;
+                }
+                R = Rf + hi;
+                // left: last index in [Lf, Ll] outside for this row (Lf is)
+                int llo = 0, lhi = lenL;  // llo: outside, lhi: inside (virtual)
+                while (lhi - llo > 1) {
+                    const int q = (llo + lhi) >> 1;
+                    if (!inside<KERN>(w.xr - segL[q], h)) llo = q; else lhi = q;
+                }
+                L = Lf + llo;
+                const int nkR = R - w.r, nkL = w.r - L;
+                gR = max(1, nkR - kR);
+                gL = max(1, nkL - kL);
+                kR = nkR;
+                kL = nkL;
+            } else {
+                const int kR0 = kR, kL0 = kL;
+                window_bounds<KERN>(xs, n, w.r, w.xr, h, kR, kL, gR, gL);
+                gR = max(1, kR - kR0);
+                gL = max(1, kL - kL0);
+                R = w.r + kR;
+                L = w.r - kL;
+            }
+            const int c = R - L - 2;
+            const bool M = valid && c > 0;  // reading Q6
+            double e2 = M ? window_e2<KERN>(w, L + 1, R, c, h, xy, P, ps, ymax) : 0.0;
+            e2 = warp_sum(e2);
+            const unsigned ball = __ballot_sync(0xffffffffu, M);
+            const int tile = ct * 4 + wp;  // 32-row tile of the partial layout
+            if (lane == 0 && tile < ntiles) {
+                tileS[(size_t)b * ntiles + tile] = e2;
+                tileN[(size_t)b * ntiles + tile] = (uint8_t)__popc(ball);
+            }
+            __syncthreads();  // segments consumed before the next bandwidth's
+        }
+    }
+}
+
 }  // namespace krcv
