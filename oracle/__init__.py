@@ -59,6 +59,8 @@ def _lib(precision: str = "ld") -> ctypes.CDLL:
     lib.kro_default_grid.restype = ctypes.c_int
     lib.kro_finalize.argtypes = [P, i64, i32, P, P]
     lib.kro_finalize.restype = ctypes.c_int
+    lib.kro_kde_lscv.argtypes = [P, i64, P, i32, i32, P, i64, P, P, P, P]
+    lib.kro_kde_lscv.restype = ctypes.c_int
     lib.kro_real_bits.restype = ctypes.c_int
     lib.kro_num_threads.restype = ctypes.c_int
     _libs[precision] = lib
@@ -200,3 +202,24 @@ def cv_refine(x, y, h, kernel: int, levels: int, m_fine: int, evaluate=None):
         if level + 1 < levels:
             grid = refine_grid(grid, r.best, m_fine)
     return np.array(hb), np.array(cb), grids
+
+
+def kde_lscv(x, h, kernel: int, rows=None, precision: str = "ld") -> Result:
+    """KDE least-squares cross-validation by the plain definition (PAPER.md
+    P@10382-10640; reading Q24): lscv[m] (full rows only), the per-bandwidth
+    row sums A (sum of Kbar over pairs, Kbar = K*K) and B (sum of K over
+    pairs) over `rows` (default: all), best index."""
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    h = np.ascontiguousarray(h, dtype=np.float64)
+    n, m = x.shape[0], h.shape[0]
+    r = None if rows is None else np.ascontiguousarray(rows, dtype=np.int64)
+    A = np.empty(m)
+    B = np.empty(m)
+    lscv = np.full(m, np.nan)
+    best = ctypes.c_int32(-1)
+    st = _lib(precision).kro_kde_lscv(x.ctypes.data, n, h.ctypes.data, m, int(kernel), _ptr(r),
+                                      0 if r is None else r.shape[0], A.ctypes.data, B.ctypes.data,
+                                      lscv.ctypes.data, ctypes.byref(best))
+    if st:
+        raise OracleError(st)
+    return Result(lscv=lscv, A=A, B=B, best=int(best.value))

@@ -397,3 +397,95 @@ int kro_num_threads(void)
     return 1;
 #endif
 }
+
+/* ------------------------------------------------------------------ */
+/* KDE least-squares cross-validation (PAPER.md P@10382-10640: "the     */
+/* methods developed here for least-squares cross-validation can be     */
+/* applied to ... optimal bandwidth selection for kernel density        */
+/* estimation"; reading Q24).                   */
+/*                                                                      */
+/*   f_h(x)        = (1/(n h)) sum_j K((x - x_j)/h)                     */
+/*   f_{h,-i}(x_i) = (1/((n-1) h)) sum_{j!=i} K((x_i - x_j)/h)          */
+/*   LSCV(h)       = int f_h^2 - (2/n) sum_i f_{h,-i}(x_i)               */
+/*   int f_h^2     = (1/(n^2 h)) sum_i sum_j Kbar((x_i - x_j)/h),        */
+/*   Kbar = K * K (self-convolution), written out below.                */
+/* Kernels normalised to integrate to 1 (Q24): uniform 1/2 I{|u|<=1},   */
+/* Epanechnikov 3/4 (1-u^2) I{|u|<=1}, triangular (1-|u|) I{|u|<1}.     */
+/* Window membership as Q1: K's window d <= h (uniform) / d < h, Kbar's */
+/* d < 2h (Kbar vanishes continuously at |u| = 2 for all three).        */
+/* The plain definition, O(n^2 m); per row i: A_i = sum_{j!=i} Kbar,    */
+/* B_i = sum_{j!=i} K; LSCV = (n Kbar(0) + sum A)/(n^2 h)               */
+/*                           - 2 sum B / (n (n-1) h).                   */
+/* ------------------------------------------------------------------ */
+static real kde_kbar(real v, int32_t kernel) /* v = |u| in [0, 2) */
+{
+    switch (kernel) {
+    case KRO_EPANECHNIKOV: /* (3/160) (2-v)^3 (v^2 + 6 v + 4) */
+        return (real)3 / (real)160 * (2 - v) * (2 - v) * (2 - v) * (v * v + 6 * v + 4);
+    case KRO_TRIANGULAR:   /* cubic B-spline */
+        if (v < 1) return (real)2 / (real)3 - v * v + v * v * v / 2;
+        return (2 - v) * (2 - v) * (2 - v) / 6;
+    default:               /* uniform: triangle */
+        return (2 - v) / 4;
+    }
+}
+
+static real kde_k(real v, int32_t kernel) /* v = |u| inside K's window */
+{
+    switch (kernel) {
+    case KRO_EPANECHNIKOV: return (real)0.75 * (1 - v * v);
+    case KRO_TRIANGULAR:   return 1 - v;
+    default:               return (real)0.5;
+    }
+}
+
+int kro_kde_lscv(const double *x, int64_t n, const double *h, int32_t m, int32_t kernel,
+                 const int64_t *rows, int64_t nrows, double *A_out, double *B_out,
+                 double *lscv_out, int32_t *best_out)
+{
+    if (!x || !h || n < 2 || m < 1 || m > KRO_MAX_M) return KRO_EARG;
+    if (kernel != KRO_UNIFORM && kernel != KRO_EPANECHNIKOV && kernel != KRO_TRIANGULAR) return KRO_EKERNEL;
+    for (int32_t b = 0; b < m; b++) {
+        if (!isfinite(h[b]) || !(h[b] > 0.0)) return KRO_EGRID;
+        if (b > 0 && h[b] < h[b - 1]) return KRO_EGRID;
+    }
+    for (int64_t i = 0; i < n; i++)
+        if (!isfinite(x[i])) return KRO_ENONFINITE;
+    int64_t R = rows ? nrows : n;
+    if (R < 0) return KRO_EARG;
+    real *A = (real *)calloc((size_t)m, sizeof(real));
+    real *B = (real *)calloc((size_t)m, sizeof(real));
+    if (!A || !B) { free(A); free(B); return KRO_ENOMEM; }
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int32_t b = 0; b < m; b++) {
+        const double hb = h[b], h2 = 2.0 * hb; /* 2h exact in binary64 */
+        real Ab = 0, Bb = 0;
+        for (int64_t r = 0; r < R; r++) {
+            int64_t i = rows ? rows[r] : r;
+            for (int64_t l = 0; l < n; l++) {
+                if (l == i) continue;
+                double d = fabs(x[l] - x[i]);
+                real v = (real)d / (real)hb;
+                if (d < h2) Ab += kde_kbar(v, kernel);
+                if (in_window(d, hb, kernel)) Bb += kde_k(v, kernel);
+            }
+        }
+        A[b] = Ab;
+        B[b] = Bb;
+    }
+    int32_t best = -1;
+    real bestv = 0;
+    for (int32_t b = 0; b < m; b++) {
+        if (A_out) A_out[b] = (double)A[b];
+        if (B_out) B_out[b] = (double)B[b];
+        if (!rows) {
+            real nn = (real)n, hb = (real)h[b];
+            real v = (nn * kde_kbar(0, kernel) + A[b]) / (nn * nn * hb) - 2 * B[b] / (nn * (nn - 1) * hb);
+            if (lscv_out) lscv_out[b] = (double)v;
+            if (!isnan((double)v) && (best < 0 || (double)v < (double)bestv)) { best = b; bestv = v; }
+        }
+    }
+    if (best_out) *best_out = best < 0 ? 0 : best;
+    free(A); free(B);
+    return KRO_OK;
+}

@@ -407,3 +407,70 @@ def test_PG_scaling_invariance_and_sorted_rejects():
     assert np.array_equal(a, b)
     with pytest.raises(oracle.OracleError):
         oracle.cv_sorted(x, y, h, G)
+
+
+# ---------------------------------------------------------------- KDE LSCV (Q24, P@10382-10640)
+def _K_norm(u, k):
+    """Normalised kernels (integrate to 1), Q24."""
+    a = abs(u)
+    if k == E:
+        return 0.75 * (1 - u * u) if a <= 1 else 0.0
+    if k == T:
+        return 1 - a if a < 1 else 0.0
+    return 0.5 if a <= 1 else 0.0
+
+
+@pytest.mark.parametrize("k", KERNELS)
+@pytest.mark.parametrize("v", [0.0, 0.3, 0.999, 1.0, 1.25, 1.7, 1.99])
+def test_KDE_Kbar_is_the_self_convolution(k, v):
+    """n = 2 isolates Kbar: LSCV = (Kbar(0) + Kbar(v))/(2h) - 2 K(v)/h, so the
+    oracle's Kbar(v) must equal the numerical convolution int K(t) K(v-t) dt
+    (scipy quad with the kernels' breakpoints) -- an independent pin of the
+    closed forms."""
+    from scipy.integrate import quad
+    h = 0.5
+    x = np.array([0.0, v * h])
+    r = oracle.kde_lscv(x, np.array([h]), k)
+    kb0 = quad(lambda t: _K_norm(t, k) ** 2, -1, 1, points=[0.0])[0]
+    kbar_v = 2 * h * r.lscv[0] + 4 * _K_norm(v, k) - kb0
+    conv = quad(lambda t: _K_norm(t, k) * _K_norm(v - t, k), -1, 1, points=sorted({0.0, v - 1, v, min(v, 1.0)}))[0]
+    assert abs(kbar_v - conv) <= 1e-12
+
+
+@pytest.mark.parametrize("k", KERNELS)
+def test_KDE_integral_term_by_quadrature(k):
+    """int f_h^2 computed by numerical integration of the density estimate
+    equals the pairwise form (n Kbar(0) + sum A)/(n^2 h); the leave-one-out
+    term equals a brute-force double loop."""
+    from scipy.integrate import quad
+    rng = np.random.default_rng(31)
+    x = np.sort(rng.uniform(0, 1, 9))
+    n, h = x.shape[0], 0.17
+    r = oracle.kde_lscv(x, np.array([h]), k)
+
+    def f(t):
+        return sum(_K_norm((t - xi) / h, k) for xi in x) / (n * h)
+
+    pts = sorted(set(np.concatenate([x - h, x, x + h]).tolist()))
+    integral = 0.0
+    for a, b in zip(pts[:-1], pts[1:]):
+        integral += quad(lambda t: f(t) ** 2, a, b)[0]
+    kb0 = quad(lambda t: _K_norm(t, k) ** 2, -1, 1, points=[0.0])[0]
+    assert abs((n * kb0 + r.A[0]) / (n * n * h) - integral) <= 1e-10 * integral
+    loo = sum(_K_norm((x[i] - x[j]) / h, k) for i in range(n) for j in range(n) if j != i)
+    assert abs(r.B[0] - loo) <= 1e-13 * loo
+    assert abs(r.lscv[0] - (integral - 2.0 / n * loo / ((n - 1) * h))) <= 1e-10 * abs(r.lscv[0])
+
+
+def test_KDE_invariances_and_rows():
+    """LSCV(h) scales as 1/s under (x, h) -> (s x, s h) with s = 2^k (exact);
+    row subsets add up to the full sums."""
+    x, _ = workloads.draw_xy("paper", 300, 5)
+    h = np.array([0.01, 0.05, 0.2, 1.5])
+    for k in KERNELS:
+        a = oracle.kde_lscv(x, h, k)
+        b = oracle.kde_lscv(x * 4.0, h * 4.0, k)
+        assert np.array_equal(a.lscv / 4.0, b.lscv) and a.best == b.best
+        p1 = oracle.kde_lscv(x, h, k, rows=np.arange(0, 150))
+        p2 = oracle.kde_lscv(x, h, k, rows=np.arange(150, 300))
+        assert cv_rel_err(p1.A + p2.A, a.A) <= 1e-14 and cv_rel_err(p1.B + p2.B, a.B) <= 1e-14
