@@ -66,6 +66,8 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-alt", action="store_true", help="skip timing the other algorithm (alt_algo)")
+    ap.add_argument("--kde", action="store_true",
+                    help="time the KDE least-squares CV (kr_kde_lscv_async, SURVEY §8(f) rank 3) on the config's x")
     ap.add_argument("--kernel", default=None, choices=["uniform", "epanechnikov", "triangular", "gaussian"],
                     help="override the config's kernel (e.g. the Gaussian dense path on C2's data)")
     ap.add_argument("--algo", default="auto", choices=["auto", "sweep", "prefix"],
@@ -429,8 +431,68 @@ def e2e_measure(args, x, y, h, k, n, m, units, dev, rank, world, plan):
             "timing": "host wall clock around the synchronous call"}
 
 
+def run_kde(args):
+    """KDE LSCV (reading Q24) on the config's x: device-timed whole searches,
+    pair-bandwidth evaluations n (n-1) m per second; one JSON line."""
+    import torch
+
+    from paper_conf_ipps_rohlfsz17_b200 import krcv
+
+    torch.cuda.set_device(0)
+    dev = torch.device("cuda", 0)
+    cfg = workloads.CONFIGS[args.config]
+    x, _, h, k = workloads.make(cfg, seed=args.seed)
+    if args.kernel:
+        k = workloads.KERNEL_IDS[args.kernel]
+    n, m = x.shape[0], h.shape[0]
+    d_x = torch.as_tensor(x, device=dev)
+    d_h = torch.as_tensor(h, device=dev)
+    ws = krcv.aligned(krcv.workspace(n, m, dev))
+    out = torch.empty(m, dtype=torch.float64, device=dev)
+    bs = torch.empty(2, dtype=torch.int32, device=dev)
+    stream = torch.cuda.current_stream(dev)
+    lib = krcv._lib()
+
+    def run():
+        st = lib.kr_kde_lscv_async(d_x.data_ptr(), n, d_h.data_ptr(), m, k, out.data_ptr(), bs.data_ptr(),
+                                   ws.data_ptr(), ws.numel(), __import__("ctypes").c_void_p(stream.cuda_stream))
+        if st:
+            raise krcv.KrcvError(st, "kr_kde_lscv_async")
+
+    for _ in range(args.warmup):
+        run()
+    torch.cuda.synchronize()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    krcv.kr_profile_enable(True)
+    tot, win = 0.0, 0.0
+    with ClockSampler(0) as clk:
+        for s_ in range(args.steps):
+            flush.fill_(s_ & 0xFF)
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            run()
+            b.record(stream)
+            stg = krcv.kr_profile_read()
+            win += stg[2]
+            tot += a.elapsed_time(b)
+    krcv.kr_profile_enable(False)
+    best = int(bs[0])
+    units = n * (n - 1) * m
+    print(json.dumps({
+        "metric": "KDE LSCV pair-bandwidth evals/s (SURVEY 8(f) rank 3)", "value": units * args.steps / (tot * 1e-3),
+        "unit": UNIT, "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot / args.steps,
+        "higher_is_better": True, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{cfg.name} x, kde lscv, {workloads.KERNEL_NAMES[k]}", "n": n, "m": m},
+        "kde_window_kernel_ms": win / args.steps, "result": {"best": best, "h_best": float(h[best]),
+                                                              "lscv_best": float(out[best])},
+        "clocks": clk.summary()}), flush=True)
+    return 0
+
+
 def main():
     args = parse()
+    if args.kde:
+        return run_kde(args)
     if args.algo != "auto":
         os.environ["KRCV_ALGO"] = args.algo
     if args.impl == "reference":

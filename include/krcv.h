@@ -144,6 +144,35 @@ int kr_cv_refine(const double *x, const double *y, int64_t n,
                  int32_t levels, int32_t m_fine,
                  double *h_best_out, double *cv_best_out);
 
+/*
+ * KDE least-squares cross-validation (P@10382-10640: the LSCV machinery
+ * "can be applied to ... optimal bandwidth selection for kernel density
+ * estimation"; reading Q24).  Kernels normalised to integrate
+ * to 1 (uniform, Epanechnikov, triangular; KR_EKERNEL otherwise):
+ *   LSCV(h) = int f_h^2 - (2/n) sum_i f_{h,-i}(x_i)
+ *           = (n Kbar(0) + sum_i A_i) / (n^2 h) - 2 sum_i B_i / (n (n-1) h),
+ *   A_i = sum_{j!=i} Kbar((x_i-x_j)/h) (Kbar = K * K), B_i = sum_{j!=i} K(.)
+ * kr_kde_lscv: host pointers, synchronous; lscv_out [m], best_out = smallest
+ * arg-min (LSCV may be negative).  Errors: KR_EARG, KR_EKERNEL, KR_EGRID,
+ * KR_ENONFINITE, KR_ENOMEM, KR_ECUDA.
+ * kr_kde_lscv_async: the same on device pointers, enqueued (workspace from
+ * kr_workspace_bytes(n, m)); d_best_status [2] = { best, status }.
+ * kr_kde_shard_async: rows [floor(shard n/P), floor((shard+1) n/P)) of the
+ * sorted order -> d_partial [KR_PARTIAL_LEN(m)] = [ sum A | sum B | status ],
+ * additive across shards; kr_kde_finalize turns the summed partial into LSCV
+ * and best on the host (h_grid host pointer).
+ */
+int kr_kde_lscv(const double *x, int64_t n, const double *h_grid, int32_t m, int32_t kernel,
+                double *lscv_out, int32_t *best_out);
+int kr_kde_lscv_async(const double *d_x, int64_t n, const double *d_h, int32_t m, int32_t kernel,
+                      double *d_lscv, int32_t *d_best_status,
+                      void *d_workspace, size_t workspace_bytes, void *cuda_stream);
+int kr_kde_shard_async(const double *d_x, int64_t n, const double *d_h, int32_t m, int32_t kernel,
+                       int32_t shard, int32_t nshards, double *d_partial,
+                       void *d_workspace, size_t workspace_bytes, void *cuda_stream);
+int kr_kde_finalize(const double *partial, int64_t n, const double *h_grid, int32_t m, int32_t kernel,
+                    double *lscv_out, int32_t *best_out);
+
 /* Host-side grid check (finite, > 0, non-decreasing, 1 <= m <= KR_MAX_M). */
 int kr_validate_grid(const double *h_grid, int32_t m);
 

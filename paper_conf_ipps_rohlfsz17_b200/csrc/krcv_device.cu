@@ -27,6 +27,7 @@
 #include "krcv_sort.cuh"
 #include "krcv_prefix.cuh"
 #include "krcv_dense.cuh"
+#include "krcv_kde.cuh"
 
 namespace krcv {
 
@@ -242,6 +243,7 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     // arrays and prefix moments in place (kr_cv_refine)
     L->tileS = off;    off = align256(off + sizeof(double) * (size_t)ntiles * (size_t)m);
     L->tileN = off;    off = align256(off + sizeof(uint8_t) * (size_t)ntiles * (size_t)m);
+    L->tileB = off;    off = align256(off + sizeof(double) * (size_t)((n + 31) / 32) * (size_t)m);  // KDE sum B
     L->partial = off;  off = align256(off + sizeof(double) * (size_t)KR_PARTIAL_LEN(m));
     L->cub_bytes = cub_bytes;
     L->total = off;
@@ -546,6 +548,51 @@ extern "C" size_t kr_workspace_bytes(int64_t n, int32_t m)
 
 // The whole device pipeline of one shard: a1 .. a5, and with fin.cv set the
 // fused finalize (single-GPU whole search).
+// a1 + a2: validation counters, stable sort of (x, y) by x into the sorted
+// AoS array with +-inf sentinels; resets the tile counter.
+static int enqueue_sort(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m,
+                        const WsLayout &L, char *ws, cudaStream_t st, int64_t *launches_out)
+{
+    uint64_t *keys_in = reinterpret_cast<uint64_t *>(ws + L.keys_in);
+    uint64_t *keys_out = reinterpret_cast<uint64_t *>(ws + L.keys_out);
+    uint32_t *vals_in = reinterpret_cast<uint32_t *>(ws + L.vals_in);
+    uint32_t *vals_out = reinterpret_cast<uint32_t *>(ws + L.vals_out);
+    double2 *xy = reinterpret_cast<double2 *>(ws + L.xy) + kPad;
+    int *counter = reinterpret_cast<int *>(ws + L.counter);
+    unsigned *status = reinterpret_cast<unsigned *>(ws + L.status);
+    const int nn = (int)n;
+    int64_t launches = 0;
+    cudaError_t e;
+    if (n <= kRankSortMaxN && !getenv_flag("KRCV_CUB_SORT")) {
+        // a1 + a2: chunk merge sort, rank by counting across chunk pairs, scatter (krcv_sort.cuh)
+        const int cfg = chunk_config(n);
+        const int chunk = cfg == 0 ? 1024 : (cfg == 1 ? 2048 : (cfg == 2 ? 4096 : 512));
+        const int nchunks = (int)((n + chunk - 1) / chunk);
+        uint32_t *khi = reinterpret_cast<uint32_t *>(keys_out);          // keys_out is free on this path
+        int *rank = reinterpret_cast<int *>(vals_out);                    // so is vals_out
+        switch (cfg) {
+        case 0: launch_rank_sort<256, 4>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
+        case 1: launch_rank_sort<256, 8>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
+        case 2: launch_rank_sort<512, 8>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
+        default: launch_rank_sort<256, 2>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
+        }
+        const int npad = nchunks * chunk;
+        rank_scatter_kernel<<<(npad + 255) / 256, 256, 0, st>>>(vals_in, rank, nn, npad, d_x, d_y, xy, counter);
+        launches += nchunks > 1 ? 1 : 0;
+        launches += 2;
+    } else {
+        pack_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, nn, d_h, m, keys_in, vals_in, status);
+        size_t cub_bytes = L.cub_bytes;
+        e = cub::DeviceRadixSort::SortPairs(ws + L.cub, cub_bytes, keys_in, keys_out, vals_in, vals_out,
+                                            nn, 0, 64, st);
+        if (e != cudaSuccess) { set_cuda_error("cub::DeviceRadixSort::SortPairs", (int)e); return KR_ECUDA; }
+        gather_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, vals_out, nn, xy, counter);
+        launches += 2 + cub_sort_launches(n);
+    }
+    *launches_out += launches;
+    return KR_OK;
+}
+
 // reuse_sorted: the workspace already holds this (x, y)'s sorted arrays (and,
 // for the window-prefix path, its prefix moments for this kernel) from the
 // previous call on it -- only the bandwidth-dependent stages run (the
@@ -608,31 +655,9 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     if (reuse_sorted) {
         e = cudaMemsetAsync(counter, 0, sizeof(int), st);
         if (e != cudaSuccess) { set_cuda_error("cudaMemsetAsync(counter)", (int)e); return KR_ECUDA; }
-    } else if (n <= kRankSortMaxN && !getenv_flag("KRCV_CUB_SORT")) {
-        // a1 + a2: chunk merge sort, rank by counting across chunk pairs, scatter (krcv_sort.cuh)
-        const int cfg = chunk_config(n);
-        const int chunk = cfg == 0 ? 1024 : (cfg == 1 ? 2048 : (cfg == 2 ? 4096 : 512));
-        const int nchunks = (int)((n + chunk - 1) / chunk);
-        uint32_t *khi = reinterpret_cast<uint32_t *>(keys_out);          // keys_out is free on this path
-        int *rank = reinterpret_cast<int *>(vals_out);                    // so is vals_out
-        switch (cfg) {
-        case 0: launch_rank_sort<256, 4>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
-        case 1: launch_rank_sort<256, 8>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
-        case 2: launch_rank_sort<512, 8>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
-        default: launch_rank_sort<256, 2>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
-        }
-        const int npad = nchunks * chunk;
-        rank_scatter_kernel<<<(npad + 255) / 256, 256, 0, st>>>(vals_in, rank, nn, npad, d_x, d_y, xy, counter);
-        launches += nchunks > 1 ? 1 : 0;
-        launches += 2;
     } else {
-        pack_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, nn, d_h, m, keys_in, vals_in, status);
-        size_t cub_bytes = L.cub_bytes;
-        e = cub::DeviceRadixSort::SortPairs(ws + L.cub, cub_bytes, keys_in, keys_out, vals_in, vals_out,
-                                            nn, 0, 64, st);
-        if (e != cudaSuccess) { set_cuda_error("cub::DeviceRadixSort::SortPairs", (int)e); return KR_ECUDA; }
-        gather_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, vals_out, nn, xy, counter);
-        launches += 2 + cub_sort_launches(n);
+        const int st2 = enqueue_sort(d_x, d_y, n, d_h, m, L, ws, st, &launches);
+        if (st2) return st2;
     }
     prof_mark(1, st);
     if (prefix && !reuse_sorted) {
@@ -744,4 +769,117 @@ extern "C" int kr_finalize_async(const double *d_partial, int64_t n, int32_t m, 
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) { set_cuda_error("finalize_kernel launch", (int)e); return KR_ECUDA; }
     return KR_OK;
+}
+
+// ---------------------------------------------------------------------------
+// KDE least-squares cross-validation (krcv_kde.cuh; reading Q24)
+// ---------------------------------------------------------------------------
+static int enqueue_kde(const double *d_x, int64_t n, const double *d_h, int32_t m, int32_t kernel, int32_t shard,
+                       int32_t nshards, double *d_partial, KdeFin fin, void *d_workspace, size_t workspace_bytes,
+                       void *cuda_stream)
+{
+    if (!d_x || !d_h || !d_workspace) return KR_EARG;
+    if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return KR_EARG;
+    if (kernel != KR_UNIFORM && kernel != KR_EPANECHNIKOV && kernel != KR_TRIANGULAR) return KR_EKERNEL;
+    if (nshards < 1 || shard < 0 || shard >= nshards) return KR_EARG;
+    if ((reinterpret_cast<uintptr_t>(d_workspace) & 255u) != 0) return KR_EARG;
+    WsLayout L;
+    if (!ws_layout(n, m, &L)) return KR_ECUDA;
+    if (workspace_bytes < L.total) return KR_EARG;
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    char *ws = static_cast<char *>(d_workspace);
+    double2 *xy = reinterpret_cast<double2 *>(ws + L.xy) + kPad;
+    int *counter = reinterpret_cast<int *>(ws + L.counter);
+    unsigned *status = reinterpret_cast<unsigned *>(ws + L.status);
+    double *tileA = reinterpret_cast<double *>(ws + L.tileS);
+    double *tileB = reinterpret_cast<double *>(ws + L.tileB);
+    if (!d_partial) d_partial = reinterpret_cast<double *>(ws + L.partial);
+    fin.done = status + 2;
+    const int nn = (int)n;
+    const int lo = (int)(((int64_t)shard * n) / nshards);
+    const int hi = (int)(((int64_t)(shard + 1) * n) / nshards);
+    const int ntiles = (hi - lo + 31) / 32;
+    int64_t launches = 0;
+    prof_mark(0, st);
+    cudaError_t e = cudaMemsetAsync(status, 0, 8 * sizeof(unsigned), st);
+    if (e != cudaSuccess) { set_cuda_error("cudaMemsetAsync(status)", (int)e); return KR_ECUDA; }
+    // the sort carries (x, y); the density estimate has no y: x rides along
+    const int st2 = enqueue_sort(d_x, d_x, n, d_h, m, L, ws, st, &launches);
+    if (st2) return st2;
+    prof_mark(1, st);
+    launch_prefix_build<kKdeMoments>(xy, nn, L, ws, st);
+    launches += 2;
+    prof_mark(2, st);
+    if (ntiles > 0) {
+        static int resident = 0, sms = 0;
+        if (!resident) {
+            int b = 0;
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kde_window_kernel<KR_EPANECHNIKOV>, kWinThreads, 0);
+            resident = b > 0 ? b : 1;
+            int dev = 0;
+            cudaGetDevice(&dev);
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+            if (sms <= 0) sms = 148;
+        }
+        int nbc = (int)(((int64_t)sms * kWinTasksPerSM + ntiles - 1) / ntiles);
+        const int max_nbc = (m + kWinMinBper - 1) / kWinMinBper;
+        nbc = nbc > max_nbc ? max_nbc : nbc;
+        nbc = nbc < 1 ? 1 : nbc;
+        int blocks = (int)(((int64_t)ntiles * nbc + kWinWarps - 1) / kWinWarps);
+        if (blocks > sms * resident) blocks = sms * resident;
+        const double *xs = reinterpret_cast<const double *>(ws + L.xs) + kPad;
+        const double *P = reinterpret_cast<const double *>(ws + L.pfx);
+        switch (kernel) {
+        case KR_UNIFORM:
+            kde_window_kernel<KR_UNIFORM><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, d_h, m, nn, lo, hi,
+                                                                          ntiles, nbc, tileA, tileB, counter);
+            break;
+        case KR_EPANECHNIKOV:
+            kde_window_kernel<KR_EPANECHNIKOV><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, d_h, m, nn,
+                                                                               lo, hi, ntiles, nbc, tileA, tileB,
+                                                                               counter);
+            break;
+        default:
+            kde_window_kernel<KR_TRIANGULAR><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, d_h, m, nn, lo,
+                                                                             hi, ntiles, nbc, tileA, tileB, counter);
+            break;
+        }
+        launches += 1;
+    }
+    prof_mark(3, st);
+    kde_reduce_kernel<<<m < 148 * 8 ? m : 148 * 8, kKdeRedThreads, 0, st>>>(tileA, tileB, ntiles, m, status,
+                                                                             d_partial, fin);
+    launches += 1;
+    prof_mark(4, st);
+    g_prof.recorded = g_prof.on;
+    g_prof.launches = launches;
+    g_prof.algo = KR_ALGO_PREFIX;
+    e = cudaGetLastError();
+    if (e != cudaSuccess) { set_cuda_error("kernel launch", (int)e); return KR_ECUDA; }
+    return KR_OK;
+}
+
+extern "C" int kr_kde_lscv_async(const double *d_x, int64_t n, const double *d_h, int32_t m, int32_t kernel,
+                                 double *d_lscv, int32_t *d_best_status, void *d_workspace, size_t workspace_bytes,
+                                 void *cuda_stream)
+{
+    if (!d_lscv || !d_best_status) return KR_EARG;
+    KdeFin fin{};
+    fin.n = (long long)n;
+    fin.kernel = kernel;
+    fin.h = d_h;
+    fin.lscv = d_lscv;
+    fin.best = d_best_status;
+    fin.status = d_best_status + 1;
+    return enqueue_kde(d_x, n, d_h, m, kernel, 0, 1, nullptr, fin, d_workspace, workspace_bytes, cuda_stream);
+}
+
+extern "C" int kr_kde_shard_async(const double *d_x, int64_t n, const double *d_h, int32_t m, int32_t kernel,
+                                  int32_t shard, int32_t nshards, double *d_partial, void *d_workspace,
+                                  size_t workspace_bytes, void *cuda_stream)
+{
+    if (!d_partial) return KR_EARG;
+    KdeFin fin{};
+    return enqueue_kde(d_x, n, d_h, m, kernel, shard, nshards, d_partial, fin, d_workspace, workspace_bytes,
+                       cuda_stream);
 }

@@ -246,6 +246,62 @@ extern "C" int kr_cv_refine(const double *x, const double *y, int64_t n, const d
     return KR_OK;
 }
 
+extern "C" int kr_kde_lscv(const double *x, int64_t n, const double *h_grid, int32_t m, int32_t kernel,
+                           double *lscv_out, int32_t *best_out)
+{
+    if (!x || !h_grid || !lscv_out || !best_out) return KR_EARG;
+    if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return KR_EARG;
+    if (kernel != KR_UNIFORM && kernel != KR_EPANECHNIKOV && kernel != KR_TRIANGULAR) return KR_EKERNEL;
+    int st = kr_validate_grid(h_grid, m);
+    if (st) return st;
+    for (int64_t i = 0; i < n; i++)
+        if (!std::isfinite(x[i])) return KR_ENONFINITE;
+    int dev = 0;
+    KR_CUDA_TRY(cudaGetDevice(&dev));
+    DevCtx *c = get_ctx(dev);
+    std::lock_guard<std::mutex> g(c->mu);
+    st = ensure_capacity(c, n, m);
+    if (st) return st;
+    cudaStream_t s = c->stream;
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dx, x, sizeof(double) * n, cudaMemcpyHostToDevice, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dh, h_grid, sizeof(double) * m, cudaMemcpyHostToDevice, s));
+    st = kr_kde_lscv_async(c->dx, n, c->dh, m, kernel, c->dcv, c->dbest, c->ws, c->ws_bytes, s);
+    if (st) return st;
+    std::vector<double> v(m);
+    int32_t bs[2] = {0, 0};
+    KR_CUDA_TRY(cudaMemcpyAsync(v.data(), c->dcv, sizeof(double) * m, cudaMemcpyDeviceToHost, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(bs, c->dbest, sizeof(int32_t) * 2, cudaMemcpyDeviceToHost, s));
+    KR_CUDA_TRY(cudaStreamSynchronize(s));
+    if (bs[1] != KR_OK) return bs[1];
+    std::memcpy(lscv_out, v.data(), sizeof(double) * m);
+    *best_out = bs[0];
+    return KR_OK;
+}
+
+extern "C" int kr_kde_finalize(const double *partial, int64_t n, const double *h_grid, int32_t m, int32_t kernel,
+                               double *lscv_out, int32_t *best_out)
+{
+    if (!partial || !h_grid || !lscv_out || !best_out || n < 2 || m < 1 || m > KR_MAX_M) return KR_EARG;
+    if (kernel != KR_UNIFORM && kernel != KR_EPANECHNIKOV && kernel != KR_TRIANGULAR) return KR_EKERNEL;
+    if (partial[2 * (int64_t)m] != 0.0) return KR_EGRID;
+    if (partial[2 * (int64_t)m + 1] != 0.0) return KR_ENONFINITE;
+    const double nn = (double)n;
+    const double kb0 = kernel == KR_UNIFORM ? 0.5 : (kernel == KR_EPANECHNIKOV ? 0.6 : 2.0 / 3.0);
+    int32_t best = -1;
+    double bv = 0.0;
+    for (int32_t b = 0; b < m; b++) {
+        const double v = (nn * kb0 + partial[b]) / (nn * nn * h_grid[b]) -
+                         2.0 * partial[m + b] / (nn * (nn - 1.0) * h_grid[b]);
+        lscv_out[b] = v;
+        if (!std::isnan(v) && (best < 0 || v < bv)) {
+            bv = v;
+            best = b;
+        }
+    }
+    *best_out = best < 0 ? 0 : best;
+    return KR_OK;
+}
+
 extern "C" int kr_finalize(const double *partial, int64_t n, int32_t m, double *cv_out, int64_t *neff_out,
                            int32_t *best_out)
 {

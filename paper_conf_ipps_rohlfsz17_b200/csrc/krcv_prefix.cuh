@@ -60,6 +60,9 @@ constexpr int kWinMinBper = 8;        // >= this many bandwidths per task
 
 // Moments per kernel (slot order).  Epanechnikov: y, u, u^2, y u, y u^2.
 // Triangular: y, u, y u.  Uniform: y.
+// Pseudo-kernel id of the KDE moment set (krcv_kde.cuh): u, u^2, ..., u^5.
+constexpr int kKdeMoments = 100;
+
 template <int KERN>
 struct NMom {
     static constexpr int v = KERN == KR_UNIFORM ? 1 : (KERN == KR_TRIANGULAR ? 3 : 5);
@@ -68,6 +71,15 @@ struct NMom {
 template <int KERN>
 __device__ __forceinline__ void moment_terms(double x, double y, double o, dd (&t)[kPfxMoments])
 {
+    if (KERN == kKdeMoments) {  // KDE: powers of u = x - o (y unused)
+        const dd u = two_sum(x, -o);
+        t[0] = u;
+        t[1] = dd_mul(u, u);
+        t[2] = dd_mul(t[1], u);
+        t[3] = dd_mul(t[1], t[1]);
+        t[4] = dd_mul(t[3], u);
+        return;
+    }
     t[0] = dd_make(y);
     if (KERN != KR_UNIFORM) {
         const dd u = two_sum(x, -o);  // exact: u.hi + u.lo == x - o

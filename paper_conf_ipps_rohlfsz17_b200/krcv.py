@@ -37,6 +37,7 @@ EXPORTS = (
     "kr_cv_shard_async", "kr_cv_shard_algo_async", "kr_cv_grid_async", "kr_finalize", "kr_finalize_async", "kr_default_grid",
     "kr_strerror", "kr_last_cuda_error", "kr_version",
     "kr_profile_enable", "kr_profile_read", "kr_launch_count", "kr_last_algo",
+    "kr_kde_lscv", "kr_kde_lscv_async", "kr_kde_shard_async", "kr_kde_finalize",
 )
 
 
@@ -92,6 +93,12 @@ def _lib() -> ctypes.CDLL:
     lib.kr_profile_read.argtypes = [P]
     lib.kr_profile_read.restype = ctypes.c_int
     lib.kr_launch_count.restype = ctypes.c_int64
+    lib.kr_kde_lscv.argtypes = [P, i64, P, i32, i32, P, P]
+    lib.kr_kde_lscv_async.argtypes = [P, i64, P, i32, i32, P, P, P, sz, P]
+    lib.kr_kde_shard_async.argtypes = [P, i64, P, i32, i32, i32, i32, P, P, sz, P]
+    lib.kr_kde_finalize.argtypes = [P, i64, P, i32, i32, P, P]
+    for f in ("kr_kde_lscv", "kr_kde_lscv_async", "kr_kde_shard_async", "kr_kde_finalize"):
+        getattr(lib, f).restype = ctypes.c_int
     lib.kr_last_algo.restype = ctypes.c_int32
     _LIB = lib
     return lib
@@ -298,3 +305,35 @@ def aligned(ws):
     """View of ws starting at a 256-byte boundary."""
     off = (-ws.data_ptr()) % 256
     return ws[off:]
+
+
+# ------------------------------------------------------------ KDE (LSCV, Q24)
+def kr_kde_lscv(x, h, kernel="epanechnikov"):
+    """KDE least-squares CV on the current CUDA device: (lscv[m], best)."""
+    x, h = _host(x), _host(h)
+    m = h.shape[0]
+    out = np.empty(m, np.float64)
+    best = ctypes.c_int32(-1)
+    _check(_lib().kr_kde_lscv(x.ctypes.data, x.shape[0], h.ctypes.data, m, _kernel_id(kernel), out.ctypes.data,
+                              ctypes.byref(best)), "kr_kde_lscv")
+    return out, int(best.value)
+
+
+def kr_kde_shard_async(d_x, d_h, kernel, shard: int, nshards: int, d_partial, d_ws, stream=None) -> None:
+    """Enqueue one row shard of the KDE LSCV -> partial [sum A | sum B | status]."""
+    import torch
+
+    s = torch.cuda.current_stream(d_x.device) if stream is None else stream
+    _check(_lib().kr_kde_shard_async(d_x.data_ptr(), d_x.numel(), d_h.data_ptr(), d_h.numel(), _kernel_id(kernel),
+                                     int(shard), int(nshards), d_partial.data_ptr(), d_ws.data_ptr(),
+                                     d_ws.numel() * d_ws.element_size(), ctypes.c_void_p(s.cuda_stream)),
+           "kr_kde_shard_async")
+
+
+def kr_kde_finalize(partial, n: int, h, kernel="epanechnikov"):
+    p, h = _host(partial), _host(h)
+    out = np.empty(h.shape[0], np.float64)
+    best = ctypes.c_int32(-1)
+    _check(_lib().kr_kde_finalize(p.ctypes.data, int(n), h.ctypes.data, h.shape[0], _kernel_id(kernel),
+                                  out.ctypes.data, ctypes.byref(best)), "kr_kde_finalize")
+    return out, int(best.value)

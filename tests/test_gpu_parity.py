@@ -366,3 +366,45 @@ def test_gaussian_wide_bandwidth_chunk():
     cv, neff, best = krcv.kr_cv_grid(x, y, h, GA, with_neff=True)
     ref = oracle.cv_direct(x, y, h, GA)
     assert cv_rel_err(cv, ref.cv) <= TIGHT and np.all(neff == 700)
+
+
+# ---------------------------------------------------------------- KDE LSCV (Q24)
+@pytest.mark.parametrize("k", [U, E, T])
+@pytest.mark.parametrize("dist,n", [("paper", 2), ("paper", 65), ("paper", 1000), ("sin_uniform", 777),
+                                    ("lognormal", 900)])
+def test_kde_lscv_parity(k, dist, n):
+    """kr_kde_lscv (window-prefix with u^1..u^5 dd prefix moments) vs the
+    oracle's plain-definition KDE LSCV in long double."""
+    x, _ = workloads.draw_xy(dist, n, 21)
+    m = 31
+    h = workloads.grid_log(x, m) if dist == "lognormal" else workloads.grid_default(x, m)
+    lscv, best = krcv.kr_kde_lscv(x, h, k)
+    ref = oracle.kde_lscv(x, h, k)
+    assert cv_rel_err(lscv, ref.lscv) <= TIGHT
+    assert best_ok(best, ref.lscv)
+
+
+@pytest.mark.parametrize("k", [U, E, T])
+def test_kde_full_size_sampled_shard(k):
+    """C2-size x (n = 20,000, 200 bandwidths): one sorted-order shard's sums
+    A and B against the oracle on exactly those rows; shards add up."""
+    import torch
+    x, _, h, _ = workloads.make("C2", seed=0)
+    m = h.shape[0]
+    d_x = torch.as_tensor(x, device="cuda")
+    d_h = torch.as_tensor(h, device="cuda")
+    ws = krcv.aligned(krcv.workspace(x.shape[0], m, "cuda"))
+    part = torch.empty(krcv.partial_len(m), dtype=torch.float64, device="cuda")
+    krcv.kr_kde_shard_async(d_x, d_h, k, 37, 64, part, ws)
+    torch.cuda.synchronize()
+    p = part.cpu().numpy()
+    ref = oracle.kde_lscv(x, h, k, rows=oracle.shard_rows(x, 37, 64))
+    assert cv_rel_err(p[:m], ref.A) <= TIGHT and cv_rel_err(p[m:2 * m], ref.B) <= TIGHT
+    tot = np.zeros(krcv.partial_len(m))
+    for r in range(4):
+        krcv.kr_kde_shard_async(d_x, d_h, k, r, 4, part, ws)
+        torch.cuda.synchronize()
+        tot += part.cpu().numpy()
+    lscv, best = krcv.kr_kde_finalize(tot, x.shape[0], h, k)
+    full, best_full = krcv.kr_kde_lscv(x, h, k)
+    assert cv_rel_err(lscv, full) <= 1e-12 and best_ok(best, full)
