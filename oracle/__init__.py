@@ -13,6 +13,11 @@ Contents
                      (P@13614-14984, P@20401-22459), long double.
 * ``exact.cv_exact``        -- Python ``fractions`` brute force of Eq.(1)-(3).
 * ``window.cv_window``      -- numpy long-double window-prefix checker (pin P10).
+* ``ll_cv``       -- C, local-linear LOO CV by its plain definition
+                     (weighted least-squares intercept, centred two-pass form;
+                     PAPER.md P@15728, reading Q25), O(n^2 m), long double.
+* ``exact.ll_cv_exact``     -- Python ``fractions`` brute force of the
+                               local-linear normal equations.
 * ``sorted_rows``           -- the x-sorted row order (stable by (x, index))
                                that defines shards.
 
@@ -61,6 +66,8 @@ def _lib(precision: str = "ld") -> ctypes.CDLL:
     lib.kro_finalize.restype = ctypes.c_int
     lib.kro_kde_lscv.argtypes = [P, i64, P, i32, i32, P, i64, P, P, P, P]
     lib.kro_kde_lscv.restype = ctypes.c_int
+    lib.kro_ll_cv.argtypes = [P, P, i64, P, i32, i32, P, i64, P, P, P, P]
+    lib.kro_ll_cv.restype = ctypes.c_int
     lib.kro_real_bits.restype = ctypes.c_int
     lib.kro_num_threads.restype = ctypes.c_int
     _libs[precision] = lib
@@ -223,3 +230,21 @@ def kde_lscv(x, h, kernel: int, rows=None, precision: str = "ld") -> Result:
     if st:
         raise OracleError(st)
     return Result(lscv=lscv, A=A, B=B, best=int(best.value))
+
+
+def ll_cv(x, y, h, kernel: int, rows=None, precision: str = "ld") -> Result:
+    """Local-linear LOO CV by the plain definition (reading Q25): for every
+    bandwidth and row, the intercept of the kernel-weighted least-squares line
+    through the in-window neighbours (row excluded); M_i = [>= 2 distinct x in
+    the window].  Returns cv, best, S (sum of M e^2 over `rows`), neff."""
+    x, y, h = _prep(x, y, h)
+    n, m = x.shape[0], h.shape[0]
+    r = None if rows is None else np.ascontiguousarray(rows, dtype=np.int64)
+    S = np.zeros(m); ne = np.zeros(m, np.int64); cv = np.zeros(m)
+    best = ctypes.c_int32(-1)
+    st = _lib(precision).kro_ll_cv(
+        _ptr(x), _ptr(y), n, _ptr(h), m, int(kernel), _ptr(r), 0 if r is None else r.shape[0],
+        _ptr(S), _ptr(ne), _ptr(cv), ctypes.byref(best))
+    if st:
+        raise OracleError(st)
+    return Result(cv=cv, best=int(best.value), S=S, neff=ne)

@@ -104,3 +104,43 @@ def cv_gauss_decimal(x, y, h, digits: int = 50):
             cvs.append(S / n)
         best = min(range(len(cvs)), key=lambda b: (cvs[b], b))
         return cvs, best
+
+
+def ll_cv_exact(x, y, h, kernel: int):
+    """Local-linear LOO CV in exact rationals (pin for ``oracle.ll_cv``,
+    reading Q25): per row and bandwidth, the 2x2 weighted normal equations
+        [S0 S1; S1 S2] [a; beta] = [T0; T1],  S_k = sum w d^k, T_k = sum w y d^k,
+    d = x_l - x_i, solved by Cramer's rule, a = (S2 T0 - S1 T1) / (S0 S2 - S1^2)
+    -- the uncentred form, deliberately not the oracle's centred one.  A row is
+    counted (M = 1) iff S0 S2 - S1^2 != 0.  Window membership as Q1 (binary64
+    test on |d|).  Returns (cv list, neff list, best)."""
+    xs = [float(v) for v in x]
+    ys = [Fraction(float(v)) for v in y]
+    n = len(xs)
+    cvs, neffs = [], []
+    for hb in (float(v) for v in h):
+        H = Fraction(hb)
+        tot, ne = Fraction(0), 0
+        for i in range(n):
+            S = [Fraction(0)] * 3
+            T = [Fraction(0)] * 2
+            for l in range(n):
+                if l == i:
+                    continue
+                d64 = abs(xs[l] - xs[i])
+                if not (d64 <= hb if kernel == UNIFORM else d64 < hb):
+                    continue
+                d = Fraction(xs[l]) - Fraction(xs[i])
+                w = _K(abs(d) / H, kernel)
+                S = [S[0] + w, S[1] + w * d, S[2] + w * d * d]
+                T = [T[0] + w * ys[l], T[1] + w * ys[l] * d]
+            det = S[0] * S[2] - S[1] * S[1]
+            if det == 0:
+                continue
+            a = (S[2] * T[0] - S[1] * T[1]) / det
+            tot += (ys[i] - a) ** 2
+            ne += 1
+        cvs.append(tot / n)
+        neffs.append(ne)
+    best = min(range(len(cvs)), key=lambda b: (cvs[b], b))
+    return cvs, neffs, best

@@ -489,3 +489,95 @@ int kro_kde_lscv(const double *x, int64_t n, const double *h, int32_t m, int32_t
     free(A); free(B);
     return KRO_OK;
 }
+
+/* ------------------------------------------------------------------ */
+/* Local-linear leave-one-out CV (PAPER.md      */
+/* §IV P@15728-15905: "The Nadaraya-Watson [19], [27] local constant    */
+/* estimator is used rather than a local linear regression" -- the      */
+/* local-linear estimator is the named alternative; reading Q25).       */
+/*                                                                      */
+/* For row i and bandwidth h the LOO local-linear estimate is the       */
+/* intercept a of the kernel-weighted least-squares line                */
+/*   min_{a,beta} sum_{l != i, l in W_i} w_il (Y_l - a - beta d_il)^2,  */
+/*   d_il = X_l - X_i (binary64), w_il = K(|d_il|/h) (Eq.(3), Q13),     */
+/* over the same window W_i as Eq.(2) (reading Q1).  The 2x2 normal     */
+/* equations are non-singular iff W_i holds at least two distinct X     */
+/* values (all weights are > 0 inside the window), so                   */
+/*   M_i = [W_i holds >= 2 distinct X]  (an integer test, as Q6),       */
+/* rows with M_i = 0 contribute 0 and CV divides by n (as Q7).          */
+/* The intercept is written in the centred (two-pass) form of the       */
+/* weighted least-squares solution, algebraically identical to          */
+/* (S2 T0 - S1 T1) / (S0 S2 - S1^2) with S_k = sum w d^k,               */
+/* T_k = sum w Y d^k:                                                   */
+/*   dbar = sum w d / sum w,  ybar = sum w Y / sum w,                   */
+/*   beta = sum w (d - dbar)(Y - ybar) / sum w (d - dbar)^2,            */
+/*   a    = ybar - beta dbar.                                           */
+/* The plain definition: O(n) per (row, bandwidth), no sort.            */
+/* ------------------------------------------------------------------ */
+static int ll_row(const double *x, const double *y, int64_t n, double hb, int32_t kernel, int64_t i, real *e2)
+{
+    real s0 = 0, sd = 0, sy = 0;
+    int64_t first = -1, distinct = 0;
+    for (int64_t l = 0; l < n; l++) {
+        if (l == i) continue;
+        double d = x[l] - x[i];
+        if (!in_window(fabs(d), hb, kernel)) continue;
+        real w = kernel_K(fabs(d), hb, kernel);
+        s0 += w;
+        sd += w * (real)d;
+        sy += w * (real)y[l];
+        if (first < 0) first = l;
+        else if (x[l] != x[first]) distinct = 1;
+    }
+    if (!distinct) return 0; /* M_i = 0 */
+    real dbar = sd / s0, ybar = sy / s0, sdd = 0, sdy = 0;
+    for (int64_t l = 0; l < n; l++) {
+        if (l == i) continue;
+        double d = x[l] - x[i];
+        if (!in_window(fabs(d), hb, kernel)) continue;
+        real w = kernel_K(fabs(d), hb, kernel);
+        real dc = (real)d - dbar;
+        sdd += w * dc * dc;
+        sdy += w * dc * ((real)y[l] - ybar);
+    }
+    real a = ybar - (sdy / sdd) * dbar;
+    real e = (real)y[i] - a;
+    *e2 = e * e;
+    return 1;
+}
+
+int kro_ll_cv(const double *x, const double *y, int64_t n, const double *h, int32_t m, int32_t kernel,
+              const int64_t *rows, int64_t nrows, double *S_out, int64_t *neff_out, double *cv_out,
+              int32_t *best_out)
+{
+    int st = kro_validate(x, y, n, h, m, kernel);
+    if (st) return st;
+    if (kernel == KRO_GAUSSIAN) return KRO_EKERNEL;
+    int64_t R = rows ? nrows : n;
+    if (R < 0) return KRO_EARG;
+    if (rows)
+        for (int64_t r = 0; r < R; r++)
+            if (rows[r] < 0 || rows[r] >= n) return KRO_EARG;
+    real *S = (real *)calloc((size_t)m, sizeof(real));
+    int64_t *ne = (int64_t *)calloc((size_t)m, sizeof(int64_t));
+    if (!S || !ne) { free(S); free(ne); return KRO_ENOMEM; }
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int32_t b = 0; b < m; b++) {
+        real Sb = 0;
+        int64_t nb = 0;
+        for (int64_t r = 0; r < R; r++) {
+            int64_t i = rows ? rows[r] : r;
+            real e2 = 0;
+            if (ll_row(x, y, n, h[b], kernel, i, &e2)) { Sb += e2; nb++; }
+        }
+        S[b] = Sb;
+        ne[b] = nb;
+    }
+    for (int32_t b = 0; b < m; b++) {
+        if (S_out) S_out[b] = (double)S[b];
+        if (neff_out) neff_out[b] = ne[b];
+    }
+    kro_finish(S, n, m, cv_out, best_out);
+    free(S); free(ne);
+    return KRO_OK;
+}

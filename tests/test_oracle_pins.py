@@ -474,3 +474,106 @@ def test_KDE_invariances_and_rows():
         p1 = oracle.kde_lscv(x, h, k, rows=np.arange(0, 150))
         p2 = oracle.kde_lscv(x, h, k, rows=np.arange(150, 300))
         assert cv_rel_err(p1.A + p2.A, a.A) <= 1e-14 and cv_rel_err(p1.B + p2.B, a.B) <= 1e-14
+
+
+# ---------------------------------------------------------------- local-linear (reading Q25)
+def test_LL_worked_example():
+    """Hand-derived fixture tests/golden/ll_worked_example.json."""
+    g = json.load(open(os.path.join(GOLDEN, "ll_worked_example.json")))
+    for case in g["cases"]:
+        k = workloads.KERNEL_IDS[case["kernel"]]
+        r = oracle.ll_cv(g["x"], g["y"], [case["h"]], k)
+        want = float(Fraction(case["cv"]))
+        assert abs(r.cv[0] - want) <= math.ulp(want) if want else r.cv[0] == 0.0
+        assert int(r.neff[0]) == case["neff"]
+
+
+@pytest.mark.parametrize("seed", range(16))
+def test_LL_exact_rational_bruteforce(seed):
+    """Cramer's-rule normal equations in exact rationals (exact.ll_cv_exact,
+    the uncentred form) vs the oracle's centred long-double form, on dyadic
+    inputs with duplicates and points exactly at h."""
+    rng = np.random.default_rng(7000 + seed)
+    n = int(rng.integers(2, 15))
+    m = int(rng.integers(1, 7))
+    x, y, h = workloads.random_dyadic(n, m, seed + 500)
+    for k in KERNELS:
+        cv_ex, ne_ex, best_ex = exact.ll_cv_exact(x, y, h, k)
+        r = oracle.ll_cv(x, y, h, k)
+        assert list(r.neff) == ne_ex, k
+        assert _frac_rel(r.cv, cv_ex) <= 1e-15, (k, r.cv, [float(c) for c in cv_ex])
+        assert r.best == best_ex or r.cv[r.best] == r.cv[best_ex]
+
+
+@pytest.mark.parametrize("k", KERNELS)
+def test_LL_reproduces_lines(k):
+    """A local-linear fit reproduces any line exactly: y = a + b x on a dyadic
+    grid (every product exact) gives e = 0 for every counted row, so CV = 0
+    to long-double rounding, while Nadaraya-Watson (which has O(h) bias on a
+    slope) does not."""
+    x = np.arange(64, dtype=np.float64) / 16.0
+    x = x[np.random.default_rng(3).permutation(64)]
+    y = 0.75 - 2.5 * x
+    h = np.array([0.0625, 0.125, 0.3, 1.0, 4.0])
+    r = oracle.ll_cv(x, y, h, k)
+    assert np.all(r.cv <= 1e-28), r.cv
+    assert r.neff[-1] == 64
+    assert oracle.cv_direct(x, y, h[2:], k).cv.min() > 1e-6
+
+
+def test_LL_uniform_large_h_is_ols_press():
+    """Uniform kernel with h >= range: every weight is 1/2, the LOO fit is
+    ordinary least squares without row i, whose residual is the PRESS residual
+    e_i / (1 - H_ii) of the full OLS fit (hat matrix H = X (X'X)^-1 X',
+    numpy.linalg)."""
+    x, y = workloads.draw_xy("sin_uniform", 400, 9)
+    X = np.stack([np.ones_like(x), x], axis=1)
+    H = X @ np.linalg.solve(X.T @ X, X.T)
+    e = y - H @ y
+    press = float(np.mean((e / (1.0 - np.diag(H))) ** 2))
+    r = float(x.max() - x.min())
+    res = oracle.ll_cv(x, y, np.array([r, 3.0 * r]), U)
+    assert cv_rel_err(res.cv, [press, press]) <= 1e-12
+
+
+@pytest.mark.parametrize("k", KERNELS)
+def test_LL_invariances(k):
+    """Adding a line to y leaves every LOO residual unchanged; (x, h) scaled by
+    2^j is bit-identical; permuting rows changes nothing; n_eff counts rows with
+    >= 2 distinct x in the window (checked against a direct count)."""
+    x, y = workloads.draw_xy("paper", 300, 4)
+    h = workloads.grid_default(x, 10)
+    base = oracle.ll_cv(x, y, h, k)
+    r = oracle.ll_cv(x, y + 3.0 - 7.0 * x, h, k)
+    assert cv_rel_err(r.cv, base.cv) <= 1e-11
+    r = oracle.ll_cv(x * 4.0, y, h * 4.0, k)
+    assert np.array_equal(r.cv, base.cv)
+    p = np.random.default_rng(0).permutation(x.shape[0])
+    r = oracle.ll_cv(x[p], y[p], h, k)
+    assert cv_rel_err(r.cv, base.cv) <= 1e-15
+    for b in (0, 1):
+        cnt = 0
+        for i in range(x.shape[0]):
+            d = np.abs(x - x[i])
+            inw = (d <= h[b]) if k == U else (d < h[b])
+            inw[i] = False
+            cnt += int(np.unique(x[inw]).shape[0] >= 2)
+        assert base.neff[b] == cnt
+
+
+def test_LL_duplicates_and_rows():
+    """Windows whose points share one x are M = 0 (singular normal
+    equations); shard rows add up to the full S."""
+    x = np.array([0.0, 0.5, 0.5, 0.5, 2.0, 2.0])
+    y = np.array([1.0, 2.0, 3.0, 5.0, 1.0, 4.0])
+    r = oracle.ll_cv(x, y, [0.25, 1.0], E)
+    # h = 0.25: rows 1-3 see only duplicates at 0.5, rows 4-5 see each other
+    # (one x), row 0 sees nothing -> no row counted.  h = 1: rows 1-3 see
+    # x = 0 and 0.5 (counted); row 0 sees only x = 0.5, rows 4-5 only x = 2
+    assert list(r.neff) == [0, 3] and r.cv[0] == 0.0
+    x, y = workloads.draw_xy("paper", 500, 2)
+    h = workloads.grid_default(x, 8)
+    full = oracle.ll_cv(x, y, h, E)
+    parts = [oracle.ll_cv(x, y, h, E, rows=oracle.shard_rows(x, s, 3)) for s in range(3)]
+    assert cv_rel_err(sum(p.S for p in parts), full.S) <= 1e-14
+    assert np.array_equal(sum(p.neff for p in parts), full.neff)
