@@ -68,6 +68,8 @@ def parse():
     ap.add_argument("--no-alt", action="store_true", help="skip timing the other algorithm (alt_algo)")
     ap.add_argument("--kde", action="store_true",
                     help="time the KDE least-squares CV (kr_kde_lscv_async, SURVEY §8(f) rank 3) on the config's x")
+    ap.add_argument("--ll", action="store_true",
+                    help="time the local-linear LOO CV (kr_ll_cv_grid_async, SURVEY §8(f) rank 4) on the config")
     ap.add_argument("--kernel", default=None, choices=["uniform", "epanechnikov", "triangular", "gaussian"],
                     help="override the config's kernel (e.g. the Gaussian dense path on C2's data)")
     ap.add_argument("--algo", default="auto", choices=["auto", "sweep", "prefix"],
@@ -489,10 +491,93 @@ def run_kde(args):
     return 0
 
 
+# Local-linear algorithmic work per (row, bandwidth), Epanechnikov, in the
+# double formula: 9 prefix differences, binomial shifts of
+# D1..D4 (10 multiply-adds) and Y0..Y3 (6), S0..S2, T0, T1 (5 FMA), det and
+# num (2 x 3), g (1), e^2 and its sum (3): 61 flops.  Uniform: 5 differences,
+# shifts D1, D2, Y1 (4 multiply-adds), det/num (6), g, e^2, sum (4): 23.
+LL_FLOPS = {0: 23, 1: 61, 2: 2 * 61}
+
+
+def run_ll(args):
+    """Local-linear LOO CV (reading Q25) on the config: device-timed whole
+    searches (kr_ll_cv_grid_async), pair-bandwidth evaluations n (n-1) m per
+    second, the window kernel's FP64 roofline fraction; one JSON line."""
+    import ctypes
+
+    import torch
+
+    from paper_conf_ipps_rohlfsz17_b200 import krcv
+
+    torch.cuda.set_device(0)
+    dev = torch.device("cuda", 0)
+    cfg = workloads.CONFIGS[args.config]
+    x, y, h, k = workloads.make(cfg, seed=args.seed)
+    if args.kernel:
+        k = workloads.KERNEL_IDS[args.kernel]
+    n, m = x.shape[0], h.shape[0]
+    d_x, d_y, d_h = (torch.as_tensor(a, device=dev) for a in (x, y, h))
+    ws = krcv.aligned(krcv.workspace(n, m, dev))
+    cv = torch.empty(m, dtype=torch.float64, device=dev)
+    bs = torch.empty(2, dtype=torch.int32, device=dev)
+    stream = torch.cuda.current_stream(dev)
+    lib = krcv._lib()
+
+    def run():
+        st = lib.kr_ll_cv_grid_async(d_x.data_ptr(), d_y.data_ptr(), n, d_h.data_ptr(), m, k, cv.data_ptr(), None,
+                                     bs.data_ptr(), ws.data_ptr(), ws.numel(), ctypes.c_void_p(stream.cuda_stream))
+        if st:
+            raise krcv.KrcvError(st, "kr_ll_cv_grid_async")
+
+    for _ in range(args.warmup):
+        run()
+    torch.cuda.synchronize()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    krcv.kr_profile_enable(True)
+    tot, win = 0.0, 0.0
+    stages = [0.0] * 4
+    with ClockSampler(0) as clk:
+        for s_ in range(args.steps):
+            flush.fill_(s_ & 0xFF)
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            run()
+            b.record(stream)
+            stg = krcv.kr_profile_read()
+            stages = [u + v for u, v in zip(stages, stg)]
+            tot += a.elapsed_time(b)
+    krcv.kr_profile_enable(False)
+    best = int(bs[0])
+    units = n * (n - 1) * m
+    kms = stages[2] / args.steps
+    flops = LL_FLOPS.get(k, 61) * n * m
+    peak = SM_COUNT * FP64_LANES_PER_SM * 2 * SM_MAX_MHZ_NOMINAL * 1e6 / 1e12  # TFLOP/s, as run_ours
+    ach = flops / (kms * 1e-3) / 1e12
+    print(json.dumps({
+        "metric": "local-linear LOO-CV pair-bandwidth evals/s (SURVEY 8(f) rank 4)",
+        "value": units * args.steps / (tot * 1e-3), "unit": UNIT, "n_gpus": 1, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": tot / args.steps, "higher_is_better": True, "dtype": "f64",
+        "data": "synthetic",
+        "config": {"workload": f"{cfg.name}, local-linear, {workloads.KERNEL_NAMES[k]}", "n": n, "m": m,
+                   "l2": "flushed between timed steps (256 MiB write, outside the events)"},
+        "roofline": {"bound": "alu", "kernel": "ll_window_kernel", "achieved": ach, "peak": peak, "unit": "TFLOP/s",
+                     "frac": ach / peak, "traffic": None, "flops_per_launch": flops,
+                     "flops_basis": f"{LL_FLOPS.get(k, 61)} flops per (row, bandwidth) in the double formula "
+                                    "(DESIGN.md 6.7); dd arithmetic and searches not counted",
+                     "kernel_ms": kms, "kernel_share_of_step": kms / (tot / args.steps)},
+        "stage_ms": {"pack_sort_gather": stages[0] / args.steps, "prefix_build": stages[1] / args.steps,
+                     "window": kms, "reduce_finalize": stages[3] / args.steps},
+        "result": {"best": best, "h_best": float(h[best]), "cv_best": float(cv[best])},
+        "clocks": clk.summary()}), flush=True)
+    return 0
+
+
 def main():
     args = parse()
     if args.kde:
         return run_kde(args)
+    if args.ll:
+        return run_ll(args)
     if args.algo != "auto":
         os.environ["KRCV_ALGO"] = args.algo
     if args.impl == "reference":

@@ -173,6 +173,37 @@ int kr_kde_shard_async(const double *d_x, int64_t n, const double *d_h, int32_t 
 int kr_kde_finalize(const double *partial, int64_t n, const double *h_grid, int32_t m, int32_t kernel,
                     double *lscv_out, int32_t *best_out);
 
+/*
+ * Local-linear leave-one-out CV (§IV P@15728-15905: "The
+ * Nadaraya-Watson local constant estimator is used rather than a local
+ * linear regression" -- the named alternative; reading Q25).
+ * Per row i and bandwidth h the LOO estimate is the intercept at x_i of the
+ * kernel-weighted least-squares line through the window of Eq.(2) (reading
+ * Q1, row i excluded), weights K(|x_l - x_i|/h) of Eq.(3) / footnote 1:
+ *   g = (S2 T0 - S1 T1) / (S0 S2 - S1^2),  S_k = sum w d^k, T_k = sum w y d^k.
+ * M_i = [the window holds >= 2 distinct x] (else the 2x2 system is
+ * singular); CV(h) = n^-1 sum_i M_i (y_i - g)^2 as Eq.(1), best as Q11.
+ * Kernels KR_UNIFORM | KR_EPANECHNIKOV | KR_TRIANGULAR (KR_EKERNEL for
+ * KR_GAUSSIAN); always the window-prefix path.
+ * kr_ll_cv_grid: host pointers, synchronous, outputs as kr_cv_grid_ex
+ *   (neff_out nullable).  Errors as kr_cv_grid.
+ * kr_ll_cv_grid_async: device pointers, enqueued on cuda_stream; workspace
+ *   from kr_workspace_bytes(n, m); d_cv [m], d_neff [m] int64 (nullable),
+ *   d_best_status [2] = { best, status }.
+ * kr_ll_shard_async: rows [floor(shard n/P), floor((shard+1) n/P)) of the
+ *   sorted order -> d_partial [KR_PARTIAL_LEN(m)], the same additive layout
+ *   as kr_cv_shard_async, so kr_finalize / kr_finalize_async apply.
+ */
+int kr_ll_cv_grid(const double *x, const double *y, int64_t n,
+                  const double *h_grid, int32_t m, int32_t kernel,
+                  double *cv_out, int64_t *neff_out, int32_t *best_out);
+int kr_ll_cv_grid_async(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m,
+                        int32_t kernel, double *d_cv, int64_t *d_neff, int32_t *d_best_status,
+                        void *d_workspace, size_t workspace_bytes, void *cuda_stream);
+int kr_ll_shard_async(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m,
+                      int32_t kernel, int32_t shard, int32_t nshards, double *d_partial,
+                      void *d_workspace, size_t workspace_bytes, void *cuda_stream);
+
 /* Host-side grid check (finite, > 0, non-decreasing, 1 <= m <= KR_MAX_M). */
 int kr_validate_grid(const double *h_grid, int32_t m);
 

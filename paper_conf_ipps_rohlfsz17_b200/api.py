@@ -72,7 +72,7 @@ class GridSearch:
     """
 
     def __init__(self, n: int, h, kernel="epanechnikov", device=None, rank: int = 0, world: int = 1,
-                 group=None, algo="auto"):
+                 group=None, algo="auto", estimator: str = "nw"):
         import torch
 
         self.torch = torch
@@ -84,6 +84,9 @@ class GridSearch:
         self.n, self.m = int(n), int(h_host.shape[0])
         self.kernel = krcv._kernel_id(kernel)
         self.algo = krcv._algo_id(algo)
+        if estimator not in ("nw", "ll"):
+            raise ValueError("estimator must be 'nw' (Nadaraya-Watson, Eq.(2)) or 'll' (local-linear, reading Q25)")
+        self.estimator = estimator
         self.rank, self.world, self.group = int(rank), int(world), group
         self.h = h_host
         self.d_h = torch.as_tensor(h_host, device=self.device)
@@ -97,6 +100,15 @@ class GridSearch:
     def run(self, d_x, d_y) -> None:
         if d_x.numel() != self.n or d_y.numel() != self.n:
             raise ValueError("x, y must have n elements")
+        if self.estimator == "ll":
+            if self.world == 1:
+                krcv.kr_ll_cv_grid_async(d_x, d_y, self.d_h, self.kernel, self.cv, self.neff, self.best_status,
+                                         self.ws)
+                return
+            krcv.kr_ll_shard_async(d_x, d_y, self.d_h, self.kernel, self.rank, self.world, self.partial, self.ws)
+            allreduce_partial(self.partial, self.group)
+            krcv.kr_finalize_async(self.partial, self.n, self.m, self.cv, self.neff, self.best_status)
+            return
         if self.world == 1:  # whole search in one enqueue, finalize fused into the reduction
             krcv.kr_cv_grid_async(d_x, d_y, self.d_h, self.kernel, self.cv, self.neff, self.best_status, self.ws,
                                   algo=self.algo)
@@ -115,11 +127,12 @@ class GridSearch:
 
 
 def cv_grid(x, y, h=None, m: int | None = None, kernel="epanechnikov", device=None, distributed: bool = False,
-            group=None, algo="auto") -> CVResult:
+            group=None, algo="auto", estimator: str = "nw") -> CVResult:
     """LOO-CV grid search.  x, y: numpy arrays or CUDA tensors; h: grid array,
     or None with m for the default grid (§IV P@16146).  With distributed=True
     every rank of the default (or given) process group must call it with the
-    same inputs; the result is identical on every rank."""
+    same inputs; the result is identical on every rank.  estimator: "nw"
+    (Nadaraya-Watson, Eq.(2)) or "ll" (local-linear, reading Q25)."""
     import torch
 
     if h is None:
@@ -135,7 +148,7 @@ def cv_grid(x, y, h=None, m: int | None = None, kernel="epanechnikov", device=No
     dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
     d_x = torch.as_tensor(x, dtype=torch.float64, device=dev).contiguous()
     d_y = torch.as_tensor(y, dtype=torch.float64, device=dev).contiguous()
-    plan = GridSearch(d_x.numel(), h, kernel, dev, rank, world, group, algo)
+    plan = GridSearch(d_x.numel(), h, kernel, dev, rank, world, group, algo, estimator)
     plan.run(d_x, d_y)
     return plan.result()
 

@@ -28,6 +28,7 @@
 #include "krcv_prefix.cuh"
 #include "krcv_dense.cuh"
 #include "krcv_kde.cuh"
+#include "krcv_ll.cuh"
 
 namespace krcv {
 
@@ -511,6 +512,39 @@ static void launch_window(int K, const double2 *xy, int n, const double *h, int 
     }
 }
 
+// Local-linear window kernel (krcv_ll.cuh): one row per lane, the same
+// task split as window_kernel.
+template <int KERN>
+static void launch_ll_window(const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
+                             const WsLayout &L, char *ws, double *tileS, uint8_t *tileN, int *counter,
+                             cudaStream_t st)
+{
+    static int resident = 0, sms = 0;
+    if (!resident) {
+        int b = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, ll_window_kernel<KERN>, kWinThreads, 0);
+        resident = b > 0 ? b : 1;
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (sms <= 0) sms = 148;
+    }
+    const int64_t want = (int64_t)sms * kWinTasksPerSM;
+    int nbc = (int)((want + ntiles - 1) / ntiles);
+    const int max_nbc = (m + kWinMinBper - 1) / kWinMinBper;
+    if (nbc > max_nbc) nbc = max_nbc;
+    if (nbc < 1) nbc = 1;
+    const int64_t tasks = (int64_t)ntiles * nbc;
+    int blocks = (int)((tasks + kWinWarps - 1) / kWinWarps);
+    if (blocks > sms * resident) blocks = sms * resident;
+    const double *xs = reinterpret_cast<const double *>(ws + L.xs) + kPad;
+    const double *P = reinterpret_cast<const double *>(ws + L.pfx);
+    const unsigned long long *ymax =
+        reinterpret_cast<const unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
+    ll_window_kernel<KERN><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc,
+                                                           ymax, tileS, tileN, counter);
+}
+
 }  // namespace krcv
 
 using namespace krcv;
@@ -599,7 +633,8 @@ static int enqueue_sort(const double *d_x, const double *d_y, int64_t n, const d
 // coarse-to-fine refinement, kr_cv_refine).
 static int enqueue(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m, int32_t kernel,
                    int32_t algo, int32_t shard, int32_t nshards, double *d_partial, FinOut fin,
-                   void *d_workspace, size_t workspace_bytes, void *cuda_stream, bool reuse_sorted = false)
+                   void *d_workspace, size_t workspace_bytes, void *cuda_stream, bool reuse_sorted = false,
+                   bool ll = false)
 {
     if (!d_x || !d_y || !d_h || !d_workspace) return KR_EARG;
     if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return KR_EARG;
@@ -607,6 +642,11 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         return KR_EKERNEL;
     if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX && algo != KR_ALGO_DENSE)
         return KR_EARG;
+    if (ll) {  // local-linear: compact kernels on the window-prefix path only
+        if (kernel == KR_GAUSSIAN) return KR_EKERNEL;
+        if (algo != KR_ALGO_AUTO && algo != KR_ALGO_PREFIX) return KR_EARG;
+        algo = KR_ALGO_PREFIX;
+    }
     // the Gaussian has no compact support: only the dense path applies, and
     // the dense path is only for it
     if ((kernel == KR_GAUSSIAN) != (algo == KR_ALGO_DENSE || (algo == KR_ALGO_AUTO && kernel == KR_GAUSSIAN)))
@@ -641,7 +681,7 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     const int variant = sweep_variant(hi - lo);
     int G = sweep_G(hi - lo);
     if (variant == 1 && G > 4) G = 4;
-    const int winK = win_rows_per_lane(hi - lo);
+    const int winK = ll ? 1 : win_rows_per_lane(hi - lo);
     const int rows_per_tile = 32 * ((winK == 3 || winK == 5) ? 1 : winK);
     const int ntiles = prefix ? (int)((hi - lo + rows_per_tile - 1) / rows_per_tile)
                               : dense ? (int)tiles_for(hi - lo, 1)
@@ -660,7 +700,10 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         if (st2) return st2;
     }
     prof_mark(1, st);
-    if (prefix && !reuse_sorted) {
+    if (prefix && !reuse_sorted && ll) {
+        launch_prefix_build<kLLMoments>(xy, nn, L, ws, st);
+        launches += 2;
+    } else if (prefix && !reuse_sorted) {
         switch (kernel) {
         case KR_UNIFORM: launch_prefix_build<KR_UNIFORM>(xy, nn, L, ws, st); break;
         case KR_EPANECHNIKOV: launch_prefix_build<KR_EPANECHNIKOV>(xy, nn, L, ws, st); break;
@@ -675,6 +718,18 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
             const int nrt = (hi - lo + kGThreads - 1) / kGThreads;
             const int nbc = (m + kGB - 1) / kGB;
             gauss_kernel<<<nrt * nbc, kGThreads, 0, st>>>(xy, nn, d_h, m, lo, hi, nbc, ntiles, tileS, tileN);
+        } else if (prefix && ll) {
+            switch (kernel) {
+            case KR_UNIFORM:
+                launch_ll_window<KR_UNIFORM>(xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
+                break;
+            case KR_EPANECHNIKOV:
+                launch_ll_window<KR_EPANECHNIKOV>(xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
+                break;
+            default:
+                launch_ll_window<KR_TRIANGULAR>(xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
+                break;
+            }
         } else if (prefix) {
             switch (kernel) {
             case KR_UNIFORM:
@@ -758,6 +813,33 @@ extern "C" int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n
 {
     return kr_cv_shard_algo_async(d_x, d_y, n, d_h, m, kernel, KR_ALGO_AUTO, shard, nshards, d_partial,
                                   d_workspace, workspace_bytes, cuda_stream);
+}
+
+// Local-linear LOO CV (krcv_ll.cuh, reading Q25): same pipeline and
+// partial layout as Nadaraya-Watson, other prefix moments and window kernel.
+extern "C" int kr_ll_cv_grid_async(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m,
+                                   int32_t kernel, double *d_cv, int64_t *d_neff, int32_t *d_best_status,
+                                   void *d_workspace, size_t workspace_bytes, void *cuda_stream)
+{
+    if (!d_cv || !d_best_status) return KR_EARG;
+    FinOut fin{};
+    fin.n = (long long)n;
+    fin.cv = d_cv;
+    fin.neff = reinterpret_cast<long long *>(d_neff);
+    fin.best = d_best_status;
+    fin.status = d_best_status + 1;
+    return enqueue(d_x, d_y, n, d_h, m, kernel, KR_ALGO_PREFIX, 0, 1, nullptr, fin, d_workspace, workspace_bytes,
+                   cuda_stream, false, true);
+}
+
+extern "C" int kr_ll_shard_async(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m,
+                                 int32_t kernel, int32_t shard, int32_t nshards, double *d_partial,
+                                 void *d_workspace, size_t workspace_bytes, void *cuda_stream)
+{
+    if (!d_partial) return KR_EARG;
+    FinOut fin{};
+    return enqueue(d_x, d_y, n, d_h, m, kernel, KR_ALGO_PREFIX, shard, nshards, d_partial, fin, d_workspace,
+                   workspace_bytes, cuda_stream, false, true);
 }
 
 extern "C" int kr_finalize_async(const double *d_partial, int64_t n, int32_t m, double *d_cv,

@@ -170,6 +170,40 @@ extern "C" int kr_cv_grid_algo(const double *x, const double *y, int64_t n, cons
     return KR_OK;
 }
 
+extern "C" int kr_ll_cv_grid(const double *x, const double *y, int64_t n, const double *h_grid, int32_t m,
+                             int32_t kernel, double *cv_out, int64_t *neff_out, int32_t *best_out)
+{
+    if (!cv_out || !best_out) return KR_EARG;
+    int st = validate_all(x, y, n, h_grid, m, kernel);
+    if (st) return st;
+    if (kernel == KR_GAUSSIAN) return KR_EKERNEL;
+    int dev = 0;
+    KR_CUDA_TRY(cudaGetDevice(&dev));
+    DevCtx *c = get_ctx(dev);
+    std::lock_guard<std::mutex> g(c->mu);
+    st = ensure_capacity(c, n, m);
+    if (st) return st;
+    cudaStream_t s = c->stream;
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dx, x, sizeof(double) * n, cudaMemcpyHostToDevice, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dy, y, sizeof(double) * n, cudaMemcpyHostToDevice, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dh, h_grid, sizeof(double) * m, cudaMemcpyHostToDevice, s));
+    st = kr_ll_cv_grid_async(c->dx, c->dy, n, c->dh, m, kernel, c->dcv, c->dneff, c->dbest, c->ws, c->ws_bytes, s);
+    if (st) return st;
+    std::vector<double> cv(m);
+    std::vector<int64_t> ne(neff_out ? m : 0);
+    int32_t bs[2] = {0, 0};
+    KR_CUDA_TRY(cudaMemcpyAsync(cv.data(), c->dcv, sizeof(double) * m, cudaMemcpyDeviceToHost, s));
+    if (neff_out)
+        KR_CUDA_TRY(cudaMemcpyAsync(ne.data(), c->dneff, sizeof(int64_t) * m, cudaMemcpyDeviceToHost, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(bs, c->dbest, sizeof(int32_t) * 2, cudaMemcpyDeviceToHost, s));
+    KR_CUDA_TRY(cudaStreamSynchronize(s));
+    if (bs[1] != KR_OK) return bs[1];
+    std::memcpy(cv_out, cv.data(), sizeof(double) * m);
+    if (neff_out) std::memcpy(neff_out, ne.data(), sizeof(int64_t) * m);
+    *best_out = bs[0];
+    return KR_OK;
+}
+
 extern "C" int kr_cv_grid_ex(const double *x, const double *y, int64_t n, const double *h_grid, int32_t m,
                              int32_t kernel, double *cv_out, int64_t *neff_out, int32_t *best_out)
 {

@@ -29,8 +29,8 @@ struct WsLayout {
                                 //              u64 bits of max |y| (window-prefix fast-path bound)
     size_t partial;             // double  [2m+2] partial vector of kr_cv_grid_async
     size_t xs;                  // double  [n + 2 kPad] sorted x, +-inf sentinels (prefix path)
-    size_t pfx;                 // double [5][2][pstride] dd prefix moments P[k][0..n], hi / lo planes
-    size_t ptot;                // double2 [5][nch] prefix tile totals
+    size_t pfx;                 // double [8][2][pstride] dd prefix moments P[k][0..n], hi / lo planes
+    size_t ptot;                // double2 [8][nch] prefix tile totals
     int64_t pstride, nch;
     size_t cub;                 // radix-sort scratch
     size_t cub_bytes;

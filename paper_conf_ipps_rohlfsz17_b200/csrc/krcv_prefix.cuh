@@ -52,7 +52,7 @@
 namespace krcv {
 
 constexpr int kPfxThreads = 256;      // prefix build CTA
-constexpr int kPfxMoments = 5;        // slots reserved in the workspace
+constexpr int kPfxMoments = 8;        // slots reserved in the workspace (local-linear uses all 8)
 constexpr int kWinWarps = 4;
 constexpr int kWinThreads = kWinWarps * 32;
 constexpr int kWinTasksPerSM = 64;    // warp tasks per SM the b-split aims for
@@ -62,10 +62,14 @@ constexpr int kWinMinBper = 8;        // >= this many bandwidths per task
 // Triangular: y, u, y u.  Uniform: y.
 // Pseudo-kernel id of the KDE moment set (krcv_kde.cuh): u, u^2, ..., u^5.
 constexpr int kKdeMoments = 100;
+// Pseudo-kernel id of the local-linear moment set (krcv_ll.cuh):
+// y, u, u^2, u^3, u^4, y u, y u^2, y u^3.
+constexpr int kLLMoments = 101;
 
 template <int KERN>
 struct NMom {
-    static constexpr int v = KERN == KR_UNIFORM ? 1 : (KERN == KR_TRIANGULAR ? 3 : 5);
+    static constexpr int v =
+        KERN == kLLMoments ? 8 : (KERN == KR_UNIFORM ? 1 : (KERN == KR_TRIANGULAR ? 3 : 5));
 };
 
 template <int KERN>
@@ -78,6 +82,19 @@ __device__ __forceinline__ void moment_terms(double x, double y, double o, dd (&
         t[2] = dd_mul(t[1], u);
         t[3] = dd_mul(t[1], t[1]);
         t[4] = dd_mul(t[3], u);
+        return;
+    }
+    if (KERN == kLLMoments) {  // local-linear: y, u .. u^4, y u .. y u^3
+        const dd u = two_sum(x, -o);
+        const dd u2 = dd_mul(u, u), u3 = dd_mul(u2, u);
+        t[0] = dd_make(y);
+        t[1] = u;
+        t[2] = u2;
+        t[3] = u3;
+        t[4] = dd_mul(u2, u2);
+        t[5] = dd_mul_d(u, y);
+        t[6] = dd_mul_d(u2, y);
+        t[7] = dd_mul_d(u3, y);
         return;
     }
     t[0] = dd_make(y);

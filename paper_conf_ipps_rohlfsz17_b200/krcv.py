@@ -38,6 +38,7 @@ EXPORTS = (
     "kr_strerror", "kr_last_cuda_error", "kr_version",
     "kr_profile_enable", "kr_profile_read", "kr_launch_count", "kr_last_algo",
     "kr_kde_lscv", "kr_kde_lscv_async", "kr_kde_shard_async", "kr_kde_finalize",
+    "kr_ll_cv_grid", "kr_ll_cv_grid_async", "kr_ll_shard_async",
 )
 
 
@@ -98,6 +99,11 @@ def _lib() -> ctypes.CDLL:
     lib.kr_kde_shard_async.argtypes = [P, i64, P, i32, i32, i32, i32, P, P, sz, P]
     lib.kr_kde_finalize.argtypes = [P, i64, P, i32, i32, P, P]
     for f in ("kr_kde_lscv", "kr_kde_lscv_async", "kr_kde_shard_async", "kr_kde_finalize"):
+        getattr(lib, f).restype = ctypes.c_int
+    lib.kr_ll_cv_grid.argtypes = [P, P, i64, P, i32, i32, P, P, P]
+    lib.kr_ll_cv_grid_async.argtypes = [P, P, i64, P, i32, i32, P, P, P, P, sz, P]
+    lib.kr_ll_shard_async.argtypes = [P, P, i64, P, i32, i32, i32, i32, P, P, sz, P]
+    for f in ("kr_ll_cv_grid", "kr_ll_cv_grid_async", "kr_ll_shard_async"):
         getattr(lib, f).restype = ctypes.c_int
     lib.kr_last_algo.restype = ctypes.c_int32
     _LIB = lib
@@ -337,3 +343,54 @@ def kr_kde_finalize(partial, n: int, h, kernel="epanechnikov"):
     _check(_lib().kr_kde_finalize(p.ctypes.data, int(n), h.ctypes.data, h.shape[0], _kernel_id(kernel),
                                   out.ctypes.data, ctypes.byref(best)), "kr_kde_finalize")
     return out, int(best.value)
+
+
+# ------------------------------------------------------- local-linear (Q25)
+def kr_ll_cv_grid(x, y, h, kernel="epanechnikov", with_neff: bool = False):
+    """Local-linear LOO-CV grid search from host arrays (kr_ll_cv_grid).
+    Returns (cv[m], best) or (cv, neff, best)."""
+    x, y, h = _host(x), _host(y), _host(h)
+    if x.shape != y.shape or x.ndim != 1:
+        raise ValueError("x and y must be 1-D arrays of equal length")
+    n, m = x.shape[0], h.shape[0]
+    cv = np.empty(m, np.float64)
+    neff = np.empty(m, np.int64)
+    best = ctypes.c_int32(-1)
+    _check(_lib().kr_ll_cv_grid(x.ctypes.data, y.ctypes.data, n, h.ctypes.data, m, _kernel_id(kernel),
+                                cv.ctypes.data, neff.ctypes.data, ctypes.byref(best)), "kr_ll_cv_grid")
+    return (cv, neff, int(best.value)) if with_neff else (cv, int(best.value))
+
+
+def kr_ll_cv_grid_async(d_x, d_y, d_h, kernel, d_cv, d_neff, d_best_status, d_ws, stream=None) -> None:
+    """Enqueue the whole single-GPU local-linear search (tensors as kr_cv_grid_async)."""
+    import torch
+
+    n, m = d_x.numel(), d_h.numel()
+    for t, name in ((d_x, "x"), (d_y, "y"), (d_h, "h"), (d_cv, "cv")):
+        if not (t.is_cuda and t.dtype == torch.float64 and t.is_contiguous()):
+            raise ValueError(f"{name} must be a contiguous float64 CUDA tensor")
+    if d_cv.numel() != m or d_best_status.numel() != 2 or d_best_status.dtype != torch.int32:
+        raise ValueError("cv must have m elements, best_status 2 int32")
+    s = torch.cuda.current_stream(d_x.device) if stream is None else stream
+    _check(_lib().kr_ll_cv_grid_async(d_x.data_ptr(), d_y.data_ptr(), n, d_h.data_ptr(), m, _kernel_id(kernel),
+                                      d_cv.data_ptr(), None if d_neff is None else d_neff.data_ptr(),
+                                      d_best_status.data_ptr(), d_ws.data_ptr(), d_ws.numel() * d_ws.element_size(),
+                                      ctypes.c_void_p(s.cuda_stream)), "kr_ll_cv_grid_async")
+
+
+def kr_ll_shard_async(d_x, d_y, d_h, kernel, shard: int, nshards: int, d_partial, d_ws, stream=None) -> None:
+    """Enqueue one row shard of the local-linear search -> additive partial
+    [S | neff | status] (finalize with kr_finalize / kr_finalize_async)."""
+    import torch
+
+    n, m = d_x.numel(), d_h.numel()
+    for t, name in ((d_x, "x"), (d_y, "y"), (d_h, "h"), (d_partial, "partial")):
+        if not (t.is_cuda and t.dtype == torch.float64 and t.is_contiguous()):
+            raise ValueError(f"{name} must be a contiguous float64 CUDA tensor")
+    if d_partial.numel() != partial_len(m):
+        raise ValueError("partial must have 2m+2 elements")
+    s = torch.cuda.current_stream(d_x.device) if stream is None else stream
+    _check(_lib().kr_ll_shard_async(d_x.data_ptr(), d_y.data_ptr(), n, d_h.data_ptr(), m, _kernel_id(kernel),
+                                    int(shard), int(nshards), d_partial.data_ptr(), d_ws.data_ptr(),
+                                    d_ws.numel() * d_ws.element_size(), ctypes.c_void_p(s.cuda_stream)),
+           "kr_ll_shard_async")
