@@ -72,7 +72,7 @@ def parse():
                     help="time the local-linear LOO CV (kr_ll_cv_grid_async, SURVEY §8(f) rank 4) on the config")
     ap.add_argument("--kernel", default=None, choices=["uniform", "epanechnikov", "triangular", "gaussian"],
                     help="override the config's kernel (e.g. the Gaussian dense path on C2's data)")
-    ap.add_argument("--algo", default="auto", choices=["auto", "sweep", "prefix"],
+    ap.add_argument("--algo", default="auto", choices=["auto", "sweep", "prefix", "hist"],
                     help="KR_ALGO_* for every call (sets KRCV_ALGO before the library loads)")
     ap.add_argument("--cpu-seconds", type=float, default=8.0,
                     help="target wall seconds of the bounded oracle sample")
@@ -287,7 +287,7 @@ def run_ours(args):
             torch.cuda.synchronize()
         barrier()
         krcv.kr_profile_enable(False)
-        used = {1: "sweep", 2: "prefix", 3: "dense"}.get(krcv.kr_last_algo(), "?")
+        used = {1: "sweep", 2: "prefix", 3: "dense", 4: "hist"}.get(krcv.kr_last_algo(), "?")
         total_ms = sum(starts[s].elapsed_time(ends[s]) for s in range(args.steps))
         main_total = sum(main_ms)
         if world > 1:
@@ -302,8 +302,9 @@ def run_ours(args):
             flops = rows_mine * (n - 1) * m * FLOPS_PER_PAIR_BW_DENSE
             basis = (f"{FLOPS_PER_PAIR_BW_DENSE} flops per (ordered pair, bandwidth) incl. the fp64 exp; "
                      "column truncation (weights < e^-64) not credited")
-        elif used == "sweep":
-            kname = "sweep_kernel (a3+a4, per-pair running sums)"
+        elif used in ("sweep", "hist"):
+            kname = ("sweep_kernel (a3+a4, per-pair running sums)" if used == "sweep" else
+                     "hist_kernel (a3+a4, bucket-by-bandwidth smem histogram + warp scan)")
             flops = rows_mine * (n - 1) * FLOPS_PER_PAIR[k] + rows_mine * m * FLOPS_PER_EMIT[k]
             basis = (f"{FLOPS_PER_PAIR[k]} flops per ordered pair x rows x (n-1) + {FLOPS_PER_EMIT[k]} per "
                      "(row, bandwidth) emit")

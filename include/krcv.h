@@ -86,10 +86,17 @@ enum {
     KR_ALGO_AUTO = 0,
     KR_ALGO_SWEEP = 1,
     KR_ALGO_PREFIX = 2,
-    KR_ALGO_DENSE = 3   /* tiled all-pairs x all-bandwidths, the only path for
+    KR_ALGO_DENSE = 3,  /* tiled all-pairs x all-bandwidths, the only path for
                            KR_GAUSSIAN (AUTO picks it); KR_EARG with the
-                           compact kernels, and SWEEP / PREFIX give KR_EARG
-                           with KR_GAUSSIAN */
+                           compact kernels, and SWEEP / PREFIX / HIST give
+                           KR_EARG with KR_GAUSSIAN */
+    KR_ALGO_HIST = 4    /* bucket-by-bandwidth shared-memory histogram + warp
+                           scan (north_star's named alternative to a per-row
+                           sort; SURVEY.md §7.1 "H", an ablation -- never
+                           chosen by AUTO): O(n^2) bucketed pairs with
+                           shared-memory atomics; sums agree with the other
+                           paths to rounding, not bitwise (atomic order).
+                           m <= 5,000 (shared-memory histogram; KR_EARG above) */
 };
 
 /* Length of the partial vector of the device path: [ S[0..m) | neff[0..m) |

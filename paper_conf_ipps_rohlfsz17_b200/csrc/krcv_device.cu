@@ -18,6 +18,7 @@
 
 #include <cmath>
 #include <cstdint>
+#include <cstdio>
 #include <cstdlib>
 
 #include "krcv.h"
@@ -29,6 +30,7 @@
 #include "krcv_dense.cuh"
 #include "krcv_kde.cuh"
 #include "krcv_ll.cuh"
+#include "krcv_hist.cuh"
 
 namespace krcv {
 
@@ -62,13 +64,14 @@ __global__ void pack_kernel(const double *__restrict__ x, const double *__restri
 // the first real record).  Also resets the sweep's tile counter.
 __global__ void gather_kernel(const double *__restrict__ x, const double *__restrict__ y,
                               const uint32_t *__restrict__ order, int n, double2 *__restrict__ xy,
-                              int *__restrict__ tile_counter)
+                              uint32_t *__restrict__ perm, int *__restrict__ tile_counter)
 {
     const int stride = gridDim.x * blockDim.x;
     const int tid = blockIdx.x * blockDim.x + threadIdx.x;
     for (int k = tid; k < n; k += stride) {
         uint32_t i = order[k];
         xy[k] = make_double2(x[i], y[i]);
+        perm[k] = i;
     }
     if (tid < kPad) {
         xy[-1 - tid] = make_double2(-INFINITY, 0.0);
@@ -230,6 +233,7 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     L->vals_out = off; off = align256(off + sizeof(uint32_t) * npad);
     L->xy = off;       off = align256(off + sizeof(double2) * ((size_t)n + 2 * kPad));
     L->counter = off;  off = align256(off + sizeof(int));
+    L->perm = off;     off = align256(off + sizeof(uint32_t) * (size_t)n);
     // window-prefix path (krcv_prefix.cuh)
     const size_t nch = (size_t)((n + kPfxTile) / kPfxTile);  // tiles covering P[0..n]
     L->pstride = (int64_t)(((size_t)n + 1 + 15) & ~size_t(15));
@@ -411,7 +415,7 @@ int auto_algo(int64_t /*n*/, int64_t /*rows*/, int32_t /*m*/, int32_t /*kernel*/
     static int forced = -1;
     if (forced < 0) {
         const char *e = getenv("KRCV_ALGO");
-        forced = !e ? 0 : (e[0] == 's' ? KR_ALGO_SWEEP : (e[0] == 'p' ? KR_ALGO_PREFIX : 0));
+        forced = !e ? 0 : (e[0] == 's' ? KR_ALGO_SWEEP : (e[0] == 'p' ? KR_ALGO_PREFIX : (e[0] == 'h' ? KR_ALGO_HIST : 0)));
     }
     return forced ? forced : KR_ALGO_PREFIX;
 }
@@ -512,6 +516,27 @@ static void launch_window(int K, const double2 *xy, int n, const double *h, int 
     }
 }
 
+// Histogram ordering (krcv_hist.cuh): `warps` warps per CTA (as many as the
+// shared-memory histograms allow) share a 32-row tile; persistent CTAs.
+template <int KERN>
+static void launch_hist(int warps, const double *d_x, const double *d_y, const uint32_t *perm, const double2 *xy,
+                        const double *h, int m, int n, int lo, int hi, int ntiles, double *tileS, uint8_t *tileN,
+                        int *counter, cudaStream_t st)
+{
+    const size_t smem = hist_smem_bytes(m, warps);
+    cudaFuncSetAttribute(hist_kernel<KERN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int resident = 0, dev = 0, sms = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&resident, hist_kernel<KERN>, warps * 32, smem);
+    if (resident < 1) resident = 1;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (sms <= 0) sms = 148;
+    int blocks = ntiles;  // one 32-row tile per CTA iteration
+    if (blocks > sms * resident) blocks = sms * resident;
+    hist_kernel<KERN><<<blocks, warps * 32, smem, st>>>(d_x, d_y, perm, xy, h, m, n, lo, hi, ntiles, tileS, tileN,
+                                                         counter);
+}
+
 // Local-linear window kernel (krcv_ll.cuh): one row per lane, the same
 // task split as window_kernel.
 template <int KERN>
@@ -541,8 +566,20 @@ static void launch_ll_window(const double2 *xy, int n, const double *h, int m, i
     const double *P = reinterpret_cast<const double *>(ws + L.pfx);
     const unsigned long long *ymax =
         reinterpret_cast<const unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
+    // KRCV_LL_STATS=1 (debug): count the branches taken, print to stderr
+    static unsigned long long *stats = nullptr;
+    const bool want_stats = getenv_flag("KRCV_LL_STATS");
+    if (want_stats && !stats) cudaMalloc(&stats, 4 * sizeof(unsigned long long));
+    if (want_stats) cudaMemsetAsync(stats, 0, 4 * sizeof(unsigned long long), st);
     ll_window_kernel<KERN><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc,
-                                                           ymax, tileS, tileN, counter);
+                                                           ymax, tileS, tileN, counter, want_stats ? stats : nullptr);
+    if (want_stats) {
+        unsigned long long v[4] = {0, 0, 0, 0};
+        cudaMemcpyAsync(v, stats, sizeof v, cudaMemcpyDeviceToHost, st);
+        cudaStreamSynchronize(st);
+        fprintf(stderr, "ll stats: direct %llu prefix_ok %llu prefix_rejected %llu rejected_window_points %llu\n",
+                v[0], v[1], v[2], v[3]);
+    }
 }
 
 }  // namespace krcv
@@ -593,6 +630,7 @@ static int enqueue_sort(const double *d_x, const double *d_y, int64_t n, const d
     uint32_t *vals_out = reinterpret_cast<uint32_t *>(ws + L.vals_out);
     double2 *xy = reinterpret_cast<double2 *>(ws + L.xy) + kPad;
     int *counter = reinterpret_cast<int *>(ws + L.counter);
+    uint32_t *perm = reinterpret_cast<uint32_t *>(ws + L.perm);
     unsigned *status = reinterpret_cast<unsigned *>(ws + L.status);
     const int nn = (int)n;
     int64_t launches = 0;
@@ -611,7 +649,8 @@ static int enqueue_sort(const double *d_x, const double *d_y, int64_t n, const d
         default: launch_rank_sort<256, 2>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
         }
         const int npad = nchunks * chunk;
-        rank_scatter_kernel<<<(npad + 255) / 256, 256, 0, st>>>(vals_in, rank, nn, npad, d_x, d_y, xy, counter);
+        rank_scatter_kernel<<<(npad + 255) / 256, 256, 0, st>>>(vals_in, rank, nn, npad, d_x, d_y, xy, perm,
+                                                                 counter);
         launches += nchunks > 1 ? 1 : 0;
         launches += 2;
     } else {
@@ -620,7 +659,7 @@ static int enqueue_sort(const double *d_x, const double *d_y, int64_t n, const d
         e = cub::DeviceRadixSort::SortPairs(ws + L.cub, cub_bytes, keys_in, keys_out, vals_in, vals_out,
                                             nn, 0, 64, st);
         if (e != cudaSuccess) { set_cuda_error("cub::DeviceRadixSort::SortPairs", (int)e); return KR_ECUDA; }
-        gather_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, vals_out, nn, xy, counter);
+        gather_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, vals_out, nn, xy, perm, counter);
         launches += 2 + cub_sort_launches(n);
     }
     *launches_out += launches;
@@ -640,7 +679,8 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return KR_EARG;
     if (kernel != KR_UNIFORM && kernel != KR_EPANECHNIKOV && kernel != KR_TRIANGULAR && kernel != KR_GAUSSIAN)
         return KR_EKERNEL;
-    if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX && algo != KR_ALGO_DENSE)
+    if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX && algo != KR_ALGO_DENSE &&
+        algo != KR_ALGO_HIST)
         return KR_EARG;
     if (ll) {  // local-linear: compact kernels on the window-prefix path only
         if (kernel == KR_GAUSSIAN) return KR_EKERNEL;
@@ -678,12 +718,21 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     if (algo == KR_ALGO_AUTO) algo = kernel == KR_GAUSSIAN ? KR_ALGO_DENSE : auto_algo(n, hi - lo, m, kernel);
     const bool prefix = algo == KR_ALGO_PREFIX;
     const bool dense = algo == KR_ALGO_DENSE;
+    const bool hist = algo == KR_ALGO_HIST;
+    int hist_warps = 0;
+    if (hist) {  // shared-memory histogram: warps per CTA that fit 227 KB
+        const size_t cap = 227 * 1024;
+        for (int w = kHistMaxWarps; w >= 1 && !hist_warps; w--)
+            if (hist_smem_bytes(m, w) <= cap) hist_warps = w;
+        if (!hist_warps) return KR_EARG;
+    }
     const int variant = sweep_variant(hi - lo);
     int G = sweep_G(hi - lo);
     if (variant == 1 && G > 4) G = 4;
     const int winK = ll ? 1 : win_rows_per_lane(hi - lo);
     const int rows_per_tile = 32 * ((winK == 3 || winK == 5) ? 1 : winK);
-    const int ntiles = prefix ? (int)((hi - lo + rows_per_tile - 1) / rows_per_tile)
+    const int ntiles = hist ? (int)((hi - lo + 31) / 32)
+                     : prefix ? (int)((hi - lo + rows_per_tile - 1) / rows_per_tile)
                               : dense ? (int)tiles_for(hi - lo, 1)
                                       : (variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G));
 
@@ -714,7 +763,23 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     prof_mark(2, st);
     if (ntiles > 0) {
         launches += 1;
-        if (dense) {
+        if (hist) {
+            const uint32_t *perm = reinterpret_cast<const uint32_t *>(ws + L.perm);
+            switch (kernel) {
+            case KR_UNIFORM:
+                launch_hist<KR_UNIFORM>(hist_warps, d_x, d_y, perm, xy, d_h, m, nn, lo, hi, ntiles, tileS, tileN,
+                                        counter, st);
+                break;
+            case KR_EPANECHNIKOV:
+                launch_hist<KR_EPANECHNIKOV>(hist_warps, d_x, d_y, perm, xy, d_h, m, nn, lo, hi, ntiles, tileS,
+                                             tileN, counter, st);
+                break;
+            default:
+                launch_hist<KR_TRIANGULAR>(hist_warps, d_x, d_y, perm, xy, d_h, m, nn, lo, hi, ntiles, tileS, tileN,
+                                           counter, st);
+                break;
+            }
+        } else if (dense) {
             const int nrt = (hi - lo + kGThreads - 1) / kGThreads;
             const int nbc = (m + kGB - 1) / kGB;
             gauss_kernel<<<nrt * nbc, kGThreads, 0, st>>>(xy, nn, d_h, m, lo, hi, nbc, ntiles, tileS, tileN);

@@ -138,7 +138,8 @@ extern "C" int kr_cv_grid_algo(const double *x, const double *y, int64_t n, cons
                                int32_t *best_out)
 {
     if (!cv_out || !best_out) return KR_EARG;
-    if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX && algo != KR_ALGO_DENSE)
+    if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX && algo != KR_ALGO_DENSE &&
+        algo != KR_ALGO_HIST)
         return KR_EARG;
     int st = validate_all(x, y, n, h_grid, m, kernel);
     if (st) return st;
@@ -240,7 +241,8 @@ extern "C" int kr_cv_refine(const double *x, const double *y, int64_t n, const d
 {
     if (!h_best_out || !cv_best_out || levels < 1 || levels > 64) return KR_EARG;
     if (levels > 1 && (m_fine < 3 || m_fine > KR_MAX_M)) return KR_EARG;
-    if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX && algo != KR_ALGO_DENSE)
+    if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX && algo != KR_ALGO_DENSE &&
+        algo != KR_ALGO_HIST)
         return KR_EARG;
     int st = validate_all(x, y, n, h_grid, m, kernel);
     if (st) return st;

@@ -22,6 +22,7 @@ struct WsLayout {
     size_t vals_in, vals_out;   // uint32 [n]  original indices
     size_t xy;                  // double2 [n + 2 kPad] (x, y) in sorted order, +-inf sentinels
     size_t counter;             // int: sweep tile counter
+    size_t perm;                // uint32 [n]  original index of each sorted record (histogram path)
     size_t tileS;               // double  [m][ntiles]  per-tile sum of M e^2
     size_t tileN;               // uint8   [m][ntiles]  per-tile sum of M
     size_t tileB;               // double  [m][ceil(n/32)] per-tile KDE sum B (tileS holds A)

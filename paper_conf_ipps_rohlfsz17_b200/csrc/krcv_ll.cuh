@@ -25,8 +25,9 @@
 // Accuracy: the prefix differences and the shift carry an absolute error
 // bounded by kappa * mag_k (kappa = (n + 64) 2^-104 covers the prefix
 // build's accumulated dd rounding, mag_k = the binomial combination of the
-// prefix magnitudes); propagated through S, T, det and num it bounds the
-// error of g.  If the bound is not below 2^-44 max|y| (or the window is small,
+// prefix magnitudes); S, T, det = S0 S2 - S1^2 and num = S2 T0 - S1 T1
+// stay in dd (det cancels badly when the window sits far to one side of the
+// row: tail rows at large h), and the propagated bound covers g.  If the bound is not below 2^-44 max|y| (or the window is small,
 // c <= kLLDirect, where the direct loop is cheaper anyway) g is computed
 // directly over the window in the centred two-pass form.
 #pragma once
@@ -81,16 +82,14 @@ __device__ double ll_direct(const double2 *__restrict__ xy, int A, int R, int r,
     return ybar - dbar * (sdy / sdd);
 }
 
-// Shifted power sums over [a, b): D[k] = sum (u - delta)^k (k = 1..DU) and
-// Y[k] = sum y (u - delta)^k (k = 0..DY; Y[0] minus ysub, subtracted in dd),
-// rounded to double, with absolute error bounds
-// eD[k], eY[k] = kappa sum_i C(k,i) |delta|^(k-i) (|P_i[a]| + |P_i[b]|)
-//              + 2^-52 |value| (the final rounding, generously).
+// Shifted power sums over [a, b) in dd: D[k] = sum (u - delta)^k
+// (k = 1..DU) and Y[k] = sum y (u - delta)^k (k = 0..DY; Y[0] minus ysub),
+// with absolute error bounds
+// eD[k], eY[k] = kappa sum_i C(k,i) |delta|^(k-i) (|P_i[a]| + |P_i[b]|).
 // Slots (kLLMoments): 0 y, 1 u, 2 u^2, 3 u^3, 4 u^4, 5 y u, 6 y u^2, 7 y u^3.
 template <int DU, int DY>
 __device__ __forceinline__ void ll_shift(const double *__restrict__ P, int ps, int a, int b, dd del, double ysub,
-                                         double kappa, double (&D)[5], double (&Y)[4], double (&eD)[5],
-                                         double (&eY)[4])
+                                         double kappa, dd (&D)[5], dd (&Y)[4], double (&eD)[5], double (&eY)[4])
 {
     const dd e = dd_neg(del);
     const double ad = fabs(del.hi);
@@ -123,8 +122,8 @@ __device__ __forceinline__ void ll_shift(const double *__restrict__ P, int ps, i
             acc = dd_add(dd_mul_d_raw(Mu[i], cb), dd_mul_raw(e, acc));
             mag = fma(cb, au[i], ad * mag);
         }
-        D[k] = dd_to_d(acc);
-        eD[k] = fma(kappa, mag, 0x1p-52 * fabs(D[k]));
+        D[k] = acc;
+        eD[k] = kappa * mag;
     }
 #pragma unroll
     for (int k = 0; k <= DY; k++) {
@@ -138,78 +137,94 @@ __device__ __forceinline__ void ll_shift(const double *__restrict__ P, int ps, i
             mag = fma(cb, ay[i], ad * mag);
         }
         if (k == 0) acc = dd_add_d(acc, -ysub);
-        Y[k] = dd_to_d(acc);
-        eY[k] = fma(kappa, mag, 0x1p-52 * fabs(Y[k]));
+        Y[k] = acc;
+        eY[k] = kappa * mag;
     }
 }
 
+// H a - b in dd (H, a, b dd): the S_k / T_k of the weighted sums
+__device__ __forceinline__ dd ll_comb(dd H, dd a, dd b) { return dd_sub(dd_mul(H, a), b); }
+
 // Local-linear g for row r, window [A, R) (c = R - A - 1 >= 2 points besides
-// r, at least two distinct x).  Returns g.
+// r, at least two distinct x).  S_k, T_k, det and num stay in dd; the error
+// bounds eS, eT propagate the prefix errors, and dd rounding adds
+// 2^-100 of the magnitudes combined.  Returns g.
 template <int KERN>
 __device__ __forceinline__ double ll_estimate(const WinRow &w, int A, int R, int c, double h,
                                               const double2 *__restrict__ xy, const double *__restrict__ P, int ps,
-                                              double ymax, double kappa)
+                                              double ymax, double kappa,
+                                              unsigned long long *__restrict__ stats)
 {
     const int r = w.r;
-    if (c <= kLLDirect) return ll_direct<KERN>(xy, A, R, r, w.xr, h);
-    // S0..S2, T0, T1 and absolute error bounds eS*, eT*
-    double S0, S1, S2, T0, T1, eS0, eS1, eS2, eT0, eT1;
+    if (c <= kLLDirect) {
+        if (stats) atomicAdd(stats + 0, 1ull);
+        return ll_direct<KERN>(xy, A, R, r, w.xr, h);
+    }
+    dd S0, S1, S2, T0, T1;
+    double eS0, eS1, eS2, eT0, eT1;
+    const dd cc = dd_make((double)c);
     if (KERN != KR_TRIANGULAR) {
-        double D[5], Y[4], eD[5], eY[4];
-        D[0] = (double)c;
-        eD[0] = 0.0;
+        dd D[5], Y[4];
+        double eD[5], eY[4];
         // row r is inside [A, R): its d-terms vanish, its y leaves Y_0 (LOO)
         if (KERN == KR_UNIFORM) {
             ll_shift<2, 1>(P, ps, A, R, w.del, w.yr, kappa, D, Y, eD, eY);
-        } else {
-            ll_shift<4, 3>(P, ps, A, R, w.del, w.yr, kappa, D, Y, eD, eY);
-        }
-        if (KERN == KR_UNIFORM) {
-            S0 = (double)c; S1 = D[1]; S2 = D[2]; T0 = Y[0]; T1 = Y[1];
+            S0 = cc; S1 = D[1]; S2 = D[2]; T0 = Y[0]; T1 = Y[1];
             eS0 = 0.0; eS1 = eD[1]; eS2 = eD[2]; eT0 = eY[0]; eT1 = eY[1];
         } else {
-            const double hh = h * h;  // rounded: <= 2^-53 relative, bounded below
-            S0 = fma(hh, (double)c, -D[2]);
-            S1 = fma(hh, D[1], -D[3]);
-            S2 = fma(hh, D[2], -D[4]);
-            T0 = fma(hh, Y[0], -Y[2]);
-            T1 = fma(hh, Y[1], -Y[3]);
-            const double q = 0x1p-52 * hh;  // hh's own rounding
-            eS0 = fma(q, (double)c, eD[2]);
-            eS1 = fma(hh, eD[1], fma(q, fabs(D[1]), eD[3]));
-            eS2 = fma(hh, eD[2], fma(q, fabs(D[2]), eD[4]));
-            eT0 = fma(hh, eY[0], fma(q, fabs(Y[0]), eY[2]));
-            eT1 = fma(hh, eY[1], fma(q, fabs(Y[1]), eY[3]));
+            ll_shift<4, 3>(P, ps, A, R, w.del, w.yr, kappa, D, Y, eD, eY);
+            const dd H = two_prod(h, h);  // h^2 exactly
+            const double hh = H.hi;
+            S0 = ll_comb(H, cc, D[2]);
+            S1 = ll_comb(H, D[1], D[3]);
+            S2 = ll_comb(H, D[2], D[4]);
+            T0 = ll_comb(H, Y[0], Y[2]);
+            T1 = ll_comb(H, Y[1], Y[3]);
+            eS0 = eD[2];
+            eS1 = fma(hh, eD[1], eD[3]);
+            eS2 = fma(hh, eD[2], eD[4]);
+            eT0 = fma(hh, eY[0], eY[2]);
+            eT1 = fma(hh, eY[1], eY[3]);
         }
     } else {
-        double DR[5], YR[4], eDR[5], eYR[4], DL[5], YL[4], eDL[5], eYL[4];
+        dd DR[5], YR[4], DL[5], YL[4];
+        double eDR[5], eYR[4], eDL[5], eYL[4];
         ll_shift<3, 2>(P, ps, r + 1, R, w.del, 0.0, kappa, DR, YR, eDR, eYR);  // row r in neither part
         ll_shift<3, 2>(P, ps, A, r, w.del, 0.0, kappa, DL, YL, eDL, eYL);
         // right d = |d|, left d = -|d|: sum |d|^k = DR_k + (-1)^k DL_k
-        S0 = fma(h, (double)c, -(DR[1] - DL[1]));
-        S1 = fma(h, DR[1] + DL[1], -(DR[2] - DL[2]));
-        S2 = fma(h, DR[2] + DL[2], -(DR[3] - DL[3]));
-        T0 = fma(h, YR[0] + YL[0], -(YR[1] - YL[1]));
-        T1 = fma(h, YR[1] + YL[1], -(YR[2] - YL[2]));
+        const dd H = dd_make(h);
+        S0 = ll_comb(H, cc, dd_sub(DR[1], DL[1]));
+        S1 = ll_comb(H, dd_add(DR[1], DL[1]), dd_sub(DR[2], DL[2]));
+        S2 = ll_comb(H, dd_add(DR[2], DL[2]), dd_sub(DR[3], DL[3]));
+        T0 = ll_comb(H, dd_add(YR[0], YL[0]), dd_sub(YR[1], YL[1]));
+        T1 = ll_comb(H, dd_add(YR[1], YL[1]), dd_sub(YR[2], YL[2]));
         eS0 = eDR[1] + eDL[1];
         eS1 = fma(h, eDR[1] + eDL[1], eDR[2] + eDL[2]);
         eS2 = fma(h, eDR[2] + eDL[2], eDR[3] + eDL[3]);
         eT0 = fma(h, eYR[0] + eYL[0], eYR[1] + eYL[1]);
         eT1 = fma(h, eYR[1] + eYL[1], eYR[2] + eYL[2]);
     }
-    // det and num in dd (the products cancel when the window is narrow
-    // relative to its offset from the row)
-    const dd det = dd_sub(two_prod(S0, S2), two_prod(S1, S1));
-    const dd num = dd_sub(two_prod(S2, T0), two_prod(S1, T1));
+    // det = S0 S2 - S1^2 and num = S2 T0 - S1 T1 in dd (they cancel when the
+    // window sits far to one side of the row)
+    const dd det = dd_sub(dd_mul(S0, S2), dd_mul(S1, S1));
+    const dd num = dd_sub(dd_mul(S2, T0), dd_mul(S1, T1));
     const double dt = dd_to_d(det), nm = dd_to_d(num);
     const double g = nm / dt;
-    const double aS0 = fabs(S0), aS1 = fabs(S1), aS2 = fabs(S2);
-    const double eps = 0x1p-52;  // rounding of the fma forming S, T
-    const double fS0 = fma(eps, aS0, eS0), fS1 = fma(eps, aS1, eS1), fS2 = fma(eps, aS2, eS2);
-    const double fT0 = fma(eps, fabs(T0), eT0), fT1 = fma(eps, fabs(T1), eT1);
-    const double edet = aS2 * fS0 + aS0 * fS2 + 2.0 * aS1 * fS1 + fS0 * fS2 + fS1 * fS1;
-    const double enum_ = aS2 * fT0 + fabs(T0) * fS2 + aS1 * fT1 + fabs(T1) * fS1 + fS2 * fT0 + fS1 * fT1;
+    // first-order propagation of eS, eT plus dd rounding (2^-100 relative to
+    // the products, generously)
+    const double aS0 = fabs(S0.hi), aS1 = fabs(S1.hi), aS2 = fabs(S2.hi);
+    const double aT0 = fabs(T0.hi), aT1 = fabs(T1.hi);
+    const double q = 0x1p-100;
+    const double fS0 = fma(q, aS0, eS0), fS1 = fma(q, aS1, eS1), fS2 = fma(q, aS2, eS2);
+    const double fT0 = fma(q, aT0, eT0), fT1 = fma(q, aT1, eT1);
+    const double edet = aS2 * fS0 + aS0 * fS2 + 2.0 * aS1 * fS1 + fS0 * fS2 + fS1 * fS1 + q * (aS0 * aS2 + aS1 * aS1);
+    const double enum_ =
+        aS2 * fT0 + aT0 * fS2 + aS1 * fT1 + aT1 * fS1 + fS2 * fT0 + fS1 * fT1 + q * (aS2 * aT0 + aS1 * aT1);
     const bool ok = dt > 0.0 && edet <= 0x1p-20 * dt && fma(fabs(g), edet, enum_) <= 0x1p-44 * dt * ymax;
+    if (stats) {
+        atomicAdd(stats + (ok ? 1 : 2), 1ull);
+        if (!ok) atomicAdd(stats + 3, (unsigned long long)c);
+    }
     if (ok) return g;
     return ll_direct<KERN>(xy, A, R, r, w.xr, h);
 }
@@ -217,12 +232,15 @@ __device__ __forceinline__ double ll_estimate(const WinRow &w, int A, int R, int
 // A warp owns 32 consecutive sorted rows (one per lane) and a chunk of the
 // bandwidth loop, as window_kernel<KERN, 1>; output in the same tile-partial
 // layout (reduce_kernel and the finalize are shared with Nadaraya-Watson).
+// stats (debug, nullable): counts of direct / prefix-accepted / prefix-
+// rejected (row, bandwidth) evaluations and the rejected windows' total size.
 template <int KERN>
 __global__ void __launch_bounds__(kWinThreads)
 ll_window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
                  int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
                  int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
-                 uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
+                 uint8_t *__restrict__ tileN, int *__restrict__ tile_counter,
+                 unsigned long long *__restrict__ stats)
 {
     const int lane = threadIdx.x & 31;
     const double o = pfx_origin(xy, n);
@@ -265,7 +283,7 @@ ll_window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, 
                 const int first = A == row.r ? A + 1 : A;
                 const int last = R - 1 == row.r ? R - 2 : R - 1;
                 if (xs[first] != xs[last]) {
-                    const double g = ll_estimate<KERN>(row, A, R, c, h, xy, P, ps, ymax, kappa);
+                    const double g = ll_estimate<KERN>(row, A, R, c, h, xy, P, ps, ymax, kappa, stats);
                     const double e = row.yr - g;
                     e2 = e * e;
                     cntM = 1;

@@ -160,7 +160,7 @@ rank_count_kernel(const uint64_t *__restrict__ keys, const uint32_t *__restrict_
 __global__ void __launch_bounds__(256)
 rank_scatter_kernel(const uint32_t *__restrict__ idx, const int *__restrict__ rank, int n, int npad,
                     const double *__restrict__ x, const double *__restrict__ y, double2 *__restrict__ xy,
-                    int *__restrict__ tile_counter)
+                    uint32_t *__restrict__ perm, int *__restrict__ tile_counter)
 {
     const int g = blockIdx.x * blockDim.x + threadIdx.x;
     if (g < kPad) {
@@ -170,7 +170,11 @@ rank_scatter_kernel(const uint32_t *__restrict__ idx, const int *__restrict__ ra
     if (g == 0) *tile_counter = 0;
     if (g >= npad) return;
     const uint32_t i = idx[g];
-    if (i < (uint32_t)n) xy[rank[g]] = make_double2(x[i], y[i]);
+    if (i < (uint32_t)n) {
+        const int r = rank[g];
+        xy[r] = make_double2(x[i], y[i]);
+        perm[r] = i;  // sorted position -> original index (histogram path's self test)
+    }
 }
 
 }  // namespace krcv

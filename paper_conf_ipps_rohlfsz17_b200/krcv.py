@@ -25,8 +25,8 @@ LIB_PATH = os.path.join(_HERE, "libkrcv.so")
 UNIFORM, EPANECHNIKOV, TRIANGULAR, GAUSSIAN = 0, 1, 2, 3
 KERNELS = {"uniform": UNIFORM, "epanechnikov": EPANECHNIKOV, "triangular": TRIANGULAR, "gaussian": GAUSSIAN}
 
-ALGO_AUTO, ALGO_SWEEP, ALGO_PREFIX, ALGO_DENSE = 0, 1, 2, 3
-ALGOS = {"auto": ALGO_AUTO, "sweep": ALGO_SWEEP, "prefix": ALGO_PREFIX, "dense": ALGO_DENSE}
+ALGO_AUTO, ALGO_SWEEP, ALGO_PREFIX, ALGO_DENSE, ALGO_HIST = 0, 1, 2, 3, 4
+ALGOS = {"auto": ALGO_AUTO, "sweep": ALGO_SWEEP, "prefix": ALGO_PREFIX, "dense": ALGO_DENSE, "hist": ALGO_HIST}
 
 KR_OK, KR_EARG, KR_EKERNEL, KR_EGRID, KR_ENONFINITE, KR_EDEGENERATE, KR_ENOMEM, KR_ECUDA = range(8)
 KR_MAX_M = 65536
