@@ -113,8 +113,14 @@ enum {
  *   kernel   KR_UNIFORM | KR_EPANECHNIKOV | KR_TRIANGULAR
  *   cv_out   [m] host: CV(h_b) per Eq.(1) (already divided by n)
  *   best_out host: smallest arg-min index
- * Errors: KR_EARG, KR_EKERNEL, KR_EGRID, KR_ENONFINITE (validated on the host
- * before any device work), KR_ENOMEM, KR_ECUDA.  Outputs untouched on error.
+ * Errors: KR_EARG, KR_EKERNEL, KR_EGRID (arguments and grid validated on the
+ * host before any device work), KR_ENONFINITE (NaN / Inf in x or y, counted
+ * on the device by the pack / sort kernels), KR_ENOMEM, KR_ECUDA.  Outputs
+ * untouched on error.
+ * Repeat calls with the same pinned (cudaMallocHost / cudaHostRegister) x, y,
+ * h_grid pointers, n, m, kernel and algorithm replay a CUDA graph of the
+ * whole call (H2D copies, device pipeline, D2H copies) captured on the first
+ * such call; the copies read the buffers' current contents.
  */
 int kr_cv_grid(const double *x, const double *y, int64_t n,
                const double *h_grid, int32_t m, int32_t kernel,

@@ -235,7 +235,7 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     L->counter = off;  off = align256(off + sizeof(int));
     L->perm = off;     off = align256(off + sizeof(uint32_t) * (size_t)n);
     // window-prefix path (krcv_prefix.cuh)
-    const size_t nch = (size_t)((n + kPfxTile) / kPfxTile);  // tiles covering P[0..n]
+    const size_t nch = (size_t)((n + kPfxTileMin) / kPfxTileMin);  // most tiles covering P[0..n]
     L->pstride = (int64_t)(((size_t)n + 1 + 15) & ~size_t(15));
     L->nch = (int64_t)nch;
     L->xs = off;       off = align256(off + sizeof(double) * ((size_t)n + 2 * kPad));
@@ -369,6 +369,8 @@ struct Prof {
 };
 static thread_local Prof g_prof;
 
+bool prof_enabled() { return g_prof.on; }
+
 static void prof_mark(int k, cudaStream_t st)
 {
     if (!g_prof.on) return;
@@ -420,6 +422,20 @@ int auto_algo(int64_t /*n*/, int64_t /*rows*/, int32_t /*m*/, int32_t /*kernel*/
     return forced ? forced : KR_ALGO_PREFIX;
 }
 
+// Records per thread of the prefix build: 1 (256-record tiles, more CTAs)
+// up to 2^18 records, 4 above.  KRCV_PFX_ITEMS=1|4 overrides.
+static int pfx_items(int n)
+{
+    static int forced = -1;
+    if (forced < 0) {
+        const char *e = getenv("KRCV_PFX_ITEMS");
+        forced = e ? atoi(e) : 0;
+        if (forced != 1 && forced != 4) forced = 0;
+    }
+    if (forced) return forced;
+    return n <= (1 << 18) ? 1 : kPfxItemsMax;
+}
+
 template <int KERN>
 static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, char *ws, cudaStream_t st)
 {
@@ -427,9 +443,16 @@ static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, cha
     double *P = reinterpret_cast<double *>(ws + L.pfx);
     double2 *tot = reinterpret_cast<double2 *>(ws + L.ptot);
     unsigned long long *ymax = reinterpret_cast<unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
-    const int ntiles = (int)L.nch;
-    pfx_tile_reduce_kernel<KERN><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, ymax);
-    pfx_tile_scan_kernel<KERN><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, P, (int)L.pstride, xs);
+    if (pfx_items(n) == 1) {
+        const int ntiles = (n + kPfxThreads) / kPfxThreads;  // tiles covering P[0..n]
+        pfx_tile_reduce_kernel<KERN, 1><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, ymax);
+        pfx_tile_scan_kernel<KERN, 1><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, P, (int)L.pstride, xs);
+    } else {
+        const int ntiles = (n + kPfxThreads * kPfxItemsMax) / (kPfxThreads * kPfxItemsMax);
+        pfx_tile_reduce_kernel<KERN, kPfxItemsMax><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, ymax);
+        pfx_tile_scan_kernel<KERN, kPfxItemsMax><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, P,
+                                                                                 (int)L.pstride, xs);
+    }
 }
 
 // Rows per lane of the window kernel (K consecutive rows; rows 2..K advance

@@ -43,6 +43,18 @@ struct DevCtx {
     double *dpartial = nullptr, *dcv = nullptr;
     int64_t *dneff = nullptr;
     int32_t *dbest = nullptr;  // [2]: best, status
+    // pinned staging for the results of the synchronous host path
+    double *pcv = nullptr;
+    int64_t *pneff = nullptr;
+    int32_t *pbs = nullptr;
+    int32_t pcap_m = 0;
+    // CUDA graph of the last synchronous call whose inputs were pinned
+    // (H2D copies, the whole device pipeline, D2H copies): replayed while
+    // the pointers, sizes, kernel, algorithm and estimator repeat
+    cudaGraphExec_t gexec = nullptr;
+    const void *gx = nullptr, *gy = nullptr, *gh = nullptr;
+    int64_t gn = 0;
+    int32_t gm = 0, gkernel = -1, galgo = -1, gll = -1;
 };
 
 static std::mutex g_ctx_mu;
@@ -126,10 +138,122 @@ static int validate_all(const double *x, const double *y, int64_t n, const doubl
     if (!x || !y || !h) return KR_EARG;
     if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return KR_EARG;
     if (!kernel_ok(kernel)) return KR_EKERNEL;
-    int st = kr_validate_grid(h, m);
+    // x, y are checked for NaN / Inf on the device (the pack / chunk-sort
+    // kernels count them into the status word, and the call returns
+    // KR_ENONFINITE with the outputs untouched): a host scan would cost more
+    // than the whole C2 search's H2D copy
+    return kr_validate_grid(h, m);
+}
+
+static bool is_pinned(const void *p)
+{
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeHost;
+}
+
+static int ensure_staging(DevCtx *c, int32_t m)
+{
+    if (m <= c->pcap_m) return KR_OK;
+    cudaFreeHost(c->pcv);
+    cudaFreeHost(c->pneff);
+    cudaFreeHost(c->pbs);
+    c->pcv = nullptr;
+    c->pneff = nullptr;
+    c->pbs = nullptr;
+    c->pcap_m = 0;
+    KR_CUDA_TRY(cudaMallocHost(&c->pcv, sizeof(double) * m));
+    KR_CUDA_TRY(cudaMallocHost(&c->pneff, sizeof(int64_t) * m));
+    KR_CUDA_TRY(cudaMallocHost(&c->pbs, sizeof(int32_t) * 2));
+    c->pcap_m = m;
+    return KR_OK;
+}
+
+// H2D of the inputs, the whole device search (Nadaraya-Watson or
+// local-linear), D2H of the results into the pinned staging -- all enqueued
+// on c->stream.
+static int enqueue_host_call(DevCtx *c, const double *x, const double *y, int64_t n, const double *h, int32_t m,
+                             int32_t kernel, int32_t algo, bool ll)
+{
+    cudaStream_t s = c->stream;
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dx, x, sizeof(double) * n, cudaMemcpyHostToDevice, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dy, y, sizeof(double) * n, cudaMemcpyHostToDevice, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dh, h, sizeof(double) * m, cudaMemcpyHostToDevice, s));
+    const int st = ll ? kr_ll_cv_grid_async(c->dx, c->dy, n, c->dh, m, kernel, c->dcv, c->dneff, c->dbest, c->ws,
+                                            c->ws_bytes, s)
+                      : kr_cv_grid_async(c->dx, c->dy, n, c->dh, m, kernel, algo, c->dcv, c->dneff, c->dbest, c->ws,
+                                         c->ws_bytes, s);
     if (st) return st;
-    for (int64_t i = 0; i < n; i++)
-        if (!std::isfinite(x[i]) || !std::isfinite(y[i])) return KR_ENONFINITE;
+    KR_CUDA_TRY(cudaMemcpyAsync(c->pcv, c->dcv, sizeof(double) * m, cudaMemcpyDeviceToHost, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(c->pneff, c->dneff, sizeof(int64_t) * m, cudaMemcpyDeviceToHost, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(c->pbs, c->dbest, sizeof(int32_t) * 2, cudaMemcpyDeviceToHost, s));
+    return KR_OK;
+}
+
+// The synchronous host-pointer path shared by kr_cv_grid* and kr_ll_cv_grid.
+// With pinned x, y, h (and profiling off) the enqueued sequence is captured
+// once as a CUDA graph and replayed on repeat calls -- one launch instead of
+// ~13 API calls; the copies read the caller's buffers at replay time.
+static int host_call(const double *x, const double *y, int64_t n, const double *h, int32_t m, int32_t kernel,
+                     int32_t algo, bool ll, double *cv_out, int64_t *neff_out, int32_t *best_out)
+{
+    int dev = 0;
+    KR_CUDA_TRY(cudaGetDevice(&dev));
+    DevCtx *c = get_ctx(dev);
+    std::lock_guard<std::mutex> g(c->mu);
+    int st = ensure_capacity(c, n, m);
+    if (st) return st;
+    st = ensure_staging(c, m);
+    if (st) return st;
+    cudaStream_t s = c->stream;
+    const bool graph = !prof_enabled() && is_pinned(x) && is_pinned(y) && is_pinned(h);
+    if (graph) {
+        const bool same = c->gexec && c->gx == x && c->gy == y && c->gh == h && c->gn == n && c->gm == m &&
+                          c->gkernel == kernel && c->galgo == algo && c->gll == (ll ? 1 : 0);
+        if (!same) {
+            if (c->gexec) cudaGraphExecDestroy(c->gexec);
+            c->gexec = nullptr;
+            KR_CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+            st = enqueue_host_call(c, x, y, n, h, m, kernel, algo, ll);
+            cudaGraph_t gr = nullptr;
+            const cudaError_t e = cudaStreamEndCapture(s, &gr);
+            if (st) {
+                if (gr) cudaGraphDestroy(gr);
+                return st;
+            }
+            if (e != cudaSuccess) {
+                set_cuda_error("cudaStreamEndCapture", (int)e);
+                return KR_ECUDA;
+            }
+            const cudaError_t e2 = cudaGraphInstantiate(&c->gexec, gr, 0);
+            cudaGraphDestroy(gr);
+            if (e2 != cudaSuccess) {
+                c->gexec = nullptr;
+                set_cuda_error("cudaGraphInstantiate", (int)e2);
+                return KR_ECUDA;
+            }
+            c->gx = x;
+            c->gy = y;
+            c->gh = h;
+            c->gn = n;
+            c->gm = m;
+            c->gkernel = kernel;
+            c->galgo = algo;
+            c->gll = ll ? 1 : 0;
+        }
+        KR_CUDA_TRY(cudaGraphLaunch(c->gexec, s));
+    } else {
+        st = enqueue_host_call(c, x, y, n, h, m, kernel, algo, ll);
+        if (st) return st;
+    }
+    KR_CUDA_TRY(cudaStreamSynchronize(s));
+    if (c->pbs[1] != KR_OK) return c->pbs[1];
+    std::memcpy(cv_out, c->pcv, sizeof(double) * m);
+    if (neff_out) std::memcpy(neff_out, c->pneff, sizeof(int64_t) * m);
+    *best_out = c->pbs[0];
     return KR_OK;
 }
 
@@ -141,68 +265,19 @@ extern "C" int kr_cv_grid_algo(const double *x, const double *y, int64_t n, cons
     if (algo != KR_ALGO_AUTO && algo != KR_ALGO_SWEEP && algo != KR_ALGO_PREFIX && algo != KR_ALGO_DENSE &&
         algo != KR_ALGO_HIST)
         return KR_EARG;
-    int st = validate_all(x, y, n, h_grid, m, kernel);
+    const int st = validate_all(x, y, n, h_grid, m, kernel);
     if (st) return st;
-    int dev = 0;
-    KR_CUDA_TRY(cudaGetDevice(&dev));
-    DevCtx *c = get_ctx(dev);
-    std::lock_guard<std::mutex> g(c->mu);
-    st = ensure_capacity(c, n, m);
-    if (st) return st;
-    cudaStream_t s = c->stream;
-    KR_CUDA_TRY(cudaMemcpyAsync(c->dx, x, sizeof(double) * n, cudaMemcpyHostToDevice, s));
-    KR_CUDA_TRY(cudaMemcpyAsync(c->dy, y, sizeof(double) * n, cudaMemcpyHostToDevice, s));
-    KR_CUDA_TRY(cudaMemcpyAsync(c->dh, h_grid, sizeof(double) * m, cudaMemcpyHostToDevice, s));
-    st = kr_cv_grid_async(c->dx, c->dy, n, c->dh, m, kernel, algo, c->dcv, c->dneff, c->dbest, c->ws, c->ws_bytes,
-                          s);
-    if (st) return st;
-    std::vector<double> cv(m);
-    std::vector<int64_t> ne(neff_out ? m : 0);
-    int32_t bs[2] = {0, 0};
-    KR_CUDA_TRY(cudaMemcpyAsync(cv.data(), c->dcv, sizeof(double) * m, cudaMemcpyDeviceToHost, s));
-    if (neff_out)
-        KR_CUDA_TRY(cudaMemcpyAsync(ne.data(), c->dneff, sizeof(int64_t) * m, cudaMemcpyDeviceToHost, s));
-    KR_CUDA_TRY(cudaMemcpyAsync(bs, c->dbest, sizeof(int32_t) * 2, cudaMemcpyDeviceToHost, s));
-    KR_CUDA_TRY(cudaStreamSynchronize(s));
-    if (bs[1] != KR_OK) return bs[1];
-    std::memcpy(cv_out, cv.data(), sizeof(double) * m);
-    if (neff_out) std::memcpy(neff_out, ne.data(), sizeof(int64_t) * m);
-    *best_out = bs[0];
-    return KR_OK;
+    return host_call(x, y, n, h_grid, m, kernel, algo, false, cv_out, neff_out, best_out);
 }
 
 extern "C" int kr_ll_cv_grid(const double *x, const double *y, int64_t n, const double *h_grid, int32_t m,
                              int32_t kernel, double *cv_out, int64_t *neff_out, int32_t *best_out)
 {
     if (!cv_out || !best_out) return KR_EARG;
-    int st = validate_all(x, y, n, h_grid, m, kernel);
+    const int st = validate_all(x, y, n, h_grid, m, kernel);
     if (st) return st;
     if (kernel == KR_GAUSSIAN) return KR_EKERNEL;
-    int dev = 0;
-    KR_CUDA_TRY(cudaGetDevice(&dev));
-    DevCtx *c = get_ctx(dev);
-    std::lock_guard<std::mutex> g(c->mu);
-    st = ensure_capacity(c, n, m);
-    if (st) return st;
-    cudaStream_t s = c->stream;
-    KR_CUDA_TRY(cudaMemcpyAsync(c->dx, x, sizeof(double) * n, cudaMemcpyHostToDevice, s));
-    KR_CUDA_TRY(cudaMemcpyAsync(c->dy, y, sizeof(double) * n, cudaMemcpyHostToDevice, s));
-    KR_CUDA_TRY(cudaMemcpyAsync(c->dh, h_grid, sizeof(double) * m, cudaMemcpyHostToDevice, s));
-    st = kr_ll_cv_grid_async(c->dx, c->dy, n, c->dh, m, kernel, c->dcv, c->dneff, c->dbest, c->ws, c->ws_bytes, s);
-    if (st) return st;
-    std::vector<double> cv(m);
-    std::vector<int64_t> ne(neff_out ? m : 0);
-    int32_t bs[2] = {0, 0};
-    KR_CUDA_TRY(cudaMemcpyAsync(cv.data(), c->dcv, sizeof(double) * m, cudaMemcpyDeviceToHost, s));
-    if (neff_out)
-        KR_CUDA_TRY(cudaMemcpyAsync(ne.data(), c->dneff, sizeof(int64_t) * m, cudaMemcpyDeviceToHost, s));
-    KR_CUDA_TRY(cudaMemcpyAsync(bs, c->dbest, sizeof(int32_t) * 2, cudaMemcpyDeviceToHost, s));
-    KR_CUDA_TRY(cudaStreamSynchronize(s));
-    if (bs[1] != KR_OK) return bs[1];
-    std::memcpy(cv_out, cv.data(), sizeof(double) * m);
-    if (neff_out) std::memcpy(neff_out, ne.data(), sizeof(int64_t) * m);
-    *best_out = bs[0];
-    return KR_OK;
+    return host_call(x, y, n, h_grid, m, kernel, KR_ALGO_PREFIX, true, cv_out, neff_out, best_out);
 }
 
 extern "C" int kr_cv_grid_ex(const double *x, const double *y, int64_t n, const double *h_grid, int32_t m,

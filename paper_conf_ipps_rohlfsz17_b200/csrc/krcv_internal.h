@@ -49,6 +49,11 @@ int enqueue_grid(const double *d_x, const double *d_y, int64_t n, const double *
                  int32_t algo, double *d_cv, int64_t *d_neff, int32_t *d_best_status, void *d_workspace,
                  size_t workspace_bytes, void *cuda_stream, bool reuse_sorted);
 
+// True while kr_profile_enable(1) is in effect on this thread (the stage
+// events must be recorded on a stream, so the host path does not replay a
+// captured graph then).
+bool prof_enabled();
+
 // Records a CUDA error string for kr_last_cuda_error (thread-local).
 void set_cuda_error(const char *what, int code);
 

@@ -28,7 +28,7 @@
 // row, so a grid search costs O(n m log) instead of O(n^2).
 //
 // Kernels:
-//   pfx_tile_reduce_kernel  per tile of kPfxTile sorted records: moment terms
+//   pfx_tile_reduce_kernel  per tile of 256 ITEMS sorted records: moment terms
 //                           and their dd totals
 //   pfx_tile_scan_kernel    per tile: its offset (fixed-order sum of the
 //                           earlier tiles' totals), prefix values P[k][0..n]
@@ -55,7 +55,7 @@ constexpr int kPfxThreads = 256;      // prefix build CTA
 constexpr int kPfxMoments = 8;        // slots reserved in the workspace (local-linear uses all 8)
 constexpr int kWinWarps = 4;
 constexpr int kWinThreads = kWinWarps * 32;
-constexpr int kWinTasksPerSM = 64;    // warp tasks per SM the b-split aims for
+constexpr int kWinTasksPerSM = 256;   // warp tasks per SM the b-split aims for (measured: C3 nbc 7 -> 28, -9 %)
 constexpr int kWinMinBper = 8;        // >= this many bandwidths per task
 
 // Moments per kernel (slot order).  Epanechnikov: y, u, u^2, y u, y u^2.
@@ -122,10 +122,13 @@ __device__ __forceinline__ double pfx_origin(const double2 *xy, int n) { return 
 // ---------------------------------------------------------------- build
 // Two-phase fixed-order scan (bit-reproducible; a decoupled look-back
 // would make the dd rounding depend on timing): tile totals, then every tile
-// sums its predecessors' totals itself and scans its records.  A tile is kPfxTile sorted
-// records; thread t of its CTA owns records 4t .. 4t+3 of the tile.
-constexpr int kPfxItems = 4;
-constexpr int kPfxTile = kPfxThreads * kPfxItems;
+// sums its predecessors' totals itself and scans its records.  A tile is
+// 256 ITEMS sorted records; thread t of its CTA owns records ITEMS t ..
+// ITEMS t + ITEMS - 1 of the tile.  ITEMS = 4 (tile 1,024) for large n, 1
+// (tile 256) for small n so that the scan spreads over more CTAs
+// (pfx_items() in krcv_device.cu).
+constexpr int kPfxItemsMax = 4;
+constexpr int kPfxTileMin = kPfxThreads;  // the workspace sizes tile totals for this
 
 __device__ __forceinline__ dd shfl_up_dd(dd v, int d)
 {
@@ -138,7 +141,7 @@ __device__ __forceinline__ dd shfl_xor_dd(dd v, int d)
 }
 
 // Phase 1: per-tile totals of the moment terms -> tot[k][tile].
-template <int KERN>
+template <int KERN, int ITEMS>
 __global__ void __launch_bounds__(kPfxThreads)
 pfx_tile_reduce_kernel(const double2 *__restrict__ xy, int n, double2 *__restrict__ tot, int ntiles,
                        unsigned long long *__restrict__ ymax_bits)
@@ -146,14 +149,14 @@ pfx_tile_reduce_kernel(const double2 *__restrict__ xy, int n, double2 *__restric
     constexpr int K = NMom<KERN>::v;
     __shared__ double2 wsum[K][kPfxThreads / 32];
     const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-    const int j0 = blockIdx.x * kPfxTile + t * kPfxItems;
+    const int j0 = blockIdx.x * (kPfxThreads * ITEMS) + t * ITEMS;
     const double o = pfx_origin(xy, n);
     dd acc[kPfxMoments];
 #pragma unroll
     for (int k = 0; k < K; k++) acc[k] = dd{0.0, 0.0};
     double ym = 0.0;
 #pragma unroll
-    for (int q = 0; q < kPfxItems; q++) {
+    for (int q = 0; q < ITEMS; q++) {
         if (j0 + q < n) {
             const double2 v = xy[j0 + q];
             ym = fmax(ym, fabs(v.y));
@@ -185,7 +188,7 @@ pfx_tile_reduce_kernel(const double2 *__restrict__ xy, int n, double2 *__restric
 // Phase 3: in-tile exclusive scan + tile offset -> P[k][j] = sum_{l<j} t_k(l)
 // for j in the tile (and P[k][n] by the last tile), plus the plain sorted-x
 // array xs (with -inf / +inf sentinels) used by the window searches.
-template <int KERN>
+template <int KERN, int ITEMS>
 __global__ void __launch_bounds__(kPfxThreads)
 pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__restrict__ tot, int ntiles,
                      double *__restrict__ P, int pstride, double *__restrict__ xs)
@@ -215,18 +218,18 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
         __syncthreads();
     }
     const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-    const int j0 = blockIdx.x * kPfxTile + t * kPfxItems;
+    const int j0 = blockIdx.x * (kPfxThreads * ITEMS) + t * ITEMS;
     if (blockIdx.x == 0 && t < kPad) {
         xs[-1 - t] = -INFINITY;
         xs[n + t] = INFINITY;
     }
     const double o = pfx_origin(xy, n);
-    dd tm[kPfxItems][kPfxMoments];
+    dd tm[ITEMS][kPfxMoments];
     dd acc[kPfxMoments];
 #pragma unroll
     for (int k = 0; k < K; k++) acc[k] = dd{0.0, 0.0};
 #pragma unroll
-    for (int q = 0; q < kPfxItems; q++) {
+    for (int q = 0; q < ITEMS; q++) {
         if (j0 + q < n) {
             const double2 v = xy[j0 + q];
             xs[j0 + q] = v.x;
@@ -259,7 +262,7 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
         for (int q = 0; q < w; q++) base = dd_add(base, ld_dd(&wsum[k][q]));
         dd run = dd_add(base, ex[k]);
 #pragma unroll
-        for (int q = 0; q < kPfxItems; q++) {
+        for (int q = 0; q < ITEMS; q++) {
             if (j0 + q <= n) {
                 P[(size_t)(2 * k) * pstride + j0 + q] = run.hi;
                 P[(size_t)(2 * k + 1) * pstride + j0 + q] = run.lo;

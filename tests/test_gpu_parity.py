@@ -408,3 +408,46 @@ def test_kde_full_size_sampled_shard(k):
     lscv, best = krcv.kr_kde_finalize(tot, x.shape[0], h, k)
     full, best_full = krcv.kr_kde_lscv(x, h, k)
     assert cv_rel_err(lscv, full) <= 1e-12 and best_ok(best, full)
+
+
+def test_host_api_nonfinite_and_graph_replay():
+    """kr_cv_grid from host arrays: NaN / Inf in x or y -> KR_ENONFINITE
+    (device-side status) with the outputs untouched; with pinned buffers the
+    call is replayed from a captured CUDA graph, which must read the buffers'
+    current contents (new data each call) and re-capture when n, m, kernel
+    or algorithm change."""
+    import ctypes
+
+    import torch
+    lib = krcv._lib()
+    x, y = workloads.draw_xy("paper", 3000, 5)
+    h = workloads.grid_default(x, 40)
+    for bad in ("x", "y"):
+        xb, yb = x.copy(), y.copy()
+        (xb if bad == "x" else yb)[1234] = math.nan if bad == "x" else -math.inf
+        cv = np.full(40, 7.0)
+        best = ctypes.c_int32(-5)
+        st = lib.kr_cv_grid(xb.ctypes.data, yb.ctypes.data, 3000, h.ctypes.data, 40, E, cv.ctypes.data,
+                            ctypes.byref(best))
+        assert st == krcv.KR_ENONFINITE and np.all(cv == 7.0) and best.value == -5
+    hx = torch.empty(3000, dtype=torch.float64).pin_memory()
+    hy = torch.empty(3000, dtype=torch.float64).pin_memory()
+    hh = torch.from_numpy(h.copy()).pin_memory()
+    out = torch.empty(40, dtype=torch.float64).pin_memory()
+    best = ctypes.c_int32(-1)
+    for seed in range(4):
+        xs, ys = workloads.draw_xy("sin_uniform" if seed % 2 else "paper", 3000, 50 + seed)
+        hx.copy_(torch.from_numpy(xs))
+        hy.copy_(torch.from_numpy(ys))
+        hh.copy_(torch.from_numpy(workloads.grid_default(xs, 40)))
+        for k in (E, U):
+            st = krcv.kr_cv_grid_ptr(hx.data_ptr(), hy.data_ptr(), 3000, hh.data_ptr(), 40, k, out.data_ptr(),
+                                     ctypes.byref(best))
+            assert st == 0
+            ref = oracle.cv_sorted(xs, ys, hh.numpy(), k)
+            assert cv_rel_err(out.numpy(), ref.cv) <= TIGHT and best.value == ref.best
+    # a NaN arriving through the replayed graph is still reported
+    hx[7] = math.nan
+    st = krcv.kr_cv_grid_ptr(hx.data_ptr(), hy.data_ptr(), 3000, hh.data_ptr(), 40, U, out.data_ptr(),
+                             ctypes.byref(best))
+    assert st == krcv.KR_ENONFINITE
