@@ -90,7 +90,7 @@ class GridSearch:
         # graph=True (single GPU): the enqueued pipeline is captured once per
         # (x, y) pointer pair as a CUDA graph and replayed -- one launch for
         # the whole search instead of one per stage
-        self.graph = bool(graph) and self.world == 1
+        self.graph = bool(graph) and int(world) == 1
         self._g = None
         self._gkey = None
         self.rank, self.world, self.group = int(rank), int(world), group

@@ -287,41 +287,42 @@ template <int KERN>
 __device__ __forceinline__ void window_bounds(const double *__restrict__ xs, int n, int r, double xr, double h,
                                               int &kR, int &kL, int gR, int gL)
 {
-    const double *__restrict__ xsr = xs + r;
+    // the row's base pointer, laundered through an empty asm so the compiler
+    // keeps it in a register instead of re-deriving xs + (r + k) in 64-bit
+    // arithmetic at every probe (4 instructions -> 1 IMAD.WIDE)
+    unsigned long long base = reinterpret_cast<unsigned long long>(xs + r);
+    asm("" : "+l"(base));
+    const double *__restrict__ xsr = reinterpret_cast<const double *>(base);
     int rlo = kR - 1, rhi = 0, rstep = gR;  // rlo: inside (or the row itself)
     int llo = kL - 1, lhi = 0, lstep = gL;
     const int kRmax = n - r, kLmax = r + 1;
-    bool rg = true, lg = true;
-    while (rg || lg) {
+    int rg = 1, lg = 1;  // int flags: bools cost byte-permute instructions here
+    while (rg | lg) {
         if (rg) {
             const int k = min(rlo + rstep, kRmax);
-            if (inside<KERN>(xsr[k] - xr, h)) {
-                rlo = k;
-                rstep *= 2;
-            } else {
-                rhi = k;
-                rg = false;
-            }
+            const int in = inside<KERN>(__ldg(xsr + k) - xr, h);
+            rlo = in ? k : rlo;
+            rhi = in ? rhi : k;
+            rstep <<= in;
+            rg = in;
         }
         if (lg) {
             const int k = min(llo + lstep, kLmax);
-            if (inside<KERN>(xr - xsr[-k], h)) {
-                llo = k;
-                lstep *= 2;
-            } else {
-                lhi = k;
-                lg = false;
-            }
+            const int in = inside<KERN>(xr - __ldg(xsr - k), h);
+            llo = in ? k : llo;
+            lhi = in ? lhi : k;
+            lstep <<= in;
+            lg = in;
         }
     }
     while (rhi - rlo > 1 || lhi - llo > 1) {
         if (rhi - rlo > 1) {
             const int k = (rlo + rhi) >> 1;
-            if (inside<KERN>(xsr[k] - xr, h)) rlo = k; else rhi = k;
+            if (inside<KERN>(__ldg(xsr + k) - xr, h)) rlo = k; else rhi = k;
         }
         if (lhi - llo > 1) {
             const int k = (llo + lhi) >> 1;
-            if (inside<KERN>(xr - xsr[-k], h)) llo = k; else lhi = k;
+            if (inside<KERN>(xr - __ldg(xsr - k), h)) llo = k; else lhi = k;
         }
     }
     kR = rhi;
@@ -475,25 +476,33 @@ __device__ __forceinline__ void window_advance(const double *__restrict__ xs, in
 {
     int rlo = max(R, r1 + 1) - 1, rhi = 0, rstep = 1;  // rlo: inside for r1 (or r1 itself)
     int llo = L, lhi = 0, lstep = 1;                   // llo: outside for r1
-    bool rg = true, lg = true;
-    while (rg || lg) {
+    int rg = 1, lg = 1;
+    while (rg | lg) {
         if (rg) {
             const int k = min(rlo + rstep, n);
-            if (inside<KERN>(xs[k] - xr1, h)) { rlo = k; rstep *= 2; } else { rhi = k; rg = false; }
+            const int in = inside<KERN>(__ldg(xs + k) - xr1, h);
+            rlo = in ? k : rlo;
+            rhi = in ? rhi : k;
+            rstep <<= in;
+            rg = in;
         }
         if (lg) {
             const int k = min(llo + lstep, r1);  // r1 itself is "inside" (d = 0)
-            if (k < r1 && !inside<KERN>(xr1 - xs[k], h)) { llo = k; lstep *= 2; } else { lhi = k; lg = false; }
+            const int out = k < r1 && !inside<KERN>(xr1 - __ldg(xs + k), h);
+            llo = out ? k : llo;
+            lhi = out ? lhi : k;
+            lstep <<= out;
+            lg = out;
         }
     }
     while (rhi - rlo > 1 || lhi - llo > 1) {
         if (rhi - rlo > 1) {
             const int k = (rlo + rhi) >> 1;
-            if (inside<KERN>(xs[k] - xr1, h)) rlo = k; else rhi = k;
+            if (inside<KERN>(__ldg(xs + k) - xr1, h)) rlo = k; else rhi = k;
         }
         if (lhi - llo > 1) {
             const int k = (llo + lhi) >> 1;
-            if (!inside<KERN>(xr1 - xs[k], h)) llo = k; else lhi = k;
+            if (!inside<KERN>(xr1 - __ldg(xs + k), h)) llo = k; else lhi = k;
         }
     }
     R = rhi;
@@ -586,21 +595,27 @@ template <int KERN>
 __device__ __forceinline__ void window_bounds2(const double *__restrict__ xs, int n, int r, double xr, double ha,
                                                double hb, int kR, int kL, int gR, int gL, int (&kout)[4])
 {
-    const double *__restrict__ xsr = xs + r;
+    unsigned long long base = reinterpret_cast<unsigned long long>(xs + r);  // see window_bounds
+    asm("" : "+l"(base));
+    const double *__restrict__ xsr = reinterpret_cast<const double *>(base);
     // chains: 0 right@ha, 1 left@ha, 2 right@hb, 3 left@hb
     int lo[4] = {kR - 1, kL - 1, kR - 1, kL - 1};
     int hi[4] = {0, 0, 0, 0};
     int st[4] = {gR, gL, 2 * gR, 2 * gL};
-    bool go[4] = {true, true, true, true};
+    int go[4] = {1, 1, 1, 1};
     const int kmax[4] = {n - r, r + 1, n - r, r + 1};
     const double hh[4] = {ha, ha, hb, hb};
-    while (go[0] || go[1] || go[2] || go[3]) {
+    while (go[0] | go[1] | go[2] | go[3]) {
 #pragma unroll
         for (int c = 0; c < 4; c++) {
             if (go[c]) {
                 const int k = min(lo[c] + st[c], kmax[c]);
-                const double d = (c & 1) ? xr - xsr[-k] : xsr[k] - xr;
-                if (inside<KERN>(d, hh[c])) { lo[c] = k; st[c] *= 2; } else { hi[c] = k; go[c] = false; }
+                const double d = (c & 1) ? xr - __ldg(xsr - k) : __ldg(xsr + k) - xr;
+                const int in = inside<KERN>(d, hh[c]);
+                lo[c] = in ? k : lo[c];
+                hi[c] = in ? hi[c] : k;
+                st[c] <<= in;
+                go[c] = in;
             }
         }
     }
@@ -609,7 +624,7 @@ __device__ __forceinline__ void window_bounds2(const double *__restrict__ xs, in
         for (int c = 0; c < 4; c++) {
             if (hi[c] - lo[c] > 1) {
                 const int k = (lo[c] + hi[c]) >> 1;
-                const double d = (c & 1) ? xr - xsr[-k] : xsr[k] - xr;
+                const double d = (c & 1) ? xr - __ldg(xsr - k) : __ldg(xsr + k) - xr;
                 if (inside<KERN>(d, hh[c])) lo[c] = k; else hi[c] = k;
             }
         }

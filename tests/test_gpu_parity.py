@@ -451,3 +451,26 @@ def test_host_api_nonfinite_and_graph_replay():
     st = krcv.kr_cv_grid_ptr(hx.data_ptr(), hy.data_ptr(), 3000, hh.data_ptr(), 40, U, out.data_ptr(),
                              ctypes.byref(best))
     assert st == krcv.KR_ENONFINITE
+
+
+def test_gridsearch_graph_replay():
+    """GridSearch(graph=True): the captured graph replays the whole search;
+    new contents in the same tensors are picked up, other tensors re-capture,
+    results equal the eager path bit for bit (same kernels, same order)."""
+    import torch
+    x, y = workloads.draw_xy("paper", 5000, 9)
+    h = workloads.grid_default(x, 60)
+    d_x, d_y = torch.as_tensor(x, device="cuda"), torch.as_tensor(y, device="cuda")
+    eager = GridSearch(5000, h, E)
+    graph = GridSearch(5000, h, E, graph=True)
+    for step in range(3):
+        if step == 2:
+            d_x, d_y = d_x.clone(), (d_y * 2.0).contiguous()
+        elif step == 1:
+            d_y.mul_(0.5)
+        eager.run(d_x, d_y)
+        graph.run(d_x, d_y)
+        a, b = eager.result(), graph.result()
+        assert torch.equal(a.cv, b.cv) and a.best == b.best and torch.equal(a.neff, b.neff)
+    ref = oracle.cv_sorted(d_x.cpu().numpy(), d_y.cpu().numpy(), h, E)
+    assert cv_rel_err(b.cv.cpu().numpy(), ref.cv) <= TIGHT
