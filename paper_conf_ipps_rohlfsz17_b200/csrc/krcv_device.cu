@@ -375,7 +375,14 @@ static void prof_mark(int k, cudaStream_t st)
 {
     if (!g_prof.on) return;
     if (!g_prof.ev[k]) cudaEventCreate(&g_prof.ev[k]);
-    cudaEventRecord(g_prof.ev[k], st);
+    // inside a stream capture (GridSearch(graph=True)) the record must be an
+    // external event-record node so that every graph replay records it
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    cudaStreamIsCapturing(st, &cs);
+    if (cs == cudaStreamCaptureStatusActive)
+        cudaEventRecordWithFlags(g_prof.ev[k], st, cudaEventRecordExternal);
+    else
+        cudaEventRecord(g_prof.ev[k], st);
 }
 
 // Kernel launches CUB's radix sort makes for `n` 64-bit keys.  Onesweep:

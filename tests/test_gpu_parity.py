@@ -474,3 +474,23 @@ def test_gridsearch_graph_replay():
         assert torch.equal(a.cv, b.cv) and a.best == b.best and torch.equal(a.neff, b.neff)
     ref = oracle.cv_sorted(d_x.cpu().numpy(), d_y.cpu().numpy(), h, E)
     assert cv_rel_err(b.cv.cpu().numpy(), ref.cv) <= TIGHT
+
+
+def test_gridsearch_graph_with_stage_events():
+    """The bench's configuration: profiling on before the capture, so the
+    stage events are event-record nodes of the graph and kr_profile_read
+    returns this replay's stage times."""
+    import torch
+    x, y, h, k = workloads.make("C2", seed=0, n=4000)
+    d_x, d_y = torch.as_tensor(x, device="cuda"), torch.as_tensor(y, device="cuda")
+    krcv.kr_profile_enable(True)
+    try:
+        plan = GridSearch(4000, h, k, graph=True)
+        for _ in range(3):
+            plan.run(d_x, d_y)
+            st = krcv.kr_profile_read()
+            assert len(st) == 4 and all(v >= 0.0 for v in st) and st[2] > 0.0
+    finally:
+        krcv.kr_profile_enable(False)
+    ref = oracle.cv_sorted(x, y, h, k)
+    assert cv_rel_err(plan.result().cv.cpu().numpy(), ref.cv) <= TIGHT
