@@ -473,10 +473,11 @@ int win_rows_per_lane(int64_t rows)
         forced = (k >= 1 && k <= 5) ? k : 0;  // 3: window_kernel_b2, 5: window_kernel_coop
     }
     if (forced) return forced;
-    // measured (profiles/r01t_*, r01u_*): two consecutive rows per lane up to
-    // ~1.5e5 rows (C2, C3); above, one row per lane with two bandwidths per
-    // step (window_kernel_b2: C4 22.9 -> 20.9 ms, C5 2.57 -> 2.43 ms)
-    return rows <= 150000 ? 2 : 3;
+    // measured (profiles/r01t_*, r01u_*, r01af_*): two consecutive rows per
+    // lane up to 5e4 rows (C2: K = 1, 2, b2 within 1 %); above, one row per
+    // lane with two bandwidths per step (window_kernel_b2: C3 1.73 -> 1.65 ms,
+    // C4 22.9 -> 20.9 ms, C5 2.57 -> 2.43 ms)
+    return rows <= 50000 ? 2 : 3;
 }
 
 template <int KERN, int K>

@@ -94,8 +94,8 @@ kde_window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy,
         const int r = valid ? i : row_hi - 1;
         const double xr = xy[r].x;
         const dd del = two_sum(xr, -o);  // exact x_r - o
-        int kR1 = 1, kL1 = 1, gR1 = 1, gL1 = 1;  // K's window (radius h)
-        int kR2 = 1, kL2 = 1, gR2 = 1, gL2 = 1;  // Kbar's window (radius 2h, open)
+        int kR1 = 1, kL1 = 1, gR1 = cold_step(xs, n, __ldg(hg + b0)), gL1 = gR1;  // K's window (radius h)
+        int kR2 = 1, kL2 = 1, gR2 = 2 * gR1, gL2 = gR2;  // Kbar's window (radius 2h, open)
         for (int b = b0; b < b1; b++) {
             const double h = __ldg(hg + b), h2 = 2.0 * h;  // 2h exact
             {

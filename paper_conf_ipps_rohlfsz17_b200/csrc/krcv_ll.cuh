@@ -266,7 +266,7 @@ ll_window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, 
             row.yr = v.y;
             row.del = two_sum(v.x, -o);
         }
-        int kR = 1, kL = 1, gR = 1, gL = 1;
+        int kR = 1, kL = 1, gR = cold_step(xs, n, __ldg(hg + b0)), gL = gR;
         for (int b = b0; b < b1; b++) {
             const double h = __ldg(hg + b);
             const int kR0 = kR, kL0 = kL;

@@ -119,6 +119,19 @@ __device__ __forceinline__ void st_dd(double2 *p, dd v) { *p = make_double2(v.hi
 // origin o: the median record of the sorted array (keeps |u| small).
 __device__ __forceinline__ double pfx_origin(const double2 *xy, int n) { return xy[n >> 1].x; }
 
+// First gallop step of a chunk's cold search at bandwidth h: half the
+// window size a uniform density would give, (n - 1) h / (x_max - x_min) / 2
+// (>= 1).  Chunks after the first start far from the row, and a gallop from
+// step 1 would spend ~2 log2(window) probes per side getting there; any step
+// keeps the search exact (the gallop / bisection verify every boundary).
+__device__ __forceinline__ int cold_step(const double *__restrict__ xs, int n, double h)
+{
+    const double span = xs[n - 1] - xs[0];
+    if (!(span > 0.0)) return 1;
+    const double e = 0.5 * (double)(n - 1) * (h / span);
+    return e >= (double)n ? n : (e < 1.0 ? 1 : (int)e);
+}
+
 // ---------------------------------------------------------------- build
 // Two-phase fixed-order scan (bit-reproducible; a decoupled look-back
 // would make the dd rounding depend on timing): tile totals, then every tile
@@ -554,7 +567,7 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
             rows[k].del = two_sum(v.x, -o);  // exact x_r - o
         }
         int kR = 1, kL = 1;  // first row: first offsets not yet known inside
-        int gR = 1, gL = 1;  // first row: previous growth of each side
+        int gR = cold_step(xs, n, __ldg(hg + b0)), gL = gR;  // first row: gallop steps
 
         for (int b = b0; b < b1; b++) {
             const double h = __ldg(hg + b);
@@ -662,7 +675,7 @@ window_kernel_b2(const double *__restrict__ xs, const double2 *__restrict__ xy, 
         w.xr = v.x;
         w.yr = v.y;
         w.del = two_sum(v.x, -o);
-        int kR = 1, kL = 1, gR = 1, gL = 1;
+        int kR = 1, kL = 1, gR = cold_step(xs, n, __ldg(hg + b0)), gL = gR;
         for (int b = b0; b < b1; b += 2) {
             const bool two = b + 1 < b1;
             const double ha = __ldg(hg + b), hb = two ? __ldg(hg + b + 1) : ha;
@@ -788,7 +801,7 @@ window_kernel_coop(const double *__restrict__ xs, const double2 *__restrict__ xy
         w.xr = v.x;
         w.yr = v.y;
         w.del = two_sum(v.x, -o);
-        int kR = 1, kL = 1, gR = 1, gL = 1;  // this row's previous boundaries (offsets) and growth
+        int kR = 1, kL = 1, gR = cold_step(xs, n, __ldg(hg + b0)), gL = gR;  // previous boundaries, growth
         // leader state (offsets from the leader row): warp 0 R of first, 1 R of
         // last, 2 L of first, 3 L of last
         const int lrow = (wp & 1) ? last : first;
