@@ -310,6 +310,31 @@ __device__ __forceinline__ void window_bounds(const double *__restrict__ xs, int
     int llo = kL - 1, lhi = 0, lstep = gL;
     const int kRmax = n - r, kLmax = r + 1;
     int rg = 1, lg = 1;  // int flags: bools cost byte-permute instructions here
+    // Predicted bracket: the boundary is expected about one growth g beyond
+    // the previous one, give or take a few sqrt(g) (Poisson spread of the
+    // points added).  Probe g - s and g + s (s = 3 sqrt(g)) on both sides at
+    // once -- four independent loads -- and bisect the bracket that holds
+    // the boundary; if both probes are inside, keep galloping from g + s.
+    // Any outcome leaves a valid state for the loops below (exactness does
+    // not depend on the prediction).
+    if (gR >= 4) {
+        const int sR = (int)(3.0f * sqrtf((float)gR));
+        const int p1 = min(rlo + max(1, gR - sR), kRmax), p2 = min(rlo + gR + sR, kRmax);
+        const int in1 = inside<KERN>(__ldg(xsr + p1) - xr, h), in2 = inside<KERN>(__ldg(xsr + p2) - xr, h);
+        rhi = !in1 ? p1 : (!in2 ? p2 : 0);
+        rlo = !in1 ? rlo : (!in2 ? p1 : p2);
+        rstep = 2 * sR + 1;
+        rg = in1 & in2;
+    }
+    if (gL >= 4) {
+        const int sL = (int)(3.0f * sqrtf((float)gL));
+        const int p1 = min(llo + max(1, gL - sL), kLmax), p2 = min(llo + gL + sL, kLmax);
+        const int in1 = inside<KERN>(xr - __ldg(xsr - p1), h), in2 = inside<KERN>(xr - __ldg(xsr - p2), h);
+        lhi = !in1 ? p1 : (!in2 ? p2 : 0);
+        llo = !in1 ? llo : (!in2 ? p1 : p2);
+        lstep = 2 * sL + 1;
+        lg = in1 & in2;
+    }
     while (rg | lg) {
         if (rg) {
             const int k = min(rlo + rstep, kRmax);
@@ -489,7 +514,29 @@ __device__ __forceinline__ void window_advance(const double *__restrict__ xs, in
 {
     int rlo = max(R, r1 + 1) - 1, rhi = 0, rstep = 1;  // rlo: inside for r1 (or r1 itself)
     int llo = L, lhi = 0, lstep = 1;                   // llo: outside for r1
-    int rg = 1, lg = 1;
+    // Common case first: each boundary moves by 0 or 1 (about one point per
+    // row gap).  The four candidates are independent loads -- one memory
+    // latency instead of two or three dependent probes per side; xs has
+    // +inf sentinels past n, so rlo + 2 <= n + 1 is always readable.
+    int rg, lg;
+    {
+        const double a1 = __ldg(xs + rlo + 1), a2 = __ldg(xs + rlo + 2);
+        const int k1 = llo + 1, k2 = llo + 2;  // <= r1 + 1: readable (r1 < n)
+        const double b1 = __ldg(xs + k1), b2 = __ldg(xs + k2);
+        const int in1 = rlo + 1 <= n && inside<KERN>(a1 - xr1, h);
+        const int in2 = rlo + 2 <= n && inside<KERN>(a2 - xr1, h);
+        const int out1 = k1 < r1 && !inside<KERN>(xr1 - b1, h);
+        const int out2 = k2 < r1 && !inside<KERN>(xr1 - b2, h);
+        // right: first outside among rlo+1, rlo+2, else keep galloping from rlo+2
+        rhi = !in1 ? rlo + 1 : (!in2 ? rlo + 2 : 0);
+        rg = in1 & in2;
+        rlo = in1 ? (in2 ? rlo + 2 : rlo + 1) : rlo;
+        // left: last outside -- llo+1, llo+2 outside move it; stop at the first inside
+        lhi = !out1 ? k1 : (!out2 ? k2 : 0);
+        lg = out1 & out2;
+        llo = out1 ? (out2 ? k2 : k1) : llo;
+        if (rg) rhi = 0;
+    }
     while (rg | lg) {
         if (rg) {
             const int k = min(rlo + rstep, n);
@@ -618,6 +665,22 @@ __device__ __forceinline__ void window_bounds2(const double *__restrict__ xs, in
     int go[4] = {1, 1, 1, 1};
     const int kmax[4] = {n - r, r + 1, n - r, r + 1};
     const double hh[4] = {ha, ha, hb, hb};
+    // predicted brackets (see window_bounds): eight independent loads
+#pragma unroll
+    for (int c = 0; c < 4; c++) {
+        const int g = st[c];
+        if (g >= 4) {
+            const int sg = (int)(3.0f * sqrtf((float)g));
+            const int p1 = min(lo[c] + max(1, g - sg), kmax[c]), p2 = min(lo[c] + g + sg, kmax[c]);
+            const double d1 = (c & 1) ? xr - __ldg(xsr - p1) : __ldg(xsr + p1) - xr;
+            const double d2 = (c & 1) ? xr - __ldg(xsr - p2) : __ldg(xsr + p2) - xr;
+            const int in1 = inside<KERN>(d1, hh[c]), in2 = inside<KERN>(d2, hh[c]);
+            hi[c] = !in1 ? p1 : (!in2 ? p2 : 0);
+            lo[c] = !in1 ? lo[c] : (!in2 ? p1 : p2);
+            st[c] = 2 * sg + 1;
+            go[c] = in1 & in2;
+        }
+    }
     while (go[0] | go[1] | go[2] | go[3]) {
 #pragma unroll
         for (int c = 0; c < 4; c++) {
