@@ -250,7 +250,6 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     L->tileN = off;    off = align256(off + sizeof(uint8_t) * (size_t)ntiles * (size_t)m);
     L->tileB = off;    off = align256(off + sizeof(double) * (size_t)((n + 31) / 32) * (size_t)m);  // KDE sum B
     L->partial = off;  off = align256(off + sizeof(double) * (size_t)KR_PARTIAL_LEN(m));
-    L->chunkdone = off; off = align256(off + sizeof(unsigned) * ((size_t)m + 2));
     L->cub_bytes = cub_bytes;
     L->total = off;
     L->ntiles_max = ntiles;
@@ -484,7 +483,7 @@ int win_rows_per_lane(int64_t rows)
 template <int KERN, int K>
 static void launch_window_k(const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
                             const WsLayout &L, char *ws, double *tileS, uint8_t *tileN, int *counter,
-                            cudaStream_t st, WinFuse fz)
+                            cudaStream_t st)
 {
     static int resident = 0;
     if (!resident) {
@@ -522,34 +521,29 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
     const double *P = reinterpret_cast<const double *>(ws + L.pfx);
     const unsigned long long *ymax =
         reinterpret_cast<const unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
-    if (fz.partial) {  // fused a5: zero the chunk completion counters
-        fz.chunk_done = reinterpret_cast<unsigned *>(ws + L.chunkdone);
-        fz.chunks_done = fz.chunk_done + nbc;
-        cudaMemsetAsync(fz.chunk_done, 0, sizeof(unsigned) * (size_t)(nbc + 1), st);
-    }
     if (K == 3)
         window_kernel_b2<KERN><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
-                                                               nbc, ymax, tileS, tileN, counter, fz);
+                                                               nbc, ymax, tileS, tileN, counter);
     else if (K == 5)
         window_kernel_coop<KERN><<<blocks, kCoopRows, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
                                                                nbc, ymax, tileS, tileN, counter);
     else
         window_kernel<KERN, (K == 3 || K == 5) ? 1 : K><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo,
                                                                             hi, ntiles, nbc, ymax, tileS, tileN,
-                                                                            counter, fz);
+                                                                            counter);
 }
 
 template <int KERN>
 static void launch_window(int K, const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
                           const WsLayout &L, char *ws, double *tileS, uint8_t *tileN, int *counter,
-                          cudaStream_t st, const WinFuse &fz)
+                          cudaStream_t st)
 {
     switch (K) {
-    case 1: launch_window_k<KERN, 1>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st, fz); break;
-    case 2: launch_window_k<KERN, 2>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st, fz); break;
-    case 3: launch_window_k<KERN, 3>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st, fz); break;
-    case 5: launch_window_k<KERN, 5>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st, WinFuse{}); break;
-    default: launch_window_k<KERN, 4>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st, fz); break;
+    case 1: launch_window_k<KERN, 1>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    case 2: launch_window_k<KERN, 2>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    case 3: launch_window_k<KERN, 3>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    case 5: launch_window_k<KERN, 5>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    default: launch_window_k<KERN, 4>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     }
 }
 
@@ -798,19 +792,6 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         launches += 2;
     }
     prof_mark(2, st);
-    // a5 fused into the window kernel's tail (WinFuse) on the window-prefix
-    // path (not the cooperative variant, not local-linear)
-    const bool fused = prefix && !ll && winK != 5 && ntiles > 0 && !getenv_flag("KRCV_NO_FUSE");
-    WinFuse fz{};
-    if (fused) {
-        fz.partial = d_partial;
-        fz.status = status;
-        fz.n = fin.n;
-        fz.cv = fin.cv;
-        fz.neff = fin.neff;
-        fz.best = fin.best;
-        fz.status_out = fin.status;
-    }
     if (ntiles > 0) {
         launches += 1;
         if (hist) {
@@ -848,13 +829,13 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         } else if (prefix) {
             switch (kernel) {
             case KR_UNIFORM:
-                launch_window<KR_UNIFORM>(winK, xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st, fz);
+                launch_window<KR_UNIFORM>(winK, xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
                 break;
             case KR_EPANECHNIKOV:
-                launch_window<KR_EPANECHNIKOV>(winK, xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st, fz);
+                launch_window<KR_EPANECHNIKOV>(winK, xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
                 break;
             default:
-                launch_window<KR_TRIANGULAR>(winK, xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st, fz);
+                launch_window<KR_TRIANGULAR>(winK, xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
                 break;
             }
         } else {
@@ -872,11 +853,9 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         }
     }
     prof_mark(3, st);
-    if (!fused) {
-        reduce_kernel<<<m < 148 * 8 ? m : 148 * 8, kReduceThreads, 0, st>>>(tileS, tileN, ntiles, m, status,
-                                                                            d_partial, fin);
-        launches += 1;
-    }
+    reduce_kernel<<<m < 148 * 8 ? m : 148 * 8, kReduceThreads, 0, st>>>(tileS, tileN, ntiles, m, status,
+                                                                        d_partial, fin);
+    launches += 1;
     prof_mark(4, st);
     g_prof.recorded = g_prof.on;
     g_prof.launches = launches;

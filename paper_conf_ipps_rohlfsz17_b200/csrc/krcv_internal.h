@@ -26,7 +26,6 @@ struct WsLayout {
     size_t tileS;               // double  [m][ntiles]  per-tile sum of M e^2
     size_t tileN;               // uint8   [m][ntiles]  per-tile sum of M
     size_t tileB;               // double  [m][ceil(n/32)] per-tile KDE sum B (tileS holds A)
-    size_t chunkdone;           // uint32  [m + 1] chunk completion counters of the fused a5
     size_t status;              // uint32  [8]  n_bad_grid, n_nonfinite, reduce completion counter, pad,
                                 //              u64 bits of max |y| (window-prefix fast-path bound)
     size_t partial;             // double  [2m+2] partial vector of kr_cv_grid_async

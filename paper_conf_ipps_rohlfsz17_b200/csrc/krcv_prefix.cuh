@@ -569,92 +569,6 @@ __device__ __forceinline__ void window_advance(const double *__restrict__ xs, in
     L = llo;
 }
 
-// a5 fused into the window kernels (replaces reduce_kernel on this path):
-// the warp that completes the last tile of a bandwidth chunk sums that
-// chunk's tile partials per bandwidth in a fixed order (lane-strided over
-// tiles, then a fixed butterfly -- bit-reproducible whichever warp does it)
-// into partial[b] / partial[m + b]; the warp that completes the last chunk
-// copies the status counters and, for a single-GPU whole search (cv set),
-// runs the finalize (CV = S/n, arg-min of reading Q11).  Counters are zeroed
-// by the host enqueue before the launch.
-struct WinFuse {
-    double *partial;              // nullptr: no fusion (reduce_kernel follows)
-    const unsigned *status;       // status words 0, 1 (bad grid, non-finite)
-    unsigned *chunk_done;         // [nbc] tiles finished per chunk
-    unsigned *chunks_done;        // chunks finished
-    long long n;
-    double *cv;                   // finalize outputs (nullptr: shard partial only)
-    long long *neff;
-    int *best, *status_out;
-};
-
-__device__ __forceinline__ void win_task_tail(const WinFuse &f, int chunk, int b0, int b1, int ntiles, int nbc,
-                                              int m, const double *tileS, const uint8_t *tileN, int lane)
-{
-    if (f.partial == nullptr) return;
-    __threadfence();  // this warp's tile partials (written by lane 0) before the count
-    unsigned last = 0;
-    if (lane == 0) last = atomicAdd(f.chunk_done + chunk, 1u) == (unsigned)ntiles - 1u;
-    last = __shfl_sync(0xffffffffu, last, 0);
-    if (!last) return;
-    __threadfence();
-    for (int b = b0; b < b1; b++) {
-        double a = 0.0;
-        unsigned c = 0;
-        for (int t = lane; t < ntiles; t += 32) {
-            a += __ldcg(tileS + (size_t)b * ntiles + t);
-            c += __ldcg(tileN + (size_t)b * ntiles + t);
-        }
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
-        c = __reduce_add_sync(0xffffffffu, c);
-        if (lane == 0) {
-            f.partial[b] = a;
-            f.partial[m + b] = (double)c;
-        }
-    }
-    __threadfence();
-    unsigned lastc = 0;
-    if (lane == 0) lastc = atomicAdd(f.chunks_done, 1u) == (unsigned)nbc - 1u;
-    lastc = __shfl_sync(0xffffffffu, lastc, 0);
-    if (!lastc) return;
-    __threadfence();
-    if (lane == 0) {
-        f.partial[2 * m] = (double)__ldcg(f.status + 0);
-        f.partial[2 * m + 1] = (double)__ldcg(f.status + 1);
-    }
-    if (f.cv == nullptr) return;
-    __syncwarp();
-    // finalize: CV = S / n, smallest arg-min, NaN never minimal (reading Q11)
-    double bv = 0.0;
-    int bi = -1;
-    for (int b = lane; b < m; b += 32) {
-        const double v = __ldcg(f.partial + b) / (double)f.n;
-        f.cv[b] = v;
-        if (f.neff) f.neff[b] = (long long)__ldcg(f.partial + m + b);
-        if (!isnan(v) && (bi < 0 || v < bv)) {
-            bv = v;
-            bi = b;
-        }
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        const double ov = __shfl_xor_sync(0xffffffffu, bv, o);
-        const int oi = __shfl_xor_sync(0xffffffffu, bi, o);
-        if (oi >= 0 && (bi < 0 || ov < bv || (ov == bv && oi < bi))) {
-            bv = ov;
-            bi = oi;
-        }
-    }
-    if (lane == 0) {
-        *f.best = bi < 0 ? 0 : bi;
-        int st = KR_OK;
-        if (__ldcg(f.status + 0) != 0u) st = KR_EGRID;
-        else if (__ldcg(f.status + 1) != 0u) st = KR_ENONFINITE;
-        *f.status_out = st;
-    }
-}
-
 // A warp owns 32 * K consecutive sorted rows: lane l the K rows
 // base + l K .. base + l K + K - 1, and a chunk of the bandwidth loop.  Per
 // bandwidth the lane's first row searches from its previous bandwidth's
@@ -665,7 +579,7 @@ __global__ void __launch_bounds__(kWinThreads)
 window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
               int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
               int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
-              uint8_t *__restrict__ tileN, int *__restrict__ tile_counter, WinFuse fuse)
+              uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
 {
     const int lane = threadIdx.x & 31;
     const double o = pfx_origin(xy, n);
@@ -730,7 +644,6 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
                 tileN[(size_t)b * ntiles + tile] = (uint8_t)cnt;
             }
         }
-        win_task_tail(fuse, chunk, b0, b1, ntiles, nbc, m, tileS, tileN, lane);
     }
 }
 
@@ -801,7 +714,7 @@ __global__ void __launch_bounds__(kWinThreads)
 window_kernel_b2(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
                  int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
                  int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
-                 uint8_t *__restrict__ tileN, int *__restrict__ tile_counter, WinFuse fuse)
+                 uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
 {
     const int lane = threadIdx.x & 31;
     const double o = pfx_origin(xy, n);
@@ -862,7 +775,6 @@ window_kernel_b2(const double *__restrict__ xs, const double2 *__restrict__ xy, 
                 }
             }
         }
-        win_task_tail(fuse, chunk, b0, b1, ntiles, nbc, m, tileS, tileN, lane);
     }
 }
 
