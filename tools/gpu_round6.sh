@@ -1,0 +1,15 @@
+#!/bin/bash
+TAG=${1:-r01}; OUT=gpurun_out; mkdir -p $OUT
+timeout 1500 python -m pytest tests -m gpu -x -q > $OUT/${TAG}_pytest_gpu.log 2>&1; echo "exit $?" >> $OUT/${TAG}_pytest_gpu.log
+timeout 600 python bench.py > $OUT/${TAG}_bench_C2.json 2> $OUT/${TAG}_bench_C2.err
+for c in C3 C5 C4; do
+  timeout 600 python bench.py --config $c --steps 10 --warmup 3 --no-cpu-baseline > $OUT/${TAG}_bench_$c.json 2> $OUT/${TAG}_bench_$c.err
+done
+for c in C2 C3; do for K in 1 2 3; do
+  KRCV_WIN_K=$K timeout 300 python bench.py --config $c --steps 10 --warmup 3 --no-cpu-baseline --no-alt > $OUT/${TAG}_bench_${c}_K$K.json 2>/dev/null
+done; done
+timeout 300 python bench.py --ll --config C2 --steps 10 --warmup 3 > $OUT/${TAG}_bench_ll_C2.json 2>&1
+timeout 300 python bench.py --kde --config C2 --steps 10 --warmup 3 > $OUT/${TAG}_bench_kde_C2.json 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:window_kernel -s 2 -c 1 \
+    -o $OUT/${TAG}_window_C2 -f python bench.py --steps 1 --warmup 2 --no-cpu-baseline --no-alt > $OUT/${TAG}_ncu_full.log 2>&1
+echo done
