@@ -231,11 +231,19 @@ def run_ours(args):
             raise SystemExit("--gpus N>1 must be launched with torchrun (one rank per GPU)")
     if not torch.cuda.is_available():
         raise SystemExit("bench.py needs a CUDA device")
+    # KRCV_BENCH_BACKEND=gloo (and more ranks than GPUs, ranks wrapping onto
+    # the available devices) exercises the multi-rank code path on a one-GPU
+    # box; the timed configuration is NCCL, one rank per GPU
+    backend = os.environ.get("KRCV_BENCH_BACKEND", "nccl")
+    local = local % torch.cuda.device_count() if backend != "nccl" else local
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     from paper_conf_ipps_rohlfsz17_b200 import krcv
     from paper_conf_ipps_rohlfsz17_b200.api import GridSearch
 
