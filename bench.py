@@ -187,6 +187,11 @@ def run_reference(args):
     rank, world, _ = dist_env()
     if rank != 0:
         return 0
+    if world > 1 and os.environ.get("OMP_NUM_THREADS") == "1":
+        # torchrun pins OMP_NUM_THREADS=1 per rank; rank 0 alone runs the
+        # oracle here, on all of the host's cores (set before the oracle's
+        # OpenMP runtime loads)
+        os.environ["OMP_NUM_THREADS"] = str(len(os.sched_getaffinity(0)))
     cfg = workloads.CONFIGS[args.config]
     x, y, h, k = workloads.make(cfg, seed=args.seed)
     if args.kernel:
@@ -356,7 +361,8 @@ def run_ours(args):
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": workload_desc(cfg, args.seed), "n": n, "m": m,
                    "kernel": workloads.KERNEL_NAMES[k], "seed": args.seed,
-                   "parallelism": f"row-shard x{world}" + (" + nccl all_reduce(2m+2 fp64)" if world > 1 else ""),
+                   "parallelism": f"row-shard x{world}" + (
+                       f" + {os.environ.get('KRCV_BENCH_BACKEND', 'nccl')} all_reduce(2m+2 fp64)" if world > 1 else ""),
                    "l2": "flushed between timed steps (256 MiB write, outside the events)",
                    "launch": ("CUDA graph replay of the whole search (GridSearch(graph=True))" if world == 1
                               else "eager enqueue per step")},
