@@ -162,29 +162,33 @@ reduce_kernel(const double *__restrict__ tileS, const uint8_t *__restrict__ tile
               const unsigned *__restrict__ status, double *__restrict__ partial, FinOut fin)
 {
     __shared__ double sS[kReduceThreads];
+    __shared__ long long sN[kReduceThreads];
     __shared__ int sI[kReduceThreads];
     __shared__ bool last;
-    // one warp per bandwidth column: lane-strided over the tiles, then a fixed
-    // butterfly (no block barriers; the order is fixed, so bit-reproducible)
-    const int lane = threadIdx.x & 31;
-    const int gw = blockIdx.x * (kReduceThreads / 32) + (threadIdx.x >> 5);
-    const int nw = gridDim.x * (kReduceThreads / 32);
-    for (int b = gw; b < m; b += nw) {
+    for (int b = blockIdx.x; b < m; b += gridDim.x) {
         double a = 0.0;
-        unsigned cnt = 0;
+        long long cnt = 0;
         const double *col = tileS + (size_t)b * ntiles;
         const uint8_t *ncol = tileN + (size_t)b * ntiles;
-        for (int t = lane; t < ntiles; t += 32) {
+        for (int t = threadIdx.x; t < ntiles; t += kReduceThreads) {
             a += col[t];
             cnt += ncol[t];
         }
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
-        cnt = __reduce_add_sync(0xffffffffu, cnt);
-        if (lane == 0) {
-            partial[b] = a;
-            partial[m + b] = (double)cnt;
+        sS[threadIdx.x] = a;
+        sN[threadIdx.x] = cnt;
+        __syncthreads();
+        for (int s = kReduceThreads / 2; s > 0; s >>= 1) {
+            if (threadIdx.x < s) {
+                sS[threadIdx.x] += sS[threadIdx.x + s];
+                sN[threadIdx.x] += sN[threadIdx.x + s];
+            }
+            __syncthreads();
         }
+        if (threadIdx.x == 0) {
+            partial[b] = sS[0];
+            partial[m + b] = (double)sN[0];
+        }
+        __syncthreads();
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         partial[2 * m] = (double)status[0];
@@ -237,7 +241,6 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     L->xs = off;       off = align256(off + sizeof(double) * ((size_t)n + 2 * kPad));
     L->pfx = off;      off = align256(off + sizeof(double2) * kPfxMoments * (size_t)L->pstride);
     L->ptot = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
-    L->pflags = off;   off = align256(off + sizeof(unsigned) * (nch + 1));
     L->status = off;   off = align256(off + 8 * sizeof(unsigned));  // bad grid, non-finite, done, pad, u64 max|y| bits
     L->cub = off;      off = align256(off + cub_bytes);
     // m-dependent buffers last: everything above has the same offset for any
@@ -447,23 +450,6 @@ static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, cha
     double *P = reinterpret_cast<double *>(ws + L.pfx);
     double2 *tot = reinterpret_cast<double2 *>(ws + L.ptot);
     unsigned long long *ymax = reinterpret_cast<unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
-    static int two = -1;
-    if (two < 0) two = getenv_flag("KRCV_PFX_TWO") ? 1 : 0;  // A/B: the two-launch build
-    if (!two) {
-        unsigned *flags = reinterpret_cast<unsigned *>(ws + L.pflags);
-        if (pfx_items(n) == 1) {
-            const int ntiles = (n + kPfxThreads) / kPfxThreads;
-            cudaMemsetAsync(flags, 0, sizeof(unsigned) * (size_t)(ntiles + 1), st);
-            pfx_build_kernel<KERN, 1><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, flags, P, (int)L.pstride,
-                                                                      xs, ymax);
-        } else {
-            const int ntiles = (n + kPfxThreads * kPfxItemsMax) / (kPfxThreads * kPfxItemsMax);
-            cudaMemsetAsync(flags, 0, sizeof(unsigned) * (size_t)(ntiles + 1), st);
-            pfx_build_kernel<KERN, kPfxItemsMax><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, flags, P,
-                                                                                 (int)L.pstride, xs, ymax);
-        }
-        return;
-    }
     if (pfx_items(n) == 1) {
         const int ntiles = (n + kPfxThreads) / kPfxThreads;  // tiles covering P[0..n]
         pfx_tile_reduce_kernel<KERN, 1><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, ymax);
@@ -867,11 +853,8 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         }
     }
     prof_mark(3, st);
-    {
-        const int rb = (m + kReduceThreads / 32 - 1) / (kReduceThreads / 32);  // a warp per bandwidth
-        reduce_kernel<<<rb < 148 * 8 ? rb : 148 * 8, kReduceThreads, 0, st>>>(tileS, tileN, ntiles, m, status,
-                                                                               d_partial, fin);
-    }
+    reduce_kernel<<<m < 148 * 8 ? m : 148 * 8, kReduceThreads, 0, st>>>(tileS, tileN, ntiles, m, status,
+                                                                        d_partial, fin);
     launches += 1;
     prof_mark(4, st);
     g_prof.recorded = g_prof.on;

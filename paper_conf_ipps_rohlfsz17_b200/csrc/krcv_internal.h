@@ -32,7 +32,6 @@ struct WsLayout {
     size_t xs;                  // double  [n + 2 kPad] sorted x, +-inf sentinels (prefix path)
     size_t pfx;                 // double [8][2][pstride] dd prefix moments P[k][0..n], hi / lo planes
     size_t ptot;                // double2 [8][nch] prefix tile totals
-    size_t pflags;              // uint32 [nch + 1] one-launch prefix build: tile flags + ticket counter
     int64_t pstride, nch;
     size_t cub;                 // radix-sort scratch
     size_t cub_bytes;

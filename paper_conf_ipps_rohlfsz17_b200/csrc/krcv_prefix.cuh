@@ -285,137 +285,6 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
     }
 }
 
-// One-launch build (default): tiles take tickets from an atomic counter (so
-// a tile only waits on tiles already running or done), compute their
-// records' moment terms once, publish their dd totals, then wait for every
-// earlier tile's flag and sum those totals in the same fixed order as
-// pfx_tile_scan_kernel (strided per thread, fixed butterfly, fixed warp
-// order) -- bit-reproducible, no second launch, no second read of xy.
-// flags[0 .. ntiles) are per-tile "totals published", flags[ntiles] the
-// ticket counter; all zeroed by the host before the launch.
-template <int KERN, int ITEMS>
-__global__ void __launch_bounds__(kPfxThreads)
-pfx_build_kernel(const double2 *__restrict__ xy, int n, double2 *__restrict__ tot, int ntiles,
-                 unsigned *__restrict__ flags, double *__restrict__ P, int pstride, double *__restrict__ xs,
-                 unsigned long long *__restrict__ ymax_bits)
-{
-    constexpr int K = NMom<KERN>::v;
-    __shared__ double2 wsum[K][kPfxThreads / 32];
-    __shared__ double2 base_s[K];
-    __shared__ int tile_s;
-    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-    if (t == 0) tile_s = (int)atomicAdd(flags + ntiles, 1u);
-    __syncthreads();
-    const int tile = tile_s;
-    const int j0 = tile * (kPfxThreads * ITEMS) + t * ITEMS;
-    if (tile == 0 && t < kPad) {
-        xs[-1 - t] = -INFINITY;
-        xs[n + t] = INFINITY;
-    }
-    const double o = pfx_origin(xy, n);
-    // 1. moment terms, thread totals, max |y|
-    dd tm[ITEMS][kPfxMoments];
-    dd acc[kPfxMoments];
-#pragma unroll
-    for (int k = 0; k < K; k++) acc[k] = dd{0.0, 0.0};
-    double ym = 0.0;
-#pragma unroll
-    for (int q = 0; q < ITEMS; q++) {
-        if (j0 + q < n) {
-            const double2 v = xy[j0 + q];
-            xs[j0 + q] = v.x;
-            ym = fmax(ym, fabs(v.y));
-            moment_terms<KERN>(v.x, v.y, o, tm[q]);
-        } else {
-#pragma unroll
-            for (int k = 0; k < K; k++) tm[q][k] = dd{0.0, 0.0};
-        }
-#pragma unroll
-        for (int k = 0; k < K; k++) acc[k] = dd_add(acc[k], tm[q][k]);
-    }
-#pragma unroll
-    for (int d = 16; d > 0; d >>= 1) ym = fmax(ym, __shfl_xor_sync(0xffffffffu, ym, d));
-    if (lane == 0 && ym > 0.0) atomicMax(ymax_bits, (unsigned long long)__double_as_longlong(ym));
-    // 2. the tile total (fixed butterfly + fixed warp order) -> publish
-    {
-        dd a[kPfxMoments];
-#pragma unroll
-        for (int k = 0; k < K; k++) {
-            a[k] = acc[k];
-#pragma unroll
-            for (int d = 16; d > 0; d >>= 1) a[k] = dd_add(a[k], shfl_xor_dd(a[k], d));
-            if (lane == 0) st_dd(&wsum[k][w], a[k]);
-        }
-        __syncthreads();
-        if (t < K) {
-            dd b = dd{0.0, 0.0};
-            for (int q = 0; q < kPfxThreads / 32; q++) b = dd_add(b, ld_dd(&wsum[t][q]));
-            st_dd(tot + (size_t)t * ntiles + tile, b);
-            __threadfence();
-        }
-        __syncthreads();
-        if (t == 0) atomicExch(flags + tile, 1u);
-    }
-    // 3. this tile's offset: wait for the earlier tiles, sum their totals
-    {
-        for (int q = t; q < tile; q += kPfxThreads)
-            while (atomicAdd(flags + q, 0u) == 0u) {
-            }
-        __threadfence();
-        dd a[kPfxMoments];
-#pragma unroll
-        for (int k = 0; k < K; k++) {
-            a[k] = dd{0.0, 0.0};
-            for (int q = t; q < tile; q += kPfxThreads) {
-                const double2 v = __ldcg(tot + (size_t)k * ntiles + q);
-                a[k] = dd_add(a[k], dd{v.x, v.y});
-            }
-#pragma unroll
-            for (int d = 16; d > 0; d >>= 1) a[k] = dd_add(a[k], shfl_xor_dd(a[k], d));
-        }
-        __syncthreads();  // wsum reuse
-#pragma unroll
-        for (int k = 0; k < K; k++)
-            if (lane == 0) st_dd(&wsum[k][w], a[k]);
-        __syncthreads();
-        if (t < K) {
-            dd b = dd{0.0, 0.0};
-            for (int q = 0; q < kPfxThreads / 32; q++) b = dd_add(b, ld_dd(&wsum[t][q]));
-            st_dd(&base_s[t], b);
-        }
-        __syncthreads();
-    }
-    // 4. in-tile exclusive scan + offset -> P (as pfx_tile_scan_kernel)
-    dd ex[kPfxMoments];
-#pragma unroll
-    for (int k = 0; k < K; k++) {
-        dd inc = acc[k];
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const dd u = shfl_up_dd(inc, d);
-            if (lane >= d) inc = dd_add(u, inc);
-        }
-        if (lane == 31) st_dd(&wsum[k][w], inc);
-        const dd u = shfl_up_dd(inc, 1);
-        ex[k] = lane == 0 ? dd{0.0, 0.0} : u;
-    }
-    __syncthreads();
-#pragma unroll
-    for (int k = 0; k < K; k++) {
-        dd base = ld_dd(&base_s[k]);
-        for (int q = 0; q < w; q++) base = dd_add(base, ld_dd(&wsum[k][q]));
-        dd run = dd_add(base, ex[k]);
-#pragma unroll
-        for (int q = 0; q < ITEMS; q++) {
-            if (j0 + q <= n) {
-                P[(size_t)(2 * k) * pstride + j0 + q] = run.hi;
-                P[(size_t)(2 * k + 1) * pstride + j0 + q] = run.lo;
-            }
-            run = dd_add(run, tm[q][k]);
-        }
-    }
-}
-
 // ---------------------------------------------------------------- windows
 // New boundaries for bandwidth h from the previous ones, in offsets from the
 // row: the right side probes xs[r + k], the left side xs[r - k]; "inside" is
