@@ -96,7 +96,7 @@ __device__ __forceinline__ void ll_shift(const double *__restrict__ P, int ps, i
     dd Mu[5], My[4];
     double au[5], ay[4];
     Mu[0] = dd_make((double)(b - a));
-    au[0] = 0.0;  // the count is exact
+    au[0] = (double)(b - a);  // exact, but the Horner intermediates reach c' |delta|^k
 #pragma unroll
     for (int k = 1; k <= DU; k++) {
         const dd pb = ld_pdd(P, ps, k, b), pa = ld_pdd(P, ps, k, a);
@@ -145,6 +145,102 @@ __device__ __forceinline__ void ll_shift(const double *__restrict__ P, int ps, i
 // H a - b in dd (H, a, b dd): the S_k / T_k of the weighted sums
 __device__ __forceinline__ dd ll_comb(dd H, dd a, dd b) { return dd_sub(dd_mul(H, a), b); }
 
+// Plain-double fast path (uniform / Epanechnikov): the hi words of P only,
+// the binomial shift, S, T, det and num in double, with a bound of the same
+// form as the dd path's -- every prefix value carries <= 2^-53 relative
+// rounding (its dd lo part dropped), every Horner / fma step <= 2^-53 of the
+// magnitude it combines (kf = 2^-49 covers them with slack), and delta's own
+// rounding (only del.hi is used) shifts each d by |del.lo|, changing
+// sum d^k by <= k |del.lo| c' h^(k-1).  Returns false when the bound is not
+// below the dd path's tolerance (the caller then takes the dd path).
+template <int KERN>
+__device__ __forceinline__ bool ll_fast(const WinRow &w, int A, int R, int c, double h,
+                                        const double *__restrict__ P, int ps, double ymax, double &g)
+{
+    constexpr int DU = KERN == KR_UNIFORM ? 2 : 4, DY = KERN == KR_UNIFORM ? 1 : 3;
+    const double kf = 0x1p-49;
+    const double e = -w.del.hi, ad = fabs(w.del.hi), dlo = fabs(w.del.lo);
+    const double c1 = (double)(c + 1);  // points in [A, R), row r included
+    double U[5], aU[5], Yr[4], aY[4];
+    U[0] = c1;
+    aU[0] = c1;  // exact, but the Horner intermediates reach c' |delta|^k
+#pragma unroll
+    for (int k = 1; k <= DU; k++) {
+        const double pb = ld_hi(P, ps, k, R), pa = ld_hi(P, ps, k, A);
+        U[k] = pb - pa;
+        aU[k] = fabs(pb) + fabs(pa);
+    }
+#pragma unroll
+    for (int k = 0; k <= DY; k++) {
+        const int slot = k == 0 ? 0 : 4 + k;
+        const double pb = ld_hi(P, ps, slot, R), pa = ld_hi(P, ps, slot, A);
+        Yr[k] = pb - pa;
+        aY[k] = fabs(pb) + fabs(pa);
+    }
+    double D[5], eD[5], Y[4], eY[4];
+    double hp = 1.0;  // h^(k-1)
+#pragma unroll
+    for (int k = 1; k <= DU; k++) {
+        double acc = U[0], mag = aU[0], cb = 1.0;
+#pragma unroll
+        for (int i = 1; i <= k; i++) {
+            cb = cb * (double)(k - i + 1) / (double)i;
+            acc = fma(acc, e, cb * U[i]);
+            mag = fma(mag, ad, cb * aU[i]);
+        }
+        D[k] = acc;
+        eD[k] = fma(kf, mag + fabs(acc), 2.0 * k * dlo * c1 * hp);
+        hp *= h;
+    }
+    hp = 1.0;
+    const double ay0 = c1 * ymax;
+#pragma unroll
+    for (int k = 0; k <= DY; k++) {
+        double acc = Yr[0], mag = aY[0], cb = 1.0;
+#pragma unroll
+        for (int i = 1; i <= k; i++) {
+            cb = cb * (double)(k - i + 1) / (double)i;
+            acc = fma(acc, e, cb * Yr[i]);
+            mag = fma(mag, ad, cb * aY[i]);
+        }
+        if (k == 0) {  // LOO: drop row r's own y
+            acc -= w.yr;
+            mag += fabs(w.yr);
+        }
+        Y[k] = acc;
+        eY[k] = fma(kf, mag + fabs(acc), k > 0 ? 2.0 * k * dlo * ay0 * hp : 0.0);
+        if (k > 0) hp *= h;
+    }
+    double S0, S1, S2, T0, T1, eS0, eS1, eS2, eT0, eT1;
+    const double q = 0x1p-52;
+    if (KERN == KR_UNIFORM) {
+        S0 = (double)c; S1 = D[1]; S2 = D[2]; T0 = Y[0]; T1 = Y[1];
+        eS0 = 0.0; eS1 = eD[1]; eS2 = eD[2]; eT0 = eY[0]; eT1 = eY[1];
+    } else {
+        const double hh = h * h;
+        S0 = fma(hh, (double)c, -D[2]);
+        S1 = fma(hh, D[1], -D[3]);
+        S2 = fma(hh, D[2], -D[4]);
+        T0 = fma(hh, Y[0], -Y[2]);
+        T1 = fma(hh, Y[1], -Y[3]);
+        // hh's rounding (q hh |.|), the fma's (q |result|), the inputs' bounds
+        eS0 = eD[2] + q * (hh * (double)c + fabs(S0));
+        eS1 = fma(hh, eD[1], eD[3]) + q * (hh * fabs(D[1]) + fabs(S1));
+        eS2 = fma(hh, eD[2], eD[4]) + q * (hh * fabs(D[2]) + fabs(S2));
+        eT0 = fma(hh, eY[0], eY[2]) + q * (hh * fabs(Y[0]) + fabs(T0));
+        eT1 = fma(hh, eY[1], eY[3]) + q * (hh * fabs(Y[1]) + fabs(T1));
+    }
+    const double s11 = S1 * S1, s1t1 = S1 * T1;
+    const double dt = fma(S0, S2, -s11), nm = fma(S2, T0, -s1t1);
+    g = nm / dt;
+    const double aS0 = fabs(S0), aS1 = fabs(S1), aS2 = fabs(S2), aT0 = fabs(T0), aT1 = fabs(T1);
+    const double edet = aS2 * eS0 + aS0 * eS2 + 2.0 * aS1 * eS1 + eS0 * eS2 + eS1 * eS1 +
+                        q * (aS0 * aS2 + s11 + fabs(dt));
+    const double enum_ = aS2 * eT0 + aT0 * eS2 + aS1 * eT1 + aT1 * eS1 + eS2 * eT0 + eS1 * eT1 +
+                         q * (aS2 * aT0 + fabs(s1t1) + fabs(nm));
+    return dt > 0.0 && edet <= 0x1p-20 * dt && fma(fabs(g), edet, enum_) <= 0x1p-44 * dt * ymax;
+}
+
 // Local-linear g for row r, window [A, R) (c = R - A - 1 >= 2 points besides
 // r, at least two distinct x).  S_k, T_k, det and num stay in dd; the error
 // bounds eS, eT propagate the prefix errors, and dd rounding adds
@@ -159,6 +255,13 @@ __device__ __forceinline__ double ll_estimate(const WinRow &w, int A, int R, int
     if (c <= kLLDirect) {
         if (stats) atomicAdd(stats + 0, 1ull);
         return ll_direct<KERN>(xy, A, R, r, w.xr, h);
+    }
+    if (KERN != KR_TRIANGULAR) {
+        double gf;
+        if (ll_fast<KERN>(w, A, R, c, h, P, ps, ymax, gf)) {
+            if (stats) atomicAdd(stats + 1, 1ull);
+            return gf;
+        }
     }
     dd S0, S1, S2, T0, T1;
     double eS0, eS1, eS2, eT0, eT1;
@@ -232,8 +335,9 @@ __device__ __forceinline__ double ll_estimate(const WinRow &w, int A, int R, int
 // A warp owns 32 consecutive sorted rows (one per lane) and a chunk of the
 // bandwidth loop, as window_kernel<KERN, 1>; output in the same tile-partial
 // layout (reduce_kernel and the finalize are shared with Nadaraya-Watson).
-// stats (debug, nullable): counts of direct / prefix-accepted / prefix-
-// rejected (row, bandwidth) evaluations and the rejected windows' total size.
+// stats (debug, nullable): counts of direct / prefix-accepted (fast double
+// or dd) / prefix-rejected (row, bandwidth) evaluations and the rejected
+// windows' total size.
 template <int KERN>
 __global__ void __launch_bounds__(kWinThreads)
 ll_window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
