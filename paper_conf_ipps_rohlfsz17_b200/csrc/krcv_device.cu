@@ -392,20 +392,20 @@ static void prof_mark(int k, cudaStream_t st)
 static int64_t cub_sort_launches(int64_t n) { return n <= kCubSingleTile ? 1 : 2 + 64 / 8; }
 
 // Small-n sort chunk configuration: 0 = 256x4 (1024), 1 = 256x8 (2048),
-// 2 = 512x8 (4096), 3 = 256x2 (512) records per CTA.  Measured
-// (profiles/r01v_*): 1024 fastest for C2 and C3 -- smaller chunks sort faster
-// on more SMs, the extra chunk pairs of the rank step are cheap.
-// KRCV_CHUNK=0..3 overrides.
+// 2 = 512x8 (4096), 3 = 256x2 (512), 4 = 128x2 (256) records per CTA.
+// Measured (profiles/r01v_*, r01al_*): 1024 beats 2048 / 4096 at C2 and C3;
+// 512 beats 1024 at C2 (sort 26 -> 22 us) -- smaller chunks sort faster on
+// more SMs while the extra chunk pairs of the rank step stay cheap at small
+// n.  KRCV_CHUNK=0..4 overrides.
 int chunk_config(int64_t n)
 {
     static int forced = -1;
     if (forced < 0) {
         const char *e = getenv("KRCV_CHUNK");
-        forced = (e && e[0] >= '0' && e[0] <= '3') ? e[0] - '0' : 4;
+        forced = (e && e[0] >= '0' && e[0] <= '4') ? e[0] - '0' : 5;
     }
-    if (forced != 4) return forced;
-    (void)n;
-    return 0;
+    if (forced != 5) return forced;
+    return n <= 40000 ? 3 : 0;
 }
 
 template <int T, int I>
@@ -669,7 +669,7 @@ static int enqueue_sort(const double *d_x, const double *d_y, int64_t n, const d
     if (n <= kRankSortMaxN && !getenv_flag("KRCV_CUB_SORT")) {
         // a1 + a2: chunk merge sort, rank by counting across chunk pairs, scatter (krcv_sort.cuh)
         const int cfg = chunk_config(n);
-        const int chunk = cfg == 0 ? 1024 : (cfg == 1 ? 2048 : (cfg == 2 ? 4096 : 512));
+        const int chunk = cfg == 0 ? 1024 : (cfg == 1 ? 2048 : (cfg == 2 ? 4096 : (cfg == 3 ? 512 : 256)));
         const int nchunks = (int)((n + chunk - 1) / chunk);
         uint32_t *khi = reinterpret_cast<uint32_t *>(keys_out);          // keys_out is free on this path
         int *rank = reinterpret_cast<int *>(vals_out);                    // so is vals_out
@@ -677,7 +677,8 @@ static int enqueue_sort(const double *d_x, const double *d_y, int64_t n, const d
         case 0: launch_rank_sort<256, 4>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
         case 1: launch_rank_sort<256, 8>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
         case 2: launch_rank_sort<512, 8>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
-        default: launch_rank_sort<256, 2>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
+        case 3: launch_rank_sort<256, 2>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
+        default: launch_rank_sort<128, 2>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
         }
         const int npad = nchunks * chunk;
         rank_scatter_kernel<<<(npad + 255) / 256, 256, 0, st>>>(vals_in, rank, nn, npad, d_x, d_y, xy, perm,
