@@ -731,10 +731,6 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
 
     cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
     char *ws = static_cast<char *>(d_workspace);
-    uint64_t *keys_in = reinterpret_cast<uint64_t *>(ws + L.keys_in);
-    uint64_t *keys_out = reinterpret_cast<uint64_t *>(ws + L.keys_out);
-    uint32_t *vals_in = reinterpret_cast<uint32_t *>(ws + L.vals_in);
-    uint32_t *vals_out = reinterpret_cast<uint32_t *>(ws + L.vals_out);
     double2 *xy = reinterpret_cast<double2 *>(ws + L.xy) + kPad;  // first real record
     int *counter = reinterpret_cast<int *>(ws + L.counter);
     double *tileS = reinterpret_cast<double *>(ws + L.tileS);

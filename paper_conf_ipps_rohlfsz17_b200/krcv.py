@@ -20,7 +20,9 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libkrcv.so")
+# KRCV_LIB selects another in-tree build variant of the same library (A/B
+# measurements of compile-time options, tools/); default libkrcv.so
+LIB_PATH = os.path.join(_HERE, os.environ.get("KRCV_LIB", "libkrcv.so"))
 
 UNIFORM, EPANECHNIKOV, TRIANGULAR, GAUSSIAN = 0, 1, 2, 3
 KERNELS = {"uniform": UNIFORM, "epanechnikov": EPANECHNIKOV, "triangular": TRIANGULAR, "gaussian": GAUSSIAN}
