@@ -55,10 +55,6 @@ constexpr int kPfxThreads = 256;      // prefix build CTA
 constexpr int kPfxMoments = 8;        // slots reserved in the workspace (local-linear uses all 8)
 constexpr int kWinWarps = 4;
 constexpr int kWinThreads = kWinWarps * 32;
-#ifndef KRCV_WIN_MIN_BLOCKS
-#define KRCV_WIN_MIN_BLOCKS 1
-#endif
-constexpr int kWinMinBlocks = KRCV_WIN_MIN_BLOCKS;  // resident CTAs the register allocation must allow
 constexpr int kWinTasksPerSM = 256;   // warp tasks per SM the b-split aims for (measured: C3 nbc 7 -> 28, -9 %)
 constexpr int kWinMinBper = 8;        // >= this many bandwidths per task
 
@@ -579,7 +575,7 @@ __device__ __forceinline__ void window_advance(const double *__restrict__ xs, in
 // boundaries (window_bounds); each next row starts from its predecessor's
 // boundaries at the same bandwidth (window_advance, ~1 probe per side).
 template <int KERN, int K>
-__global__ void __launch_bounds__(kWinThreads, kWinMinBlocks)
+__global__ void __launch_bounds__(kWinThreads)
 window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
               int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
               int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
@@ -714,7 +710,7 @@ __device__ __forceinline__ void window_bounds2(const double *__restrict__ xs, in
 }
 
 template <int KERN>
-__global__ void __launch_bounds__(kWinThreads, kWinMinBlocks)
+__global__ void __launch_bounds__(kWinThreads)
 window_kernel_b2(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
                  int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
                  int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
