@@ -148,6 +148,17 @@ class ClockSampler:
                 "sm_max_mhz": self.max_mhz, "reasons": names, "samples": len(self.samples)}
 
 
+def ncu_traffic(config: str, algo: str):
+    """DRAM bytes per launch of the dominant kernel from the committed ncu
+    capture for this (config, algo) (profiles/ncu_traffic.json), else None."""
+    try:
+        with open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "ncu_traffic.json")) as f:
+            e = json.load(f).get(f"{config}/{algo}")
+        return None if e is None else e["bytes"]
+    except (OSError, ValueError, KeyError):
+        return None
+
+
 # --------------------------------------------------------------- cpu oracle
 def oracle_sample(x, y, h, k, target_s: float):
     """Time the oracle (Program-3 algorithm) on a bounded row sample of the
@@ -335,7 +346,8 @@ def run_ours(args):
             "stage_ms": {"pack_sort_gather": sum(sort_ms) / args.steps, "prefix_build": sum(build_ms) / args.steps,
                          "sweep": sum(main_ms) / args.steps, "reduce_finalize": sum(red_ms) / args.steps},
             "roofline": {"bound": "alu", "kernel": kname, "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
-                         "frac": achieved / peak, "traffic": None, "flops_per_launch": flops, "flops_basis": basis,
+                         "frac": achieved / peak, "traffic": ncu_traffic(args.config, used),
+                         "flops_per_launch": flops, "flops_basis": basis,
                          "peak_note": "FP64: 148 SM x 64 FMA lanes x 2 flop x 1965 MHz (derived, DESIGN.md)",
                          "kernel_ms": main_total / args.steps,
                          "kernel_share_of_step": main_total / total_ms},
