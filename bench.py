@@ -360,12 +360,6 @@ def run_ours(args):
 
     # ---- end-to-end through the public API, host buffers, H2D/D2H inside
     e2e = e2e_measure(args, x, y, h, k, n, m, units, dev, rank, world, plan)
-    traffic_json = os.path.join(ROOT, "profiles", "dram_traffic.json")
-    if os.path.exists(traffic_json):
-        try:
-            main["roofline"]["traffic"] = json.load(open(traffic_json)).get(args.config, {}).get(main["algo"])
-        except Exception:
-            pass
 
     out = {
         "metric": METRIC, "value": main["value"], "unit": UNIT, "n_gpus": world, "steps": args.steps,
