@@ -104,24 +104,31 @@ __device__ __forceinline__ void finalize_body(const double *partial, long long n
             bi = b;
         }
     }
-    sv[threadIdx.x] = bv;
-    si[threadIdx.x] = bi;
-    __syncthreads();
-    for (int s = THREADS / 2; s > 0; s >>= 1) {
-        if (threadIdx.x < s) {
-            const double ov = sv[threadIdx.x + s];
-            const int oi = si[threadIdx.x + s];
-            const int mi = si[threadIdx.x];
-            const double mv = sv[threadIdx.x];
-            if (oi >= 0 && (mi < 0 || ov < mv || (ov == mv && oi < mi))) {
-                sv[threadIdx.x] = ov;
-                si[threadIdx.x] = oi;
-            }
+    // (min value, lowest index) is associative and commutative: any tree
+    // gives the same index.  Butterfly per warp, then warp 0 over the warps.
+    auto take = [](double &mv, int &mi, double ov, int oi) {
+        if (oi >= 0 && (mi < 0 || ov < mv || (ov == mv && oi < mi))) {
+            mv = ov;
+            mi = oi;
         }
-        __syncthreads();
+    };
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1)
+        take(bv, bi, __shfl_xor_sync(0xffffffffu, bv, o), __shfl_xor_sync(0xffffffffu, bi, o));
+    if ((threadIdx.x & 31) == 0) {
+        sv[threadIdx.x >> 5] = bv;
+        si[threadIdx.x >> 5] = bi;
+    }
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        bv = threadIdx.x < THREADS / 32 ? sv[threadIdx.x] : 0.0;
+        bi = threadIdx.x < THREADS / 32 ? si[threadIdx.x] : -1;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1)
+            take(bv, bi, __shfl_xor_sync(0xffffffffu, bv, o), __shfl_xor_sync(0xffffffffu, bi, o));
     }
     if (threadIdx.x == 0) {
-        *best = si[0] < 0 ? 0 : si[0];
+        *best = bi < 0 ? 0 : bi;
         int st = KR_OK;
         if (__ldcg(partial + 2 * m) != 0.0) st = KR_EGRID;
         else if (__ldcg(partial + 2 * m + 1) != 0.0) st = KR_ENONFINITE;
@@ -174,19 +181,29 @@ reduce_kernel(const double *__restrict__ tileS, const uint8_t *__restrict__ tile
             a += col[t];
             cnt += ncol[t];
         }
-        sS[threadIdx.x] = a;
-        sN[threadIdx.x] = cnt;
-        __syncthreads();
-        for (int s = kReduceThreads / 2; s > 0; s >>= 1) {
-            if (threadIdx.x < s) {
-                sS[threadIdx.x] += sS[threadIdx.x + s];
-                sN[threadIdx.x] += sN[threadIdx.x + s];
-            }
-            __syncthreads();
+        // fixed tree: butterfly within each warp, then warp 0 adds the eight
+        // warp sums in order (bit-reproducible, one barrier)
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            a += __shfl_xor_sync(0xffffffffu, a, o);
+            cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
         }
+        const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+        if (lane == 0) {
+            sS[w] = a;
+            sN[w] = cnt;
+        }
+        __syncthreads();
         if (threadIdx.x == 0) {
-            partial[b] = sS[0];
-            partial[m + b] = (double)sN[0];
+            double t = 0.0;
+            long long c = 0;
+#pragma unroll
+            for (int q = 0; q < kReduceThreads / 32; q++) {
+                t += sS[q];
+                c += sN[q];
+            }
+            partial[b] = t;
+            partial[m + b] = (double)c;
         }
         __syncthreads();
     }
@@ -470,7 +487,8 @@ int win_rows_per_lane(int64_t rows)
     if (forced < 0) {
         const char *e = getenv("KRCV_WIN_K");
         const int k = e ? atoi(e) : 0;
-        forced = (k >= 1 && k <= 5) ? k : 0;  // 3: window_kernel_b2, 5: window_kernel_coop
+        forced = (k >= 1 && k <= 8) ? k : 0;  // 3: window_kernel_b2, 5: window_kernel_coop,
+                                              // 6/7/8: window_kernel_seg with 2/4/1 rows per lane
     }
     if (forced) return forced;
     // measured (profiles/r01t_*, r01u_*, r01af_*): two consecutive rows per
@@ -478,6 +496,17 @@ int win_rows_per_lane(int64_t rows)
     // lane with two bandwidths per step (window_kernel_b2: C3 1.73 -> 1.65 ms,
     // C4 22.9 -> 20.9 ms, C5 2.57 -> 2.43 ms)
     return rows <= 50000 ? 2 : 3;
+}
+
+// Rows per lane of window-kernel variant K (KRCV_WIN_K numbering).
+static int win_lane_rows(int K)
+{
+    switch (K) {
+    case 3: case 5: case 8: return 1;
+    case 6: return 2;
+    case 7: return 4;
+    default: return K;
+    }
 }
 
 template <int KERN, int K>
@@ -492,6 +521,9 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_b2<KERN>, kWinThreads, 0);
         else if (K == 5)
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_coop<KERN>, kCoopRows, 0);
+        else if (K >= 6)
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_seg<KERN, K == 6 ? 2 : (K == 7 ? 4 : 1)>,
+                                                          kWinThreads, 0);
         else
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel<KERN, K>, kWinThreads, 0);
         resident = b > 0 ? b : 1;
@@ -527,6 +559,9 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
     else if (K == 5)
         window_kernel_coop<KERN><<<blocks, kCoopRows, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
                                                                nbc, ymax, tileS, tileN, counter);
+    else if (K >= 6)
+        window_kernel_seg<KERN, K == 6 ? 2 : (K == 7 ? 4 : 1)><<<blocks, kWinThreads, 0, st>>>(
+            xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter);
     else
         window_kernel<KERN, (K == 3 || K == 5) ? 1 : K><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo,
                                                                             hi, ntiles, nbc, ymax, tileS, tileN,
@@ -543,6 +578,9 @@ static void launch_window(int K, const double2 *xy, int n, const double *h, int 
     case 2: launch_window_k<KERN, 2>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     case 3: launch_window_k<KERN, 3>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     case 5: launch_window_k<KERN, 5>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    case 6: launch_window_k<KERN, 6>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    case 7: launch_window_k<KERN, 7>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    case 8: launch_window_k<KERN, 8>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     default: launch_window_k<KERN, 4>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     }
 }
@@ -758,7 +796,7 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     int G = sweep_G(hi - lo);
     if (variant == 1 && G > 4) G = 4;
     const int winK = ll ? 1 : win_rows_per_lane(hi - lo);
-    const int rows_per_tile = 32 * ((winK == 3 || winK == 5) ? 1 : winK);
+    const int rows_per_tile = 32 * win_lane_rows(winK);
     const int ntiles = hist ? (int)((hi - lo + 31) / 32)
                      : prefix ? (int)((hi - lo + rows_per_tile - 1) / rows_per_tile)
                               : dense ? (int)tiles_for(hi - lo, 1)

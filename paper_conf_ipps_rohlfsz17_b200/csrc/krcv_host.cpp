@@ -40,13 +40,14 @@ struct DevCtx {
     double *dx = nullptr, *dy = nullptr, *dh = nullptr;
     int64_t cap_n = 0;
     int32_t cap_m = 0;
-    double *dpartial = nullptr, *dcv = nullptr;
+    double *dpartial = nullptr;
+    // results of the synchronous host path, one block [best, status | cv[m] |
+    // neff[m]] on the device and its pinned mirror: one D2H copy per call
+    char *dres = nullptr;
+    double *dcv = nullptr;
     int64_t *dneff = nullptr;
     int32_t *dbest = nullptr;  // [2]: best, status
-    // pinned staging for the results of the synchronous host path
-    double *pcv = nullptr;
-    int64_t *pneff = nullptr;
-    int32_t *pbs = nullptr;
+    char *pres = nullptr;
     int32_t pcap_m = 0;
     // CUDA graph of the last synchronous call whose inputs were pinned
     // (H2D copies, the whole device pipeline, D2H copies): replayed while
@@ -77,6 +78,9 @@ static DevCtx *get_ctx(int dev)
         }                                                   \
     } while (0)
 
+// [best, status] (8 B) | cv[m] | neff[m]
+static size_t res_bytes(int32_t m) { return 8 + (sizeof(double) + sizeof(int64_t)) * (size_t)m; }
+
 static int ensure_capacity(DevCtx *c, int64_t n, int32_t m)
 {
     if (!c->stream) KR_CUDA_TRY(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
@@ -92,18 +96,18 @@ static int ensure_capacity(DevCtx *c, int64_t n, int32_t m)
     if (m > c->cap_m) {
         cudaFree(c->dh);
         cudaFree(c->dpartial);
-        cudaFree(c->dcv);
-        cudaFree(c->dneff);
-        cudaFree(c->dbest);
+        cudaFree(c->dres);
         c->dh = c->dpartial = c->dcv = nullptr;
+        c->dres = nullptr;
         c->dneff = nullptr;
         c->dbest = nullptr;
         c->cap_m = 0;
         KR_CUDA_TRY(cudaMalloc(&c->dh, sizeof(double) * m));
         KR_CUDA_TRY(cudaMalloc(&c->dpartial, sizeof(double) * KR_PARTIAL_LEN(m)));
-        KR_CUDA_TRY(cudaMalloc(&c->dcv, sizeof(double) * m));
-        KR_CUDA_TRY(cudaMalloc(&c->dneff, sizeof(int64_t) * m));
-        KR_CUDA_TRY(cudaMalloc(&c->dbest, sizeof(int32_t) * 2));
+        KR_CUDA_TRY(cudaMalloc(&c->dres, res_bytes(m)));
+        c->dbest = reinterpret_cast<int32_t *>(c->dres);
+        c->dcv = reinterpret_cast<double *>(c->dres + 8);
+        c->dneff = reinterpret_cast<int64_t *>(c->dres + 8 + sizeof(double) * m);
         c->cap_m = m;
     }
     size_t need = kr_workspace_bytes(n, m);
@@ -158,16 +162,10 @@ static bool is_pinned(const void *p)
 static int ensure_staging(DevCtx *c, int32_t m)
 {
     if (m <= c->pcap_m) return KR_OK;
-    cudaFreeHost(c->pcv);
-    cudaFreeHost(c->pneff);
-    cudaFreeHost(c->pbs);
-    c->pcv = nullptr;
-    c->pneff = nullptr;
-    c->pbs = nullptr;
+    cudaFreeHost(c->pres);
+    c->pres = nullptr;
     c->pcap_m = 0;
-    KR_CUDA_TRY(cudaMallocHost(&c->pcv, sizeof(double) * m));
-    KR_CUDA_TRY(cudaMallocHost(&c->pneff, sizeof(int64_t) * m));
-    KR_CUDA_TRY(cudaMallocHost(&c->pbs, sizeof(int32_t) * 2));
+    KR_CUDA_TRY(cudaMallocHost(&c->pres, res_bytes(m)));
     c->pcap_m = m;
     return KR_OK;
 }
@@ -182,14 +180,16 @@ static int enqueue_host_call(DevCtx *c, const double *x, const double *y, int64_
     KR_CUDA_TRY(cudaMemcpyAsync(c->dx, x, sizeof(double) * n, cudaMemcpyHostToDevice, s));
     KR_CUDA_TRY(cudaMemcpyAsync(c->dy, y, sizeof(double) * n, cudaMemcpyHostToDevice, s));
     KR_CUDA_TRY(cudaMemcpyAsync(c->dh, h, sizeof(double) * m, cudaMemcpyHostToDevice, s));
-    const int st = ll ? kr_ll_cv_grid_async(c->dx, c->dy, n, c->dh, m, kernel, c->dcv, c->dneff, c->dbest, c->ws,
+    // the result block laid out for this call's m (fits the capacity's)
+    int32_t *dbest = reinterpret_cast<int32_t *>(c->dres);
+    double *dcv = reinterpret_cast<double *>(c->dres + 8);
+    int64_t *dneff = reinterpret_cast<int64_t *>(c->dres + 8 + sizeof(double) * m);
+    const int st = ll ? kr_ll_cv_grid_async(c->dx, c->dy, n, c->dh, m, kernel, dcv, dneff, dbest, c->ws,
                                             c->ws_bytes, s)
-                      : kr_cv_grid_async(c->dx, c->dy, n, c->dh, m, kernel, algo, c->dcv, c->dneff, c->dbest, c->ws,
+                      : kr_cv_grid_async(c->dx, c->dy, n, c->dh, m, kernel, algo, dcv, dneff, dbest, c->ws,
                                          c->ws_bytes, s);
     if (st) return st;
-    KR_CUDA_TRY(cudaMemcpyAsync(c->pcv, c->dcv, sizeof(double) * m, cudaMemcpyDeviceToHost, s));
-    KR_CUDA_TRY(cudaMemcpyAsync(c->pneff, c->dneff, sizeof(int64_t) * m, cudaMemcpyDeviceToHost, s));
-    KR_CUDA_TRY(cudaMemcpyAsync(c->pbs, c->dbest, sizeof(int32_t) * 2, cudaMemcpyDeviceToHost, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(c->pres, c->dres, res_bytes(m), cudaMemcpyDeviceToHost, s));  // one copy
     return KR_OK;
 }
 
@@ -250,10 +250,11 @@ static int host_call(const double *x, const double *y, int64_t n, const double *
         if (st) return st;
     }
     KR_CUDA_TRY(cudaStreamSynchronize(s));
-    if (c->pbs[1] != KR_OK) return c->pbs[1];
-    std::memcpy(cv_out, c->pcv, sizeof(double) * m);
-    if (neff_out) std::memcpy(neff_out, c->pneff, sizeof(int64_t) * m);
-    *best_out = c->pbs[0];
+    const int32_t *pbs = reinterpret_cast<const int32_t *>(c->pres);  // layout of enqueue_host_call
+    if (pbs[1] != KR_OK) return pbs[1];
+    std::memcpy(cv_out, c->pres + 8, sizeof(double) * m);
+    if (neff_out) std::memcpy(neff_out, c->pres + 8 + sizeof(double) * m, sizeof(int64_t) * m);
+    *best_out = pbs[0];
     return KR_OK;
 }
 

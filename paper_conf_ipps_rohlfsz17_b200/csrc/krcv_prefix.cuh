@@ -779,6 +779,251 @@ window_kernel_b2(const double *__restrict__ xs, const double2 *__restrict__ xy, 
 }
 
 // ---------------------------------------------------------------------------
+// Segment variant (window_kernel_seg<K, KR>): the boundary searches of a
+// warp's 32 KR consecutive rows read one shared-memory segment per side
+// instead of probing global memory one dependent load at a time.
+//
+// Both boundaries are monotone in the row: R_j (first index right of j
+// outside the window) and L_j (last index left of j outside) never decrease
+// as x_j grows, and at a larger bandwidth R_j grows and L_j shrinks.  So at
+// h_b every right boundary of the tile lies between the first row's and the
+// last row's, and those move by about the previous step's growth g.  Per
+// bandwidth the warp
+//   1. predicts the segment [S, E] of the sorted x that holds all the tile's
+//      right boundaries (first row's previous R + g - 3 sqrt g ... last row's
+//      previous R + g + 3 sqrt g), likewise for the left;
+//   2. loads it coalesced into its shared-memory slice (one round trip);
+//   3. verifies the prediction exactly -- xs[S] inside the first row's window
+//      (hence every row's) and xs[E] outside the last row's (hence every
+//      row's), the mirror conditions on the left -- with the same binary64
+//      predicate (reading Q1);
+//   4. every lane bisects its first row's boundaries in shared memory (lower
+//      end: the row's previous boundary) and advances its next rows from
+//      their predecessor's (typically 0-2 steps).
+// A failed check or a segment longer than kSegMax (sparse tiles) falls back,
+// warp-uniformly, to the global searches of window_kernel for that
+// bandwidth; the first bandwidth of a chunk always does (no prediction yet).
+// The boundaries found are the same indices either way, so the window sums
+// and the emitted partials are bit-identical to window_kernel's.
+constexpr int kSegMax = 512;
+
+__device__ __forceinline__ int seg_spread(int g) { return (int)(3.0f * sqrtf((float)g)) + 2; }
+
+// first q in (lo, hi] with seg[q] outside the right window of (xr, h);
+// lo inside, hi outside.  Gallops from lo (the next row's boundary usually
+// moves by 0-2), then bisects.
+template <int KERN>
+__device__ __forceinline__ int seg_first_out(const double *seg, int lo, int hi, double xr, double h)
+{
+    int step = 1;
+    for (;;) {
+        const int k = min(lo + step, hi);
+        if (k == hi) break;
+        if (!inside<KERN>(seg[k] - xr, h)) { hi = k; break; }
+        lo = k;
+        step <<= 1;
+    }
+    while (hi - lo > 1) {
+        const int k = (lo + hi) >> 1;
+        if (inside<KERN>(seg[k] - xr, h)) lo = k; else hi = k;
+    }
+    return hi;
+}
+
+// last q in [lo, hi) with seg[q] outside the left window of (xr, h); lo
+// outside, hi inside.  Gallop from lo, then bisect.
+template <int KERN>
+__device__ __forceinline__ int seg_last_out(const double *seg, int lo, int hi, double xr, double h)
+{
+    int step = 1;
+    for (;;) {
+        const int k = min(lo + step, hi);
+        if (k == hi) break;
+        if (inside<KERN>(xr - seg[k], h)) { hi = k; break; }
+        lo = k;
+        step <<= 1;
+    }
+    while (hi - lo > 1) {
+        const int k = (lo + hi) >> 1;
+        if (!inside<KERN>(xr - seg[k], h)) lo = k; else hi = k;
+    }
+    return lo;
+}
+
+template <int KERN, int KR>
+__global__ void __launch_bounds__(kWinThreads)
+window_kernel_seg(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
+                  int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
+                  int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
+                  uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
+{
+    __shared__ double s_seg[kWinWarps][2][kSegMax];
+    const int lane = threadIdx.x & 31;
+    double *segR = s_seg[threadIdx.x >> 5][0];
+    double *segL = s_seg[threadIdx.x >> 5][1];
+    const double o = pfx_origin(xy, n);
+    const double ymax = __longlong_as_double((long long)*ymax_bits);
+    const int bper = (m + nbc - 1) / nbc;
+    const int ps = pstride;
+    for (;;) {
+        int task = 0;
+        if (lane == 0) task = atomicAdd(tile_counter, 1);
+        task = __shfl_sync(0xffffffffu, task, 0);
+        if (task >= ntiles * nbc) return;  // warp-uniform
+        const int chunk = task / ntiles;  // chunk-major (see window_kernel)
+        const int tile = task - chunk * ntiles;
+        const int b0 = chunk * bper, b1 = min(m, b0 + bper);
+
+        const int i0 = row_lo + tile * 32 * KR + lane * KR;
+        WinRow rows[KR];
+        int nvalid = 0;
+#pragma unroll
+        for (int k = 0; k < KR; k++) {
+            const int i = i0 + k;
+            nvalid += i < row_hi ? 1 : 0;
+            rows[k].r = min(i, row_hi - 1);  // clamped rows do identical work, discarded
+            const double2 v = xy[rows[k].r];
+            rows[k].xr = v.x;
+            rows[k].yr = v.y;
+            rows[k].del = two_sum(v.x, -o);
+        }
+        // the tile's first and last row (monotonicity anchors of the checks)
+        const double xfirst = __shfl_sync(0xffffffffu, rows[0].xr, 0);
+        const double xlast = __shfl_sync(0xffffffffu, rows[KR - 1].xr, 31);
+        // this lane's first row: boundaries (absolute) and growth at the previous bandwidth
+        int R0 = rows[0].r + 1, L0 = rows[0].r - 1;
+        int gR = cold_step(xs, n, __ldg(hg + b0)), gL = gR;
+        // warp-level anchors: first row's R/L, last row's R/L and their growth
+        int Rf = 0, Rl = 0, Lf = 0, Ll = 0, gRf = 0, gRl = 0, gLf = 0, gLl = 0;
+        double hprev = 0.0;
+
+        for (int b = b0; b < b1; b++) {
+            const double h = __ldg(hg + b);
+            if (b == b0 + 1) {  // no growth observed yet: density estimate from the first windows
+                const double f = (h - hprev) / hprev;
+                const int rf = __shfl_sync(0xffffffffu, rows[0].r, 0), rl = __shfl_sync(0xffffffffu, rows[KR - 1].r, 31);
+                gRf = (int)fmin(ceil((Rf - rf) * f), (double)n);
+                gRl = (int)fmin(ceil((Rl - rl) * f), (double)n);
+                gLf = (int)fmin(ceil((rf - Lf) * f), (double)n);
+                gLl = (int)fmin(ceil((rl - Ll) * f), (double)n);
+            }
+            int Rk[KR], Lk[KR];
+            bool seg_ok = false;
+            if (b > b0) {
+                // 1. predicted segments (warp-uniform)
+                const bool rfull = Rf >= n, lfull = Ll <= -1;  // every row's window reaches the end
+                // (64-bit: growth and spread may reach n each)
+                int S = (int)min((long long)Rf - 1 + max(0, gRf - seg_spread(gRf)), (long long)n);
+                const int E = (int)min((long long)n, (long long)Rl + gRl + seg_spread(gRl));
+                S = min(S, E);
+                const int SL = (int)max(-1LL, (long long)Lf - gLf - seg_spread(gLf));
+                int EL = Ll + 1 - max(0, gLl - seg_spread(gLl));
+                EL = max(EL, SL);
+                const int lenR = rfull ? 1 : E - S + 1, lenL = lfull ? 1 : EL - SL + 1;
+                if (lenR <= kSegMax && lenL <= kSegMax) {
+                    // 2. coalesced loads into the warp's slice
+                    __syncwarp();
+                    if (!rfull)
+                        for (int q = lane; q < lenR; q += 32) segR[q] = __ldg(xs + S + q);
+                    if (!lfull)
+                        for (int q = lane; q < lenL; q += 32) segL[q] = __ldg(xs + SL + q);
+                    __syncwarp();
+                    // 3. exact check of the prediction
+                    bool ok = true;
+                    if (!rfull) ok = ok && inside<KERN>(segR[0] - xfirst, h) && !inside<KERN>(segR[lenR - 1] - xlast, h);
+                    if (!lfull) ok = ok && !inside<KERN>(xfirst - segL[0], h) && inside<KERN>(xlast - segL[lenL - 1], h);
+                    seg_ok = ok;  // identical in every lane (same loads, same predicate)
+                    if (ok) {
+                        // 4. per-lane searches in shared memory
+#pragma unroll
+                        for (int k = 0; k < KR; k++) {
+                            const double xr = rows[k].xr;
+                            if (rfull) {
+                                Rk[k] = n;
+                            } else {
+                                // lower end: row 0 its previous boundary - 1, row k its predecessor's - 1
+                                if (k == 0) {  // bisect (previous R - 1 is inside)
+                                    int lo = max(0, R0 - 1 - S), hh = lenR - 1;
+                                    while (hh - lo > 1) {
+                                        const int q = (lo + hh) >> 1;
+                                        if (inside<KERN>(segR[q] - xr, h)) lo = q; else hh = q;
+                                    }
+                                    Rk[0] = S + hh;
+                                } else {  // gallop from the predecessor's boundary
+                                    Rk[k] = S + seg_first_out<KERN>(segR, Rk[k - 1] - 1 - S, lenR - 1, xr, h);
+                                }
+                            }
+                            if (lfull) {
+                                Lk[k] = -1;
+                            } else if (k == 0) {
+                                // row 0: last outside in [0, previous L + 1 - SL]; previous L + 1 is inside
+                                const int hi = min(lenL - 1, L0 + 1 - SL);
+                                int lo = 0, hh = hi;
+                                while (hh - lo > 1) {
+                                    const int q = (lo + hh) >> 1;
+                                    if (!inside<KERN>(xr - segL[q], h)) lo = q; else hh = q;
+                                }
+                                Lk[0] = SL + lo;
+                            } else {
+                                Lk[k] = SL + seg_last_out<KERN>(segL, Lk[k - 1] - SL, lenL - 1, xr, h);
+                            }
+                        }
+                    }
+                }
+            }
+            if (!seg_ok) {  // global searches (window_kernel's)
+                int kR = R0 - rows[0].r, kL = rows[0].r - L0;
+                window_bounds<KERN>(xs, n, rows[0].r, rows[0].xr, h, kR, kL, gR, gL);
+                int R = rows[0].r + kR, L = rows[0].r - kL;
+                Rk[0] = R;
+                Lk[0] = L;
+#pragma unroll
+                for (int k = 1; k < KR; k++) {
+                    if (rows[k].r != rows[k - 1].r) window_advance<KERN>(xs, n, rows[k].r, rows[k].xr, h, R, L);
+                    Rk[k] = R;
+                    Lk[k] = L;
+                }
+            }
+            gR = max(1, Rk[0] - R0);
+            gL = max(1, L0 - Lk[0]);
+            R0 = Rk[0];
+            L0 = Lk[0];
+            {
+                const int nRf = __shfl_sync(0xffffffffu, Rk[0], 0), nLf = __shfl_sync(0xffffffffu, Lk[0], 0);
+                const int nRl = __shfl_sync(0xffffffffu, Rk[KR - 1], 31), nLl = __shfl_sync(0xffffffffu, Lk[KR - 1], 31);
+                if (b > b0) {
+                    gRf = nRf - Rf;
+                    gRl = nRl - Rl;
+                    gLf = Lf - nLf;
+                    gLl = Ll - nLl;
+                }
+                Rf = nRf;
+                Rl = nRl;
+                Lf = nLf;
+                Ll = nLl;
+            }
+            hprev = h;
+            double e2 = 0.0;
+            int cntM = 0;
+#pragma unroll
+            for (int k = 0; k < KR; k++) {
+                const int c = Rk[k] - Lk[k] - 2;
+                if (k < nvalid && c > 0) {  // reading Q6
+                    e2 += window_e2<KERN>(rows[k], Lk[k] + 1, Rk[k], c, h, xy, P, ps, ymax);
+                    cntM += 1;
+                }
+            }
+            e2 = warp_sum(e2);
+            const int cnt = __reduce_add_sync(0xffffffffu, cntM);  // <= 32 KR <= 128: fits the u8 slot
+            if (lane == 0) {
+                tileS[(size_t)b * ntiles + tile] = e2;
+                tileN[(size_t)b * ntiles + tile] = (uint8_t)cnt;
+            }
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
 // Cooperative variant (window_kernel_coop): a CTA owns kCoopRows = 128
 // consecutive sorted rows and a chunk of the bandwidth loop.  Per bandwidth:
 //   1. four "leader" boundaries -- right and left boundary of the tile's first

@@ -8,7 +8,7 @@ from __future__ import annotations
 
 import numpy as np
 import pytest
-from hypothesis import HealthCheck, given, settings
+from hypothesis import HealthCheck, example, given, settings
 from hypothesis import strategies as st
 
 import oracle
@@ -48,20 +48,35 @@ def problems(draw):
     return x, y, h
 
 
-SETTINGS = settings(max_examples=40, deadline=None, suppress_health_check=[HealthCheck.too_slow])
+# derandomize: the same examples on every run (the round-end GPU run must be
+# reproducible); the example set was widened instead (max_examples)
+SETTINGS = settings(max_examples=60, deadline=None, derandomize=True, database=None,
+                    suppress_health_check=[HealthCheck.too_slow])
+
+
+def zero_floor(y) -> float:
+    """Floor for exact-zero CV (constant y, P6; helpers.cv_rel_err): fp64 noise
+    there is ~1e-32 max y^2 (measured 1.4e-32 y^2, hist/triangular, n = 2), and
+    TOL times the floor must exceed it; 1e-20 max y^2 allows 1e-29 y^2 at
+    TOL = 1e-9, while one misplaced window member changes CV by O(y^2 / n)."""
+    return 1e-20 * float(np.max(np.asarray(y) ** 2))
 
 
 @pytest.mark.parametrize("algo", ["sweep", "prefix", "hist"])
 @pytest.mark.parametrize("k", [0, 1, 2])
 @SETTINGS
 @given(p=problems())
+# found by random runs: constant y, exact CV 0, the oracle's triangular
+# quotient leaves 4.7e-38, the GPU's 4.9e-32 (zero_floor)
+@example(p=(np.array([0.0, 1.625]), np.array([3.0, 3.0]), np.array([3.0])))
+@example(p=(np.array([0.0, 0.0]), np.array([1.875, 1.875]), np.array([2.18257963])))
 def test_property_nw(algo, k, p):
     x, y, h = p
     cv, neff, best = krcv.kr_cv_grid(x, y, h, k, with_neff=True, algo=algo)
     ref = oracle.cv_direct(x, y, h, k)
     assert np.array_equal(neff, ref.neff)
-    assert cv_rel_err(cv, ref.cv) <= TOL
-    assert best_ok(best, ref.cv, 1e-9)
+    assert cv_rel_err(cv, ref.cv, zero_floor(y)) <= TOL
+    assert best_ok(best, ref.cv, 1e-9, zero_floor(y))
 
 
 @pytest.mark.parametrize("k", [0, 1, 2])
@@ -72,8 +87,8 @@ def test_property_local_linear(k, p):
     cv, neff, best = krcv.kr_ll_cv_grid(x, y, h, k, with_neff=True)
     ref = oracle.ll_cv(x, y, h, k)
     assert np.array_equal(neff, ref.neff)
-    assert cv_rel_err(cv, ref.cv) <= 1e-7  # ill-conditioned 2-point fits amplify rounding
-    assert best_ok(best, ref.cv, 1e-7)
+    assert cv_rel_err(cv, ref.cv, zero_floor(y)) <= 1e-7  # ill-conditioned 2-point fits amplify rounding
+    assert best_ok(best, ref.cv, 1e-7, zero_floor(y))
 
 
 @SETTINGS
@@ -83,4 +98,4 @@ def test_property_gaussian(p):
     cv, neff, best = krcv.kr_cv_grid(x, y, h, 3, with_neff=True)
     ref = oracle.cv_direct(x, y, h, 3)
     assert np.array_equal(neff, ref.neff)
-    assert cv_rel_err(cv, ref.cv) <= TOL
+    assert cv_rel_err(cv, ref.cv, zero_floor(y)) <= TOL
