@@ -487,8 +487,9 @@ int win_rows_per_lane(int64_t rows)
     if (forced < 0) {
         const char *e = getenv("KRCV_WIN_K");
         const int k = e ? atoi(e) : 0;
-        forced = (k >= 1 && k <= 8) ? k : 0;  // 3: window_kernel_b2, 5: window_kernel_coop,
-                                              // 6/7/8: window_kernel_seg with 2/4/1 rows per lane
+        forced = (k >= 1 && k <= 10) ? k : 0;  // 3: window_kernel_b2, 5: window_kernel_coop,
+                                               // 6/7/8: window_kernel_seg with 2/4/1 rows per lane,
+                                               // 9/10: window_kernel_blk with 2/4 blocks of 32 rows
     }
     if (forced) return forced;
     // measured (profiles/r01t_*, r01u_*, r01af_*): two consecutive rows per
@@ -503,8 +504,8 @@ static int win_lane_rows(int K)
 {
     switch (K) {
     case 3: case 5: case 8: return 1;
-    case 6: return 2;
-    case 7: return 4;
+    case 6: case 9: return 2;
+    case 7: case 10: return 4;
     default: return K;
     }
 }
@@ -521,6 +522,8 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_b2<KERN>, kWinThreads, 0);
         else if (K == 5)
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_coop<KERN>, kCoopRows, 0);
+        else if (K >= 9)
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_blk<KERN, K == 9 ? 2 : 4>, kWinThreads, 0);
         else if (K >= 6)
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_seg<KERN, K == 6 ? 2 : (K == 7 ? 4 : 1)>,
                                                           kWinThreads, 0);
@@ -559,6 +562,9 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
     else if (K == 5)
         window_kernel_coop<KERN><<<blocks, kCoopRows, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
                                                                nbc, ymax, tileS, tileN, counter);
+    else if (K >= 9)
+        window_kernel_blk<KERN, K == 9 ? 2 : 4><<<blocks, kWinThreads, 0, st>>>(
+            xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter);
     else if (K >= 6)
         window_kernel_seg<KERN, K == 6 ? 2 : (K == 7 ? 4 : 1)><<<blocks, kWinThreads, 0, st>>>(
             xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter);
@@ -581,6 +587,8 @@ static void launch_window(int K, const double2 *xy, int n, const double *h, int 
     case 6: launch_window_k<KERN, 6>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     case 7: launch_window_k<KERN, 7>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     case 8: launch_window_k<KERN, 8>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    case 9: launch_window_k<KERN, 9>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    case 10: launch_window_k<KERN, 10>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     default: launch_window_k<KERN, 4>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     }
 }

@@ -1179,4 +1179,162 @@ window_kernel_coop(const double *__restrict__ xs, const double2 *__restrict__ xy
     }
 }
 
+// ---------------------------------------------------------------------------
+// Block variant (window_kernel_blk<K, KB>): lanes hold CONSECUTIVE rows (lane l
+// row base + 32 k + l of block k), and each block's boundary searches start
+// from an exact lower bound instead of a prediction.  Because R_j and L_j are
+// monotone in the row, the boundaries of block k lie at or beyond those of the
+// previous block's last row (lane 31): the segment xs[S .. S + 63] starting
+// there is loaded coalesced (two doubles per lane, one round trip) and every
+// lane finds its boundary in it by a 6-step branchless bisection over warp
+// shuffles.  Lanes whose boundary lies beyond the 64-element segment (sparse
+// data) continue with their own gallop from its end.  Block 0's lower bounds
+// are the tile's first row's own boundaries, found by one warp-cooperative
+// 32-ary search per side (warp_boundary) from the previous bandwidth's.
+// Same predicate (reading Q1), same windows, same window_e2 as window_kernel;
+// the tile groups 32 KB consecutive rows like window_kernel<K, KB>, but a
+// lane sums different rows, so CV agrees with it to rounding, not bitwise.
+
+// first outside right of absolute index lo (inside for row (r, xr), or lo = r)
+template <int KERN>
+__device__ __forceinline__ int right_from(const double *__restrict__ xs, int n, double xr, double h, int lo)
+{
+    int step = 1, hi;
+    for (;;) {
+        const int k = min(lo + step, n);  // xs[n] = +inf: outside
+        if (!inside<KERN>(__ldg(xs + k) - xr, h)) { hi = k; break; }
+        lo = k;
+        step <<= 1;
+    }
+    while (hi - lo > 1) {
+        const int k = (lo + hi) >> 1;
+        if (inside<KERN>(__ldg(xs + k) - xr, h)) lo = k; else hi = k;
+    }
+    return hi;
+}
+
+// last outside left of row r at or after absolute index lo (outside for (r, xr))
+template <int KERN>
+__device__ __forceinline__ int left_from(const double *__restrict__ xs, int r, double xr, double h, int lo)
+{
+    int step = 1, hi;
+    for (;;) {
+        const int k = min(lo + step, r);  // r itself is inside (d = 0)
+        if (k == r || inside<KERN>(xr - __ldg(xs + k), h)) { hi = k; break; }
+        lo = k;
+        step <<= 1;
+    }
+    while (hi - lo > 1) {
+        const int k = (lo + hi) >> 1;
+        if (!inside<KERN>(xr - __ldg(xs + k), h)) lo = k; else hi = k;
+    }
+    return lo;
+}
+
+// element q (0..63) of the warp's two-register segment (lane l holds l, 32 + l)
+__device__ __forceinline__ double seg_at(double c0, double c1, int q)
+{
+    const double v0 = __shfl_sync(0xffffffffu, c0, q & 31);
+    const double v1 = __shfl_sync(0xffffffffu, c1, q & 31);
+    return q < 32 ? v0 : v1;
+}
+
+template <int KERN, int KB>
+__global__ void __launch_bounds__(kWinThreads)
+window_kernel_blk(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
+                  int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
+                  int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
+                  uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
+{
+    const int lane = threadIdx.x & 31;
+    const double o = pfx_origin(xy, n);
+    const double ymax = __longlong_as_double((long long)*ymax_bits);
+    const int bper = (m + nbc - 1) / nbc;
+    const int ps = pstride;
+    for (;;) {
+        int task = 0;
+        if (lane == 0) task = atomicAdd(tile_counter, 1);
+        task = __shfl_sync(0xffffffffu, task, 0);
+        if (task >= ntiles * nbc) return;  // warp-uniform
+        const int chunk = task / ntiles;  // chunk-major (see window_kernel)
+        const int tile = task - chunk * ntiles;
+        const int b0 = chunk * bper, b1 = min(m, b0 + bper);
+        const int base = row_lo + tile * 32 * KB;  // < row_hi
+        const double xb = xy[base].x;
+        // the first row's boundaries (offsets from base) and growth at the previous bandwidth
+        int kR = 1, kL = 1, gR = cold_step(xs, n, __ldg(hg + b0)), gL = gR;
+        for (int b = b0; b < b1; b++) {
+            const double h = __ldg(hg + b);
+            // block 0's lower bounds: the first row's own boundaries (warp-cooperative)
+            {
+                const int nR = warp_boundary<KERN, true>(xs, n, base, xb, h, kR - 1, gR, lane);
+                const int nL = warp_boundary<KERN, false>(xs, n, base, xb, h, kL - 1, gL, lane);
+                gR = max(1, nR - kR);
+                gL = max(1, nL - kL);
+                kR = nR;
+                kL = nL;
+            }
+            int SR = base + kR, SL = base - kL;  // R of the row before the block (or the first row), L likewise
+            double e2 = 0.0;
+            int cntM = 0;
+#pragma unroll
+            for (int k = 0; k < KB; k++) {
+                const int i = base + 32 * k + lane;
+                const bool valid = i < row_hi;
+                WinRow w;
+                w.r = valid ? i : row_hi - 1;  // clamped rows do identical work, discarded
+                const double2 v = xy[w.r];
+                w.xr = v.x;
+                w.yr = v.y;
+                w.del = two_sum(v.x, -o);
+                // right: xs[SR - 1] is inside for every row of the block (or a row
+                // at or before it); the first outside lies at SR or beyond
+                const double r0 = __ldg(xs + min(SR + lane, n)), r1 = __ldg(xs + min(SR + 32 + lane, n));
+                // (indices >= the row are never compared; clamped to stay inside xs)
+                const double l0 = __ldg(xs + min(SL + lane, n)), l1 = __ldg(xs + min(SL + 32 + lane, n));
+                // (the shuffles run in every lane; lanes whose boundary lies past
+                // the segment then take their own gallop)
+                int R, L;
+                {
+                    // inside count of xs[SR .. SR + 63] (a prefix: the predicate is monotone)
+                    const double last = __shfl_sync(0xffffffffu, r1, 31);
+                    const bool beyond = SR + 63 < n && inside<KERN>(last - w.xr, h);
+                    int idx = 0;
+#pragma unroll
+                    for (int st = 32; st > 0; st >>= 1)
+                        idx += inside<KERN>(seg_at(r0, r1, idx + st - 1) - w.xr, h) ? st : 0;
+                    R = beyond ? right_from<KERN>(xs, n, w.xr, h, SR + 63) : min(SR + idx, n);
+                }
+                {
+                    // xs[SL] is outside for every row of the block; outside count of
+                    // xs[SL .. SL + 63] (indices >= the row are inside: d <= 0)
+                    const double last = __shfl_sync(0xffffffffu, l1, 31);
+                    const bool beyond = SL + 63 < w.r && !inside<KERN>(w.xr - last, h);
+                    int idx = 0;
+#pragma unroll
+                    for (int st = 32; st > 0; st >>= 1) {
+                        const int q = idx + st - 1;
+                        const double v = seg_at(l0, l1, q);
+                        idx += (SL + q < w.r && !inside<KERN>(w.xr - v, h)) ? st : 0;
+                    }
+                    L = beyond ? left_from<KERN>(xs, w.r, w.xr, h, SL + 63) : SL + idx - 1;
+                }
+                SR = __shfl_sync(0xffffffffu, R, 31);
+                SL = __shfl_sync(0xffffffffu, L, 31);
+                const int c = R - L - 2;
+                if (valid && c > 0) {  // reading Q6
+                    e2 += window_e2<KERN>(w, L + 1, R, c, h, xy, P, ps, ymax);
+                    cntM += 1;
+                }
+            }
+            e2 = warp_sum(e2);
+            const int cnt = __reduce_add_sync(0xffffffffu, cntM);  // <= 32 KB <= 128: fits the u8 slot
+            if (lane == 0) {
+                tileS[(size_t)b * ntiles + tile] = e2;
+                tileN[(size_t)b * ntiles + tile] = (uint8_t)cnt;
+            }
+        }
+    }
+}
+
 }  // namespace krcv

@@ -1,5 +1,9 @@
 """GPU: the window-kernel variants find the same boundaries.
 
+`window_kernel_blk` (KRCV_WIN_K = 9 / 10: 2 / 4 blocks of 32 consecutive rows)
+sums a tile's rows in another order than window_kernel<K, 2 / 4>: n_eff and
+best must be identical, CV equal to rounding.
+
 `window_kernel_seg` (KRCV_WIN_K = 6 / 7 / 8: 2 / 4 / 1 rows per lane) searches
 in a shared-memory segment with an exact check of its prediction and falls
 back to `window_kernel`'s global searches; with the same rows per lane
@@ -88,4 +92,22 @@ def test_seg_kernel_bit_identical(tmp_path, base, seg):
     for c in cases:
         assert a[c]["cv"] == b[c]["cv"], c
         assert a[c]["neff"] == b[c]["neff"], c
+        assert a[c]["best"] == b[c]["best"], c
+
+
+@pytest.mark.parametrize("base,blk", [(2, 9), (4, 10)])
+def test_blk_kernel_same_windows(tmp_path, base, blk):
+    cases = _cases()
+    path = str(tmp_path / "cases.npz")
+    arrs = {}
+    for c, (x, y, h, k) in cases.items():
+        arrs[c + "_x"], arrs[c + "_y"], arrs[c + "_h"], arrs[c + "_k"] = x, y, h, np.array(k)
+    np.savez(path, **arrs)
+    a, b = _run(base, path), _run(blk, path)
+    for c in cases:
+        ca = np.array(a[c]["cv"], np.uint64).view(np.float64)
+        cb = np.array(b[c]["cv"], np.uint64).view(np.float64)
+        assert a[c]["neff"] == b[c]["neff"], c
+        scale = max(float(np.max(np.abs(ca))), 1e-300)
+        assert float(np.max(np.abs(ca - cb))) <= 1e-13 * scale, c
         assert a[c]["best"] == b[c]["best"], c
