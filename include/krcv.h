@@ -326,6 +326,17 @@ int32_t kr_last_algo(void);
 /* Library version, e.g. "krcv 0.1.0 sm_100a". */
 const char *kr_version(void);
 
+/*
+ * kr_release -- frees the state the synchronous host-pointer entry points
+ * (kr_cv_grid*, kr_ll_cv_grid, kr_kde_lscv, kr_cv_refine) keep between calls
+ * on every device: device buffers, pinned staging, the captured CUDA graph
+ * and the library's stream.  The next call re-creates them.  Must not run
+ * concurrently with a host call.  Device-pointer (async) calls own no library
+ * state and are unaffected.  Returns KR_OK, or KR_ECUDA if a device could
+ * not be selected (the others are still released).
+ */
+int kr_release(void);
+
 #ifdef __cplusplus
 }
 #endif

@@ -468,3 +468,45 @@ extern "C" const char *kr_strerror(int status)
 extern "C" const char *kr_last_cuda_error(void) { return g_last_cuda_error.c_str(); }
 
 extern "C" const char *kr_version(void) { return "krcv 0.1.0 sm_100a"; }
+
+// Frees what the synchronous host entry points keep between calls on every
+// device (buffers, pinned staging, the captured graph, the stream); the next
+// call re-creates them.  The caller must not have a host call in flight.
+extern "C" int kr_release(void)
+{
+    std::lock_guard<std::mutex> g(g_ctx_mu);
+    int prev = 0;
+    cudaGetDevice(&prev);
+    int st = KR_OK;
+    for (size_t d = 0; d < g_ctx.size(); d++) {
+        DevCtx *c = g_ctx[d];
+        if (!c) continue;
+        std::lock_guard<std::mutex> lk(c->mu);
+        if (cudaSetDevice((int)d) != cudaSuccess) { st = KR_ECUDA; continue; }
+        if (c->stream) cudaStreamSynchronize(c->stream);
+        if (c->gexec) cudaGraphExecDestroy(c->gexec);
+        cudaFree(c->ws);
+        cudaFree(c->dx);
+        cudaFree(c->dy);
+        cudaFree(c->dh);
+        cudaFree(c->dpartial);
+        cudaFree(c->dres);
+        cudaFreeHost(c->pres);
+        if (c->stream) cudaStreamDestroy(c->stream);
+        c->gexec = nullptr;
+        c->gx = c->gy = c->gh = nullptr;
+        c->ws = nullptr;
+        c->ws_bytes = 0;
+        c->dx = c->dy = c->dh = c->dpartial = c->dcv = nullptr;
+        c->dres = nullptr;
+        c->dneff = nullptr;
+        c->dbest = nullptr;
+        c->pres = nullptr;
+        c->pcap_m = 0;
+        c->cap_n = 0;
+        c->cap_m = 0;
+        c->stream = nullptr;
+    }
+    cudaSetDevice(prev);
+    return st;
+}

@@ -37,7 +37,7 @@ KR_MAX_M = 65536
 EXPORTS = (
     "kr_cv_grid", "kr_cv_grid_ex", "kr_cv_grid_algo", "kr_cv_refine", "kr_validate_grid", "kr_workspace_bytes",
     "kr_cv_shard_async", "kr_cv_shard_algo_async", "kr_cv_grid_async", "kr_finalize", "kr_finalize_async", "kr_default_grid",
-    "kr_strerror", "kr_last_cuda_error", "kr_version",
+    "kr_strerror", "kr_last_cuda_error", "kr_version", "kr_release",
     "kr_profile_enable", "kr_profile_read", "kr_launch_count", "kr_last_algo",
     "kr_kde_lscv", "kr_kde_lscv_async", "kr_kde_shard_async", "kr_kde_finalize",
     "kr_ll_cv_grid", "kr_ll_cv_grid_async", "kr_ll_shard_async",
@@ -213,6 +213,11 @@ def kr_strerror(status: int) -> str:
 
 def kr_version() -> str:
     return _lib().kr_version().decode()
+
+
+def kr_release() -> None:
+    """Free the state the synchronous host entry points keep between calls."""
+    _check(_lib().kr_release(), "kr_release")
 
 
 def kr_workspace_bytes(n: int, m: int) -> int:
