@@ -22,6 +22,10 @@
 #include <cstdlib>
 
 #include "krcv.h"
+#include <nvtx3/nvToolsExt.h>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
 #include "krcv_internal.h"
 #include "krcv_sweep.cuh"
 #include "krcv_sweep_gxg.cuh"
@@ -220,6 +224,22 @@ reduce_kernel(const double *__restrict__ tileS, const uint8_t *__restrict__ tile
     __threadfence();
     finalize_body<kReduceThreads>(partial, fin.n, m, fin.cv, fin.neff, fin.best, fin.status, sS, sI);
     if (threadIdx.x == 0) *fin.done = 0u;
+}
+
+// ---------------------------------------------------------------------------
+// tracing and fault injection (krcv_internal.h)
+// ---------------------------------------------------------------------------
+NvtxScope::NvtxScope(const char *name) { nvtxRangePushA(name); }
+NvtxScope::~NvtxScope() { nvtxRangePop(); }
+
+bool injected_failure(const char *stage)
+{
+    const char *e = getenv("KRCV_FAIL_AT");
+    if (!e || strcmp(e, stage) != 0) return false;
+    char buf[96];
+    snprintf(buf, sizeof buf, "injected failure at %s (KRCV_FAIL_AT)", stage);
+    set_error_text(buf);
+    return true;
 }
 
 // ---------------------------------------------------------------------------
@@ -811,6 +831,7 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
                                       : (variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G));
 
     int64_t launches = 0;
+    NvtxScope nv_all("krcv: grid-search shard (a1-a5)");
     prof_mark(0, st);
     // reuse keeps max|y| (words 4-5); the host validated x, y and the grid
     cudaError_t e = cudaMemsetAsync(status, 0, (reuse_sorted ? 3 : 8) * sizeof(unsigned), st);
@@ -819,10 +840,13 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         e = cudaMemsetAsync(counter, 0, sizeof(int), st);
         if (e != cudaSuccess) { set_cuda_error("cudaMemsetAsync(counter)", (int)e); return KR_ECUDA; }
     } else {
+        if (injected_failure("sort")) return KR_ECUDA;
+        NvtxScope nv("krcv: a1+a2 pack, validate, sort");
         const int st2 = enqueue_sort(d_x, d_y, n, d_h, m, L, ws, st, &launches);
         if (st2) return st2;
     }
     prof_mark(1, st);
+    if (prefix && !reuse_sorted && injected_failure("prefix")) return KR_ECUDA;
     if (prefix && !reuse_sorted && ll) {
         launch_prefix_build<kLLMoments>(xy, nn, L, ws, st);
         launches += 2;
@@ -835,7 +859,9 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         launches += 2;
     }
     prof_mark(2, st);
+    if (injected_failure("sweep")) return KR_ECUDA;
     if (ntiles > 0) {
+        NvtxScope nv("krcv: a3+a4 windows, LOO estimates, squared errors");
         launches += 1;
         if (hist) {
             const uint32_t *perm = reinterpret_cast<const uint32_t *>(ws + L.perm);
@@ -896,6 +922,8 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         }
     }
     prof_mark(3, st);
+    if (injected_failure("reduce")) return KR_ECUDA;
+    NvtxScope nv_red("krcv: a5 reduction (+ finalize)");
     reduce_kernel<<<m < 148 * 8 ? m : 148 * 8, kReduceThreads, 0, st>>>(tileS, tileN, ntiles, m, status,
                                                                         d_partial, fin);
     launches += 1;

@@ -26,6 +26,8 @@ void set_cuda_error(const char *what, int code)
     g_last_cuda_error = buf;
 }
 
+void set_error_text(const char *text) { g_last_cuda_error = text; }
+
 static bool kernel_ok(int32_t k)
 {
     return k == KR_UNIFORM || k == KR_EPANECHNIKOV || k == KR_TRIANGULAR || k == KR_GAUSSIAN;

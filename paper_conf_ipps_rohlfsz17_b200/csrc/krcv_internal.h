@@ -56,5 +56,22 @@ bool prof_enabled();
 
 // Records a CUDA error string for kr_last_cuda_error (thread-local).
 void set_cuda_error(const char *what, int code);
+void set_error_text(const char *text);
+
+// Fault injection: with KRCV_FAIL_AT=<stage> in the
+// environment (stage: sort, prefix, sweep, reduce) the enqueue stops before
+// that stage and returns KR_ECUDA, kr_last_cuda_error naming the stage --
+// tests/test_gpu_faults.py checks the error unwinding (nothing written, the
+// next call clean).  Read per call; unset costs one getenv.
+bool injected_failure(const char *stage);
+
+// NVTX range for the host-side enqueue of a stage (nsys / ncu --nvtx);
+// header-only NVTX v3, a no-op without an attached tool.
+struct NvtxScope {
+    explicit NvtxScope(const char *name);
+    ~NvtxScope();
+    NvtxScope(const NvtxScope &) = delete;
+    NvtxScope &operator=(const NvtxScope &) = delete;
+};
 
 }  // namespace krcv
