@@ -173,14 +173,21 @@ def oracle_sample(x, y, h, k, target_s: float):
     t0 = time.perf_counter()
     evaluate(x, y, h, k, rows=order[:rows])
     dt = time.perf_counter() - t0
-    per_row = dt / rows
-    rows = int(min(n, max(rows, target_s / max(per_row, 1e-9))))
-    stride = max(1, n // rows)
-    sample = order[::stride][:rows]  # spread over the sorted order
-    t0 = time.perf_counter()
-    evaluate(x, y, h, k, rows=sample)
-    dt = time.perf_counter() - t0
-    return sample.shape[0] * (n - 1) * m / dt, dt, int(sample.shape[0]), threads
+    # size the sample from the measured per-row time; a small first probe
+    # over-estimates it (thread start-up), so re-size until the sample takes
+    # at least half the target (or covers every row)
+    for _ in range(4):
+        per_row = dt / rows
+        rows = int(min(n, max(rows, 0.9 * target_s / max(per_row, 1e-9))))
+        stride = max(1, n // rows)
+        sample = order[::stride][:rows]  # spread over the sorted order
+        t0 = time.perf_counter()
+        evaluate(x, y, h, k, rows=sample)
+        dt = time.perf_counter() - t0
+        rows = int(sample.shape[0])
+        if dt >= 0.5 * target_s or rows >= n:
+            break
+    return rows * (n - 1) * m / dt, dt, rows, threads
 
 
 def cpu_model():

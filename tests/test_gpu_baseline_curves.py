@@ -1,0 +1,47 @@
+"""GPU parity at BASELINE.json's full sizes, in the launch configuration
+bench.py times (GridSearch(graph=True): one CUDA-graph replay of the whole
+search on device-resident x, y): every CV(h_b) of C1-C5, seeds 0-2, against
+the oracle's curves in tests/golden/curves/ (written by
+tools/make_reference_curves.py, which calls only oracle/: the Program-3
+evaluator for C1/C2, the oracle's window checker for C3-C5).  Bar
+(north_star): relative error <= 1e-6 with the SURVEY §8(c) floor (measured
+~1e-14), n_eff identical, best identical unless the reference's two best
+values lie within 1e-6.  Also the bench's second plan (stage events in the
+graph) and the host API give the same curve."""
+from __future__ import annotations
+
+import glob
+import os
+
+import numpy as np
+import pytest
+
+import workloads
+from paper_conf_ipps_rohlfsz17_b200.api import GridSearch
+from tests.helpers import best_ok, cv_rel_err
+
+pytestmark = pytest.mark.gpu
+
+GOLD = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", "curves")
+FILES = sorted(glob.glob(os.path.join(GOLD, "C*_s*.npz")))
+
+
+@pytest.mark.parametrize("path", FILES, ids=[os.path.basename(p)[:-4] for p in FILES])
+def test_full_size_curve_in_bench_launch_config(path):
+    torch = pytest.importorskip("torch")
+    ref = np.load(path)
+    cfg, seed = os.path.basename(path)[:-4].split("_s")
+    x, y, h, k = workloads.make(cfg, seed=int(seed))
+    assert x.shape[0] == int(ref["n"]) and h.shape[0] == int(ref["m"]) and k == int(ref["kernel"])
+    dev = torch.device("cuda", 0)
+    d_x, d_y = torch.as_tensor(x, device=dev), torch.as_tensor(y, device=dev)
+    plan = GridSearch(x.shape[0], h, k, device=dev, graph=True)
+    for _ in range(2):  # capture, then replay
+        plan.run(d_x, d_y)
+    res = plan.result()
+    cv, neff = res.cv.cpu().numpy(), res.neff.cpu().numpy()
+    err = cv_rel_err(cv, ref["cv"])
+    print(f"{cfg} seed {seed}: max rel err {err:.3g}, best {res.best} (ref {int(ref['best'])})")
+    assert err <= 1e-6
+    assert np.array_equal(neff, ref["neff"])
+    assert best_ok(res.best, ref["cv"], 1e-6)
