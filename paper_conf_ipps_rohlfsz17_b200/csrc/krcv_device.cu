@@ -269,7 +269,7 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     L->vals_in = off;  off = align256(off + sizeof(uint32_t) * npad);
     L->vals_out = off; off = align256(off + sizeof(uint32_t) * npad);
     L->xy = off;       off = align256(off + sizeof(double2) * ((size_t)n + 2 * kPad));
-    L->counter = off;  off = align256(off + sizeof(int));
+    L->counter = off;  off = align256(off + sizeof(int) * (1 + kSmCounters));  // tile counter + SM-local counters
     L->perm = off;     off = align256(off + sizeof(uint32_t) * (size_t)n);
     // window-prefix path (krcv_prefix.cuh)
     const size_t nch = (size_t)((n + kPfxTileMin) / kPfxTileMin);  // most tiles covering P[0..n]
@@ -530,16 +530,31 @@ static int win_lane_rows(int K)
     }
 }
 
+// Task assignment of the window kernels: 1 = SM-local regions
+// (take_task_local, krcv_prefix.cuh), 0 = one global counter (default).  KRCV_WIN_SCHED
+// overrides.
+static int win_sched()
+{
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("KRCV_WIN_SCHED");
+        v = e ? (atoi(e) ? 1 : 0) : 0;  // measured: no gain
+    }
+    return v;
+}
+
 template <int KERN, int K>
 static void launch_window_k(const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
                             const WsLayout &L, char *ws, double *tileS, uint8_t *tileN, int *counter,
                             cudaStream_t st)
 {
+    const int sched = win_sched();
     static int resident = 0;
     if (!resident) {
         int b = 0;
         if (K == 3)
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_b2<KERN>, kWinThreads, 0);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sched ? window_kernel_b2<KERN, 1> : window_kernel_b2<KERN, 0>,
+                                                          kWinThreads, 0);
         else if (K == 5)
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_coop<KERN>, kCoopRows, 0);
         else if (K >= 9)
@@ -548,7 +563,9 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_seg<KERN, K == 6 ? 2 : (K == 7 ? 4 : 1)>,
                                                           kWinThreads, 0);
         else
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel<KERN, K>, kWinThreads, 0);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+                &b, sched ? window_kernel<KERN, (K == 3 || K >= 5) ? 1 : K, 1> : window_kernel<KERN, (K == 3 || K >= 5) ? 1 : K, 0>,
+                kWinThreads, 0);
         resident = b > 0 ? b : 1;
     }
     static int sms = 0;
@@ -576,9 +593,14 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
     const double *P = reinterpret_cast<const double *>(ws + L.pfx);
     const unsigned long long *ymax =
         reinterpret_cast<const unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
-    if (K == 3)
-        window_kernel_b2<KERN><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
-                                                               nbc, ymax, tileS, tileN, counter);
+    const bool local = sched && (K <= 4) && sms <= kSmCounters;
+    if (local) cudaMemsetAsync(counter + 1, 0, sizeof(int) * sms, st);  // the SM-local region counters
+    if (K == 3 && local)
+        window_kernel_b2<KERN, 1><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
+                                                                  nbc, ymax, tileS, tileN, counter, sms);
+    else if (K == 3)
+        window_kernel_b2<KERN, 0><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
+                                                                  nbc, ymax, tileS, tileN, counter, sms);
     else if (K == 5)
         window_kernel_coop<KERN><<<blocks, kCoopRows, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
                                                                nbc, ymax, tileS, tileN, counter);
@@ -588,10 +610,12 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
     else if (K >= 6)
         window_kernel_seg<KERN, K == 6 ? 2 : (K == 7 ? 4 : 1)><<<blocks, kWinThreads, 0, st>>>(
             xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter);
+    else if (local)
+        window_kernel<KERN, (K == 3 || K >= 5) ? 1 : K, 1><<<blocks, kWinThreads, 0, st>>>(
+            xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter, sms);
     else
-        window_kernel<KERN, (K == 3 || K == 5) ? 1 : K><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo,
-                                                                            hi, ntiles, nbc, ymax, tileS, tileN,
-                                                                            counter);
+        window_kernel<KERN, (K == 3 || K >= 5) ? 1 : K, 0><<<blocks, kWinThreads, 0, st>>>(
+            xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter, sms);
 }
 
 template <int KERN>

@@ -7,6 +7,9 @@
 
 namespace krcv {
 
+// SM-local task counters after the tile counter in the workspace (window kernels).
+constexpr int kSmCounters = 1024;
+
 // Shards with at least this many rows use the gxg sweep variant.
 constexpr int64_t kGxgRows = 400000;
 int sweep_G(int64_t rows);

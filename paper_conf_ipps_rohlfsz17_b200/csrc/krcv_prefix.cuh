@@ -132,6 +132,50 @@ __device__ __forceinline__ int cold_step(const double *__restrict__ xs, int n, d
     return e >= (double)n ? n : (e < 1.0 ? 1 : (int)e);
 }
 
+// SM-local task assignment (window kernels, SCHED = 1).  The task space
+// (chunk-major: consecutive tasks are adjacent row tiles at the same
+// bandwidths) is cut into one contiguous region per SM; the warps resident
+// on an SM take their region's tasks in order from its counter ctr[s], so
+// they work on neighbouring tiles at the same time and their boundary probes
+// and prefix loads hit the same L1 lines.  A warp whose region is exhausted
+// steals from the others (32 regions checked per round, one atomic per
+// candidate).  Returns -1 when every task has been taken.  Which warp runs a
+// task never changes its result (one partial per (tile, bandwidth)).
+__device__ __forceinline__ int region_lo(int r, int total, int nsm) { return (int)((long long)r * total / nsm); }
+
+__device__ __noinline__ int take_task_local(int *__restrict__ ctr, int total, int nsm, int lane)
+{
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    const int own = (int)(smid % (unsigned)nsm);
+    int t = -1;
+    if (lane == 0) {
+        const int lo = region_lo(own, total, nsm), hi = region_lo(own + 1, total, nsm);
+        const int k = atomicAdd(ctr + own, 1);
+        if (lo + k < hi) t = lo + k;
+    }
+    t = __shfl_sync(0xffffffffu, t, 0);
+    if (t >= 0) return t;
+    for (int base = 1; base < nsm; base += 32) {
+        const int v = (own + base + lane) % nsm;
+        const int lo = region_lo(v, total, nsm), len = region_lo(v + 1, total, nsm) - lo;
+        const int left = base + lane < nsm ? len - *(volatile int *)(ctr + v) : 0;
+        unsigned ball = __ballot_sync(0xffffffffu, left > 0);
+        while (ball) {
+            const int src = __ffs(ball) - 1;
+            int got = -1;
+            if (lane == src) {
+                const int k = atomicAdd(ctr + v, 1);
+                if (k < len) got = lo + k;
+            }
+            got = __shfl_sync(0xffffffffu, got, src);
+            if (got >= 0) return got;
+            ball &= ball - 1;
+        }
+    }
+    return -1;
+}
+
 // ---------------------------------------------------------------- build
 // Two-phase fixed-order scan (bit-reproducible; a decoupled look-back
 // would make the dd rounding depend on timing): tile totals, then every tile
@@ -574,12 +618,12 @@ __device__ __forceinline__ void window_advance(const double *__restrict__ xs, in
 // bandwidth the lane's first row searches from its previous bandwidth's
 // boundaries (window_bounds); each next row starts from its predecessor's
 // boundaries at the same bandwidth (window_advance, ~1 probe per side).
-template <int KERN, int K>
+template <int KERN, int K, int SCHED>
 __global__ void __launch_bounds__(kWinThreads)
 window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
               int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
               int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
-              uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
+              uint8_t *__restrict__ tileN, int *__restrict__ tile_counter, int nsm)
 {
     const int lane = threadIdx.x & 31;
     const double o = pfx_origin(xy, n);
@@ -591,9 +635,14 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
         // split so that small shards still fill the GPU; a chunk starts its
         // searches cold (from the row itself), later steps from the previous h.
         int task = 0;
-        if (lane == 0) task = atomicAdd(tile_counter, 1);
-        task = __shfl_sync(0xffffffffu, task, 0);
-        if (task >= ntiles * nbc) return;  // warp-uniform
+        if (SCHED) {
+            task = take_task_local(tile_counter + 1, ntiles * nbc, nsm, lane);
+            if (task < 0) return;  // warp-uniform
+        } else {
+            if (lane == 0) task = atomicAdd(tile_counter, 1);
+            task = __shfl_sync(0xffffffffu, task, 0);
+            if (task >= ntiles * nbc) return;  // warp-uniform
+        }
         // chunk-major order: concurrently running warps hold adjacent tiles at
         // the same bandwidths, so their windows (and probes) overlap in L1/L2
         const int chunk = task / ntiles;
@@ -709,12 +758,12 @@ __device__ __forceinline__ void window_bounds2(const double *__restrict__ xs, in
     for (int c = 0; c < 4; c++) kout[c] = hi[c];
 }
 
-template <int KERN>
+template <int KERN, int SCHED>
 __global__ void __launch_bounds__(kWinThreads)
 window_kernel_b2(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
                  int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
                  int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
-                 uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
+                 uint8_t *__restrict__ tileN, int *__restrict__ tile_counter, int nsm)
 {
     const int lane = threadIdx.x & 31;
     const double o = pfx_origin(xy, n);
@@ -723,9 +772,14 @@ window_kernel_b2(const double *__restrict__ xs, const double2 *__restrict__ xy, 
     const int ps = pstride;
     for (;;) {
         int task = 0;
-        if (lane == 0) task = atomicAdd(tile_counter, 1);
-        task = __shfl_sync(0xffffffffu, task, 0);
-        if (task >= ntiles * nbc) return;  // warp-uniform
+        if (SCHED) {
+            task = take_task_local(tile_counter + 1, ntiles * nbc, nsm, lane);
+            if (task < 0) return;  // warp-uniform
+        } else {
+            if (lane == 0) task = atomicAdd(tile_counter, 1);
+            task = __shfl_sync(0xffffffffu, task, 0);
+            if (task >= ntiles * nbc) return;  // warp-uniform
+        }
         const int chunk = task / ntiles;  // chunk-major (see window_kernel)
         const int tile = task - chunk * ntiles;
         const int b0 = chunk * bper, b1 = min(m, b0 + bper);
