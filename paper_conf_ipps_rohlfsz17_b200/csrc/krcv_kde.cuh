@@ -71,6 +71,63 @@ __device__ __forceinline__ void kde_power_sums(const double *__restrict__ P, int
     }
 }
 
+// Plain-double fast path of kde_power_sums (hi words of P only, Horner in
+// double) with a rigorous bound of its error.  Each raw moment difference
+// M_i = P_hi[b] - P_hi[a] is off by at most 2^-52 (|P_hi[b]| + |P_hi[a]|)
+// (hi word rounding of the dd prefix + the subtraction); Horner's 2k roundings
+// and the rounding of delta (k 2^-53 relative, first order) are bounded by
+// the same binomial sum of magnitudes E_k = sum_i C(k,i) Mb_i |delta|^(k-i),
+// so |S_k - S_k(fast)| <= (3k + 4) 2^-52 (E_k right + E_k left) (twice the
+// first-order estimate: the magnitudes are themselves rounded).  Empty sides
+// contribute exactly 0 (P_hi[b] == P_hi[a]) and no error.
+template <int DEG>
+__device__ __forceinline__ void kde_power_sums_fast(const double *__restrict__ P, int ps, int r, int A, int R,
+                                                    double dl, double (&S)[6], double (&err)[6])
+{
+    const double e = -dl, ae = fabs(dl);
+    double TR[6], TL[6], ER[6], EL[6];
+#pragma unroll
+    for (int side = 0; side < 2; side++) {
+        const int a = side == 0 ? r + 1 : A, b = side == 0 ? R : r;
+        const bool empty = b <= a;
+        double M[6], Mb[6];
+        M[0] = empty ? 0.0 : (double)(b - a);
+        Mb[0] = M[0];
+#pragma unroll
+        for (int k = 1; k <= DEG; k++) {
+            const double pb = ld_hi(P, ps, k - 1, b), pa = ld_hi(P, ps, k - 1, a);
+            M[k] = empty ? 0.0 : pb - pa;
+            Mb[k] = empty ? 0.0 : fabs(pb) + fabs(pa);
+        }
+        double *T = side == 0 ? TR : TL;
+        double *E = side == 0 ? ER : EL;
+#pragma unroll
+        for (int k = 1; k <= DEG; k++) {
+            if (DEG == 5 && k == 4) continue;  // S4 is never needed
+            double acc = M[0], mag = Mb[0], cbin = 1.0;
+#pragma unroll
+            for (int i = 1; i <= k; i++) {
+                cbin = cbin * (double)(k - i + 1) / (double)i;  // exact small integers
+                acc = fma(e, acc, cbin * M[i]);
+                mag = fma(ae, mag, cbin * Mb[i]);
+            }
+            T[k] = acc;
+            E[k] = mag;
+        }
+    }
+#pragma unroll
+    for (int k = 1; k <= DEG; k++) {
+        if (DEG == 5 && k == 4) continue;
+        S[k] = (k & 1) ? TR[k] - TL[k] : TR[k] + TL[k];
+        err[k] = (3.0 * k + 4.0) * 0x1p-52 * (ER[k] + EL[k]);
+    }
+}
+
+// Fast results are kept when the bound on the error of A_i (B_i) is below
+// kKdeFastTol times the largest value A_i (B_i) can take, c Kbar(0) (c K(0)):
+// per row an absolute error <= 2^-44 of its possible contribution.
+constexpr double kKdeFastTol = 0x1p-44;
+
 template <int KERN>
 __global__ void __launch_bounds__(kWinThreads)
 kde_window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
@@ -114,22 +171,39 @@ kde_window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy,
             const double c1 = (double)(R1 - A1 - 1), c2 = (double)(R2 - A2 - 1);
             const double ih = 1.0 / h, ih2 = ih * ih, ih3 = ih2 * ih;
             double Ai, Bi;
-            if (KERN == KR_UNIFORM) {
+            if (KERN == KR_UNIFORM) {  // one power sum: dd directly (the fast path measured slower here)
                 double S[6];
                 kde_power_sums<1>(P, ps, r, A2, R2, del, S);
                 Bi = 0.5 * c1;
                 Ai = 0.25 * fma(-S[1], ih, 2.0 * c2);
             } else if (KERN == KR_EPANECHNIKOV) {
-                double S1[6], S2[6];
-                kde_power_sums<2>(P, ps, r, A1, R1, del, S1);
-                kde_power_sums<5>(P, ps, r, A2, R2, del, S2);
-                Bi = 0.75 * fma(-S1[2], ih2, c1);
+                double S1[6], S2[6], e1[6], e2[6];
                 const double ih5 = ih3 * ih2;
+                kde_power_sums_fast<2>(P, ps, r, A1, R1, del.hi, S1, e1);
+                kde_power_sums_fast<5>(P, ps, r, A2, R2, del.hi, S2, e2);
+                const double errB = 0.75 * e1[2] * ih2;
+                const double errA = (3.0 / 160.0) * (40.0 * e2[2] * ih2 + 20.0 * e2[3] * ih3 + e2[5] * ih5 +
+                                                     8.0 * 0x1p-53 * (32.0 * c2 + 40.0 * fabs(S2[2]) * ih2 +
+                                                                      20.0 * fabs(S2[3]) * ih3 + fabs(S2[5]) * ih5));
+                if (!(errB <= kKdeFastTol * 0.75 * c1)) kde_power_sums<2>(P, ps, r, A1, R1, del, S1);
+                if (!(errA <= kKdeFastTol * 0.6 * c2)) kde_power_sums<5>(P, ps, r, A2, R2, del, S2);
+                Bi = 0.75 * fma(-S1[2], ih2, c1);
                 Ai = (3.0 / 160.0) * (32.0 * c2 - 40.0 * S2[2] * ih2 + 20.0 * S2[3] * ih3 - S2[5] * ih5);
             } else {
-                double S1[6], S2[6];
-                kde_power_sums<3>(P, ps, r, A1, R1, del, S1);
-                kde_power_sums<3>(P, ps, r, A2, R2, del, S2);
+                double S1[6], S2[6], e1[6], e2[6];
+                kde_power_sums_fast<3>(P, ps, r, A1, R1, del.hi, S1, e1);
+                kde_power_sums_fast<3>(P, ps, r, A2, R2, del.hi, S2, e2);
+                const double errB = e1[1] * ih;
+                const double errA = e1[2] * ih2 + 0.5 * e1[3] * ih3 +
+                                    (12.0 * (e2[1] + e1[1]) * ih + 6.0 * (e2[2] + e1[2]) * ih2 +
+                                     (e2[3] + e1[3]) * ih3) / 6.0 +
+                                    8.0 * 0x1p-53 * (c1 + c2 + (fabs(S2[1]) + fabs(S1[1])) * 2.0 * ih +
+                                                     (fabs(S2[2]) + fabs(S1[2])) * ih2 +
+                                                     (fabs(S2[3]) + fabs(S1[3])) * ih3);
+                if (!(errB <= kKdeFastTol * c1 && errA <= kKdeFastTol * (2.0 / 3.0) * c2)) {
+                    kde_power_sums<3>(P, ps, r, A1, R1, del, S1);
+                    kde_power_sums<3>(P, ps, r, A2, R2, del, S2);
+                }
                 Bi = fma(-S1[1], ih, c1);
                 const double inner = (2.0 / 3.0) * c1 - S1[2] * ih2 + 0.5 * S1[3] * ih3;
                 const double outer = (8.0 * (c2 - c1) - 12.0 * (S2[1] - S1[1]) * ih + 6.0 * (S2[2] - S1[2]) * ih2 -
