@@ -268,6 +268,21 @@ def test_grid_sizes(m):
     _check(x, y, h, E)
 
 
+@pytest.mark.parametrize("k", [U, E, T])
+def test_max_grid_size(k):
+    """The largest grid the ABI accepts (KR_MAX_M = 65,536 bandwidths): tile
+    partials, the reduction grid-stride loop and the fused finalize's arg-min
+    at their limit, with a log grid so that windows range from empty to all."""
+    x, y = workloads.draw_xy("lognormal", 300, 4)
+    r = float(x.max() - x.min())
+    h = np.geomspace(1e-6 * r, 2.0 * r, krcv.KR_MAX_M)
+    cv, neff, best = _gpu(x, y, h, k)
+    ref = oracle.cv_sorted(x, y, h, k)
+    assert np.array_equal(neff, ref.neff)
+    assert cv_rel_err(cv, ref.cv) <= TIGHT
+    assert best_ok(best, ref.cv)
+
+
 @pytest.mark.parametrize("cfg,n", [("C2", 20000), ("C5", 5000), ("C1", 1000), ("C2", 4097), ("C2", 131072)])
 def test_rank_sort_matches_cub_sort_bitwise(cfg, n, monkeypatch):
     """The two a2 implementations (chunked rank sort for n <= 131072, CUB
