@@ -468,16 +468,22 @@ int auto_algo(int64_t /*n*/, int64_t /*rows*/, int32_t /*m*/, int32_t /*kernel*/
 
 // Records per thread of the prefix build: 1 (256-record tiles, more CTAs)
 // up to 2^18 records, 4 above.  KRCV_PFX_ITEMS=1|4 overrides.
+// 0 = the one-CTA build (pfx_one_cta_kernel) for n <= kPfxOneCtaMax: its
+// per-thread sequential dd chains only pay off for a few records per thread
+// (profiles/experiments/r01be_*).
+// KRCV_PFX_ITEMS=0|1|4 overrides.
+constexpr int kPfxOneCtaMax = 1024;  // measured: C1 (n = 1,000) 10.2 -> 8.2 us, C2 (n = 20,000) 18 -> 187 us
+
 static int pfx_items(int n)
 {
     static int forced = -1;
     if (forced < 0) {
         const char *e = getenv("KRCV_PFX_ITEMS");
-        forced = e ? atoi(e) : 0;
-        if (forced != 1 && forced != 4) forced = 0;
+        forced = e ? atoi(e) : -2;
+        if (forced != 0 && forced != 1 && forced != 4) forced = -2;
     }
-    if (forced) return forced;
-    return n <= (1 << 18) ? 1 : kPfxItemsMax;
+    if (forced != -2) return forced;
+    return n <= kPfxOneCtaMax ? 0 : (n <= (1 << 18) ? 1 : kPfxItemsMax);
 }
 
 template <int KERN>
@@ -487,7 +493,10 @@ static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, cha
     double *P = reinterpret_cast<double *>(ws + L.pfx);
     double2 *tot = reinterpret_cast<double2 *>(ws + L.ptot);
     unsigned long long *ymax = reinterpret_cast<unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
-    if (pfx_items(n) == 1) {
+    const int items = pfx_items(n);
+    if (items == 0) {
+        pfx_one_cta_kernel<KERN><<<1, kPfx1Threads, 0, st>>>(xy, n, P, (int)L.pstride, xs, ymax);
+    } else if (items == 1) {
         const int ntiles = (n + kPfxThreads) / kPfxThreads;  // tiles covering P[0..n]
         pfx_tile_reduce_kernel<KERN, 1><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, ymax);
         pfx_tile_scan_kernel<KERN, 1><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, P, (int)L.pstride, xs);

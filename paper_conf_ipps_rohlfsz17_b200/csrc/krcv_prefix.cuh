@@ -329,6 +329,103 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
     }
 }
 
+// One-CTA build for small n (a single launch instead of two; the two-phase
+// build is latency-bound there).  Thread t owns the contiguous records
+// [t I, t I + I), I = ceil(n / kPfx1Threads): pass 1 sums its terms in order,
+// a fixed-order block scan (warp shuffles, then warp 0 over the warp totals)
+// gives each thread its exclusive offset, pass 2 recomputes the terms and
+// writes the running prefix P[k][j] (j = 0 .. n), xs and the sentinels.
+// Every sum is in a fixed order: bit-reproducible, like the two-phase build
+// (whose different order rounds differently in the last dd bits).
+constexpr int kPfx1Threads = 512;
+
+template <int KERN>
+__global__ void __launch_bounds__(kPfx1Threads)
+pfx_one_cta_kernel(const double2 *__restrict__ xy, int n, double *__restrict__ P, int pstride,
+                   double *__restrict__ xs, unsigned long long *__restrict__ ymax_bits)
+{
+    constexpr int K = NMom<KERN>::v;
+    constexpr int W = kPfx1Threads / 32;
+    __shared__ double2 wtot[K][W];
+    __shared__ double2 woff[K][W];
+    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+    const int I = (n + kPfx1Threads - 1) / kPfx1Threads;
+    const int j0 = min(n, t * I), j1 = min(n, j0 + I);
+    const double o = pfx_origin(xy, n);
+    if (t < kPad) {
+        xs[-1 - t] = -INFINITY;
+        xs[n + t] = INFINITY;
+    }
+    // pass 1: this thread's totals
+    dd acc[kPfxMoments];
+#pragma unroll
+    for (int k = 0; k < K; k++) acc[k] = dd{0.0, 0.0};
+    double ym = 0.0;
+    for (int j = j0; j < j1; j++) {
+        const double2 v = xy[j];
+        ym = fmax(ym, fabs(v.y));
+        dd tm[kPfxMoments];
+        moment_terms<KERN>(v.x, v.y, o, tm);
+#pragma unroll
+        for (int k = 0; k < K; k++) acc[k] = dd_add(acc[k], tm[k]);
+    }
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) ym = fmax(ym, __shfl_xor_sync(0xffffffffu, ym, d));
+    if (lane == 0 && ym > 0.0) atomicMax(ymax_bits, (unsigned long long)__double_as_longlong(ym));
+    // exclusive scan of the thread totals: within the warp, then over the warps
+    dd ex[kPfxMoments];
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        dd inc = acc[k];
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const dd u = shfl_up_dd(inc, d);
+            if (lane >= d) inc = dd_add(u, inc);
+        }
+        if (lane == 31) st_dd(&wtot[k][w], inc);
+        const dd u = shfl_up_dd(inc, 1);
+        ex[k] = lane == 0 ? dd{0.0, 0.0} : u;
+    }
+    __syncthreads();
+    if (w == 0) {
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            dd inc = lane < W ? ld_dd(&wtot[k][lane]) : dd{0.0, 0.0};
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const dd u = shfl_up_dd(inc, d);
+                if (lane >= d) inc = dd_add(u, inc);
+            }
+            const dd u = shfl_up_dd(inc, 1);
+            if (lane < W) st_dd(&woff[k][lane], lane == 0 ? dd{0.0, 0.0} : u);
+        }
+    }
+    __syncthreads();
+    // pass 2: running prefix over this thread's records
+    dd run[kPfxMoments];
+#pragma unroll
+    for (int k = 0; k < K; k++) run[k] = dd_add(ld_dd(&woff[k][w]), ex[k]);
+    for (int j = j0; j < j1; j++) {
+        const double2 v = xy[j];
+        xs[j] = v.x;
+        dd tm[kPfxMoments];
+        moment_terms<KERN>(v.x, v.y, o, tm);
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            P[(size_t)(2 * k) * pstride + j] = run[k].hi;
+            P[(size_t)(2 * k + 1) * pstride + j] = run[k].lo;
+            run[k] = dd_add(run[k], tm[k]);
+        }
+    }
+    if (j1 == n && j0 < n) {  // the thread holding the last record writes P[k][n]
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            P[(size_t)(2 * k) * pstride + n] = run[k].hi;
+            P[(size_t)(2 * k + 1) * pstride + n] = run[k].lo;
+        }
+    }
+}
+
 // ---------------------------------------------------------------- windows
 // New boundaries for bandwidth h from the previous ones, in offsets from the
 // row: the right side probes xs[r + k], the left side xs[r - k]; "inside" is
