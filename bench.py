@@ -323,10 +323,12 @@ def run_ours(args):
             return sum(starts[s].elapsed_time(ends[s]) for s in range(args.steps)), st, launches, clk
 
         krcv.kr_profile_enable(False)
-        plan = GridSearch(n, h, k, device=dev, rank=rank, world=world, algo=algo, graph=(world == 1))
+        plan = GridSearch(n, h, k, device=dev, rank=rank, world=world, algo=algo, graph=(world == 1),
+                          balance=(world > 1))
         total_ms, _, launches, clk = run_steps(plan, False)
         krcv.kr_profile_enable(True)
-        pplan = GridSearch(n, h, k, device=dev, rank=rank, world=world, algo=algo, graph=(world == 1))
+        pplan = GridSearch(n, h, k, device=dev, rank=rank, world=world, algo=algo, graph=(world == 1),
+                          balance=(world > 1))
         prof_total_ms, st, _, _ = run_steps(pplan, True)
         krcv.kr_profile_enable(False)
         del pplan
@@ -387,6 +389,7 @@ def run_ours(args):
         "config": {"workload": workload_desc(cfg, args.seed), "n": n, "m": m,
                    "kernel": workloads.KERNEL_NAMES[k], "seed": args.seed,
                    "parallelism": f"row-shard x{world}" + (
+                       " (cost-balanced cuts from rank 0's calibration in the first warm-up step)"
                        f" + {os.environ.get('KRCV_BENCH_BACKEND', 'nccl')} all_reduce(2m+2 fp64)" if world > 1 else ""),
                    "l2": "flushed between timed steps (256 MiB write, outside the events)",
                    "launch": ("CUDA graph replay of the whole search (GridSearch(graph=True))" if world == 1

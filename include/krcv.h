@@ -256,6 +256,21 @@ int kr_cv_shard_algo_async(const double *d_x, const double *d_y, int64_t n,
                            void *cuda_stream);
 
 /*
+ * kr_cv_rows_async -- kr_cv_shard_algo_async for an explicit range of rows:
+ * rows [row_lo, row_hi) of the stable x-sorted order (0 <= row_lo <= row_hi
+ * <= n, else KR_EARG; an empty range gives a zero partial).  Any set of
+ * disjoint ranges covering [0, n) sums to the unsharded partial, so ranks may
+ * take unequal row counts of equal cost (cost-balanced
+ * partition; the oracle reproduces a range as sorted_rows(x)[lo:hi]).
+ * Arguments, layout, ownership and errors otherwise as kr_cv_shard_algo_async.
+ */
+int kr_cv_rows_async(const double *d_x, const double *d_y, int64_t n,
+                     const double *d_h, int32_t m, int32_t kernel, int32_t algo,
+                     int64_t row_lo, int64_t row_hi,
+                     double *d_partial, void *d_workspace, size_t workspace_bytes,
+                     void *cuda_stream);
+
+/*
  * kr_cv_grid_async -- the whole single-GPU grid search on caller-owned device
  * memory, enqueued on `cuda_stream` without synchronising (capturable):
  * kr_cv_shard_algo_async(shard 0 of 1) with the finalize fused into the

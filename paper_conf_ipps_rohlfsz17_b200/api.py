@@ -64,6 +64,32 @@ def finalize_partial(partial, n: int, m: int):
     return torch.from_numpy(cv), torch.from_numpy(neff), best
 
 
+def balanced_cuts(cost, n: int, world: int, align: int = 64) -> list[int]:
+    """Row cut points [0, c_1, ..., c_{P-1}, n] of the sorted order that give
+    every rank the same share of the measured cost.  cost[s]
+    is the time of segment s of S equal segments [floor(s n / S),
+    floor((s+1) n / S)); the cumulative cost is interpolated linearly inside
+    a segment and every inner cut is rounded to a multiple of `align` rows
+    (whole window-kernel tiles), kept non-decreasing within [0, n]."""
+    cost = np.maximum(np.asarray(cost, np.float64), 0.0)
+    S = cost.shape[0]
+    if world <= 1 or S == 0 or not np.isfinite(cost).all() or cost.sum() <= 0.0:
+        return [(r * n) // max(world, 1) for r in range(max(world, 1))] + [n]
+    bounds = np.array([(s * n) // S for s in range(S + 1)], np.float64)
+    cum = np.concatenate([[0.0], np.cumsum(cost)])
+    cuts = [0]
+    for r in range(1, world):
+        target = cum[-1] * r / world
+        s = int(np.searchsorted(cum, target, side="right")) - 1
+        s = min(max(s, 0), S - 1)
+        frac = 0.0 if cost[s] <= 0.0 else (target - cum[s]) / cost[s]
+        row = bounds[s] + frac * (bounds[s + 1] - bounds[s])
+        c = int(round(row / align)) * align
+        cuts.append(min(max(c, cuts[-1]), n))
+    cuts.append(n)
+    return cuts
+
+
 class GridSearch:
     """Reusable device plan for one (n, m, kernel) on one GPU / one rank.
 
@@ -72,7 +98,7 @@ class GridSearch:
     """
 
     def __init__(self, n: int, h, kernel="epanechnikov", device=None, rank: int = 0, world: int = 1,
-                 group=None, algo="auto", estimator: str = "nw", graph: bool = False):
+                 group=None, algo="auto", estimator: str = "nw", graph: bool = False, balance: bool = False):
         import torch
 
         self.torch = torch
@@ -94,6 +120,13 @@ class GridSearch:
         self._g = None
         self._gkey = None
         self.rank, self.world, self.group = int(rank), int(world), group
+        # balance=True (Nadaraya-Watson, world > 1): on the first run, rank 0
+        # times the device path on 4 P equal row segments, cuts the sorted
+        # rows at equal cumulative cost (balanced_cuts) and broadcasts the
+        # cuts; every later run takes rows [cut_r, cut_{r+1}) through
+        # kr_cv_rows_async.  Equal-row shards otherwise.
+        self.balance = bool(balance) and self.world > 1 and estimator == "nw"
+        self.rows = None
         self.h = h_host
         self.d_h = torch.as_tensor(h_host, device=self.device)
         self._ws_raw = krcv.workspace(self.n, self.m, self.device)
@@ -137,10 +170,45 @@ class GridSearch:
             krcv.kr_cv_grid_async(d_x, d_y, self.d_h, self.kernel, self.cv, self.neff, self.best_status, self.ws,
                                   algo=self.algo)
             return
-        krcv.kr_cv_shard_async(d_x, d_y, self.d_h, self.kernel, self.rank, self.world, self.partial, self.ws,
-                               algo=self.algo)
+        if self.balance:
+            if self.rows is None:
+                self.rows = self._balanced_rows(d_x, d_y)
+            krcv.kr_cv_rows_async(d_x, d_y, self.d_h, self.kernel, self.rows[0], self.rows[1], self.partial,
+                                  self.ws, algo=self.algo)
+        else:
+            krcv.kr_cv_shard_async(d_x, d_y, self.d_h, self.kernel, self.rank, self.world, self.partial, self.ws,
+                                   algo=self.algo)
         allreduce_partial(self.partial, self.group)
         krcv.kr_finalize_async(self.partial, self.n, self.m, self.cv, self.neff, self.best_status)
+
+    def _balanced_rows(self, d_x, d_y):
+        """(lo, hi) of this rank from rank 0's cost measurement (broadcast)."""
+        torch = self.torch
+        import torch.distributed as dist
+
+        cuts = torch.zeros(self.world + 1, dtype=torch.int64)
+        if self.rank == 0:
+            S = 4 * self.world
+            cost = np.zeros(S)
+            was_on = krcv.kr_profile_enabled()
+            krcv.kr_profile_enable(True)
+            try:
+                for s in range(S):
+                    lo, hi = (s * self.n) // S, ((s + 1) * self.n) // S
+                    for _ in range(2):  # the second run is timed warm
+                        krcv.kr_cv_rows_async(d_x, d_y, self.d_h, self.kernel, lo, hi, self.partial, self.ws,
+                                              algo=self.algo)
+                        cost[s] = krcv.kr_profile_read()[2]  # the window / sweep stage
+            finally:
+                krcv.kr_profile_enable(was_on)
+            cuts = torch.tensor(balanced_cuts(cost, self.n, self.world), dtype=torch.int64)
+        if dist.is_available() and dist.is_initialized():
+            dev_cuts = cuts.to(self.device) if dist.get_backend(self.group) == "nccl" else cuts
+            dist.broadcast(dev_cuts, src=dist.get_global_rank(self.group, 0) if self.group is not None else 0,
+                           group=self.group)
+            cuts = dev_cuts.cpu()
+        c = [int(v) for v in cuts.tolist()]
+        return c[self.rank], c[self.rank + 1]
 
     def result(self) -> CVResult:
         bs = self.best_status.cpu()
@@ -151,12 +219,14 @@ class GridSearch:
 
 
 def cv_grid(x, y, h=None, m: int | None = None, kernel="epanechnikov", device=None, distributed: bool = False,
-            group=None, algo="auto", estimator: str = "nw") -> CVResult:
+            group=None, algo="auto", estimator: str = "nw", balance: bool = False) -> CVResult:
     """LOO-CV grid search.  x, y: numpy arrays or CUDA tensors; h: grid array,
     or None with m for the default grid (§IV P@16146).  With distributed=True
     every rank of the default (or given) process group must call it with the
     same inputs; the result is identical on every rank.  estimator: "nw"
-    (Nadaraya-Watson, Eq.(2)) or "ll" (local-linear, reading Q25)."""
+    (Nadaraya-Watson, Eq.(2)) or "ll" (local-linear, reading Q25).
+    balance: cost-balanced row cuts (GridSearch) -- a one-off calibration
+    that pays off for plans run repeatedly, not for one call."""
     import torch
 
     if h is None:
@@ -172,7 +242,7 @@ def cv_grid(x, y, h=None, m: int | None = None, kernel="epanechnikov", device=No
     dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
     d_x = torch.as_tensor(x, dtype=torch.float64, device=dev).contiguous()
     d_y = torch.as_tensor(y, dtype=torch.float64, device=dev).contiguous()
-    plan = GridSearch(d_x.numel(), h, kernel, dev, rank, world, group, algo, estimator)
+    plan = GridSearch(d_x.numel(), h, kernel, dev, rank, world, group, algo, estimator, balance=balance)
     plan.run(d_x, d_y)
     return plan.result()
 

@@ -804,7 +804,7 @@ static int enqueue_sort(const double *d_x, const double *d_y, int64_t n, const d
 static int enqueue(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m, int32_t kernel,
                    int32_t algo, int32_t shard, int32_t nshards, double *d_partial, FinOut fin,
                    void *d_workspace, size_t workspace_bytes, void *cuda_stream, bool reuse_sorted = false,
-                   bool ll = false)
+                   bool ll = false, int64_t range_lo = -1, int64_t range_hi = -1)
 {
     if (!d_x || !d_y || !d_h || !d_workspace) return KR_EARG;
     if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return KR_EARG;
@@ -822,7 +822,9 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     // the dense path is only for it
     if ((kernel == KR_GAUSSIAN) != (algo == KR_ALGO_DENSE || (algo == KR_ALGO_AUTO && kernel == KR_GAUSSIAN)))
         return KR_EARG;
-    if (nshards < 1 || shard < 0 || shard >= nshards) return KR_EARG;
+    const bool ranged = range_lo >= 0;  // explicit rows [range_lo, range_hi) (kr_cv_rows_async)
+    if (ranged ? !(range_lo <= range_hi && range_hi <= n) : (nshards < 1 || shard < 0 || shard >= nshards))
+        return KR_EARG;
     if ((reinterpret_cast<uintptr_t>(d_workspace) & 255u) != 0) return KR_EARG;
     WsLayout L;
     if (!ws_layout(n, m, &L)) return KR_ECUDA;
@@ -840,8 +842,8 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     const int nn = (int)n;
 
     // Rows of this shard in sorted order.
-    const int lo = (int)(((int64_t)shard * n) / nshards);
-    const int hi = (int)(((int64_t)(shard + 1) * n) / nshards);
+    const int lo = ranged ? (int)range_lo : (int)(((int64_t)shard * n) / nshards);
+    const int hi = ranged ? (int)range_hi : (int)(((int64_t)(shard + 1) * n) / nshards);
     if (algo == KR_ALGO_AUTO) algo = kernel == KR_GAUSSIAN ? KR_ALGO_DENSE : auto_algo(n, hi - lo, m, kernel);
     const bool prefix = algo == KR_ALGO_PREFIX;
     const bool dense = algo == KR_ALGO_DENSE;
@@ -1003,6 +1005,18 @@ extern "C" int kr_cv_grid_async(const double *d_x, const double *d_y, int64_t n,
 {
     return enqueue_grid(d_x, d_y, n, d_h, m, kernel, algo, d_cv, d_neff, d_best_status, d_workspace,
                         workspace_bytes, cuda_stream, false);
+}
+
+extern "C" int kr_cv_rows_async(const double *d_x, const double *d_y, int64_t n,
+                                const double *d_h, int32_t m, int32_t kernel, int32_t algo,
+                                int64_t row_lo, int64_t row_hi,
+                                double *d_partial, void *d_workspace, size_t workspace_bytes,
+                                void *cuda_stream)
+{
+    if (!d_partial || row_lo < 0) return KR_EARG;
+    FinOut fin{};
+    return enqueue(d_x, d_y, n, d_h, m, kernel, algo, 0, 1, d_partial, fin, d_workspace, workspace_bytes,
+                   cuda_stream, false, false, row_lo, row_hi);
 }
 
 extern "C" int kr_cv_shard_async(const double *d_x, const double *d_y, int64_t n,

@@ -36,7 +36,7 @@ KR_MAX_M = 65536
 # Every symbol include/krcv.h declares (checked by tests/test_abi.py).
 EXPORTS = (
     "kr_cv_grid", "kr_cv_grid_ex", "kr_cv_grid_algo", "kr_cv_refine", "kr_validate_grid", "kr_workspace_bytes",
-    "kr_cv_shard_async", "kr_cv_shard_algo_async", "kr_cv_grid_async", "kr_finalize", "kr_finalize_async", "kr_default_grid",
+    "kr_cv_shard_async", "kr_cv_shard_algo_async", "kr_cv_rows_async", "kr_cv_grid_async", "kr_finalize", "kr_finalize_async", "kr_default_grid",
     "kr_strerror", "kr_last_cuda_error", "kr_version", "kr_release",
     "kr_profile_enable", "kr_profile_read", "kr_launch_count", "kr_last_algo",
     "kr_kde_lscv", "kr_kde_lscv_async", "kr_kde_shard_async", "kr_kde_finalize",
@@ -79,12 +79,13 @@ def _lib() -> ctypes.CDLL:
     lib.kr_workspace_bytes.restype = sz
     lib.kr_cv_shard_async.argtypes = [P, P, i64, P, i32, i32, i32, i32, P, P, sz, P]
     lib.kr_cv_shard_algo_async.argtypes = [P, P, i64, P, i32, i32, i32, i32, i32, P, P, sz, P]
+    lib.kr_cv_rows_async.argtypes = [P, P, i64, P, i32, i32, i32, i64, i64, P, P, sz, P]
     lib.kr_cv_grid_async.argtypes = [P, P, i64, P, i32, i32, i32, P, P, P, P, sz, P]
     lib.kr_finalize.argtypes = [P, i64, i32, P, P, P]
     lib.kr_finalize_async.argtypes = [P, i64, i32, P, P, P, P, P]
     lib.kr_default_grid.argtypes = [P, i64, i32, P]
     for f in ("kr_cv_grid", "kr_cv_grid_ex", "kr_cv_grid_algo", "kr_cv_refine", "kr_validate_grid", "kr_cv_shard_async",
-              "kr_cv_shard_algo_async", "kr_cv_grid_async",
+              "kr_cv_shard_algo_async", "kr_cv_rows_async", "kr_cv_grid_async",
               "kr_finalize", "kr_finalize_async", "kr_default_grid"):
         getattr(lib, f).restype = ctypes.c_int
     lib.kr_strerror.argtypes = [ctypes.c_int]
@@ -225,6 +226,25 @@ def kr_workspace_bytes(n: int, m: int) -> int:
 
 
 # ---------------------------------------------------------------- device API
+def kr_cv_rows_async(d_x, d_y, d_h, kernel, row_lo: int, row_hi: int, d_partial, d_ws, stream=None,
+                     algo="auto") -> None:
+    """Enqueue the device pipeline for rows [row_lo, row_hi) of the sorted
+    order (cost-balanced sharding); tensors as kr_cv_shard_async."""
+    import torch
+
+    n, m = d_x.numel(), d_h.numel()
+    for t, name in ((d_x, "x"), (d_y, "y"), (d_h, "h"), (d_partial, "partial")):
+        if not (t.is_cuda and t.dtype == torch.float64 and t.is_contiguous()):
+            raise ValueError(f"{name} must be a contiguous float64 CUDA tensor")
+    if d_partial.numel() != partial_len(m):
+        raise ValueError("partial must have 2m+2 elements")
+    s = torch.cuda.current_stream(d_x.device) if stream is None else stream
+    st = _lib().kr_cv_rows_async(d_x.data_ptr(), d_y.data_ptr(), n, d_h.data_ptr(), m, _kernel_id(kernel),
+                                 _algo_id(algo), int(row_lo), int(row_hi), d_partial.data_ptr(), d_ws.data_ptr(),
+                                 d_ws.numel() * d_ws.element_size(), ctypes.c_void_p(s.cuda_stream))
+    _check(st, "kr_cv_rows_async")
+
+
 def kr_cv_shard_async(d_x, d_y, d_h, kernel, shard: int, nshards: int, d_partial, d_ws, stream=None,
                       algo="auto") -> None:
     """Enqueue the sharded device pipeline.  All tensor arguments are CUDA
@@ -284,8 +304,17 @@ def kr_finalize_async(d_partial, n: int, m: int, d_cv, d_neff, d_best_status, st
     _check(st, "kr_finalize_async")
 
 
+_PROFILING = {"on": False}
+
+
 def kr_profile_enable(on: bool) -> None:
     _lib().kr_profile_enable(1 if on else 0)
+    _PROFILING["on"] = bool(on)
+
+
+def kr_profile_enabled() -> bool:
+    """Whether kr_profile_enable(True) is in effect (as set through this binding)."""
+    return _PROFILING["on"]
 
 
 def kr_profile_read():

@@ -84,3 +84,38 @@ def test_shard_bounds_partition():
             assert all(hi - lo in (n // P, n // P + 1) for lo, hi in b)
     with pytest.raises(ValueError):
         api.shard_bounds(10, 2, 2)
+
+
+# ------------------------------------------------------------ balanced cuts
+def test_balanced_cuts_uniform_cost_is_equal_rows():
+    from paper_conf_ipps_rohlfsz17_b200.api import balanced_cuts
+    cuts = balanced_cuts(np.ones(32), 64 * 1000, 8)
+    assert cuts == [r * 8000 for r in range(9)]
+
+
+def test_balanced_cuts_equalise_skewed_cost():
+    """A slow tail (the C5 shape) moves the cuts so every rank's share of the
+    cost is within one alignment block of 1/P, and the cuts tile [0, n)."""
+    from paper_conf_ipps_rohlfsz17_b200.api import balanced_cuts
+    rng = np.random.default_rng(3)
+    S, n, P = 128, 1_000_000, 8
+    cost = 1.0 + rng.uniform(0, 0.2, S)
+    cost[-8:] *= 4.0
+    cuts = balanced_cuts(cost, n, P)
+    assert cuts[0] == 0 and cuts[-1] == n and all(a <= b for a, b in zip(cuts, cuts[1:]))
+    assert all(c % 64 == 0 for c in cuts[1:-1])
+    # per-row cost, piecewise constant over the segments
+    bounds = [(s * n) // S for s in range(S + 1)]
+    row_cost = np.repeat(cost / np.diff(bounds), np.diff(bounds))
+    share = np.array([row_cost[a:b].sum() for a, b in zip(cuts, cuts[1:])]) / row_cost.sum()
+    assert np.max(np.abs(share - 1.0 / P)) <= 64 * row_cost.max() / row_cost.sum() + 1e-12
+    equal = np.array([row_cost[(r * n) // P:((r + 1) * n) // P].sum() for r in range(P)]) / row_cost.sum()
+    assert share.max() < equal.max()
+
+
+def test_balanced_cuts_degenerate_inputs():
+    from paper_conf_ipps_rohlfsz17_b200.api import balanced_cuts
+    assert balanced_cuts(np.zeros(16), 1000, 4) == [0, 250, 500, 750, 1000]   # no cost measured
+    assert balanced_cuts(np.ones(16), 1000, 1) == [0, 1000]
+    cuts = balanced_cuts(np.r_[np.zeros(15), 1.0], 100, 4)                   # all cost in the last segment
+    assert cuts[0] == 0 and cuts[-1] == 100 and all(a <= b for a, b in zip(cuts, cuts[1:]))

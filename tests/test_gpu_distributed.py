@@ -25,7 +25,7 @@ def _free_port() -> int:
         return s.getsockname()[1]
 
 
-def _worker(rank, world, port, cfg, n, estimator, algo, q):
+def _worker(rank, world, port, cfg, n, estimator, algo, q, balance=False):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
@@ -34,20 +34,22 @@ def _worker(rank, world, port, cfg, n, estimator, algo, q):
 
         torch.cuda.set_device(0)
         x, y, h, k = workloads.make(cfg, seed=6, n=n)
-        r = api.cv_grid(x, y, h, kernel=k, distributed=True, algo=algo, estimator=estimator)
+        r = api.cv_grid(x, y, h, kernel=k, distributed=True, algo=algo, estimator=estimator, balance=balance)
         q.put((rank, r.cv.cpu().numpy(), r.neff.cpu().numpy(), r.best))
     finally:
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world,cfg,n,estimator,algo", [
-    (2, "C2", 3000, "nw", "auto"),
-    (3, "C5", 2500, "nw", "auto"),
-    (2, "C2", 3000, "nw", "sweep"),
-    (2, "C1", 1000, "nw", "hist"),
-    (3, "C2", 2000, "ll", "auto"),
+@pytest.mark.parametrize("world,cfg,n,estimator,algo,balance", [
+    (2, "C2", 3000, "nw", "auto", False),
+    (3, "C5", 2500, "nw", "auto", False),
+    (2, "C2", 3000, "nw", "sweep", False),
+    (2, "C1", 1000, "nw", "hist", False),
+    (3, "C2", 2000, "ll", "auto", False),
+    (3, "C5", 2500, "nw", "auto", True),    # cost-balanced cuts (rank 0 calibrates, broadcast)
+    (2, "C2", 3000, "nw", "sweep", True),
 ])
-def test_sharded_device_path_matches_single_gpu(world, cfg, n, estimator, algo):
+def test_sharded_device_path_matches_single_gpu(world, cfg, n, estimator, algo, balance):
     import oracle
     import workloads
     from paper_conf_ipps_rohlfsz17_b200 import api
@@ -56,7 +58,8 @@ def test_sharded_device_path_matches_single_gpu(world, cfg, n, estimator, algo):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, cfg, n, estimator, algo, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, cfg, n, estimator, algo, q, balance))
+             for r in range(world)]
     for p in procs:
         p.start()
     res = [q.get(timeout=600) for _ in range(world)]

@@ -173,6 +173,36 @@ def test_full_size_sampled_shard(cfg, P, shard):
     assert part[2 * m] == 0 and part[2 * m + 1] == 0
 
 
+def test_row_ranges_sum_to_unsharded_and_match_oracle():
+    """kr_cv_rows_async: disjoint unequal row ranges (incl. an empty one and
+    ranges cutting through window-kernel tiles) add up to the unsharded
+    partial, and one range equals the oracle on exactly those sorted rows."""
+    import torch
+    x, y, h, k = workloads.make("C5", seed=2, n=6000)
+    m = h.shape[0]
+    d_x, d_y, d_h = (torch.as_tensor(v, device="cuda") for v in (x, y, h))
+    ws = krcv.aligned(krcv.workspace(x.shape[0], m, "cuda"))
+    part = torch.empty(krcv.partial_len(m), dtype=torch.float64, device="cuda")
+    full = _device_partial(x, y, h, k, 0, 1)
+    cuts = [0, 1, 777, 777, 2048, 4001, 5999, 6000]
+    tot = np.zeros(krcv.partial_len(m))
+    for lo, hi in zip(cuts, cuts[1:]):
+        krcv.kr_cv_rows_async(d_x, d_y, d_h, k, lo, hi, part, ws, algo=ALGO["a"])
+        torch.cuda.synchronize()
+        p = part.cpu().numpy()
+        tot += p
+        if (lo, hi) == (777, 2048):
+            ref = oracle.cv_sorted(x, y, h, k, rows=oracle.sorted_rows(x)[lo:hi])
+            assert cv_rel_err(p[:m], ref.S) <= TIGHT
+            assert np.array_equal(p[m:2 * m].astype(np.int64), ref.neff)
+    assert cv_rel_err(tot[:m], full[:m]) <= 1e-14
+    assert np.array_equal(tot[m:], full[m:])
+    with pytest.raises(krcv.KrcvError):
+        krcv.kr_cv_rows_async(d_x, d_y, d_h, k, 10, 5, part, ws)       # hi < lo
+    with pytest.raises(krcv.KrcvError):
+        krcv.kr_cv_rows_async(d_x, d_y, d_h, k, 0, 6001, part, ws)     # past n
+
+
 @pytest.mark.parametrize("P", [2, 3, 8, 64])
 def test_shard_emulation_sums_to_unsharded(P):
     """T4: shards 0..P-1 on one GPU, summed on the host == unsharded run."""
