@@ -1,0 +1,64 @@
+"""The C-ABI used from plain C (examples/krcv_example.c): compiled with gcc
+against include/krcv.h and linked to libkrcv.so, without Python or PyTorch in
+the process.  CPU tier: the host-only entry points (version, default grid,
+grid validation, argument errors); GPU tier: a whole C2-size search, whose
+optimum must be the oracle's on the same inputs."""
+from __future__ import annotations
+
+import os
+import re
+import shutil
+import subprocess
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+LIBDIR = os.path.join(ROOT, "paper_conf_ipps_rohlfsz17_b200")
+
+
+def _build(tmp_path):
+    if shutil.which("gcc") is None:
+        pytest.skip("gcc not available")
+    exe = str(tmp_path / "krcv_example")
+    subprocess.run(["gcc", "-O2", "-std=c11", "-Wall", "-I", os.path.join(ROOT, "include"),
+                    os.path.join(ROOT, "examples", "krcv_example.c"), "-L", LIBDIR, "-lkrcv",
+                    f"-Wl,-rpath,{LIBDIR}", "-o", exe], check=True, capture_output=True, text=True)
+    return exe
+
+
+def test_c_consumer_host_only(tmp_path):
+    p = subprocess.run([_build(tmp_path), "--host-only"], capture_output=True, text=True, timeout=120)
+    assert p.returncode == 0, p.stdout + p.stderr
+    assert "sm_100a" in p.stdout and "host-only ABI checks: ok" in p.stdout
+
+
+@pytest.mark.gpu
+def test_c_consumer_full_search(tmp_path):
+    import numpy as np
+
+    import oracle
+    p = subprocess.run([_build(tmp_path), "3000", "40"], capture_output=True, text=True, timeout=300)
+    assert p.returncode == 0, p.stdout + p.stderr
+    mt = re.search(r"best b = (\d+), h = (\S+), CV = (\S+)", p.stdout)
+    assert mt, p.stdout
+    # the same xorshift inputs, regenerated here for the oracle
+    s = 0x9E3779B97F4A7C15
+    mask = (1 << 64) - 1
+
+    def urand():
+        nonlocal s
+        s ^= (s << 13) & mask
+        s ^= s >> 7
+        s ^= (s << 17) & mask
+        return (s >> 11) * 2.0 ** -53
+
+    n, m = 3000, 40
+    x = np.empty(n)
+    y = np.empty(n)
+    for i in range(n):
+        x[i] = urand()
+        y[i] = 0.5 * x[i] + 10.0 * x[i] * x[i] + 0.5 * urand()
+    h = oracle.default_grid(x, m)
+    ref = oracle.cv_sorted(x, y, h, oracle.EPANECHNIKOV)
+    assert int(mt.group(1)) == ref.best
+    assert abs(float(mt.group(3)) - ref.cv[ref.best]) <= 1e-9 * ref.cv[ref.best]
