@@ -37,6 +37,10 @@ static bool kernel_ok(int32_t k)
 struct DevCtx {
     std::mutex mu;
     cudaStream_t stream = nullptr;
+    // side streams and events that fork the three input copies into parallel
+    // branches (x on `stream`, y and h on side[0], side[1]) and join them
+    cudaStream_t side[2] = {nullptr, nullptr};
+    cudaEvent_t ev_fork = nullptr, ev_join[2] = {nullptr, nullptr};
     void *ws = nullptr;
     size_t ws_bytes = 0;
     double *dx = nullptr, *dy = nullptr, *dh = nullptr;
@@ -44,7 +48,8 @@ struct DevCtx {
     int32_t cap_m = 0;
     double *dpartial = nullptr;
     // results of the synchronous host path, one block [best, status | cv[m] |
-    // neff[m]] on the device and its pinned mirror: one D2H copy per call
+    // neff[m]] on the device (refinement, KDE) and its pinned mapped mirror, which
+    // the finalize of kr_cv_grid* / kr_ll_cv_grid writes directly (no D2H copy)
     char *dres = nullptr;
     double *dcv = nullptr;
     int64_t *dneff = nullptr;
@@ -85,7 +90,14 @@ static size_t res_bytes(int32_t m) { return 8 + (sizeof(double) + sizeof(int64_t
 
 static int ensure_capacity(DevCtx *c, int64_t n, int32_t m)
 {
-    if (!c->stream) KR_CUDA_TRY(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
+    if (!c->stream) {
+        KR_CUDA_TRY(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
+        for (int i = 0; i < 2; i++) {
+            KR_CUDA_TRY(cudaStreamCreateWithFlags(&c->side[i], cudaStreamNonBlocking));
+            KR_CUDA_TRY(cudaEventCreateWithFlags(&c->ev_join[i], cudaEventDisableTiming));
+        }
+        KR_CUDA_TRY(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+    }
     if (n > c->cap_n) {
         cudaFree(c->dx);
         cudaFree(c->dy);
@@ -179,19 +191,29 @@ static int enqueue_host_call(DevCtx *c, const double *x, const double *y, int64_
                              int32_t kernel, int32_t algo, bool ll)
 {
     cudaStream_t s = c->stream;
+    // the three input copies run as parallel branches (one copy engine each)
+    KR_CUDA_TRY(cudaEventRecord(c->ev_fork, s));
+    for (int i = 0; i < 2; i++) KR_CUDA_TRY(cudaStreamWaitEvent(c->side[i], c->ev_fork, 0));
     KR_CUDA_TRY(cudaMemcpyAsync(c->dx, x, sizeof(double) * n, cudaMemcpyHostToDevice, s));
-    KR_CUDA_TRY(cudaMemcpyAsync(c->dy, y, sizeof(double) * n, cudaMemcpyHostToDevice, s));
-    KR_CUDA_TRY(cudaMemcpyAsync(c->dh, h, sizeof(double) * m, cudaMemcpyHostToDevice, s));
-    // the result block laid out for this call's m (fits the capacity's)
-    int32_t *dbest = reinterpret_cast<int32_t *>(c->dres);
-    double *dcv = reinterpret_cast<double *>(c->dres + 8);
-    int64_t *dneff = reinterpret_cast<int64_t *>(c->dres + 8 + sizeof(double) * m);
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dy, y, sizeof(double) * n, cudaMemcpyHostToDevice, c->side[0]));
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dh, h, sizeof(double) * m, cudaMemcpyHostToDevice, c->side[1]));
+    for (int i = 0; i < 2; i++) {
+        KR_CUDA_TRY(cudaEventRecord(c->ev_join[i], c->side[i]));
+        KR_CUDA_TRY(cudaStreamWaitEvent(s, c->ev_join[i], 0));
+    }
+    // the finalize (fused into the reduction's last CTA) writes the result
+    // block -- [best, status | cv[m] | neff[m]] laid out for this call's m --
+    // straight into the mapped pinned staging: no device-to-host copy
+    char *pres = nullptr;
+    KR_CUDA_TRY(cudaHostGetDevicePointer(reinterpret_cast<void **>(&pres), c->pres, 0));
+    int32_t *dbest = reinterpret_cast<int32_t *>(pres);
+    double *dcv = reinterpret_cast<double *>(pres + 8);
+    int64_t *dneff = reinterpret_cast<int64_t *>(pres + 8 + sizeof(double) * m);
     const int st = ll ? kr_ll_cv_grid_async(c->dx, c->dy, n, c->dh, m, kernel, dcv, dneff, dbest, c->ws,
                                             c->ws_bytes, s)
                       : kr_cv_grid_async(c->dx, c->dy, n, c->dh, m, kernel, algo, dcv, dneff, dbest, c->ws,
                                          c->ws_bytes, s);
     if (st) return st;
-    KR_CUDA_TRY(cudaMemcpyAsync(c->pres, c->dres, res_bytes(m), cudaMemcpyDeviceToHost, s));  // one copy
     return KR_OK;
 }
 
@@ -495,6 +517,14 @@ extern "C" int kr_release(void)
         cudaFree(c->dres);
         cudaFreeHost(c->pres);
         if (c->stream) cudaStreamDestroy(c->stream);
+        for (int i = 0; i < 2; i++) {
+            if (c->side[i]) cudaStreamDestroy(c->side[i]);
+            if (c->ev_join[i]) cudaEventDestroy(c->ev_join[i]);
+            c->side[i] = nullptr;
+            c->ev_join[i] = nullptr;
+        }
+        if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+        c->ev_fork = nullptr;
         c->gexec = nullptr;
         c->gx = c->gy = c->gh = nullptr;
         c->ws = nullptr;
