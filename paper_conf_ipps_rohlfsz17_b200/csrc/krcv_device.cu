@@ -27,6 +27,7 @@
 #include <cstdlib>
 #include <cstring>
 #include "krcv_internal.h"
+#include "krcv_pdl.cuh"
 #include "krcv_sweep.cuh"
 #include "krcv_sweep_gxg.cuh"
 #include "krcv_sort.cuh"
@@ -70,6 +71,7 @@ __global__ void gather_kernel(const double *__restrict__ x, const double *__rest
                               const uint32_t *__restrict__ order, int n, double2 *__restrict__ xy,
                               uint32_t *__restrict__ perm, int *__restrict__ tile_counter)
 {
+    pdl_wait();  // krcv_pdl.cuh
     const int stride = gridDim.x * blockDim.x;
     const int tid = blockIdx.x * blockDim.x + threadIdx.x;
     for (int k = tid; k < n; k += stride) {
@@ -172,6 +174,7 @@ __global__ void __launch_bounds__(kReduceThreads)
 reduce_kernel(const double *__restrict__ tileS, const uint8_t *__restrict__ tileN, int ntiles, int m,
               const unsigned *__restrict__ status, double *__restrict__ partial, FinOut fin)
 {
+    pdl_wait();  // krcv_pdl.cuh
     __shared__ double sS[kReduceThreads];
     __shared__ long long sN[kReduceThreads];
     __shared__ int sI[kReduceThreads];
@@ -224,6 +227,37 @@ reduce_kernel(const double *__restrict__ tileS, const uint8_t *__restrict__ tile
     __threadfence();
     finalize_body<kReduceThreads>(partial, fin.n, m, fin.cv, fin.neff, fin.best, fin.status, sS, sI);
     if (threadIdx.x == 0) *fin.done = 0u;
+}
+
+// ---------------------------------------------------------------------------
+// Programmatic dependent launch (krcv_pdl.cuh): only kernels that start with
+// pdl_wait() are launched this way.  KRCV_PDL=0 launches them plainly.
+// ---------------------------------------------------------------------------
+static bool pdl_enabled()
+{
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("KRCV_PDL");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
+
+template <typename... KArgs, typename... Args>
+static void launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                       Args... args)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);  // errors surface via cudaGetLastError
 }
 
 // ---------------------------------------------------------------------------
@@ -450,7 +484,7 @@ static void launch_rank_sort(const double *d_x, const double *d_y, int n, const 
                              uint32_t *khi, uint32_t *idx, int *rank, unsigned *status, int nchunks, cudaStream_t st)
 {
     chunk_sort_kernel<T, I><<<nchunks, T, 0, st>>>(d_x, d_y, n, d_h, m, keys, khi, idx, rank, status);
-    if (nchunks > 1) rank_count_kernel<T, I><<<dim3(nchunks, nchunks), T, 0, st>>>(keys, khi, idx, rank);
+    if (nchunks > 1) launch_pdl(rank_count_kernel<T, I>, dim3(nchunks, nchunks), dim3(T), 0, st, keys, khi, idx, rank);
 }
 
 // KR_ALGO_AUTO: the window-prefix path does O(n m log) work against the
@@ -498,13 +532,15 @@ static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, cha
         pfx_one_cta_kernel<KERN><<<1, kPfx1Threads, 0, st>>>(xy, n, P, (int)L.pstride, xs, ymax);
     } else if (items == 1) {
         const int ntiles = (n + kPfxThreads) / kPfxThreads;  // tiles covering P[0..n]
-        pfx_tile_reduce_kernel<KERN, 1><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, ymax);
-        pfx_tile_scan_kernel<KERN, 1><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, P, (int)L.pstride, xs);
+        launch_pdl(pfx_tile_reduce_kernel<KERN, 1>, dim3(ntiles), dim3(kPfxThreads), 0, st, xy, n, tot, ntiles, ymax);
+        launch_pdl(pfx_tile_scan_kernel<KERN, 1>, dim3(ntiles), dim3(kPfxThreads), 0, st, xy, n,
+                   (const double2 *)tot, ntiles, P, (int)L.pstride, xs);
     } else {
         const int ntiles = (n + kPfxThreads * kPfxItemsMax) / (kPfxThreads * kPfxItemsMax);
-        pfx_tile_reduce_kernel<KERN, kPfxItemsMax><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, ymax);
-        pfx_tile_scan_kernel<KERN, kPfxItemsMax><<<ntiles, kPfxThreads, 0, st>>>(xy, n, tot, ntiles, P,
-                                                                                 (int)L.pstride, xs);
+        launch_pdl(pfx_tile_reduce_kernel<KERN, kPfxItemsMax>, dim3(ntiles), dim3(kPfxThreads), 0, st, xy, n, tot,
+                   ntiles, ymax);
+        launch_pdl(pfx_tile_scan_kernel<KERN, kPfxItemsMax>, dim3(ntiles), dim3(kPfxThreads), 0, st, xy, n,
+                   (const double2 *)tot, ntiles, P, (int)L.pstride, xs);
     }
 }
 
@@ -608,8 +644,8 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
         window_kernel_b2<KERN, 1><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
                                                                   nbc, ymax, tileS, tileN, counter, sms);
     else if (K == 3)
-        window_kernel_b2<KERN, 0><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
-                                                                  nbc, ymax, tileS, tileN, counter, sms);
+        launch_pdl(window_kernel_b2<KERN, 0>, dim3(blocks), dim3(kWinThreads), 0, st, xs, (const double2 *)xy, P,
+                   (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter, sms);
     else if (K == 5)
         window_kernel_coop<KERN><<<blocks, kCoopRows, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
                                                                nbc, ymax, tileS, tileN, counter);
@@ -623,8 +659,9 @@ static void launch_window_k(const double2 *xy, int n, const double *h, int m, in
         window_kernel<KERN, (K == 3 || K >= 5) ? 1 : K, 1><<<blocks, kWinThreads, 0, st>>>(
             xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter, sms);
     else
-        window_kernel<KERN, (K == 3 || K >= 5) ? 1 : K, 0><<<blocks, kWinThreads, 0, st>>>(
-            xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter, sms);
+        launch_pdl(window_kernel<KERN, (K == 3 || K >= 5) ? 1 : K, 0>, dim3(blocks), dim3(kWinThreads), 0, st, xs,
+                   (const double2 *)xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN,
+                   counter, sms);
 }
 
 template <int KERN>
@@ -780,7 +817,7 @@ static int enqueue_sort(const double *d_x, const double *d_y, int64_t n, const d
         default: launch_rank_sort<128, 2>(d_x, d_y, nn, d_h, m, keys_in, khi, vals_in, rank, status, nchunks, st); break;
         }
         const int npad = nchunks * chunk;
-        rank_scatter_kernel<<<(npad + 255) / 256, 256, 0, st>>>(vals_in, rank, nn, npad, d_x, d_y, xy, perm,
+        launch_pdl(rank_scatter_kernel, dim3((npad + 255) / 256), dim3(256), 0, st, vals_in, rank, nn, npad, d_x, d_y, xy, perm,
                                                                  counter);
         launches += nchunks > 1 ? 1 : 0;
         launches += 2;
@@ -790,7 +827,7 @@ static int enqueue_sort(const double *d_x, const double *d_y, int64_t n, const d
         e = cub::DeviceRadixSort::SortPairs(ws + L.cub, cub_bytes, keys_in, keys_out, vals_in, vals_out,
                                             nn, 0, 64, st);
         if (e != cudaSuccess) { set_cuda_error("cub::DeviceRadixSort::SortPairs", (int)e); return KR_ECUDA; }
-        gather_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, vals_out, nn, xy, perm, counter);
+        launch_pdl(gather_kernel, dim3(grid_for(n, 256)), dim3(256), 0, st, d_x, d_y, vals_out, nn, xy, perm, counter);
         launches += 2 + cub_sort_launches(n);
     }
     *launches_out += launches;
@@ -959,8 +996,8 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     prof_mark(3, st);
     if (injected_failure("reduce")) return KR_ECUDA;
     NvtxScope nv_red("krcv: a5 reduction (+ finalize)");
-    reduce_kernel<<<m < 148 * 8 ? m : 148 * 8, kReduceThreads, 0, st>>>(tileS, tileN, ntiles, m, status,
-                                                                        d_partial, fin);
+    launch_pdl(reduce_kernel, dim3(m < 148 * 8 ? m : 148 * 8), dim3(kReduceThreads), 0, st, (const double *)tileS,
+               (const uint8_t *)tileN, ntiles, m, (const unsigned *)status, d_partial, fin);
     launches += 1;
     prof_mark(4, st);
     g_prof.recorded = g_prof.on;

@@ -40,6 +40,8 @@
 //                      the same tile-partial layout the sweep uses (a5).
 #pragma once
 
+#include "krcv_pdl.cuh"
+
 #include <cuda_runtime.h>
 
 #include <climits>
@@ -203,6 +205,7 @@ __global__ void __launch_bounds__(kPfxThreads)
 pfx_tile_reduce_kernel(const double2 *__restrict__ xy, int n, double2 *__restrict__ tot, int ntiles,
                        unsigned long long *__restrict__ ymax_bits)
 {
+    pdl_wait();  // krcv_pdl.cuh
     constexpr int K = NMom<KERN>::v;
     __shared__ double2 wsum[K][kPfxThreads / 32];
     const int t = threadIdx.x, lane = t & 31, w = t >> 5;
@@ -250,6 +253,7 @@ __global__ void __launch_bounds__(kPfxThreads)
 pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__restrict__ tot, int ntiles,
                      double *__restrict__ P, int pstride, double *__restrict__ xs)
 {
+    pdl_wait();  // krcv_pdl.cuh
     constexpr int K = NMom<KERN>::v;
     __shared__ double2 wsum[K][kPfxThreads / 32];
     __shared__ double2 base_s[K];
@@ -722,6 +726,7 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
               int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
               uint8_t *__restrict__ tileN, int *__restrict__ tile_counter, int nsm)
 {
+    pdl_wait();  // krcv_pdl.cuh
     const int lane = threadIdx.x & 31;
     const double o = pfx_origin(xy, n);
     const double ymax = __longlong_as_double((long long)*ymax_bits);
@@ -862,6 +867,7 @@ window_kernel_b2(const double *__restrict__ xs, const double2 *__restrict__ xy, 
                  int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
                  uint8_t *__restrict__ tileN, int *__restrict__ tile_counter, int nsm)
 {
+    pdl_wait();  // krcv_pdl.cuh
     const int lane = threadIdx.x & 31;
     const double o = pfx_origin(xy, n);
     const double ymax = __longlong_as_double((long long)*ymax_bits);

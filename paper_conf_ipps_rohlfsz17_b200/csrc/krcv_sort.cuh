@@ -19,6 +19,8 @@
 //      sort by x.
 #pragma once
 
+#include "krcv_pdl.cuh"
+
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -110,6 +112,7 @@ __global__ void __launch_bounds__(kChunkThreads)
 rank_count_kernel(const uint64_t *__restrict__ keys, const uint32_t *__restrict__ khi,
                   const uint32_t *__restrict__ idx, int *__restrict__ rank)
 {
+    pdl_wait();  // krcv_pdl.cuh
     constexpr int kChunk = kChunkThreads * kChunkItems;
     const int c = blockIdx.x, cc = blockIdx.y;
     if (c == cc) return;
@@ -162,6 +165,7 @@ rank_scatter_kernel(const uint32_t *__restrict__ idx, const int *__restrict__ ra
                     const double *__restrict__ x, const double *__restrict__ y, double2 *__restrict__ xy,
                     uint32_t *__restrict__ perm, int *__restrict__ tile_counter)
 {
+    pdl_wait();  // krcv_pdl.cuh
     const int g = blockIdx.x * blockDim.x + threadIdx.x;
     if (g < kPad) {
         xy[-1 - g] = make_double2(-INFINITY, 0.0);
