@@ -148,15 +148,29 @@ class ClockSampler:
                 "sm_max_mhz": self.max_mhz, "reasons": names, "samples": len(self.samples)}
 
 
-def ncu_traffic(config: str, algo: str):
-    """DRAM bytes per launch of the dominant kernel from the committed ncu
-    capture for this (config, algo) (profiles/ncu_traffic.json), else None."""
+def ncu_entry(config: str, algo: str):
+    """The committed ncu capture's entry for this (config, algo)
+    (profiles/ncu_traffic.json), else None."""
     try:
         with open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "ncu_traffic.json")) as f:
-            e = json.load(f).get(f"{config}/{algo}")
-        return None if e is None else e["bytes"]
-    except (OSError, ValueError, KeyError):
+            return json.load(f).get(f"{config}/{algo}")
+    except (OSError, ValueError):
         return None
+
+
+def ncu_traffic(config: str, algo: str):
+    """DRAM bytes per launch of the dominant kernel from the committed ncu
+    capture for this (config, algo), else None."""
+    e = ncu_entry(config, algo)
+    return None if e is None else e.get("bytes")
+
+
+def ncu_context(config: str, algo: str):
+    """Pipe / issue / L1 counters of the same capture (what bounds frac)."""
+    e = ncu_entry(config, algo)
+    if e is None:
+        return None
+    return {k: v for k, v in e.items() if k not in ("bytes", "kernel")} or None
 
 
 # --------------------------------------------------------------- cpu oracle
@@ -365,6 +379,7 @@ def run_ours(args):
                          "sweep": sum(main_ms) / args.steps, "reduce_finalize": sum(red_ms) / args.steps},
             "roofline": {"bound": "alu", "kernel": kname, "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
                          "frac": achieved / peak, "traffic": ncu_traffic(args.config, used),
+                         "ncu": ncu_context(args.config, used),
                          "flops_per_launch": flops, "flops_basis": basis,
                          "peak_note": "FP64: 148 SM x 64 FMA lanes x 2 flop x 1965 MHz (derived, DESIGN.md)",
                          "kernel_ms": main_total / args.steps,
