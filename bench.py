@@ -56,6 +56,24 @@ FLOPS_PER_WINDOW = {0: 6, 1: 25, 2: 30}
 FLOPS_PER_PAIR_BW_DENSE = 35
 
 
+def fp64_peak():
+    """(TFLOP/s, note) of the FP64 roofline denominator: the DFMA throughput
+    measured on a B200 of this pool by tools/fp64_peak.py (committed as
+    profiles/fp64_peak.json with its clock record), else the derived nominal
+    figure 148 x 64 x 2 x 1965 MHz."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "fp64_peak.json")) as f:
+            d = json.load(f)
+        c = d.get("clocks", {})
+        return float(d["dfma_tflops"]), (
+            f"FP64 DFMA throughput measured by tools/fp64_peak.py on {d.get('gpu', 'B200')} "
+            f"({d.get('when', '?')}, SM {c.get('sm_mhz')} of {c.get('sm_max_mhz')} MHz, reasons {c.get('reasons')}; "
+            f"profiles/fp64_peak.json) -- of measured")
+    except (OSError, ValueError, KeyError):
+        return (SM_COUNT * FP64_LANES_PER_SM * 2 * SM_MAX_MHZ_NOMINAL * 1e6 / 1e12,
+                "FP64: 148 SM x 64 FMA lanes x 2 flop x 1965 MHz (derived nominal; no measurement committed)")
+
+
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -334,28 +352,29 @@ def run_ours(args):
                     launches += krcv.kr_launch_count() + (1 if world > 1 else 0)  # + finalize (fused at N=1)
                 torch.cuda.synchronize()
             barrier()
-            return sum(starts[s].elapsed_time(ends[s]) for s in range(args.steps)), st, launches, clk
+            # median step; the driver's clock brackets all K
+            return statistics.median(starts[s].elapsed_time(ends[s]) for s in range(args.steps)), st, launches, clk
 
         krcv.kr_profile_enable(False)
         plan = GridSearch(n, h, k, device=dev, rank=rank, world=world, algo=algo, graph=(world == 1),
                           balance=(world > 1))
-        total_ms, _, launches, clk = run_steps(plan, False)
+        step_ms, _, launches, clk = run_steps(plan, False)
         krcv.kr_profile_enable(True)
         pplan = GridSearch(n, h, k, device=dev, rank=rank, world=world, algo=algo, graph=(world == 1),
                           balance=(world > 1))
-        prof_total_ms, st, _, _ = run_steps(pplan, True)
+        prof_step_ms, st, _, _ = run_steps(pplan, True)
         krcv.kr_profile_enable(False)
         del pplan
         sort_ms, build_ms, main_ms, red_ms = ([v[i] for v in st] for i in range(4))
         used = {1: "sweep", 2: "prefix", 3: "dense", 4: "hist"}.get(krcv.kr_last_algo(), "?")
-        main_total = sum(main_ms)
+        main_med = statistics.median(main_ms)  # dominant kernel, median over the profiled steps
         if world > 1:
-            t = torch.tensor([total_ms, main_total, prof_total_ms], dtype=torch.float64, device=dev)
+            t = torch.tensor([step_ms, main_med, prof_step_ms], dtype=torch.float64, device=dev)
             torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-            total_ms, main_total, prof_total_ms = float(t[0]), float(t[1]), float(t[2])
+            step_ms, main_med, prof_step_ms = float(t[0]), float(t[1]), float(t[2])
         res = plan.result()
-        main_s = (main_total / args.steps) * 1e-3
-        peak = SM_COUNT * FP64_LANES_PER_SM * 2 * SM_MAX_MHZ_NOMINAL * 1e6 / 1e12  # TFLOP/s
+        main_s = main_med * 1e-3
+        peak, peak_note = fp64_peak()  # TFLOP/s
         if used == "dense":
             kname = "gauss_kernel (a3+a4, tiled all-pairs, Gaussian)"
             flops = rows_mine * (n - 1) * m * FLOPS_PER_PAIR_BW_DENSE
@@ -374,19 +393,20 @@ def run_ours(args):
                      "row, LOO estimate, squared error (DESIGN.md §6.2); searches not counted")
         achieved = flops / main_s / 1e12
         return {
-            "algo": used, "value": units * args.steps / (total_ms * 1e-3), "ms_per_step": total_ms / args.steps,
-            "stage_ms": {"pack_sort_gather": sum(sort_ms) / args.steps, "prefix_build": sum(build_ms) / args.steps,
-                         "sweep": sum(main_ms) / args.steps, "reduce_finalize": sum(red_ms) / args.steps},
+            "algo": used, "value": units / (step_ms * 1e-3), "ms_per_step": step_ms,
+            "stage_ms": {"pack_sort_gather": statistics.median(sort_ms), "prefix_build": statistics.median(build_ms),
+                         "sweep": main_med, "reduce_finalize": statistics.median(red_ms)},
             "roofline": {"bound": "alu", "kernel": kname, "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
                          "frac": achieved / peak, "traffic": ncu_traffic(args.config, used),
                          "ncu": ncu_context(args.config, used),
                          "flops_per_launch": flops, "flops_basis": basis,
-                         "peak_note": "FP64: 148 SM x 64 FMA lanes x 2 flop x 1965 MHz (derived, DESIGN.md)",
-                         "kernel_ms": main_total / args.steps,
-                         "kernel_share_of_step": main_total / prof_total_ms,
+                         "peak_note": peak_note,
+                         "kernel_ms": main_med,
+                         "kernel_share_of_step": main_med / prof_step_ms,
                          "timing": "kernel_ms from stage CUDA events of a second, profiled run (events in its "
                                    "graph); value/ms_per_step from graph replays without stage events"},
-            "ms_per_step_profiled": prof_total_ms / args.steps,
+            "ms_per_step_profiled": prof_step_ms,
+            "timing_stat": "median over the K timed steps",
             "result": {"best": res.best, "h_best": float(h[res.best]), "cv_best": float(res.cv[res.best])},
             "clocks": clk.summary(), "gpu_launches": launches, "plan": plan,
         }
@@ -491,10 +511,10 @@ def e2e_measure(args, x, y, h, k, n, m, units, dev, rank, world, plan):
         times = [float(t[0]) / len(times)] * len(times)
         api = "GridSearch.run (row-sharded, NCCL all-reduce) with pinned H2D/D2H per step"
         d2h = 8 * m + 8
-    tot = sum(times)
-    return {"value": units * len(times) / tot, "unit": UNIT, "h2d_bytes_per_step": 16 * n + 8 * m,
-            "d2h_bytes_per_step": d2h, "ms_per_search": 1e3 * tot / len(times), "api": api,
-            "timing": "host wall clock around the synchronous call"}
+    med = statistics.median(times)
+    return {"value": units / med, "unit": UNIT, "h2d_bytes_per_step": 16 * n + 8 * m,
+            "d2h_bytes_per_step": d2h, "ms_per_search": 1e3 * med, "api": api,
+            "timing": "host wall clock around the synchronous call, median over the K steps"}
 
 
 def run_kde(args):
@@ -615,7 +635,7 @@ def run_ll(args):
     units = n * (n - 1) * m
     kms = stages[2] / args.steps
     flops = LL_FLOPS.get(k, 61) * n * m
-    peak = SM_COUNT * FP64_LANES_PER_SM * 2 * SM_MAX_MHZ_NOMINAL * 1e6 / 1e12  # TFLOP/s, as run_ours
+    peak, _ = fp64_peak()  # TFLOP/s, as run_ours
     ach = flops / (kms * 1e-3) / 1e12
     print(json.dumps({
         "metric": "local-linear LOO-CV pair-bandwidth evals/s (SURVEY 8(f) rank 4)",

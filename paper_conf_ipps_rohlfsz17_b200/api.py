@@ -215,7 +215,9 @@ class GridSearch:
         st = int(bs[1])
         if st != krcv.KR_OK:
             raise krcv.KrcvError(st, "device status")
-        return CVResult(cv=self.cv, neff=self.neff, best=int(bs[0]), h=self.h)
+        # copies: the plan's buffers are overwritten by the next run() (or
+        # graph replay), a result handed out must not change under the caller
+        return CVResult(cv=self.cv.clone(), neff=self.neff.clone(), best=int(bs[0]), h=self.h)
 
 
 def cv_grid(x, y, h=None, m: int | None = None, kernel="epanechnikov", device=None, distributed: bool = False,

@@ -85,6 +85,17 @@ static DevCtx *get_ctx(int dev)
         }                                                   \
     } while (0)
 
+// The captured host-path graph (DevCtx::gexec) has c->dx, c->dy, c->dh,
+// c->ws and the pinned staging c->pres baked into its nodes: any
+// reallocation of one of them must drop it, or a later replay with the same
+// caller pointers would copy into / launch on freed memory.
+static void drop_graph(DevCtx *c)
+{
+    if (c->gexec) cudaGraphExecDestroy(c->gexec);
+    c->gexec = nullptr;
+    c->gx = c->gy = c->gh = nullptr;
+}
+
 // [best, status] (8 B) | cv[m] | neff[m]
 static size_t res_bytes(int32_t m) { return 8 + (sizeof(double) + sizeof(int64_t)) * (size_t)m; }
 
@@ -99,6 +110,7 @@ static int ensure_capacity(DevCtx *c, int64_t n, int32_t m)
         KR_CUDA_TRY(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
     }
     if (n > c->cap_n) {
+        drop_graph(c);
         cudaFree(c->dx);
         cudaFree(c->dy);
         c->dx = c->dy = nullptr;
@@ -108,6 +120,7 @@ static int ensure_capacity(DevCtx *c, int64_t n, int32_t m)
         c->cap_n = n;
     }
     if (m > c->cap_m) {
+        drop_graph(c);
         cudaFree(c->dh);
         cudaFree(c->dpartial);
         cudaFree(c->dres);
@@ -127,6 +140,7 @@ static int ensure_capacity(DevCtx *c, int64_t n, int32_t m)
     size_t need = kr_workspace_bytes(n, m);
     if (need == 0) return KR_ECUDA;
     if (need > c->ws_bytes) {
+        drop_graph(c);
         cudaFree(c->ws);
         c->ws = nullptr;
         c->ws_bytes = 0;
@@ -176,6 +190,7 @@ static bool is_pinned(const void *p)
 static int ensure_staging(DevCtx *c, int32_t m)
 {
     if (m <= c->pcap_m) return KR_OK;
+    drop_graph(c);
     cudaFreeHost(c->pres);
     c->pres = nullptr;
     c->pcap_m = 0;

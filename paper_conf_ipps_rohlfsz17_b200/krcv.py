@@ -226,6 +226,31 @@ def kr_workspace_bytes(n: int, m: int) -> int:
 
 
 # ---------------------------------------------------------------- device API
+def _check_f64(name: str, t, numel=None) -> None:
+    """Contiguous float64 CUDA tensor (of ``numel`` elements when given)."""
+    import torch
+
+    if not (t.is_cuda and t.dtype == torch.float64 and t.is_contiguous()):
+        raise ValueError(f"{name} must be a contiguous float64 CUDA tensor")
+    if numel is not None and t.numel() != numel:
+        raise ValueError(f"{name} must have {numel} elements, got {t.numel()}")
+
+
+def _check_best_status(t) -> None:
+    """Exactly two contiguous int32 CUDA elements: (best, status)."""
+    import torch
+
+    if not (t.is_cuda and t.dtype == torch.int32 and t.is_contiguous() and t.numel() == 2):
+        raise ValueError("best_status must be a contiguous int32 CUDA tensor of 2 elements")
+
+
+def _check_neff(t, m: int) -> None:
+    import torch
+
+    if t is not None and not (t.is_cuda and t.dtype == torch.int64 and t.is_contiguous() and t.numel() == m):
+        raise ValueError("neff must be None or a contiguous int64 CUDA tensor of m elements")
+
+
 def kr_cv_rows_async(d_x, d_y, d_h, kernel, row_lo: int, row_hi: int, d_partial, d_ws, stream=None,
                      algo="auto") -> None:
     """Enqueue the device pipeline for rows [row_lo, row_hi) of the sorted
@@ -296,6 +321,10 @@ def kr_finalize_async(d_partial, n: int, m: int, d_cv, d_neff, d_best_status, st
     d_best_status int32[2] -> (best, status)."""
     import torch
 
+    _check_f64("partial", d_partial, partial_len(m))
+    _check_f64("cv", d_cv, m)
+    _check_neff(d_neff, m)
+    _check_best_status(d_best_status)
     s = torch.cuda.current_stream(d_partial.device) if stream is None else stream
     st = _lib().kr_finalize_async(d_partial.data_ptr(), int(n), int(m), d_cv.data_ptr(),
                                   None if d_neff is None else d_neff.data_ptr(),
@@ -365,6 +394,9 @@ def kr_kde_shard_async(d_x, d_h, kernel, shard: int, nshards: int, d_partial, d_
     """Enqueue one row shard of the KDE LSCV -> partial [sum A | sum B | status]."""
     import torch
 
+    _check_f64("x", d_x)
+    _check_f64("h", d_h)
+    _check_f64("partial", d_partial, partial_len(d_h.numel()))
     s = torch.cuda.current_stream(d_x.device) if stream is None else stream
     _check(_lib().kr_kde_shard_async(d_x.data_ptr(), d_x.numel(), d_h.data_ptr(), d_h.numel(), _kernel_id(kernel),
                                      int(shard), int(nshards), d_partial.data_ptr(), d_ws.data_ptr(),
@@ -374,6 +406,8 @@ def kr_kde_shard_async(d_x, d_h, kernel, shard: int, nshards: int, d_partial, d_
 
 def kr_kde_finalize(partial, n: int, h, kernel="epanechnikov"):
     p, h = _host(partial), _host(h)
+    if p.shape[0] != partial_len(h.shape[0]):
+        raise ValueError("partial must have length 2m+2")
     out = np.empty(h.shape[0], np.float64)
     best = ctypes.c_int32(-1)
     _check(_lib().kr_kde_finalize(p.ctypes.data, int(n), h.ctypes.data, h.shape[0], _kernel_id(kernel),
