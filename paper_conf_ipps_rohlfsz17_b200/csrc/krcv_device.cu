@@ -26,12 +26,15 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
+#include <vector>
 #include "krcv_internal.h"
 #include "krcv_pdl.cuh"
 #include "krcv_sweep.cuh"
 #include "krcv_sweep_gxg.cuh"
 #include "krcv_sort.cuh"
 #include "krcv_prefix.cuh"
+#include "krcv_window.cuh"
 #include "krcv_dense.cuh"
 #include "krcv_kde.cuh"
 #include "krcv_ll.cuh"
@@ -170,8 +173,9 @@ struct FinOut {
     unsigned *done;
 };
 
+template <typename CountT>  // uint8_t (one partial per 32-row tile) or uint32_t (win_kernel's row blocks)
 __global__ void __launch_bounds__(kReduceThreads)
-reduce_kernel(const double *__restrict__ tileS, const uint8_t *__restrict__ tileN, int ntiles, int m,
+reduce_kernel(const double *__restrict__ tileS, const CountT *__restrict__ tileN, int ntiles, int m,
               const unsigned *__restrict__ status, double *__restrict__ partial, FinOut fin)
 {
     pdl_wait();  // krcv_pdl.cuh
@@ -183,7 +187,7 @@ reduce_kernel(const double *__restrict__ tileS, const uint8_t *__restrict__ tile
         double a = 0.0;
         long long cnt = 0;
         const double *col = tileS + (size_t)b * ntiles;
-        const uint8_t *ncol = tileN + (size_t)b * ntiles;
+        const CountT *ncol = tileN + (size_t)b * ntiles;
         for (int t = threadIdx.x; t < ntiles; t += kReduceThreads) {
             a += col[t];
             cnt += ncol[t];
@@ -235,12 +239,11 @@ reduce_kernel(const double *__restrict__ tileS, const uint8_t *__restrict__ tile
 // ---------------------------------------------------------------------------
 static bool pdl_enabled()
 {
-    static int v = -1;
-    if (v < 0) {
+    static const bool v = [] {
         const char *e = getenv("KRCV_PDL");
-        v = (e && e[0] == '0') ? 0 : 1;
-    }
-    return v == 1;
+        return !(e && e[0] == '0');
+    }();
+    return v;
 }
 
 template <typename... KArgs, typename... Args>
@@ -258,6 +261,70 @@ static void launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t sme
     cfg.attrs = at;
     cfg.numAttrs = 1;
     cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);  // errors surface via cudaGetLastError
+}
+
+// ---------------------------------------------------------------------------
+// Per-device launch facts, safe under concurrent first calls (include/krcv.h
+// promises re-entrant entry points): the SM count of each device, and the
+// resident CTAs per SM of each (kernel, block size, smem) on each device,
+// computed once under a mutex and cached.  Environment overrides are read
+// into function-local statics with thread-safe (C++11 "magic static")
+// initialisation.
+// ---------------------------------------------------------------------------
+struct DevInfo {
+    int sms = 148;
+};
+
+static int current_device()
+{
+    int dev = 0;
+    cudaGetDevice(&dev);
+    return dev;
+}
+
+static const DevInfo &dev_info()
+{
+    constexpr int kMaxDev = 64;
+    static std::mutex mu;
+    static DevInfo info[kMaxDev];
+    static bool have[kMaxDev] = {};
+    const int dev = current_device();
+    const int d = dev >= 0 && dev < kMaxDev ? dev : 0;
+    std::lock_guard<std::mutex> g(mu);
+    if (!have[d]) {
+        int sms = 0;
+        if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && sms > 0)
+            info[d].sms = sms;
+        else
+            cudaGetLastError();
+        have[d] = true;
+    }
+    return info[d];
+}
+
+static int occupancy(const void *func, int threads, size_t smem = 0)
+{
+    struct Key {
+        int dev;
+        const void *f;
+        int threads;
+        size_t smem;
+        int value;
+    };
+    static std::mutex mu;
+    static std::vector<Key> cache;
+    const int dev = current_device();
+    std::lock_guard<std::mutex> g(mu);
+    for (const Key &k : cache)
+        if (k.dev == dev && k.f == func && k.threads == threads && k.smem == smem) return k.value;
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, func, threads, smem) != cudaSuccess) {
+        cudaGetLastError();
+        b = 1;
+    }
+    if (b < 1) b = 1;
+    cache.push_back(Key{dev, func, threads, smem, b});
+    return b;
 }
 
 // ---------------------------------------------------------------------------
@@ -317,8 +384,15 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     // m-dependent buffers last: everything above has the same offset for any
     // m, so a refinement level with another grid size can reuse the sorted
     // arrays and prefix moments in place (kr_cv_refine)
+    // bucket table of win_kernel (krcv_window.cuh): int32 [Qmax + 1], Qmax = min(kBktFmax n, kBktQmax)
+    const int64_t qmax = (int64_t)kBktFmax * n < kBktQmax ? (int64_t)kBktFmax * n : kBktQmax;
+    L->bt = off;       off = align256(off + sizeof(int) * (size_t)(qmax + 1));
     L->tileS = off;    off = align256(off + sizeof(double) * (size_t)ntiles * (size_t)m);
-    L->tileN = off;    off = align256(off + sizeof(uint8_t) * (size_t)ntiles * (size_t)m);
+    // counts: uint8 per 32-row tile (sweep, r01 window, LL, hist, dense) or
+    // uint32 per row block of win_kernel (at most one block per 32 rows)
+    const size_t n32 = (size_t)((n + 31) / 32);
+    const size_t nbytes = (size_t)ntiles > 4 * n32 ? (size_t)ntiles : 4 * n32;
+    L->tileN = off;    off = align256(off + nbytes * (size_t)m);
     L->tileB = off;    off = align256(off + sizeof(double) * (size_t)((n + 31) / 32) * (size_t)m);  // KDE sum B
     L->partial = off;  off = align256(off + sizeof(double) * (size_t)KR_PARTIAL_LEN(m));
     L->cub_bytes = cub_bytes;
@@ -333,12 +407,11 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
 // combine overhead).  KRCV_SWEEP_G overrides (1, 2, 4; 8 for split).
 int sweep_G(int64_t /*rows*/)
 {
-    static int forced = -1;
-    if (forced < 0) {
+    static const int forced = [] {
         const char *e = getenv("KRCV_SWEEP_G");
-        int g = e ? atoi(e) : 0;
-        forced = (g == 1 || g == 2 || g == 4 || g == 8) ? g : 0;
-    }
+        const int g = e ? atoi(e) : 0;
+        return (g == 1 || g == 2 || g == 4 || g == 8) ? g : 0;
+    }();
     return forced ? forced : 4;
 }
 
@@ -369,11 +442,10 @@ static int grid_for(int64_t work, int threads)
 // (DESIGN.md §6).  KRCV_SWEEP=split|gxg overrides.
 int sweep_variant(int64_t rows)
 {
-    static int v = -1;
-    if (v < 0) {
+    static const int v = [] {
         const char *e = getenv("KRCV_SWEEP");
-        v = !e ? 2 : (e[0] == 's' ? 0 : (e[0] == 'g' ? 1 : 2));
-    }
+        return !e ? 2 : (e[0] == 's' ? 0 : (e[0] == 'g' ? 1 : 2));
+    }();
     if (v != 2) return v;
     return rows >= kGxgRows ? 1 : 0;
 }
@@ -382,22 +454,10 @@ template <int KERN, int G, bool GXG>
 static void launch_sweep_g(const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
                            double *tileS, uint8_t *tileN, int *counter, cudaStream_t st)
 {
-    static int resident = 0;  // CTAs per SM at full occupancy (persistent grid)
-    if (!resident) {
-        int b = 0;
-        if (GXG)
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sweep_gxg_kernel<KERN, G>, kSweepThreads, 0);
-        else
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sweep_kernel<KERN, G>, kSweepThreads, 0);
-        resident = b > 0 ? b : 1;
-    }
-    static int sms = 0;
-    if (!sms) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (sms <= 0) sms = 148;
-    }
+    // CTAs per SM at full occupancy (persistent grid)
+    const int resident = occupancy(GXG ? (const void *)sweep_gxg_kernel<KERN, G> : (const void *)sweep_kernel<KERN, G>,
+                                   kSweepThreads);
+    const int sms = dev_info().sms;
     int blocks = (ntiles + kSweepWarps - 1) / kSweepWarps;
     if (blocks > sms * resident) blocks = sms * resident;
     if (GXG)
@@ -470,11 +530,10 @@ static int64_t cub_sort_launches(int64_t n) { return n <= kCubSingleTile ? 1 : 2
 // n.  KRCV_CHUNK=0..4 overrides.
 int chunk_config(int64_t n)
 {
-    static int forced = -1;
-    if (forced < 0) {
+    static const int forced = [] {
         const char *e = getenv("KRCV_CHUNK");
-        forced = (e && e[0] >= '0' && e[0] <= '4') ? e[0] - '0' : 5;
-    }
+        return (e && e[0] >= '0' && e[0] <= '4') ? e[0] - '0' : 5;
+    }();
     if (forced != 5) return forced;
     return n <= 40000 ? 3 : 0;
 }
@@ -492,11 +551,10 @@ static void launch_rank_sort(const double *d_x, const double *d_y, int n, const 
 // KRCV_ALGO=sweep|prefix overrides (benchmarks, A/B tests).
 int auto_algo(int64_t /*n*/, int64_t /*rows*/, int32_t /*m*/, int32_t /*kernel*/)
 {
-    static int forced = -1;
-    if (forced < 0) {
+    static const int forced = [] {
         const char *e = getenv("KRCV_ALGO");
-        forced = !e ? 0 : (e[0] == 's' ? KR_ALGO_SWEEP : (e[0] == 'p' ? KR_ALGO_PREFIX : (e[0] == 'h' ? KR_ALGO_HIST : 0)));
-    }
+        return !e ? 0 : (e[0] == 's' ? KR_ALGO_SWEEP : (e[0] == 'p' ? KR_ALGO_PREFIX : (e[0] == 'h' ? KR_ALGO_HIST : 0)));
+    }();
     return forced ? forced : KR_ALGO_PREFIX;
 }
 
@@ -510,12 +568,11 @@ constexpr int kPfxOneCtaMax = 1024;  // measured: C1 (n = 1,000) 10.2 -> 8.2 us,
 
 static int pfx_items(int n)
 {
-    static int forced = -1;
-    if (forced < 0) {
+    static const int forced = [] {
         const char *e = getenv("KRCV_PFX_ITEMS");
-        forced = e ? atoi(e) : -2;
-        if (forced != 0 && forced != 1 && forced != 4) forced = -2;
-    }
+        const int v = e ? atoi(e) : -2;
+        return (v == 0 || v == 1 || v == 4) ? v : -2;
+    }();
     if (forced != -2) return forced;
     return n <= kPfxOneCtaMax ? 0 : (n <= (1 << 18) ? 1 : kPfxItemsMax);
 }
@@ -527,141 +584,73 @@ static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, cha
     double *P = reinterpret_cast<double *>(ws + L.pfx);
     double2 *tot = reinterpret_cast<double2 *>(ws + L.ptot);
     unsigned long long *ymax = reinterpret_cast<unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
+    unsigned long long *gap = reinterpret_cast<unsigned long long *>(ws + L.status + 6 * sizeof(unsigned));
     const int items = pfx_items(n);
     if (items == 0) {
-        pfx_one_cta_kernel<KERN><<<1, kPfx1Threads, 0, st>>>(xy, n, P, (int)L.pstride, xs, ymax);
+        pfx_one_cta_kernel<KERN><<<1, kPfx1Threads, 0, st>>>(xy, n, P, (int)L.pstride, xs, ymax, gap);
     } else if (items == 1) {
         const int ntiles = (n + kPfxThreads) / kPfxThreads;  // tiles covering P[0..n]
         launch_pdl(pfx_tile_reduce_kernel<KERN, 1>, dim3(ntiles), dim3(kPfxThreads), 0, st, xy, n, tot, ntiles, ymax);
         launch_pdl(pfx_tile_scan_kernel<KERN, 1>, dim3(ntiles), dim3(kPfxThreads), 0, st, xy, n,
-                   (const double2 *)tot, ntiles, P, (int)L.pstride, xs);
+                   (const double2 *)tot, ntiles, P, (int)L.pstride, xs, gap);
     } else {
         const int ntiles = (n + kPfxThreads * kPfxItemsMax) / (kPfxThreads * kPfxItemsMax);
         launch_pdl(pfx_tile_reduce_kernel<KERN, kPfxItemsMax>, dim3(ntiles), dim3(kPfxThreads), 0, st, xy, n, tot,
                    ntiles, ymax);
         launch_pdl(pfx_tile_scan_kernel<KERN, kPfxItemsMax>, dim3(ntiles), dim3(kPfxThreads), 0, st, xy, n,
-                   (const double2 *)tot, ntiles, P, (int)L.pstride, xs);
+                   (const double2 *)tot, ntiles, P, (int)L.pstride, xs, gap);
     }
 }
 
-// Rows per lane of the window kernel (K consecutive rows; rows 2..K advance
-// from their predecessor's boundaries).  KRCV_WIN_K overrides (1, 2, 4).
+// Window kernel of r01 (window_kernel<K> / window_kernel_b2), kept for A/B
+// runs: K consecutive rows per lane (K = 1, 2) or one row per lane with two
+// bandwidths per step (3).  KRCV_WIN_K overrides.
 int win_rows_per_lane(int64_t rows)
 {
-    static int forced = -1;
-    if (forced < 0) {
+    static const int forced = [] {
         const char *e = getenv("KRCV_WIN_K");
         const int k = e ? atoi(e) : 0;
-        forced = (k >= 1 && k <= 10) ? k : 0;  // 3: window_kernel_b2, 5: window_kernel_coop,
-                                               // 6/7/8: window_kernel_seg with 2/4/1 rows per lane,
-                                               // 9/10: window_kernel_blk with 2/4 blocks of 32 rows
-    }
+        return (k >= 1 && k <= 3) ? k : 0;
+    }();
     if (forced) return forced;
     // measured (profiles/r01t_*, r01u_*, r01af_*): two consecutive rows per
-    // lane up to 5e4 rows (C2: K = 1, 2, b2 within 1 %); above, one row per
-    // lane with two bandwidths per step (window_kernel_b2: C3 1.73 -> 1.65 ms,
-    // C4 22.9 -> 20.9 ms, C5 2.57 -> 2.43 ms)
+    // lane up to 5e4 rows, above one row per lane with two bandwidths per step
     return rows <= 50000 ? 2 : 3;
 }
 
-// Rows per lane of window-kernel variant K (KRCV_WIN_K numbering).
-static int win_lane_rows(int K)
-{
-    switch (K) {
-    case 3: case 5: case 8: return 1;
-    case 6: case 9: return 2;
-    case 7: case 10: return 4;
-    default: return K;
-    }
-}
-
-// Task assignment of the window kernels: 1 = SM-local regions
-// (take_task_local, krcv_prefix.cuh), 0 = one global counter (default).  KRCV_WIN_SCHED
-// overrides.
-static int win_sched()
-{
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("KRCV_WIN_SCHED");
-        v = e ? (atoi(e) ? 1 : 0) : 0;  // measured: no gain
-    }
-    return v;
-}
+static int win_lane_rows(int K) { return K == 3 ? 1 : K; }
 
 template <int KERN, int K>
 static void launch_window_k(const double2 *xy, int n, const double *h, int m, int lo, int hi, int ntiles,
                             const WsLayout &L, char *ws, double *tileS, uint8_t *tileN, int *counter,
                             cudaStream_t st)
 {
-    const int sched = win_sched();
-    static int resident = 0;
-    if (!resident) {
-        int b = 0;
-        if (K == 3)
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, sched ? window_kernel_b2<KERN, 1> : window_kernel_b2<KERN, 0>,
-                                                          kWinThreads, 0);
-        else if (K == 5)
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_coop<KERN>, kCoopRows, 0);
-        else if (K >= 9)
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_blk<KERN, K == 9 ? 2 : 4>, kWinThreads, 0);
-        else if (K >= 6)
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, window_kernel_seg<KERN, K == 6 ? 2 : (K == 7 ? 4 : 1)>,
-                                                          kWinThreads, 0);
-        else
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-                &b, sched ? window_kernel<KERN, (K == 3 || K >= 5) ? 1 : K, 1> : window_kernel<KERN, (K == 3 || K >= 5) ? 1 : K, 0>,
-                kWinThreads, 0);
-        resident = b > 0 ? b : 1;
-    }
-    static int sms = 0;
-    if (!sms) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (sms <= 0) sms = 148;
-    }
+    const DevInfo &di = dev_info();
+    const int resident = occupancy(K == 3 ? (const void *)window_kernel_b2<KERN> : (const void *)window_kernel<KERN, K == 3 ? 1 : K>,
+                                   kWinThreads);
     // Split the bandwidth loop into nbc chunks until there are enough warp
     // tasks to fill every SM (~kWinTasksPerSM resident warps each), keeping
     // >= kWinMinBper bandwidths per chunk to amortise the cold searches.
-    const int64_t want = (int64_t)sms * kWinTasksPerSM;
+    const int64_t want = (int64_t)di.sms * kWinTasksPerSM;
     int nbc = (int)((want + ntiles - 1) / ntiles);
     nbc = nbc < 1 ? 1 : nbc;
     const int max_nbc = (m + kWinMinBper - 1) / kWinMinBper;
     if (nbc > max_nbc) nbc = max_nbc;
     if (nbc < 1) nbc = 1;
-    const char *fe = getenv("KRCV_WIN_NBC");
-    if (fe && atoi(fe) > 0) nbc = atoi(fe) < m ? atoi(fe) : m;
     const int64_t tasks = (int64_t)ntiles * nbc;
-    int blocks = (int)((tasks + kWinWarps - 1) / kWinWarps);  // kWinWarps == kCoopRows / 32
-    if (blocks > sms * resident) blocks = sms * resident;
+    int blocks = (int)((tasks + kWinWarps - 1) / kWinWarps);
+    if (blocks > di.sms * resident) blocks = di.sms * resident;
     const double *xs = reinterpret_cast<const double *>(ws + L.xs) + kPad;
     const double *P = reinterpret_cast<const double *>(ws + L.pfx);
     const unsigned long long *ymax =
         reinterpret_cast<const unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
-    const bool local = sched && (K <= 4) && sms <= kSmCounters;
-    if (local) cudaMemsetAsync(counter + 1, 0, sizeof(int) * sms, st);  // the SM-local region counters
-    if (K == 3 && local)
-        window_kernel_b2<KERN, 1><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
-                                                                  nbc, ymax, tileS, tileN, counter, sms);
-    else if (K == 3)
-        launch_pdl(window_kernel_b2<KERN, 0>, dim3(blocks), dim3(kWinThreads), 0, st, xs, (const double2 *)xy, P,
-                   (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter, sms);
-    else if (K == 5)
-        window_kernel_coop<KERN><<<blocks, kCoopRows, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles,
-                                                               nbc, ymax, tileS, tileN, counter);
-    else if (K >= 9)
-        window_kernel_blk<KERN, K == 9 ? 2 : 4><<<blocks, kWinThreads, 0, st>>>(
-            xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter);
-    else if (K >= 6)
-        window_kernel_seg<KERN, K == 6 ? 2 : (K == 7 ? 4 : 1)><<<blocks, kWinThreads, 0, st>>>(
-            xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter);
-    else if (local)
-        window_kernel<KERN, (K == 3 || K >= 5) ? 1 : K, 1><<<blocks, kWinThreads, 0, st>>>(
-            xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter, sms);
+    if (K == 3)
+        launch_pdl(window_kernel_b2<KERN>, dim3(blocks), dim3(kWinThreads), 0, st, xs, (const double2 *)xy, P,
+                   (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN, counter);
     else
-        launch_pdl(window_kernel<KERN, (K == 3 || K >= 5) ? 1 : K, 0>, dim3(blocks), dim3(kWinThreads), 0, st, xs,
+        launch_pdl(window_kernel<KERN, K == 3 ? 1 : K>, dim3(blocks), dim3(kWinThreads), 0, st, xs,
                    (const double2 *)xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc, ymax, tileS, tileN,
-                   counter, sms);
+                   counter);
 }
 
 template <int KERN>
@@ -671,16 +660,79 @@ static void launch_window(int K, const double2 *xy, int n, const double *h, int 
 {
     switch (K) {
     case 1: launch_window_k<KERN, 1>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
-    case 2: launch_window_k<KERN, 2>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     case 3: launch_window_k<KERN, 3>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
-    case 5: launch_window_k<KERN, 5>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
-    case 6: launch_window_k<KERN, 6>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
-    case 7: launch_window_k<KERN, 7>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
-    case 8: launch_window_k<KERN, 8>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
-    case 9: launch_window_k<KERN, 9>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
-    case 10: launch_window_k<KERN, 10>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
-    default: launch_window_k<KERN, 4>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
+    default: launch_window_k<KERN, 2>(xy, n, h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st); break;
     }
+}
+
+// Window kernel selection: 1 = win_kernel (bucket-table lookups,
+// krcv_window.cuh; default), 0 = r01's window_kernel / window_kernel_b2
+// (KRCV_WIN=r01, A/B runs).
+static bool use_win2()
+{
+    static const bool v = [] {
+        const char *e = getenv("KRCV_WIN");
+        return !(e && strcmp(e, "r01") == 0);
+    }();
+    return v;
+}
+
+// Task shape of win_kernel for a shard of `rows` rows: BC bandwidths per
+// chunk (<= kWin2Chunk) and TB tiles of 32 rows per block, chosen so that
+// there are about kWin2TasksPerWarp tasks per resident warp (load balance)
+// with as few partials as that allows.
+struct Win2Shape {
+    int BC, nbc, TB, nblk;
+};
+constexpr int kWin2TasksPerWarp = 4;
+
+template <int KERN>
+static Win2Shape win2_shape(int64_t rows, int m)
+{
+    Win2Shape w;
+    const int64_t n32 = (rows + 31) / 32;
+    const int64_t warps = (int64_t)dev_info().sms * occupancy((const void *)win_kernel<KERN>, kWin2Threads) * kWin2Warps;
+    const int64_t target = kWin2TasksPerWarp * warps;
+    int64_t bc = (int64_t)m * n32 / (target > 0 ? target : 1);
+    bc = bc < 8 ? 8 : (bc > kWin2Chunk ? kWin2Chunk : bc);
+    if (bc > m) bc = m;
+    w.BC = (int)bc;
+    w.nbc = (int)((m + bc - 1) / bc);
+    int64_t tb = n32 * w.nbc / (target > 0 ? target : 1);
+    tb = tb < 1 ? 1 : (tb > 16 ? 16 : tb);
+    w.TB = (int)tb;
+    w.nblk = (int)((n32 + tb - 1) / tb);
+    return w;
+}
+
+template <int KERN>
+static void launch_win2(const double2 *xy, int n, const double *h, int m, int lo, int hi, const Win2Shape &w,
+                        bool build_table, const WsLayout &L, char *ws, double *tileS, uint32_t *tileN, int *counter,
+                        cudaStream_t st)
+{
+    const double *xs = reinterpret_cast<const double *>(ws + L.xs) + kPad;
+    const double *P = reinterpret_cast<const double *>(ws + L.pfx);
+    int *BT = reinterpret_cast<int *>(ws + L.bt);
+    const unsigned long long *ymax =
+        reinterpret_cast<const unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
+    const unsigned long long *gap =
+        reinterpret_cast<const unsigned long long *>(ws + L.status + 6 * sizeof(unsigned));
+    BktParams *prm = reinterpret_cast<BktParams *>(ws + L.status + 32);
+    const int sms = dev_info().sms;
+    if (build_table) {
+        const int64_t qmax = (int64_t)kBktFmax * n < kBktQmax ? (int64_t)kBktFmax * n : kBktQmax;
+        const int64_t nseg = (n + qmax + 1 + kBktSeg - 1) / kBktSeg;
+        int64_t blocks = (nseg + kBktFillThreads - 1) / kBktFillThreads;
+        if (blocks > (int64_t)sms * 8) blocks = (int64_t)sms * 8;
+        launch_pdl(bkt_fill_kernel, dim3((int)blocks), dim3(kBktFillThreads), 0, st, xs, n, gap, BT, prm);
+    }
+    const int resident = occupancy((const void *)win_kernel<KERN>, kWin2Threads);
+    const int64_t tasks = (int64_t)w.nblk * w.nbc;
+    int blocks = (int)((tasks + kWin2Warps - 1) / kWin2Warps);
+    if (blocks > sms * resident) blocks = sms * resident;
+    launch_pdl(win_kernel<KERN>, dim3(blocks), dim3(kWin2Threads), 0, st, xs, xy, P, (int)L.pstride,
+               (const int *)BT, (const BktParams *)prm, h, m, n, lo, hi, w.TB, w.nblk, w.BC, w.nbc, ymax, tileS,
+               tileN, counter);
 }
 
 // Histogram ordering (krcv_hist.cuh): `warps` warps per CTA (as many as the
@@ -692,12 +744,8 @@ static void launch_hist(int warps, const double *d_x, const double *d_y, const u
 {
     const size_t smem = hist_smem_bytes(m, warps);
     cudaFuncSetAttribute(hist_kernel<KERN>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    int resident = 0, dev = 0, sms = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&resident, hist_kernel<KERN>, warps * 32, smem);
-    if (resident < 1) resident = 1;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (sms <= 0) sms = 148;
+    const int resident = occupancy((const void *)hist_kernel<KERN>, warps * 32, smem);
+    const int sms = dev_info().sms;
     int blocks = ntiles;  // one 32-row tile per CTA iteration
     if (blocks > sms * resident) blocks = sms * resident;
     hist_kernel<KERN><<<blocks, warps * 32, smem, st>>>(d_x, d_y, perm, xy, h, m, n, lo, hi, ntiles, tileS, tileN,
@@ -711,16 +759,8 @@ static void launch_ll_window(const double2 *xy, int n, const double *h, int m, i
                              const WsLayout &L, char *ws, double *tileS, uint8_t *tileN, int *counter,
                              cudaStream_t st)
 {
-    static int resident = 0, sms = 0;
-    if (!resident) {
-        int b = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, ll_window_kernel<KERN>, kWinThreads, 0);
-        resident = b > 0 ? b : 1;
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (sms <= 0) sms = 148;
-    }
+    const int resident = occupancy((const void *)ll_window_kernel<KERN>, kWinThreads);
+    const int sms = dev_info().sms;
     const int64_t want = (int64_t)sms * kWinTasksPerSM;
     int nbc = (int)((want + ntiles - 1) / ntiles);
     const int max_nbc = (m + kWinMinBper - 1) / kWinMinBper;
@@ -734,16 +774,17 @@ static void launch_ll_window(const double2 *xy, int n, const double *h, int m, i
     const unsigned long long *ymax =
         reinterpret_cast<const unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
     // KRCV_LL_STATS=1 (debug): count the branches taken, print to stderr
-    static unsigned long long *stats = nullptr;
+    unsigned long long *stats = nullptr;
     const bool want_stats = getenv_flag("KRCV_LL_STATS");
-    if (want_stats && !stats) cudaMalloc(&stats, 4 * sizeof(unsigned long long));
-    if (want_stats) cudaMemsetAsync(stats, 0, 4 * sizeof(unsigned long long), st);
+    if (want_stats && cudaMalloc(&stats, 4 * sizeof(unsigned long long)) != cudaSuccess) stats = nullptr;
+    if (stats) cudaMemsetAsync(stats, 0, 4 * sizeof(unsigned long long), st);
     ll_window_kernel<KERN><<<blocks, kWinThreads, 0, st>>>(xs, xy, P, (int)L.pstride, h, m, n, lo, hi, ntiles, nbc,
-                                                           ymax, tileS, tileN, counter, want_stats ? stats : nullptr);
-    if (want_stats) {
+                                                           ymax, tileS, tileN, counter, stats);
+    if (stats) {
         unsigned long long v[4] = {0, 0, 0, 0};
         cudaMemcpyAsync(v, stats, sizeof v, cudaMemcpyDeviceToHost, st);
         cudaStreamSynchronize(st);
+        cudaFree(stats);
         fprintf(stderr, "ll stats: direct %llu prefix_ok %llu prefix_rejected %llu rejected_window_points %llu\n",
                 v[0], v[1], v[2], v[3]);
     }
@@ -895,9 +936,19 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     const int variant = sweep_variant(hi - lo);
     int G = sweep_G(hi - lo);
     if (variant == 1 && G > 4) G = 4;
+    const bool win2 = prefix && !ll && use_win2();  // win_kernel (krcv_window.cuh)
+    Win2Shape w2{};
+    if (win2) {
+        switch (kernel) {
+        case KR_UNIFORM: w2 = win2_shape<KR_UNIFORM>(hi - lo, m); break;
+        case KR_EPANECHNIKOV: w2 = win2_shape<KR_EPANECHNIKOV>(hi - lo, m); break;
+        default: w2 = win2_shape<KR_TRIANGULAR>(hi - lo, m); break;
+        }
+    }
     const int winK = ll ? 1 : win_rows_per_lane(hi - lo);
     const int rows_per_tile = 32 * win_lane_rows(winK);
     const int ntiles = hist ? (int)((hi - lo + 31) / 32)
+                     : win2 ? w2.nblk
                      : prefix ? (int)((hi - lo + rows_per_tile - 1) / rows_per_tile)
                               : dense ? (int)tiles_for(hi - lo, 1)
                                       : (variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G));
@@ -967,6 +1018,21 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
                 launch_ll_window<KR_TRIANGULAR>(xy, nn, d_h, m, lo, hi, ntiles, L, ws, tileS, tileN, counter, st);
                 break;
             }
+        } else if (win2) {
+            uint32_t *tileN32 = reinterpret_cast<uint32_t *>(ws + L.tileN);
+            const bool table = !reuse_sorted;  // the table depends on xs only
+            switch (kernel) {
+            case KR_UNIFORM:
+                launch_win2<KR_UNIFORM>(xy, nn, d_h, m, lo, hi, w2, table, L, ws, tileS, tileN32, counter, st);
+                break;
+            case KR_EPANECHNIKOV:
+                launch_win2<KR_EPANECHNIKOV>(xy, nn, d_h, m, lo, hi, w2, table, L, ws, tileS, tileN32, counter, st);
+                break;
+            default:
+                launch_win2<KR_TRIANGULAR>(xy, nn, d_h, m, lo, hi, w2, table, L, ws, tileS, tileN32, counter, st);
+                break;
+            }
+            launches += table ? 1 : 0;
         } else if (prefix) {
             switch (kernel) {
             case KR_UNIFORM:
@@ -996,8 +1062,14 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     prof_mark(3, st);
     if (injected_failure("reduce")) return KR_ECUDA;
     NvtxScope nv_red("krcv: a5 reduction (+ finalize)");
-    launch_pdl(reduce_kernel, dim3(m < 148 * 8 ? m : 148 * 8), dim3(kReduceThreads), 0, st, (const double *)tileS,
-               (const uint8_t *)tileN, ntiles, m, (const unsigned *)status, d_partial, fin);
+    if (win2)
+        launch_pdl(reduce_kernel<uint32_t>, dim3(m < 148 * 8 ? m : 148 * 8), dim3(kReduceThreads), 0, st,
+                   (const double *)tileS, (const uint32_t *)(ws + L.tileN), ntiles, m, (const unsigned *)status,
+                   d_partial, fin);
+    else
+        launch_pdl(reduce_kernel<uint8_t>, dim3(m < 148 * 8 ? m : 148 * 8), dim3(kReduceThreads), 0, st,
+                   (const double *)tileS, (const uint8_t *)tileN, ntiles, m, (const unsigned *)status, d_partial,
+                   fin);
     launches += 1;
     prof_mark(4, st);
     g_prof.recorded = g_prof.on;
@@ -1144,16 +1216,8 @@ static int enqueue_kde(const double *d_x, int64_t n, const double *d_h, int32_t 
     launches += 2;
     prof_mark(2, st);
     if (ntiles > 0) {
-        static int resident = 0, sms = 0;
-        if (!resident) {
-            int b = 0;
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kde_window_kernel<KR_EPANECHNIKOV>, kWinThreads, 0);
-            resident = b > 0 ? b : 1;
-            int dev = 0;
-            cudaGetDevice(&dev);
-            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-            if (sms <= 0) sms = 148;
-        }
+        const int resident = occupancy((const void *)kde_window_kernel<KR_EPANECHNIKOV>, kWinThreads);
+        const int sms = dev_info().sms;
         int nbc = (int)(((int64_t)sms * kWinTasksPerSM + ntiles - 1) / ntiles);
         const int max_nbc = (m + kWinMinBper - 1) / kWinMinBper;
         nbc = nbc > max_nbc ? max_nbc : nbc;

@@ -26,11 +26,14 @@ struct WsLayout {
     size_t xy;                  // double2 [n + 2 kPad] (x, y) in sorted order, +-inf sentinels
     size_t counter;             // int: sweep tile counter
     size_t perm;                // uint32 [n]  original index of each sorted record (histogram path)
+    size_t bt;                  // int32   [Qmax + 1] bucket table of win_kernel (krcv_window.cuh)
     size_t tileS;               // double  [m][ntiles]  per-tile sum of M e^2
     size_t tileN;               // uint8   [m][ntiles]  per-tile sum of M
     size_t tileB;               // double  [m][ceil(n/32)] per-tile KDE sum B (tileS holds A)
     size_t status;              // uint32  [8]  n_bad_grid, n_nonfinite, reduce completion counter, pad,
-                                //              u64 bits of max |y| (window-prefix fast-path bound)
+                                //              u64 bits of max |y| (window-prefix fast-path bound),
+                                //              u64 complement bits of the min x-span of kGapSpan+1 records;
+                                //              then (byte 32) the BktParams of the call (256 B region)
     size_t partial;             // double  [2m+2] partial vector of kr_cv_grid_async
     size_t xs;                  // double  [n + 2 kPad] sorted x, +-inf sentinels (prefix path)
     size_t pfx;                 // double [8][2][pstride] dd prefix moments P[k][0..n], hi / lo planes

@@ -59,6 +59,25 @@ constexpr int kWinWarps = 4;
 constexpr int kWinThreads = kWinWarps * 32;
 constexpr int kWinTasksPerSM = 256;   // warp tasks per SM the b-split aims for (measured: C3 nbc 7 -> 28, -9 %)
 constexpr int kWinMinBper = 8;        // >= this many bandwidths per task
+// Density statistic for the bucket table (krcv_window.cuh): the smallest
+// x-distance spanned by kGapSpan + 1 consecutive sorted records, stored as
+// the complement of its bit pattern (non-negative doubles order like their
+// bits, so the complement orders inversely and atomicMax keeps the minimum;
+// the status memset's 0 is below every stored value).
+constexpr int kGapSpan = 64;
+
+__device__ __forceinline__ void gap_stat(const double2 *__restrict__ xy, int n, int j, double &gmin)
+{
+    if (j + kGapSpan < n) gmin = fmin(gmin, xy[j + kGapSpan].x - xy[j].x);
+}
+
+__device__ __forceinline__ void gap_publish(double gmin, unsigned long long *__restrict__ gap_bits)
+{
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) gmin = fmin(gmin, __shfl_xor_sync(0xffffffffu, gmin, d));
+    if ((threadIdx.x & 31) == 0 && gmin < INFINITY)
+        atomicMax(gap_bits, ~(unsigned long long)__double_as_longlong(fmax(gmin, 0.0)));
+}
 
 // Moments per kernel (slot order).  Epanechnikov: y, u, u^2, y u, y u^2.
 // Triangular: y, u, y u.  Uniform: y.
@@ -115,6 +134,65 @@ __device__ __forceinline__ void moment_terms(double x, double y, double o, dd (&
     }
 }
 
+// Prefix storage.  Nadaraya-Watson moment sets (uniform / Epanechnikov /
+// triangular) are stored as records, array of structures: the hi words of
+// index j at P[j S .. j S + S), the lo words at P[ps S + j S ..], S doubles
+// per record (Epanechnikov 6: y, u, u^2, y u, y u^2, j; triangular 4: y, u,
+// y u, j; uniform 2: y, j -- the last slot is the index j itself as a double,
+// so a window count is a difference of two loaded slots).  One record is one
+// or three 16-byte loads.  The KDE and local-linear sets keep the
+// structure-of-arrays planes (hi of moment k at P + 2k ps, lo at
+// P + (2k+1) ps).
+template <int KERN>
+struct PfxRec {
+    static constexpr int S = KERN == KR_EPANECHNIKOV ? 6 : (KERN == KR_TRIANGULAR ? 4 : (KERN == KR_UNIFORM ? 2 : 0));
+};
+
+template <int KERN>
+__device__ __forceinline__ void pk_store(double *__restrict__ P, int ps, int k, int j, dd v)
+{
+    constexpr int S = PfxRec<KERN>::S;
+    if (S) {
+        P[(size_t)j * S + k] = v.hi;
+        P[(size_t)ps * S + (size_t)j * S + k] = v.lo;
+    } else {
+        P[(size_t)(2 * k) * ps + j] = v.hi;
+        P[(size_t)(2 * k + 1) * ps + j] = v.lo;
+    }
+}
+
+// the record's index slot (AoS layouts only)
+template <int KERN>
+__device__ __forceinline__ void pk_store_index(double *__restrict__ P, int ps, int j)
+{
+    constexpr int S = PfxRec<KERN>::S;
+    if (S) {
+        P[(size_t)j * S + S - 1] = (double)j;
+        P[(size_t)ps * S + (size_t)j * S + S - 1] = 0.0;
+    }
+}
+
+template <int KERN>
+__device__ __forceinline__ double pk_hi(const double *__restrict__ P, int ps, int k, int j)
+{
+    constexpr int S = PfxRec<KERN>::S;
+    return S ? P[(size_t)j * S + k] : P[(size_t)(2 * k) * ps + j];
+}
+
+template <int KERN>
+__device__ __forceinline__ dd pk_dd(const double *__restrict__ P, int ps, int k, int j)
+{
+    constexpr int S = PfxRec<KERN>::S;
+    return S ? dd{P[(size_t)j * S + k], P[(size_t)ps * S + (size_t)j * S + k]}
+             : dd{P[(size_t)(2 * k) * ps + j], P[(size_t)(2 * k + 1) * ps + j]};
+}
+
+template <int KERN>
+__device__ __forceinline__ dd pk_wsum(const double *__restrict__ P, int ps, int k, int a, int b)
+{
+    return dd_sub(pk_dd<KERN>(P, ps, k, b), pk_dd<KERN>(P, ps, k, a));
+}
+
 __device__ __forceinline__ dd ld_dd(const double2 *p) { const double2 v = *p; return dd{v.x, v.y}; }
 __device__ __forceinline__ void st_dd(double2 *p, dd v) { *p = make_double2(v.hi, v.lo); }
 
@@ -132,50 +210,6 @@ __device__ __forceinline__ int cold_step(const double *__restrict__ xs, int n, d
     if (!(span > 0.0)) return 1;
     const double e = 0.5 * (double)(n - 1) * (h / span);
     return e >= (double)n ? n : (e < 1.0 ? 1 : (int)e);
-}
-
-// SM-local task assignment (window kernels, SCHED = 1).  The task space
-// (chunk-major: consecutive tasks are adjacent row tiles at the same
-// bandwidths) is cut into one contiguous region per SM; the warps resident
-// on an SM take their region's tasks in order from its counter ctr[s], so
-// they work on neighbouring tiles at the same time and their boundary probes
-// and prefix loads hit the same L1 lines.  A warp whose region is exhausted
-// steals from the others (32 regions checked per round, one atomic per
-// candidate).  Returns -1 when every task has been taken.  Which warp runs a
-// task never changes its result (one partial per (tile, bandwidth)).
-__device__ __forceinline__ int region_lo(int r, int total, int nsm) { return (int)((long long)r * total / nsm); }
-
-__device__ __noinline__ int take_task_local(int *__restrict__ ctr, int total, int nsm, int lane)
-{
-    unsigned smid;
-    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-    const int own = (int)(smid % (unsigned)nsm);
-    int t = -1;
-    if (lane == 0) {
-        const int lo = region_lo(own, total, nsm), hi = region_lo(own + 1, total, nsm);
-        const int k = atomicAdd(ctr + own, 1);
-        if (lo + k < hi) t = lo + k;
-    }
-    t = __shfl_sync(0xffffffffu, t, 0);
-    if (t >= 0) return t;
-    for (int base = 1; base < nsm; base += 32) {
-        const int v = (own + base + lane) % nsm;
-        const int lo = region_lo(v, total, nsm), len = region_lo(v + 1, total, nsm) - lo;
-        const int left = base + lane < nsm ? len - *(volatile int *)(ctr + v) : 0;
-        unsigned ball = __ballot_sync(0xffffffffu, left > 0);
-        while (ball) {
-            const int src = __ffs(ball) - 1;
-            int got = -1;
-            if (lane == src) {
-                const int k = atomicAdd(ctr + v, 1);
-                if (k < len) got = lo + k;
-            }
-            got = __shfl_sync(0xffffffffu, got, src);
-            if (got >= 0) return got;
-            ball &= ball - 1;
-        }
-    }
-    return -1;
 }
 
 // ---------------------------------------------------------------- build
@@ -251,7 +285,8 @@ pfx_tile_reduce_kernel(const double2 *__restrict__ xy, int n, double2 *__restric
 template <int KERN, int ITEMS>
 __global__ void __launch_bounds__(kPfxThreads)
 pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__restrict__ tot, int ntiles,
-                     double *__restrict__ P, int pstride, double *__restrict__ xs)
+                     double *__restrict__ P, int pstride, double *__restrict__ xs,
+                     unsigned long long *__restrict__ gap_bits)
 {
     pdl_wait();  // krcv_pdl.cuh
     constexpr int K = NMom<KERN>::v;
@@ -287,6 +322,7 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
     const double o = pfx_origin(xy, n);
     dd tm[ITEMS][kPfxMoments];
     dd acc[kPfxMoments];
+    double gmin = INFINITY;
 #pragma unroll
     for (int k = 0; k < K; k++) acc[k] = dd{0.0, 0.0};
 #pragma unroll
@@ -294,6 +330,7 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
         if (j0 + q < n) {
             const double2 v = xy[j0 + q];
             xs[j0 + q] = v.x;
+            if (PfxRec<KERN>::S) gap_stat(xy, n, j0 + q, gmin);
             moment_terms<KERN>(v.x, v.y, o, tm[q]);
         } else {
 #pragma unroll
@@ -302,6 +339,7 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
 #pragma unroll
         for (int k = 0; k < K; k++) acc[k] = dd_add(acc[k], tm[q][k]);
     }
+    if (PfxRec<KERN>::S) gap_publish(gmin, gap_bits);
     // exclusive scan of the thread totals across the CTA
     dd ex[kPfxMoments];
 #pragma unroll
@@ -325,8 +363,8 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
 #pragma unroll
         for (int q = 0; q < ITEMS; q++) {
             if (j0 + q <= n) {
-                P[(size_t)(2 * k) * pstride + j0 + q] = run.hi;
-                P[(size_t)(2 * k + 1) * pstride + j0 + q] = run.lo;
+                pk_store<KERN>(P, pstride, k, j0 + q, run);
+                if (k == 0) pk_store_index<KERN>(P, pstride, j0 + q);
             }
             run = dd_add(run, tm[q][k]);
         }
@@ -346,7 +384,8 @@ constexpr int kPfx1Threads = 512;
 template <int KERN>
 __global__ void __launch_bounds__(kPfx1Threads)
 pfx_one_cta_kernel(const double2 *__restrict__ xy, int n, double *__restrict__ P, int pstride,
-                   double *__restrict__ xs, unsigned long long *__restrict__ ymax_bits)
+                   double *__restrict__ xs, unsigned long long *__restrict__ ymax_bits,
+                   unsigned long long *__restrict__ gap_bits)
 {
     constexpr int K = NMom<KERN>::v;
     constexpr int W = kPfx1Threads / 32;
@@ -364,10 +403,11 @@ pfx_one_cta_kernel(const double2 *__restrict__ xy, int n, double *__restrict__ P
     dd acc[kPfxMoments];
 #pragma unroll
     for (int k = 0; k < K; k++) acc[k] = dd{0.0, 0.0};
-    double ym = 0.0;
+    double ym = 0.0, gmin = INFINITY;
     for (int j = j0; j < j1; j++) {
         const double2 v = xy[j];
         ym = fmax(ym, fabs(v.y));
+        if (PfxRec<KERN>::S) gap_stat(xy, n, j, gmin);
         dd tm[kPfxMoments];
         moment_terms<KERN>(v.x, v.y, o, tm);
 #pragma unroll
@@ -376,6 +416,7 @@ pfx_one_cta_kernel(const double2 *__restrict__ xy, int n, double *__restrict__ P
 #pragma unroll
     for (int d = 16; d > 0; d >>= 1) ym = fmax(ym, __shfl_xor_sync(0xffffffffu, ym, d));
     if (lane == 0 && ym > 0.0) atomicMax(ymax_bits, (unsigned long long)__double_as_longlong(ym));
+    if (PfxRec<KERN>::S) gap_publish(gmin, gap_bits);
     // exclusive scan of the thread totals: within the warp, then over the warps
     dd ex[kPfxMoments];
 #pragma unroll
@@ -416,17 +457,15 @@ pfx_one_cta_kernel(const double2 *__restrict__ xy, int n, double *__restrict__ P
         moment_terms<KERN>(v.x, v.y, o, tm);
 #pragma unroll
         for (int k = 0; k < K; k++) {
-            P[(size_t)(2 * k) * pstride + j] = run[k].hi;
-            P[(size_t)(2 * k + 1) * pstride + j] = run[k].lo;
+            pk_store<KERN>(P, pstride, k, j, run[k]);
             run[k] = dd_add(run[k], tm[k]);
         }
+        pk_store_index<KERN>(P, pstride, j);
     }
     if (j1 == n && j0 < n) {  // the thread holding the last record writes P[k][n]
 #pragma unroll
-        for (int k = 0; k < K; k++) {
-            P[(size_t)(2 * k) * pstride + n] = run[k].hi;
-            P[(size_t)(2 * k + 1) * pstride + n] = run[k].lo;
-        }
+        for (int k = 0; k < K; k++) pk_store<KERN>(P, pstride, k, n, run[k]);
+        pk_store_index<KERN>(P, pstride, n);
     }
 }
 
@@ -564,10 +603,10 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
     const double dl = del.hi, adl = fabs(del.hi);
     double g;
     if (KERN == KR_UNIFORM) {
-        const double pb = ld_hi(P, ps, 0, R), pa = ld_hi(P, ps, 0, A);
+        const double pb = pk_hi<KERN>(P, ps, 0, R), pa = pk_hi<KERN>(P, ps, 0, A);
         double sy = (pb - pa) - yr;
         if (!(kFastSlack * (fabs(pb) + fabs(pa) + fabs(yr)) <= kFastTol * (double)c * ymax))
-            sy = dd_sub_to_d(wsum(P, ps, 0, A, R), dd_make(yr));
+            sy = dd_sub_to_d(pk_wsum<KERN>(P, ps, 0, A, R), dd_make(yr));
         g = sy / (double)c;
     } else {
         const double hk = (KERN == KR_EPANECHNIKOV) ? h * h : h;
@@ -575,19 +614,22 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
         bool fast = false;
         if (KERN == KR_EPANECHNIKOV) {
             // fast path: hi words only, plain double (error test: see kFastTol)
-            const double y_b = ld_hi(P, ps, 0, R), y_a = ld_hi(P, ps, 0, A);
-            const double u_b = ld_hi(P, ps, 1, R), u_a = ld_hi(P, ps, 1, A);
-            const double uu_b = ld_hi(P, ps, 2, R), uu_a = ld_hi(P, ps, 2, A);
-            const double yu_b = ld_hi(P, ps, 3, R), yu_a = ld_hi(P, ps, 3, A);
-            const double yuu_b = ld_hi(P, ps, 4, R), yuu_a = ld_hi(P, ps, 4, A);
-            const double c1 = (double)(c + 1);  // range count, row r included (its terms vanish)
+            // records R and A (PfxRec: y, u, u^2, y u, y u^2, j): three 16-byte loads each
+            const double2 *pr = reinterpret_cast<const double2 *>(P) + (size_t)R * 3;
+            const double2 *pa = reinterpret_cast<const double2 *>(P) + (size_t)A * 3;
+            const double2 r01 = __ldg(pr), r23 = __ldg(pr + 1), r45 = __ldg(pr + 2);
+            const double2 a01 = __ldg(pa), a23 = __ldg(pa + 1), a45 = __ldg(pa + 2);
+            const double y_b = r01.x, y_a = a01.x, u_b = r01.y, u_a = a01.y;
+            const double uu_b = r23.x, uu_a = a23.x, yu_b = r23.y, yu_a = a23.y;
+            const double yuu_b = r45.x, yuu_a = a45.x;
+            const double c1 = r45.y - a45.y;  // range count R - A, row r included (its terms vanish); exact
             const double Sy = y_b - y_a, Su = u_b - u_a, Suu = uu_b - uu_a;
             const double Syu = yu_b - yu_a, Syuu = yuu_b - yuu_a;
             s1 = fma(-dl, fma(-c1, dl, 2.0 * Su), Suu);
             sy1 = fma(-dl, fma(-dl, Sy, 2.0 * Syu), Syuu);
             sy = Sy - yr;
             num = fma(hk, sy, -sy1);
-            den = fma(hk, (double)c, -s1);
+            den = fma(hk, c1 - 1.0, -s1);
             const double ay = fabs(y_b) + fabs(y_a);
             const double E1 = fabs(uu_b) + fabs(uu_a) + 2.0 * adl * (fabs(u_b) + fabs(u_a)) +
                               2.0 * c1 * adl * (adl + h);
@@ -598,23 +640,23 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
         }
         if (!fast) {
             if (KERN == KR_EPANECHNIKOV) {
-                const dd Sy = wsum(P, ps, 0, A, R);
-                const dd Su = wsum(P, ps, 1, A, R);
-                const dd Suu = wsum(P, ps, 2, A, R);
-                const dd Syu = wsum(P, ps, 3, A, R);
-                const dd Syuu = wsum(P, ps, 4, A, R);
+                const dd Sy = pk_wsum<KERN>(P, ps, 0, A, R);
+                const dd Su = pk_wsum<KERN>(P, ps, 1, A, R);
+                const dd Suu = pk_wsum<KERN>(P, ps, 2, A, R);
+                const dd Syu = pk_wsum<KERN>(P, ps, 3, A, R);
+                const dd Syuu = pk_wsum<KERN>(P, ps, 4, A, R);
                 const dd t1 = dd_sub(dd_twice(Su), dd_mul_d_raw(del, (double)(c + 1)));
                 s1 = dd_sub_to_d(Suu, dd_mul_raw(del, t1));
                 const dd t2 = dd_sub(dd_twice(Syu), dd_mul_raw(del, Sy));
                 sy1 = dd_sub_to_d(Syuu, dd_mul_raw(del, t2));
                 sy = dd_sub_to_d(Sy, dd_make(yr));
             } else {  // triangular: right (r, R) and left [A, r) separately
-                const dd SyR = wsum(P, ps, 0, r + 1, R);
-                const dd SuR = wsum(P, ps, 1, r + 1, R);
-                const dd SyuR = wsum(P, ps, 2, r + 1, R);
-                const dd SyL = wsum(P, ps, 0, A, r);
-                const dd SuL = wsum(P, ps, 1, A, r);
-                const dd SyuL = wsum(P, ps, 2, A, r);
+                const dd SyR = pk_wsum<KERN>(P, ps, 0, r + 1, R);
+                const dd SuR = pk_wsum<KERN>(P, ps, 1, r + 1, R);
+                const dd SyuR = pk_wsum<KERN>(P, ps, 2, r + 1, R);
+                const dd SyL = pk_wsum<KERN>(P, ps, 0, A, r);
+                const dd SuL = pk_wsum<KERN>(P, ps, 1, A, r);
+                const dd SyuL = pk_wsum<KERN>(P, ps, 2, A, r);
                 const int cR = R - r - 1, cL = r - A;
                 // sum d  = (SuR - cR delta) + (cL delta - SuL)
                 const dd dR = dd_sub(SuR, dd_mul_d_raw(del, (double)cR));
@@ -719,12 +761,12 @@ __device__ __forceinline__ void window_advance(const double *__restrict__ xs, in
 // bandwidth the lane's first row searches from its previous bandwidth's
 // boundaries (window_bounds); each next row starts from its predecessor's
 // boundaries at the same bandwidth (window_advance, ~1 probe per side).
-template <int KERN, int K, int SCHED>
+template <int KERN, int K>
 __global__ void __launch_bounds__(kWinThreads)
 window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
               int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
               int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
-              uint8_t *__restrict__ tileN, int *__restrict__ tile_counter, int nsm)
+              uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
 {
     pdl_wait();  // krcv_pdl.cuh
     const int lane = threadIdx.x & 31;
@@ -737,14 +779,9 @@ window_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, con
         // split so that small shards still fill the GPU; a chunk starts its
         // searches cold (from the row itself), later steps from the previous h.
         int task = 0;
-        if (SCHED) {
-            task = take_task_local(tile_counter + 1, ntiles * nbc, nsm, lane);
-            if (task < 0) return;  // warp-uniform
-        } else {
-            if (lane == 0) task = atomicAdd(tile_counter, 1);
-            task = __shfl_sync(0xffffffffu, task, 0);
-            if (task >= ntiles * nbc) return;  // warp-uniform
-        }
+        if (lane == 0) task = atomicAdd(tile_counter, 1);
+        task = __shfl_sync(0xffffffffu, task, 0);
+        if (task >= ntiles * nbc) return;  // warp-uniform
         // chunk-major order: concurrently running warps hold adjacent tiles at
         // the same bandwidths, so their windows (and probes) overlap in L1/L2
         const int chunk = task / ntiles;
@@ -860,12 +897,12 @@ __device__ __forceinline__ void window_bounds2(const double *__restrict__ xs, in
     for (int c = 0; c < 4; c++) kout[c] = hi[c];
 }
 
-template <int KERN, int SCHED>
+template <int KERN>
 __global__ void __launch_bounds__(kWinThreads)
 window_kernel_b2(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
                  int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
                  int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
-                 uint8_t *__restrict__ tileN, int *__restrict__ tile_counter, int nsm)
+                 uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
 {
     pdl_wait();  // krcv_pdl.cuh
     const int lane = threadIdx.x & 31;
@@ -875,14 +912,9 @@ window_kernel_b2(const double *__restrict__ xs, const double2 *__restrict__ xy, 
     const int ps = pstride;
     for (;;) {
         int task = 0;
-        if (SCHED) {
-            task = take_task_local(tile_counter + 1, ntiles * nbc, nsm, lane);
-            if (task < 0) return;  // warp-uniform
-        } else {
-            if (lane == 0) task = atomicAdd(tile_counter, 1);
-            task = __shfl_sync(0xffffffffu, task, 0);
-            if (task >= ntiles * nbc) return;  // warp-uniform
-        }
+        if (lane == 0) task = atomicAdd(tile_counter, 1);
+        task = __shfl_sync(0xffffffffu, task, 0);
+        if (task >= ntiles * nbc) return;  // warp-uniform
         const int chunk = task / ntiles;  // chunk-major (see window_kernel)
         const int tile = task - chunk * ntiles;
         const int b0 = chunk * bper, b1 = min(m, b0 + bper);
@@ -930,565 +962,6 @@ window_kernel_b2(const double *__restrict__ xs, const double2 *__restrict__ xy, 
                     tileS[(size_t)(b + 1) * ntiles + tile] = e2b;
                     tileN[(size_t)(b + 1) * ntiles + tile] = (uint8_t)__popc(ballb);
                 }
-            }
-        }
-    }
-}
-
-// ---------------------------------------------------------------------------
-// Segment variant (window_kernel_seg<K, KR>): the boundary searches of a
-// warp's 32 KR consecutive rows read one shared-memory segment per side
-// instead of probing global memory one dependent load at a time.
-//
-// Both boundaries are monotone in the row: R_j (first index right of j
-// outside the window) and L_j (last index left of j outside) never decrease
-// as x_j grows, and at a larger bandwidth R_j grows and L_j shrinks.  So at
-// h_b every right boundary of the tile lies between the first row's and the
-// last row's, and those move by about the previous step's growth g.  Per
-// bandwidth the warp
-//   1. predicts the segment [S, E] of the sorted x that holds all the tile's
-//      right boundaries (first row's previous R + g - 3 sqrt g ... last row's
-//      previous R + g + 3 sqrt g), likewise for the left;
-//   2. loads it coalesced into its shared-memory slice (one round trip);
-//   3. verifies the prediction exactly -- xs[S] inside the first row's window
-//      (hence every row's) and xs[E] outside the last row's (hence every
-//      row's), the mirror conditions on the left -- with the same binary64
-//      predicate (reading Q1);
-//   4. every lane bisects its first row's boundaries in shared memory (lower
-//      end: the row's previous boundary) and advances its next rows from
-//      their predecessor's (typically 0-2 steps).
-// A failed check or a segment longer than kSegMax (sparse tiles) falls back,
-// warp-uniformly, to the global searches of window_kernel for that
-// bandwidth; the first bandwidth of a chunk always does (no prediction yet).
-// The boundaries found are the same indices either way, so the window sums
-// and the emitted partials are bit-identical to window_kernel's.
-constexpr int kSegMax = 512;
-
-__device__ __forceinline__ int seg_spread(int g) { return (int)(3.0f * sqrtf((float)g)) + 2; }
-
-// first q in (lo, hi] with seg[q] outside the right window of (xr, h);
-// lo inside, hi outside.  Gallops from lo (the next row's boundary usually
-// moves by 0-2), then bisects.
-template <int KERN>
-__device__ __forceinline__ int seg_first_out(const double *seg, int lo, int hi, double xr, double h)
-{
-    int step = 1;
-    for (;;) {
-        const int k = min(lo + step, hi);
-        if (k == hi) break;
-        if (!inside<KERN>(seg[k] - xr, h)) { hi = k; break; }
-        lo = k;
-        step <<= 1;
-    }
-    while (hi - lo > 1) {
-        const int k = (lo + hi) >> 1;
-        if (inside<KERN>(seg[k] - xr, h)) lo = k; else hi = k;
-    }
-    return hi;
-}
-
-// last q in [lo, hi) with seg[q] outside the left window of (xr, h); lo
-// outside, hi inside.  Gallop from lo, then bisect.
-template <int KERN>
-__device__ __forceinline__ int seg_last_out(const double *seg, int lo, int hi, double xr, double h)
-{
-    int step = 1;
-    for (;;) {
-        const int k = min(lo + step, hi);
-        if (k == hi) break;
-        if (inside<KERN>(xr - seg[k], h)) { hi = k; break; }
-        lo = k;
-        step <<= 1;
-    }
-    while (hi - lo > 1) {
-        const int k = (lo + hi) >> 1;
-        if (!inside<KERN>(xr - seg[k], h)) lo = k; else hi = k;
-    }
-    return lo;
-}
-
-template <int KERN, int KR>
-__global__ void __launch_bounds__(kWinThreads)
-window_kernel_seg(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
-                  int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
-                  int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
-                  uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
-{
-    __shared__ double s_seg[kWinWarps][2][kSegMax];
-    const int lane = threadIdx.x & 31;
-    double *segR = s_seg[threadIdx.x >> 5][0];
-    double *segL = s_seg[threadIdx.x >> 5][1];
-    const double o = pfx_origin(xy, n);
-    const double ymax = __longlong_as_double((long long)*ymax_bits);
-    const int bper = (m + nbc - 1) / nbc;
-    const int ps = pstride;
-    for (;;) {
-        int task = 0;
-        if (lane == 0) task = atomicAdd(tile_counter, 1);
-        task = __shfl_sync(0xffffffffu, task, 0);
-        if (task >= ntiles * nbc) return;  // warp-uniform
-        const int chunk = task / ntiles;  // chunk-major (see window_kernel)
-        const int tile = task - chunk * ntiles;
-        const int b0 = chunk * bper, b1 = min(m, b0 + bper);
-
-        const int i0 = row_lo + tile * 32 * KR + lane * KR;
-        WinRow rows[KR];
-        int nvalid = 0;
-#pragma unroll
-        for (int k = 0; k < KR; k++) {
-            const int i = i0 + k;
-            nvalid += i < row_hi ? 1 : 0;
-            rows[k].r = min(i, row_hi - 1);  // clamped rows do identical work, discarded
-            const double2 v = xy[rows[k].r];
-            rows[k].xr = v.x;
-            rows[k].yr = v.y;
-            rows[k].del = two_sum(v.x, -o);
-        }
-        // the tile's first and last row (monotonicity anchors of the checks)
-        const double xfirst = __shfl_sync(0xffffffffu, rows[0].xr, 0);
-        const double xlast = __shfl_sync(0xffffffffu, rows[KR - 1].xr, 31);
-        // this lane's first row: boundaries (absolute) and growth at the previous bandwidth
-        int R0 = rows[0].r + 1, L0 = rows[0].r - 1;
-        int gR = cold_step(xs, n, __ldg(hg + b0)), gL = gR;
-        // warp-level anchors: first row's R/L, last row's R/L and their growth
-        int Rf = 0, Rl = 0, Lf = 0, Ll = 0, gRf = 0, gRl = 0, gLf = 0, gLl = 0;
-        double hprev = 0.0;
-
-        for (int b = b0; b < b1; b++) {
-            const double h = __ldg(hg + b);
-            if (b == b0 + 1) {  // no growth observed yet: density estimate from the first windows
-                const double f = (h - hprev) / hprev;
-                const int rf = __shfl_sync(0xffffffffu, rows[0].r, 0), rl = __shfl_sync(0xffffffffu, rows[KR - 1].r, 31);
-                gRf = (int)fmin(ceil((Rf - rf) * f), (double)n);
-                gRl = (int)fmin(ceil((Rl - rl) * f), (double)n);
-                gLf = (int)fmin(ceil((rf - Lf) * f), (double)n);
-                gLl = (int)fmin(ceil((rl - Ll) * f), (double)n);
-            }
-            int Rk[KR], Lk[KR];
-            bool seg_ok = false;
-            if (b > b0) {
-                // 1. predicted segments (warp-uniform)
-                const bool rfull = Rf >= n, lfull = Ll <= -1;  // every row's window reaches the end
-                // (64-bit: growth and spread may reach n each)
-                int S = (int)min((long long)Rf - 1 + max(0, gRf - seg_spread(gRf)), (long long)n);
-                const int E = (int)min((long long)n, (long long)Rl + gRl + seg_spread(gRl));
-                S = min(S, E);
-                const int SL = (int)max(-1LL, (long long)Lf - gLf - seg_spread(gLf));
-                int EL = Ll + 1 - max(0, gLl - seg_spread(gLl));
-                EL = max(EL, SL);
-                const int lenR = rfull ? 1 : E - S + 1, lenL = lfull ? 1 : EL - SL + 1;
-                if (lenR <= kSegMax && lenL <= kSegMax) {
-                    // 2. coalesced loads into the warp's slice
-                    __syncwarp();
-                    if (!rfull)
-                        for (int q = lane; q < lenR; q += 32) segR[q] = __ldg(xs + S + q);
-                    if (!lfull)
-                        for (int q = lane; q < lenL; q += 32) segL[q] = __ldg(xs + SL + q);
-                    __syncwarp();
-                    // 3. exact check of the prediction
-                    bool ok = true;
-                    if (!rfull) ok = ok && inside<KERN>(segR[0] - xfirst, h) && !inside<KERN>(segR[lenR - 1] - xlast, h);
-                    if (!lfull) ok = ok && !inside<KERN>(xfirst - segL[0], h) && inside<KERN>(xlast - segL[lenL - 1], h);
-                    seg_ok = ok;  // identical in every lane (same loads, same predicate)
-                    if (ok) {
-                        // 4. per-lane searches in shared memory
-#pragma unroll
-                        for (int k = 0; k < KR; k++) {
-                            const double xr = rows[k].xr;
-                            if (rfull) {
-                                Rk[k] = n;
-                            } else {
-                                // lower end: row 0 its previous boundary - 1, row k its predecessor's - 1
-                                if (k == 0) {  // bisect (previous R - 1 is inside)
-                                    int lo = max(0, R0 - 1 - S), hh = lenR - 1;
-                                    while (hh - lo > 1) {
-                                        const int q = (lo + hh) >> 1;
-                                        if (inside<KERN>(segR[q] - xr, h)) lo = q; else hh = q;
-                                    }
-                                    Rk[0] = S + hh;
-                                } else {  // gallop from the predecessor's boundary
-                                    Rk[k] = S + seg_first_out<KERN>(segR, Rk[k - 1] - 1 - S, lenR - 1, xr, h);
-                                }
-                            }
-                            if (lfull) {
-                                Lk[k] = -1;
-                            } else if (k == 0) {
-                                // row 0: last outside in [0, previous L + 1 - SL]; previous L + 1 is inside
-                                const int hi = min(lenL - 1, L0 + 1 - SL);
-                                int lo = 0, hh = hi;
-                                while (hh - lo > 1) {
-                                    const int q = (lo + hh) >> 1;
-                                    if (!inside<KERN>(xr - segL[q], h)) lo = q; else hh = q;
-                                }
-                                Lk[0] = SL + lo;
-                            } else {
-                                Lk[k] = SL + seg_last_out<KERN>(segL, Lk[k - 1] - SL, lenL - 1, xr, h);
-                            }
-                        }
-                    }
-                }
-            }
-            if (!seg_ok) {  // global searches (window_kernel's)
-                int kR = R0 - rows[0].r, kL = rows[0].r - L0;
-                window_bounds<KERN>(xs, n, rows[0].r, rows[0].xr, h, kR, kL, gR, gL);
-                int R = rows[0].r + kR, L = rows[0].r - kL;
-                Rk[0] = R;
-                Lk[0] = L;
-#pragma unroll
-                for (int k = 1; k < KR; k++) {
-                    if (rows[k].r != rows[k - 1].r) window_advance<KERN>(xs, n, rows[k].r, rows[k].xr, h, R, L);
-                    Rk[k] = R;
-                    Lk[k] = L;
-                }
-            }
-            gR = max(1, Rk[0] - R0);
-            gL = max(1, L0 - Lk[0]);
-            R0 = Rk[0];
-            L0 = Lk[0];
-            {
-                const int nRf = __shfl_sync(0xffffffffu, Rk[0], 0), nLf = __shfl_sync(0xffffffffu, Lk[0], 0);
-                const int nRl = __shfl_sync(0xffffffffu, Rk[KR - 1], 31), nLl = __shfl_sync(0xffffffffu, Lk[KR - 1], 31);
-                if (b > b0) {
-                    gRf = nRf - Rf;
-                    gRl = nRl - Rl;
-                    gLf = Lf - nLf;
-                    gLl = Ll - nLl;
-                }
-                Rf = nRf;
-                Rl = nRl;
-                Lf = nLf;
-                Ll = nLl;
-            }
-            hprev = h;
-            double e2 = 0.0;
-            int cntM = 0;
-#pragma unroll
-            for (int k = 0; k < KR; k++) {
-                const int c = Rk[k] - Lk[k] - 2;
-                if (k < nvalid && c > 0) {  // reading Q6
-                    e2 += window_e2<KERN>(rows[k], Lk[k] + 1, Rk[k], c, h, xy, P, ps, ymax);
-                    cntM += 1;
-                }
-            }
-            e2 = warp_sum(e2);
-            const int cnt = __reduce_add_sync(0xffffffffu, cntM);  // <= 32 KR <= 128: fits the u8 slot
-            if (lane == 0) {
-                tileS[(size_t)b * ntiles + tile] = e2;
-                tileN[(size_t)b * ntiles + tile] = (uint8_t)cnt;
-            }
-        }
-    }
-}
-
-// ---------------------------------------------------------------------------
-// Cooperative variant (window_kernel_coop): a CTA owns kCoopRows = 128
-// consecutive sorted rows and a chunk of the bandwidth loop.  Per bandwidth:
-//   1. four "leader" boundaries -- right and left boundary of the tile's first
-//      and last row -- each found by one warp with 32 parallel probes per
-//      round (a 32-ary search from the previous bandwidth's boundary: one or
-//      two dependent round trips instead of ~8);
-//   2. since every row's boundaries lie between its tile's leaders (both are
-//      monotone in the row), the two segments [R_first, R_last] and
-//      [L_first, L_last] of the sorted x are staged in shared memory
-//      (coalesced) and every thread bisects its own boundaries there;
-//   3. the window arithmetic and the per-warp partials are window_e2's.
-// Segments longer than kCoopSeg (sparse data: a tile spanning a wide x range)
-// fall back, CTA-uniformly, to every thread's own global search.
-constexpr int kCoopRows = 128;
-constexpr int kCoopSeg = 1024;
-
-// 32-ary search by one warp: the first offset k > lo (offsets from row r,
-// direction by RIGHT) that is outside the window of row (r, xr) at h, given
-// that lo is inside (0 = the row itself) and the boundary is expected about
-// g past lo.  Returns the same value in every lane.
-template <int KERN, bool RIGHT>
-__device__ __forceinline__ int warp_boundary(const double *__restrict__ xs, int n, int r, double xr, double h, int lo,
-                                             int g, int lane)
-{
-    const int kmax = RIGHT ? n - r : r + 1;  // sentinel offset: outside
-    int s = max(1, (2 * g + 31) / 32);
-    for (;;) {
-        const int k = min(lo + (lane + 1) * s, kmax);
-        const double d = RIGHT ? xs[r + k] - xr : xr - xs[r - k];
-        const unsigned in = __ballot_sync(0xffffffffu, inside<KERN>(d, h));
-        const int cnt = __popc(in);  // inside probes form a prefix
-        if (cnt == 32) {             // all 32 inside: move on, widen
-            lo = min(lo + 32 * s, kmax);
-            s *= 2;
-            continue;
-        }
-        const int hi = min(lo + (cnt + 1) * s, kmax);  // first probed outside
-        lo = lo + cnt * s;                              // last probed inside
-        if (hi - lo <= 1) return hi;
-        s = (hi - lo + 31) / 32;  // refine inside (lo, hi)
-        if (s == 1) {
-            const int k2 = min(lo + lane + 1, hi);
-            const double d2 = RIGHT ? xs[r + k2] - xr : xr - xs[r - k2];
-            const unsigned in2 = __ballot_sync(0xffffffffu, k2 < hi && inside<KERN>(d2, h));
-            return lo + __popc(in2) + 1;
-        }
-    }
-}
-
-template <int KERN>
-__global__ void __launch_bounds__(kCoopRows)
-window_kernel_coop(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
-                   int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
-                   int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
-                   uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
-{
-    __shared__ double segR[kCoopSeg], segL[kCoopSeg];
-    __shared__ int s_lead[4];  // R_first, R_last (absolute), L_first, L_last (absolute)
-    __shared__ int s_task;
-    const int t = threadIdx.x, lane = t & 31, wp = t >> 5;
-    const double o = pfx_origin(xy, n);
-    const double ymax = __longlong_as_double((long long)*ymax_bits);
-    const int bper = (m + nbc - 1) / nbc;
-    const int ps = pstride;
-    const int ctiles = (ntiles + 3) / 4;  // CTA tiles of 128 rows (ntiles counts 32-row tiles)
-    for (;;) {
-        __syncthreads();
-        if (t == 0) s_task = atomicAdd(tile_counter, 1);
-        __syncthreads();
-        const int task = s_task;
-        if (task >= ctiles * nbc) return;  // block-uniform
-        const int chunk = task / ctiles;
-        const int ct = task - chunk * ctiles;
-        const int b0 = chunk * bper, b1 = min(m, b0 + bper);
-        const int first = row_lo + ct * kCoopRows;
-        const int last = min(row_hi, first + kCoopRows) - 1;
-
-        const int i = first + t;
-        const bool valid = i <= last;
-        WinRow w;
-        w.r = valid ? i : last;
-        const double2 v = xy[w.r];
-        w.xr = v.x;
-        w.yr = v.y;
-        w.del = two_sum(v.x, -o);
-        int kR = 1, kL = 1, gR = cold_step(xs, n, __ldg(hg + b0)), gL = gR;  // previous boundaries, growth
-        // leader state (offsets from the leader row): warp 0 R of first, 1 R of
-        // last, 2 L of first, 3 L of last
-        const int lrow = (wp & 1) ? last : first;
-        const double lx = xy[lrow].x;
-        int lk = 1, lg = 1;
-
-        for (int b = b0; b < b1; b++) {
-            const double h = __ldg(hg + b);
-            // 1. leaders
-            {
-                const int k = (wp < 2) ? warp_boundary<KERN, true>(xs, n, lrow, lx, h, lk - 1, lg, lane)
-                                       : warp_boundary<KERN, false>(xs, n, lrow, lx, h, lk - 1, lg, lane);
-                lg = max(1, k - lk);
-                lk = k;
-                if (lane == 0) s_lead[wp] = (wp < 2) ? lrow + k : lrow - k;
-            }
-            __syncthreads();
-            const int Rf = s_lead[0], Rl = s_lead[1], Lf = s_lead[2], Ll = s_lead[3];
-            const int lenR = Rl - Rf + 1, lenL = Ll - Lf + 1;
-            const bool seg = lenR <= kCoopSeg && lenL <= kCoopSeg;  // block-uniform
-            if (seg) {
-                for (int q = t; q < lenR; q += kCoopRows) segR[q] = xs[Rf + q];
-                for (int q = t; q < lenL; q += kCoopRows) segL[q] = xs[Lf + q];
-            }
-            __syncthreads();
-            int R, L;
-            if (seg) {
-                // right: first index in [Rf, Rl] outside for this row (Rl is)
-                int lo = -1, hi = lenR - 1;  // lo: inside (virtual), hi: outside
-                while (hi - lo > 1) {
-                    const int q = (lo + hi) >> 1;
-                    if (inside<KERN>(segR[q] - w.xr, h)) lo = q; else hi = q;
-                }
-                R = Rf + hi;
-                // left: last index in [Lf, Ll] outside for this row (Lf is)
-                int llo = 0, lhi = lenL;  // llo: outside, lhi: inside (virtual)
-                while (lhi - llo > 1) {
-                    const int q = (llo + lhi) >> 1;
-                    if (!inside<KERN>(w.xr - segL[q], h)) llo = q; else lhi = q;
-                }
-                L = Lf + llo;
-                const int nkR = R - w.r, nkL = w.r - L;
-                gR = max(1, nkR - kR);
-                gL = max(1, nkL - kL);
-                kR = nkR;
-                kL = nkL;
-            } else {
-                const int kR0 = kR, kL0 = kL;
-                window_bounds<KERN>(xs, n, w.r, w.xr, h, kR, kL, gR, gL);
-                gR = max(1, kR - kR0);
-                gL = max(1, kL - kL0);
-                R = w.r + kR;
-                L = w.r - kL;
-            }
-            const int c = R - L - 2;
-            const bool M = valid && c > 0;  // reading Q6
-            double e2 = M ? window_e2<KERN>(w, L + 1, R, c, h, xy, P, ps, ymax) : 0.0;
-            e2 = warp_sum(e2);
-            const unsigned ball = __ballot_sync(0xffffffffu, M);
-            const int tile = ct * 4 + wp;  // 32-row tile of the partial layout
-            if (lane == 0 && tile < ntiles) {
-                tileS[(size_t)b * ntiles + tile] = e2;
-                tileN[(size_t)b * ntiles + tile] = (uint8_t)__popc(ball);
-            }
-            __syncthreads();  // segments consumed before the next bandwidth's
-        }
-    }
-}
-
-// ---------------------------------------------------------------------------
-// Block variant (window_kernel_blk<K, KB>): lanes hold CONSECUTIVE rows (lane l
-// row base + 32 k + l of block k), and each block's boundary searches start
-// from an exact lower bound instead of a prediction.  Because R_j and L_j are
-// monotone in the row, the boundaries of block k lie at or beyond those of the
-// previous block's last row (lane 31): the segment xs[S .. S + 63] starting
-// there is loaded coalesced (two doubles per lane, one round trip) and every
-// lane finds its boundary in it by a 6-step branchless bisection over warp
-// shuffles.  Lanes whose boundary lies beyond the 64-element segment (sparse
-// data) continue with their own gallop from its end.  Block 0's lower bounds
-// are the tile's first row's own boundaries, found by one warp-cooperative
-// 32-ary search per side (warp_boundary) from the previous bandwidth's.
-// Same predicate (reading Q1), same windows, same window_e2 as window_kernel;
-// the tile groups 32 KB consecutive rows like window_kernel<K, KB>, but a
-// lane sums different rows, so CV agrees with it to rounding, not bitwise.
-
-// first outside right of absolute index lo (inside for row (r, xr), or lo = r)
-template <int KERN>
-__device__ __forceinline__ int right_from(const double *__restrict__ xs, int n, double xr, double h, int lo)
-{
-    int step = 1, hi;
-    for (;;) {
-        const int k = min(lo + step, n);  // xs[n] = +inf: outside
-        if (!inside<KERN>(__ldg(xs + k) - xr, h)) { hi = k; break; }
-        lo = k;
-        step <<= 1;
-    }
-    while (hi - lo > 1) {
-        const int k = (lo + hi) >> 1;
-        if (inside<KERN>(__ldg(xs + k) - xr, h)) lo = k; else hi = k;
-    }
-    return hi;
-}
-
-// last outside left of row r at or after absolute index lo (outside for (r, xr))
-template <int KERN>
-__device__ __forceinline__ int left_from(const double *__restrict__ xs, int r, double xr, double h, int lo)
-{
-    int step = 1, hi;
-    for (;;) {
-        const int k = min(lo + step, r);  // r itself is inside (d = 0)
-        if (k == r || inside<KERN>(xr - __ldg(xs + k), h)) { hi = k; break; }
-        lo = k;
-        step <<= 1;
-    }
-    while (hi - lo > 1) {
-        const int k = (lo + hi) >> 1;
-        if (!inside<KERN>(xr - __ldg(xs + k), h)) lo = k; else hi = k;
-    }
-    return lo;
-}
-
-// element q (0..63) of the warp's two-register segment (lane l holds l, 32 + l)
-__device__ __forceinline__ double seg_at(double c0, double c1, int q)
-{
-    const double v0 = __shfl_sync(0xffffffffu, c0, q & 31);
-    const double v1 = __shfl_sync(0xffffffffu, c1, q & 31);
-    return q < 32 ? v0 : v1;
-}
-
-template <int KERN, int KB>
-__global__ void __launch_bounds__(kWinThreads)
-window_kernel_blk(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P,
-                  int pstride, const double *__restrict__ hg, int m, int n, int row_lo, int row_hi, int ntiles,
-                  int nbc, const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
-                  uint8_t *__restrict__ tileN, int *__restrict__ tile_counter)
-{
-    const int lane = threadIdx.x & 31;
-    const double o = pfx_origin(xy, n);
-    const double ymax = __longlong_as_double((long long)*ymax_bits);
-    const int bper = (m + nbc - 1) / nbc;
-    const int ps = pstride;
-    for (;;) {
-        int task = 0;
-        if (lane == 0) task = atomicAdd(tile_counter, 1);
-        task = __shfl_sync(0xffffffffu, task, 0);
-        if (task >= ntiles * nbc) return;  // warp-uniform
-        const int chunk = task / ntiles;  // chunk-major (see window_kernel)
-        const int tile = task - chunk * ntiles;
-        const int b0 = chunk * bper, b1 = min(m, b0 + bper);
-        const int base = row_lo + tile * 32 * KB;  // < row_hi
-        const double xb = xy[base].x;
-        // the first row's boundaries (offsets from base) and growth at the previous bandwidth
-        int kR = 1, kL = 1, gR = cold_step(xs, n, __ldg(hg + b0)), gL = gR;
-        for (int b = b0; b < b1; b++) {
-            const double h = __ldg(hg + b);
-            // block 0's lower bounds: the first row's own boundaries (warp-cooperative)
-            {
-                const int nR = warp_boundary<KERN, true>(xs, n, base, xb, h, kR - 1, gR, lane);
-                const int nL = warp_boundary<KERN, false>(xs, n, base, xb, h, kL - 1, gL, lane);
-                gR = max(1, nR - kR);
-                gL = max(1, nL - kL);
-                kR = nR;
-                kL = nL;
-            }
-            int SR = base + kR, SL = base - kL;  // R of the row before the block (or the first row), L likewise
-            double e2 = 0.0;
-            int cntM = 0;
-#pragma unroll
-            for (int k = 0; k < KB; k++) {
-                const int i = base + 32 * k + lane;
-                const bool valid = i < row_hi;
-                WinRow w;
-                w.r = valid ? i : row_hi - 1;  // clamped rows do identical work, discarded
-                const double2 v = xy[w.r];
-                w.xr = v.x;
-                w.yr = v.y;
-                w.del = two_sum(v.x, -o);
-                // right: xs[SR - 1] is inside for every row of the block (or a row
-                // at or before it); the first outside lies at SR or beyond
-                const double r0 = __ldg(xs + min(SR + lane, n)), r1 = __ldg(xs + min(SR + 32 + lane, n));
-                // (indices >= the row are never compared; clamped to stay inside xs)
-                const double l0 = __ldg(xs + min(SL + lane, n)), l1 = __ldg(xs + min(SL + 32 + lane, n));
-                // (the shuffles run in every lane; lanes whose boundary lies past
-                // the segment then take their own gallop)
-                int R, L;
-                {
-                    // inside count of xs[SR .. SR + 63] (a prefix: the predicate is monotone)
-                    const double last = __shfl_sync(0xffffffffu, r1, 31);
-                    const bool beyond = SR + 63 < n && inside<KERN>(last - w.xr, h);
-                    int idx = 0;
-#pragma unroll
-                    for (int st = 32; st > 0; st >>= 1)
-                        idx += inside<KERN>(seg_at(r0, r1, idx + st - 1) - w.xr, h) ? st : 0;
-                    R = beyond ? right_from<KERN>(xs, n, w.xr, h, SR + 63) : min(SR + idx, n);
-                }
-                {
-                    // xs[SL] is outside for every row of the block; outside count of
-                    // xs[SL .. SL + 63] (indices >= the row are inside: d <= 0)
-                    const double last = __shfl_sync(0xffffffffu, l1, 31);
-                    const bool beyond = SL + 63 < w.r && !inside<KERN>(w.xr - last, h);
-                    int idx = 0;
-#pragma unroll
-                    for (int st = 32; st > 0; st >>= 1) {
-                        const int q = idx + st - 1;
-                        const double v = seg_at(l0, l1, q);
-                        idx += (SL + q < w.r && !inside<KERN>(w.xr - v, h)) ? st : 0;
-                    }
-                    L = beyond ? left_from<KERN>(xs, w.r, w.xr, h, SL + 63) : SL + idx - 1;
-                }
-                SR = __shfl_sync(0xffffffffu, R, 31);
-                SL = __shfl_sync(0xffffffffu, L, 31);
-                const int c = R - L - 2;
-                if (valid && c > 0) {  // reading Q6
-                    e2 += window_e2<KERN>(w, L + 1, R, c, h, xy, P, ps, ymax);
-                    cntM += 1;
-                }
-            }
-            e2 = warp_sum(e2);
-            const int cnt = __reduce_add_sync(0xffffffffu, cntM);  // <= 32 KB <= 128: fits the u8 slot
-            if (lane == 0) {
-                tileS[(size_t)b * ntiles + tile] = e2;
-                tileN[(size_t)b * ntiles + tile] = (uint8_t)cnt;
             }
         }
     }

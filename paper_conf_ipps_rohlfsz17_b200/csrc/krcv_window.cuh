@@ -1,0 +1,265 @@
+// krcv_window.cuh -- the window-prefix hot loop with bucket-table boundary
+// lookups (a3 + a4 of SURVEY.md §8).
+//
+// The method (§III P@13614-14984, §IV.B P@21724-22104): for every
+// row i and every bandwidth h_b of the ascending grid, the neighbours within
+// h_b of x_i, their running sums c, sum y, sum d^2, sum y d^2 (reading Q3),
+// the LOO estimate Eq.(2) and the squared error of Eq.(1).  On the globally
+// sorted array row r's window at h is the index range [A, R) minus r itself:
+//     R = first k > r  with  NOT (xs[k] - x_r < h)   (<= for uniform, Q1)
+//     A = first k <= r with       x_r - xs[k] < h
+// and the running sums are differences of prefix sums (krcv_prefix.cuh).
+//
+// What this kernel changes against r01's window_kernel (krcv_prefix.cuh,
+// kept for A/B runs as KRCV_WIN=r01): the boundaries are no longer searched
+// from the previous bandwidth's (a dependent galloping chain of ~8 probes per
+// side), but looked up.  A bucket table over the x range,
+//     BT[q] = first k with bkt(xs[k]) >= q,   q = 0 .. Q,
+//     bkt(v) = lo32(fma(v, Q / span, 1.5 * 2^52 - x_min Q / span))
+// (bkt is round-to-nearest of (v - x_min) Q / span, read from the low mantissa
+// word; monotone non-decreasing in v), maps t = x_r + h to a hint
+// k0 = BT[bkt(t)]: every k < k0 has xs[k] < t and every k >= BT[bkt(t) + 1]
+// has xs[k] > t.  The exact predicate differs from "xs[k] < t" only for
+// values within an ulp of t, so four independent probes k0 - 1 .. k0 + 2
+// decide the boundary whenever the bucket holds <= 2 points below t; a
+// gallop + bisection from the hint covers every other case (ties, crowded
+// buckets), so the hint never decides an index, only how fast it is found.
+// Q = F n with F = 2^k chosen per call from the data's peak density (the
+// smallest x-span of kGapSpan + 1 sorted records, krcv_prefix.cuh), so the
+// densest region still averages about half a point per bucket (F <= kBktFmax).
+// Sides whose window reaches the end of the data (x_max - x_r < h, resp.
+// x_r - x_min < h) take R = n (A = 0) with no lookup at all.
+//
+// Every (row, bandwidth) is independent, so a warp task is a block of TB
+// tiles of 32 consecutive sorted rows (lane = row, coalesced loads) times a
+// chunk of <= 64 bandwidths; per (tile, bandwidth) the warp's squared errors
+// are summed by a fixed butterfly and lane (b - b0) mod 32 accumulates the
+// chunk's sums over the TB tiles in registers.  One partial per (block,
+// bandwidth) -- TB times fewer than one per tile (the tile
+// partials were 6x the algorithmic DRAM bytes at C4) -- written once,
+// reduced in a fixed order by reduce_kernel: bit-reproducible.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "krcv.h"
+#include "krcv_pdl.cuh"
+#include "krcv_prefix.cuh"
+
+namespace krcv {
+
+constexpr int kBktFmax = 32;             // buckets per point, at most
+constexpr int64_t kBktQmax = 1LL << 28;  // buckets, at most
+constexpr double kBktMagic = 6755399441055744.0;  // 1.5 * 2^52: fma(.) + magic keeps the integer in the low word
+constexpr int kBktFillThreads = 256;
+constexpr int kBktSeg = 16;              // merge-path items per thread of the table fill
+
+// Table parameters, written by bkt_fill_kernel's first thread, read by the
+// window kernel (both compute them from the same inputs).
+struct BktParams {
+    double invw;  // Q / span
+    double C;     // kBktMagic - x_min Q / span
+    int Q;        // buckets 0 .. Q
+    int F;
+};
+
+__device__ __forceinline__ int bkt_raw(double v, double invw, double C)
+{
+    return __double2loint(fma(v, invw, C));
+}
+
+// Parameters of the table for this call: F from the peak density.
+__device__ __forceinline__ BktParams bkt_params(const double *__restrict__ xs, int n,
+                                                const unsigned long long *__restrict__ gap_bits)
+{
+    BktParams p;
+    const double lo = xs[0], span = xs[n - 1] - xs[0];
+    const unsigned long long gb = *gap_bits;
+    int F = 1;
+    if (gb != 0ull && span > 0.0) {
+        const double gap = __longlong_as_double((long long)~gb);  // min x-span of kGapSpan + 1 records
+        // ratio of the peak density kGapSpan / gap to the mean (n - 1) / span,
+        // times 2: about half a point per bucket where the data is densest
+        const double ratio = gap > 0.0 ? 2.0 * (double)kGapSpan * span / (gap * (double)(n - 1)) : 1e300;
+        while (F < kBktFmax && (double)F < ratio) F <<= 1;
+    }
+    int64_t Q = (int64_t)F * n;
+    if (Q > kBktQmax) Q = kBktQmax;
+    p.F = F;
+    p.Q = (int)Q;
+    p.invw = span > 0.0 ? (double)Q / span : 0.0;
+    p.C = kBktMagic - lo * p.invw;
+    return p;
+}
+
+// BT[q] = #{k : bkt(xs[k]) < q} for q = 0 .. Q: the merge of the sorted
+// bucket ids A[k] = clamp(bkt(xs[k]), 0, Q) with the sequence 0 .. Q (A[k]
+// goes first iff A[k] < q), cut into segments of kBktSeg merged items by a
+// binary search on each segment's diagonal (merge path), so long runs of
+// empty buckets (the sparse tail of a heavy-tailed x) are spread over many
+// threads.  Grid-stride over segments; the grid is sized for Q <= kBktFmax n.
+__global__ void __launch_bounds__(kBktFillThreads)
+bkt_fill_kernel(const double *__restrict__ xs, int n, const unsigned long long *__restrict__ gap_bits,
+                int *__restrict__ BT, BktParams *__restrict__ prm)
+{
+    pdl_wait();  // krcv_pdl.cuh
+    const BktParams p = bkt_params(xs, n, gap_bits);
+    if (blockIdx.x == 0 && threadIdx.x == 0) *prm = p;
+    const int Q = p.Q;
+    auto A = [&](int k) { return min(max(bkt_raw(xs[k], p.invw, p.C), 0), Q); };
+    const int64_t total = (int64_t)n + Q + 1;
+    const int64_t nseg = (total + kBktSeg - 1) / kBktSeg;
+    for (int64_t sg = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; sg < nseg;
+         sg += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t d = sg * kBktSeg;
+        // split of the first d merged items: i from A, d - i from B.  Smallest
+        // i with "B[d - i - 1] before A[i]" (A[i] >= d - i - 1), monotone in i.
+        int64_t lo = d - (Q + 1) > 0 ? d - (Q + 1) : 0;
+        int64_t hi = d < n ? d : n;
+        while (lo < hi) {
+            const int64_t mid = (lo + hi) >> 1;
+            if ((int64_t)A((int)mid) >= d - mid - 1) hi = mid; else lo = mid + 1;
+        }
+        int i = (int)lo;
+        int64_t j = d - lo;
+        int ai = i < n ? A(i) : 0;
+        for (int s = 0; s < kBktSeg && (int64_t)i + j < total; s++) {
+            if (i < n && (j > Q || (int64_t)ai < j)) {
+                i++;
+                ai = i < n ? A(i) : 0;
+            } else {
+                BT[j] = i;
+                j++;
+            }
+        }
+    }
+}
+
+// First k in [lo, hi] with p(k) true, p monotone (false ... true), p(hi)
+// true, and p(lo - 1) false wherever it is read (the +-inf sentinels and row
+// r make that hold for both sides).  Four probes around the hint k0 settle
+// the common case; otherwise gallop from the hint in the direction the probes
+// point, then bisect.  Exact for any hint.
+template <class Pred>
+__device__ __forceinline__ int first_true(Pred p, int lo, int hi, int k0)
+{
+    const int k = min(max(k0, lo), hi);
+    const bool pa = p(k - 1), pb = p(k), pc = p(k + 1), pd = p(k + 2);
+    if (!pa && pd) return k + (pb ? 0 : (pc ? 1 : 2));
+    int a, b;  // p(a) false (a >= lo - 1), p(b) true
+    if (pa) {  // boundary at or below k - 1: gallop down
+        b = k - 1;
+        int step = 1;
+        a = b - 1;
+        while (a >= lo && p(a)) {
+            b = a;
+            step <<= 1;
+            a = b - step;
+        }
+        a = max(a, lo - 1);
+    } else {   // p(k + 2) false: gallop up
+        a = k + 2;
+        int step = 1;
+        b = min(a + 1, hi);
+        while (b < hi && !p(b)) {
+            a = b;
+            step <<= 1;
+            b = min(a + step, hi);
+        }
+    }
+    while (b - a > 1) {
+        const int mid = (a + b) >> 1;
+        if (p(mid)) b = mid; else a = mid;
+    }
+    return b;
+}
+
+constexpr int kWin2Warps = 4;
+constexpr int kWin2Threads = kWin2Warps * 32;
+constexpr int kWin2Chunk = 64;  // bandwidths per task, at most (two accumulators per lane)
+
+// task = (block of TB tiles of 32 sorted rows, chunk of <= 64 bandwidths),
+// chunk-major so that concurrently running warps hold adjacent blocks at the
+// same bandwidths.  Output: tileS[b][blk], tileN[b][blk] (blk = block index).
+template <int KERN>
+__global__ void __launch_bounds__(kWin2Threads)
+win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P, int pstride,
+           const int *__restrict__ BT, const BktParams *__restrict__ prm, const double *__restrict__ hg, int m,
+           int n, int row_lo, int row_hi, int TB, int nblk, int BC, int nbc,
+           const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
+           uint32_t *__restrict__ tileN, int *__restrict__ task_counter)
+{
+    pdl_wait();  // krcv_pdl.cuh
+    const int lane = threadIdx.x & 31;
+    const double o = pfx_origin(xy, n);
+    const double ymax = __longlong_as_double((long long)*ymax_bits);
+    const double xmin = xs[0], xmax = xs[n - 1];
+    const double invw = prm->invw, C = prm->C;
+    const int Q = prm->Q;
+    const int ntasks = nblk * nbc;
+    for (;;) {
+        int task = 0;
+        if (lane == 0) task = atomicAdd(task_counter, 1);
+        task = __shfl_sync(0xffffffffu, task, 0);
+        if (task >= ntasks) return;  // warp-uniform
+        const int chunk = task / nblk;
+        const int blk = task - chunk * nblk;
+        const int b0 = chunk * BC, b1 = min(m, b0 + BC);
+        double acc0 = 0.0, acc1 = 0.0;
+        uint32_t cnt0 = 0, cnt1 = 0;
+        for (int t = 0; t < TB; t++) {
+            const int base = row_lo + (blk * TB + t) * 32;
+            if (base >= row_hi) break;  // warp-uniform
+            const int i = base + lane;
+            const bool valid = i < row_hi;
+            WinRow w;
+            w.r = valid ? i : row_hi - 1;  // clamped rows do identical work, discarded
+            const double2 v = xy[w.r];
+            w.xr = v.x;
+            w.yr = v.y;
+            w.del = two_sum(v.x, -o);  // exact x_r - o
+            const int r = w.r;
+            const double xr = w.xr;
+            const double dmax = xmax - xr, dmin = xr - xmin;
+            for (int b = b0; b < b1; b++) {
+                const double h = __ldg(hg + b);
+                int R = n, A = 0;
+                if (!inside<KERN>(dmax, h)) {  // window ends inside the data: look R up
+                    const int k0 = __ldg(BT + min(max(bkt_raw(xr + h, invw, C), 0), Q));
+                    R = first_true([&](int k) { return !inside<KERN>(__ldg(xs + k) - xr, h); }, r + 1, n, k0);
+                }
+                if (!inside<KERN>(dmin, h)) {
+                    const int k0 = __ldg(BT + min(max(bkt_raw(xr - h, invw, C), 0), Q));
+                    A = first_true([&](int k) { return inside<KERN>(xr - __ldg(xs + k), h); }, 0, r, k0);
+                }
+                const int c = R - A - 1;
+                const bool M = valid && c > 0;  // reading Q6
+                double e2 = M ? window_e2<KERN>(w, A, R, c, h, xy, P, pstride, ymax) : 0.0;
+                e2 = warp_sum(e2);  // fixed butterfly: every lane holds the tile's sum
+                const uint32_t nb = __popc(__ballot_sync(0xffffffffu, M));
+                const int bl = b - b0;
+                if (lane == (bl & 31)) {
+                    if (bl < 32) {
+                        acc0 += e2;
+                        cnt0 += nb;
+                    } else {
+                        acc1 += e2;
+                        cnt1 += nb;
+                    }
+                }
+            }
+        }
+        if (b0 + lane < b1) {
+            tileS[(size_t)(b0 + lane) * nblk + blk] = acc0;
+            tileN[(size_t)(b0 + lane) * nblk + blk] = cnt0;
+        }
+        if (b0 + 32 + lane < b1) {
+            tileS[(size_t)(b0 + 32 + lane) * nblk + blk] = acc1;
+            tileN[(size_t)(b0 + 32 + lane) * nblk + blk] = cnt1;
+        }
+    }
+}
+
+}  // namespace krcv

@@ -2,8 +2,8 @@
 synccheck and initcheck over tests/sanitize/gpu_driver.py, which runs every
 CUDA path of libkrcv.so once at small sizes (both sort paths, prefix build,
 window kernel, sweep, histogram, Gaussian, KDE, local-linear, refinement,
-reduction + fused finalize, the non-finite error path).  The shared-memory
-window variants (KRCV_WIN_K = 5 coop, 6 seg) get their own racecheck run.
+reduction + fused finalize, the non-finite error path).  The
+default window kernel and r01's (KRCV_WIN=r01) each get a racecheck run.
 Any sanitizer report fails the test (--error-exitcode)."""
 from __future__ import annotations
 
@@ -42,6 +42,6 @@ def test_compute_sanitizer_initcheck():
     _run("initcheck")
 
 
-@pytest.mark.parametrize("win", ["2", "5", "6"])
+@pytest.mark.parametrize("win", ["default", "r01"])
 def test_compute_sanitizer_racecheck(win):
-    _run("racecheck", {"KRCV_WIN_K": win})
+    _run("racecheck", {} if win == "default" else {"KRCV_WIN": "r01", "KRCV_WIN_K": "2"})

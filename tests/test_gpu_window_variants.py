@@ -1,17 +1,16 @@
-"""GPU: the window-kernel variants find the same boundaries.
+"""GPU: the window kernels find the same boundaries.
 
-`window_kernel_blk` (KRCV_WIN_K = 9 / 10: 2 / 4 blocks of 32 consecutive rows)
-sums a tile's rows in another order than window_kernel<K, 2 / 4>: n_eff and
-best must be identical, CV equal to rounding.
-
-`window_kernel_seg` (KRCV_WIN_K = 6 / 7 / 8: 2 / 4 / 1 rows per lane) searches
-in a shared-memory segment with an exact check of its prediction and falls
-back to `window_kernel`'s global searches; with the same rows per lane
-(KRCV_WIN_K = 2 / 4 / 1) the two kernels group rows into the same tiles, so
-their CV curves must agree bit for bit.  The library reads KRCV_WIN_K once per
-process, so each variant runs in a subprocess.  Inputs stress the fallback:
-heavy-tailed x (sparse tiles, segments longer than the cap), duplicates,
-points exactly at a bandwidth, a jump in the grid, tiny n.
+`win_kernel` (krcv_window.cuh, the default) looks every boundary up in a
+bucket table and verifies it with the exact binary64 predicate of reading Q1;
+r01's `window_kernel<K>` / `window_kernel_b2` (KRCV_WIN=r01, KRCV_WIN_K = 1 /
+2 / 3) search from the previous bandwidth's boundaries.  The windows -- hence
+n_eff -- must be identical, and so must best; the CV curves are equal to
+rounding (the kernels sum a bandwidth's squared errors in different orders:
+one partial per 32-row tile vs per block of tiles).  The library reads the
+selection once per process, so each variant runs in a subprocess.  Inputs
+stress the lookups: heavy-tailed x (crowded and empty buckets, F at its cap),
+duplicates, points exactly at a bandwidth, a jump in the grid, tiny n, all x
+equal (zero span), two distinct values.
 """
 from __future__ import annotations
 
@@ -69,41 +68,35 @@ def _cases():
     hj = np.concatenate([np.linspace(1e-4, 1e-3, 20), np.linspace(0.2, 1.0, 20)])
     cases["jump"] = (xs, ys, hj, "epanechnikov")
     cases["tiny"] = (xs[:37], ys[:37], np.linspace(0.01, 1.0, 30), "epanechnikov")
+    cases["const_x"] = (np.full(300, 0.5), ys[:300], np.array([1e-3, 0.1, 1.0]), "epanechnikov")
+    cases["two_values"] = (np.repeat([0.0, 1.0], 150), ys[:300], np.array([0.5, 1.0, 1.0, 2.0]), "uniform")
     return cases
 
 
-def _run(k: int, path: str):
-    env = dict(os.environ, KRCV_WIN_K=str(k))
+def _run(env_extra: dict, path: str):
+    env = dict(os.environ, **env_extra)
     p = subprocess.run([sys.executable, "-c", CHILD, path], cwd=ROOT, env=env, capture_output=True, text=True,
                        timeout=600)
     assert p.returncode == 0, p.stderr[-2000:]
     return json.loads(p.stdout.strip().splitlines()[-1])
 
 
-@pytest.mark.parametrize("base,seg", [(2, 6), (4, 7), (1, 8)])
-def test_seg_kernel_bit_identical(tmp_path, base, seg):
+@pytest.fixture(scope="module")
+def case_path(tmp_path_factory):
     cases = _cases()
-    path = str(tmp_path / "cases.npz")
+    path = str(tmp_path_factory.mktemp("winvar") / "cases.npz")
     arrs = {}
     for c, (x, y, h, k) in cases.items():
         arrs[c + "_x"], arrs[c + "_y"], arrs[c + "_h"], arrs[c + "_k"] = x, y, h, np.array(k)
     np.savez(path, **arrs)
-    a, b = _run(base, path), _run(seg, path)
-    for c in cases:
-        assert a[c]["cv"] == b[c]["cv"], c
-        assert a[c]["neff"] == b[c]["neff"], c
-        assert a[c]["best"] == b[c]["best"], c
+    return path, cases
 
 
-@pytest.mark.parametrize("base,blk", [(2, 9), (4, 10)])
-def test_blk_kernel_same_windows(tmp_path, base, blk):
-    cases = _cases()
-    path = str(tmp_path / "cases.npz")
-    arrs = {}
-    for c, (x, y, h, k) in cases.items():
-        arrs[c + "_x"], arrs[c + "_y"], arrs[c + "_h"], arrs[c + "_k"] = x, y, h, np.array(k)
-    np.savez(path, **arrs)
-    a, b = _run(base, path), _run(blk, path)
+@pytest.mark.parametrize("r01k", ["1", "2", "3"])
+def test_win_kernel_same_windows_as_r01(case_path, r01k):
+    path, cases = case_path
+    a = _run({}, path)
+    b = _run({"KRCV_WIN": "r01", "KRCV_WIN_K": r01k}, path)
     for c in cases:
         ca = np.array(a[c]["cv"], np.uint64).view(np.float64)
         cb = np.array(b[c]["cv"], np.uint64).view(np.float64)
@@ -111,3 +104,19 @@ def test_blk_kernel_same_windows(tmp_path, base, blk):
         scale = max(float(np.max(np.abs(ca))), 1e-300)
         assert float(np.max(np.abs(ca - cb))) <= 1e-13 * scale, c
         assert a[c]["best"] == b[c]["best"], c
+
+
+def test_win_kernel_matches_oracle(case_path):
+    """The default kernel on the same stress inputs against Program 3."""
+    import oracle
+    from tests.helpers import best_ok, cv_rel_err
+
+    path, cases = case_path
+    a = _run({}, path)
+    kid = {"uniform": 0, "epanechnikov": 1, "triangular": 2}
+    for c, (x, y, h, k) in cases.items():
+        ref = oracle.cv_sorted(x, y, h, kid[k])
+        got = np.array(a[c]["cv"], np.uint64).view(np.float64)
+        assert cv_rel_err(got, ref.cv) <= 1e-10, c
+        assert np.array_equal(np.asarray(a[c]["neff"]), ref.neff), c
+        assert best_ok(a[c]["best"], ref.cv), c
