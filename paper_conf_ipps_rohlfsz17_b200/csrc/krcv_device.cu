@@ -173,10 +173,15 @@ struct FinOut {
     unsigned *done;
 };
 
-template <typename CountT>  // uint8_t (one partial per 32-row tile) or uint32_t (win_kernel's row blocks)
+// Partial layouts: [m][ntiles] with every column entry valid (slots == 0:
+// one partial per 32-row tile, uint8 counts), or win_kernel's warp slots
+// (slots = S > 0, uint32 counts, krcv_window.cuh): bandwidth b of chunk
+// c = b / bc was run by all S slots when ntiles >= S, else by the ntiles slots
+// (c ntiles + t) mod S, t = 0 .. ntiles-1 -- summed in that (fixed) order.
+template <typename CountT>
 __global__ void __launch_bounds__(kReduceThreads)
 reduce_kernel(const double *__restrict__ tileS, const CountT *__restrict__ tileN, int ntiles, int m,
-              const unsigned *__restrict__ status, double *__restrict__ partial, FinOut fin)
+              const unsigned *__restrict__ status, double *__restrict__ partial, FinOut fin, int slots, int bc)
 {
     pdl_wait();  // krcv_pdl.cuh
     __shared__ double sS[kReduceThreads];
@@ -186,11 +191,24 @@ reduce_kernel(const double *__restrict__ tileS, const CountT *__restrict__ tileN
     for (int b = blockIdx.x; b < m; b += gridDim.x) {
         double a = 0.0;
         long long cnt = 0;
-        const double *col = tileS + (size_t)b * ntiles;
-        const CountT *ncol = tileN + (size_t)b * ntiles;
-        for (int t = threadIdx.x; t < ntiles; t += kReduceThreads) {
-            a += col[t];
-            cnt += ncol[t];
+        if (slots == 0) {
+            const double *col = tileS + (size_t)b * ntiles;
+            const CountT *ncol = tileN + (size_t)b * ntiles;
+            for (int t = threadIdx.x; t < ntiles; t += kReduceThreads) {
+                a += col[t];
+                cnt += ncol[t];
+            }
+        } else {
+            const int nsl = ntiles >= slots ? slots : ntiles;
+            const int first = ntiles >= slots ? 0 : (int)(((int64_t)(b / bc) * ntiles) % slots);
+            const double *col = tileS + (size_t)b * slots;
+            const CountT *ncol = tileN + (size_t)b * slots;
+            for (int q = threadIdx.x; q < nsl; q += kReduceThreads) {
+                int sl = first + q;
+                sl = sl >= slots ? sl - slots : sl;
+                a += col[sl];
+                cnt += ncol[sl];
+            }
         }
         // fixed tree: butterfly within each warp, then warp 0 adds the eight
         // warp sums in order (bit-reproducible, one barrier)
@@ -302,6 +320,11 @@ static const DevInfo &dev_info()
     return info[d];
 }
 
+// partial slots win_kernel may use on this device (workspace sizing): at
+// most 64 resident warps per SM (the uniform instantiation's 56 registers
+// allow 9 CTAs = 36 warps per SM)
+static int64_t win2_max_slots() { return (int64_t)dev_info().sms * 64; }
+
 static int occupancy(const void *func, int threads, size_t smem = 0)
 {
     struct Key {
@@ -377,7 +400,11 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     L->pstride = (int64_t)(((size_t)n + 1 + 15) & ~size_t(15));
     L->nch = (int64_t)nch;
     L->xs = off;       off = align256(off + sizeof(double) * ((size_t)n + 2 * kPad));
-    L->pfx = off;      off = align256(off + sizeof(double2) * kPfxMoments * (size_t)L->pstride);
+    // prefix moments: SoA planes (KDE, local-linear: 8 x 2 x pstride doubles) or the
+    // blocked records of the NW sets (2 x 5 x pk_slots doubles at most)
+    const size_t pfx_soa = sizeof(double2) * kPfxMoments * (size_t)L->pstride;
+    const size_t pfx_rec = sizeof(double) * 2 * pk_lo_off<KR_EPANECHNIKOV>((int)L->pstride);
+    L->pfx = off;      off = align256(off + (pfx_soa > pfx_rec ? pfx_soa : pfx_rec));
     L->ptot = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
     L->status = off;   off = align256(off + 8 * sizeof(unsigned));  // bad grid, non-finite, done, pad, u64 max|y| bits
     L->cub = off;      off = align256(off + cub_bytes);
@@ -387,11 +414,11 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     // bucket table of win_kernel (krcv_window.cuh): int32 [Qmax + 1], Qmax = min(kBktFmax n, kBktQmax)
     const int64_t qmax = (int64_t)kBktFmax * n < kBktQmax ? (int64_t)kBktFmax * n : kBktQmax;
     L->bt = off;       off = align256(off + sizeof(int) * (size_t)(qmax + 1));
-    L->tileS = off;    off = align256(off + sizeof(double) * (size_t)ntiles * (size_t)m);
-    // counts: uint8 per 32-row tile (sweep, r01 window, LL, hist, dense) or
-    // uint32 per row block of win_kernel (at most one block per 32 rows)
-    const size_t n32 = (size_t)((n + 31) / 32);
-    const size_t nbytes = (size_t)ntiles > 4 * n32 ? (size_t)ntiles : 4 * n32;
+    // partials: one per 32-row tile (sweep, r01 window, LL, hist, dense; uint8
+    // counts) or one per win_kernel warp slot (uint32 counts)
+    const size_t slots = (size_t)win2_max_slots();
+    L->tileS = off;    off = align256(off + sizeof(double) * ((size_t)ntiles > slots ? (size_t)ntiles : slots) * (size_t)m);
+    const size_t nbytes = (size_t)ntiles > 4 * slots ? (size_t)ntiles : 4 * slots;
     L->tileN = off;    off = align256(off + nbytes * (size_t)m);
     L->tileB = off;    off = align256(off + sizeof(double) * (size_t)((n + 31) / 32) * (size_t)m);  // KDE sum B
     L->partial = off;  off = align256(off + sizeof(double) * (size_t)KR_PARTIAL_LEN(m));
@@ -678,36 +705,40 @@ static bool use_win2()
 }
 
 // Task shape of win_kernel for a shard of `rows` rows: BC bandwidths per
-// chunk (<= kWin2Chunk) and TB tiles of 32 rows per block, chosen so that
-// there are about kWin2TasksPerWarp tasks per resident warp (load balance)
-// with as few partials as that allows.
+// chunk (1 .. kWin2Chunk), so that there are about kWin2TasksPerWarp tasks per
+// warp slot; S = the persistent grid's warp slots.
 struct Win2Shape {
-    int BC, nbc, TB, nblk;
+    int BC, nbc, ntiles, blocks, S;
 };
-constexpr int kWin2TasksPerWarp = 4;
+constexpr int kWin2TasksPerWarp = 8;  // static round-robin: >= 8 tasks per slot keeps the tail short
 
 template <int KERN>
 static Win2Shape win2_shape(int64_t rows, int m)
 {
     Win2Shape w;
-    const int64_t n32 = (rows + 31) / 32;
-    const int64_t warps = (int64_t)dev_info().sms * occupancy((const void *)win_kernel<KERN>, kWin2Threads) * kWin2Warps;
-    const int64_t target = kWin2TasksPerWarp * warps;
-    int64_t bc = (int64_t)m * n32 / (target > 0 ? target : 1);
-    bc = bc < 8 ? 8 : (bc > kWin2Chunk ? kWin2Chunk : bc);
+    w.ntiles = (int)((rows + 31) / 32);
+    const int resident = occupancy((const void *)win_kernel<KERN>, kWin2Threads);
+    const int64_t slots = (int64_t)dev_info().sms * resident * kWin2Warps;
+    const int64_t target = kWin2TasksPerWarp * slots;
+    int64_t bc = (int64_t)m * ((w.ntiles + 1) / 2) / (target > 0 ? target : 1);
+    bc = bc < 1 ? 1 : (bc > kWin2Chunk ? kWin2Chunk : bc);
     if (bc > m) bc = m;
     w.BC = (int)bc;
     w.nbc = (int)((m + bc - 1) / bc);
-    int64_t tb = n32 * w.nbc / (target > 0 ? target : 1);
-    tb = tb < 1 ? 1 : (tb > 16 ? 16 : tb);
-    w.TB = (int)tb;
-    w.nblk = (int)((n32 + tb - 1) / tb);
+    // no more slots than tasks (a slot without a task would leave its partials unwritten)
+    const int64_t tasks = (int64_t)((w.ntiles + 1) / 2) * w.nbc;
+    int64_t blocks = (int64_t)dev_info().sms * resident;
+    if (blocks * kWin2Warps > win2_max_slots()) blocks = win2_max_slots() / kWin2Warps;
+    if (blocks * kWin2Warps > tasks) blocks = tasks / kWin2Warps;
+    if (blocks < 1) blocks = 1;
+    w.blocks = (int)blocks;
+    w.S = (int)blocks * kWin2Warps;
     return w;
 }
 
 template <int KERN>
 static void launch_win2(const double2 *xy, int n, const double *h, int m, int lo, int hi, const Win2Shape &w,
-                        bool build_table, const WsLayout &L, char *ws, double *tileS, uint32_t *tileN, int *counter,
+                        bool build_table, const WsLayout &L, char *ws, double *tileS, uint32_t *tileN,
                         cudaStream_t st)
 {
     const double *xs = reinterpret_cast<const double *>(ws + L.xs) + kPad;
@@ -726,13 +757,9 @@ static void launch_win2(const double2 *xy, int n, const double *h, int m, int lo
         if (blocks > (int64_t)sms * 8) blocks = (int64_t)sms * 8;
         launch_pdl(bkt_fill_kernel, dim3((int)blocks), dim3(kBktFillThreads), 0, st, xs, n, gap, BT, prm);
     }
-    const int resident = occupancy((const void *)win_kernel<KERN>, kWin2Threads);
-    const int64_t tasks = (int64_t)w.nblk * w.nbc;
-    int blocks = (int)((tasks + kWin2Warps - 1) / kWin2Warps);
-    if (blocks > sms * resident) blocks = sms * resident;
-    launch_pdl(win_kernel<KERN>, dim3(blocks), dim3(kWin2Threads), 0, st, xs, xy, P, (int)L.pstride,
-               (const int *)BT, (const BktParams *)prm, h, m, n, lo, hi, w.TB, w.nblk, w.BC, w.nbc, ymax, tileS,
-               tileN, counter);
+    launch_pdl(win_kernel<KERN>, dim3(w.blocks), dim3(kWin2Threads), 0, st, xs, xy, P, (int)L.pstride,
+               (const int *)BT, (const BktParams *)prm, h, m, n, lo, hi, w.ntiles, w.BC, w.nbc, ymax, tileS,
+               tileN);
 }
 
 // Histogram ordering (krcv_hist.cuh): `warps` warps per CTA (as many as the
@@ -948,7 +975,7 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     const int winK = ll ? 1 : win_rows_per_lane(hi - lo);
     const int rows_per_tile = 32 * win_lane_rows(winK);
     const int ntiles = hist ? (int)((hi - lo + 31) / 32)
-                     : win2 ? w2.nblk
+                     : win2 ? (w2.ntiles + 1) / 2  // win_kernel tasks per chunk: tile pairs
                      : prefix ? (int)((hi - lo + rows_per_tile - 1) / rows_per_tile)
                               : dense ? (int)tiles_for(hi - lo, 1)
                                       : (variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G));
@@ -1023,13 +1050,13 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
             const bool table = !reuse_sorted;  // the table depends on xs only
             switch (kernel) {
             case KR_UNIFORM:
-                launch_win2<KR_UNIFORM>(xy, nn, d_h, m, lo, hi, w2, table, L, ws, tileS, tileN32, counter, st);
+                launch_win2<KR_UNIFORM>(xy, nn, d_h, m, lo, hi, w2, table, L, ws, tileS, tileN32, st);
                 break;
             case KR_EPANECHNIKOV:
-                launch_win2<KR_EPANECHNIKOV>(xy, nn, d_h, m, lo, hi, w2, table, L, ws, tileS, tileN32, counter, st);
+                launch_win2<KR_EPANECHNIKOV>(xy, nn, d_h, m, lo, hi, w2, table, L, ws, tileS, tileN32, st);
                 break;
             default:
-                launch_win2<KR_TRIANGULAR>(xy, nn, d_h, m, lo, hi, w2, table, L, ws, tileS, tileN32, counter, st);
+                launch_win2<KR_TRIANGULAR>(xy, nn, d_h, m, lo, hi, w2, table, L, ws, tileS, tileN32, st);
                 break;
             }
             launches += table ? 1 : 0;
@@ -1065,11 +1092,11 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     if (win2)
         launch_pdl(reduce_kernel<uint32_t>, dim3(m < 148 * 8 ? m : 148 * 8), dim3(kReduceThreads), 0, st,
                    (const double *)tileS, (const uint32_t *)(ws + L.tileN), ntiles, m, (const unsigned *)status,
-                   d_partial, fin);
+                   d_partial, fin, w2.S, w2.BC);  // tasks per chunk: tile pairs
     else
         launch_pdl(reduce_kernel<uint8_t>, dim3(m < 148 * 8 ? m : 148 * 8), dim3(kReduceThreads), 0, st,
                    (const double *)tileS, (const uint8_t *)tileN, ntiles, m, (const unsigned *)status, d_partial,
-                   fin);
+                   fin, 0, 0);
     launches += 1;
     prof_mark(4, st);
     g_prof.recorded = g_prof.on;

@@ -135,56 +135,79 @@ __device__ __forceinline__ void moment_terms(double x, double y, double o, dd (&
 }
 
 // Prefix storage.  Nadaraya-Watson moment sets (uniform / Epanechnikov /
-// triangular) are stored as records, array of structures: the hi words of
-// index j at P[j S .. j S + S), the lo words at P[ps S + j S ..], S doubles
-// per record (Epanechnikov 6: y, u, u^2, y u, y u^2, j; triangular 4: y, u,
-// y u, j; uniform 2: y, j -- the last slot is the index j itself as a double,
-// so a window count is a difference of two loaded slots).  One record is one
-// or three 16-byte loads.  The KDE and local-linear sets keep the
-// structure-of-arrays planes (hi of moment k at P + 2k ps, lo at
-// P + (2k+1) ps).
+// triangular) are stored in blocks of kRecBlock indices, each block holding
+// the block's values plane after plane: Epanechnikov planes (y, u) and
+// (u^2, y u) of 16-byte pairs and (y u^2) of doubles -- 40 bytes per index;
+// triangular (y, u) and (y u); uniform (y).  Moment slot k of index j is at
+// double offset  (j / kRecBlock) BS + plane_off(k) + (j % kRecBlock) w(k) + sub(k).
+// A warp whose 32 lanes read 32 consecutive indices loads 512 contiguous
+// bytes per pair plane (4 L1 wavefronts; an array of 40-byte structures would
+// span 10 lines per load), and the planes of one index are a fixed 16 / 32 KB
+// apart: immediate offsets of one address.  The lo words follow the hi words
+// at double offset pk_lo_off(ps).  (No padding: the whole C4 working set --
+// hi records, sorted x, bucket table -- must stay inside the 126 MB L2;
+// profiles/r02f_* measured 12-15 GB of DRAM reads per launch when it did not.)
+// The KDE and local-linear sets keep structure-of-arrays planes (hi of moment
+// k at P + 2k ps, lo at P + (2k+1) ps).
+constexpr int kRecBlock = 1024;
+
 template <int KERN>
 struct PfxRec {
-    static constexpr int S = KERN == KR_EPANECHNIKOV ? 6 : (KERN == KR_TRIANGULAR ? 4 : (KERN == KR_UNIFORM ? 2 : 0));
+    static constexpr int S = KERN == KR_EPANECHNIKOV ? 5 : (KERN == KR_TRIANGULAR ? 3 : (KERN == KR_UNIFORM ? 1 : 0));
+    static constexpr int BS = S * kRecBlock;  // doubles per block (all planes)
+    // plane of slot k: width 2 for slots 0..2*(S/2)-1, width 1 for the odd last slot
+    static __host__ __device__ constexpr int width(int k) { return k < 2 * (S / 2) ? 2 : 1; }
+    static __host__ __device__ constexpr int plane_off(int k) { return (k / 2) * 2 * kRecBlock; }
+    static __host__ __device__ constexpr int sub(int k) { return k < 2 * (S / 2) ? (k & 1) : 0; }
 };
+
+// index slots reserved for prefix stride ps (>= n + 1): whole blocks
+__host__ __device__ __forceinline__ size_t pk_slots(int ps)
+{
+    return ((size_t)ps + kRecBlock - 1) / kRecBlock * kRecBlock;
+}
+
+// doubles of one (hi or lo) record array for prefix stride ps
+template <int KERN>
+__host__ __device__ __forceinline__ size_t pk_lo_off(int ps)
+{
+    return (size_t)PfxRec<KERN>::S * pk_slots(ps);
+}
+
+// double offset of moment slot k of index j (j >= 0): one shift and one
+// 32 x 32 -> 64-bit multiply-add plus constants
+template <int KERN>
+__device__ __forceinline__ size_t pk_off(int k, int j)
+{
+    using R = PfxRec<KERN>;
+    const unsigned u = (unsigned)j;
+    return (size_t)(u >> 10) * (unsigned)R::BS +
+           (size_t)((u & (kRecBlock - 1)) * (unsigned)R::width(k) + (unsigned)(R::plane_off(k) + R::sub(k)));
+}
 
 template <int KERN>
 __device__ __forceinline__ void pk_store(double *__restrict__ P, int ps, int k, int j, dd v)
 {
-    constexpr int S = PfxRec<KERN>::S;
-    if (S) {
-        P[(size_t)j * S + k] = v.hi;
-        P[(size_t)ps * S + (size_t)j * S + k] = v.lo;
+    if (PfxRec<KERN>::S) {
+        P[pk_off<KERN>(k, j)] = v.hi;
+        P[pk_lo_off<KERN>(ps) + pk_off<KERN>(k, j)] = v.lo;
     } else {
         P[(size_t)(2 * k) * ps + j] = v.hi;
         P[(size_t)(2 * k + 1) * ps + j] = v.lo;
     }
 }
 
-// the record's index slot (AoS layouts only)
-template <int KERN>
-__device__ __forceinline__ void pk_store_index(double *__restrict__ P, int ps, int j)
-{
-    constexpr int S = PfxRec<KERN>::S;
-    if (S) {
-        P[(size_t)j * S + S - 1] = (double)j;
-        P[(size_t)ps * S + (size_t)j * S + S - 1] = 0.0;
-    }
-}
-
 template <int KERN>
 __device__ __forceinline__ double pk_hi(const double *__restrict__ P, int ps, int k, int j)
 {
-    constexpr int S = PfxRec<KERN>::S;
-    return S ? P[(size_t)j * S + k] : P[(size_t)(2 * k) * ps + j];
+    return PfxRec<KERN>::S ? P[pk_off<KERN>(k, j)] : P[(size_t)(2 * k) * ps + j];
 }
 
 template <int KERN>
 __device__ __forceinline__ dd pk_dd(const double *__restrict__ P, int ps, int k, int j)
 {
-    constexpr int S = PfxRec<KERN>::S;
-    return S ? dd{P[(size_t)j * S + k], P[(size_t)ps * S + (size_t)j * S + k]}
-             : dd{P[(size_t)(2 * k) * ps + j], P[(size_t)(2 * k + 1) * ps + j]};
+    return PfxRec<KERN>::S ? dd{P[pk_off<KERN>(k, j)], P[pk_lo_off<KERN>(ps) + pk_off<KERN>(k, j)]}
+                           : dd{P[(size_t)(2 * k) * ps + j], P[(size_t)(2 * k + 1) * ps + j]};
 }
 
 template <int KERN>
@@ -364,7 +387,6 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
         for (int q = 0; q < ITEMS; q++) {
             if (j0 + q <= n) {
                 pk_store<KERN>(P, pstride, k, j0 + q, run);
-                if (k == 0) pk_store_index<KERN>(P, pstride, j0 + q);
             }
             run = dd_add(run, tm[q][k]);
         }
@@ -460,12 +482,10 @@ pfx_one_cta_kernel(const double2 *__restrict__ xy, int n, double *__restrict__ P
             pk_store<KERN>(P, pstride, k, j, run[k]);
             run[k] = dd_add(run[k], tm[k]);
         }
-        pk_store_index<KERN>(P, pstride, j);
     }
     if (j1 == n && j0 < n) {  // the thread holding the last record writes P[k][n]
 #pragma unroll
         for (int k = 0; k < K; k++) pk_store<KERN>(P, pstride, k, n, run[k]);
-        pk_store_index<KERN>(P, pstride, n);
     }
 }
 
@@ -579,6 +599,21 @@ __device__ __forceinline__ dd wsum(const double *__restrict__ P, int ps, int k, 
 // denominator (and, for the numerator, of den * max|y|), which bounds the
 // fast path's relative error in den and its absolute error in g_{-i} by
 // kFastTol (times max|y|).  Otherwise the window is recomputed in dd.
+// a / b for finite b != 0 with normal 1/b: hardware reciprocal estimate, two
+// Newton steps and one residual correction -- within 1 ulp of the correctly
+// rounded quotient, branch-free (IEEE division adds a slow-path test).
+__device__ __forceinline__ double fast_div(double a, double b)
+{
+    double r;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(b));
+    double e = fma(-b, r, 1.0);
+    r = fma(r, e, r);
+    e = fma(-b, r, 1.0);
+    r = fma(r, e, r);
+    const double q = a * r;
+    return fma(r, fma(-b, q, a), q);
+}
+
 constexpr double kFastSlack = 16.0 * 0x1p-53;
 constexpr double kFastTol = 0x1p-44;
 
@@ -607,22 +642,26 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
         double sy = (pb - pa) - yr;
         if (!(kFastSlack * (fabs(pb) + fabs(pa) + fabs(yr)) <= kFastTol * (double)c * ymax))
             sy = dd_sub_to_d(pk_wsum<KERN>(P, ps, 0, A, R), dd_make(yr));
-        g = sy / (double)c;
+        g = fast_div(sy, (double)c);
     } else {
         const double hk = (KERN == KR_EPANECHNIKOV) ? h * h : h;
         double sy, s1, sy1, num, den;
         bool fast = false;
         if (KERN == KR_EPANECHNIKOV) {
             // fast path: hi words only, plain double (error test: see kFastTol)
-            // records R and A (PfxRec: y, u, u^2, y u, y u^2, j): three 16-byte loads each
-            const double2 *pr = reinterpret_cast<const double2 *>(P) + (size_t)R * 3;
-            const double2 *pa = reinterpret_cast<const double2 *>(P) + (size_t)A * 3;
-            const double2 r01 = __ldg(pr), r23 = __ldg(pr + 1), r45 = __ldg(pr + 2);
-            const double2 a01 = __ldg(pa), a23 = __ldg(pa + 1), a45 = __ldg(pa + 2);
+            // records R and A (PfxRec planes (y, u), (u^2, y u), (y u^2)): two 16-byte and one
+            // 8-byte load each, fixed offsets from one address
+            const double *pr = P + pk_off<KERN>(0, R);
+            const double *pa = P + pk_off<KERN>(0, A);
+            const double2 r01 = __ldg(reinterpret_cast<const double2 *>(pr));
+            const double2 r23 = __ldg(reinterpret_cast<const double2 *>(pr + 2 * kRecBlock));
+            const double2 a01 = __ldg(reinterpret_cast<const double2 *>(pa));
+            const double2 a23 = __ldg(reinterpret_cast<const double2 *>(pa + 2 * kRecBlock));
+            const double yuu_b = __ldg(pr + 4 * kRecBlock - (int)((unsigned)R & (kRecBlock - 1))),
+                         yuu_a = __ldg(pa + 4 * kRecBlock - (int)((unsigned)A & (kRecBlock - 1)));
             const double y_b = r01.x, y_a = a01.x, u_b = r01.y, u_a = a01.y;
             const double uu_b = r23.x, uu_a = a23.x, yu_b = r23.y, yu_a = a23.y;
-            const double yuu_b = r45.x, yuu_a = a45.x;
-            const double c1 = r45.y - a45.y;  // range count R - A, row r included (its terms vanish); exact
+            const double c1 = (double)(c + 1);  // range count R - A, row r included (its terms vanish)
             const double Sy = y_b - y_a, Su = u_b - u_a, Suu = uu_b - uu_a;
             const double Syu = yu_b - yu_a, Syuu = yuu_b - yuu_a;
             s1 = fma(-dl, fma(-c1, dl, 2.0 * Su), Suu);
@@ -640,11 +679,19 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
         }
         if (!fast) {
             if (KERN == KR_EPANECHNIKOV) {
-                const dd Sy = pk_wsum<KERN>(P, ps, 0, A, R);
-                const dd Su = pk_wsum<KERN>(P, ps, 1, A, R);
-                const dd Suu = pk_wsum<KERN>(P, ps, 2, A, R);
-                const dd Syu = pk_wsum<KERN>(P, ps, 3, A, R);
-                const dd Syuu = pk_wsum<KERN>(P, ps, 4, A, R);
+                // the records' hi and lo words at fixed offsets from two addresses
+                const size_t lo = pk_lo_off<KERN>(ps);
+                const double *pr = P + pk_off<KERN>(0, R), *pa = P + pk_off<KERN>(0, A);
+                const int orr = 4 * kRecBlock - (int)((unsigned)R & (kRecBlock - 1));
+                const int oaa = 4 * kRecBlock - (int)((unsigned)A & (kRecBlock - 1));
+                auto wd = [&](int offr, int offa) {
+                    return dd_sub(dd{pr[offr], pr[lo + offr]}, dd{pa[offa], pa[lo + offa]});
+                };
+                const dd Sy = wd(0, 0);
+                const dd Su = wd(1, 1);
+                const dd Suu = wd(2 * kRecBlock, 2 * kRecBlock);
+                const dd Syu = wd(2 * kRecBlock + 1, 2 * kRecBlock + 1);
+                const dd Syuu = wd(orr, oaa);
                 const dd t1 = dd_sub(dd_twice(Su), dd_mul_d_raw(del, (double)(c + 1)));
                 s1 = dd_sub_to_d(Suu, dd_mul_raw(del, t1));
                 const dd t2 = dd_sub(dd_twice(Syu), dd_mul_raw(del, Sy));
@@ -684,7 +731,7 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
                 den += wt;
             }
         }
-        g = num / den;
+        g = fast_div(num, den);
     }
     const double e = yr - g;
     return e * e;

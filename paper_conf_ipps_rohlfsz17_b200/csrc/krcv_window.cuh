@@ -26,18 +26,13 @@
 // buckets), so the hint never decides an index, only how fast it is found.
 // Q = F n with F = 2^k chosen per call from the data's peak density (the
 // smallest x-span of kGapSpan + 1 sorted records, krcv_prefix.cuh), so the
-// densest region still averages about half a point per bucket (F <= kBktFmax).
+// densest region still averages at most one point per bucket (F <= kBktFmax).
 // Sides whose window reaches the end of the data (x_max - x_r < h, resp.
 // x_r - x_min < h) take R = n (A = 0) with no lookup at all.
 //
-// Every (row, bandwidth) is independent, so a warp task is a block of TB
-// tiles of 32 consecutive sorted rows (lane = row, coalesced loads) times a
-// chunk of <= 64 bandwidths; per (tile, bandwidth) the warp's squared errors
-// are summed by a fixed butterfly and lane (b - b0) mod 32 accumulates the
-// chunk's sums over the TB tiles in registers.  One partial per (block,
-// bandwidth) -- TB times fewer than one per tile (the tile
-// partials were 6x the algorithmic DRAM bytes at C4) -- written once,
-// reduced in a fixed order by reduce_kernel: bit-reproducible.
+// Every (row, bandwidth) is independent, so a warp task is a tile of 32
+// consecutive sorted rows (lane = row, coalesced loads) times a chunk of <= 32
+// bandwidths, scheduled on persistent warp slots (see win_kernel).
 #pragma once
 
 #include <cuda_runtime.h>
@@ -54,7 +49,7 @@ constexpr int kBktFmax = 32;             // buckets per point, at most
 constexpr int64_t kBktQmax = 1LL << 28;  // buckets, at most
 constexpr double kBktMagic = 6755399441055744.0;  // 1.5 * 2^52: fma(.) + magic keeps the integer in the low word
 constexpr int kBktFillThreads = 256;
-constexpr int kBktSeg = 16;              // merge-path items per thread of the table fill
+constexpr int kBktSeg = 8;               // merge-path items per thread of the table fill (more threads: the diagonal searches are latency-bound)
 
 // Table parameters, written by bkt_fill_kernel's first thread, read by the
 // window kernel (both compute them from the same inputs).
@@ -80,9 +75,11 @@ __device__ __forceinline__ BktParams bkt_params(const double *__restrict__ xs, i
     int F = 1;
     if (gb != 0ull && span > 0.0) {
         const double gap = __longlong_as_double((long long)~gb);  // min x-span of kGapSpan + 1 records
-        // ratio of the peak density kGapSpan / gap to the mean (n - 1) / span,
-        // times 2: about half a point per bucket where the data is densest
-        const double ratio = gap > 0.0 ? 2.0 * (double)kGapSpan * span / (gap * (double)(n - 1)) : 1e300;
+        // ratio of the peak density kGapSpan / gap to the mean (n - 1) / span:
+        // F = the next power of two, at most one point per bucket where the data
+        // is densest (uniform x: F = 2; a larger table costs L2 capacity, which
+        // the C4 working set needs -- profiles/r02f_*)
+        const double ratio = gap > 0.0 ? (double)kGapSpan * span / (gap * (double)(n - 1)) : 1e300;
         while (F < kBktFmax && (double)F < ratio) F <<= 1;
     }
     int64_t Q = (int64_t)F * n;
@@ -178,86 +175,132 @@ __device__ __forceinline__ int first_true(Pred p, int lo, int hi, int k0)
 
 constexpr int kWin2Warps = 4;
 constexpr int kWin2Threads = kWin2Warps * 32;
-constexpr int kWin2Chunk = 64;  // bandwidths per task, at most (two accumulators per lane)
+constexpr int kWin2Chunk = 32;  // bandwidths per task, at most (lane (b - b0) keeps bandwidth b's running sum)
+// CTAs per SM the register allocation must allow: 8 -> 64 registers, 32
+// warps per SM (measured faster than 6 -> 80 and 4 -> 128 registers: the
+// kernel is latency-bound, profiles/r02d_*, r02e_*).  KRCV_WIN2_MINB at build
+// time overrides (tuning runs).
+#ifndef KRCV_WIN2_MINB
+#define KRCV_WIN2_MINB 8
+#endif
+constexpr int kWin2MinBlocks = KRCV_WIN2_MINB;
 
-// task = (block of TB tiles of 32 sorted rows, chunk of <= 64 bandwidths),
-// chunk-major so that concurrently running warps hold adjacent blocks at the
-// same bandwidths.  Output: tileS[b][blk], tileN[b][blk] (blk = block index).
+// Schedule.  Task k = (chunk c = k / npairs of <= 32 bandwidths, tile pair
+// t = k % npairs: 64 consecutive sorted rows, two per lane), chunk-major.  The grid is
+// persistent: S = gridDim.x * kWin2Warps warp slots, slot s runs tasks s, s + S,
+// s + 2S, ... (static, no atomics).  So the tasks in flight at any moment are S
+// consecutive tiles of one chunk -- a band of 32 S rows whose windows at
+// nearby bandwidths touch a band of the sorted arrays that stays in L2 (an
+// earlier schedule with every row block in flight touched the whole array per
+// bandwidth and read 7-12 GB from DRAM per C4 launch, profiles/r02f_*,
+// r02g_*).  Per (tile, bandwidth) the squared errors are summed by a fixed
+// butterfly and lane b - b0 adds the sum to the slot's running sum for b over
+// the slot's consecutive tasks of the same chunk; the sum is written once per
+// (slot, chunk) to tileS[b][s] (tileN likewise).  reduce_slots_kernel adds the
+// slots of each bandwidth in slot order: bit-reproducible, and S m partials
+// instead of one per (tile, bandwidth) (the per-tile partials
+// were 6x the algorithmic DRAM bytes at C4).
+// No shared memory: the probes and prefix records live in L1, and shared
+// memory a CTA reserves is taken from the L1 carve-out (a shared-memory batch
+// reduction measured 12% slower at C4 for that reason, profiles/r02e_*).
+// Squared LOO error of one row at bandwidth h (0 if the row is invalid or has
+// an empty window, reading Q6), M through *M.
 template <int KERN>
-__global__ void __launch_bounds__(kWin2Threads)
+__device__ __forceinline__ double row_e2(const WinRow &w, bool valid, double dmax, double dmin, double h,
+                                         const double *__restrict__ xs, const double2 *__restrict__ xy,
+                                         const double *__restrict__ P, int pstride, const int *__restrict__ BT,
+                                         double invw, double C, int Q, int n, double ymax, bool &M)
+{
+    const int r = w.r;
+    const double xr = w.xr;
+    int R = n, A = 0;
+    if (!inside<KERN>(dmax, h)) {  // window ends inside the data: look R up
+        const int k0 = __ldg(BT + min(max(bkt_raw(xr + h, invw, C), 0), Q));
+        R = first_true([&](int q) { return !inside<KERN>(__ldg(xs + q) - xr, h); }, r + 1, n, k0);
+    }
+    if (!inside<KERN>(dmin, h)) {
+        const int k0 = __ldg(BT + min(max(bkt_raw(xr - h, invw, C), 0), Q));
+        A = first_true([&](int q) { return inside<KERN>(xr - __ldg(xs + q), h); }, 0, r, k0);
+    }
+    const int c = R - A - 1;
+    M = valid && c > 0;  // reading Q6
+    return M ? window_e2<KERN>(w, A, R, c, h, xy, P, pstride, ymax) : 0.0;
+}
+
+template <int KERN>
+__global__ void __launch_bounds__(kWin2Threads, kWin2MinBlocks)
 win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P, int pstride,
            const int *__restrict__ BT, const BktParams *__restrict__ prm, const double *__restrict__ hg, int m,
-           int n, int row_lo, int row_hi, int TB, int nblk, int BC, int nbc,
+           int n, int row_lo, int row_hi, int ntiles, int BC, int nbc,
            const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
-           uint32_t *__restrict__ tileN, int *__restrict__ task_counter)
+           uint32_t *__restrict__ tileN)
 {
     pdl_wait();  // krcv_pdl.cuh
     const int lane = threadIdx.x & 31;
+    const int S = gridDim.x * kWin2Warps;
+    const int slot = blockIdx.x * kWin2Warps + (threadIdx.x >> 5);
     const double o = pfx_origin(xy, n);
     const double ymax = __longlong_as_double((long long)*ymax_bits);
     const double xmin = xs[0], xmax = xs[n - 1];
     const double invw = prm->invw, C = prm->C;
     const int Q = prm->Q;
-    const int ntasks = nblk * nbc;
-    for (;;) {
-        int task = 0;
-        if (lane == 0) task = atomicAdd(task_counter, 1);
-        task = __shfl_sync(0xffffffffu, task, 0);
-        if (task >= ntasks) return;  // warp-uniform
-        const int chunk = task / nblk;
-        const int blk = task - chunk * nblk;
-        const int b0 = chunk * BC, b1 = min(m, b0 + BC);
-        double acc0 = 0.0, acc1 = 0.0;
-        uint32_t cnt0 = 0, cnt1 = 0;
-        for (int t = 0; t < TB; t++) {
-            const int base = row_lo + (blk * TB + t) * 32;
-            if (base >= row_hi) break;  // warp-uniform
-            const int i = base + lane;
-            const bool valid = i < row_hi;
-            WinRow w;
-            w.r = valid ? i : row_hi - 1;  // clamped rows do identical work, discarded
-            const double2 v = xy[w.r];
-            w.xr = v.x;
-            w.yr = v.y;
-            w.del = two_sum(v.x, -o);  // exact x_r - o
-            const int r = w.r;
-            const double xr = w.xr;
-            const double dmax = xmax - xr, dmin = xr - xmin;
-            for (int b = b0; b < b1; b++) {
-                const double h = __ldg(hg + b);
-                int R = n, A = 0;
-                if (!inside<KERN>(dmax, h)) {  // window ends inside the data: look R up
-                    const int k0 = __ldg(BT + min(max(bkt_raw(xr + h, invw, C), 0), Q));
-                    R = first_true([&](int k) { return !inside<KERN>(__ldg(xs + k) - xr, h); }, r + 1, n, k0);
-                }
-                if (!inside<KERN>(dmin, h)) {
-                    const int k0 = __ldg(BT + min(max(bkt_raw(xr - h, invw, C), 0), Q));
-                    A = first_true([&](int k) { return inside<KERN>(xr - __ldg(xs + k), h); }, 0, r, k0);
-                }
-                const int c = R - A - 1;
-                const bool M = valid && c > 0;  // reading Q6
-                double e2 = M ? window_e2<KERN>(w, A, R, c, h, xy, P, pstride, ymax) : 0.0;
-                e2 = warp_sum(e2);  // fixed butterfly: every lane holds the tile's sum
-                const uint32_t nb = __popc(__ballot_sync(0xffffffffu, M));
-                const int bl = b - b0;
-                if (lane == (bl & 31)) {
-                    if (bl < 32) {
-                        acc0 += e2;
-                        cnt0 += nb;
-                    } else {
-                        acc1 += e2;
-                        cnt1 += nb;
-                    }
-                }
+    // a task is a pair of adjacent tiles (64 rows): two rows per lane share
+    // one butterfly per bandwidth
+    const int npairs = (ntiles + 1) / 2;
+    const int64_t ntasks = (int64_t)npairs * nbc;
+    int cur = -1;  // chunk of the running sums
+    double acc = 0.0;
+    uint32_t cnt = 0;
+    for (int64_t k = slot;; k += S) {
+        const int chunk = k < ntasks ? (int)(k / npairs) : nbc;  // warp-uniform
+        if (chunk != cur) {  // flush the previous chunk's sums, start the next
+            if (cur >= 0 && cur * BC + lane < min(m, (cur + 1) * BC)) {
+                tileS[(size_t)(cur * BC + lane) * S + slot] = acc;
+                tileN[(size_t)(cur * BC + lane) * S + slot] = cnt;
             }
+            if (chunk >= nbc) return;
+            cur = chunk;
+            acc = 0.0;
+            cnt = 0;
         }
-        if (b0 + lane < b1) {
-            tileS[(size_t)(b0 + lane) * nblk + blk] = acc0;
-            tileN[(size_t)(b0 + lane) * nblk + blk] = cnt0;
+        const int t = (int)(k - (int64_t)chunk * npairs);
+        const int b0 = chunk * BC, b1 = min(m, b0 + BC);
+        WinRow w0, w1;
+        bool v0, v1;
+        double dmax0, dmin0, dmax1, dmin1;
+        {
+            const int i = row_lo + t * 64 + lane;
+            v0 = i < row_hi;
+            w0.r = v0 ? i : row_hi - 1;  // clamped rows do identical work, discarded
+            const double2 v = xy[w0.r];
+            w0.xr = v.x;
+            w0.yr = v.y;
+            w0.del = two_sum(v.x, -o);  // exact x_r - o
+            dmax0 = xmax - v.x;
+            dmin0 = v.x - xmin;
         }
-        if (b0 + 32 + lane < b1) {
-            tileS[(size_t)(b0 + 32 + lane) * nblk + blk] = acc1;
-            tileN[(size_t)(b0 + 32 + lane) * nblk + blk] = cnt1;
+        {
+            const int i = row_lo + t * 64 + 32 + lane;
+            v1 = i < row_hi;
+            w1.r = v1 ? i : row_hi - 1;
+            const double2 v = xy[w1.r];
+            w1.xr = v.x;
+            w1.yr = v.y;
+            w1.del = two_sum(v.x, -o);
+            dmax1 = xmax - v.x;
+            dmin1 = v.x - xmin;
+        }
+        for (int b = b0; b < b1; b++) {
+            const double h = __ldg(hg + b);
+            bool M0, M1;
+            double e2 = row_e2<KERN>(w0, v0, dmax0, dmin0, h, xs, xy, P, pstride, BT, invw, C, Q, n, ymax, M0);
+            e2 += row_e2<KERN>(w1, v1, dmax1, dmin1, h, xs, xy, P, pstride, BT, invw, C, Q, n, ymax, M1);
+            e2 = warp_sum(e2);  // fixed butterfly: every lane holds the pair's sum
+            const uint32_t nb = __popc(__ballot_sync(0xffffffffu, M0)) + __popc(__ballot_sync(0xffffffffu, M1));
+            if (lane == b - b0) {
+                acc += e2;
+                cnt += nb;
+            }
         }
     }
 }
