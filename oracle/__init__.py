@@ -18,6 +18,12 @@ Contents
                      PAPER.md P@15728, reading Q25), O(n^2 m), long double.
 * ``exact.ll_cv_exact``     -- Python ``fractions`` brute force of the
                                local-linear normal equations.
+* ``nw_jackknife`` / ``kde_jackknife`` -- C, leave-one-out (delete-one
+                     jackknife) confidence intervals at a bandwidth (PAPER.md
+                     P@10560, reading Q26), plain definitions, long double;
+                     ``cv_ci`` / ``kde_ci`` run them at the CV / LSCV optimum.
+* ``exact.nw_jackknife_exact`` / ``exact.kde_jackknife_exact`` -- Python
+                     ``fractions``: the jackknife by explicit deletion.
 * ``sorted_rows``           -- the x-sorted row order (stable by (x, index))
                                that defines shards.
 
@@ -68,6 +74,10 @@ def _lib(precision: str = "ld") -> ctypes.CDLL:
     lib.kro_kde_lscv.restype = ctypes.c_int
     lib.kro_ll_cv.argtypes = [P, P, i64, P, i32, i32, P, i64, P, P, P, P]
     lib.kro_ll_cv.restype = ctypes.c_int
+    lib.kro_nw_jackknife.argtypes = [P, P, i64, ctypes.c_double, i32, P, P, P]
+    lib.kro_nw_jackknife.restype = ctypes.c_int
+    lib.kro_kde_jackknife.argtypes = [P, i64, ctypes.c_double, i32, P, P]
+    lib.kro_kde_jackknife.restype = ctypes.c_int
     lib.kro_real_bits.restype = ctypes.c_int
     lib.kro_num_threads.restype = ctypes.c_int
     _libs[precision] = lib
@@ -248,3 +258,50 @@ def ll_cv(x, y, h, kernel: int, rows=None, precision: str = "ld") -> Result:
     if st:
         raise OracleError(st)
     return Result(cv=cv, best=int(best.value), S=S, neff=ne)
+
+
+def nw_jackknife(x, y, h: float, kernel: int, precision: str = "ld") -> Result:
+    """Delete-one jackknife interval pieces for the Nadaraya-Watson estimate at
+    every observation at bandwidth h (reading Q26): est[n] (full-sample
+    estimate, the point itself included), se[n] (NaN where the window holds
+    only the point), nwin[n] (window sizes)."""
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    y = np.ascontiguousarray(y, dtype=np.float64)
+    n = x.shape[0]
+    est, se, nw = np.empty(n), np.empty(n), np.empty(n, np.int64)
+    st = _lib(precision).kro_nw_jackknife(x.ctypes.data, y.ctypes.data, n, float(h), int(kernel),
+                                          est.ctypes.data, se.ctypes.data, nw.ctypes.data)
+    if st:
+        raise OracleError(st)
+    return Result(est=est, se=se, nwin=nw)
+
+
+def kde_jackknife(x, h: float, kernel: int, precision: str = "ld") -> Result:
+    """Delete-one jackknife interval pieces for the kernel density estimate at
+    every observation at bandwidth h (reading Q26): est[n] = f_h(x_i), se[n]."""
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    n = x.shape[0]
+    est, se = np.empty(n), np.empty(n)
+    st = _lib(precision).kro_kde_jackknife(x.ctypes.data, n, float(h), int(kernel), est.ctypes.data,
+                                           se.ctypes.data)
+    if st:
+        raise OracleError(st)
+    return Result(est=est, se=se)
+
+
+def cv_ci(x, y, h, kernel: int) -> Result:
+    """The CV-optimal bandwidth (Program 3, cv_sorted) and the jackknife
+    interval pieces there (reading Q26): best, h_best, est, se, nwin."""
+    r = cv_sorted(x, y, h, kernel)
+    hb = float(np.asarray(h, dtype=np.float64)[r.best])
+    j = nw_jackknife(x, y, hb, kernel)
+    return Result(best=r.best, h_best=hb, est=j.est, se=j.se, nwin=j.nwin)
+
+
+def kde_ci(x, h, kernel: int) -> Result:
+    """The LSCV-optimal bandwidth (kde_lscv) and the jackknife interval pieces
+    of the density estimate there (reading Q26): best, h_best, est, se."""
+    r = kde_lscv(x, h, kernel)
+    hb = float(np.asarray(h, dtype=np.float64)[r.best])
+    j = kde_jackknife(x, hb, kernel)
+    return Result(best=r.best, h_best=hb, est=j.est, se=j.se)

@@ -144,3 +144,69 @@ def ll_cv_exact(x, y, h, kernel: int):
         neffs.append(ne)
     best = min(range(len(cvs)), key=lambda b: (cvs[b], b))
     return cvs, neffs, best
+
+
+def _window(xs, i, l, hb, kernel):
+    d64 = abs(xs[l] - xs[i])
+    return d64 <= hb if kernel == UNIFORM else d64 < hb
+
+
+def nw_jackknife_exact(x, y, hb: float, kernel: int):
+    """Reading Q26 in exact rationals, by explicit deletion: for each point i,
+    g_i = the Nadaraya-Watson estimate at x_i from the whole sample (i
+    included), and for every j = 0..n-1 the estimate g_i^(-j) from the sample
+    WITHOUT observation j, recomputed from scratch; the jackknife variance
+    (n-1)/n sum_j (g_i^(-j) - mean_j g_i^(-j))^2.  No algebraic shortcut (the
+    oracle's Delta_j form is what this checks).  Returns (est list, var list);
+    var is None where some deletion empties the window."""
+    xs = [float(v) for v in x]
+    ys = [Fraction(float(v)) for v in y]
+    n = len(xs)
+    H = Fraction(float(hb))
+
+    def estimate(i, skip):
+        num = den = Fraction(0)
+        for l in range(n):
+            if l == skip or not _window(xs, i, l, float(hb), kernel):
+                continue
+            w = _K(abs(Fraction(xs[l]) - Fraction(xs[i])) / H, kernel)
+            num += w * ys[l]
+            den += w
+        return None if den == 0 else num / den
+
+    est, var = [], []
+    for i in range(n):
+        est.append(estimate(i, -1))
+        dels = [estimate(i, j) for j in range(n)]
+        if any(v is None for v in dels):
+            var.append(None)
+            continue
+        mean = sum(dels) / n
+        var.append(Fraction(n - 1, n) * sum((v - mean) ** 2 for v in dels))
+    return est, var
+
+
+def kde_jackknife_exact(x, hb: float, kernel: int):
+    """Reading Q26 for the density, in exact rationals by explicit deletion:
+    f_i = (1/(n h)) sum_j K(d_ij/h) with Q24's normalised kernels, the
+    delete-one estimates f_i^(-j) = (1/((n-1) h)) sum_{l != j} K(d_il/h)
+    recomputed from scratch, and their jackknife variance.  Returns
+    (est list, var list)."""
+    xs = [float(v) for v in x]
+    n = len(xs)
+    H = Fraction(float(hb))
+
+    def k(i, l):
+        if not _window(xs, i, l, float(hb), kernel):
+            return Fraction(0)
+        return _K(abs(Fraction(xs[l]) - Fraction(xs[i])) / H, kernel)
+
+    est, var = [], []
+    for i in range(n):
+        kk = [k(i, l) for l in range(n)]
+        tot = sum(kk)
+        est.append(tot / (n * H))
+        dels = [(tot - kk[j]) / ((n - 1) * H) for j in range(n)]
+        mean = sum(dels) / n
+        var.append(Fraction(n - 1, n) * sum((v - mean) ** 2 for v in dels))
+    return est, var

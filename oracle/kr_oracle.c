@@ -581,3 +581,106 @@ int kro_ll_cv(const double *x, const double *y, int64_t n, const double *h, int3
     free(S); free(ne);
     return KRO_OK;
 }
+
+/* ------------------------------------------------------------------ */
+/* Leave-one-out (delete-one jackknife) confidence intervals at a given */
+/* bandwidth -- the CV-optimal one in use (§II P@10560-10640:  */
+/* "the estimation of leave-one-out cross-validated confidence          */
+/* intervals for kernel density estimates and kernel regressions";      */
+/* SURVEY.md §8(f) rank 3; reading Q26).                     */
+/*                                                                      */
+/* Kernel regression (Nadaraya-Watson, Eq.(2) with the point itself):   */
+/*   W+_i = { j : d_ij in the window (Q1) }  (i itself included, d = 0) */
+/*   w_ij = K(d_ij / h) (Eq.(3), Q13), D_i = sum w_ij,                  */
+/*   N_i = sum w_ij Y_j, g_i = N_i / D_i                                */
+/*   delete-one estimates g_i^(-j) = (N_i - w_ij Y_j) / (D_i - w_ij)    */
+/*   (= g_i for j outside W+_i), jackknife variance                     */
+/*   V_i = (n-1)/n sum_j (g_i^(-j) - mean_j g_i^(-j))^2                 */
+/* written with Delta_j = g_i^(-j) - g_i = -w_ij (Y_j - g_i)/(D_i-w_ij) */
+/* (zero outside W+_i) as                                               */
+/*   V_i = (n-1)/n [ sum Delta_j^2 - (sum Delta_j)^2 / n ].             */
+/* A point whose window holds only itself has no delete-one estimate at */
+/* j = i: its se is NaN (no interval).  Output in the caller's order.   */
+/*                                                                      */
+/* Kernel density (Q24's normalised kernels):                           */
+/*   K_ij = K(d_ij / h) / h on K's window, f_i = (1/n) sum_j K_ij       */
+/*   delete-one f_i^(-j) = (n f_i - K_ij)/(n-1); its jackknife variance */
+/*   reduces to the sample variance of the K_ij over j = 0..n-1:        */
+/*   V_i = sum_j (K_ij - f_i)^2 / (n (n-1))                             */
+/*       = [ sum_{W+} (K_ij - f_i)^2 + (n - |W+_i|) f_i^2 ] / (n(n-1)). */
+/* The interval is est_i -+ z se_i, se_i = sqrt(V_i) (z from the        */
+/* caller's level).  Both: the plain definitions, O(n) per point.       */
+/* ------------------------------------------------------------------ */
+int kro_nw_jackknife(const double *x, const double *y, int64_t n, double h, int32_t kernel,
+                     double *est_out, double *se_out, int64_t *nwin_out)
+{
+    if (!x || !y || !est_out || !se_out || n < 2) return KRO_EARG;
+    if (kernel != KRO_UNIFORM && kernel != KRO_EPANECHNIKOV && kernel != KRO_TRIANGULAR) return KRO_EKERNEL;
+    if (!isfinite(h) || !(h > 0.0)) return KRO_EGRID;
+    for (int64_t i = 0; i < n; i++)
+        if (!isfinite(x[i]) || !isfinite(y[i])) return KRO_ENONFINITE;
+    const real nn = (real)n;
+#pragma omp parallel for schedule(dynamic, 64)
+    for (int64_t i = 0; i < n; i++) {
+        real D = 0, N = 0;
+        int64_t c = 0;
+        for (int64_t j = 0; j < n; j++) {
+            double d = fabs(x[j] - x[i]);
+            if (!in_window(d, h, kernel)) continue;
+            real w = kernel_K(d, h, kernel);
+            D += w;
+            N += w * (real)y[j];
+            c++;
+        }
+        real g = N / D;
+        real s1 = 0, s2 = 0;
+        int ok = 1;
+        for (int64_t j = 0; j < n; j++) {
+            double d = fabs(x[j] - x[i]);
+            if (!in_window(d, h, kernel)) continue;
+            real w = kernel_K(d, h, kernel);
+            real rest = D - w;
+            if (!(rest > 0)) { ok = 0; break; }
+            real delta = -w * ((real)y[j] - g) / rest;
+            s1 += delta;
+            s2 += delta * delta;
+        }
+        est_out[i] = (double)g;
+        se_out[i] = ok ? (double)sqrtl((nn - 1) / nn * (s2 - s1 * s1 / nn)) : NAN;
+        if (nwin_out) nwin_out[i] = c;
+    }
+    return KRO_OK;
+}
+
+int kro_kde_jackknife(const double *x, int64_t n, double h, int32_t kernel, double *est_out, double *se_out)
+{
+    if (!x || !est_out || !se_out || n < 2) return KRO_EARG;
+    if (kernel != KRO_UNIFORM && kernel != KRO_EPANECHNIKOV && kernel != KRO_TRIANGULAR) return KRO_EKERNEL;
+    if (!isfinite(h) || !(h > 0.0)) return KRO_EGRID;
+    for (int64_t i = 0; i < n; i++)
+        if (!isfinite(x[i])) return KRO_ENONFINITE;
+    const real nn = (real)n, hh = (real)h;
+#pragma omp parallel for schedule(dynamic, 64)
+    for (int64_t i = 0; i < n; i++) {
+        real S = 0;
+        int64_t c = 0;
+        for (int64_t j = 0; j < n; j++) {
+            double d = fabs(x[j] - x[i]);
+            if (!in_window(d, h, kernel)) continue;
+            S += kde_k((real)d / hh, kernel) / hh;
+            c++;
+        }
+        real f = S / nn;
+        real q = 0;
+        for (int64_t j = 0; j < n; j++) {
+            double d = fabs(x[j] - x[i]);
+            if (!in_window(d, h, kernel)) continue;
+            real t = kde_k((real)d / hh, kernel) / hh - f;
+            q += t * t;
+        }
+        q += (nn - (real)c) * f * f;
+        est_out[i] = (double)f;
+        se_out[i] = (double)sqrtl(q / (nn * (nn - 1)));
+    }
+    return KRO_OK;
+}

@@ -3,10 +3,13 @@ bench.py times (GridSearch(graph=True): one CUDA-graph replay of the whole
 search on device-resident x, y): every CV(h_b) of C1-C5, seeds 0-2, against
 the oracle's curves in tests/golden/curves/ (written by
 tools/make_reference_curves.py, which calls only oracle/: the Program-3
-evaluator for C1/C2, the oracle's window checker for C3-C5).  Bar
-(north_star): relative error <= 1e-6 with the SURVEY §8(c) floor (measured
-~1e-14), n_eff identical, best identical unless the reference's two best
-values lie within 1e-6.  Also the bench's second plan (stage events in the
+evaluator kro_cv_sorted for C1, C2, C3 and C5, the oracle's window checker for
+C4, whose Program-3 run would take ~1.4e5 core-seconds).  Bar (north_star):
+relative error <= 1e-6 with the SURVEY §8(c) floor, n_eff identical, best
+identical unless the reference's two best values lie within 1e-6; against a
+Program-3 curve the test also asserts 1e-10 (measured ~1e-14), so an error
+the size of the window checker's own (6.7e-10 at C5, stored beside the
+Program-3 curve) would fail it.  Also the bench's second plan (stage events in the
 graph) and the host API give the same curve."""
 from __future__ import annotations
 
@@ -43,5 +46,7 @@ def test_full_size_curve_in_bench_launch_config(path):
     err = cv_rel_err(cv, ref["cv"])
     print(f"{cfg} seed {seed}: max rel err {err:.3g}, best {res.best} (ref {int(ref['best'])})")
     assert err <= 1e-6
+    if "kro_cv_sorted" in str(ref["evaluator"]):
+        assert err <= 1e-10, err
     assert np.array_equal(neff, ref["neff"])
     assert best_ok(res.best, ref["cv"], 1e-6)
