@@ -314,6 +314,49 @@ int kr_finalize_async(const double *d_partial, int64_t n, int32_t m,
  */
 int kr_default_grid(const double *x, int64_t n, int32_t m, double *h_out);
 
+/*
+ * Leave-one-out cross-validated confidence intervals (§II
+ * P@10560-10640: "the estimation of leave-one-out cross-validated confidence
+ * intervals for kernel density estimates and kernel regressions"; reading
+ * Q26).  Each call runs the grid search first (kr_cv_grid /
+ * kr_kde_lscv semantics, same outputs), then at the optimal bandwidth
+ * h* = h_grid[best] computes for every observation i (outputs in the caller's
+ * order):
+ *   kr_cv_ci : est_out[i] = g(x_i), the Nadaraya-Watson estimate from the whole
+ *              sample (x_i itself included, Eq.(2) with l = i allowed), and
+ *              se_out[i] = the delete-one jackknife standard error
+ *              sqrt((n-1)/n sum_j (g^(-j)(x_i) - mean_j g^(-j)(x_i))^2),
+ *              g^(-j) the estimate without observation j -- NaN when the
+ *              window of x_i holds only x_i (no estimate without it);
+ *   kr_kde_ci: est_out[i] = f(x_i) = (1/(n h*)) sum_j K((x_i - x_j)/h*)
+ *              (Q24's normalised kernels), se_out[i] its jackknife standard
+ *              error, which is the sample standard deviation of the terms
+ *              K((x_i - x_j)/h*)/h* over j divided by sqrt(n).
+ * The (1 - alpha) interval is est_i -+ z_{1-alpha/2} se_i (the caller's z).
+ * Kernels: uniform, Epanechnikov, triangular (the window is compact).
+ * Host pointers, synchronous, current CUDA device.  cv_out / lscv_out [m]
+ * (the curve of the search), est_out, se_out [n], best_out.
+ * Errors: as kr_cv_grid / kr_kde_lscv; KR_EKERNEL for the Gaussian.
+ */
+int kr_cv_ci(const double *x, const double *y, int64_t n, const double *h_grid, int32_t m, int32_t kernel,
+             double *cv_out, double *est_out, double *se_out, int32_t *best_out);
+int kr_kde_ci(const double *x, int64_t n, const double *h_grid, int32_t m, int32_t kernel,
+              double *lscv_out, double *est_out, double *se_out, int32_t *best_out);
+
+/*
+ * Device-pointer forms, enqueued on cuda_stream (no host synchronisation:
+ * h* is read on the device from the search's best index).  Workspace as
+ * kr_cv_grid_async (kr_workspace_bytes(n, m)).  d_cv / d_lscv [m],
+ * d_est, d_se [n] fp64, d_best_status [2] int32 {best, status}: read after
+ * the stream work completes; est/se are meaningful only if status == KR_OK.
+ */
+int kr_cv_ci_async(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m, int32_t kernel,
+                   double *d_cv, double *d_est, double *d_se, int32_t *d_best_status,
+                   void *d_workspace, size_t workspace_bytes, void *cuda_stream);
+int kr_kde_ci_async(const double *d_x, int64_t n, const double *d_h, int32_t m, int32_t kernel,
+                    double *d_lscv, double *d_est, double *d_se, int32_t *d_best_status,
+                    void *d_workspace, size_t workspace_bytes, void *cuda_stream);
+
 /* Static message for a status code (never NULL). */
 const char *kr_strerror(int status);
 

@@ -9,6 +9,7 @@ from .krcv import (  # noqa: F401
     EPANECHNIKOV, TRIANGULAR, UNIFORM, KERNELS, KrcvError,
     kr_cv_grid, kr_cv_shard_async, kr_default_grid, kr_finalize, kr_finalize_async,
     kr_strerror, kr_validate_grid, kr_version, kr_workspace_bytes,
+    kr_cv_ci, kr_kde_ci, confidence_intervals,
 )
 from .api import CVResult, GridSearch, cv_grid  # noqa: F401
 

@@ -35,6 +35,7 @@
 #include "krcv_sort.cuh"
 #include "krcv_prefix.cuh"
 #include "krcv_window.cuh"
+#include "krcv_ci.cuh"
 #include "krcv_dense.cuh"
 #include "krcv_kde.cuh"
 #include "krcv_ll.cuh"
@@ -1306,4 +1307,62 @@ extern "C" int kr_kde_shard_async(const double *d_x, int64_t n, const double *d_
     KdeFin fin{};
     return enqueue_kde(d_x, n, d_h, m, kernel, shard, nshards, d_partial, fin, d_workspace, workspace_bytes,
                        cuda_stream);
+}
+
+// ---------------------------------------------------------------------------
+// Leave-one-out (jackknife) confidence intervals at the CV-optimal bandwidth
+// (krcv_ci.cuh; reading Q26): the grid search, then one launch reading best
+// on the device.
+// ---------------------------------------------------------------------------
+template <bool KDE>
+static int enqueue_ci(int64_t n, const double *d_h, int32_t kernel, double *d_est, double *d_se,
+                      const int32_t *d_best_status, void *d_workspace, int32_t m, void *cuda_stream)
+{
+    WsLayout L;
+    if (!ws_layout(n, m, &L)) return KR_ECUDA;
+    char *ws = static_cast<char *>(d_workspace);
+    const double2 *xy = reinterpret_cast<const double2 *>(ws + L.xy) + kPad;
+    const uint32_t *perm = reinterpret_cast<const uint32_t *>(ws + L.perm);
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    const dim3 grid((unsigned)((n + kCiThreads - 1) / kCiThreads)), block(kCiThreads);
+    const int nn = (int)n;
+    switch (kernel) {
+    case KR_UNIFORM:
+        launch_pdl(ci_kernel<KR_UNIFORM, KDE>, grid, block, 0, st, xy, perm, nn, d_h, d_best_status, d_est, d_se);
+        break;
+    case KR_EPANECHNIKOV:
+        launch_pdl(ci_kernel<KR_EPANECHNIKOV, KDE>, grid, block, 0, st, xy, perm, nn, d_h, d_best_status, d_est,
+                   d_se);
+        break;
+    default:
+        launch_pdl(ci_kernel<KR_TRIANGULAR, KDE>, grid, block, 0, st, xy, perm, nn, d_h, d_best_status, d_est, d_se);
+        break;
+    }
+    g_prof.launches += 1;
+    const cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) { set_cuda_error("ci_kernel launch", (int)e); return KR_ECUDA; }
+    return KR_OK;
+}
+
+extern "C" int kr_cv_ci_async(const double *d_x, const double *d_y, int64_t n, const double *d_h, int32_t m,
+                              int32_t kernel, double *d_cv, double *d_est, double *d_se, int32_t *d_best_status,
+                              void *d_workspace, size_t workspace_bytes, void *cuda_stream)
+{
+    if (!d_est || !d_se) return KR_EARG;
+    if (kernel == KR_GAUSSIAN) return KR_EKERNEL;  // Q26: compact windows
+    const int st = enqueue_grid(d_x, d_y, n, d_h, m, kernel, KR_ALGO_AUTO, d_cv, nullptr, d_best_status, d_workspace,
+                                workspace_bytes, cuda_stream, false);
+    if (st) return st;
+    return enqueue_ci<false>(n, d_h, kernel, d_est, d_se, d_best_status, d_workspace, m, cuda_stream);
+}
+
+extern "C" int kr_kde_ci_async(const double *d_x, int64_t n, const double *d_h, int32_t m, int32_t kernel,
+                               double *d_lscv, double *d_est, double *d_se, int32_t *d_best_status,
+                               void *d_workspace, size_t workspace_bytes, void *cuda_stream)
+{
+    if (!d_est || !d_se) return KR_EARG;
+    const int st = kr_kde_lscv_async(d_x, n, d_h, m, kernel, d_lscv, d_best_status, d_workspace, workspace_bytes,
+                                     cuda_stream);
+    if (st) return st;
+    return enqueue_ci<true>(n, d_h, kernel, d_est, d_se, d_best_status, d_workspace, m, cuda_stream);
 }

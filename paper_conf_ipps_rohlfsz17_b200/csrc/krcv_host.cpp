@@ -59,6 +59,9 @@ struct DevCtx {
     // CUDA graph of the last synchronous call whose inputs were pinned
     // (H2D copies, the whole device pipeline, D2H copies): replayed while
     // the pointers, sizes, kernel, algorithm and estimator repeat
+    // confidence-interval outputs [n] (kr_cv_ci / kr_kde_ci)
+    double *dest = nullptr, *dse = nullptr;
+    int64_t cap_ci = 0;
     cudaGraphExec_t gexec = nullptr;
     const void *gx = nullptr, *gy = nullptr, *gh = nullptr;
     int64_t gn = 0;
@@ -429,6 +432,68 @@ extern "C" int kr_kde_lscv(const double *x, int64_t n, const double *h_grid, int
     return KR_OK;
 }
 
+// Leave-one-out (jackknife) confidence intervals at the CV / LSCV optimum
+// (reading Q26): the device search, the interval kernel, one copy back.
+static int host_ci(bool kde, const double *x, const double *y, int64_t n, const double *h_grid, int32_t m,
+                   int32_t kernel, double *curve_out, double *est_out, double *se_out, int32_t *best_out)
+{
+    if (!curve_out || !est_out || !se_out || !best_out) return KR_EARG;
+    int st = kde ? (x && h_grid ? KR_OK : KR_EARG) : validate_all(x, y, n, h_grid, m, kernel);
+    if (st) return st;
+    if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return KR_EARG;
+    if (kernel != KR_UNIFORM && kernel != KR_EPANECHNIKOV && kernel != KR_TRIANGULAR) return KR_EKERNEL;
+    if (kde) {
+        st = kr_validate_grid(h_grid, m);
+        if (st) return st;
+        for (int64_t i = 0; i < n; i++)
+            if (!std::isfinite(x[i])) return KR_ENONFINITE;
+    }
+    int dev = 0;
+    KR_CUDA_TRY(cudaGetDevice(&dev));
+    DevCtx *c = get_ctx(dev);
+    std::lock_guard<std::mutex> g(c->mu);
+    st = ensure_capacity(c, n, m);
+    if (st) return st;
+    if (n > c->cap_ci) {
+        cudaFree(c->dest);
+        cudaFree(c->dse);
+        c->dest = c->dse = nullptr;
+        c->cap_ci = 0;
+        KR_CUDA_TRY(cudaMalloc(&c->dest, sizeof(double) * n));
+        KR_CUDA_TRY(cudaMalloc(&c->dse, sizeof(double) * n));
+        c->cap_ci = n;
+    }
+    cudaStream_t s = c->stream;
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dx, x, sizeof(double) * n, cudaMemcpyHostToDevice, s));
+    if (!kde) KR_CUDA_TRY(cudaMemcpyAsync(c->dy, y, sizeof(double) * n, cudaMemcpyHostToDevice, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(c->dh, h_grid, sizeof(double) * m, cudaMemcpyHostToDevice, s));
+    st = kde ? kr_kde_ci_async(c->dx, n, c->dh, m, kernel, c->dcv, c->dest, c->dse, c->dbest, c->ws, c->ws_bytes, s)
+             : kr_cv_ci_async(c->dx, c->dy, n, c->dh, m, kernel, c->dcv, c->dest, c->dse, c->dbest, c->ws,
+                              c->ws_bytes, s);
+    if (st) return st;
+    int32_t bs[2] = {0, 0};
+    KR_CUDA_TRY(cudaMemcpyAsync(bs, c->dbest, sizeof(int32_t) * 2, cudaMemcpyDeviceToHost, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(curve_out, c->dcv, sizeof(double) * m, cudaMemcpyDeviceToHost, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(est_out, c->dest, sizeof(double) * n, cudaMemcpyDeviceToHost, s));
+    KR_CUDA_TRY(cudaMemcpyAsync(se_out, c->dse, sizeof(double) * n, cudaMemcpyDeviceToHost, s));
+    KR_CUDA_TRY(cudaStreamSynchronize(s));
+    if (bs[1] != KR_OK) return bs[1];
+    *best_out = bs[0];
+    return KR_OK;
+}
+
+extern "C" int kr_cv_ci(const double *x, const double *y, int64_t n, const double *h_grid, int32_t m, int32_t kernel,
+                        double *cv_out, double *est_out, double *se_out, int32_t *best_out)
+{
+    return host_ci(false, x, y, n, h_grid, m, kernel, cv_out, est_out, se_out, best_out);
+}
+
+extern "C" int kr_kde_ci(const double *x, int64_t n, const double *h_grid, int32_t m, int32_t kernel,
+                         double *lscv_out, double *est_out, double *se_out, int32_t *best_out)
+{
+    return host_ci(true, x, nullptr, n, h_grid, m, kernel, lscv_out, est_out, se_out, best_out);
+}
+
 extern "C" int kr_kde_finalize(const double *partial, int64_t n, const double *h_grid, int32_t m, int32_t kernel,
                                double *lscv_out, int32_t *best_out)
 {
@@ -530,6 +595,10 @@ extern "C" int kr_release(void)
         cudaFree(c->dh);
         cudaFree(c->dpartial);
         cudaFree(c->dres);
+        cudaFree(c->dest);
+        cudaFree(c->dse);
+        c->dest = c->dse = nullptr;
+        c->cap_ci = 0;
         cudaFreeHost(c->pres);
         if (c->stream) cudaStreamDestroy(c->stream);
         for (int i = 0; i < 2; i++) {

@@ -41,6 +41,7 @@ EXPORTS = (
     "kr_profile_enable", "kr_profile_read", "kr_launch_count", "kr_last_algo",
     "kr_kde_lscv", "kr_kde_lscv_async", "kr_kde_shard_async", "kr_kde_finalize",
     "kr_ll_cv_grid", "kr_ll_cv_grid_async", "kr_ll_shard_async",
+    "kr_cv_ci", "kr_kde_ci", "kr_cv_ci_async", "kr_kde_ci_async",
 )
 
 
@@ -107,6 +108,12 @@ def _lib() -> ctypes.CDLL:
     lib.kr_ll_cv_grid_async.argtypes = [P, P, i64, P, i32, i32, P, P, P, P, sz, P]
     lib.kr_ll_shard_async.argtypes = [P, P, i64, P, i32, i32, i32, i32, P, P, sz, P]
     for f in ("kr_ll_cv_grid", "kr_ll_cv_grid_async", "kr_ll_shard_async"):
+        getattr(lib, f).restype = ctypes.c_int
+    lib.kr_cv_ci.argtypes = [P, P, i64, P, i32, i32, P, P, P, P]
+    lib.kr_kde_ci.argtypes = [P, i64, P, i32, i32, P, P, P, P]
+    lib.kr_cv_ci_async.argtypes = [P, P, i64, P, i32, i32, P, P, P, P, P, sz, P]
+    lib.kr_kde_ci_async.argtypes = [P, i64, P, i32, i32, P, P, P, P, P, sz, P]
+    for f in ("kr_cv_ci", "kr_kde_ci", "kr_cv_ci_async", "kr_kde_ci_async"):
         getattr(lib, f).restype = ctypes.c_int
     lib.kr_last_algo.restype = ctypes.c_int32
     _LIB = lib
@@ -464,3 +471,80 @@ def kr_ll_shard_async(d_x, d_y, d_h, kernel, shard: int, nshards: int, d_partial
                                     int(shard), int(nshards), d_partial.data_ptr(), d_ws.data_ptr(),
                                     d_ws.numel() * d_ws.element_size(), ctypes.c_void_p(s.cuda_stream)),
            "kr_ll_shard_async")
+
+
+# ------------------------------------- LOO confidence intervals (Q26)
+def kr_cv_ci(x, y, h, kernel="epanechnikov"):
+    """Grid search, then at the CV-optimal bandwidth the Nadaraya-Watson
+    estimate and its delete-one jackknife standard error at every observation
+    (reading Q26): (cv[m], est[n], se[n], best).  se is NaN where a point's
+    window holds only itself."""
+    x, y, h = _host(x), _host(y), _host(h)
+    if x.shape != y.shape or x.ndim != 1:
+        raise ValueError("x and y must be 1-D arrays of equal length")
+    n, m = x.shape[0], h.shape[0]
+    cv, est, se = np.empty(m), np.empty(n), np.empty(n)
+    best = ctypes.c_int32(-1)
+    _check(_lib().kr_cv_ci(x.ctypes.data, y.ctypes.data, n, h.ctypes.data, m, _kernel_id(kernel), cv.ctypes.data,
+                           est.ctypes.data, se.ctypes.data, ctypes.byref(best)), "kr_cv_ci")
+    return cv, est, se, int(best.value)
+
+
+def kr_kde_ci(x, h, kernel="epanechnikov"):
+    """KDE LSCV grid search, then at the optimal bandwidth the density estimate
+    and its delete-one jackknife standard error at every observation
+    (reading Q26): (lscv[m], est[n], se[n], best)."""
+    x, h = _host(x), _host(h)
+    n, m = x.shape[0], h.shape[0]
+    lscv, est, se = np.empty(m), np.empty(n), np.empty(n)
+    best = ctypes.c_int32(-1)
+    _check(_lib().kr_kde_ci(x.ctypes.data, n, h.ctypes.data, m, _kernel_id(kernel), lscv.ctypes.data,
+                            est.ctypes.data, se.ctypes.data, ctypes.byref(best)), "kr_kde_ci")
+    return lscv, est, se, int(best.value)
+
+
+def kr_cv_ci_async(d_x, d_y, d_h, kernel, d_cv, d_est, d_se, d_best_status, d_ws, stream=None) -> None:
+    """Device form of kr_cv_ci (CUDA tensors; enqueued on `stream`)."""
+    import torch
+
+    n, m = d_x.numel(), d_h.numel()
+    for t, name in ((d_x, "x"), (d_y, "y"), (d_h, "h")):
+        _check_f64(name, t)
+    _check_f64("y", d_y, n)
+    _check_f64("cv", d_cv, m)
+    _check_f64("est", d_est, n)
+    _check_f64("se", d_se, n)
+    _check_best_status(d_best_status)
+    s = torch.cuda.current_stream(d_x.device) if stream is None else stream
+    _check(_lib().kr_cv_ci_async(d_x.data_ptr(), d_y.data_ptr(), n, d_h.data_ptr(), m, _kernel_id(kernel),
+                                 d_cv.data_ptr(), d_est.data_ptr(), d_se.data_ptr(), d_best_status.data_ptr(),
+                                 d_ws.data_ptr(), d_ws.numel() * d_ws.element_size(), ctypes.c_void_p(s.cuda_stream)),
+           "kr_cv_ci_async")
+
+
+def kr_kde_ci_async(d_x, d_h, kernel, d_lscv, d_est, d_se, d_best_status, d_ws, stream=None) -> None:
+    """Device form of kr_kde_ci (CUDA tensors; enqueued on `stream`)."""
+    import torch
+
+    n, m = d_x.numel(), d_h.numel()
+    _check_f64("x", d_x)
+    _check_f64("h", d_h)
+    _check_f64("lscv", d_lscv, m)
+    _check_f64("est", d_est, n)
+    _check_f64("se", d_se, n)
+    _check_best_status(d_best_status)
+    s = torch.cuda.current_stream(d_x.device) if stream is None else stream
+    _check(_lib().kr_kde_ci_async(d_x.data_ptr(), n, d_h.data_ptr(), m, _kernel_id(kernel), d_lscv.data_ptr(),
+                                  d_est.data_ptr(), d_se.data_ptr(), d_best_status.data_ptr(), d_ws.data_ptr(),
+                                  d_ws.numel() * d_ws.element_size(), ctypes.c_void_p(s.cuda_stream)),
+           "kr_kde_ci_async")
+
+
+def confidence_intervals(est, se, level: float = 0.95):
+    """(lo, hi) = est -+ z se with z = Phi^-1((1 + level) / 2) (arithmetic on
+    the outputs of kr_cv_ci / kr_kde_ci; no device work)."""
+    from statistics import NormalDist
+
+    z = NormalDist().inv_cdf(0.5 + 0.5 * float(level))
+    est, se = np.asarray(est, np.float64), np.asarray(se, np.float64)
+    return est - z * se, est + z * se
