@@ -50,6 +50,14 @@ FLOPS_PER_EMIT = {0: 4, 1: 9, 2: 9}
 # formula (prefix differences, shift to the row frame, estimate, error);
 # DESIGN.md §6.2.
 FLOPS_PER_WINDOW = {0: 6, 1: 25, 2: 30}
+# FP64 operations of the two boundary lookups of one (row, bandwidth) in
+# win_kernel (per side: x_r +- h, the bucket index FMA, four probes of
+# subtract + compare): the search share of the work, for frac_incl_search.
+SEARCH_FP64_PER_WINDOW = 20
+# Small-message NCCL all-reduce latency over NVLink assumed by the P-GPU
+# projection of other_configs (the 2m+2 fp64 partial vector, <= 16 KB); NOT
+# measured here -- this environment has one GPU.
+ALLREDUCE_US_ASSUMED = 20.0
 # Dense Gaussian path: per (pair, bandwidth) x = t c (1), e^-x evaluated on
 # the FP64 pipe (Cody-Waite 2 FMA + degree-12 Horner 12 FMA + rounding trick
 # 2 + scale 1 = 31 flops), num FMA (2), den add (1).  DESIGN.md §6.5.
@@ -92,6 +100,8 @@ def parse():
                     help="override the config's kernel (e.g. the Gaussian dense path on C2's data)")
     ap.add_argument("--algo", default="auto", choices=["auto", "sweep", "prefix", "hist"],
                     help="KR_ALGO_* for every call (sets KRCV_ALGO before the library loads)")
+    ap.add_argument("--no-extra", action="store_true",
+                    help="skip the single-GPU C3/C4/C5 lines under other_configs (default run only)")
     ap.add_argument("--cpu-seconds", type=float, default=8.0,
                     help="target wall seconds of the bounded oracle sample")
     return ap.parse_args()
@@ -315,14 +325,23 @@ def run_ours(args):
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
     stream = torch.cuda.current_stream(dev)
     rows_mine = ((rank + 1) * n) // world - (rank * n) // world
+    main_wl = {"name": args.config, "x": x, "y": y, "h": h, "k": k, "n": n, "m": m, "d_x": d_x, "d_y": d_y, "units": units,
+               "rows_mine": rows_mine}
 
     def barrier():
         if world > 1:
             torch.distributed.barrier()
 
-    def timed(algo):
+    def timed(algo, wl=None, steps=None, warmup=None):
         """W warm-up + K device-timed grid searches with `algo`; L2 flushed
-        between steps (outside the events); max over ranks."""
+        between steps (outside the events); max over ranks.  wl: another
+        workload (bench_extra_configs), default the config's."""
+        wl = wl or main_wl
+        nsteps = steps or args.steps
+        nwarm = warmup or args.warmup
+        x, y, h, k, n, m = wl["x"], wl["y"], wl["h"], wl["k"], wl["n"], wl["m"]
+        cname = wl["name"]
+        d_x, d_y, units, rows_mine = wl["d_x"], wl["d_y"], wl["units"], wl["rows_mine"]
         # single GPU: the whole search is replayed from a CUDA graph
         # (GridSearch(graph=True)).  Two plans: the headline steps replay a
         # graph WITHOUT the library's stage events; a second, profiled plan
@@ -330,17 +349,17 @@ def run_ours(args):
         # capture) gives the per-stage times, the dominant kernel's time for
         # the roofline and its share of a profiled step.
         def run_steps(plan, profiled):
-            for _ in range(args.warmup):
+            for _ in range(nwarm):
                 plan.run(d_x, d_y)
             plan.result()
             torch.cuda.synchronize()
-            starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-            ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+            starts = [torch.cuda.Event(enable_timing=True) for _ in range(nsteps)]
+            ends = [torch.cuda.Event(enable_timing=True) for _ in range(nsteps)]
             st, launches = [], 0
             barrier()
             torch.cuda.synchronize()
             with ClockSampler(local) as clk:
-                for s in range(args.steps):
+                for s in range(nsteps):
                     flush.fill_(s & 0xFF)
                     starts[s].record(stream)
                     plan.run(d_x, d_y)
@@ -353,7 +372,7 @@ def run_ours(args):
                 torch.cuda.synchronize()
             barrier()
             # median step; the driver's clock brackets all K
-            return statistics.median(starts[s].elapsed_time(ends[s]) for s in range(args.steps)), st, launches, clk
+            return statistics.median(starts[s].elapsed_time(ends[s]) for s in range(nsteps)), st, launches, clk
 
         krcv.kr_profile_enable(False)
         plan = GridSearch(n, h, k, device=dev, rank=rank, world=world, algo=algo, graph=(world == 1),
@@ -387,19 +406,27 @@ def run_ours(args):
             basis = (f"{FLOPS_PER_PAIR[k]} flops per ordered pair x rows x (n-1) + {FLOPS_PER_EMIT[k]} per "
                      "(row, bandwidth) emit")
         else:
-            kname = "window_kernel (a3+a4, window-prefix)"
+            kname = "win_kernel (a3+a4, window-prefix with bucket-table boundary lookups)"
             flops = rows_mine * m * FLOPS_PER_WINDOW[k]
             basis = (f"{FLOPS_PER_WINDOW[k]} flops per (row, bandwidth): prefix differences, shift to the "
-                     "row, LOO estimate, squared error (DESIGN.md §6.2); searches not counted")
+                     "row, LOO estimate, squared error (DESIGN.md §6.2); searches not counted (see "
+                     "frac_incl_search)")
         achieved = flops / main_s / 1e12
+        extra = {}
+        if used == "prefix":
+            fs = rows_mine * m * (FLOPS_PER_WINDOW[k] + SEARCH_FP64_PER_WINDOW)
+            extra = {"flops_incl_search": fs, "frac_incl_search": fs / main_s / 1e12 / peak,
+                     "search_basis": f"+{SEARCH_FP64_PER_WINDOW} FP64 ops per (row, bandwidth) for the two "
+                                     "boundary lookups (x_r +- h, bucket index, four probes of subtract + "
+                                     "compare per side; DESIGN.md §6.2)"}
         return {
             "algo": used, "value": units / (step_ms * 1e-3), "ms_per_step": step_ms,
             "stage_ms": {"pack_sort_gather": statistics.median(sort_ms), "prefix_build": statistics.median(build_ms),
                          "sweep": main_med, "reduce_finalize": statistics.median(red_ms)},
             "roofline": {"bound": "alu", "kernel": kname, "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
-                         "frac": achieved / peak, "traffic": ncu_traffic(args.config, used),
-                         "ncu": ncu_context(args.config, used),
-                         "flops_per_launch": flops, "flops_basis": basis,
+                         "frac": achieved / peak, "traffic": ncu_traffic(cname, used),
+                         "ncu": ncu_context(cname, used),
+                         "flops_per_launch": flops, "flops_basis": basis, **extra,
                          "peak_note": peak_note,
                          "kernel_ms": main_med,
                          "kernel_share_of_step": main_med / prof_step_ms,
@@ -445,6 +472,8 @@ def run_ours(args):
         alt.pop("plan")
         out["alt_algo"] = {key: alt[key] for key in ("algo", "value", "ms_per_step", "stage_ms", "roofline",
                                                       "result", "clocks")}
+    if world == 1 and args.config == "C2" and not args.no_extra:
+        out["other_configs"] = bench_extra_configs(args, timed, dev, krcv, torch)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         v, dt, rows, threads = oracle_sample(x, y, h, k, args.cpu_seconds)
         out["cpu_baseline"] = {
@@ -459,6 +488,60 @@ def run_ours(args):
     if world > 1:
         torch.distributed.destroy_process_group()
     return 0
+
+
+def bench_extra_configs(args, timed, dev, krcv, torch):
+    """The other BASELINE.json configurations on this one GPU (C3, C4, C5:
+    configs[2..4]) in the same launch configuration as the headline, each with
+    its stage times and roofline, plus the row-shard balance of the window
+    stage at P = 8 (the eight equal sorted-row shards timed one after another
+    on this GPU through kr_cv_rows_async) and the projected P-GPU time
+        T(P) = pack/sort + prefix/table build (replicated on every rank)
+               + window * (max shard / mean shard) / P + reduce
+               + ALLREDUCE_US_ASSUMED
+    and efficiency T(1) / (P T(P)).  A projection from single-GPU stage times,
+    not a multi-GPU measurement (this environment has one GPU)."""
+    res = {}
+    for name in ("C3", "C4", "C5"):
+        cfg = workloads.CONFIGS[name]
+        x, y, h, k = workloads.make(cfg, seed=args.seed)
+        n, m = x.shape[0], h.shape[0]
+        wl = {"name": name, "x": x, "y": y, "h": h, "k": k, "n": n, "m": m, "d_x": torch.as_tensor(x, device=dev),
+              "d_y": torch.as_tensor(y, device=dev), "units": n * (n - 1) * m, "rows_mine": n}
+        r = timed("auto", wl, steps=5 if name == "C4" else 10, warmup=3)
+        r.pop("plan")
+        # window-stage balance of 8 equal row shards
+        d_h = torch.as_tensor(h, device=dev)
+        ws = krcv.aligned(krcv.workspace(n, m, dev))
+        part = torch.zeros(krcv.partial_len(m), dtype=torch.float64, device=dev)
+        krcv.kr_profile_enable(True)
+        shard_ms = []
+        for s in range(8):
+            lo, hi = (s * n) // 8, ((s + 1) * n) // 8
+            for _ in range(2):  # the second run is timed (warm)
+                krcv.kr_cv_rows_async(wl["d_x"], wl["d_y"], d_h, k, lo, hi, part, ws)
+                t = krcv.kr_profile_read()
+            shard_ms.append(t[2])
+        krcv.kr_profile_enable(False)
+        del ws
+        st = r["stage_ms"]
+        imb = max(shard_ms) / (sum(shard_ms) / len(shard_ms))
+        t1 = r["ms_per_step"]
+        proj = {}
+        for P in (2, 4, 8):
+            tp = st["pack_sort_gather"] + st["prefix_build"] + st["sweep"] * (imb if P == 8 else 1.0) / P + \
+                st["reduce_finalize"] + ALLREDUCE_US_ASSUMED * 1e-3
+            proj[str(P)] = {"ms": tp, "efficiency": t1 / (P * tp)}
+        res[name] = {"workload": workload_desc(cfg, args.seed), "value": r["value"], "unit": UNIT,
+                     "ms_per_step": t1, "stage_ms": st, "roofline": r["roofline"], "result": r["result"],
+                     "clocks": r["clocks"], "gpu_launches": r["gpu_launches"],
+                     "shard8_window_ms": shard_ms, "shard8_imbalance": imb,
+                     "projected_scaling": proj,
+                     "projection_note": ("T(P) = replicated sort + prefix/table build + window x imbalance(P=8, "
+                                         "measured on 8 equal shards) / P + reduce + "
+                                         f"{ALLREDUCE_US_ASSUMED} us assumed all-reduce; one-GPU stage times, "
+                                         "not a multi-GPU measurement")}
+    return res
 
 
 def e2e_measure(args, x, y, h, k, n, m, units, dev, rank, world, plan):

@@ -6,7 +6,11 @@
  *   gcc -O2 -I include examples/krcv_example.c \
  *       -L paper_conf_ipps_rohlfsz17_b200 -lkrcv \
  *       -Wl,-rpath,$PWD/paper_conf_ipps_rohlfsz17_b200 -o krcv_example
- *   ./krcv_example [n] [m]          (--host-only: ABI checks without a GPU)
+ *   ./krcv_example [n] [m] [--dump] (--host-only: ABI checks without a GPU)
+ *
+ * --dump prints the whole CV curve and n_eff (kr_cv_grid_ex) and the
+ * leave-one-out confidence intervals at the optimum (kr_cv_ci) of every
+ * observation, one value per line in %.17g, for tests/test_c_consumer.py.
  */
 #include <stdint.h>
 #include <stdio.h>
@@ -51,6 +55,19 @@ int main(int argc, char **argv)
     st = kr_cv_grid(x, y, n, h, m, KR_EPANECHNIKOV, cv, &best);
     if (st) { fprintf(stderr, "kr_cv_grid: %s (%s)\n", kr_strerror(st), kr_last_cuda_error()); return 1; }
     printf("n = %lld, m = %d: best b = %d, h = %.9g, CV = %.12g\n", (long long)n, m, best, h[best], cv[best]);
+    if (argc > 3 && strcmp(argv[3], "--dump") == 0) {
+        int64_t *neff = malloc(sizeof(int64_t) * m);
+        double *est = malloc(sizeof(double) * n), *se = malloc(sizeof(double) * n);
+        int32_t best2 = -1, best3 = -1;
+        if (!neff || !est || !se) return 2;
+        st = kr_cv_grid_ex(x, y, n, h, m, KR_EPANECHNIKOV, cv, neff, &best2);
+        if (st || best2 != best) { fprintf(stderr, "kr_cv_grid_ex: %s\n", kr_strerror(st)); return 1; }
+        for (int32_t b = 0; b < m; b++) printf("curve %d %.17g %lld\n", b, cv[b], (long long)neff[b]);
+        st = kr_cv_ci(x, y, n, h, m, KR_EPANECHNIKOV, cv, est, se, &best3);
+        if (st || best3 != best) { fprintf(stderr, "kr_cv_ci: %s\n", kr_strerror(st)); return 1; }
+        for (int64_t i = 0; i < n; i++) printf("ci %lld %.17g %.17g\n", (long long)i, est[i], se[i]);
+        free(neff); free(est); free(se);
+    }
     kr_release();
     free(x); free(y); free(h); free(cv);
     return 0;

@@ -220,10 +220,20 @@ int kr_ll_shard_async(const double *d_x, const double *d_y, int64_t n, const dou
 /* Host-side grid check (finite, > 0, non-decreasing, 1 <= m <= KR_MAX_M). */
 int kr_validate_grid(const double *h_grid, int32_t m);
 
-/* Device workspace size in bytes for kr_cv_shard_async at (n, m).  Returns 0
- * for invalid (n, m).  Requires a CUDA device (the radix-sort scratch size
- * is queried from the runtime). */
+/* Device workspace size in bytes at (n, m), enough for EVERY device entry
+ * point (all algorithms, the KDE family).  Returns 0 for invalid (n, m).
+ * Requires a CUDA device (the radix-sort scratch size and the SM count are
+ * queried from the runtime). */
 size_t kr_workspace_bytes(int64_t n, int32_t m);
+
+/* The workspace one Nadaraya-Watson / local-linear / interval call needs with
+ * `algo` (KR_ALGO_*; KR_ALGO_AUTO resolves as the call would) -- the
+ * per-algorithm partial-sum blocks only (the split sweep's per-tile partials
+ * are the largest; the default window-prefix path needs a few MB per 1,000
+ * bandwidths) -- and the one the KDE entry points need.  An entry point given
+ * less than its requirement returns KR_EARG.  0 for invalid (n, m). */
+size_t kr_workspace_bytes_algo(int64_t n, int32_t m, int32_t kernel, int32_t algo);
+size_t kr_kde_workspace_bytes(int64_t n, int32_t m);
 
 /*
  * kr_cv_shard_async -- device path for caller-owned device memory and row

@@ -376,7 +376,16 @@ constexpr int64_t kCubSingleTile = 0;
 
 static inline size_t align256(size_t v) { return (v + 255) & ~size_t(255); }
 
-bool ws_layout(int64_t n, int32_t m, WsLayout *L)
+// Workspace classes (size the partials per algorithm; the KDE
+// sum-B block only for the KDE entry points).  Everything before the bucket
+// table has the same offset in every class (kr_cv_refine reuses it in place).
+int ws_class_for(int32_t algo, int32_t kernel, int64_t rows)
+{
+    if (algo == KR_ALGO_AUTO) algo = kernel == KR_GAUSSIAN ? KR_ALGO_DENSE : auto_algo(rows, rows, 0, kernel);
+    return algo == KR_ALGO_SWEEP ? kWsSweep : kWsDefault;
+}
+
+bool ws_layout(int64_t n, int32_t m, WsLayout *L, int cls)
 {
     size_t cub_bytes = 0;
     cudaError_t e = cub::DeviceRadixSort::SortPairs(
@@ -394,7 +403,7 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     L->vals_in = off;  off = align256(off + sizeof(uint32_t) * npad);
     L->vals_out = off; off = align256(off + sizeof(uint32_t) * npad);
     L->xy = off;       off = align256(off + sizeof(double2) * ((size_t)n + 2 * kPad));
-    L->counter = off;  off = align256(off + sizeof(int) * (1 + kSmCounters));  // tile counter + SM-local counters
+    L->counter = off;  off = align256(off + sizeof(int) * 32);  // tile counter
     L->perm = off;     off = align256(off + sizeof(uint32_t) * (size_t)n);
     // window-prefix path (krcv_prefix.cuh)
     const size_t nch = (size_t)((n + kPfxTileMin) / kPfxTileMin);  // most tiles covering P[0..n]
@@ -415,13 +424,18 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L)
     // bucket table of win_kernel (krcv_window.cuh): int32 [Qmax + 1], Qmax = min(kBktFmax n, kBktQmax)
     const int64_t qmax = (int64_t)kBktFmax * n < kBktQmax ? (int64_t)kBktFmax * n : kBktQmax;
     L->bt = off;       off = align256(off + sizeof(int) * (size_t)(qmax + 1));
-    // partials: one per 32-row tile (sweep, r01 window, LL, hist, dense; uint8
-    // counts) or one per win_kernel warp slot (uint32 counts)
+    // partials: one per win_kernel warp slot (uint32 counts), one per 32-row
+    // tile (r01 window, local-linear, histogram, dense, KDE; uint8 counts) and,
+    // for the sweep class, one per 32/G-row tile of the split sweep
     const size_t slots = (size_t)win2_max_slots();
-    L->tileS = off;    off = align256(off + sizeof(double) * ((size_t)ntiles > slots ? (size_t)ntiles : slots) * (size_t)m);
-    const size_t nbytes = (size_t)ntiles > 4 * slots ? (size_t)ntiles : 4 * slots;
+    const size_t t32 = (size_t)((n + 31) / 32);
+    size_t tiles = t32;
+    if (cls == kWsSweep || cls == kWsAll) tiles = (size_t)ntiles > tiles ? (size_t)ntiles : tiles;
+    L->tileS = off;    off = align256(off + sizeof(double) * (tiles > slots ? tiles : slots) * (size_t)m);
+    const size_t nbytes = tiles > 4 * slots ? tiles : 4 * slots;
     L->tileN = off;    off = align256(off + nbytes * (size_t)m);
-    L->tileB = off;    off = align256(off + sizeof(double) * (size_t)((n + 31) / 32) * (size_t)m);  // KDE sum B
+    L->tileB = off;
+    if (cls == kWsKde || cls == kWsAll) off = align256(off + sizeof(double) * t32 * (size_t)m);  // KDE sum B
     L->partial = off;  off = align256(off + sizeof(double) * (size_t)KR_PARTIAL_LEN(m));
     L->cub_bytes = cub_bytes;
     L->total = off;
@@ -737,10 +751,26 @@ static Win2Shape win2_shape(int64_t rows, int m)
     return w;
 }
 
+// the bucket table of win_kernel (krcv_window.cuh) from the sorted x: part of
+// the O(n) build stage, after the prefix scan (which publishes the density
+// statistic it sizes the table with)
+static void launch_bkt_fill(int n, const WsLayout &L, char *ws, cudaStream_t st)
+{
+    const double *xs = reinterpret_cast<const double *>(ws + L.xs) + kPad;
+    int *BT = reinterpret_cast<int *>(ws + L.bt);
+    const unsigned long long *gap =
+        reinterpret_cast<const unsigned long long *>(ws + L.status + 6 * sizeof(unsigned));
+    BktParams *prm = reinterpret_cast<BktParams *>(ws + L.status + 32);
+    const int64_t qmax = (int64_t)kBktFmax * n < kBktQmax ? (int64_t)kBktFmax * n : kBktQmax;
+    const int64_t nseg = (n + qmax + 1 + kBktSeg - 1) / kBktSeg;
+    int64_t blocks = (nseg + kBktFillThreads - 1) / kBktFillThreads;
+    if (blocks > (int64_t)dev_info().sms * 8) blocks = (int64_t)dev_info().sms * 8;
+    launch_pdl(bkt_fill_kernel, dim3((int)blocks), dim3(kBktFillThreads), 0, st, xs, n, gap, BT, prm);
+}
+
 template <int KERN>
 static void launch_win2(const double2 *xy, int n, const double *h, int m, int lo, int hi, const Win2Shape &w,
-                        bool build_table, const WsLayout &L, char *ws, double *tileS, uint32_t *tileN,
-                        cudaStream_t st)
+                        const WsLayout &L, char *ws, double *tileS, uint32_t *tileN, cudaStream_t st)
 {
     const double *xs = reinterpret_cast<const double *>(ws + L.xs) + kPad;
     const double *P = reinterpret_cast<const double *>(ws + L.pfx);
@@ -750,14 +780,6 @@ static void launch_win2(const double2 *xy, int n, const double *h, int m, int lo
     const unsigned long long *gap =
         reinterpret_cast<const unsigned long long *>(ws + L.status + 6 * sizeof(unsigned));
     BktParams *prm = reinterpret_cast<BktParams *>(ws + L.status + 32);
-    const int sms = dev_info().sms;
-    if (build_table) {
-        const int64_t qmax = (int64_t)kBktFmax * n < kBktQmax ? (int64_t)kBktFmax * n : kBktQmax;
-        const int64_t nseg = (n + qmax + 1 + kBktSeg - 1) / kBktSeg;
-        int64_t blocks = (nseg + kBktFillThreads - 1) / kBktFillThreads;
-        if (blocks > (int64_t)sms * 8) blocks = (int64_t)sms * 8;
-        launch_pdl(bkt_fill_kernel, dim3((int)blocks), dim3(kBktFillThreads), 0, st, xs, n, gap, BT, prm);
-    }
     launch_pdl(win_kernel<KERN>, dim3(w.blocks), dim3(kWin2Threads), 0, st, xs, xy, P, (int)L.pstride,
                (const int *)BT, (const BktParams *)prm, h, m, n, lo, hi, w.ntiles, w.BC, w.nbc, ymax, tileS,
                tileN);
@@ -849,7 +871,23 @@ extern "C" size_t kr_workspace_bytes(int64_t n, int32_t m)
 {
     if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return 0;
     WsLayout L;
-    if (!ws_layout(n, m, &L)) return 0;
+    if (!ws_layout(n, m, &L, kWsAll)) return 0;
+    return L.total;
+}
+
+extern "C" size_t kr_workspace_bytes_algo(int64_t n, int32_t m, int32_t kernel, int32_t algo)
+{
+    if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return 0;
+    WsLayout L;
+    if (!ws_layout(n, m, &L, ws_class_for(algo, kernel, n))) return 0;
+    return L.total;
+}
+
+extern "C" size_t kr_kde_workspace_bytes(int64_t n, int32_t m)
+{
+    if (n < 2 || n > 2147483647LL || m < 1 || m > KR_MAX_M) return 0;
+    WsLayout L;
+    if (!ws_layout(n, m, &L, kWsKde)) return 0;
     return L.total;
 }
 
@@ -933,7 +971,7 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         return KR_EARG;
     if ((reinterpret_cast<uintptr_t>(d_workspace) & 255u) != 0) return KR_EARG;
     WsLayout L;
-    if (!ws_layout(n, m, &L)) return KR_ECUDA;
+    if (!ws_layout(n, m, &L, ws_class_for(algo, kernel, n))) return KR_ECUDA;
     if (workspace_bytes < L.total) return KR_EARG;
 
     cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
@@ -1008,6 +1046,10 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         default: launch_prefix_build<KR_TRIANGULAR>(xy, nn, L, ws, st); break;
         }
         launches += 2;
+        if (win2) {  // win_kernel's bucket table (depends on xs only: kept on reuse)
+            launch_bkt_fill(nn, L, ws, st);
+            launches += 1;
+        }
     }
     prof_mark(2, st);
     if (injected_failure("sweep")) return KR_ECUDA;
@@ -1048,19 +1090,17 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
             }
         } else if (win2) {
             uint32_t *tileN32 = reinterpret_cast<uint32_t *>(ws + L.tileN);
-            const bool table = !reuse_sorted;  // the table depends on xs only
             switch (kernel) {
             case KR_UNIFORM:
-                launch_win2<KR_UNIFORM>(xy, nn, d_h, m, lo, hi, w2, table, L, ws, tileS, tileN32, st);
+                launch_win2<KR_UNIFORM>(xy, nn, d_h, m, lo, hi, w2, L, ws, tileS, tileN32, st);
                 break;
             case KR_EPANECHNIKOV:
-                launch_win2<KR_EPANECHNIKOV>(xy, nn, d_h, m, lo, hi, w2, table, L, ws, tileS, tileN32, st);
+                launch_win2<KR_EPANECHNIKOV>(xy, nn, d_h, m, lo, hi, w2, L, ws, tileS, tileN32, st);
                 break;
             default:
-                launch_win2<KR_TRIANGULAR>(xy, nn, d_h, m, lo, hi, w2, table, L, ws, tileS, tileN32, st);
+                launch_win2<KR_TRIANGULAR>(xy, nn, d_h, m, lo, hi, w2, L, ws, tileS, tileN32, st);
                 break;
             }
-            launches += table ? 1 : 0;
         } else if (prefix) {
             switch (kernel) {
             case KR_UNIFORM:
@@ -1217,7 +1257,7 @@ static int enqueue_kde(const double *d_x, int64_t n, const double *d_h, int32_t 
     if (nshards < 1 || shard < 0 || shard >= nshards) return KR_EARG;
     if ((reinterpret_cast<uintptr_t>(d_workspace) & 255u) != 0) return KR_EARG;
     WsLayout L;
-    if (!ws_layout(n, m, &L)) return KR_ECUDA;
+    if (!ws_layout(n, m, &L, kWsKde)) return KR_ECUDA;
     if (workspace_bytes < L.total) return KR_EARG;
     cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
     char *ws = static_cast<char *>(d_workspace);
@@ -1318,8 +1358,8 @@ template <bool KDE>
 static int enqueue_ci(int64_t n, const double *d_h, int32_t kernel, double *d_est, double *d_se,
                       const int32_t *d_best_status, void *d_workspace, int32_t m, void *cuda_stream)
 {
-    WsLayout L;
-    if (!ws_layout(n, m, &L)) return KR_ECUDA;
+    WsLayout L;  // only the m-independent offsets are read here: any class
+    if (!ws_layout(n, m, &L, kWsDefault)) return KR_ECUDA;
     char *ws = static_cast<char *>(d_workspace);
     const double2 *xy = reinterpret_cast<const double2 *>(ws + L.xy) + kPad;
     const uint32_t *perm = reinterpret_cast<const uint32_t *>(ws + L.perm);

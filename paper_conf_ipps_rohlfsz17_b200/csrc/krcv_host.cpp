@@ -102,7 +102,7 @@ static void drop_graph(DevCtx *c)
 // [best, status] (8 B) | cv[m] | neff[m]
 static size_t res_bytes(int32_t m) { return 8 + (sizeof(double) + sizeof(int64_t)) * (size_t)m; }
 
-static int ensure_capacity(DevCtx *c, int64_t n, int32_t m)
+static int ensure_capacity(DevCtx *c, int64_t n, int32_t m, size_t need)
 {
     if (!c->stream) {
         KR_CUDA_TRY(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
@@ -140,7 +140,6 @@ static int ensure_capacity(DevCtx *c, int64_t n, int32_t m)
         c->dneff = reinterpret_cast<int64_t *>(c->dres + 8 + sizeof(double) * m);
         c->cap_m = m;
     }
-    size_t need = kr_workspace_bytes(n, m);
     if (need == 0) return KR_ECUDA;
     if (need > c->ws_bytes) {
         drop_graph(c);
@@ -246,7 +245,8 @@ static int host_call(const double *x, const double *y, int64_t n, const double *
     KR_CUDA_TRY(cudaGetDevice(&dev));
     DevCtx *c = get_ctx(dev);
     std::lock_guard<std::mutex> g(c->mu);
-    int st = ensure_capacity(c, n, m);
+    int st = ensure_capacity(c, n, m, ll ? kr_workspace_bytes_algo(n, m, kernel, KR_ALGO_PREFIX)
+                                         : kr_workspace_bytes_algo(n, m, kernel, algo));
     if (st) return st;
     st = ensure_staging(c, m);
     if (st) return st;
@@ -369,7 +369,7 @@ extern "C" int kr_cv_refine(const double *x, const double *y, int64_t n, const d
     DevCtx *c = get_ctx(dev);
     std::lock_guard<std::mutex> g(c->mu);
     const int32_t mcap = levels > 1 && m_fine > m ? m_fine : m;
-    st = ensure_capacity(c, n, mcap);
+    st = ensure_capacity(c, n, mcap, kr_workspace_bytes_algo(n, mcap, kernel, algo));
     if (st) return st;
     cudaStream_t s = c->stream;
     KR_CUDA_TRY(cudaMemcpyAsync(c->dx, x, sizeof(double) * n, cudaMemcpyHostToDevice, s));
@@ -414,7 +414,7 @@ extern "C" int kr_kde_lscv(const double *x, int64_t n, const double *h_grid, int
     KR_CUDA_TRY(cudaGetDevice(&dev));
     DevCtx *c = get_ctx(dev);
     std::lock_guard<std::mutex> g(c->mu);
-    st = ensure_capacity(c, n, m);
+    st = ensure_capacity(c, n, m, kr_kde_workspace_bytes(n, m));
     if (st) return st;
     cudaStream_t s = c->stream;
     KR_CUDA_TRY(cudaMemcpyAsync(c->dx, x, sizeof(double) * n, cudaMemcpyHostToDevice, s));
@@ -452,7 +452,7 @@ static int host_ci(bool kde, const double *x, const double *y, int64_t n, const 
     KR_CUDA_TRY(cudaGetDevice(&dev));
     DevCtx *c = get_ctx(dev);
     std::lock_guard<std::mutex> g(c->mu);
-    st = ensure_capacity(c, n, m);
+    st = ensure_capacity(c, n, m, kde ? kr_kde_workspace_bytes(n, m) : kr_workspace_bytes_algo(n, m, kernel, KR_ALGO_AUTO));
     if (st) return st;
     if (n > c->cap_ci) {
         cudaFree(c->dest);

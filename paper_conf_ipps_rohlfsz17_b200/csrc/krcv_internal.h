@@ -7,8 +7,6 @@
 
 namespace krcv {
 
-// SM-local task counters after the tile counter in the workspace (window kernels).
-constexpr int kSmCounters = 1024;
 
 // Shards with at least this many rows use the gxg sweep variant.
 constexpr int64_t kGxgRows = 400000;
@@ -45,8 +43,16 @@ struct WsLayout {
     int64_t ntiles_max;
 };
 
+// Workspace classes: the partial-sum blocks an algorithm needs (the other
+// buffers are common): default = win_kernel slots + one partial per 32-row
+// tile (window-prefix, local-linear, dense, histogram, intervals); sweep = +
+// the split sweep's 32/G-row tiles; kde = + the KDE sum-B block; all = every
+// entry point (kr_workspace_bytes).
+enum { kWsDefault = 0, kWsSweep = 1, kWsKde = 2, kWsAll = 3 };
+int ws_class_for(int32_t algo, int32_t kernel, int64_t rows);
+
 // Fills `out`; returns false if the CUDA runtime refuses the sort-size query.
-bool ws_layout(int64_t n, int32_t m, WsLayout *out);
+bool ws_layout(int64_t n, int32_t m, WsLayout *out, int cls);
 
 // Whole single-GPU search (kr_cv_grid_async) with an optional reuse of the
 // sorted arrays / prefix moments already in the workspace (kr_cv_refine).

@@ -42,6 +42,7 @@ EXPORTS = (
     "kr_kde_lscv", "kr_kde_lscv_async", "kr_kde_shard_async", "kr_kde_finalize",
     "kr_ll_cv_grid", "kr_ll_cv_grid_async", "kr_ll_shard_async",
     "kr_cv_ci", "kr_kde_ci", "kr_cv_ci_async", "kr_kde_ci_async",
+    "kr_workspace_bytes_algo", "kr_kde_workspace_bytes",
 )
 
 
@@ -78,6 +79,10 @@ def _lib() -> ctypes.CDLL:
     lib.kr_validate_grid.argtypes = [P, i32]
     lib.kr_workspace_bytes.argtypes = [i64, i32]
     lib.kr_workspace_bytes.restype = sz
+    lib.kr_workspace_bytes_algo.argtypes = [i64, i32, i32, i32]
+    lib.kr_workspace_bytes_algo.restype = sz
+    lib.kr_kde_workspace_bytes.argtypes = [i64, i32]
+    lib.kr_kde_workspace_bytes.restype = sz
     lib.kr_cv_shard_async.argtypes = [P, P, i64, P, i32, i32, i32, i32, P, P, sz, P]
     lib.kr_cv_shard_algo_async.argtypes = [P, P, i64, P, i32, i32, i32, i32, i32, P, P, sz, P]
     lib.kr_cv_rows_async.argtypes = [P, P, i64, P, i32, i32, i32, i64, i64, P, P, sz, P]
@@ -228,7 +233,14 @@ def kr_release() -> None:
     _check(_lib().kr_release(), "kr_release")
 
 
-def kr_workspace_bytes(n: int, m: int) -> int:
+def kr_workspace_bytes(n: int, m: int, kernel=None, algo=None, kde: bool = False) -> int:
+    """Workspace bytes: for every entry point (default), for one algorithm
+    (kernel and algo given: kr_workspace_bytes_algo) or for the KDE family."""
+    if kde:
+        return int(_lib().kr_kde_workspace_bytes(int(n), int(m)))
+    if algo is not None:
+        k = EPANECHNIKOV if kernel is None else _kernel_id(kernel)
+        return int(_lib().kr_workspace_bytes_algo(int(n), int(m), k, _algo_id(algo)))
     return int(_lib().kr_workspace_bytes(int(n), int(m)))
 
 
@@ -369,11 +381,12 @@ def kr_launch_count() -> int:
     return int(_lib().kr_launch_count())
 
 
-def workspace(n: int, m: int, device=None):
-    """A device workspace tensor (PyTorch caching allocator, 256-B aligned)."""
+def workspace(n: int, m: int, device=None, kernel=None, algo=None, kde: bool = False):
+    """A device workspace tensor (PyTorch caching allocator; take aligned()).
+    Sized for every entry point unless algo (with kernel) or kde narrows it."""
     import torch
 
-    nbytes = kr_workspace_bytes(n, m)
+    nbytes = kr_workspace_bytes(n, m, kernel, algo, kde)
     if nbytes == 0:
         raise KrcvError(KR_ECUDA, "kr_workspace_bytes")
     return torch.empty(nbytes + 256, dtype=torch.uint8, device=device)

@@ -1,8 +1,10 @@
 """The C-ABI used from plain C (examples/krcv_example.c): compiled with gcc
 against include/krcv.h and linked to libkrcv.so, without Python or PyTorch in
 the process.  CPU tier: the host-only entry points (version, default grid,
-grid validation, argument errors); GPU tier: a whole C2-size search, whose
-optimum must be the oracle's on the same inputs."""
+grid validation, argument errors); GPU tier: a whole search from plain C --
+the full CV curve and n_eff (kr_cv_grid_ex) against the oracle element by
+element, the optimum, and the leave-one-out confidence intervals at it
+(kr_cv_ci, reading Q26) for every observation."""
 from __future__ import annotations
 
 import os
@@ -37,7 +39,7 @@ def test_c_consumer_full_search(tmp_path):
     import numpy as np
 
     import oracle
-    p = subprocess.run([_build(tmp_path), "3000", "40"], capture_output=True, text=True, timeout=300)
+    p = subprocess.run([_build(tmp_path), "3000", "40", "--dump"], capture_output=True, text=True, timeout=300)
     assert p.returncode == 0, p.stdout + p.stderr
     mt = re.search(r"best b = (\d+), h = (\S+), CV = (\S+)", p.stdout)
     assert mt, p.stdout
@@ -62,3 +64,20 @@ def test_c_consumer_full_search(tmp_path):
     ref = oracle.cv_sorted(x, y, h, oracle.EPANECHNIKOV)
     assert int(mt.group(1)) == ref.best
     assert abs(float(mt.group(3)) - ref.cv[ref.best]) <= 1e-9 * ref.cv[ref.best]
+    from tests.helpers import cv_rel_err
+
+    curve = [ln.split() for ln in p.stdout.splitlines() if ln.startswith("curve ")]
+    assert [int(c[1]) for c in curve] == list(range(m))
+    cv = np.array([float(c[2]) for c in curve])
+    neff = np.array([int(c[3]) for c in curve])
+    assert cv_rel_err(cv, ref.cv) <= 1e-10
+    assert np.array_equal(neff, ref.neff)
+    ci = [ln.split() for ln in p.stdout.splitlines() if ln.startswith("ci ")]
+    assert [int(c[1]) for c in ci] == list(range(n))
+    est = np.array([float(c[2]) for c in ci])
+    se = np.array([float(c[3]) for c in ci])
+    jk = oracle.nw_jackknife(x, y, float(h[ref.best]), oracle.EPANECHNIKOV)
+    assert np.max(np.abs(est - jk.est) / np.abs(jk.est)) <= 1e-10
+    ok = ~np.isnan(jk.se)
+    assert np.array_equal(np.isnan(se), ~ok)
+    assert np.max(np.abs(se[ok] - jk.se[ok]) / jk.se[ok]) <= 1e-10
