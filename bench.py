@@ -375,11 +375,11 @@ def run_ours(args):
             return statistics.median(starts[s].elapsed_time(ends[s]) for s in range(nsteps)), st, launches, clk
 
         krcv.kr_profile_enable(False)
-        plan = GridSearch(n, h, k, device=dev, rank=rank, world=world, algo=algo, graph=(world == 1),
+        plan = GridSearch(n, h, k, device=dev, rank=rank, world=world, algo=algo, graph=True,
                           balance=(world > 1))
         step_ms, _, launches, clk = run_steps(plan, False)
         krcv.kr_profile_enable(True)
-        pplan = GridSearch(n, h, k, device=dev, rank=rank, world=world, algo=algo, graph=(world == 1),
+        pplan = GridSearch(n, h, k, device=dev, rank=rank, world=world, algo=algo, graph=True,
                           balance=(world > 1))
         prof_step_ms, st, _, _ = run_steps(pplan, True)
         krcv.kr_profile_enable(False)
@@ -436,10 +436,13 @@ def run_ours(args):
             "timing_stat": "median over the K timed steps",
             "result": {"best": res.best, "h_best": float(h[res.best]), "cv_best": float(res.cv[res.best])},
             "clocks": clk.summary(), "gpu_launches": launches, "plan": plan,
+            "launch": ("CUDA graph replay of the whole step" + (" incl. the NCCL all-reduce" if world > 1 else "")
+                       if plan.graph else f"eager enqueue per step (graph capture refused: {plan.graph_error})"),
         }
 
     main = timed(args.algo)
     plan = main.pop("plan")
+    main_launch = main.pop("launch")
 
     # ---- end-to-end through the public API, host buffers, H2D/D2H inside
     e2e = e2e_measure(args, x, y, h, k, n, m, units, dev, rank, world, plan)
@@ -454,8 +457,7 @@ def run_ours(args):
                        " (cost-balanced cuts from rank 0's calibration in the first warm-up step)"
                        f" + {os.environ.get('KRCV_BENCH_BACKEND', 'nccl')} all_reduce(2m+2 fp64)" if world > 1 else ""),
                    "l2": "flushed between timed steps (256 MiB write, outside the events)",
-                   "launch": ("CUDA graph replay of the whole search (GridSearch(graph=True))" if world == 1
-                              else "eager enqueue per step")},
+                   "launch": main_launch},
         "algo": main["algo"],
         "roofline": main["roofline"],
         "stage_ms": main["stage_ms"],
@@ -470,6 +472,7 @@ def run_ours(args):
         other = "sweep" if main["algo"] == "prefix" else "prefix"
         alt = timed(other)
         alt.pop("plan")
+        alt.pop("launch")
         out["alt_algo"] = {key: alt[key] for key in ("algo", "value", "ms_per_step", "stage_ms", "roofline",
                                                       "result", "clocks")}
     if world == 1 and args.config == "C2" and not args.no_extra:
@@ -510,6 +513,7 @@ def bench_extra_configs(args, timed, dev, krcv, torch):
               "d_y": torch.as_tensor(y, device=dev), "units": n * (n - 1) * m, "rows_mine": n}
         r = timed("auto", wl, steps=5 if name == "C4" else 10, warmup=3)
         r.pop("plan")
+        r.pop("launch")
         # window-stage balance of 8 equal row shards
         d_h = torch.as_tensor(h, device=dev)
         ws = krcv.aligned(krcv.workspace(n, m, dev))

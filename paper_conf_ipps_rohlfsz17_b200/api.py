@@ -45,6 +45,14 @@ def allreduce_partial(partial, group=None) -> None:
         dist.all_reduce(partial, op=dist.ReduceOp.SUM, group=group)
 
 
+def _nccl_group(group=None) -> bool:
+    """True when torch.distributed is initialised with an NCCL group (whose
+    collectives a CUDA graph can capture)."""
+    import torch.distributed as dist
+
+    return bool(dist.is_available() and dist.is_initialized() and dist.get_backend(group) == "nccl")
+
+
 def finalize_partial(partial, n: int, m: int):
     """CV = S/n, n_eff and the arg-min from a reduced partial vector.  CUDA
     tensors are finalized on the device (kr_finalize_async), CPU tensors with
@@ -113,10 +121,15 @@ class GridSearch:
         if estimator not in ("nw", "ll"):
             raise ValueError("estimator must be 'nw' (Nadaraya-Watson, Eq.(2)) or 'll' (local-linear, reading Q25)")
         self.estimator = estimator
-        # graph=True (single GPU): the enqueued pipeline is captured once per
-        # (x, y) pointer pair as a CUDA graph and replayed -- one launch for
-        # the whole search instead of one per stage
-        self.graph = bool(graph) and int(world) == 1
+        # graph=True: the enqueued pipeline is captured once per (x, y) pointer
+        # pair as a CUDA graph and replayed -- one launch for the whole search
+        # instead of one per stage.  With world > 1 (NCCL process group) the
+        # captured step includes the shard's pipeline, the NCCL all-reduce of
+        # the partial vector and the finalize; if the capture is refused (a
+        # non-NCCL group, an NCCL/driver without graph support) the plan falls
+        # back to eager enqueue and says so in self.graph_error.
+        self.graph = bool(graph) and (int(world) == 1 or _nccl_group(group))
+        self.graph_error = None
         self._g = None
         self._gkey = None
         self.rank, self.world, self.group = int(rank), int(world), group
@@ -143,13 +156,23 @@ class GridSearch:
             torch = self.torch
             key = (d_x.data_ptr(), d_y.data_ptr())
             if self._g is None or self._gkey != key:
-                self._enqueue(d_x, d_y)  # eager first: one-time launch configuration queries
+                # eager first: one-time launch configuration queries (and, for
+                # world > 1 with balance, the cost calibration and broadcast)
+                self._enqueue(d_x, d_y)
                 cur = torch.cuda.current_stream(self.device)
                 side = torch.cuda.Stream(self.device)
                 side.wait_stream(cur)
                 g = torch.cuda.CUDAGraph()
-                with torch.cuda.graph(g, stream=side, capture_error_mode="thread_local"):
+                try:
+                    with torch.cuda.graph(g, stream=side, capture_error_mode="thread_local"):
+                        self._enqueue(d_x, d_y)
+                except Exception as e:  # noqa: BLE001 -- capture refused: eager from now on
+                    if self.world == 1:
+                        raise
+                    cur.wait_stream(side)
+                    self.graph, self._g, self.graph_error = False, None, f"{type(e).__name__}: {e}"
                     self._enqueue(d_x, d_y)
+                    return
                 cur.wait_stream(side)
                 self._g, self._gkey = g, key
             self._g.replay()

@@ -735,13 +735,13 @@ static Win2Shape win2_shape(int64_t rows, int m)
     const int resident = occupancy((const void *)win_kernel<KERN>, kWin2Threads);
     const int64_t slots = (int64_t)dev_info().sms * resident * kWin2Warps;
     const int64_t target = kWin2TasksPerWarp * slots;
-    int64_t bc = (int64_t)m * ((w.ntiles + 1) / 2) / (target > 0 ? target : 1);
+    int64_t bc = (int64_t)m * ((w.ntiles + kWin2Rows - 1) / kWin2Rows) / (target > 0 ? target : 1);
     bc = bc < 1 ? 1 : (bc > kWin2Chunk ? kWin2Chunk : bc);
     if (bc > m) bc = m;
     w.BC = (int)bc;
     w.nbc = (int)((m + bc - 1) / bc);
     // no more slots than tasks (a slot without a task would leave its partials unwritten)
-    const int64_t tasks = (int64_t)((w.ntiles + 1) / 2) * w.nbc;
+    const int64_t tasks = (int64_t)((w.ntiles + kWin2Rows - 1) / kWin2Rows) * w.nbc;
     int64_t blocks = (int64_t)dev_info().sms * resident;
     if (blocks * kWin2Warps > win2_max_slots()) blocks = win2_max_slots() / kWin2Warps;
     if (blocks * kWin2Warps > tasks) blocks = tasks / kWin2Warps;
@@ -1014,7 +1014,7 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     const int winK = ll ? 1 : win_rows_per_lane(hi - lo);
     const int rows_per_tile = 32 * win_lane_rows(winK);
     const int ntiles = hist ? (int)((hi - lo + 31) / 32)
-                     : win2 ? (w2.ntiles + 1) / 2  // win_kernel tasks per chunk: tile pairs
+                     : win2 ? (w2.ntiles + kWin2Rows - 1) / kWin2Rows  // win_kernel tasks per chunk
                      : prefix ? (int)((hi - lo + rows_per_tile - 1) / rows_per_tile)
                               : dense ? (int)tiles_for(hi - lo, 1)
                                       : (variant == 1 ? (int)tiles_for(hi - lo, 1) : (int)tiles_for(hi - lo, G));

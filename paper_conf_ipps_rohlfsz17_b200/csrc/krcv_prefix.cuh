@@ -150,10 +150,18 @@ __device__ __forceinline__ void moment_terms(double x, double y, double o, dd (&
 // The KDE and local-linear sets keep structure-of-arrays planes (hi of moment
 // k at P + 2k ps, lo at P + (2k+1) ps).
 constexpr int kRecBlock = 1024;
+// KRCV_REC_AOS=1 (build time, A/B runs): records as an array of structures of
+// S + 1 doubles (the moments, then the index j as a double) instead of the
+// blocked planes.
+#ifndef KRCV_REC_AOS
+#define KRCV_REC_AOS 0
+#endif
+constexpr bool kRecAos = KRCV_REC_AOS != 0;
 
 template <int KERN>
 struct PfxRec {
-    static constexpr int S = KERN == KR_EPANECHNIKOV ? 5 : (KERN == KR_TRIANGULAR ? 3 : (KERN == KR_UNIFORM ? 1 : 0));
+    static constexpr int S0 = KERN == KR_EPANECHNIKOV ? 5 : (KERN == KR_TRIANGULAR ? 3 : (KERN == KR_UNIFORM ? 1 : 0));
+    static constexpr int S = (kRecAos && S0) ? S0 + 1 : S0;  // doubles per index (AoS: + the index slot)
     static constexpr int BS = S * kRecBlock;  // doubles per block (all planes)
     // plane of slot k: width 2 for slots 0..2*(S/2)-1, width 1 for the odd last slot
     static __host__ __device__ constexpr int width(int k) { return k < 2 * (S / 2) ? 2 : 1; }
@@ -180,6 +188,7 @@ template <int KERN>
 __device__ __forceinline__ size_t pk_off(int k, int j)
 {
     using R = PfxRec<KERN>;
+    if (kRecAos) return (size_t)j * R::S + k;
     const unsigned u = (unsigned)j;
     return (size_t)(u >> 10) * (unsigned)R::BS +
            (size_t)((u & (kRecBlock - 1)) * (unsigned)R::width(k) + (unsigned)(R::plane_off(k) + R::sub(k)));
@@ -194,6 +203,17 @@ __device__ __forceinline__ void pk_store(double *__restrict__ P, int ps, int k, 
     } else {
         P[(size_t)(2 * k) * ps + j] = v.hi;
         P[(size_t)(2 * k + 1) * ps + j] = v.lo;
+    }
+}
+
+// the AoS layout's index slot (the blocked layout has none)
+template <int KERN>
+__device__ __forceinline__ void pk_store_index(double *__restrict__ P, int ps, int j)
+{
+    constexpr int S = PfxRec<KERN>::S;
+    if (kRecAos && S) {
+        P[(size_t)j * S + S - 1] = (double)j;
+        P[pk_lo_off<KERN>(ps) + (size_t)j * S + S - 1] = 0.0;
     }
 }
 
@@ -387,6 +407,7 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
         for (int q = 0; q < ITEMS; q++) {
             if (j0 + q <= n) {
                 pk_store<KERN>(P, pstride, k, j0 + q, run);
+                if (k == 0) pk_store_index<KERN>(P, pstride, j0 + q);
             }
             run = dd_add(run, tm[q][k]);
         }
@@ -482,10 +503,12 @@ pfx_one_cta_kernel(const double2 *__restrict__ xy, int n, double *__restrict__ P
             pk_store<KERN>(P, pstride, k, j, run[k]);
             run[k] = dd_add(run[k], tm[k]);
         }
+        pk_store_index<KERN>(P, pstride, j);
     }
     if (j1 == n && j0 < n) {  // the thread holding the last record writes P[k][n]
 #pragma unroll
         for (int k = 0; k < K; k++) pk_store<KERN>(P, pstride, k, n, run[k]);
+        pk_store_index<KERN>(P, pstride, n);
     }
 }
 
@@ -602,8 +625,12 @@ __device__ __forceinline__ dd wsum(const double *__restrict__ P, int ps, int k, 
 // a / b for finite b != 0 with normal 1/b: hardware reciprocal estimate, two
 // Newton steps and one residual correction -- within 1 ulp of the correctly
 // rounded quotient, branch-free (IEEE division adds a slow-path test).
+#ifndef KRCV_FASTDIV
+#define KRCV_FASTDIV 1
+#endif
 __device__ __forceinline__ double fast_div(double a, double b)
 {
+    if (!KRCV_FASTDIV) return a / b;
     double r;
     asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(b));
     double e = fma(-b, r, 1.0);
@@ -653,15 +680,25 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
             // 8-byte load each, fixed offsets from one address
             const double *pr = P + pk_off<KERN>(0, R);
             const double *pa = P + pk_off<KERN>(0, A);
+            const int q2 = kRecAos ? 2 : 2 * kRecBlock;  // offset of the (u^2, y u) pair
             const double2 r01 = __ldg(reinterpret_cast<const double2 *>(pr));
-            const double2 r23 = __ldg(reinterpret_cast<const double2 *>(pr + 2 * kRecBlock));
+            const double2 r23 = __ldg(reinterpret_cast<const double2 *>(pr + q2));
             const double2 a01 = __ldg(reinterpret_cast<const double2 *>(pa));
-            const double2 a23 = __ldg(reinterpret_cast<const double2 *>(pa + 2 * kRecBlock));
-            const double yuu_b = __ldg(pr + 4 * kRecBlock - (int)((unsigned)R & (kRecBlock - 1))),
-                         yuu_a = __ldg(pa + 4 * kRecBlock - (int)((unsigned)A & (kRecBlock - 1)));
+            const double2 a23 = __ldg(reinterpret_cast<const double2 *>(pa + q2));
+            double yuu_b, yuu_a, c1;
+            if (kRecAos) {  // (y u^2, j) pair: the count is a difference of loaded slots
+                const double2 r45 = __ldg(reinterpret_cast<const double2 *>(pr + 4));
+                const double2 a45 = __ldg(reinterpret_cast<const double2 *>(pa + 4));
+                yuu_b = r45.x;
+                yuu_a = a45.x;
+                c1 = r45.y - a45.y;
+            } else {
+                yuu_b = __ldg(pr + 4 * kRecBlock - (int)((unsigned)R & (kRecBlock - 1)));
+                yuu_a = __ldg(pa + 4 * kRecBlock - (int)((unsigned)A & (kRecBlock - 1)));
+                c1 = (double)(c + 1);  // range count R - A, row r included (its terms vanish)
+            }
             const double y_b = r01.x, y_a = a01.x, u_b = r01.y, u_a = a01.y;
             const double uu_b = r23.x, uu_a = a23.x, yu_b = r23.y, yu_a = a23.y;
-            const double c1 = (double)(c + 1);  // range count R - A, row r included (its terms vanish)
             const double Sy = y_b - y_a, Su = u_b - u_a, Suu = uu_b - uu_a;
             const double Syu = yu_b - yu_a, Syuu = yuu_b - yuu_a;
             s1 = fma(-dl, fma(-c1, dl, 2.0 * Su), Suu);
@@ -682,15 +719,16 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
                 // the records' hi and lo words at fixed offsets from two addresses
                 const size_t lo = pk_lo_off<KERN>(ps);
                 const double *pr = P + pk_off<KERN>(0, R), *pa = P + pk_off<KERN>(0, A);
-                const int orr = 4 * kRecBlock - (int)((unsigned)R & (kRecBlock - 1));
-                const int oaa = 4 * kRecBlock - (int)((unsigned)A & (kRecBlock - 1));
+                const int q2 = kRecAos ? 2 : 2 * kRecBlock;
+                const int orr = kRecAos ? 4 : 4 * kRecBlock - (int)((unsigned)R & (kRecBlock - 1));
+                const int oaa = kRecAos ? 4 : 4 * kRecBlock - (int)((unsigned)A & (kRecBlock - 1));
                 auto wd = [&](int offr, int offa) {
                     return dd_sub(dd{pr[offr], pr[lo + offr]}, dd{pa[offa], pa[lo + offa]});
                 };
                 const dd Sy = wd(0, 0);
                 const dd Su = wd(1, 1);
-                const dd Suu = wd(2 * kRecBlock, 2 * kRecBlock);
-                const dd Syu = wd(2 * kRecBlock + 1, 2 * kRecBlock + 1);
+                const dd Suu = wd(q2, q2);
+                const dd Syu = wd(q2 + 1, q2 + 1);
                 const dd Syuu = wd(orr, oaa);
                 const dd t1 = dd_sub(dd_twice(Su), dd_mul_d_raw(del, (double)(c + 1)));
                 s1 = dd_sub_to_d(Suu, dd_mul_raw(del, t1));

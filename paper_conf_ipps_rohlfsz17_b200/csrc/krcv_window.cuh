@@ -46,6 +46,9 @@
 namespace krcv {
 
 constexpr int kBktFmax = 32;             // buckets per point, at most
+#ifndef KRCV_BKT_FX
+#define KRCV_BKT_FX 1.0                  // (build-time A/B) buckets per point at the peak density
+#endif
 constexpr int64_t kBktQmax = 1LL << 28;  // buckets, at most
 constexpr double kBktMagic = 6755399441055744.0;  // 1.5 * 2^52: fma(.) + magic keeps the integer in the low word
 constexpr int kBktFillThreads = 256;
@@ -79,7 +82,7 @@ __device__ __forceinline__ BktParams bkt_params(const double *__restrict__ xs, i
         // F = the next power of two, at most one point per bucket where the data
         // is densest (uniform x: F = 2; a larger table costs L2 capacity, which
         // the C4 working set needs -- profiles/r02f_*)
-        const double ratio = gap > 0.0 ? (double)kGapSpan * span / (gap * (double)(n - 1)) : 1e300;
+        const double ratio = gap > 0.0 ? KRCV_BKT_FX * (double)kGapSpan * span / (gap * (double)(n - 1)) : 1e300;
         while (F < kBktFmax && (double)F < ratio) F <<= 1;
     }
     int64_t Q = (int64_t)F * n;
@@ -175,6 +178,10 @@ __device__ __forceinline__ int first_true(Pred p, int lo, int hi, int k0)
 
 constexpr int kWin2Warps = 4;
 constexpr int kWin2Threads = kWin2Warps * 32;
+#ifndef KRCV_WIN2_ROWS
+#define KRCV_WIN2_ROWS 2
+#endif
+constexpr int kWin2Rows = KRCV_WIN2_ROWS;  // tiles of 32 rows per task = rows per lane (1 or 2)
 constexpr int kWin2Chunk = 32;  // bandwidths per task, at most (lane (b - b0) keeps bandwidth b's running sum)
 // CTAs per SM the register allocation must allow: 8 -> 64 registers, 32
 // warps per SM (measured faster than 6 -> 80 and 4 -> 128 registers: the
@@ -244,9 +251,9 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
     const double xmin = xs[0], xmax = xs[n - 1];
     const double invw = prm->invw, C = prm->C;
     const int Q = prm->Q;
-    // a task is a pair of adjacent tiles (64 rows): two rows per lane share
-    // one butterfly per bandwidth
-    const int npairs = (ntiles + 1) / 2;
+    // a task is kWin2Rows adjacent tiles (2: 64 rows, two rows per lane
+    // sharing one butterfly per bandwidth)
+    const int npairs = (ntiles + kWin2Rows - 1) / kWin2Rows;
     const int64_t ntasks = (int64_t)npairs * nbc;
     int cur = -1;  // chunk of the running sums
     double acc = 0.0;
@@ -266,10 +273,10 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
         const int t = (int)(k - (int64_t)chunk * npairs);
         const int b0 = chunk * BC, b1 = min(m, b0 + BC);
         WinRow w0, w1;
-        bool v0, v1;
-        double dmax0, dmin0, dmax1, dmin1;
+        bool v0, v1 = false;
+        double dmax0, dmin0, dmax1 = 0.0, dmin1 = 0.0;
         {
-            const int i = row_lo + t * 64 + lane;
+            const int i = row_lo + t * 32 * kWin2Rows + lane;
             v0 = i < row_hi;
             w0.r = v0 ? i : row_hi - 1;  // clamped rows do identical work, discarded
             const double2 v = xy[w0.r];
@@ -279,7 +286,7 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
             dmax0 = xmax - v.x;
             dmin0 = v.x - xmin;
         }
-        {
+        if (kWin2Rows == 2) {
             const int i = row_lo + t * 64 + 32 + lane;
             v1 = i < row_hi;
             w1.r = v1 ? i : row_hi - 1;
@@ -294,9 +301,12 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
             const double h = __ldg(hg + b);
             bool M0, M1;
             double e2 = row_e2<KERN>(w0, v0, dmax0, dmin0, h, xs, xy, P, pstride, BT, invw, C, Q, n, ymax, M0);
-            e2 += row_e2<KERN>(w1, v1, dmax1, dmin1, h, xs, xy, P, pstride, BT, invw, C, Q, n, ymax, M1);
-            e2 = warp_sum(e2);  // fixed butterfly: every lane holds the pair's sum
-            const uint32_t nb = __popc(__ballot_sync(0xffffffffu, M0)) + __popc(__ballot_sync(0xffffffffu, M1));
+            M1 = false;
+            if (kWin2Rows == 2)
+                e2 += row_e2<KERN>(w1, v1, dmax1, dmin1, h, xs, xy, P, pstride, BT, invw, C, Q, n, ymax, M1);
+            e2 = warp_sum(e2);  // fixed butterfly: every lane holds the task's sum
+            const uint32_t nb = __popc(__ballot_sync(0xffffffffu, M0)) +
+                                (kWin2Rows == 2 ? __popc(__ballot_sync(0xffffffffu, M1)) : 0u);
             if (lane == b - b0) {
                 acc += e2;
                 cnt += nb;
