@@ -1,0 +1,13 @@
+#!/bin/bash
+# r02p: a5 (column sums + finalize) fused into win_kernel via per-chunk completion counters
+set -u
+OUT=gpurun_out; mkdir -p $OUT
+python -c "import __graft_entry__ as g; g.build()" > $OUT/r02p_build.log 2>&1
+timeout 1500 python -m pytest tests/test_gpu_parity.py tests/test_gpu_window_variants.py tests/test_gpu_distributed.py tests/test_gpu_faults.py tests/test_gpu_baseline_curves.py tests/test_gpu_host_path.py -m gpu -x -q -p no:cacheprovider > $OUT/r02p_pytest.log 2>&1; echo "exit $?" >> $OUT/r02p_pytest.log
+for C in C2 C3 C4 C5; do
+  timeout 300 python bench.py --config $C --no-alt --no-cpu-baseline --no-extra --steps 10 --warmup 3 > $OUT/r02p_bench_$C.json 2> $OUT/r02p_bench_$C.err
+done
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/r02p_launches_C2.csv \
+    python bench.py --steps 2 --warmup 1 --no-alt --no-cpu-baseline --no-extra > $OUT/r02p_launch_bench.log 2>&1
+OMP_NUM_THREADS=1 timeout 600 python tools/oracle_single_thread.py --out $OUT/r02p_oracle_single_thread.json > $OUT/r02p_oracle_1t.log 2>&1
+echo done
