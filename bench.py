@@ -437,7 +437,9 @@ def run_ours(args):
             "result": {"best": res.best, "h_best": float(h[res.best]), "cv_best": float(res.cv[res.best])},
             "clocks": clk.summary(), "gpu_launches": launches, "plan": plan,
             "launch": ("CUDA graph replay of the whole step" + (" incl. the NCCL all-reduce" if world > 1 else "")
-                       if plan.graph else f"eager enqueue per step (graph capture refused: {plan.graph_error})"),
+                       if plan.graph else
+                       (f"eager enqueue per step (graph capture refused: {plan.graph_error})" if plan.graph_error
+                        else "eager enqueue per step (non-NCCL process group: collectives not capturable)")),
         }
 
     main = timed(args.algo)

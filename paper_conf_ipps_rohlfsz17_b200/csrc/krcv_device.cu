@@ -619,8 +619,13 @@ static int pfx_items(int n)
     return n <= kPfxOneCtaMax ? 0 : (n <= (1 << 18) ? 1 : kPfxItemsMax);
 }
 
+static void launch_bkt_fill(int n, const WsLayout &L, char *ws, cudaStream_t st);
+
+// The O(n) build of the window-prefix path: prefix moments, xs and (table:
+// win_kernel's) the bucket table.  Returns the launches enqueued.
 template <int KERN>
-static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, char *ws, cudaStream_t st)
+static int launch_prefix_build(const double2 *xy, int n, const WsLayout &L, char *ws, cudaStream_t st,
+                               bool table = false)
 {
     double *xs = reinterpret_cast<double *>(ws + L.xs) + kPad;
     double *P = reinterpret_cast<double *>(ws + L.pfx);
@@ -628,8 +633,20 @@ static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, cha
     unsigned long long *ymax = reinterpret_cast<unsigned long long *>(ws + L.status + 4 * sizeof(unsigned));
     unsigned long long *gap = reinterpret_cast<unsigned long long *>(ws + L.status + 6 * sizeof(unsigned));
     const int items = pfx_items(n);
+    const int tiles1 = (n + kPfxThreads) / kPfxThreads;  // 256-record tiles covering P[0..n]
+    if (items == 1 && PfxRec<KERN>::S && tiles1 <= dev_info().sms && !getenv_flag("KRCV_PFX_UNFUSED")) {
+        // every tile co-resident (<= one CTA per SM): the fused build
+        unsigned *arrive = reinterpret_cast<unsigned *>(ws + L.status) + 3;  // zeroed by the status memset
+        int *BT = table ? reinterpret_cast<int *>(ws + L.bt) : nullptr;
+        BktParams *prm = reinterpret_cast<BktParams *>(ws + L.status + 32);
+        launch_pdl(pfx_fused_kernel<KERN>, dim3(tiles1), dim3(kFusedPfxThreads), 0, st, xy, n, tot, tiles1, ymax,
+                   gap, P, (int)L.pstride, xs, BT, prm, arrive);
+        return 1;
+    }
+    int launches = 2;
     if (items == 0) {
         pfx_one_cta_kernel<KERN><<<1, kPfx1Threads, 0, st>>>(xy, n, P, (int)L.pstride, xs, ymax, gap);
+        launches = 1;
     } else if (items == 1) {
         const int ntiles = (n + kPfxThreads) / kPfxThreads;  // tiles covering P[0..n]
         launch_pdl(pfx_tile_reduce_kernel<KERN, 1>, dim3(ntiles), dim3(kPfxThreads), 0, st, xy, n, tot, ntiles, ymax);
@@ -642,6 +659,11 @@ static void launch_prefix_build(const double2 *xy, int n, const WsLayout &L, cha
         launch_pdl(pfx_tile_scan_kernel<KERN, kPfxItemsMax>, dim3(ntiles), dim3(kPfxThreads), 0, st, xy, n,
                    (const double2 *)tot, ntiles, P, (int)L.pstride, xs, gap);
     }
+    if (table) {
+        launch_bkt_fill(n, L, ws, st);
+        launches += 1;
+    }
+    return launches;
 }
 
 // Window kernel of r01 (window_kernel<K> / window_kernel_b2), kept for A/B
@@ -1040,15 +1062,11 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         launch_prefix_build<kLLMoments>(xy, nn, L, ws, st);
         launches += 2;
     } else if (prefix && !reuse_sorted) {
+        // win_kernel's bucket table is part of the build (depends on xs only: kept on reuse)
         switch (kernel) {
-        case KR_UNIFORM: launch_prefix_build<KR_UNIFORM>(xy, nn, L, ws, st); break;
-        case KR_EPANECHNIKOV: launch_prefix_build<KR_EPANECHNIKOV>(xy, nn, L, ws, st); break;
-        default: launch_prefix_build<KR_TRIANGULAR>(xy, nn, L, ws, st); break;
-        }
-        launches += 2;
-        if (win2) {  // win_kernel's bucket table (depends on xs only: kept on reuse)
-            launch_bkt_fill(nn, L, ws, st);
-            launches += 1;
+        case KR_UNIFORM: launches += launch_prefix_build<KR_UNIFORM>(xy, nn, L, ws, st, win2); break;
+        case KR_EPANECHNIKOV: launches += launch_prefix_build<KR_EPANECHNIKOV>(xy, nn, L, ws, st, win2); break;
+        default: launches += launch_prefix_build<KR_TRIANGULAR>(xy, nn, L, ws, st, win2); break;
         }
     }
     prof_mark(2, st);

@@ -276,6 +276,16 @@ __device__ __forceinline__ dd shfl_xor_dd(dd v, int d)
     return dd{__shfl_xor_sync(0xffffffffu, v.hi, d), __shfl_xor_sync(0xffffffffu, v.lo, d)};
 }
 
+template <int KERN, int ITEMS, bool GAP>
+__device__ __forceinline__ void pfx_reduce_body(const double2 *__restrict__ xy, int n, double2 *__restrict__ tot,
+                                                int ntiles, unsigned long long *__restrict__ ymax_bits,
+                                                unsigned long long *__restrict__ gap_bits, int tile);
+template <int KERN, int ITEMS, bool GAP, bool CG>
+__device__ __forceinline__ void pfx_scan_body(const double2 *__restrict__ xy, int n, const double2 *__restrict__ tot,
+                                              int ntiles, double *__restrict__ P, int pstride,
+                                              double *__restrict__ xs, unsigned long long *__restrict__ gap_bits,
+                                              int tile);
+
 // Phase 1: per-tile totals of the moment terms -> tot[k][tile].
 template <int KERN, int ITEMS>
 __global__ void __launch_bounds__(kPfxThreads)
@@ -283,20 +293,31 @@ pfx_tile_reduce_kernel(const double2 *__restrict__ xy, int n, double2 *__restric
                        unsigned long long *__restrict__ ymax_bits)
 {
     pdl_wait();  // krcv_pdl.cuh
+    pfx_reduce_body<KERN, ITEMS, false>(xy, n, tot, ntiles, ymax_bits, nullptr, blockIdx.x);
+}
+
+// Phase 1 body (also used by the fused build, krcv_window.cuh): tile `tile`'s
+// dd totals -> tot[k][tile], max|y|, and with GAP the density statistic.
+template <int KERN, int ITEMS, bool GAP>
+__device__ __forceinline__ void pfx_reduce_body(const double2 *__restrict__ xy, int n, double2 *__restrict__ tot,
+                                                int ntiles, unsigned long long *__restrict__ ymax_bits,
+                                                unsigned long long *__restrict__ gap_bits, int tile)
+{
     constexpr int K = NMom<KERN>::v;
     __shared__ double2 wsum[K][kPfxThreads / 32];
     const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-    const int j0 = blockIdx.x * (kPfxThreads * ITEMS) + t * ITEMS;
+    const int j0 = tile * (kPfxThreads * ITEMS) + t * ITEMS;
     const double o = pfx_origin(xy, n);
     dd acc[kPfxMoments];
 #pragma unroll
     for (int k = 0; k < K; k++) acc[k] = dd{0.0, 0.0};
-    double ym = 0.0;
+    double ym = 0.0, gmin = INFINITY;
 #pragma unroll
     for (int q = 0; q < ITEMS; q++) {
         if (j0 + q < n) {
             const double2 v = xy[j0 + q];
             ym = fmax(ym, fabs(v.y));
+            if (GAP && PfxRec<KERN>::S) gap_stat(xy, n, j0 + q, gmin);
             dd tm[kPfxMoments];
             moment_terms<KERN>(v.x, v.y, o, tm);
 #pragma unroll
@@ -314,11 +335,12 @@ pfx_tile_reduce_kernel(const double2 *__restrict__ xy, int n, double2 *__restric
 #pragma unroll
     for (int d = 16; d > 0; d >>= 1) ym = fmax(ym, __shfl_xor_sync(0xffffffffu, ym, d));
     if (lane == 0 && ym > 0.0) atomicMax(ymax_bits, (unsigned long long)__double_as_longlong(ym));
+    if (GAP && PfxRec<KERN>::S) gap_publish(gmin, gap_bits);
     __syncthreads();
     if (t < K) {
         dd a = dd{0.0, 0.0};
         for (int q = 0; q < kPfxThreads / 32; q++) a = dd_add(a, ld_dd(&wsum[t][q]));
-        st_dd(tot + (size_t)t * ntiles + blockIdx.x, a);
+        st_dd(tot + (size_t)t * ntiles + tile, a);
     }
 }
 
@@ -332,6 +354,18 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
                      unsigned long long *__restrict__ gap_bits)
 {
     pdl_wait();  // krcv_pdl.cuh
+    pfx_scan_body<KERN, ITEMS, true, false>(xy, n, tot, ntiles, P, pstride, xs, gap_bits, blockIdx.x);
+}
+
+// Phase 3 body (also used by the fused build): tile `tile`'s offset, scan,
+// records and xs; GAP: the density statistic here; CG: read the other tiles'
+// totals through L2 (they were written in this same launch).
+template <int KERN, int ITEMS, bool GAP, bool CG>
+__device__ __forceinline__ void pfx_scan_body(const double2 *__restrict__ xy, int n, const double2 *__restrict__ tot,
+                                              int ntiles, double *__restrict__ P, int pstride,
+                                              double *__restrict__ xs, unsigned long long *__restrict__ gap_bits,
+                                              int tile)
+{
     constexpr int K = NMom<KERN>::v;
     __shared__ double2 wsum[K][kPfxThreads / 32];
     __shared__ double2 base_s[K];
@@ -343,7 +377,10 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
 #pragma unroll
         for (int k = 0; k < K; k++) {
             a[k] = dd{0.0, 0.0};
-            for (int q = t; q < (int)blockIdx.x; q += kPfxThreads) a[k] = dd_add(a[k], ld_dd(tot + (size_t)k * ntiles + q));
+            for (int q = t; q < tile; q += kPfxThreads) {
+                const double2 *pq = tot + (size_t)k * ntiles + q;
+                a[k] = dd_add(a[k], CG ? dd{__ldcg(&pq->x), __ldcg(&pq->y)} : ld_dd(pq));
+            }
 #pragma unroll
             for (int d = 16; d > 0; d >>= 1) a[k] = dd_add(a[k], shfl_xor_dd(a[k], d));
             if (lane == 0) st_dd(&wsum[k][w], a[k]);
@@ -357,8 +394,8 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
         __syncthreads();
     }
     const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-    const int j0 = blockIdx.x * (kPfxThreads * ITEMS) + t * ITEMS;
-    if (blockIdx.x == 0 && t < kPad) {
+    const int j0 = tile * (kPfxThreads * ITEMS) + t * ITEMS;
+    if (tile == 0 && t < kPad) {
         xs[-1 - t] = -INFINITY;
         xs[n + t] = INFINITY;
     }
@@ -373,7 +410,7 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
         if (j0 + q < n) {
             const double2 v = xy[j0 + q];
             xs[j0 + q] = v.x;
-            if (PfxRec<KERN>::S) gap_stat(xy, n, j0 + q, gmin);
+            if (GAP && PfxRec<KERN>::S) gap_stat(xy, n, j0 + q, gmin);
             moment_terms<KERN>(v.x, v.y, o, tm[q]);
         } else {
 #pragma unroll
@@ -382,7 +419,7 @@ pfx_tile_scan_kernel(const double2 *__restrict__ xy, int n, const double2 *__res
 #pragma unroll
         for (int k = 0; k < K; k++) acc[k] = dd_add(acc[k], tm[q][k]);
     }
-    if (PfxRec<KERN>::S) gap_publish(gmin, gap_bits);
+    if (GAP && PfxRec<KERN>::S) gap_publish(gmin, gap_bits);
     // exclusive scan of the thread totals across the CTA
     dd ex[kPfxMoments];
 #pragma unroll

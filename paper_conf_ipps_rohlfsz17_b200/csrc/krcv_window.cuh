@@ -37,6 +37,7 @@
 
 #include <cuda_runtime.h>
 
+#include <climits>
 #include <cstdint>
 
 #include "krcv.h"
@@ -69,12 +70,10 @@ __device__ __forceinline__ int bkt_raw(double v, double invw, double C)
 }
 
 // Parameters of the table for this call: F from the peak density.
-__device__ __forceinline__ BktParams bkt_params(const double *__restrict__ xs, int n,
-                                                const unsigned long long *__restrict__ gap_bits)
+__device__ __forceinline__ BktParams bkt_params_of(double lo, double hi, int n, unsigned long long gb)
 {
     BktParams p;
-    const double lo = xs[0], span = xs[n - 1] - xs[0];
-    const unsigned long long gb = *gap_bits;
+    const double span = hi - lo;
     int F = 1;
     if (gb != 0ull && span > 0.0) {
         const double gap = __longlong_as_double((long long)~gb);  // min x-span of kGapSpan + 1 records
@@ -92,6 +91,71 @@ __device__ __forceinline__ BktParams bkt_params(const double *__restrict__ xs, i
     p.invw = span > 0.0 ? (double)Q / span : 0.0;
     p.C = kBktMagic - lo * p.invw;
     return p;
+}
+
+__device__ __forceinline__ BktParams bkt_params(const double *__restrict__ xs, int n,
+                                                const unsigned long long *__restrict__ gap_bits)
+{
+    return bkt_params_of(xs[0], xs[n - 1], n, *gap_bits);
+}
+
+// Fused O(n) build for a shard problem whose 256-record prefix tiles all fit
+// on the GPU at once (ntiles <= #SMs, so every CTA is co-resident): phase 1
+// (tile totals, max|y|, density statistic), a grid barrier (arrival counter,
+// zeroed by the call's status memset), phase 3 (the tile's offset from the
+// totals of the earlier tiles in fixed order, the scan, the records and xs --
+// the same bodies as pfx_tile_reduce_kernel / pfx_tile_scan_kernel, so the
+// records are bit-identical), then this tile's stretch of the bucket table:
+// q in (bkt(x_{j0-1}), bkt(x_{j1-1})] (from 0 for the first tile, to Q for
+// the last), BT[q] = the first of the tile's records with bucket >= q, by a
+// binary search over the tile's bucket ids in shared memory -- the same table
+// bkt_fill_kernel builds.  One launch instead of three.
+constexpr int kFusedPfxThreads = kPfxThreads;  // one record per thread (ITEMS = 1)
+
+__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned *p)
+{
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+template <int KERN>
+__global__ void __launch_bounds__(kFusedPfxThreads)
+pfx_fused_kernel(const double2 *__restrict__ xy, int n, double2 *__restrict__ tot, int ntiles,
+                 unsigned long long *__restrict__ ymax_bits, unsigned long long *__restrict__ gap_bits,
+                 double *__restrict__ P, int pstride, double *__restrict__ xs, int *__restrict__ BT,
+                 BktParams *__restrict__ prm, unsigned *__restrict__ arrive)
+{
+    pdl_wait();  // krcv_pdl.cuh
+    __shared__ int sA[kFusedPfxThreads];
+    pfx_reduce_body<KERN, 1, true>(xy, n, tot, ntiles, ymax_bits, gap_bits, blockIdx.x);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        atomicAdd(arrive, 1u);
+        while (ld_acquire_u32(arrive) < gridDim.x) __nanosleep(32);
+        __threadfence();
+    }
+    __syncthreads();
+    pfx_scan_body<KERN, 1, false, true>(xy, n, tot, ntiles, P, pstride, xs, gap_bits, blockIdx.x);
+    if (!BT) return;
+    const BktParams p = bkt_params_of(__ldg(&xy[0].x), __ldg(&xy[n - 1].x), n, __ldcg(gap_bits));
+    if (blockIdx.x == 0 && threadIdx.x == 0) *prm = p;
+    auto A = [&](double v) { return min(max(bkt_raw(v, p.invw, p.C), 0), p.Q); };
+    const int j0 = blockIdx.x * kFusedPfxThreads, j1 = min(j0 + kFusedPfxThreads, n), cnt = j1 - j0;
+    const int t = threadIdx.x;
+    sA[t] = t < cnt ? A(__ldg(&xy[j0 + t].x)) : INT_MAX;
+    __syncthreads();
+    const int qlo = j0 == 0 ? 0 : A(__ldg(&xy[j0 - 1].x)) + 1;
+    const int qhi = j1 == n ? p.Q : sA[cnt - 1];
+    for (int q = qlo + t; q <= qhi; q += kFusedPfxThreads) {
+        int lo = 0, hi = cnt;
+        while (lo < hi) {
+            const int mid = (lo + hi) >> 1;
+            if (sA[mid] >= q) hi = mid; else lo = mid + 1;
+        }
+        BT[q] = j0 + lo;
+    }
 }
 
 // BT[q] = #{k : bkt(xs[k]) < q} for q = 0 .. Q: the merge of the sorted
