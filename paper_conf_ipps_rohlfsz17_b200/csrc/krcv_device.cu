@@ -756,7 +756,12 @@ static Win2Shape win2_shape(int64_t rows, int m)
     w.ntiles = (int)((rows + 31) / 32);
     const int resident = occupancy((const void *)win_kernel<KERN>, kWin2Threads);
     const int64_t slots = (int64_t)dev_info().sms * resident * kWin2Warps;
-    const int64_t target = kWin2TasksPerWarp * slots;
+    static const int tpw = [] {  // KRCV_WIN2_TPW overrides (A/B runs)
+        const char *e = getenv("KRCV_WIN2_TPW");
+        const int v = e ? atoi(e) : 0;
+        return v > 0 ? v : kWin2TasksPerWarp;
+    }();
+    const int64_t target = (int64_t)tpw * slots;
     int64_t bc = (int64_t)m * ((w.ntiles + kWin2Rows - 1) / kWin2Rows) / (target > 0 ? target : 1);
     bc = bc < 1 ? 1 : (bc > kWin2Chunk ? kWin2Chunk : bc);
     if (bc > m) bc = m;
