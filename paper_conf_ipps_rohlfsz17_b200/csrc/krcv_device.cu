@@ -747,7 +747,13 @@ static bool use_win2()
 struct Win2Shape {
     int BC, nbc, ntiles, blocks, S;
 };
-constexpr int kWin2TasksPerWarp = 8;  // static round-robin: >= 8 tasks per slot keeps the tail short
+// Task shape (measured, profiles/r02/r02v_*): about 16 tasks per warp slot
+// (C3 1.192 -> 1.160 ms, C5 1.653 -> 1.600 ms against 8), but chunks of at
+// least 3 bandwidths (C2: 16 per slot would mean one-bandwidth tasks, whose
+// per-task row setup costs more than the balance gains: 65.5 -> 60.4 us
+// window at 3 bandwidths)
+constexpr int kWin2TasksPerWarp = 16;
+constexpr int kWin2MinChunk = 3;
 
 template <int KERN>
 static Win2Shape win2_shape(int64_t rows, int m)
@@ -763,7 +769,7 @@ static Win2Shape win2_shape(int64_t rows, int m)
     }();
     const int64_t target = (int64_t)tpw * slots;
     int64_t bc = (int64_t)m * ((w.ntiles + kWin2Rows - 1) / kWin2Rows) / (target > 0 ? target : 1);
-    bc = bc < 1 ? 1 : (bc > kWin2Chunk ? kWin2Chunk : bc);
+    bc = bc < kWin2MinChunk ? kWin2MinChunk : (bc > kWin2Chunk ? kWin2Chunk : bc);
     if (bc > m) bc = m;
     w.BC = (int)bc;
     w.nbc = (int)((m + bc - 1) / bc);

@@ -246,7 +246,11 @@ constexpr int kWin2Threads = kWin2Warps * 32;
 #define KRCV_WIN2_ROWS 2
 #endif
 constexpr int kWin2Rows = KRCV_WIN2_ROWS;  // tiles of 32 rows per task = rows per lane (1 or 2)
-constexpr int kWin2Chunk = 32;  // bandwidths per task, at most (lane (b - b0) keeps bandwidth b's running sum)
+#ifndef KRCV_WIN2_ACC
+#define KRCV_WIN2_ACC 1
+#endif
+constexpr int kWin2Acc = KRCV_WIN2_ACC;  // running sums per lane (build-time A/B: 1 or 2)
+constexpr int kWin2Chunk = 32 * kWin2Acc;  // bandwidths per task, at most (lane (b - b0) % 32 keeps b's sum)
 // CTAs per SM the register allocation must allow: 8 -> 64 registers, 32
 // warps per SM (measured faster than 6 -> 80 and 4 -> 128 registers: the
 // kernel is latency-bound, profiles/r02d_*, r02e_*).  KRCV_WIN2_MINB at build
@@ -320,19 +324,28 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
     const int npairs = (ntiles + kWin2Rows - 1) / kWin2Rows;
     const int64_t ntasks = (int64_t)npairs * nbc;
     int cur = -1;  // chunk of the running sums
-    double acc = 0.0;
-    uint32_t cnt = 0;
+    double acc[kWin2Acc];
+    uint32_t cnt[kWin2Acc];
+#pragma unroll
+    for (int a = 0; a < kWin2Acc; a++) {
+        acc[a] = 0.0;
+        cnt[a] = 0;
+    }
     for (int64_t k = slot;; k += S) {
         const int chunk = k < ntasks ? (int)(k / npairs) : nbc;  // warp-uniform
         if (chunk != cur) {  // flush the previous chunk's sums, start the next
-            if (cur >= 0 && cur * BC + lane < min(m, (cur + 1) * BC)) {
-                tileS[(size_t)(cur * BC + lane) * S + slot] = acc;
-                tileN[(size_t)(cur * BC + lane) * S + slot] = cnt;
+#pragma unroll
+            for (int a = 0; a < kWin2Acc; a++) {
+                const int bw = cur * BC + 32 * a + lane;
+                if (cur >= 0 && bw < min(m, (cur + 1) * BC)) {
+                    tileS[(size_t)bw * S + slot] = acc[a];
+                    tileN[(size_t)bw * S + slot] = cnt[a];
+                }
+                acc[a] = 0.0;
+                cnt[a] = 0;
             }
             if (chunk >= nbc) return;
             cur = chunk;
-            acc = 0.0;
-            cnt = 0;
         }
         const int t = (int)(k - (int64_t)chunk * npairs);
         const int b0 = chunk * BC, b1 = min(m, b0 + BC);
@@ -371,9 +384,14 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
             e2 = warp_sum(e2);  // fixed butterfly: every lane holds the task's sum
             const uint32_t nb = __popc(__ballot_sync(0xffffffffu, M0)) +
                                 (kWin2Rows == 2 ? __popc(__ballot_sync(0xffffffffu, M1)) : 0u);
-            if (lane == b - b0) {
-                acc += e2;
-                cnt += nb;
+            const int bl = b - b0;
+            if (lane == (bl & 31)) {
+#pragma unroll
+                for (int a = 0; a < kWin2Acc; a++)
+                    if ((bl >> 5) == a) {
+                        acc[a] += e2;
+                        cnt[a] += nb;
+                    }
             }
         }
     }
