@@ -749,7 +749,10 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
             const double E2 = fabs(yuu_b) + fabs(yuu_a) + 2.0 * adl * (fabs(yu_b) + fabs(yu_a)) +
                               2.0 * adl * adl * ay + 2.0 * c1 * ymax * adl * (adl + h);
             const double E0 = ay + fabs(yr);
-            fast = kFastSlack * E1 <= kFastTol * den && kFastSlack * fma(hk, E0, E2) <= kFastTol * den * ymax;
+            // kFastSlack E1 <= kFastTol den, kFastSlack (hk E0 + E2) <= kFastTol den ymax, with the
+            // exact power-of-two ratio kFastTol / kFastSlack folded in
+            constexpr double kR = kFastTol / kFastSlack;
+            fast = E1 <= kR * den && fma(hk, E0, E2) <= den * (kR * ymax);
         }
         if (!fast) {
             if (KERN == KR_EPANECHNIKOV) {

@@ -331,8 +331,11 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
         acc[a] = 0.0;
         cnt[a] = 0;
     }
+    // task k = slot + i S -> (chunk, t) advanced incrementally (no 64-bit
+    // division per task)
+    int kchunk = slot / npairs, kt = slot - kchunk * npairs;
     for (int64_t k = slot;; k += S) {
-        const int chunk = k < ntasks ? (int)(k / npairs) : nbc;  // warp-uniform
+        const int chunk = k < ntasks ? kchunk : nbc;  // warp-uniform
         if (chunk != cur) {  // flush the previous chunk's sums, start the next
 #pragma unroll
             for (int a = 0; a < kWin2Acc; a++) {
@@ -347,7 +350,13 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
             if (chunk >= nbc) return;
             cur = chunk;
         }
-        const int t = (int)(k - (int64_t)chunk * npairs);
+        const int t = kt;
+        kt += S % npairs;
+        kchunk += S / npairs;
+        if (kt >= npairs) {
+            kt -= npairs;
+            kchunk += 1;
+        }
         const int b0 = chunk * BC, b1 = min(m, b0 + BC);
         WinRow w0, w1;
         bool v0, v1 = false;
