@@ -1,10 +1,11 @@
 """T7 device half: run every CUDA path once at small sizes
 so that compute-sanitizer (memcheck / racecheck / synccheck / initcheck) sees
 every kernel: the chunked rank sort and the CUB onesweep sort, the prefix
-build, the window kernel (variant from KRCV_WIN_K), the per-pair sweep, the
+build (two-phase, fused with its grid barrier, one-CTA), the bucket table,
+the window kernel (KRCV_WIN=r01 selects r01's), the per-pair sweep, the
 histogram ordering, the dense Gaussian kernel, KDE LSCV, local-linear CV,
-refinement, the reduction with its fused finalize, and the shard + finalize
-path.  Host arrays only (no torch kernels in the trace).  Test
+the leave-one-out confidence intervals, refinement, the reduction with its
+fused finalize, and the shard + finalize path.  Host arrays only (no torch kernels in the trace).  Test
 infrastructure: called by tests/test_gpu_sanitizer.py."""
 import sys
 
@@ -27,6 +28,13 @@ def main() -> int:
         krcv.kr_cv_refine(x, y, h, k, levels=2, m_fine=9)
         krcv.kr_kde_lscv(x, h, k)
         krcv.kr_ll_cv_grid(x, y, h, k)
+        krcv.kr_cv_ci(x, y, h, k)
+        krcv.kr_kde_ci(x, h, k)
+    # the fused O(n) build (n > 1,024 and <= 148 x 256) and the two-phase one above it
+    for nn in (5_000, 60_000):
+        xm = rng.uniform(0, 1, nn)
+        ym = xm + rng.normal(0, 0.1, nn)
+        krcv.kr_cv_grid(xm, ym, np.linspace(0.001, 1.0, 7), "epanechnikov", algo="prefix")
     krcv.kr_cv_grid(x, y, h, "gaussian")
     krcv.kr_cv_grid(x[:2], y[:2], h, "epanechnikov")  # n = 2
     # CUB onesweep sort path (n > 131,072), window-prefix only (the sweep is O(n^2))
