@@ -387,14 +387,19 @@ int ws_class_for(int32_t algo, int32_t kernel, int64_t rows)
 
 bool ws_layout(int64_t n, int32_t m, WsLayout *L, int cls)
 {
-    size_t cub_bytes = 0;
+    size_t cub_bytes = 0, cub32 = 0;
     cudaError_t e = cub::DeviceRadixSort::SortPairs(
         nullptr, cub_bytes, (const uint64_t *)nullptr, (uint64_t *)nullptr,
         (const uint32_t *)nullptr, (uint32_t *)nullptr, (int)n, 0, 64, (cudaStream_t)0);
+    if (e == cudaSuccess)
+        e = cub::DeviceRadixSort::SortPairs(nullptr, cub32, (const uint32_t *)nullptr, (uint32_t *)nullptr,
+                                            (const uint32_t *)nullptr, (uint32_t *)nullptr, (int)n, 0, 32,
+                                            (cudaStream_t)0);
     if (e != cudaSuccess) {
         set_cuda_error("cub::DeviceRadixSort::SortPairs(size query)", (int)e);
         return false;
     }
+    cub_bytes = cub_bytes > cub32 ? cub_bytes : cub32;
     const int64_t ntiles = max_tiles(n);
     size_t off = 0;
     const size_t npad = (size_t)((n + kChunk - 1) / kChunk) * kChunk;  // chunked rank sort
@@ -416,7 +421,8 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L, int cls)
     const size_t pfx_rec = sizeof(double) * 2 * pk_lo_off<KR_EPANECHNIKOV>((int)L->pstride);
     L->pfx = off;      off = align256(off + (pfx_soa > pfx_rec ? pfx_soa : pfx_rec));
     L->ptot = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
-    L->status = off;   off = align256(off + 8 * sizeof(unsigned));  // bad grid, non-finite, done, pad, u64 max|y| bits
+    // 256 B: counters, max|y|, density statistic (bytes 0-31), BktParams (32), q32 key range (64-79)
+    L->status = off;   off = align256(off + 8 * sizeof(unsigned));
     L->cub = off;      off = align256(off + cub_bytes);
     // m-dependent buffers last: everything above has the same offset for any
     // m, so a refinement level with another grid size can reuse the sorted
@@ -942,7 +948,15 @@ static int enqueue_sort(const double *d_x, const double *d_y, int64_t n, const d
     const int nn = (int)n;
     int64_t launches = 0;
     cudaError_t e;
-    if (n <= kRankSortMaxN && !getenv_flag("KRCV_CUB_SORT")) {
+    static const int sort_mode = [] {  // KRCV_SORT=cub64 | q32 | rank (A/B runs); KRCV_CUB_SORT=1 = cub64
+        const char *e = getenv("KRCV_SORT");
+        if (e && strcmp(e, "cub64") == 0) return 1;
+        if (e && strcmp(e, "q32") == 0) return 2;
+        if (e && strcmp(e, "rank") == 0) return 3;
+        return getenv_flag("KRCV_CUB_SORT") ? 1 : 0;
+    }();
+    const bool use_rank = sort_mode == 3 || (sort_mode == 0 && n <= kRankSortMaxN);
+    if (use_rank) {
         // a1 + a2: chunk merge sort, rank by counting across chunk pairs, scatter (krcv_sort.cuh)
         const int cfg = chunk_config(n);
         const int chunk = cfg == 0 ? 1024 : (cfg == 1 ? 2048 : (cfg == 2 ? 4096 : (cfg == 3 ? 512 : 256)));
@@ -961,6 +975,22 @@ static int enqueue_sort(const double *d_x, const double *d_y, int64_t n, const d
                                                                  counter);
         launches += nchunks > 1 ? 1 : 0;
         launches += 2;
+    } else if (sort_mode != 1) {
+        // 32-bit quantised keys, 4 radix passes, exact fix-up of equal-key runs (krcv_sort.cuh)
+        unsigned long long *kmin_c = reinterpret_cast<unsigned long long *>(ws + L.status + 64);
+        unsigned long long *kmax = reinterpret_cast<unsigned long long *>(ws + L.status + 72);
+        uint32_t *q_in = reinterpret_cast<uint32_t *>(keys_out);   // free on this path
+        uint32_t *q_out = reinterpret_cast<uint32_t *>(keys_in);
+        pack_range_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, nn, d_h, m, status, kmin_c, kmax);
+        launch_pdl(quant_kernel, dim3(grid_for(n, 256)), dim3(256), 0, st, d_x, nn, (const unsigned long long *)kmin_c,
+                   (const unsigned long long *)kmax, q_in, vals_in);
+        size_t cub_bytes = L.cub_bytes;
+        e = cub::DeviceRadixSort::SortPairs(ws + L.cub, cub_bytes, q_in, q_out, vals_in, vals_out, nn, 0, 32, st);
+        if (e != cudaSuccess) { set_cuda_error("cub::DeviceRadixSort::SortPairs", (int)e); return KR_ECUDA; }
+        launch_pdl(q32_fixup_kernel, dim3(grid_for(n, 256)), dim3(256), 0, st, d_x, nn, (const uint32_t *)q_out,
+                   vals_out);
+        launch_pdl(gather_kernel, dim3(grid_for(n, 256)), dim3(256), 0, st, d_x, d_y, vals_out, nn, xy, perm, counter);
+        launches += 4 + 2 + 32 / 8;
     } else {
         pack_kernel<<<grid_for(n, 256), 256, 0, st>>>(d_x, d_y, nn, d_h, m, keys_in, vals_in, status);
         size_t cub_bytes = L.cub_bytes;
@@ -1056,7 +1086,8 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     NvtxScope nv_all("krcv: grid-search shard (a1-a5)");
     prof_mark(0, st);
     // reuse keeps max|y| (words 4-5); the host validated x, y and the grid
-    cudaError_t e = cudaMemsetAsync(status, 0, (reuse_sorted ? 3 : 8) * sizeof(unsigned), st);
+    // words 0-7: counters, max|y|, density statistic; bytes 64-79: the key range of the q32 sort
+    cudaError_t e = cudaMemsetAsync(status, 0, (reuse_sorted ? 3 : 20) * sizeof(unsigned), st);
     if (e != cudaSuccess) { set_cuda_error("cudaMemsetAsync(status)", (int)e); return KR_ECUDA; }
     if (reuse_sorted) {
         e = cudaMemsetAsync(counter, 0, sizeof(int), st);
@@ -1303,7 +1334,7 @@ static int enqueue_kde(const double *d_x, int64_t n, const double *d_h, int32_t 
     const int ntiles = (hi - lo + 31) / 32;
     int64_t launches = 0;
     prof_mark(0, st);
-    cudaError_t e = cudaMemsetAsync(status, 0, 8 * sizeof(unsigned), st);
+    cudaError_t e = cudaMemsetAsync(status, 0, 20 * sizeof(unsigned), st);
     if (e != cudaSuccess) { set_cuda_error("cudaMemsetAsync(status)", (int)e); return KR_ECUDA; }
     // the sort carries (x, y); the density estimate has no y: x rides along
     const int st2 = enqueue_sort(d_x, d_x, n, d_h, m, L, ws, st, &launches);

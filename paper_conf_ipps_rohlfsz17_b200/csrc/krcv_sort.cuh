@@ -181,4 +181,99 @@ rank_scatter_kernel(const uint32_t *__restrict__ idx, const int *__restrict__ ra
     }
 }
 
+// ---------------------------------------------------------------------------
+// Large-n sort on a 32-bit quantised key (a2 for n > kRankSortMaxN).  The
+// 64-bit order-preserving keys of x are reduced to q = (key - kmin) >> s with
+// s = max(0, bitlen(kmax - kmin) - 32), a monotone map onto 32 bits, so a
+// stable 4-pass radix sort of (q, index) orders the records by x up to runs
+// of equal q; each such run (x values within 2^s key units of each other --
+// a few records at most for real data) is then put in exact (key, index)
+// order by insertion sort (already-sorted runs, e.g. duplicates, cost one
+// comparison per record).  Half the passes of the 64-bit sort, the same
+// total order (stable by original index).
+// ---------------------------------------------------------------------------
+// pack: validation counters (as pack_kernel) and the key range, kept as
+// atomicMax of the complemented minimum / of the maximum (zero-initialised
+// by the call's status memset)
+__global__ void pack_range_kernel(const double *__restrict__ x, const double *__restrict__ y, int n,
+                                  const double *__restrict__ h, int m, unsigned *__restrict__ status,
+                                  unsigned long long *__restrict__ kmin_c, unsigned long long *__restrict__ kmax)
+{
+    const int stride = gridDim.x * blockDim.x;
+    const int tid = blockIdx.x * blockDim.x + threadIdx.x;
+    unsigned bad = 0, gbad = 0;
+    unsigned long long lo = ~0ull, hi = 0ull;
+    for (int i = tid; i < n; i += stride) {
+        const double xv = x[i], yv = y[i];
+        bad += (!isfinite(xv) || !isfinite(yv)) ? 1u : 0u;
+        const unsigned long long k = order_key(xv);
+        lo = k < lo ? k : lo;
+        hi = k > hi ? k : hi;
+    }
+    for (int b = tid; b < m; b += stride) {
+        const double hb = h[b];
+        gbad += (!isfinite(hb) || !(hb > 0.0) || (b > 0 && hb < h[b - 1])) ? 1u : 0u;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const unsigned long long a = __shfl_xor_sync(0xffffffffu, lo, o), c = __shfl_xor_sync(0xffffffffu, hi, o);
+        lo = a < lo ? a : lo;
+        hi = c > hi ? c : hi;
+    }
+    if ((threadIdx.x & 31) == 0 && hi >= lo) {
+        atomicMax(kmin_c, ~lo);
+        atomicMax(kmax, hi);
+    }
+    if (bad) atomicAdd(&status[1], bad);
+    if (gbad) atomicAdd(&status[0], gbad);
+}
+
+__device__ __forceinline__ int q32_shift(unsigned long long kmin, unsigned long long kmax)
+{
+    const unsigned long long r = kmax - kmin;
+    const int bits = r ? 64 - __clzll((long long)r) : 0;
+    return bits > 32 ? bits - 32 : 0;
+}
+
+__global__ void quant_kernel(const double *__restrict__ x, int n, const unsigned long long *__restrict__ kmin_c,
+                             const unsigned long long *__restrict__ kmax, uint32_t *__restrict__ q,
+                             uint32_t *__restrict__ idx)
+{
+    pdl_wait();  // krcv_pdl.cuh
+    const unsigned long long lo = ~*kmin_c, hi = *kmax;
+    const int s = q32_shift(lo, hi);
+    const int stride = gridDim.x * blockDim.x;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+        q[i] = (uint32_t)((order_key(x[i]) - lo) >> s);
+        idx[i] = (uint32_t)i;
+    }
+}
+
+// exact (key, index) order inside every run of equal q (sorted positions)
+__global__ void q32_fixup_kernel(const double *__restrict__ x, int n, const uint32_t *__restrict__ q,
+                                 uint32_t *__restrict__ idx)
+{
+    pdl_wait();  // krcv_pdl.cuh
+    const int stride = gridDim.x * blockDim.x;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+        const uint32_t qi = q[i];
+        if ((i > 0 && q[i - 1] == qi) || i + 1 >= n || q[i + 1] != qi) continue;  // not the start of a run >= 2
+        int e = i + 2;
+        while (e < n && q[e] == qi) e++;
+        for (int a = i + 1; a < e; a++) {  // insertion sort by (key, index); stable input order is index order
+            const uint32_t v = idx[a];
+            const unsigned long long kv = order_key(x[v]);
+            int b = a - 1;
+            while (b >= i) {
+                const uint32_t u = idx[b];
+                const unsigned long long ku = order_key(x[u]);
+                if (ku < kv || (ku == kv && u < v)) break;
+                idx[b + 1] = u;
+                b--;
+            }
+            idx[b + 1] = v;
+        }
+    }
+}
+
 }  // namespace krcv

@@ -46,7 +46,10 @@
 
 namespace krcv {
 
-constexpr int kBktFmax = 32;             // buckets per point, at most
+#ifndef KRCV_BKT_FMAX
+#define KRCV_BKT_FMAX 32
+#endif
+constexpr int kBktFmax = KRCV_BKT_FMAX;  // buckets per point, at most (build-time A/B)
 #ifndef KRCV_BKT_FX
 #define KRCV_BKT_FX 1.0                  // (build-time A/B) buckets per point at the peak density
 #endif
