@@ -801,8 +801,7 @@ static void launch_bkt_fill(int n, const WsLayout &L, char *ws, cudaStream_t st)
         reinterpret_cast<const unsigned long long *>(ws + L.status + 6 * sizeof(unsigned));
     BktParams *prm = reinterpret_cast<BktParams *>(ws + L.status + 32);
     const int64_t qmax = (int64_t)kBktFmax * n < kBktQmax ? (int64_t)kBktFmax * n : kBktQmax;
-    const int64_t nseg = (n + qmax + 1 + kBktSeg - 1) / kBktSeg;
-    int64_t blocks = (nseg + kBktFillThreads - 1) / kBktFillThreads;
+    int64_t blocks = (n + qmax + 1 + kBktTile - 1) / kBktTile;
     if (blocks > (int64_t)dev_info().sms * 8) blocks = (int64_t)dev_info().sms * 8;
     launch_pdl(bkt_fill_kernel, dim3((int)blocks), dim3(kBktFillThreads), 0, st, xs, n, gap, BT, prm);
 }

@@ -220,12 +220,36 @@ __global__ void pack_range_kernel(const double *__restrict__ x, const double *__
         lo = a < lo ? a : lo;
         hi = c > hi ? c : hi;
     }
-    if ((threadIdx.x & 31) == 0 && hi >= lo) {
-        atomicMax(kmin_c, ~lo);
-        atomicMax(kmax, hi);
+    // one atomic per CTA (per warp, thousands of same-address atomics
+    // serialised in L2: 11 us at n = 200,000, profiles/r02/r02ad_*)
+    __shared__ unsigned long long slo[32], shi[32];
+    __shared__ unsigned sbad[32], sgbad[32];
+    const int w = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+    if ((threadIdx.x & 31) == 0) {
+        slo[w] = lo;
+        shi[w] = hi;
     }
-    if (bad) atomicAdd(&status[1], bad);
-    if (gbad) atomicAdd(&status[0], gbad);
+    bad = __reduce_add_sync(0xffffffffu, bad);
+    gbad = __reduce_add_sync(0xffffffffu, gbad);
+    if ((threadIdx.x & 31) == 0) {
+        sbad[w] = bad;
+        sgbad[w] = gbad;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int q = 1; q < nw; q++) {
+            lo = slo[q] < lo ? slo[q] : lo;
+            hi = shi[q] > hi ? shi[q] : hi;
+            bad += sbad[q];
+            gbad += sgbad[q];
+        }
+        if (hi >= lo) {
+            atomicMax(kmin_c, ~lo);
+            atomicMax(kmax, hi);
+        }
+        if (bad) atomicAdd(&status[1], bad);
+        if (gbad) atomicAdd(&status[0], gbad);
+    }
 }
 
 __device__ __forceinline__ int q32_shift(unsigned long long kmin, unsigned long long kmax)

@@ -56,7 +56,6 @@ constexpr int kBktFmax = KRCV_BKT_FMAX;  // buckets per point, at most (build-ti
 constexpr int64_t kBktQmax = 1LL << 28;  // buckets, at most
 constexpr double kBktMagic = 6755399441055744.0;  // 1.5 * 2^52: fma(.) + magic keeps the integer in the low word
 constexpr int kBktFillThreads = 256;
-constexpr int kBktSeg = 8;               // merge-path items per thread of the table fill (more threads: the diagonal searches are latency-bound)
 
 // Table parameters, written by bkt_fill_kernel's first thread, read by the
 // window kernel (both compute them from the same inputs).
@@ -102,17 +101,26 @@ __device__ __forceinline__ BktParams bkt_params(const double *__restrict__ xs, i
     return bkt_params_of(xs[0], xs[n - 1], n, *gap_bits);
 }
 
-// Fused O(n) build for a shard problem whose 256-record prefix tiles all fit
-// on the GPU at once (ntiles <= #SMs, so every CTA is co-resident): phase 1
-// (tile totals, max|y|, density statistic), a grid barrier (arrival counter,
-// zeroed by the call's status memset), phase 3 (the tile's offset from the
-// totals of the earlier tiles in fixed order, the scan, the records and xs --
-// the same bodies as pfx_tile_reduce_kernel / pfx_tile_scan_kernel, so the
-// records are bit-identical), then this tile's stretch of the bucket table:
-// q in (bkt(x_{j0-1}), bkt(x_{j1-1})] (from 0 for the first tile, to Q for
-// the last), BT[q] = the first of the tile's records with bucket >= q, by a
-// binary search over the tile's bucket ids in shared memory -- the same table
-// bkt_fill_kernel builds.  One launch instead of three.
+// Fused O(n) build for a problem whose 256-record prefix tiles all fit on
+// the GPU at once (ntiles <= #SMs, so every CTA is co-resident), one record
+// per thread.  It is latency-bound (two warps per SM sub-partition, long
+// dependent dd chains), so every step is done once:
+//   1. the record's moment terms (kept in registers), the warp's inclusive dd
+//      scan of them, the density statistic and max|y|; the warp totals give
+//      the tile's warp offsets and total in one fixed-order pass (5 threads,
+//      one per moment), the total -> tot[k][tile];
+//   2. a grid barrier (arrival counter, zeroed by the call's status memset);
+//   3. the tile's offset: the totals of the earlier tiles in fixed order
+//      (strided per thread, butterfly per warp, warp partials in order);
+//      P[j] = offset + warp offset + the lane's exclusive scan; records, xs;
+//   4. this tile's stretch of the bucket table: q in (bkt(x_{j0-1}),
+//      bkt(x_{j1-1})] (from 0 for the first tile, to Q for the last), BT[q] =
+//      the first of the tile's records with bucket >= q, by a binary search
+//      over the tile's bucket ids in shared memory -- the table
+//      bkt_fill_kernel builds.
+// One launch instead of three; every sum in a fixed order (bit-reproducible;
+// its rounding differs from the two-phase build's in the last dd bits, as the
+// two-phase build's differs from the one-CTA build's).
 constexpr int kFusedPfxThreads = kPfxThreads;  // one record per thread (ITEMS = 1)
 
 __device__ __forceinline__ unsigned ld_acquire_u32(const unsigned *p)
@@ -130,24 +138,116 @@ pfx_fused_kernel(const double2 *__restrict__ xy, int n, double2 *__restrict__ to
                  BktParams *__restrict__ prm, unsigned *__restrict__ arrive)
 {
     pdl_wait();  // krcv_pdl.cuh
+    constexpr int K = NMom<KERN>::v;
+    constexpr int W = kFusedPfxThreads / 32;
+    __shared__ double2 wtot[K][W];  // warp totals, then the warps' exclusive offsets
+    __shared__ double2 base_s[K];
     __shared__ int sA[kFusedPfxThreads];
-    pfx_reduce_body<KERN, 1, true>(xy, n, tot, ntiles, ymax_bits, gap_bits, blockIdx.x);
+    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+    const int tile = blockIdx.x;
+    const int j = tile * kFusedPfxThreads + t;
+    if (tile == 0 && t < kPad) {
+        xs[-1 - t] = -INFINITY;
+        xs[n + t] = INFINITY;
+    }
+    // 1. terms, warp scan, statistics
+    const double o = pfx_origin(xy, n);
+    dd tm[kPfxMoments], inc[kPfxMoments];
+    double xj = 0.0, ym = 0.0, gmin = INFINITY;
+    if (j < n) {
+        const double2 v = xy[j];
+        xj = v.x;
+        ym = fabs(v.y);
+        gap_stat(xy, n, j, gmin);
+        moment_terms<KERN>(v.x, v.y, o, tm);
+    } else {
+#pragma unroll
+        for (int k = 0; k < K; k++) tm[k] = dd{0.0, 0.0};
+    }
+#pragma unroll
+    for (int k = 0; k < K; k++) inc[k] = tm[k];
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            const dd u = shfl_up_dd(inc[k], d);
+            if (lane >= d) inc[k] = dd_add(u, inc[k]);
+        }
+    }
+    if (lane == 31) {
+#pragma unroll
+        for (int k = 0; k < K; k++) st_dd(&wtot[k][w], inc[k]);
+    }
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) ym = fmax(ym, __shfl_xor_sync(0xffffffffu, ym, d));
+    if (lane == 0 && ym > 0.0) atomicMax(ymax_bits, (unsigned long long)__double_as_longlong(ym));
+    gap_publish(gmin, gap_bits);
     __syncthreads();
-    if (threadIdx.x == 0) {
+    if (t < K) {  // warp offsets (exclusive, in warp order) and the tile total
+        dd run = dd{0.0, 0.0};
+        for (int q = 0; q < W; q++) {
+            const dd v = ld_dd(&wtot[t][q]);
+            st_dd(&wtot[t][q], run);
+            run = q == 0 ? v : dd_add(run, v);
+        }
+        st_dd(tot + (size_t)t * ntiles + tile, run);
+    }
+    __syncthreads();
+    // 2. grid barrier
+    if (t == 0) {
         __threadfence();
         atomicAdd(arrive, 1u);
         while (ld_acquire_u32(arrive) < gridDim.x) __nanosleep(32);
         __threadfence();
     }
     __syncthreads();
-    pfx_scan_body<KERN, 1, false, true>(xy, n, tot, ntiles, P, pstride, xs, gap_bits, blockIdx.x);
+    // 3. the tile's offset, the records
+    {
+        dd a[kPfxMoments];
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            a[k] = dd{0.0, 0.0};
+            for (int q = t; q < tile; q += kFusedPfxThreads) {
+                const double2 *pq = tot + (size_t)k * ntiles + q;
+                a[k] = dd_add(a[k], dd{__ldcg(&pq->x), __ldcg(&pq->y)});
+            }
+        }
+        if (tile > 32 * w) {  // warps whose strided range holds earlier tiles
+#pragma unroll
+            for (int d = 16; d > 0; d >>= 1) {
+#pragma unroll
+                for (int k = 0; k < K; k++) a[k] = dd_add(a[k], shfl_xor_dd(a[k], d));
+            }
+        }
+        __shared__ double2 psum[K][W];
+        if (lane == 0) {
+#pragma unroll
+            for (int k = 0; k < K; k++) st_dd(&psum[k][w], a[k]);
+        }
+        __syncthreads();
+        if (t < K) {
+            dd b = dd{0.0, 0.0};
+            const int nw = min(W, (tile + 31) / 32);
+            for (int q = 0; q < nw; q++) b = dd_add(b, ld_dd(&psum[t][q]));
+            st_dd(&base_s[t], b);
+        }
+        __syncthreads();
+    }
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        const dd u = shfl_up_dd(inc[k], 1);
+        const dd ex = lane == 0 ? dd{0.0, 0.0} : u;
+        if (j <= n) pk_store<KERN>(P, pstride, k, j, dd_add(dd_add(ld_dd(&base_s[k]), ld_dd(&wtot[k][w])), ex));
+    }
+    if (j <= n) pk_store_index<KERN>(P, pstride, j);
+    if (j < n) xs[j] = xj;
+    // 4. bucket table
     if (!BT) return;
     const BktParams p = bkt_params_of(__ldg(&xy[0].x), __ldg(&xy[n - 1].x), n, __ldcg(gap_bits));
-    if (blockIdx.x == 0 && threadIdx.x == 0) *prm = p;
+    if (tile == 0 && t == 0) *prm = p;
     auto A = [&](double v) { return min(max(bkt_raw(v, p.invw, p.C), 0), p.Q); };
-    const int j0 = blockIdx.x * kFusedPfxThreads, j1 = min(j0 + kFusedPfxThreads, n), cnt = j1 - j0;
-    const int t = threadIdx.x;
-    sA[t] = t < cnt ? A(__ldg(&xy[j0 + t].x)) : INT_MAX;
+    const int j0 = tile * kFusedPfxThreads, j1 = min(j0 + kFusedPfxThreads, n), cnt = j1 - j0;
+    sA[t] = t < cnt ? A(xj) : INT_MAX;
     __syncthreads();
     const int qlo = j0 == 0 ? 0 : A(__ldg(&xy[j0 - 1].x)) + 1;
     const int qhi = j1 == n ? p.Q : sA[cnt - 1];
@@ -163,44 +263,90 @@ pfx_fused_kernel(const double2 *__restrict__ xy, int n, double2 *__restrict__ to
 
 // BT[q] = #{k : bkt(xs[k]) < q} for q = 0 .. Q: the merge of the sorted
 // bucket ids A[k] = clamp(bkt(xs[k]), 0, Q) with the sequence 0 .. Q (A[k]
-// goes first iff A[k] < q), cut into segments of kBktSeg merged items by a
-// binary search on each segment's diagonal (merge path), so long runs of
-// empty buckets (the sparse tail of a heavy-tailed x) are spread over many
-// threads.  Grid-stride over segments; the grid is sized for Q <= kBktFmax n.
+// goes first iff A[k] < q), cut by merge path at two levels so long runs of
+// empty buckets (the sparse tail of a heavy-tailed x) are spread evenly:
+// a CTA takes kBktTile consecutive merged items, its two warps find the
+// tile's ends on the diagonals (32 probes per round: log32 rounds of
+// dependent loads instead of log2), the CTA stages the tile's bucket ids in
+// shared memory, and each thread merges kBktItems items from its own split
+// (a binary search in shared memory).  Grid-stride over tiles.
+constexpr int kBktItems = 16;
+constexpr int kBktTile = kBktFillThreads * kBktItems;
+
+// smallest i in [lo, hi] with p(i) true (p monotone, p(hi) taken as true),
+// found by all 32 lanes of a warp together; every lane returns it
+template <class Pred>
+__device__ __forceinline__ int64_t warp_first_true(Pred p, int64_t lo, int64_t hi, int lane)
+{
+    while (hi > lo) {
+        // lane l tests the end of sub-range l of ceil(len / 32) items; lane
+        // 31's sub-range ends at hi (true by definition)
+        const int64_t step = (hi - lo + 31) / 32;
+        const int64_t q = lo + (int64_t)(lane + 1) * step - 1;
+        const bool t = lane == 31 || q >= hi || p(q);
+        const int f = __ffs(__ballot_sync(0xffffffffu, t)) - 1;
+        const int64_t end = lo + (int64_t)(f + 1) * step - 1;
+        hi = (f == 31 || end > hi) ? hi : end;
+        lo = lo + (int64_t)f * step;
+    }
+    return hi;
+}
+
 __global__ void __launch_bounds__(kBktFillThreads)
 bkt_fill_kernel(const double *__restrict__ xs, int n, const unsigned long long *__restrict__ gap_bits,
                 int *__restrict__ BT, BktParams *__restrict__ prm)
 {
     pdl_wait();  // krcv_pdl.cuh
+    __shared__ int sA[kBktTile];
+    __shared__ int sBT[kBktTile];  // the tile's table entries, stored coalesced at the end
+    __shared__ int64_t split[2];
     const BktParams p = bkt_params(xs, n, gap_bits);
     if (blockIdx.x == 0 && threadIdx.x == 0) *prm = p;
     const int Q = p.Q;
-    auto A = [&](int k) { return min(max(bkt_raw(xs[k], p.invw, p.C), 0), Q); };
+    auto A = [&](int64_t k) { return (int64_t)min(max(bkt_raw(xs[k], p.invw, p.C), 0), Q); };
     const int64_t total = (int64_t)n + Q + 1;
-    const int64_t nseg = (total + kBktSeg - 1) / kBktSeg;
-    for (int64_t sg = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; sg < nseg;
-         sg += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t d = sg * kBktSeg;
-        // split of the first d merged items: i from A, d - i from B.  Smallest
-        // i with "B[d - i - 1] before A[i]" (A[i] >= d - i - 1), monotone in i.
-        int64_t lo = d - (Q + 1) > 0 ? d - (Q + 1) : 0;
-        int64_t hi = d < n ? d : n;
-        while (lo < hi) {
-            const int64_t mid = (lo + hi) >> 1;
-            if ((int64_t)A((int)mid) >= d - mid - 1) hi = mid; else lo = mid + 1;
+    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+    for (int64_t D0 = (int64_t)blockIdx.x * kBktTile; D0 < total; D0 += (int64_t)gridDim.x * kBktTile) {
+        const int64_t D1 = D0 + kBktTile < total ? D0 + kBktTile : total;
+        if (w < 2) {
+            // split of the first d merged items: i from A, d - i from 0..Q;
+            // the smallest i with A[i] >= d - i - 1 (monotone in i)
+            const int64_t d = w == 0 ? D0 : D1;
+            const int64_t lo = d - (Q + 1) > 0 ? d - (Q + 1) : 0;
+            const int64_t hi = d < n ? d : n;
+            const int64_t s = warp_first_true([&](int64_t i) { return A(i) >= d - i - 1; }, lo, hi, lane);
+            if (lane == 0) split[w] = s;
         }
-        int i = (int)lo;
-        int64_t j = d - lo;
-        int ai = i < n ? A(i) : 0;
-        for (int s = 0; s < kBktSeg && (int64_t)i + j < total; s++) {
-            if (i < n && (j > Q || (int64_t)ai < j)) {
-                i++;
-                ai = i < n ? A(i) : 0;
-            } else {
-                BT[j] = i;
-                j++;
+        __syncthreads();
+        const int64_t i0 = split[0], i1 = split[1];
+        const int cnt = (int)(i1 - i0);  // <= kBktTile
+        for (int k = t; k < cnt; k += kBktFillThreads) sA[k] = (int)A(i0 + k);
+        __syncthreads();
+        // this thread's items: local diagonal dl = t kBktItems of the tile
+        const int dl = t * kBktItems;
+        const int64_t d = D0 + dl;
+        const int jn = (int)(D1 - D0) - cnt;  // bucket items of the tile: q = D0 - i0 ..
+        const int64_t jb = D0 - i0;
+        if (d < D1) {
+            int lo = dl - jn > 0 ? dl - jn : 0, hi = dl < cnt ? dl : cnt;
+            while (lo < hi) {
+                const int mid = (lo + hi) >> 1;
+                if ((int64_t)sA[mid] >= d - (i0 + mid) - 1) hi = mid; else lo = mid + 1;
+            }
+            int i = lo;
+            int64_t j = d - (i0 + i);
+            for (int s = 0; s < kBktItems && D0 + dl + s < D1; s++) {
+                if (i < cnt && (int64_t)sA[i] < j) {
+                    i++;
+                } else {
+                    sBT[j - jb] = (int)(i0 + i);
+                    j++;
+                }
             }
         }
+        __syncthreads();
+        for (int k = t; k < jn; k += kBktFillThreads) BT[jb + k] = sBT[k];
+        __syncthreads();  // sA / sBT / split reused by the next tile
     }
 }
 
