@@ -499,8 +499,9 @@ def bench_extra_configs(args, timed, dev, krcv, torch):
     """The other BASELINE.json configurations on this one GPU (C3, C4, C5:
     configs[2..4]) in the same launch configuration as the headline, each with
     its stage times and roofline, plus the row-shard balance of the window
-    stage at P = 8 (the eight equal sorted-row shards timed one after another
-    on this GPU through kr_cv_rows_async) and the projected P-GPU time
+    stage at P = 2, 4, 8 (the P sorted-row shards timed one after another on
+    this GPU through kr_cv_rows_async; equal rows and cost-balanced cuts) and
+    the projected P-GPU time
         T(P) = pack/sort + prefix/table build (replicated on every rank)
                + window * (max shard / mean shard) / P + reduce
                + ALLREDUCE_US_ASSUMED
@@ -516,37 +517,63 @@ def bench_extra_configs(args, timed, dev, krcv, torch):
         r = timed("auto", wl, steps=5 if name == "C4" else 10, warmup=3)
         r.pop("plan")
         r.pop("launch")
-        # window-stage balance of 8 equal row shards
+        # window-stage balance of P row shards: equal rows, and the
+        # cost-balanced cuts bench.py uses at N > 1 (api.balanced_cuts from 4P
+        # calibration segments)
+        from paper_conf_ipps_rohlfsz17_b200 import api as _api
+
         d_h = torch.as_tensor(h, device=dev)
         ws = krcv.aligned(krcv.workspace(n, m, dev))
         part = torch.zeros(krcv.partial_len(m), dtype=torch.float64, device=dev)
         krcv.kr_profile_enable(True)
-        shard_ms = []
-        for s in range(8):
-            lo, hi = (s * n) // 8, ((s + 1) * n) // 8
+
+        def window_ms(lo, hi):
             for _ in range(2):  # the second run is timed (warm)
                 krcv.kr_cv_rows_async(wl["d_x"], wl["d_y"], d_h, k, lo, hi, part, ws)
                 t = krcv.kr_profile_read()
-            shard_ms.append(t[2])
+            return t[2]
+
+        imb_eq, imb_bal, cuts_bal = {}, {}, {}
+        shard8 = []
+        for P in (2, 4, 8):
+            eq = [window_ms((s * n) // P, ((s + 1) * n) // P) for s in range(P)]
+            if P == 8:
+                shard8 = eq
+            imb_eq[P] = max(eq) / (sum(eq) / P)
+            calib = [window_ms((s * n) // (4 * P), ((s + 1) * n) // (4 * P)) for s in range(4 * P)]
+            cuts = _api.balanced_cuts(calib, n, P)
+            bal = [window_ms(cuts[s], cuts[s + 1]) for s in range(P)]
+            imb_bal[P] = max(bal) / (sum(bal) / P)
+            cuts_bal[P] = cuts
         krcv.kr_profile_enable(False)
         del ws
         st = r["stage_ms"]
-        imb = max(shard_ms) / (sum(shard_ms) / len(shard_ms))
         t1 = r["ms_per_step"]
-        proj = {}
+        fixed = st["reduce_finalize"] + ALLREDUCE_US_ASSUMED * 1e-3
+        repl = st["pack_sort_gather"] + st["prefix_build"]
+        proj, proj_eq, bound = {}, {}, {}
         for P in (2, 4, 8):
-            tp = st["pack_sort_gather"] + st["prefix_build"] + st["sweep"] * (imb if P == 8 else 1.0) / P + \
-                st["reduce_finalize"] + ALLREDUCE_US_ASSUMED * 1e-3
-            proj[str(P)] = {"ms": tp, "efficiency": t1 / (P * tp)}
+            tp = repl + st["sweep"] * imb_bal[P] / P + fixed
+            proj[str(P)] = {"ms": tp, "efficiency": t1 / (P * tp), "imbalance": imb_bal[P]}
+            tq = repl + st["sweep"] * imb_eq[P] / P + fixed
+            proj_eq[str(P)] = {"ms": tq, "efficiency": t1 / (P * tq), "imbalance": imb_eq[P]}
+            tb = st["sweep"] * imb_bal[P] / P + fixed
+            bound[str(P)] = t1 / (P * tb)
         res[name] = {"workload": workload_desc(cfg, args.seed), "value": r["value"], "unit": UNIT,
                      "ms_per_step": t1, "stage_ms": st, "roofline": r["roofline"], "result": r["result"],
                      "clocks": r["clocks"], "gpu_launches": r["gpu_launches"],
-                     "shard8_window_ms": shard_ms, "shard8_imbalance": imb,
+                     "shard8_window_ms": shard8, "shard8_imbalance": imb_eq[8],
                      "projected_scaling": proj,
-                     "projection_note": ("T(P) = replicated sort + prefix/table build + window x imbalance(P=8, "
-                                         "measured on 8 equal shards) / P + reduce + "
-                                         f"{ALLREDUCE_US_ASSUMED} us assumed all-reduce; one-GPU stage times, "
-                                         "not a multi-GPU measurement")}
+                     "projected_scaling_equal_rows": proj_eq,
+                     "efficiency_bound_no_replicated_stage": bound,
+                     "balanced_cuts": {str(P): c for P, c in cuts_bal.items()},
+                     "projection_note": ("T(P) = replicated sort + prefix/table build + window x imbalance(P) / P "
+                                         f"+ reduce + {ALLREDUCE_US_ASSUMED} us assumed all-reduce; imbalance = "
+                                         "max/mean window time of the P shards, timed one after another on this "
+                                         "GPU (cost-balanced cuts, as bench.py runs N > 1; equal rows in "
+                                         "projected_scaling_equal_rows); efficiency_bound_no_replicated_stage "
+                                         "drops the sort + build (the Amdahl bound of a fully distributed O(n) "
+                                         "stage); one-GPU stage times, not a multi-GPU measurement")}
     return res
 
 

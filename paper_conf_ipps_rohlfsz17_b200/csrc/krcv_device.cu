@@ -622,7 +622,9 @@ static int pfx_items(int n)
         return (v == 0 || v == 1 || v == 4) ? v : -2;
     }();
     if (forced != -2) return forced;
-    return n <= kPfxOneCtaMax ? 0 : (n <= (1 << 18) ? 1 : kPfxItemsMax);
+    // measured (profiles/r02/r02ag_*): 1,024-record tiles from C5's n = 200,000
+    // on (build 55 -> 51 us), equal at C3
+    return n <= kPfxOneCtaMax ? 0 : (n <= (1 << 17) ? 1 : kPfxItemsMax);
 }
 
 static void launch_bkt_fill(int n, const WsLayout &L, char *ws, cudaStream_t st);

@@ -400,24 +400,43 @@ __device__ __forceinline__ void pfx_scan_body(const double2 *__restrict__ xy, in
         xs[n + t] = INFINITY;
     }
     const double o = pfx_origin(xy, n);
-    dd tm[ITEMS][kPfxMoments];
+    // ITEMS > 1: the tile's records staged through shared memory (coalesced
+    // loads and xs stores; each thread then reads its ITEMS consecutive
+    // records), and the moment terms recomputed for the record stores instead
+    // of held in registers across the scan (124 -> fewer registers: the
+    // kernel is latency-bound at 2 CTAs per SM otherwise, profiles/r02/r02ab_*)
+    __shared__ double2 sxy[ITEMS > 1 ? kPfxThreads * ITEMS : 1];
+    if (ITEMS > 1) {
+        const int tb = tile * (kPfxThreads * ITEMS);
+#pragma unroll
+        for (int q = 0; q < ITEMS; q++) {
+            const int jj = tb + q * kPfxThreads + t;
+            const double2 v = jj < n ? xy[jj] : make_double2(0.0, 0.0);
+            sxy[q * kPfxThreads + t] = v;
+            if (jj < n) xs[jj] = v.x;
+        }
+        __syncthreads();
+    }
+    auto rec = [&](int q) { return ITEMS > 1 ? sxy[t * ITEMS + q] : xy[j0 + q]; };
+    dd tm[ITEMS > 1 ? 1 : ITEMS][kPfxMoments];
     dd acc[kPfxMoments];
     double gmin = INFINITY;
 #pragma unroll
     for (int k = 0; k < K; k++) acc[k] = dd{0.0, 0.0};
 #pragma unroll
     for (int q = 0; q < ITEMS; q++) {
+        dd (&tq)[kPfxMoments] = tm[ITEMS > 1 ? 0 : q];
         if (j0 + q < n) {
-            const double2 v = xy[j0 + q];
-            xs[j0 + q] = v.x;
+            const double2 v = rec(q);
+            if (ITEMS == 1) xs[j0 + q] = v.x;
             if (GAP && PfxRec<KERN>::S) gap_stat(xy, n, j0 + q, gmin);
-            moment_terms<KERN>(v.x, v.y, o, tm[q]);
+            moment_terms<KERN>(v.x, v.y, o, tq);
         } else {
 #pragma unroll
-            for (int k = 0; k < K; k++) tm[q][k] = dd{0.0, 0.0};
+            for (int k = 0; k < K; k++) tq[k] = dd{0.0, 0.0};
         }
 #pragma unroll
-        for (int k = 0; k < K; k++) acc[k] = dd_add(acc[k], tm[q][k]);
+        for (int k = 0; k < K; k++) acc[k] = dd_add(acc[k], tq[k]);
     }
     if (GAP && PfxRec<KERN>::S) gap_publish(gmin, gap_bits);
     // exclusive scan of the thread totals across the CTA
@@ -435,18 +454,38 @@ __device__ __forceinline__ void pfx_scan_body(const double2 *__restrict__ xy, in
         ex[k] = lane == 0 ? dd{0.0, 0.0} : u;
     }
     __syncthreads();
+    if (ITEMS == 1) {
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            dd base = ld_dd(&base_s[k]);
+            for (int q = 0; q < w; q++) base = dd_add(base, ld_dd(&wsum[k][q]));
+            const dd run = dd_add(base, ex[k]);
+            if (j0 <= n) {
+                pk_store<KERN>(P, pstride, k, j0, run);
+                if (k == 0) pk_store_index<KERN>(P, pstride, j0);
+            }
+        }
+        return;
+    }
+    dd run[kPfxMoments];
 #pragma unroll
     for (int k = 0; k < K; k++) {
         dd base = ld_dd(&base_s[k]);
         for (int q = 0; q < w; q++) base = dd_add(base, ld_dd(&wsum[k][q]));
-        dd run = dd_add(base, ex[k]);
+        run[k] = dd_add(base, ex[k]);
+    }
 #pragma unroll
-        for (int q = 0; q < ITEMS; q++) {
-            if (j0 + q <= n) {
-                pk_store<KERN>(P, pstride, k, j0 + q, run);
-                if (k == 0) pk_store_index<KERN>(P, pstride, j0 + q);
-            }
-            run = dd_add(run, tm[q][k]);
+    for (int q = 0; q < ITEMS; q++) {
+        if (j0 + q > n) break;
+#pragma unroll
+        for (int k = 0; k < K; k++) pk_store<KERN>(P, pstride, k, j0 + q, run[k]);
+        pk_store_index<KERN>(P, pstride, j0 + q);
+        if (q + 1 < ITEMS && j0 + q < n) {  // the same terms as the first pass (deterministic)
+            const double2 v = rec(q);
+            dd tq[kPfxMoments];
+            moment_terms<KERN>(v.x, v.y, o, tq);
+#pragma unroll
+            for (int k = 0; k < K; k++) run[k] = dd_add(run[k], tq[k]);
         }
     }
 }
