@@ -614,16 +614,27 @@ int auto_algo(int64_t /*n*/, int64_t /*rows*/, int32_t /*m*/, int32_t /*kernel*/
 // KRCV_PFX_ITEMS=0|1|4 overrides.
 constexpr int kPfxOneCtaMax = 1024;  // measured: C1 (n = 1,000) 10.2 -> 8.2 us, C2 (n = 20,000) 18 -> 187 us
 
-static int pfx_items(int n)
+// KRCV_PFX_ITEMS=0|1|4 forces the build's tile size (A/B runs), else -2
+static int pfx_items_forced()
 {
     static const int forced = [] {
         const char *e = getenv("KRCV_PFX_ITEMS");
         const int v = e ? atoi(e) : -2;
         return (v == 0 || v == 1 || v == 4) ? v : -2;
     }();
+    return forced;
+}
+
+// The moment sets without the fused build (KDE, local-linear): one CTA for
+// n <= 1,024, then 256-record tiles, 1,024-record tiles from n > 131,072
+// (measured, profiles/r02/r02ag_*: C5 build 55 -> 51 us, equal at C3).  The
+// regression sets take the fused build wherever its tiles are co-resident,
+// at n <= 1,024 too (C1 build 14.3 -> 12.3 us, step 0.039 -> 0.035 ms,
+// profiles/r02/r02ak_*).
+static int pfx_items(int n)
+{
+    const int forced = pfx_items_forced();
     if (forced != -2) return forced;
-    // measured (profiles/r02/r02ag_*): 1,024-record tiles from C5's n = 200,000
-    // on (build 55 -> 51 us), equal at C3
     return n <= kPfxOneCtaMax ? 0 : (n <= (1 << 17) ? 1 : kPfxItemsMax);
 }
 
@@ -642,7 +653,8 @@ static int launch_prefix_build(const double2 *xy, int n, const WsLayout &L, char
     unsigned long long *gap = reinterpret_cast<unsigned long long *>(ws + L.status + 6 * sizeof(unsigned));
     const int items = pfx_items(n);
     const int tiles1 = (n + kPfxThreads) / kPfxThreads;  // 256-record tiles covering P[0..n]
-    if (items == 1 && PfxRec<KERN>::S && tiles1 <= dev_info().sms && !getenv_flag("KRCV_PFX_UNFUSED")) {
+    const bool fusable = items == 1 || (items == 0 && pfx_items_forced() == -2);
+    if (fusable && PfxRec<KERN>::S && tiles1 <= dev_info().sms && !getenv_flag("KRCV_PFX_UNFUSED")) {
         // every tile co-resident (<= one CTA per SM): the fused build
         unsigned *arrive = reinterpret_cast<unsigned *>(ws + L.status) + 3;  // zeroed by the status memset
         int *BT = table ? reinterpret_cast<int *>(ws + L.bt) : nullptr;
@@ -759,7 +771,12 @@ struct Win2Shape {
 // (C3 1.192 -> 1.160 ms, C5 1.653 -> 1.600 ms against 8), but chunks of at
 // least 3 bandwidths (C2: 16 per slot would mean one-bandwidth tasks, whose
 // per-task row setup costs more than the balance gains: 65.5 -> 60.4 us
-// window at 3 bandwidths)
+// window at 3 bandwidths).  A rule minimising the slot imbalance
+// ceil(tasks / S) (BC + c0) instead (C2: 14-bandwidth chunks, one task per
+// slot) measured slower at C2 / C3 / C5 (59 -> 70 us, +3 %, +5 %) and 1 %
+// faster at C4: the chunk-major round-robin keeps few chunks -- a narrow
+// band of bandwidths, so of boundary positions -- in flight, and large
+// chunks widen it (profiles/r02/r02aj_*).
 constexpr int kWin2TasksPerWarp = 16;
 constexpr int kWin2MinChunk = 3;
 
@@ -776,8 +793,15 @@ static Win2Shape win2_shape(int64_t rows, int m)
         return v > 0 ? v : kWin2TasksPerWarp;
     }();
     const int64_t target = (int64_t)tpw * slots;
-    int64_t bc = (int64_t)m * ((w.ntiles + kWin2Rows - 1) / kWin2Rows) / (target > 0 ? target : 1);
+    const int64_t npairs = (w.ntiles + kWin2Rows - 1) / kWin2Rows;
+    int64_t bc = (int64_t)m * npairs / (target > 0 ? target : 1);
     bc = bc < kWin2MinChunk ? kWin2MinChunk : (bc > kWin2Chunk ? kWin2Chunk : bc);
+    // too few tasks to fill the slots even at the minimum chunk (C1): smaller
+    // chunks, up to one task per slot (C1 0.041 -> 0.037 ms, profiles/r02/r02aj_*)
+    if (npairs * ((m + bc - 1) / bc) < slots) {
+        const int64_t b = (m * npairs + slots - 1) / (slots > 0 ? slots : 1);
+        bc = b < 1 ? 1 : (b < bc ? b : bc);
+    }
     if (bc > m) bc = m;
     w.BC = (int)bc;
     w.nbc = (int)((m + bc - 1) / bc);
