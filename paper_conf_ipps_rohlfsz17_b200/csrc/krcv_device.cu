@@ -421,6 +421,10 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L, int cls)
     const size_t pfx_rec = sizeof(double) * 2 * pk_lo_off<KR_EPANECHNIKOV>((int)L->pstride);
     L->pfx = off;      off = align256(off + (pfx_soa > pfx_rec ? pfx_soa : pfx_rec));
     L->ptot = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
+    // anchored hi records of the Epanechnikov fast path (krcv_window.cuh), window-prefix classes
+    L->pfxa = off;
+    if ((cls == kWsDefault || cls == kWsAll) && n <= kAncMaxN)
+        off = align256(off + sizeof(double) * kAncMax * pk_lo_off<KR_EPANECHNIKOV>((int)L->pstride));
     // 256 B: counters, max|y|, density statistic (bytes 0-31), BktParams (32), q32 key range (64-79)
     L->status = off;   off = align256(off + 8 * sizeof(unsigned));
     L->cub = off;      off = align256(off + cub_bytes);
@@ -640,6 +644,23 @@ static int pfx_items(int n)
 
 static void launch_bkt_fill(int n, const WsLayout &L, char *ws, cudaStream_t st);
 
+// win_kernel's anchored records (Epanechnikov, after the prefix build): one
+// thread per (index 0..n, anchor).
+template <int KERN>
+static int launch_anchors(int n, const WsLayout &L, char *ws, cudaStream_t st, bool table)
+{
+    const int J = anchors_for(n);
+    if (KERN != KR_EPANECHNIKOV || !table || J == 0) return 0;
+    const double *xs = reinterpret_cast<const double *>(ws + L.xs) + kPad;
+    const double *P = reinterpret_cast<const double *>(ws + L.pfx);
+    double *PA = reinterpret_cast<double *>(ws + L.pfxa);
+    double *OJ = reinterpret_cast<double *>(ws + L.status + 96);
+    const int64_t blocks = ((int64_t)n + kAncThreads) / kAncThreads * J;  // indices 0..n of every copy
+    launch_pdl(anchor_kernel<KR_EPANECHNIKOV>, dim3((unsigned)blocks), dim3(kAncThreads), 0, st, xs, P,
+               (int)L.pstride, n, J, PA, OJ);
+    return 1;
+}
+
 // The O(n) build of the window-prefix path: prefix moments, xs and (table:
 // win_kernel's) the bucket table.  Returns the launches enqueued.
 template <int KERN>
@@ -661,7 +682,7 @@ static int launch_prefix_build(const double2 *xy, int n, const WsLayout &L, char
         BktParams *prm = reinterpret_cast<BktParams *>(ws + L.status + 32);
         launch_pdl(pfx_fused_kernel<KERN>, dim3(tiles1), dim3(kFusedPfxThreads), 0, st, xy, n, tot, tiles1, ymax,
                    gap, P, (int)L.pstride, xs, BT, prm, arrive);
-        return 1;
+        return 1 + launch_anchors<KERN>(n, L, ws, st, table);
     }
     int launches = 2;
     if (items == 0) {
@@ -683,7 +704,7 @@ static int launch_prefix_build(const double2 *xy, int n, const WsLayout &L, char
         launch_bkt_fill(n, L, ws, st);
         launches += 1;
     }
-    return launches;
+    return launches + launch_anchors<KERN>(n, L, ws, st, table);
 }
 
 // Window kernel of r01 (window_kernel<K> / window_kernel_b2), kept for A/B
@@ -785,7 +806,8 @@ static Win2Shape win2_shape(int64_t rows, int m)
 {
     Win2Shape w;
     w.ntiles = (int)((rows + 31) / 32);
-    const int resident = occupancy((const void *)win_kernel<KERN>, kWin2Threads);
+    // (both anchor variants have the same launch bounds: 64 registers, 8 CTAs per SM)
+    const int resident = occupancy((const void *)win_kernel<KERN, false>, kWin2Threads);
     const int64_t slots = (int64_t)dev_info().sms * resident * kWin2Warps;
     static const int tpw = [] {  // KRCV_WIN2_TPW overrides (A/B runs)
         const char *e = getenv("KRCV_WIN2_TPW");
@@ -816,6 +838,32 @@ static Win2Shape win2_shape(int64_t rows, int m)
     return w;
 }
 
+// Anchors of the Epanechnikov fast path (krcv_window.cuh, anchor_kernel): J
+// copies of the prefix hi words anchored at the centres of J index regions;
+// 0 = none (the fast path reads the global records).  None below kAncMinN
+// (C2: the window kernel gains nothing, the build costs 6 us); above, the
+// most of 8 / 4 / 2 / 1 whose copies under one band of win_kernel's rows
+// (its S slots x 64 rows in flight: J band / n + 1 copies of 40 n bytes) stay
+// within kAncHotBytes of L2 -- measured C3 / C5 best at 8, C4 at 4
+// (profiles/r02/r02aq_*).  KRCV_ANCHORS = 0 .. 8 overrides (A/B runs).
+int anchors_for(int64_t n)
+{
+    static const int forced = [] {
+        const char *e = getenv("KRCV_ANCHORS");
+        return e ? atoi(e) : -1;
+    }();
+    if (n > kAncMaxN) return 0;
+    if (forced >= 0) return forced > kAncMax ? kAncMax : forced;
+    if (n < kAncMinN) return 0;
+    const double band = (double)dev_info().sms * kWin2MinBlocks * kWin2Warps * 32.0 * kWin2Rows;  // rows in flight
+    const double frac = band < (double)n ? band / (double)n : 1.0;
+    for (int J = kAncMax; J > 1; J >>= 1) {
+        const double hot = (J * frac + 1.0 < J ? J * frac + 1.0 : J) * 40.0 * (double)n;
+        if (hot <= kAncHotBytes) return J;
+    }
+    return 1;
+}
+
 // the bucket table of win_kernel (krcv_window.cuh) from the sorted x: part of
 // the O(n) build stage, after the prefix scan (which publishes the density
 // statistic it sizes the table with)
@@ -844,9 +892,17 @@ static void launch_win2(const double2 *xy, int n, const double *h, int m, int lo
     const unsigned long long *gap =
         reinterpret_cast<const unsigned long long *>(ws + L.status + 6 * sizeof(unsigned));
     BktParams *prm = reinterpret_cast<BktParams *>(ws + L.status + 32);
-    launch_pdl(win_kernel<KERN>, dim3(w.blocks), dim3(kWin2Threads), 0, st, xs, xy, P, (int)L.pstride,
-               (const int *)BT, (const BktParams *)prm, h, m, n, lo, hi, w.ntiles, w.BC, w.nbc, ymax, tileS,
-               tileN);
+    const double *PA = reinterpret_cast<const double *>(ws + L.pfxa);
+    const double *OJ = reinterpret_cast<const double *>(ws + L.status + 96);
+    const int J = KERN == KR_EPANECHNIKOV ? anchors_for(n) : 0;
+    if (J > 0)
+        launch_pdl(win_kernel<KERN, KERN == KR_EPANECHNIKOV>, dim3(w.blocks), dim3(kWin2Threads), 0, st, xs, xy, P,
+                   (int)L.pstride, (const int *)BT, (const BktParams *)prm, h, m, n, lo, hi, w.ntiles, w.BC, w.nbc,
+                   ymax, tileS, tileN, PA, J, OJ);
+    else
+        launch_pdl(win_kernel<KERN, false>, dim3(w.blocks), dim3(kWin2Threads), 0, st, xs, xy, P, (int)L.pstride,
+                   (const int *)BT, (const BktParams *)prm, h, m, n, lo, hi, w.ntiles, w.BC, w.nbc, ymax, tileS,
+                   tileN, PA, 0, OJ);
 }
 
 // Histogram ordering (krcv_hist.cuh): `warps` warps per CTA (as many as the

@@ -31,17 +31,24 @@ struct WsLayout {
     size_t status;              // uint32  [8]  n_bad_grid, n_nonfinite, reduce completion counter, pad,
                                 //              u64 bits of max |y| (window-prefix fast-path bound),
                                 //              u64 complement bits of the min x-span of kGapSpan+1 records;
-                                //              then (byte 32) the BktParams of the call (256 B region)
+                                //              then (byte 32) the BktParams of the call, (bytes 64-79) the
+                                //              q32 key range, (bytes 96-159) the anchors' origins o_j
+                                //              (anchor_kernel; 256 B region)
     size_t partial;             // double  [2m+2] partial vector of kr_cv_grid_async
     size_t xs;                  // double  [n + 2 kPad] sorted x, +-inf sentinels (prefix path)
     size_t pfx;                 // double [8][2][pstride] dd prefix moments P[k][0..n], hi / lo planes
     size_t ptot;                // double2 [8][nch] prefix tile totals
+    size_t pfxa;                // double [5 kAncMax pk_slots] anchored hi records of win_kernel (0 bytes
+                                //        for the sweep / KDE classes and above kAncMaxN)
     int64_t pstride, nch;
     size_t cub;                 // radix-sort scratch
     size_t cub_bytes;
     size_t total;
     int64_t ntiles_max;
 };
+
+// win_kernel's anchors for n points (krcv_window.cuh; 0 = none)
+int anchors_for(int64_t n);
 
 // Workspace classes: the partial-sum blocks an algorithm needs (the other
 // buffers are common): default = win_kernel slots + one partial per 32-row

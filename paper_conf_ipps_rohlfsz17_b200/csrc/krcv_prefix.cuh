@@ -727,13 +727,27 @@ struct WinRow {
     dd del;      // x_r - o, exact
 };
 
+// The Epanechnikov fast path's anchored record set for a row (win_kernel,
+// krcv_window.cuh): pa = the anchored copies (hi words, blocked layout, copy
+// j at virtual indices j S + k), joff = j S for the row's anchor j, the row's
+// shift dla = fl(x_r - o_j), and the global origin o (the dd path recomputes
+// x_r - o from it).  Anchored words are within (eps/2 + 2^-57) of their
+// magnitude of the exact anchored sums, or NaN (the fast test then fails and
+// the window is recomputed from the global dd records).  Without it the fast
+// path reads the global records about o with del.hi.
+struct WinAnc {
+    const double *pa;
+    int joff;
+    double dla, o;
+};
+
 // Squared LOO error of row `w` at bandwidth h with window [A, R) \ {r}
 // (c = R - A - 1 >= 1): prefix differences (fast path or dd), Q14 guard,
 // Eq.(2), Eq.(1)'s (y_r - g)^2.  Triangular needs P[r], P[r+1] (pr, pr1).
 template <int KERN>
 __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c, double h,
                                             const double2 *__restrict__ xy, const double *__restrict__ P, int ps,
-                                            double ymax)
+                                            double ymax, const WinAnc *an = nullptr)
 {
     const int r = w.r;
     const double xr = w.xr, yr = w.yr;
@@ -754,8 +768,11 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
             // fast path: hi words only, plain double (error test: see kFastTol)
             // records R and A (PfxRec planes (y, u), (u^2, y u), (y u^2)): two 16-byte and one
             // 8-byte load each, fixed offsets from one address
-            const double *pr = P + pk_off<KERN>(0, R);
-            const double *pa = P + pk_off<KERN>(0, A);
+            const double *base = an ? an->pa : P;
+            const int Rv = an ? R + an->joff : R, Av = an ? A + an->joff : A;  // virtual indices of copy j
+            const double *pr = base + pk_off<KERN>(0, Rv);
+            const double *pa = base + pk_off<KERN>(0, Av);
+            const double dlf = an ? an->dla : dl, adlf = fabs(dlf);
             const int q2 = kRecAos ? 2 : 2 * kRecBlock;  // offset of the (u^2, y u) pair
             const double2 r01 = __ldg(reinterpret_cast<const double2 *>(pr));
             const double2 r23 = __ldg(reinterpret_cast<const double2 *>(pr + q2));
@@ -769,24 +786,24 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
                 yuu_a = a45.x;
                 c1 = r45.y - a45.y;
             } else {
-                yuu_b = __ldg(pr + 4 * kRecBlock - (int)((unsigned)R & (kRecBlock - 1)));
-                yuu_a = __ldg(pa + 4 * kRecBlock - (int)((unsigned)A & (kRecBlock - 1)));
+                yuu_b = __ldg(pr + 4 * kRecBlock - (int)((unsigned)Rv & (kRecBlock - 1)));
+                yuu_a = __ldg(pa + 4 * kRecBlock - (int)((unsigned)Av & (kRecBlock - 1)));
                 c1 = (double)(c + 1);  // range count R - A, row r included (its terms vanish)
             }
             const double y_b = r01.x, y_a = a01.x, u_b = r01.y, u_a = a01.y;
             const double uu_b = r23.x, uu_a = a23.x, yu_b = r23.y, yu_a = a23.y;
             const double Sy = y_b - y_a, Su = u_b - u_a, Suu = uu_b - uu_a;
             const double Syu = yu_b - yu_a, Syuu = yuu_b - yuu_a;
-            s1 = fma(-dl, fma(-c1, dl, 2.0 * Su), Suu);
-            sy1 = fma(-dl, fma(-dl, Sy, 2.0 * Syu), Syuu);
+            s1 = fma(-dlf, fma(-c1, dlf, 2.0 * Su), Suu);
+            sy1 = fma(-dlf, fma(-dlf, Sy, 2.0 * Syu), Syuu);
             sy = Sy - yr;
             num = fma(hk, sy, -sy1);
             den = fma(hk, c1 - 1.0, -s1);
             const double ay = fabs(y_b) + fabs(y_a);
-            const double E1 = fabs(uu_b) + fabs(uu_a) + 2.0 * adl * (fabs(u_b) + fabs(u_a)) +
-                              2.0 * c1 * adl * (adl + h);
-            const double E2 = fabs(yuu_b) + fabs(yuu_a) + 2.0 * adl * (fabs(yu_b) + fabs(yu_a)) +
-                              2.0 * adl * adl * ay + 2.0 * c1 * ymax * adl * (adl + h);
+            double E1 = fabs(uu_b) + fabs(uu_a) + 2.0 * adlf * (fabs(u_b) + fabs(u_a)) +
+                        2.0 * c1 * adlf * (adlf + h);
+            double E2 = fabs(yuu_b) + fabs(yuu_a) + 2.0 * adlf * (fabs(yu_b) + fabs(yu_a)) +
+                        2.0 * adlf * adlf * ay + 2.0 * c1 * ymax * adlf * (adlf + h);
             const double E0 = ay + fabs(yr);
             // kFastSlack E1 <= kFastTol den, kFastSlack (hk E0 + E2) <= kFastTol den ymax, with the
             // exact power-of-two ratio kFastTol / kFastSlack folded in
@@ -809,6 +826,7 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
                 const dd Suu = wd(q2, q2);
                 const dd Syu = wd(q2 + 1, q2 + 1);
                 const dd Syuu = wd(orr, oaa);
+                const dd del = an ? two_sum(xr, -an->o) : w.del;  // x_r - o, exact
                 const dd t1 = dd_sub(dd_twice(Su), dd_mul_d_raw(del, (double)(c + 1)));
                 s1 = dd_sub_to_d(Suu, dd_mul_raw(del, t1));
                 const dd t2 = dd_sub(dd_twice(Syu), dd_mul_raw(del, Sy));

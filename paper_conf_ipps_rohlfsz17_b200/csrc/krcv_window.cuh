@@ -350,6 +350,100 @@ bkt_fill_kernel(const double *__restrict__ xs, int n, const unsigned long long *
     }
 }
 
+// ---------------------------------------------------------------------------
+// Anchored records (Epanechnikov fast path; DESIGN.md §6.2 "anchored
+// records").  The fast path reads hi words of prefix differences and shifts
+// them to the row: its error is eps times the magnitudes it combines -- the
+// prefix values at A and R, accumulated from index 0 about the global origin
+// o, and (x_r - o)^2 per window point -- so rows far from o at small h fail
+// the bound and take the dd path (18 % of (row, b) at C2-C4, 36 % at C5).  J
+// anchors s_j = floor((2 j + 1) n / (2 J)) (the centres of J equal index
+// regions) each get a copy of the hi words anchored there and taken about
+// o_j = xs[s_j]:
+//     V_j[k] = sum_{l in [s_j, k)} term_j(l)     (k >= s_j; minus the sum
+//              over [k, s_j) below), term_j = (y, u', u'^2, y u', y u'^2),
+//     u' = x - o_j,
+// computed from the global dd records P[k] - P[s_j] (S) by the exact shift
+// Delta = o_j - o (dd), c = k - s_j:
+//     V_y = S_y, V_u = S_u - c Delta, V_uu = S_uu - 2 Delta S_u + c Delta^2,
+//     V_yu = S_yu - Delta S_y, V_yuu = S_yuu - 2 Delta S_yu + Delta^2 S_y,
+// normalised and rounded to nearest.  A task's rows use the copy of their
+// region: their prefix magnitudes and shift are local.  Error of a stored
+// word beyond its rounding: the dd arithmetic's and the difference of the
+// two dd prefix values' own scan errors, bounded by
+// kappa(k) Gamma = (|k - s_j| + 2048) 2^-100 times the operand magnitudes
+// Gamma of the value (the fixed-order tiled scan accumulates its error
+// between s_j and k); where kappa Gamma > 2^-57 |V| in any of the five planes
+// the copy holds NaN at k (the fast test fails, the window is recomputed
+// from the global dd records), so every stored word is within
+// (eps/2 + 2^-57) |V| of the exact anchored sum -- inside the fast-path
+// bound's slack (kFastSlack = 16 eps).  The dd path is unchanged.
+// Copy j occupies virtual indices j S .. j S + n of one blocked record array
+// (S = pk_slots), so the fast path only adds j S to its two indices.
+constexpr int kAncMax = 8;             // anchors, at most
+constexpr int64_t kAncMaxN = 1LL << 25;  // no anchors above (their copies: 40 kAncMax B per point)
+constexpr int64_t kAncMinN = 50000;    // no anchors below (measured: no gain at C2, profiles/r02/r02aq_*)
+constexpr double kAncHotBytes = 96.0 * 1024 * 1024;  // anchored copies hot in L2 under one band, at most
+constexpr int kAncThreads = 256;
+__host__ __device__ __forceinline__ int anc_s(int j, int J, int n)
+{
+    return (int)(((int64_t)(2 * j + 1) * n) / (2 * J));
+}
+__host__ __device__ __forceinline__ int anc_of(int r, int J, int n)
+{
+    const int j = (int)(((int64_t)r * J) / n);
+    return j < J ? j : J - 1;
+}
+
+// One thread per (index k, anchor j): block b covers indices
+// (b / J) 256 .. + 255 of copy j = b mod J, so the J copies of a stretch of
+// records are written together and P[k] is read from DRAM once (anchor-major
+// blocks re-streamed P J times: C4 J = 8 build 94 -> 274 us).  OJ[j] = o_j
+// (the window kernel's table).
+template <int KERN>
+__global__ void __launch_bounds__(kAncThreads)
+anchor_kernel(const double *__restrict__ xs, const double *__restrict__ P, int ps, int n, int J,
+              double *__restrict__ PA, double *__restrict__ OJ)
+{
+    static_assert(PfxRec<KERN>::S == 5 && !kRecAos, "anchored records: the Epanechnikov blocked layout");
+    pdl_wait();  // krcv_pdl.cuh
+    const int j = (int)(blockIdx.x % (unsigned)J);
+    const int s = anc_s(j, J, n);
+    const double o = xs[n >> 1];      // pfx_origin: the median sorted record
+    const dd D = two_sum(xs[s], -o);  // o_j - o, exact
+    const dd D2 = dd_mul(D, D);
+    const double aD = fabs(D.hi) * (1.0 + 0x1p-52), aD2 = aD * aD * (1.0 + 0x1p-51);  // >= |Delta|, Delta^2
+    if (blockIdx.x < (unsigned)J && threadIdx.x == 0) OJ[j] = xs[s];
+    const int k = (int)(blockIdx.x / (unsigned)J) * blockDim.x + threadIdx.x;
+    if (k > n) return;
+    dd S[5];
+    double M[5];
+#pragma unroll
+    for (int q = 0; q < 5; q++) {
+        const dd a = pk_dd<KERN>(P, ps, q, k), b = pk_dd<KERN>(P, ps, q, s);
+        S[q] = dd_sub(a, b);
+        M[q] = fabs(a.hi) + fabs(a.lo) + fabs(b.hi) + fabs(b.lo);
+    }
+    const double c = (double)(k - s);  // exact
+    const double ac = fabs(c);
+    double V[5];
+    V[0] = S[0].hi;
+    V[1] = dd_sub(S[1], dd_mul_d(D, c)).hi;
+    V[2] = dd_add(dd_sub(S[2], dd_twice(dd_mul(D, S[1]))), dd_mul_d(D2, c)).hi;
+    V[3] = dd_sub(S[3], dd_mul(D, S[0])).hi;
+    V[4] = dd_add(dd_sub(S[4], dd_twice(dd_mul(D, S[3]))), dd_mul(D2, S[0])).hi;
+    // operand magnitudes Gamma of each value (upper bounds), kappa(k) Gamma <= 2^-57 |V| or NaN
+    const double G[5] = {M[0], M[1] + ac * aD, M[2] + 2.0 * aD * M[1] + ac * aD2, M[3] + aD * M[0],
+                         M[4] + 2.0 * aD * M[3] + aD2 * M[0]};
+    const double kap = (ac + 2048.0) * 0x1p-100 * (1.0 + 0x1p-48);
+    bool ok = true;
+#pragma unroll
+    for (int q = 0; q < 5; q++) ok = ok && kap * G[q] * (1.0 + 0x1p-50) <= 0x1p-57 * fabs(V[q]);
+    const int v = j * (int)pk_slots(ps) + k;  // virtual index of (copy j, k)
+#pragma unroll
+    for (int q = 0; q < 5; q++) PA[pk_off<KERN>(q, v)] = ok ? V[q] : __longlong_as_double(0x7ff8000000000000LL);
+}
+
 // First k in [lo, hi] with p(k) true, p monotone (false ... true), p(hi)
 // true, and p(lo - 1) false wherever it is read (the +-inf sentinels and row
 // r make that hold for both sides).  Four probes around the hint k0 settle
@@ -433,7 +527,8 @@ template <int KERN>
 __device__ __forceinline__ double row_e2(const WinRow &w, bool valid, double dmax, double dmin, double h,
                                          const double *__restrict__ xs, const double2 *__restrict__ xy,
                                          const double *__restrict__ P, int pstride, const int *__restrict__ BT,
-                                         double invw, double C, int Q, int n, double ymax, bool &M)
+                                         double invw, double C, int Q, int n, double ymax, bool &M,
+                                         const WinAnc *an = nullptr)
 {
     const int r = w.r;
     const double xr = w.xr;
@@ -448,17 +543,18 @@ __device__ __forceinline__ double row_e2(const WinRow &w, bool valid, double dma
     }
     const int c = R - A - 1;
     M = valid && c > 0;  // reading Q6
-    return M ? window_e2<KERN>(w, A, R, c, h, xy, P, pstride, ymax) : 0.0;
+    return M ? window_e2<KERN>(w, A, R, c, h, xy, P, pstride, ymax, an) : 0.0;
 }
 
-template <int KERN>
+template <int KERN, bool ANC>
 __global__ void __launch_bounds__(kWin2Threads, kWin2MinBlocks)
 win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P, int pstride,
            const int *__restrict__ BT, const BktParams *__restrict__ prm, const double *__restrict__ hg, int m,
            int n, int row_lo, int row_hi, int ntiles, int BC, int nbc,
            const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
-           uint32_t *__restrict__ tileN)
+           uint32_t *__restrict__ tileN, const double *__restrict__ PA, int J, const double *__restrict__ OJ)
 {
+    static_assert(!ANC || KERN == KR_EPANECHNIKOV, "anchored records: Epanechnikov only");
     pdl_wait();  // krcv_pdl.cuh
     const int lane = threadIdx.x & 31;
     const int S = gridDim.x * kWin2Warps;
@@ -468,6 +564,9 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
     const double xmin = xs[0], xmax = xs[n - 1];
     const double invw = prm->invw, C = prm->C;
     const int Q = prm->Q;
+    // anchored records (ANC): the anchor of a task is the region of its middle row (any anchor is exact)
+    const double rJ = (double)J / (double)n;
+    const int Sv = ANC ? (int)pk_slots(pstride) : 0;  // virtual indices per anchored copy
     // a task is kWin2Rows adjacent tiles (2: 64 rows, two rows per lane
     // sharing one butterfly per bandwidth)
     const int npairs = (ntiles + kWin2Rows - 1) / kWin2Rows;
@@ -508,6 +607,8 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
         }
         const int b0 = chunk * BC, b1 = min(m, b0 + BC);
         WinRow w0, w1;
+        int joff = 0;
+        double dla0 = 0.0, dla1 = 0.0;
         bool v0, v1 = false;
         double dmax0, dmin0, dmax1 = 0.0, dmin1 = 0.0;
         {
@@ -517,7 +618,7 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
             const double2 v = xy[w0.r];
             w0.xr = v.x;
             w0.yr = v.y;
-            w0.del = two_sum(v.x, -o);  // exact x_r - o
+            if (!ANC) w0.del = two_sum(v.x, -o);  // exact x_r - o (the anchored dd path recomputes it)
             dmax0 = xmax - v.x;
             dmin0 = v.x - xmin;
         }
@@ -528,17 +629,27 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
             const double2 v = xy[w1.r];
             w1.xr = v.x;
             w1.yr = v.y;
-            w1.del = two_sum(v.x, -o);
+            if (!ANC) w1.del = two_sum(v.x, -o);
             dmax1 = xmax - v.x;
             dmin1 = v.x - xmin;
+        }
+        if (ANC) {  // warp-uniform: the task's anchor
+            const int j = min(J - 1, (int)((double)(row_lo + t * 32 * kWin2Rows + 16 * kWin2Rows) * rJ));
+            const double oj = __ldg(OJ + j);
+            joff = j * Sv;
+            dla0 = w0.xr - oj;
+            dla1 = w1.xr - oj;
         }
         for (int b = b0; b < b1; b++) {
             const double h = __ldg(hg + b);
             bool M0, M1;
-            double e2 = row_e2<KERN>(w0, v0, dmax0, dmin0, h, xs, xy, P, pstride, BT, invw, C, Q, n, ymax, M0);
+            const WinAnc an0{PA, joff, dla0, o}, an1{PA, joff, dla1, o};
+            double e2 = row_e2<KERN>(w0, v0, dmax0, dmin0, h, xs, xy, P, pstride, BT, invw, C, Q, n, ymax, M0,
+                                     ANC ? &an0 : nullptr);
             M1 = false;
             if (kWin2Rows == 2)
-                e2 += row_e2<KERN>(w1, v1, dmax1, dmin1, h, xs, xy, P, pstride, BT, invw, C, Q, n, ymax, M1);
+                e2 += row_e2<KERN>(w1, v1, dmax1, dmin1, h, xs, xy, P, pstride, BT, invw, C, Q, n, ymax, M1,
+                                   ANC ? &an1 : nullptr);
             e2 = warp_sum(e2);  // fixed butterfly: every lane holds the task's sum
             const uint32_t nb = __popc(__ballot_sync(0xffffffffu, M0)) +
                                 (kWin2Rows == 2 ? __popc(__ballot_sync(0xffffffffu, M1)) : 0u);
