@@ -502,8 +502,10 @@ def bench_extra_configs(args, timed, dev, krcv, torch):
     stage at P = 2, 4, 8 (the P sorted-row shards timed one after another on
     this GPU through kr_cv_rows_async; equal rows and cost-balanced cuts) and
     the projected P-GPU time
-        T(P) = pack/sort + prefix/table build (replicated on every rank)
-               + window * (max shard / mean shard) / P + reduce
+        T(P) = pack/sort + prefix/table build (replicated on every rank; of
+               the anchored copies only those of the rank's rows, the
+               slowest shard's build timed) + window * (max shard / mean
+               shard) / P + reduce
                + ALLREDUCE_US_ASSUMED
     and efficiency T(1) / (P T(P)).  A projection from single-GPU stage times,
     not a multi-GPU measurement (this environment has one GPU)."""
@@ -527,13 +529,16 @@ def bench_extra_configs(args, timed, dev, krcv, torch):
         part = torch.zeros(krcv.partial_len(m), dtype=torch.float64, device=dev)
         krcv.kr_profile_enable(True)
 
-        def window_ms(lo, hi):
+        def stages_ms(lo, hi):
             for _ in range(2):  # the second run is timed (warm)
                 krcv.kr_cv_rows_async(wl["d_x"], wl["d_y"], d_h, k, lo, hi, part, ws)
                 t = krcv.kr_profile_read()
-            return t[2]
+            return t
 
-        imb_eq, imb_bal, cuts_bal = {}, {}, {}
+        def window_ms(lo, hi):
+            return stages_ms(lo, hi)[2]
+
+        imb_eq, imb_bal, cuts_bal, build_bal = {}, {}, {}, {}
         shard8 = []
         for P in (2, 4, 8):
             eq = [window_ms((s * n) // P, ((s + 1) * n) // P) for s in range(P)]
@@ -542,8 +547,12 @@ def bench_extra_configs(args, timed, dev, krcv, torch):
             imb_eq[P] = max(eq) / (sum(eq) / P)
             calib = [window_ms((s * n) // (4 * P), ((s + 1) * n) // (4 * P)) for s in range(4 * P)]
             cuts = _api.balanced_cuts(calib, n, P)
-            bal = [window_ms(cuts[s], cuts[s + 1]) for s in range(P)]
+            tb = [stages_ms(cuts[s], cuts[s + 1]) for s in range(P)]
+            bal = [t[2] for t in tb]
             imb_bal[P] = max(bal) / (sum(bal) / P)
+            # a rank's O(n) build: the prefix, the table and only the anchored
+            # copies its rows use -- the slowest shard's
+            build_bal[P] = max(t[1] for t in tb)
             cuts_bal[P] = cuts
         krcv.kr_profile_enable(False)
         del ws
@@ -553,8 +562,10 @@ def bench_extra_configs(args, timed, dev, krcv, torch):
         repl = st["pack_sort_gather"] + st["prefix_build"]
         proj, proj_eq, bound = {}, {}, {}
         for P in (2, 4, 8):
-            tp = repl + st["sweep"] * imb_bal[P] / P + fixed
-            proj[str(P)] = {"ms": tp, "efficiency": t1 / (P * tp), "imbalance": imb_bal[P]}
+            repl_p = st["pack_sort_gather"] + build_bal[P]
+            tp = repl_p + st["sweep"] * imb_bal[P] / P + fixed
+            proj[str(P)] = {"ms": tp, "efficiency": t1 / (P * tp), "imbalance": imb_bal[P],
+                            "replicated_ms": repl_p}
             tq = repl + st["sweep"] * imb_eq[P] / P + fixed
             proj_eq[str(P)] = {"ms": tq, "efficiency": t1 / (P * tq), "imbalance": imb_eq[P]}
             tb = st["sweep"] * imb_bal[P] / P + fixed
@@ -567,7 +578,9 @@ def bench_extra_configs(args, timed, dev, krcv, torch):
                      "projected_scaling_equal_rows": proj_eq,
                      "efficiency_bound_no_replicated_stage": bound,
                      "balanced_cuts": {str(P): c for P, c in cuts_bal.items()},
-                     "projection_note": ("T(P) = replicated sort + prefix/table build + window x imbalance(P) / P "
+                     "projection_note": ("T(P) = replicated sort + the slowest balanced shard's prefix/table/anchor "
+                                         "build (a rank builds only its rows' anchored copies; equal rows: the "
+                                         "whole single-GPU build) + window x imbalance(P) / P "
                                          f"+ reduce + {ALLREDUCE_US_ASSUMED} us assumed all-reduce; imbalance = "
                                          "max/mean window time of the P shards, timed one after another on this "
                                          "GPU (cost-balanced cuts, as bench.py runs N > 1; equal rows in "

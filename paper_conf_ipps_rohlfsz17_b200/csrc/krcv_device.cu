@@ -595,7 +595,8 @@ static void launch_rank_sort(const double *d_x, const double *d_y, int n, const 
                              uint32_t *khi, uint32_t *idx, int *rank, unsigned *status, int nchunks, cudaStream_t st)
 {
     chunk_sort_kernel<T, I><<<nchunks, T, 0, st>>>(d_x, d_y, n, d_h, m, keys, khi, idx, rank, status);
-    if (nchunks > 1) launch_pdl(rank_count_kernel<T, I>, dim3(nchunks, nchunks), dim3(T), 0, st, keys, khi, idx, rank);
+    if (nchunks <= 1) return;
+    launch_pdl(rank_count_kernel<T, I>, dim3(nchunks, nchunks), dim3(T), 0, st, keys, khi, idx, rank);
 }
 
 // KR_ALGO_AUTO: the window-prefix path does O(n m log) work against the
@@ -645,19 +646,22 @@ static int pfx_items(int n)
 static void launch_bkt_fill(int n, const WsLayout &L, char *ws, cudaStream_t st);
 
 // win_kernel's anchored records (Epanechnikov, after the prefix build): one
-// thread per (index 0..n, anchor).
+// thread per (index 0..n, anchor), only the copies of the anchors whose
+// regions hold rows [row_lo, row_hi) of this call (a shard of P ranks builds
+// about J / P of them).
 template <int KERN>
-static int launch_anchors(int n, const WsLayout &L, char *ws, cudaStream_t st, bool table)
+static int launch_anchors(int n, const WsLayout &L, char *ws, cudaStream_t st, bool table, int row_lo, int row_hi)
 {
     const int J = anchors_for(n);
-    if (KERN != KR_EPANECHNIKOV || !table || J == 0) return 0;
+    if (KERN != KR_EPANECHNIKOV || !table || J == 0 || row_hi <= row_lo) return 0;
+    const int j0 = anc_of(row_lo, J, n), j1 = anc_of(row_hi - 1, J, n);
     const double *xs = reinterpret_cast<const double *>(ws + L.xs) + kPad;
     const double *P = reinterpret_cast<const double *>(ws + L.pfx);
     double *PA = reinterpret_cast<double *>(ws + L.pfxa);
     double *OJ = reinterpret_cast<double *>(ws + L.status + 96);
-    const int64_t blocks = ((int64_t)n + kAncThreads) / kAncThreads * J;  // indices 0..n of every copy
+    const int64_t blocks = ((int64_t)n + kAncThreads) / kAncThreads * (j1 - j0 + 1);  // indices 0..n per copy
     launch_pdl(anchor_kernel<KR_EPANECHNIKOV>, dim3((unsigned)blocks), dim3(kAncThreads), 0, st, xs, P,
-               (int)L.pstride, n, J, PA, OJ);
+               (int)L.pstride, n, J, j0, j1 - j0 + 1, PA, OJ);
     return 1;
 }
 
@@ -665,7 +669,7 @@ static int launch_anchors(int n, const WsLayout &L, char *ws, cudaStream_t st, b
 // win_kernel's) the bucket table.  Returns the launches enqueued.
 template <int KERN>
 static int launch_prefix_build(const double2 *xy, int n, const WsLayout &L, char *ws, cudaStream_t st,
-                               bool table = false)
+                               bool table = false, int row_lo = 0, int row_hi = 0)
 {
     double *xs = reinterpret_cast<double *>(ws + L.xs) + kPad;
     double *P = reinterpret_cast<double *>(ws + L.pfx);
@@ -682,7 +686,7 @@ static int launch_prefix_build(const double2 *xy, int n, const WsLayout &L, char
         BktParams *prm = reinterpret_cast<BktParams *>(ws + L.status + 32);
         launch_pdl(pfx_fused_kernel<KERN>, dim3(tiles1), dim3(kFusedPfxThreads), 0, st, xy, n, tot, tiles1, ymax,
                    gap, P, (int)L.pstride, xs, BT, prm, arrive);
-        return 1 + launch_anchors<KERN>(n, L, ws, st, table);
+        return 1 + launch_anchors<KERN>(n, L, ws, st, table, row_lo, row_hi);
     }
     int launches = 2;
     if (items == 0) {
@@ -704,7 +708,7 @@ static int launch_prefix_build(const double2 *xy, int n, const WsLayout &L, char
         launch_bkt_fill(n, L, ws, st);
         launches += 1;
     }
-    return launches + launch_anchors<KERN>(n, L, ws, st, table);
+    return launches + launch_anchors<KERN>(n, L, ws, st, table, row_lo, row_hi);
 }
 
 // Window kernel of r01 (window_kernel<K> / window_kernel_b2), kept for A/B
@@ -895,14 +899,16 @@ static void launch_win2(const double2 *xy, int n, const double *h, int m, int lo
     const double *PA = reinterpret_cast<const double *>(ws + L.pfxa);
     const double *OJ = reinterpret_cast<const double *>(ws + L.status + 96);
     const int J = KERN == KR_EPANECHNIKOV ? anchors_for(n) : 0;
+    // the anchors launch_anchors built for these rows (the kernel clamps its choice to them)
+    const int j0 = J > 0 && hi > lo ? anc_of(lo, J, n) : 0, j1 = J > 0 && hi > lo ? anc_of(hi - 1, J, n) : 0;
     if (J > 0)
         launch_pdl(win_kernel<KERN, KERN == KR_EPANECHNIKOV>, dim3(w.blocks), dim3(kWin2Threads), 0, st, xs, xy, P,
                    (int)L.pstride, (const int *)BT, (const BktParams *)prm, h, m, n, lo, hi, w.ntiles, w.BC, w.nbc,
-                   ymax, tileS, tileN, PA, J, OJ);
+                   ymax, tileS, tileN, PA, J, j0, j1, OJ);
     else
         launch_pdl(win_kernel<KERN, false>, dim3(w.blocks), dim3(kWin2Threads), 0, st, xs, xy, P, (int)L.pstride,
                    (const int *)BT, (const BktParams *)prm, h, m, n, lo, hi, w.ntiles, w.BC, w.nbc, ymax, tileS,
-                   tileN, PA, 0, OJ);
+                   tileN, PA, 0, 0, 0, OJ);
 }
 
 // Histogram ordering (krcv_hist.cuh): `warps` warps per CTA (as many as the
@@ -1188,7 +1194,9 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         // win_kernel's bucket table is part of the build (depends on xs only: kept on reuse)
         switch (kernel) {
         case KR_UNIFORM: launches += launch_prefix_build<KR_UNIFORM>(xy, nn, L, ws, st, win2); break;
-        case KR_EPANECHNIKOV: launches += launch_prefix_build<KR_EPANECHNIKOV>(xy, nn, L, ws, st, win2); break;
+        case KR_EPANECHNIKOV:
+            launches += launch_prefix_build<KR_EPANECHNIKOV>(xy, nn, L, ws, st, win2, lo, hi);
+            break;
         default: launches += launch_prefix_build<KR_TRIANGULAR>(xy, nn, L, ws, st, win2); break;
         }
     }

@@ -395,26 +395,26 @@ __host__ __device__ __forceinline__ int anc_of(int r, int J, int n)
     return j < J ? j : J - 1;
 }
 
-// One thread per (index k, anchor j): block b covers indices
-// (b / J) 256 .. + 255 of copy j = b mod J, so the J copies of a stretch of
-// records are written together and P[k] is read from DRAM once (anchor-major
-// blocks re-streamed P J times: C4 J = 8 build 94 -> 274 us).  OJ[j] = o_j
-// (the window kernel's table).
+// One thread per (index k, anchor j) for the nj anchors j0 .. j0 + nj - 1:
+// block b covers indices (b / nj) 256 .. + 255 of copy j = j0 + b mod nj, so
+// the copies of a stretch of records are written together and P[k] is read
+// from DRAM once (anchor-major blocks re-streamed P J times: C4 J = 8 build
+// 94 -> 274 us).  OJ[j] = o_j (the window kernel's table).
 template <int KERN>
 __global__ void __launch_bounds__(kAncThreads)
-anchor_kernel(const double *__restrict__ xs, const double *__restrict__ P, int ps, int n, int J,
+anchor_kernel(const double *__restrict__ xs, const double *__restrict__ P, int ps, int n, int J, int j0, int nj,
               double *__restrict__ PA, double *__restrict__ OJ)
 {
     static_assert(PfxRec<KERN>::S == 5 && !kRecAos, "anchored records: the Epanechnikov blocked layout");
     pdl_wait();  // krcv_pdl.cuh
-    const int j = (int)(blockIdx.x % (unsigned)J);
+    const int j = j0 + (int)(blockIdx.x % (unsigned)nj);
     const int s = anc_s(j, J, n);
     const double o = xs[n >> 1];      // pfx_origin: the median sorted record
     const dd D = two_sum(xs[s], -o);  // o_j - o, exact
     const dd D2 = dd_mul(D, D);
     const double aD = fabs(D.hi) * (1.0 + 0x1p-52), aD2 = aD * aD * (1.0 + 0x1p-51);  // >= |Delta|, Delta^2
-    if (blockIdx.x < (unsigned)J && threadIdx.x == 0) OJ[j] = xs[s];
-    const int k = (int)(blockIdx.x / (unsigned)J) * blockDim.x + threadIdx.x;
+    if (blockIdx.x < (unsigned)nj && threadIdx.x == 0) OJ[j] = xs[s];
+    const int k = (int)(blockIdx.x / (unsigned)nj) * blockDim.x + threadIdx.x;
     if (k > n) return;
     dd S[5];
     double M[5];
@@ -552,7 +552,8 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
            const int *__restrict__ BT, const BktParams *__restrict__ prm, const double *__restrict__ hg, int m,
            int n, int row_lo, int row_hi, int ntiles, int BC, int nbc,
            const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
-           uint32_t *__restrict__ tileN, const double *__restrict__ PA, int J, const double *__restrict__ OJ)
+           uint32_t *__restrict__ tileN, const double *__restrict__ PA, int J, int j0, int j1,
+           const double *__restrict__ OJ)
 {
     static_assert(!ANC || KERN == KR_EPANECHNIKOV, "anchored records: Epanechnikov only");
     pdl_wait();  // krcv_pdl.cuh
@@ -633,8 +634,9 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
             dmax1 = xmax - v.x;
             dmin1 = v.x - xmin;
         }
-        if (ANC) {  // warp-uniform: the task's anchor
-            const int j = min(J - 1, (int)((double)(row_lo + t * 32 * kWin2Rows + 16 * kWin2Rows) * rJ));
+        if (ANC) {  // warp-uniform: the task's anchor, among the copies built for rows [row_lo, row_hi)
+            const int mid = min(row_lo + t * 32 * kWin2Rows + 16 * kWin2Rows, row_hi - 1);
+            const int j = min(j1, max(j0, (int)((double)mid * rJ)));
             const double oj = __ldg(OJ + j);
             joff = j * Sv;
             dla0 = w0.xr - oj;

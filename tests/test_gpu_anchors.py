@@ -65,3 +65,41 @@ def test_anchored_matches_oracle_and_unanchored(anchor_cases, unanchored, refs, 
         base = np.array(unanchored[c]["cv"], np.uint64).view(np.float64)
         scale = max(float(np.max(np.abs(base))), 1e-300)
         assert float(np.max(np.abs(got - base))) <= 1e-13 * scale, (c, J)
+
+
+def test_anchored_row_ranges_sum_to_unsharded():
+    """A row range builds only the anchored copies of its rows' regions (DESIGN.md
+    §6.2) and clamps every task's anchor to them: disjoint ranges -- cutting
+    through anchor regions (n / 8 = 7,500 rows here), ending one and two rows
+    past a region boundary, spanning several regions, empty -- on one reused
+    workspace add up to the unsharded partial (windows exactly, sums to
+    rounding), and one range equals Program 3 on exactly those sorted rows."""
+    import torch
+
+    import oracle
+    import workloads
+    from paper_conf_ipps_rohlfsz17_b200 import krcv
+    from tests.helpers import cv_rel_err
+
+    x, y, h, k = workloads.make("C5", seed=4, n=60000)
+    h = h[::8].copy()
+    m = h.shape[0]
+    d_x, d_y, d_h = (torch.as_tensor(v, device="cuda") for v in (x, y, h))
+    ws = krcv.aligned(krcv.workspace(x.shape[0], m, "cuda"))
+    part = torch.empty(krcv.partial_len(m), dtype=torch.float64, device="cuda")
+    krcv.kr_cv_rows_async(d_x, d_y, d_h, k, 0, 60000, part, ws)
+    torch.cuda.synchronize()
+    full = part.cpu().numpy().copy()
+    cuts = [0, 7490, 7501, 7502, 7502, 22500, 22530, 51000, 59999, 60000]
+    tot = np.zeros(krcv.partial_len(m))
+    for lo, hi in zip(cuts, cuts[1:]):
+        krcv.kr_cv_rows_async(d_x, d_y, d_h, k, lo, hi, part, ws)
+        torch.cuda.synchronize()
+        p = part.cpu().numpy()
+        tot += p
+        if (lo, hi) == (7490, 7501):
+            ref = oracle.cv_sorted(x, y, h, k, rows=oracle.sorted_rows(x)[lo:hi])
+            assert cv_rel_err(p[:m], ref.S) <= 1e-10
+            assert np.array_equal(p[m:2 * m].astype(np.int64), ref.neff)
+    assert cv_rel_err(tot[:m], full[:m]) <= 1e-13
+    assert np.array_equal(tot[m:], full[m:])
