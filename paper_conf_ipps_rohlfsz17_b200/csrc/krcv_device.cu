@@ -423,8 +423,8 @@ bool ws_layout(int64_t n, int32_t m, WsLayout *L, int cls)
     L->ptot = off;     off = align256(off + sizeof(double2) * kPfxMoments * nch);
     // anchored hi records of the Epanechnikov fast path (krcv_window.cuh), window-prefix classes
     L->pfxa = off;
-    if ((cls == kWsDefault || cls == kWsAll) && n <= kAncMaxN)
-        off = align256(off + sizeof(double) * kAncMax * pk_lo_off<KR_EPANECHNIKOV>((int)L->pstride));
+    if (cls == kWsDefault || cls == kWsAll)  // anchors_for: 0 below n = 50,000 and above kAncMaxN
+        off = align256(off + sizeof(double) * anchors_for(n) * pk_lo_off<KR_EPANECHNIKOV>((int)L->pstride));
     // 256 B: counters, max|y|, density statistic (bytes 0-31), BktParams (32), q32 key range (64-79)
     L->status = off;   off = align256(off + 8 * sizeof(unsigned));
     L->cub = off;      off = align256(off + cub_bytes);

@@ -38,8 +38,8 @@ struct WsLayout {
     size_t xs;                  // double  [n + 2 kPad] sorted x, +-inf sentinels (prefix path)
     size_t pfx;                 // double [8][2][pstride] dd prefix moments P[k][0..n], hi / lo planes
     size_t ptot;                // double2 [8][nch] prefix tile totals
-    size_t pfxa;                // double [5 kAncMax pk_slots] anchored hi records of win_kernel (0 bytes
-                                //        for the sweep / KDE classes and above kAncMaxN)
+    size_t pfxa;                // double [5 J pk_slots] anchored hi records of win_kernel, J = anchors_for(n)
+                                //        (0 bytes for the sweep / KDE classes, below 50,000 and above kAncMaxN)
     int64_t pstride, nch;
     size_t cub;                 // radix-sort scratch
     size_t cub_bytes;

@@ -717,6 +717,9 @@ __device__ __forceinline__ double fast_div(double a, double b)
     return fma(r, fma(-b, q, a), q);
 }
 
+#ifndef KRCV_EFACT
+#define KRCV_EFACT 1  // factored fast-path bound (build-time A/B)
+#endif
 constexpr double kFastSlack = 16.0 * 0x1p-53;
 constexpr double kFastTol = 0x1p-44;
 
@@ -800,10 +803,20 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
             num = fma(hk, sy, -sy1);
             den = fma(hk, c1 - 1.0, -s1);
             const double ay = fabs(y_b) + fabs(y_a);
-            double E1 = fabs(uu_b) + fabs(uu_a) + 2.0 * adlf * (fabs(u_b) + fabs(u_a)) +
-                        2.0 * c1 * adlf * (adlf + h);
-            double E2 = fabs(yuu_b) + fabs(yuu_a) + 2.0 * adlf * (fabs(yu_b) + fabs(yu_a)) +
-                        2.0 * adlf * adlf * ay + 2.0 * c1 * ymax * adlf * (adlf + h);
+            // E1 = |uu_b| + |uu_a| + 2|d| (|u_b| + |u_a|) + 2 c1 |d| (|d| + h),
+            // E2 = |yuu_b| + |yuu_a| + 2|d| (|yu_b| + |yu_a|) + 2 d^2 ay + 2 c1 max|y| |d| (|d| + h),
+            // factored (the same bounds to rounding, which the slack covers)
+#if KRCV_EFACT
+            const double dh = adlf + h, d2 = 2.0 * adlf;
+            const double E1 = fma(d2, fma(c1, dh, fabs(u_b) + fabs(u_a)), fabs(uu_b) + fabs(uu_a));
+            const double E2 = fma(d2, fma(c1 * ymax, dh, fma(adlf, ay, fabs(yu_b) + fabs(yu_a))),
+                                  fabs(yuu_b) + fabs(yuu_a));
+#else
+            const double E1 = fabs(uu_b) + fabs(uu_a) + 2.0 * adlf * (fabs(u_b) + fabs(u_a)) +
+                              2.0 * c1 * adlf * (adlf + h);
+            const double E2 = fabs(yuu_b) + fabs(yuu_a) + 2.0 * adlf * (fabs(yu_b) + fabs(yu_a)) +
+                              2.0 * adlf * adlf * ay + 2.0 * c1 * ymax * adlf * (adlf + h);
+#endif
             const double E0 = ay + fabs(yr);
             // kFastSlack E1 <= kFastTol den, kFastSlack (hk E0 + E2) <= kFastTol den ymax, with the
             // exact power-of-two ratio kFastTol / kFastSlack folded in
@@ -854,7 +867,7 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
             num = fma(hk, sy, -sy1);
             den = fma(hk, (double)c, -s1);
         }
-        if (!(den >= 0x1p-20 * hk * (double)c)) {  // reading Q14
+        if (!(den >= 0x1p-20 * hk * (double)c)) {  // reading Q14 ((double)c: exact)
             num = 0.0;
             den = 0.0;
             for (int q = A; q < R; q++) {

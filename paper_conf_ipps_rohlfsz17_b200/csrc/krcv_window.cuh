@@ -656,7 +656,12 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
             const uint32_t nb = __popc(__ballot_sync(0xffffffffu, M0)) +
                                 (kWin2Rows == 2 ? __popc(__ballot_sync(0xffffffffu, M1)) : 0u);
             const int bl = b - b0;
-            if (lane == (bl & 31)) {
+            if (kWin2Acc == 1) {  // bl < 32: lane bl keeps bandwidth b's sums
+                if (lane == bl) {
+                    acc[0] += e2;
+                    cnt[0] += nb;
+                }
+            } else if (lane == (bl & 31)) {
 #pragma unroll
                 for (int a = 0; a < kWin2Acc; a++)
                     if ((bl >> 5) == a) {
