@@ -846,7 +846,7 @@ static Win2Shape win2_shape(int64_t rows, int m)
 // copies of the prefix hi words anchored at the centres of J index regions;
 // 0 = none (the fast path reads the global records).  None below kAncMinN
 // (C2: the window kernel gains nothing, the build costs 6 us); above, the
-// most of 8 / 4 / 2 / 1 whose copies under one band of win_kernel's rows
+// most of 16 / 8 / 4 / 2 / 1 whose copies under one band of win_kernel's rows
 // (its S slots x 64 rows in flight: J band / n + 1 copies of 40 n bytes) stay
 // within kAncHotBytes of L2 -- measured C3 / C5 best at 8, C4 at 4
 // (profiles/r02/r02aq_*).  KRCV_ANCHORS = 0 .. 8 overrides (A/B runs).

@@ -32,7 +32,7 @@ struct WsLayout {
                                 //              u64 bits of max |y| (window-prefix fast-path bound),
                                 //              u64 complement bits of the min x-span of kGapSpan+1 records;
                                 //              then (byte 32) the BktParams of the call, (bytes 64-79) the
-                                //              q32 key range, (bytes 96-159) the anchors' origins o_j
+                                //              q32 key range, (bytes 96-223) the anchors' origins o_j
                                 //              (anchor_kernel; 256 B region)
     size_t partial;             // double  [2m+2] partial vector of kr_cv_grid_async
     size_t xs;                  // double  [n + 2 kPad] sorted x, +-inf sentinels (prefix path)

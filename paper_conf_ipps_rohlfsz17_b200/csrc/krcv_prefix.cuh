@@ -839,11 +839,11 @@ __device__ __forceinline__ double window_e2(const WinRow &w, int A, int R, int c
                 const dd Suu = wd(q2, q2);
                 const dd Syu = wd(q2 + 1, q2 + 1);
                 const dd Syuu = wd(orr, oaa);
-                const dd del = an ? two_sum(xr, -an->o) : w.del;  // x_r - o, exact
-                const dd t1 = dd_sub(dd_twice(Su), dd_mul_d_raw(del, (double)(c + 1)));
-                s1 = dd_sub_to_d(Suu, dd_mul_raw(del, t1));
-                const dd t2 = dd_sub(dd_twice(Syu), dd_mul_raw(del, Sy));
-                sy1 = dd_sub_to_d(Syuu, dd_mul_raw(del, t2));
+                const dd dlt = an ? two_sum(xr, -an->o) : del;  // x_r - o, exact (anchored rows keep none)
+                const dd t1 = dd_sub(dd_twice(Su), dd_mul_d_raw(dlt, (double)(c + 1)));
+                s1 = dd_sub_to_d(Suu, dd_mul_raw(dlt, t1));
+                const dd t2 = dd_sub(dd_twice(Syu), dd_mul_raw(dlt, Sy));
+                sy1 = dd_sub_to_d(Syuu, dd_mul_raw(dlt, t2));
                 sy = dd_sub_to_d(Sy, dd_make(yr));
             } else {  // triangular: right (r, R) and left [A, r) separately
                 const dd SyR = pk_wsum<KERN>(P, ps, 0, r + 1, R);

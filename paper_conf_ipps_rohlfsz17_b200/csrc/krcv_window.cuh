@@ -380,7 +380,7 @@ bkt_fill_kernel(const double *__restrict__ xs, int n, const unsigned long long *
 // bound's slack (kFastSlack = 16 eps).  The dd path is unchanged.
 // Copy j occupies virtual indices j S .. j S + n of one blocked record array
 // (S = pk_slots), so the fast path only adds j S to its two indices.
-constexpr int kAncMax = 8;             // anchors, at most
+constexpr int kAncMax = 16;            // anchors, at most (o_j table: status bytes 96-223)
 constexpr int64_t kAncMaxN = 1LL << 25;  // no anchors above (their copies: 40 kAncMax B per point)
 constexpr int64_t kAncMinN = 50000;    // no anchors below (measured: no gain at C2, profiles/r02/r02aq_*)
 constexpr double kAncHotBytes = 96.0 * 1024 * 1024;  // anchored copies hot in L2 under one band, at most
@@ -619,7 +619,7 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
             const double2 v = xy[w0.r];
             w0.xr = v.x;
             w0.yr = v.y;
-            if (!ANC) w0.del = two_sum(v.x, -o);  // exact x_r - o (the anchored dd path recomputes it)
+            w0.del = ANC ? dd{0.0, 0.0} : two_sum(v.x, -o);  // exact x_r - o (the anchored dd path recomputes it)
             dmax0 = xmax - v.x;
             dmin0 = v.x - xmin;
         }
@@ -630,7 +630,7 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
             const double2 v = xy[w1.r];
             w1.xr = v.x;
             w1.yr = v.y;
-            if (!ANC) w1.del = two_sum(v.x, -o);
+            w1.del = ANC ? dd{0.0, 0.0} : two_sum(v.x, -o);
             dmax1 = xmax - v.x;
             dmin1 = v.x - xmin;
         }

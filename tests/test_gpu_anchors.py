@@ -50,7 +50,7 @@ def refs(anchor_cases):
     return {c: oracle.cv_sorted(x, y, h, 1) for c, (x, y, h, _) in anchor_cases[1].items()}
 
 
-@pytest.mark.parametrize("J", ["1", "3", "8", "default"])
+@pytest.mark.parametrize("J", ["1", "3", "8", "16", "default"])
 def test_anchored_matches_oracle_and_unanchored(anchor_cases, unanchored, refs, J):
     from tests.helpers import best_ok, cv_rel_err
 

@@ -160,7 +160,8 @@ def _device_partial(x, y, h, k, shard, nshards):
     return part.cpu().numpy()
 
 
-@pytest.mark.parametrize("cfg,P,shard", [("C3", 64, 17), ("C5", 64, 0), ("C5", 64, 63), ("C4", 4096, 2048)])
+@pytest.mark.parametrize("cfg,P,shard", [("C3", 64, 17), ("C5", 64, 0), ("C5", 64, 63), ("C4", 4096, 2048),
+                                         ("C4", 4096, 40)])
 def test_full_size_sampled_shard(cfg, P, shard):
     """Full BASELINE sizes in the bench launch configuration: one row shard of
     the sorted order, checked against the oracle on exactly those rows."""
