@@ -898,17 +898,22 @@ static void launch_win2(const double2 *xy, int n, const double *h, int m, int lo
     BktParams *prm = reinterpret_cast<BktParams *>(ws + L.status + 32);
     const double *PA = reinterpret_cast<const double *>(ws + L.pfxa);
     const double *OJ = reinterpret_cast<const double *>(ws + L.status + 96);
+    Win2Sched sc;
+    sc.npairs = (w.ntiles + kWin2Rows - 1) / kWin2Rows;
+    sc.s_div = w.S / sc.npairs;
+    sc.s_mod = w.S % sc.npairs;
+    sc.ntasks = (long long)sc.npairs * w.nbc;
     const int J = KERN == KR_EPANECHNIKOV ? anchors_for(n) : 0;
     // the anchors launch_anchors built for these rows (the kernel clamps its choice to them)
     const int j0 = J > 0 && hi > lo ? anc_of(lo, J, n) : 0, j1 = J > 0 && hi > lo ? anc_of(hi - 1, J, n) : 0;
     if (J > 0)
         launch_pdl(win_kernel<KERN, KERN == KR_EPANECHNIKOV>, dim3(w.blocks), dim3(kWin2Threads), 0, st, xs, xy, P,
                    (int)L.pstride, (const int *)BT, (const BktParams *)prm, h, m, n, lo, hi, w.ntiles, w.BC, w.nbc,
-                   ymax, tileS, tileN, PA, J, j0, j1, OJ);
+                   ymax, tileS, tileN, PA, J, j0, j1, OJ, sc);
     else
         launch_pdl(win_kernel<KERN, false>, dim3(w.blocks), dim3(kWin2Threads), 0, st, xs, xy, P, (int)L.pstride,
                    (const int *)BT, (const BktParams *)prm, h, m, n, lo, hi, w.ntiles, w.BC, w.nbc, ymax, tileS,
-                   tileN, PA, 0, 0, 0, OJ);
+                   tileN, PA, 0, 0, 0, OJ, sc);
 }
 
 // Histogram ordering (krcv_hist.cuh): `warps` warps per CTA (as many as the

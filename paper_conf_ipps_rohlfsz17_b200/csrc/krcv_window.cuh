@@ -546,6 +546,14 @@ __device__ __forceinline__ double row_e2(const WinRow &w, bool valid, double dma
     return M ? window_e2<KERN>(w, A, R, c, h, xy, P, pstride, ymax, an) : 0.0;
 }
 
+// Task-schedule constants of a win_kernel launch (host-computed): npairs
+// tile pairs per chunk, ntasks = npairs nbc, S / npairs and S mod npairs for
+// the incremental task index (S = the grid's warp slots).
+struct Win2Sched {
+    int npairs, s_div, s_mod;
+    long long ntasks;
+};
+
 template <int KERN, bool ANC>
 __global__ void __launch_bounds__(kWin2Threads, kWin2MinBlocks)
 win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const double *__restrict__ P, int pstride,
@@ -553,7 +561,7 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
            int n, int row_lo, int row_hi, int ntiles, int BC, int nbc,
            const unsigned long long *__restrict__ ymax_bits, double *__restrict__ tileS,
            uint32_t *__restrict__ tileN, const double *__restrict__ PA, int J, int j0, int j1,
-           const double *__restrict__ OJ)
+           const double *__restrict__ OJ, Win2Sched sc)
 {
     static_assert(!ANC || KERN == KR_EPANECHNIKOV, "anchored records: Epanechnikov only");
     pdl_wait();  // krcv_pdl.cuh
@@ -570,8 +578,10 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
     const int Sv = ANC ? (int)pk_slots(pstride) : 0;  // virtual indices per anchored copy
     // a task is kWin2Rows adjacent tiles (2: 64 rows, two rows per lane
     // sharing one butterfly per bandwidth)
-    const int npairs = (ntiles + kWin2Rows - 1) / kWin2Rows;
-    const int64_t ntasks = (int64_t)npairs * nbc;
+    // schedule constants from the host (kernel parameters: the 64-register
+    // kernel would otherwise recompute S mod npairs per task)
+    const int npairs = sc.npairs;
+    const int64_t ntasks = sc.ntasks;
     int cur = -1;  // chunk of the running sums
     double acc[kWin2Acc];
     uint32_t cnt[kWin2Acc];
@@ -600,8 +610,8 @@ win_kernel(const double *__restrict__ xs, const double2 *__restrict__ xy, const 
             cur = chunk;
         }
         const int t = kt;
-        kt += S % npairs;
-        kchunk += S / npairs;
+        kt += sc.s_mod;
+        kchunk += sc.s_div;
         if (kt >= npairs) {
             kt -= npairs;
             kchunk += 1;
