@@ -230,7 +230,9 @@ size_t kr_workspace_bytes(int64_t n, int32_t m);
  * `algo` (KR_ALGO_*; KR_ALGO_AUTO resolves as the call would) -- the
  * per-algorithm partial-sum blocks only (the split sweep's per-tile partials
  * are the largest; the default window-prefix path needs a few MB per 1,000
- * bandwidths) -- and the one the KDE entry points need.  An entry point given
+ * bandwidths, plus, from n = 50,000 to 2^25, J <= 16 anchored copies of the
+ * prefix records at 40 n bytes each -- J = 4 (160 MB) at n = 10^6, DESIGN.md
+ * §6.2) -- and the one the KDE entry points need.  An entry point given
  * less than its requirement returns KR_EARG.  0 for invalid (n, m). */
 size_t kr_workspace_bytes_algo(int64_t n, int32_t m, int32_t kernel, int32_t algo);
 size_t kr_kde_workspace_bytes(int64_t n, int32_t m);
