@@ -96,7 +96,9 @@ enum {
                            chosen by AUTO): O(n^2) bucketed pairs with
                            shared-memory atomics; sums agree with the other
                            paths to rounding, not bitwise (atomic order).
-                           m <= 5,000 (shared-memory histogram; KR_EARG above) */
+                           Grids larger than one shared-memory histogram
+                           (m > ~4,800) run in slices of ~2,600 bandwidths,
+                           one O(n^2) pass each */
 };
 
 /* Length of the partial vector of the device path: [ S[0..m) | neff[0..m) |

@@ -1147,12 +1147,15 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
     const bool prefix = algo == KR_ALGO_PREFIX;
     const bool dense = algo == KR_ALGO_DENSE;
     const bool hist = algo == KR_ALGO_HIST;
-    int hist_warps = 0;
+    int hist_warps = 0, hist_mc = m;
     if (hist) {  // shared-memory histogram: warps per CTA that fit 227 KB
         const size_t cap = 227 * 1024;
         for (int w = kHistMaxWarps; w >= 1 && !hist_warps; w--)
             if (hist_smem_bytes(m, w) <= cap) hist_warps = w;
-        if (!hist_warps) return KR_EARG;
+        if (!hist_warps) {  // grid too large for one histogram: slices of the grid, two warps per CTA
+            hist_warps = 2;
+            hist_mc = (int)(cap / hist_smem_bytes(1, hist_warps));
+        }
     }
     const int variant = sweep_variant(hi - lo);
     int G = sweep_G(hi - lo);
@@ -1211,20 +1214,36 @@ static int enqueue(const double *d_x, const double *d_y, int64_t n, const double
         NvtxScope nv("krcv: a3+a4 windows, LOO estimates, squared errors");
         launches += 1;
         if (hist) {
+            // Grids larger than one shared-memory histogram run as slices
+            // [b0, b0 + mc) of the grid: a neighbour's bucket within a slice is
+            // the first of ITS bandwidths whose window holds it (bucket 0 =
+            // inside h_b0 already), so each slice's running sums are exactly the
+            // full grid's at those bandwidths; the slice writes its rows of the
+            // [m][ntiles] partials.  The tile counter is reset between slices.
             const uint32_t *perm = reinterpret_cast<const uint32_t *>(ws + L.perm);
-            switch (kernel) {
-            case KR_UNIFORM:
-                launch_hist<KR_UNIFORM>(hist_warps, d_x, d_y, perm, xy, d_h, m, nn, lo, hi, ntiles, tileS, tileN,
-                                        counter, st);
-                break;
-            case KR_EPANECHNIKOV:
-                launch_hist<KR_EPANECHNIKOV>(hist_warps, d_x, d_y, perm, xy, d_h, m, nn, lo, hi, ntiles, tileS,
-                                             tileN, counter, st);
-                break;
-            default:
-                launch_hist<KR_TRIANGULAR>(hist_warps, d_x, d_y, perm, xy, d_h, m, nn, lo, hi, ntiles, tileS, tileN,
-                                           counter, st);
-                break;
+            for (int b0 = 0; b0 < m; b0 += hist_mc) {
+                const int mc = m - b0 < hist_mc ? m - b0 : hist_mc;
+                if (b0 > 0) {
+                    e = cudaMemsetAsync(counter, 0, sizeof(int), st);
+                    if (e != cudaSuccess) { set_cuda_error("cudaMemsetAsync(counter)", (int)e); return KR_ECUDA; }
+                    launches += 1;
+                }
+                double *tS = tileS + (size_t)b0 * ntiles;
+                uint8_t *tN = tileN + (size_t)b0 * ntiles;
+                switch (kernel) {
+                case KR_UNIFORM:
+                    launch_hist<KR_UNIFORM>(hist_warps, d_x, d_y, perm, xy, d_h + b0, mc, nn, lo, hi, ntiles, tS, tN,
+                                            counter, st);
+                    break;
+                case KR_EPANECHNIKOV:
+                    launch_hist<KR_EPANECHNIKOV>(hist_warps, d_x, d_y, perm, xy, d_h + b0, mc, nn, lo, hi, ntiles, tS,
+                                                 tN, counter, st);
+                    break;
+                default:
+                    launch_hist<KR_TRIANGULAR>(hist_warps, d_x, d_y, perm, xy, d_h + b0, mc, nn, lo, hi, ntiles, tS,
+                                               tN, counter, st);
+                    break;
+                }
             }
         } else if (dense) {
             const int nrt = (hi - lo + kGThreads - 1) / kGThreads;

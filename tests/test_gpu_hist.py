@@ -67,15 +67,18 @@ def test_hist_C2_full_size_sampled_shard(k):
     assert np.array_equal(p[m:2 * m].astype(np.int64), ref.neff)
 
 
-def test_hist_grid_size_limits():
-    """m = 4,099 runs with one warp per CTA; m = 6,000 does not fit the
-    shared-memory histogram (KR_EARG); the Gaussian kernel is rejected."""
+@pytest.mark.parametrize("k", [U, E, T])
+def test_hist_grid_size_limits(k):
+    """m = 4,099 runs in one shared-memory histogram with one warp per CTA;
+    m = 6,000 and 12,345 do not fit one and run as slices of the grid (a
+    bucket is the first bandwidth of the slice whose window holds the
+    neighbour, so each slice's running sums are the full grid's); the
+    Gaussian kernel is rejected."""
     x, y = workloads.draw_xy("paper", 300, 2)
-    h = workloads.grid_default(x, 4099)
-    _check(x, y, h, E)
-    with pytest.raises(krcv.KrcvError) as e:
-        krcv.kr_cv_grid(x, y, workloads.grid_default(x, 6000), E, algo="hist")
-    assert e.value.status == krcv.KR_EARG
+    _check(x, y, workloads.grid_default(x, 4099), k)
+    _check(x, y, workloads.grid_default(x, 6000), k)
+    r = float(x.max() - x.min())
+    _check(x, y, np.geomspace(1e-4 * r, 2.0 * r, 12345), k)
     with pytest.raises(krcv.KrcvError) as e:
         krcv.kr_cv_grid(x, y, workloads.grid_default(x, 10), GA, algo="hist")
     assert e.value.status == krcv.KR_EARG
