@@ -818,10 +818,15 @@ static Win2Shape win2_shape(int64_t rows, int m)
         const int v = e ? atoi(e) : 0;
         return v > 0 ? v : kWin2TasksPerWarp;
     }();
+    static const int min_chunk = [] {  // KRCV_WIN2_MINCHUNK overrides (A/B runs)
+        const char *e = getenv("KRCV_WIN2_MINCHUNK");
+        const int v = e ? atoi(e) : 0;
+        return v > 0 ? v : kWin2MinChunk;
+    }();
     const int64_t target = (int64_t)tpw * slots;
     const int64_t npairs = (w.ntiles + kWin2Rows - 1) / kWin2Rows;
     int64_t bc = (int64_t)m * npairs / (target > 0 ? target : 1);
-    bc = bc < kWin2MinChunk ? kWin2MinChunk : (bc > kWin2Chunk ? kWin2Chunk : bc);
+    bc = bc < min_chunk ? min_chunk : (bc > kWin2Chunk ? kWin2Chunk : bc);
     // too few tasks to fill the slots even at the minimum chunk (C1): smaller
     // chunks, up to one task per slot (C1 0.041 -> 0.037 ms, profiles/r02/r02aj_*)
     if (npairs * ((m + bc - 1) / bc) < slots) {
